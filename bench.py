@@ -1,0 +1,319 @@
+#!/usr/bin/env python
+"""Benchmark of the GPApriori support-counting hot path on B200.
+
+One STEP = one full pass of the hot path over the workload:
+validation + generation-1 histogram, static-bitset build, and every generation's candidate
+generation, GPU support counting, (all-reduce), threshold -- i.e. one gpa_mine() call.
+
+  value  = sum_{k>=2} |C_k| * N  /  step time     (candidate x transaction / s, whole job)
+           inputs (CSR) already resident in HBM when the timed region starts;
+  e2e    = the same metric through gpa_mine() with pinned HOST buffers: the H2D copy of the CSR
+           and the D2H of every generation's counts are inside the timed region.
+
+Workload: BASELINE.json configs[4], T40I10D10M (10M transactions, 1,000 items, minsup 0.005) --
+the configuration the north star grades (HBM-bound bitset, 1.25 GB > 126 MB L2, so no L2 flush
+is needed between steps).  Multi-GPU (torchrun): the transaction axis is sharded across ranks
+(contiguous, 102,400-transaction chunks), counts are summed with NCCL all-reduce inside the
+library; the total work is fixed ("strong" scaling), time = max over ranks.
+
+--impl reference times the CPU oracle (oracle/, the parity reference) as it stands on the
+host cores, on a bounded prefix sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import gen  # noqa: E402
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=5)
+    p.add_argument("--warmup", type=int, default=3)
+    p.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    p.add_argument("--config", default="t40i10d10m", choices=list(gen.CONFIGS))
+    p.add_argument("--kernel", default="auto", choices=["auto", "v0", "prefix", "pairs"])
+    p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--cpu-sample-tx", type=int, default=0, help="oracle sample size (0 = auto)")
+    return p.parse_args()
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled every 200 ms during the timed region."""
+
+    FIELDS = "clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown," \
+             "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown," \
+             "clocks_event_reasons.sw_power_cap"
+
+    def __init__(self, device: int):
+        self.device = device
+        self.samples = []
+        self._stop = threading.Event()
+        self._t = None
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                out = subprocess.run(["nvidia-smi", "-i", str(self.device), f"--query-gpu={self.FIELDS}",
+                                      "--format=csv,noheader,nounits"], capture_output=True, text=True, timeout=5)
+                vals = [v.strip() for v in out.stdout.strip().split(",")]
+                if len(vals) == 7:
+                    self.samples.append(vals)
+            except Exception:
+                pass
+            self._stop.wait(0.2)
+
+    def __enter__(self):
+        self._t = threading.Thread(target=self._run, daemon=True)
+        self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        self._t.join()
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"], "samples": 0}
+        sm = [float(s[0]) for s in self.samples if s[0].replace(".", "").isdigit()]
+        mx = [float(s[1]) for s in self.samples if s[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({n for s in self.samples for n, v in zip(names, s[3:]) if v.lower() == "active"})
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.samples)}
+
+
+def shard_range(n_tx: int, rank: int, world: int):
+    """Contiguous rank ranges on generator-chunk boundaries (multiples of 512 transactions)."""
+    ch = gen.chunk_size()
+    n_chunks = (n_tx + ch - 1) // ch
+    c0 = n_chunks * rank // world
+    c1 = n_chunks * (rank + 1) // world
+    return min(n_tx, c0 * ch), min(n_tx, c1 * ch)
+
+
+def cpu_sample_size(cfg, requested):
+    if requested:
+        return requested
+    return {"t40i10d10m": 409_600, "t40i10d100k": 25_000, "accidents": 100_000}.get(cfg.name, cfg.n_tx)
+
+
+def run_oracle_sample(cfg, n_sample):
+    """The oracle (as it stands) on the first n_sample transactions of the workload, threshold
+    ratio unchanged.  Returns (cand_tx, seconds, threads, description)."""
+    import oracle
+    ds = gen.make(cfg.name, tx_begin=0, tx_end=min(n_sample, cfg.n_tx))
+    theta = oracle.min_count(ds.n_tx, cfg.minsup)
+    threads = max(1, len(os.sched_getaffinity(0)))
+    t0 = time.perf_counter()
+    r = oracle.mine_ds(ds, theta, threads=threads)
+    dt = time.perf_counter() - t0
+    cand_tx = sum(len(lv.cand) for lv in r.levels[1:]) * ds.n_tx
+    desc = (f"oracle.mine on the first {ds.n_tx} transactions of {cfg.name} (minsup {cfg.minsup}, "
+            f"min_count {theta}); {len(r.levels)} generations")
+    return cand_tx, dt, threads, desc
+
+
+def reference_arm(args, cfg, rank, world):
+    """--impl reference: the CPU oracle timed on the host cores (rank 0 only)."""
+    if rank != 0:
+        return
+    n_sample = cpu_sample_size(cfg, args.cpu_sample_tx)
+    for _ in range(args.warmup):
+        run_oracle_sample(cfg, min(n_sample, 20_000))
+    vals, secs = [], []
+    desc, threads, cand_tx = "", 1, 0
+    for _ in range(args.steps):
+        cand_tx, dt, threads, desc = run_oracle_sample(cfg, n_sample)
+        vals.append(cand_tx / dt)
+        secs.append(dt)
+    v = float(np.median(vals))
+    line = {
+        "impl": "reference", "metric": "support-count cand*tx/s (whole mining pass)", "value": v,
+        "unit": "cand*tx/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": float(np.median(secs)) * 1e3, "higher_is_better": True, "scaling": "strong",
+        "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+        "config": {"workload": cfg.name, "n_tx": cfg.n_tx, "n_items": cfg.n_items, "minsup": cfg.minsup,
+                   "sample_tx": n_sample},
+        "cpu_baseline": {"value": v, "unit": "cand*tx/s", "cores": threads, "kind": "oracle", "sample": desc},
+        "e2e": {"value": v, "unit": "cand*tx/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    args = parse()
+    cfg = gen.CONFIGS[args.config]
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus and rank == 0:
+        print(f"# note: WORLD_SIZE={world} but --gpus={args.gpus}; using WORLD_SIZE", file=sys.stderr)
+    if args.impl == "reference":
+        reference_arm(args, cfg, rank, world)
+        return
+
+    import torch
+    import torch.distributed as tdist
+    import paper_conf_cluster_zhangzb11a_b200 as gpa
+
+    torch.cuda.set_device(local)
+    dist = None
+    if world > 1:
+        tdist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        dist = gpa.Dist.from_torch(local)
+
+    # ---- this rank's shard of the workload (synthetic, seeded)
+    b0, b1 = shard_range(cfg.n_tx, rank, world)
+    ds = gen.make(cfg.name, tx_begin=b0, tx_end=b1)
+    theta = gpa.min_count(cfg.n_tx, cfg.minsup)
+    kern = {"auto": gpa.KERNEL_AUTO, "v0": gpa.KERNEL_V0, "prefix": gpa.KERNEL_PREFIX,
+            "pairs": gpa.KERNEL_PAIRS}[args.kernel]
+    stream = torch.cuda.current_stream()
+    opts = gpa.Options(count_kernel=kern, stream=stream.cuda_stream, device=local)
+    d_off = torch.from_numpy(ds.offsets.view(np.int64)).cuda()
+    d_items = torch.from_numpy(ds.items.view(np.int32)).cuda()
+    torch.cuda.synchronize()
+
+    def barrier():
+        if world > 1:
+            tdist.barrier(device_ids=[local])
+        torch.cuda.synchronize()
+
+    def max_over_ranks(x: float) -> float:
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device="cuda")
+        tdist.all_reduce(t, op=tdist.ReduceOp.MAX)
+        return float(t.item())
+
+    # ---- warm-up
+    res = None
+    for _ in range(max(args.warmup, 0)):
+        res = gpa.mine(d_off, d_items, ds.n_items, min_count=theta, dist=dist, options=opts)
+    # ---- timed: K steps, inputs resident in HBM
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    level_ms = {}
+    barrier()
+    with ClockSampler(local) as clocks:
+        ev0.record(stream)
+        for _ in range(args.steps):
+            res = gpa.mine(d_off, d_items, ds.n_items, min_count=theta, dist=dist, options=opts)
+            for lv in res.levels[1:]:
+                level_ms.setdefault(lv.k, []).append(lv.stats["count_ms"])
+        ev1.record(stream)
+        barrier()
+    step_ms = max_over_ranks(ev0.elapsed_time(ev1) / args.steps)
+    n_tx = res.n_tx
+    cand_tx = res.cand_tx
+    value = cand_tx / (step_ms * 1e-3)
+    launches_per_step = 2 + sum(lv.stats["launches"] for lv in res.levels[1:])  # hist + bitset + counting
+
+    # ---- dominant kernel: largest count time per step (generation 2: the tiled pair kernel)
+    dom = max(res.levels[1:], key=lambda lv: float(np.mean(level_ms[lv.k])))
+    dom_ms = max_over_ranks(float(np.mean(level_ms[dom.k])))
+    dom_work = dom.n_cand * n_tx
+    kernel_name = dom.stats["kernel_name"]
+    peaks = {}
+    try:
+        peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        pass
+    clk = clocks.summary()
+    sm_max = clk.get("sm_max_mhz") or peaks.get("sm_max_mhz", 1965.0)
+    if kernel_name == "pairs":
+        # ALU bound: 148 SMs x 16 POPC/clk/SM x 32 tx per word (profiles/r01_microbench_popc.txt)
+        peak = 148 * 16 * 32 * sm_max * 1e6 / 1e12
+        roof = {"bound": "alu", "achieved": dom_work / (dom_ms * 1e-3) / 1e12, "peak": peak, "unit": "Tcand*tx/s",
+                "peak_basis": f"148 SM x 16 POPC/clk x 32 tx/word x {sm_max:.0f} MHz (POPC rate measured)"}
+    else:
+        hbm = peaks.get("hbm_gbs", 6650.0)
+        rowbytes = dom.n_cand  # placeholder replaced below
+        groups = max(dom.stats["n_groups"], 1)
+        rowbytes = (groups * (dom.k - 1) + dom.n_cand) * (n_tx / 8)
+        roof = {"bound": "hbm", "achieved": rowbytes / (dom_ms * 1e-3) / 1e9, "peak": hbm, "unit": "GB/s",
+                "peak_basis": "MEASURED_PEAKS.json hbm_gbs"}
+    roof["frac"] = roof["achieved"] / roof["peak"]
+    roof["traffic"] = None
+    roof["kernel"] = f"count_{kernel_name} (generation {dom.k})"
+    roof["kernel_ms"] = dom_ms
+    roof["work_per_launch"] = dom_work
+
+    # ---- end to end: pinned host CSR, H2D + every D2H inside the timed region
+    e2e = None
+    if not args.no_e2e:
+        h_off = torch.from_numpy(ds.offsets.view(np.int64)).pin_memory()
+        h_items = torch.from_numpy(ds.items.view(np.int32)).pin_memory()
+        opts_h = gpa.Options(count_kernel=kern, stream=stream.cuda_stream, device=local)
+        gpa.mine(h_off, h_items, ds.n_items, min_count=theta, dist=dist, options=opts_h)
+        barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(args.steps):
+            r2 = gpa.mine(h_off, h_items, ds.n_items, min_count=theta, dist=dist, options=opts_h)
+        e1.record(stream)
+        barrier()
+        e2e_ms = max_over_ranks(e0.elapsed_time(e1) / args.steps)
+        assert r2.frequent() == res.frequent()
+        h2d = int(ds.offsets.nbytes + ds.items.nbytes)
+        d2h = 4 * sum(lv.n_cand for lv in r2.levels)  # every generation's counts (+ the histogram)
+        e2e = {"value": cand_tx / (e2e_ms * 1e-3), "unit": "cand*tx/s", "ms_per_step": e2e_ms,
+               "h2d_bytes_per_step": h2d * world, "d2h_bytes_per_step": d2h}
+
+    # ---- CPU baseline: the oracle on a bounded sample (rank 0, N = 1 only)
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        ct, dt, threads, desc = run_oracle_sample(cfg, cpu_sample_size(cfg, args.cpu_sample_tx))
+        cpu = {"value": ct / dt, "unit": "cand*tx/s", "cores": threads, "kind": "oracle", "sample": desc,
+               "seconds": dt}
+
+    if rank == 0:
+        line = {
+            "metric": "support-count cand*tx/s (whole mining pass)",
+            "value": value,
+            "unit": "cand*tx/s",
+            "n_gpus": world,
+            "steps": args.steps,
+            "warmup": args.warmup,
+            "ms_per_step": step_ms,
+            "higher_is_better": True,
+            "scaling": "strong",
+            "vs_baseline": None,
+            "dtype": "u32",
+            "data": "synthetic",
+            "config": {"workload": cfg.name, "n_tx": n_tx, "n_items": cfg.n_items, "minsup": cfg.minsup,
+                       "min_count": theta, "generations": len(res.levels), "cand_tx_per_step": cand_tx,
+                       "frequent_itemsets": sum(lv.n_freq for lv in res.levels),
+                       "l2_flush": "not needed: bitset 1.25 GB and CSR 1.6 GB exceed the 126 MB L2"
+                       if cfg.name == "t40i10d10m" else "none (small config)",
+                       "parallelism": f"tx-shard x{world}", "kernel": args.kernel},
+            "roofline": roof,
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+            "gpu_launches": launches_per_step * args.steps,
+            "clocks": clk,
+            "kernel_time_ms": {f"k{k}": float(np.mean(v)) for k, v in sorted(level_ms.items())},
+            "count_throughput": cand_tx / (sum(float(np.mean(v)) for v in level_ms.values()) * 1e-3),
+            "phase_ms_last_step": res.timing_ms,
+        }
+        print(json.dumps(line), flush=True)
+    if dist is not None:
+        dist.close()
+        tdist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,53 @@
+// Internal helpers shared by the library's runtime (.cpp) and kernel (.cu) translation units.
+// Nothing here is part of the C ABI (include/gpapriori.h is).
+#pragma once
+#include <cstdint>
+#include <cstdio>
+#include <string>
+#include <cuda_runtime.h>
+#include "gpapriori.h"
+
+namespace gpa {
+
+struct Error {
+  gpa_status status;
+  std::string msg;
+};
+
+[[noreturn]] void fail(gpa_status st, const char* fmt, ...) __attribute__((format(printf, 2, 3)));
+void set_last_error(gpa_status st, const std::string& msg);
+
+#define GPA_CUDA(call)                                                                              \
+  do {                                                                                              \
+    cudaError_t e_ = (call);                                                                        \
+    if (e_ != cudaSuccess)                                                                          \
+      ::gpa::fail(GPA_ERR_CUDA, "%s failed: %s (%s:%d)", #call, cudaGetErrorString(e_), __FILE__, __LINE__); \
+  } while (0)
+
+#define GPA_REQUIRE(cond, st, ...)                                                                  \
+  do {                                                                                              \
+    if (!(cond)) ::gpa::fail(st, __VA_ARGS__);                                                      \
+  } while (0)
+
+// Row layout of the static bitset: pitch (in 32-bit words) is a multiple of this many words
+// (128 bytes = 1024 transactions).  The paper aligns rows to 64 bytes (P18@1685); 128 B
+// matches the B200 L2 line / TMA 128B-swizzle span used by the tiled kernel.
+constexpr uint64_t kPitchWords = 32;
+
+inline uint64_t pitch_words_for(uint64_t n_tx) {
+  uint64_t w = (n_tx + 31) / 32;
+  w = (w + kPitchWords - 1) / kPitchWords * kPitchWords;
+  return w ? w : kPitchWords;
+}
+
+// Index of pair (a, b), a < b, among all pairs of n rows in lexicographic order.
+__host__ __device__ inline uint64_t pair_index(uint64_t a, uint64_t b, uint64_t n) {
+  return a * n - a * (a + 1) / 2 + (b - a - 1);
+}
+
+// Flags written by the validation/histogram kernel.
+constexpr uint32_t kFlagBadOffsets = 1u;
+constexpr uint32_t kFlagBadItem = 2u;
+constexpr uint32_t kFlagNonCanonical = 4u;
+
+}  // namespace gpa

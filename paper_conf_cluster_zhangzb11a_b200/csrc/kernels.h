@@ -1,0 +1,47 @@
+// Launch wrappers of the sm_100a kernels (defined in csrc/kernels/*.cu).  All are
+// asynchronous on `stream`; all device pointers live on the current device.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace gpa {
+
+// ---- generation 1 (P13@338: "test their frequencies by scanning the transaction database")
+// Validates the CSR (offsets monotone, items < n_items, canonical order) into *flags and
+// accumulates hist[item] += 1 per (transaction, item) incidence.  hist must be zeroed.
+void launch_hist_validate(const uint64_t* offsets, const uint32_t* items, uint64_t n_tx, uint32_t n_items,
+                          uint32_t* hist, uint32_t* flags, int n_sms, cudaStream_t stream);
+// Same histogram for non-canonical input: an item counts once per transaction (set semantics).
+void launch_hist_dedup(const uint64_t* offsets, const uint32_t* items, uint64_t n_tx, uint32_t n_items,
+                       uint32_t* hist, int n_sms, cudaStream_t stream);
+
+// ---- static bitset (P18@755): rows[r][t/32] bit t%32 = [item_of_row[r] in t]
+void launch_bitset_build(const uint64_t* offsets, const uint32_t* items, uint64_t n_tx,
+                         const int32_t* row_of_item, uint32_t n_rows, uint64_t pitch_words, uint32_t* rows,
+                         cudaStream_t stream);
+
+// ---- support counting (complete intersection, P18@394-2515)
+// Paper design: one CTA per candidate, AND of all k rows, popc, block reduction.
+void launch_count_v0(const uint32_t* rows, uint64_t pitch_words, const uint32_t* cand_rows, uint32_t k,
+                     uint64_t M, uint32_t* counts, cudaStream_t stream);
+
+// Prefix-staged streaming: groups share a (k-1)-prefix; counts must be zeroed (atomic adds).
+struct PrefixTask {
+  uint32_t group;   // prefix group
+  uint32_t first;   // index of the first sibling (global candidate index)
+  uint32_t n;       // siblings in this task (<= kPrefixMaxSiblings)
+  uint32_t pad;
+};
+constexpr uint32_t kPrefixMaxSiblings = 32;
+// returns the number of CTAs launched
+uint64_t launch_count_prefix(const uint32_t* rows, uint64_t pitch_words, const uint32_t* prefix_rows, uint32_t km1,
+                             const uint32_t* ext_rows, const PrefixTask* tasks, uint32_t n_tasks, uint32_t* counts,
+                             cudaStream_t stream);
+
+// k = 2 TMA-tiled kernel: all pairs (a < b) of the n_rows rows; counts[pair_index] must be zeroed.
+// tmap: opaque 128-byte CUtensorMap built by make_pairs_tensor_map.
+bool make_pairs_tensor_map(void* tmap128, const uint32_t* rows, uint32_t n_rows, uint64_t pitch_words);
+uint64_t launch_count_pairs(const void* tmap128, uint32_t n_rows, uint64_t pitch_words, uint32_t* counts,
+                            int n_sms, cudaStream_t stream);
+
+}  // namespace gpa

@@ -1,0 +1,437 @@
+// Static bitset construction and the counting engine (host side of the library).
+//
+// gpa_bitset_create / gpa_mine share bitset_build():
+//   upload (host CSR only) -> device validation + generation-1 histogram (P13@338)
+//   -> all-reduce of the histogram across ranks -> rows = items with count >= row_min_count,
+//   ascending item id -> device transpose of the CSR into the static bitset (P18@755).
+// count_grouped / count_all_pairs run the sm_100a counting kernels on a candidate batch and
+// leave the (rank-summed) counts in bs->d_counts.
+#include <algorithm>
+#include <chrono>
+#include <numeric>
+
+#include "internal.h"
+
+namespace gpa {
+
+namespace {
+
+double now_ms() {
+  return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now().time_since_epoch()).count();
+}
+
+float event_ms(cudaEvent_t a, cudaEvent_t b) {
+  float ms = 0;
+  GPA_CUDA(cudaEventElapsedTime(&ms, a, b));
+  return ms;
+}
+
+void validate_options(const gpa_options& o) {
+  GPA_REQUIRE(o.count_kernel <= GPA_KERNEL_PAIRS, GPA_ERR_INVALID, "unknown count_kernel %u", o.count_kernel);
+  GPA_REQUIRE(o.max_k <= GPA_MAX_K, GPA_ERR_INVALID, "max_k %u > GPA_MAX_K", o.max_k);
+  GPA_REQUIRE(!o.reserved[0] && !o.reserved[1] && !o.reserved[2], GPA_ERR_INVALID, "reserved option fields must be 0");
+}
+
+}  // namespace
+
+gpa_bitset* bitset_build(const gpa_tx_csr* db, uint64_t row_min_count, const gpa_dist* dist, const gpa_options* opt_in) {
+  GPA_REQUIRE(db, GPA_ERR_INVALID, "db is NULL");
+  GPA_REQUIRE(db->memory == GPA_MEM_HOST || db->memory == GPA_MEM_DEVICE, GPA_ERR_INVALID, "db->memory must be "
+              "GPA_MEM_HOST or GPA_MEM_DEVICE");
+  GPA_REQUIRE(db->offsets || db->n_tx == 0, GPA_ERR_INVALID, "db->offsets is NULL");
+  gpa_options opt;
+  gpa_options_default(&opt);
+  if (opt_in) opt = *opt_in;
+  validate_options(opt);
+  dist_check(dist);
+  DeviceInfo di = use_device(dist ? dist->device : opt.device);
+
+  auto* bs = new gpa_bitset();
+  struct Guard {
+    gpa_bitset* b;
+    ~Guard() { if (b) bitset_free(b); }
+  } guard{bs};
+  bs->device = di.device;
+  bs->n_sms = di.n_sms;
+  bs->dist = dist;
+  bs->opt = opt;
+  bs->n_items = db->n_items;
+  bs->n_tx_local = db->n_tx;
+  if (opt.stream) {
+    bs->stream = static_cast<cudaStream_t>(opt.stream);
+  } else {
+    GPA_CUDA(cudaStreamCreateWithFlags(&bs->stream, cudaStreamNonBlocking));
+    bs->own_stream = true;
+  }
+  GPA_CUDA(cudaEventCreate(&bs->ev0));
+  GPA_CUDA(cudaEventCreate(&bs->ev1));
+  GPA_CUDA(cudaEventCreate(&bs->ev2));
+  cudaStream_t s = bs->stream;
+
+  // ---- input on the device
+  double t0 = now_ms();
+  const uint64_t n_tx = db->n_tx;
+  uint64_t nnz = 0;
+  DBuf<uint64_t> d_off;
+  DBuf<uint32_t> d_items;
+  const uint64_t* off_dev = db->offsets;
+  const uint32_t* items_dev = db->items;
+  uint64_t first_off = 0;
+  if (db->memory == GPA_MEM_HOST) {
+    if (n_tx) {
+      first_off = db->offsets[0];
+      nnz = db->offsets[n_tx];
+    }
+    GPA_REQUIRE(first_off == 0, GPA_ERR_INVALID, "offsets[0] must be 0");
+    GPA_REQUIRE(db->items || nnz == 0, GPA_ERR_INVALID, "db->items is NULL");
+    d_off.alloc(n_tx + 1, s);
+    GPA_CUDA(cudaMemcpyAsync(d_off.p, db->offsets, (n_tx + 1) * sizeof(uint64_t), cudaMemcpyHostToDevice, s));
+    if (nnz) {
+      d_items.alloc(nnz, s);
+      GPA_CUDA(cudaMemcpyAsync(d_items.p, db->items, nnz * sizeof(uint32_t), cudaMemcpyHostToDevice, s));
+    }
+    off_dev = d_off.p;
+    items_dev = d_items.p;
+  } else if (n_tx) {
+    GPA_CUDA(cudaMemcpyAsync(&first_off, db->offsets, sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+    GPA_CUDA(cudaStreamSynchronize(s));
+    GPA_REQUIRE(first_off == 0, GPA_ERR_INVALID, "offsets[0] must be 0");
+  }
+  GPA_CUDA(cudaStreamSynchronize(s));
+  double t1 = now_ms();
+  bs->build_ms[0] = t1 - t0;
+
+  // ---- validation + generation-1 histogram (+ n_tx) ; one all-reduce each
+  const uint32_t n_items = db->n_items;
+  DBuf<uint32_t> d_hist, d_flags;
+  DBuf<uint64_t> d_ntx;
+  d_hist.alloc(std::max<uint32_t>(n_items, 1), s);
+  d_flags.alloc(1, s);
+  d_ntx.alloc(1, s);
+  GPA_CUDA(cudaMemsetAsync(d_hist.p, 0, std::max<uint32_t>(n_items, 1) * sizeof(uint32_t), s));
+  GPA_CUDA(cudaMemsetAsync(d_flags.p, 0, sizeof(uint32_t), s));
+  GPA_CUDA(cudaMemcpyAsync(d_ntx.p, &bs->n_tx_local, sizeof(uint64_t), cudaMemcpyHostToDevice, s));
+  launch_hist_validate(off_dev, items_dev, n_tx, n_items, d_hist.p, d_flags.p, bs->n_sms, s);
+  uint32_t flags = 0;
+  GPA_CUDA(cudaMemcpyAsync(&flags, d_flags.p, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+  GPA_CUDA(cudaStreamSynchronize(s));
+  if ((flags & kFlagNonCanonical) && !(flags & (kFlagBadItem | kFlagBadOffsets))) {
+    GPA_CUDA(cudaMemsetAsync(d_hist.p, 0, n_items * sizeof(uint32_t), s));
+    launch_hist_dedup(off_dev, items_dev, n_tx, n_items, d_hist.p, bs->n_sms, s);
+  }
+  allreduce_max_u32(dist, d_flags.p, 1, s);   // every rank takes the same accept / reject decision
+  allreduce_sum_u32(dist, d_hist.p, n_items, s);
+  allreduce_sum_u64(dist, d_ntx.p, 1, s);
+  bs->item_counts.assign(n_items, 0);
+  if (n_items)
+    GPA_CUDA(cudaMemcpyAsync(bs->item_counts.data(), d_hist.p, n_items * sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+  GPA_CUDA(cudaMemcpyAsync(&flags, d_flags.p, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+  GPA_CUDA(cudaMemcpyAsync(&bs->n_tx_global, d_ntx.p, sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+  GPA_CUDA(cudaStreamSynchronize(s));
+  GPA_REQUIRE(!(flags & kFlagBadOffsets), GPA_ERR_INVALID, "offsets are not non-decreasing%s",
+              dist ? " (on some rank)" : "");
+  GPA_REQUIRE(!(flags & kFlagBadItem), GPA_ERR_INVALID, "an item id is >= n_items (%u)%s", n_items,
+              dist ? " (on some rank)" : "");
+  GPA_REQUIRE(bs->n_tx_global < (1ull << 32), GPA_ERR_INVALID, "n_tx must be < 2^32 (32-bit supports)");
+  double t2 = now_ms();
+  bs->build_ms[1] = t2 - t1;
+
+  // ---- rows: items with count >= row_min_count, ascending id (Q8, Q14)
+  bs->row_of_item.assign(n_items, -1);
+  for (uint32_t i = 0; i < n_items; ++i) {
+    if (bs->item_counts[i] >= row_min_count && bs->item_counts[i] > 0) {
+      bs->row_of_item[i] = (int32_t)bs->item_of_row.size();
+      bs->item_of_row.push_back(i);
+    }
+  }
+  bs->n_rows = (uint32_t)bs->item_of_row.size();
+  bs->pitch_words = pitch_words_for(n_tx);
+  if (bs->n_rows) {
+    DBuf<int32_t> d_map;
+    d_map.alloc(n_items, s);
+    GPA_CUDA(cudaMemcpyAsync(d_map.p, bs->row_of_item.data(), n_items * sizeof(int32_t), cudaMemcpyHostToDevice, s));
+    bs->rows.alloc((size_t)bs->n_rows * bs->pitch_words, s);
+    launch_bitset_build(off_dev, items_dev, n_tx, d_map.p, bs->n_rows, bs->pitch_words, bs->rows.p, s);
+  }
+  GPA_CUDA(cudaStreamSynchronize(s));
+  bs->build_ms[2] = now_ms() - t2;
+  guard.b = nullptr;
+  return bs;
+}
+
+void bitset_free(gpa_bitset* bs) {
+  if (!bs) return;
+  if (bs->stream) cudaStreamSynchronize(bs->stream);
+  bs->rows.reset();
+  bs->d_counts.reset();
+  bs->d_prefix.reset();
+  bs->d_ext.reset();
+  bs->d_flat.reset();
+  bs->d_tasks.reset();
+  if (bs->stream) cudaStreamSynchronize(bs->stream);
+  if (bs->ev0) cudaEventDestroy(bs->ev0);
+  if (bs->ev1) cudaEventDestroy(bs->ev1);
+  if (bs->ev2) cudaEventDestroy(bs->ev2);
+  if (bs->own_stream && bs->stream) cudaStreamDestroy(bs->stream);
+  delete bs;
+}
+
+// ------------------------------------------------------------------ counting engine
+
+namespace {
+
+void finish_counts(gpa_bitset* bs, size_t M, CountStats* st) {
+  cudaStream_t s = bs->stream;
+  GPA_CUDA(cudaEventRecord(bs->ev1, s));
+  allreduce_sum_u32(bs->dist, bs->d_counts.p, M, s);
+  GPA_CUDA(cudaEventRecord(bs->ev2, s));
+  GPA_CUDA(cudaEventSynchronize(bs->ev2));
+  if (st) {
+    st->count_ms = event_ms(bs->ev0, bs->ev1);
+    st->allreduce_ms = bs->dist ? event_ms(bs->ev1, bs->ev2) : 0.0;
+  }
+}
+
+void count_flat_v0(gpa_bitset* bs, const std::vector<uint32_t>& flat, uint32_t k, uint64_t M, CountStats* st) {
+  cudaStream_t s = bs->stream;
+  bs->d_flat.ensure(std::max<size_t>(flat.size(), 1), s);
+  bs->d_counts.ensure(std::max<uint64_t>(M, 1), s);
+  GPA_CUDA(cudaMemcpyAsync(bs->d_flat.p, flat.data(), flat.size() * sizeof(uint32_t), cudaMemcpyHostToDevice, s));
+  GPA_CUDA(cudaEventRecord(bs->ev0, s));
+  if (bs->n_rows) launch_count_v0(bs->rows.p, bs->pitch_words, bs->d_flat.p, k, M, bs->d_counts.p, s);
+  else GPA_CUDA(cudaMemsetAsync(bs->d_counts.p, 0, M * sizeof(uint32_t), s));
+  if (st) { st->kernel = GPA_KERNEL_V0; st->launches = 1; }
+  finish_counts(bs, M, st);
+}
+
+}  // namespace
+
+void count_grouped(gpa_bitset* bs, const GroupedBatch& b, uint32_t kernel, CountStats* st) {
+  cudaStream_t s = bs->stream;
+  const uint64_t M = b.size(), G = b.groups();
+  const uint32_t km1 = b.k - 1;
+  if (M == 0) return;
+  if (kernel == GPA_KERNEL_AUTO) kernel = GPA_KERNEL_PREFIX;
+  if (kernel == GPA_KERNEL_PAIRS) kernel = GPA_KERNEL_PREFIX;  // grouped batches use the prefix kernel
+  if (kernel == GPA_KERNEL_V0 || km1 == 0) {
+    std::vector<uint32_t> flat(M * b.k);
+    for (uint64_t g = 0; g < G; ++g)
+      for (uint64_t j = b.ext_off[g]; j < b.ext_off[g + 1]; ++j) {
+        std::copy(b.prefix.begin() + g * km1, b.prefix.begin() + (g + 1) * km1, flat.begin() + j * b.k);
+        flat[j * b.k + km1] = b.ext[j];
+      }
+    count_flat_v0(bs, flat, b.k, M, st);
+    return;
+  }
+  GPA_REQUIRE(G < (1ull << 32) && M < (1ull << 32), GPA_ERR_INVALID, "candidate batch too large");
+  // tasks: each group split into chunks of <= kPrefixMaxSiblings siblings
+  std::vector<PrefixTask> tasks;
+  tasks.reserve(M / 8 + G);
+  for (uint64_t g = 0; g < G; ++g)
+    for (uint64_t j = b.ext_off[g]; j < b.ext_off[g + 1]; j += kPrefixMaxSiblings) {
+      uint32_t n = (uint32_t)std::min<uint64_t>(kPrefixMaxSiblings, b.ext_off[g + 1] - j);
+      tasks.push_back(PrefixTask{(uint32_t)g, (uint32_t)j, n, 0});
+    }
+  bs->d_prefix.ensure(b.prefix.size(), s);
+  bs->d_ext.ensure(M, s);
+  bs->d_tasks.ensure(tasks.size(), s);
+  bs->d_counts.ensure(M, s);
+  GPA_CUDA(cudaMemcpyAsync(bs->d_prefix.p, b.prefix.data(), b.prefix.size() * sizeof(uint32_t), cudaMemcpyHostToDevice, s));
+  GPA_CUDA(cudaMemcpyAsync(bs->d_ext.p, b.ext.data(), M * sizeof(uint32_t), cudaMemcpyHostToDevice, s));
+  GPA_CUDA(cudaMemcpyAsync(bs->d_tasks.p, tasks.data(), tasks.size() * sizeof(PrefixTask), cudaMemcpyHostToDevice, s));
+  GPA_CUDA(cudaMemsetAsync(bs->d_counts.p, 0, M * sizeof(uint32_t), s));
+  GPA_CUDA(cudaEventRecord(bs->ev0, s));
+  // a task index must fit the kernel's 32-bit grid decode: launch in slices of tasks if needed
+  const uint64_t max_tasks = 1u << 20;
+  uint32_t launches = 0;
+  for (uint64_t t0 = 0; t0 < tasks.size(); t0 += max_tasks) {
+    uint32_t nt = (uint32_t)std::min<uint64_t>(max_tasks, tasks.size() - t0);
+    launch_count_prefix(bs->rows.p, bs->pitch_words, bs->d_prefix.p, km1, bs->d_ext.p, bs->d_tasks.p + t0, nt,
+                        bs->d_counts.p, s);
+    ++launches;
+  }
+  if (st) { st->kernel = GPA_KERNEL_PREFIX; st->launches = launches; }
+  finish_counts(bs, M, st);
+}
+
+void count_all_pairs(gpa_bitset* bs, uint32_t kernel, CountStats* st) {
+  cudaStream_t s = bs->stream;
+  const uint64_t n = bs->n_rows;
+  const uint64_t M = n * (n - 1) / 2;
+  if (n < 2) return;
+  if (kernel == GPA_KERNEL_AUTO) kernel = GPA_KERNEL_PAIRS;
+  if (kernel != GPA_KERNEL_PAIRS) {
+    GroupedBatch b;
+    b.k = 2;
+    b.ext_off.push_back(0);
+    for (uint64_t a = 0; a + 1 < n; ++a) {
+      b.prefix.push_back((uint32_t)a);
+      for (uint64_t c = a + 1; c < n; ++c) b.ext.push_back((uint32_t)c);
+      b.ext_off.push_back(b.ext.size());
+    }
+    count_grouped(bs, b, kernel, st);
+    return;
+  }
+  if (!bs->tmap_ready) {
+    make_pairs_tensor_map(bs->tmap, bs->rows.p, bs->n_rows, bs->pitch_words);
+    bs->tmap_ready = true;
+  }
+  bs->d_counts.ensure(M, s);
+  GPA_CUDA(cudaMemsetAsync(bs->d_counts.p, 0, M * sizeof(uint32_t), s));
+  GPA_CUDA(cudaEventRecord(bs->ev0, s));
+  launch_count_pairs(bs->tmap, bs->n_rows, bs->pitch_words, bs->d_counts.p, bs->n_sms, s);
+  if (st) { st->kernel = GPA_KERNEL_PAIRS; st->launches = 1; }
+  finish_counts(bs, M, st);
+}
+
+}  // namespace gpa
+
+// ---------------------------------------------------------------- C ABI: options, threshold, bitset
+
+extern "C" void gpa_options_default(gpa_options* opt) {
+  if (!opt) return;
+  memset(opt, 0, sizeof(*opt));
+  opt->count_kernel = GPA_KERNEL_AUTO;
+  opt->device = -1;
+}
+
+extern "C" uint64_t gpa_min_count(uint64_t n_tx, uint64_t num, uint64_t den) {
+  if (den == 0) return 0;
+  unsigned __int128 q = ((unsigned __int128)n_tx * num + den - 1) / den;
+  if (q > UINT64_MAX) q = UINT64_MAX;
+  return q < 1 ? 1 : (uint64_t)q;
+}
+
+extern "C" gpa_status gpa_bitset_create(const gpa_tx_csr* db, uint32_t row_min_count, const gpa_dist* dist,
+                                        const gpa_options* opt, gpa_bitset** out) {
+  return gpa::guard([&] {
+    GPA_REQUIRE(out, GPA_ERR_INVALID, "out is NULL");
+    *out = gpa::bitset_build(db, row_min_count, dist, opt);
+  });
+}
+
+extern "C" gpa_status gpa_bitset_destroy(gpa_bitset* bs) {
+  return gpa::guard([&] { gpa::bitset_free(bs); });
+}
+
+extern "C" gpa_status gpa_bitset_info(const gpa_bitset* bs, uint64_t* n_tx_local, uint64_t* n_tx_global,
+                                      uint32_t* n_rows, uint64_t* row_pitch_bytes) {
+  return gpa::guard([&] {
+    GPA_REQUIRE(bs, GPA_ERR_INVALID, "bitset is NULL");
+    if (n_tx_local) *n_tx_local = bs->n_tx_local;
+    if (n_tx_global) *n_tx_global = bs->n_tx_global;
+    if (n_rows) *n_rows = bs->n_rows;
+    if (row_pitch_bytes) *row_pitch_bytes = bs->pitch_words * 4;
+  });
+}
+
+extern "C" gpa_status gpa_bitset_item_counts(const gpa_bitset* bs, uint32_t* counts_out) {
+  return gpa::guard([&] {
+    GPA_REQUIRE(bs && counts_out, GPA_ERR_INVALID, "NULL argument");
+    std::copy(bs->item_counts.begin(), bs->item_counts.end(), counts_out);
+  });
+}
+
+extern "C" gpa_status gpa_bitset_rows(const gpa_bitset* bs, uint32_t* item_of_row_out) {
+  return gpa::guard([&] {
+    GPA_REQUIRE(bs && (item_of_row_out || bs->n_rows == 0), GPA_ERR_INVALID, "NULL argument");
+    std::copy(bs->item_of_row.begin(), bs->item_of_row.end(), item_of_row_out);
+  });
+}
+
+extern "C" gpa_status gpa_bitset_export(const gpa_bitset* bs, uint32_t* host_out) {
+  return gpa::guard([&] {
+    GPA_REQUIRE(bs && (host_out || bs->n_rows == 0), GPA_ERR_INVALID, "NULL argument");
+    if (!bs->n_rows) return;
+    gpa::use_device(bs->device);
+    GPA_CUDA(cudaMemcpyAsync(host_out, bs->rows.p, (size_t)bs->n_rows * bs->pitch_words * 4, cudaMemcpyDeviceToHost,
+                             bs->stream));
+    GPA_CUDA(cudaStreamSynchronize(bs->stream));
+  });
+}
+
+extern "C" gpa_status gpa_count(gpa_bitset* bs, const uint32_t* cand, uint32_t k, uint64_t M, uint32_t kernel,
+                                uint32_t* counts_out) {
+  return gpa::guard([&] {
+    GPA_REQUIRE(bs, GPA_ERR_INVALID, "bitset is NULL");
+    GPA_REQUIRE(k >= 1 && k <= GPA_MAX_K, GPA_ERR_INVALID, "k must be in [1, %u]", GPA_MAX_K);
+    GPA_REQUIRE(kernel <= GPA_KERNEL_PAIRS, GPA_ERR_INVALID, "unknown kernel %u", kernel);
+    if (M == 0) return;
+    GPA_REQUIRE(cand && counts_out, GPA_ERR_INVALID, "NULL argument");
+    GPA_REQUIRE(M <= (UINT64_MAX / 8) / k && M < (1ull << 32), GPA_ERR_INVALID, "M * k overflows");
+    gpa::dist_check(bs->dist);
+    gpa::use_device(bs->device);
+    // validate + translate to row ids
+    std::vector<uint32_t> rows(M * k);
+    for (uint64_t m = 0; m < M; ++m) {
+      for (uint32_t j = 0; j < k; ++j) {
+        const uint32_t it = cand[m * k + j];
+        GPA_REQUIRE(it < bs->n_items, GPA_ERR_INVALID, "candidate %llu: item %u >= n_items", (unsigned long long)m, it);
+        GPA_REQUIRE(j == 0 || it > cand[m * k + j - 1], GPA_ERR_INVALID,
+                    "candidate %llu is not strictly increasing", (unsigned long long)m);
+        const int32_t r = bs->row_of_item[it];
+        GPA_REQUIRE(r >= 0, GPA_ERR_RANGE, "item %u has no bitset row", it);
+        rows[m * k + j] = (uint32_t)r;
+      }
+    }
+    uint32_t kern = kernel == GPA_KERNEL_AUTO ? bs->opt.count_kernel : kernel;
+    if (k == 1) kern = GPA_KERNEL_V0;
+    if (kern == GPA_KERNEL_AUTO)
+      kern = (k == 2 && (double)M * 8 >= (double)bs->n_rows * bs->n_rows) ? GPA_KERNEL_PAIRS : GPA_KERNEL_PREFIX;
+    if (kern == GPA_KERNEL_PAIRS && k != 2) kern = GPA_KERNEL_PREFIX;
+    if (kern == GPA_KERNEL_PAIRS) {
+      gpa::count_all_pairs(bs, GPA_KERNEL_PAIRS, nullptr);
+      const uint64_t n = bs->n_rows, P = n * (n - 1) / 2;
+      std::vector<uint32_t> all(P);
+      if (P) {
+        GPA_CUDA(cudaMemcpyAsync(all.data(), bs->d_counts.p, P * 4, cudaMemcpyDeviceToHost, bs->stream));
+        GPA_CUDA(cudaStreamSynchronize(bs->stream));
+      }
+      for (uint64_t m = 0; m < M; ++m) counts_out[m] = all[gpa::pair_index(rows[2 * m], rows[2 * m + 1], n)];
+      return;
+    }
+    if (kern == GPA_KERNEL_V0) {
+      gpa::GroupedBatch b;  // V0 path takes the flat batch in caller order: one group per candidate
+      b.k = k;
+      b.ext_off.resize(M + 1);
+      b.prefix.resize(M * (k - 1));
+      b.ext.resize(M);
+      for (uint64_t m = 0; m < M; ++m) {
+        std::copy(rows.begin() + m * k, rows.begin() + m * k + k - 1, b.prefix.begin() + m * (k - 1));
+        b.ext[m] = rows[m * k + k - 1];
+        b.ext_off[m] = m;
+      }
+      b.ext_off[M] = M;
+      gpa::count_grouped(bs, b, GPA_KERNEL_V0, nullptr);
+      GPA_CUDA(cudaMemcpyAsync(counts_out, bs->d_counts.p, M * 4, cudaMemcpyDeviceToHost, bs->stream));
+      GPA_CUDA(cudaStreamSynchronize(bs->stream));
+      return;
+    }
+    // PREFIX: group by (k-1)-prefix (sort candidate indices lexicographically)
+    std::vector<uint64_t> order(M);
+    std::iota(order.begin(), order.end(), 0);
+    std::sort(order.begin(), order.end(), [&](uint64_t a, uint64_t b) {
+      return std::lexicographical_compare(rows.begin() + a * k, rows.begin() + a * k + k, rows.begin() + b * k,
+                                          rows.begin() + b * k + k);
+    });
+    gpa::GroupedBatch b;
+    b.k = k;
+    b.ext.resize(M);
+    for (uint64_t i = 0; i < M; ++i) {
+      const uint64_t m = order[i];
+      const bool new_group = i == 0 || !std::equal(rows.begin() + m * k, rows.begin() + m * k + k - 1,
+                                                    rows.begin() + order[i - 1] * k);
+      if (new_group) {
+        b.ext_off.push_back(i);
+        b.prefix.insert(b.prefix.end(), rows.begin() + m * k, rows.begin() + m * k + k - 1);
+      }
+      b.ext[i] = rows[m * k + k - 1];
+    }
+    b.ext_off.push_back(M);
+    gpa::count_grouped(bs, b, GPA_KERNEL_PREFIX, nullptr);
+    std::vector<uint32_t> sorted(M);
+    GPA_CUDA(cudaMemcpyAsync(sorted.data(), bs->d_counts.p, M * 4, cudaMemcpyDeviceToHost, bs->stream));
+    GPA_CUDA(cudaStreamSynchronize(bs->stream));
+    for (uint64_t i = 0; i < M; ++i) counts_out[order[i]] = sorted[i];
+  });
+}

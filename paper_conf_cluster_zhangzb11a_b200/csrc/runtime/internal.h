@@ -1,0 +1,155 @@
+// Runtime-internal declarations (handles, device buffers, counting engine).
+#pragma once
+#include <cstdint>
+#include <cstring>
+#include <string>
+#include <utility>
+#include <vector>
+#include <new>
+#include <exception>
+
+#include <cuda_runtime.h>
+#include <nccl.h>
+
+#include "../common.h"
+#include "../kernels.h"
+
+struct gpa_dist {
+  ncclComm_t comm = nullptr;
+  int rank = 0, world = 1, device = 0;
+  bool failed = false;
+};
+
+namespace gpa {
+
+// Device buffer allocated from the device's stream-ordered pool (cudaMallocAsync).  The pool's
+// release threshold is raised once per device so repeated calls reuse memory without a
+// cudaMalloc / cudaFree round trip.
+template <class T>
+struct DBuf {
+  T* p = nullptr;
+  size_t n = 0;
+  cudaStream_t s = nullptr;
+  DBuf() = default;
+  DBuf(const DBuf&) = delete;
+  DBuf& operator=(const DBuf&) = delete;
+  DBuf(DBuf&& o) noexcept { swap(o); }
+  DBuf& operator=(DBuf&& o) noexcept { reset(); swap(o); return *this; }
+  ~DBuf() { reset(); }
+  void swap(DBuf& o) noexcept { std::swap(p, o.p); std::swap(n, o.n); std::swap(s, o.s); }
+  void reset() noexcept {
+    if (p) cudaFreeAsync(p, s);
+    p = nullptr; n = 0;
+  }
+  void alloc(size_t count, cudaStream_t stream) {
+    reset();
+    s = stream;
+    n = count;
+    if (count == 0) return;
+    cudaError_t e = cudaMallocAsync(reinterpret_cast<void**>(&p), count * sizeof(T), stream);
+    if (e != cudaSuccess) {
+      p = nullptr;
+      n = 0;
+      cudaGetLastError();
+      fail(e == cudaErrorMemoryAllocation ? GPA_ERR_OOM : GPA_ERR_CUDA, "device allocation of %zu bytes failed: %s",
+           count * sizeof(T), cudaGetErrorString(e));
+    }
+  }
+  // grow-only reuse
+  void ensure(size_t count, cudaStream_t stream) {
+    if (count > n || stream != s) alloc(count, stream);
+  }
+};
+
+struct DeviceInfo {
+  int device;
+  int n_sms;
+};
+DeviceInfo use_device(int requested);   // cudaSetDevice + one-time pool setup
+
+// NCCL helpers (no-ops without dist)
+void dist_check(const gpa_dist* d);
+void allreduce_sum_u32(const gpa_dist* d, uint32_t* buf, size_t n, cudaStream_t s);
+void allreduce_sum_u64(const gpa_dist* d, uint64_t* buf, size_t n, cudaStream_t s);
+void allreduce_max_u32(const gpa_dist* d, uint32_t* buf, size_t n, cudaStream_t s);
+
+// Candidate batch grouped by (k-1)-prefix, in ROW ids.  Candidates are prefix + ext[j] for
+// j in [ext_off[g], ext_off[g+1]); global candidate index = position in ext.
+struct GroupedBatch {
+  uint32_t k = 0;
+  std::vector<uint32_t> prefix;    // G * (k-1)
+  std::vector<uint64_t> ext_off;   // G + 1
+  std::vector<uint32_t> ext;       // M
+  uint64_t groups() const { return ext_off.empty() ? 0 : ext_off.size() - 1; }
+  uint64_t size() const { return ext.size(); }
+};
+
+// Join + prune of L_{k-1} (n x (k-1) row ids, lexicographic, distinct) into C_k grouped by
+// (k-1)-prefix; candidates come out in lexicographic order.
+GroupedBatch candgen_join_prune(const std::vector<uint32_t>& L, uint64_t n, uint32_t km1);
+
+const char* last_error_cstr();
+
+// Run f() and translate exceptions into a gpa_status + thread-local message (no exception
+// crosses the C ABI).
+template <class F>
+gpa_status guard(F&& f) {
+  try {
+    f();
+    return GPA_OK;
+  } catch (const Error& e) {
+    set_last_error(e.status, e.msg);
+    return e.status;
+  } catch (const std::bad_alloc&) {
+    set_last_error(GPA_ERR_OOM, "host allocation failed");
+    return GPA_ERR_OOM;
+  } catch (const std::exception& e) {
+    set_last_error(GPA_ERR_INVALID, std::string("internal error: ") + e.what());
+    return GPA_ERR_INVALID;
+  } catch (...) {
+    set_last_error(GPA_ERR_INVALID, "internal error");
+    return GPA_ERR_INVALID;
+  }
+}
+
+struct CountStats {
+  uint32_t kernel = 0;
+  uint32_t launches = 0;
+  double count_ms = 0;
+  double allreduce_ms = 0;
+};
+
+}  // namespace gpa
+
+struct gpa_bitset {
+  int device = 0;
+  int n_sms = 148;
+  cudaStream_t stream = nullptr;
+  bool own_stream = false;
+  const gpa_dist* dist = nullptr;
+  gpa_options opt{};
+  uint64_t n_tx_local = 0, n_tx_global = 0;
+  uint32_t n_items = 0, n_rows = 0;
+  uint64_t pitch_words = 0;
+  gpa::DBuf<uint32_t> rows;
+  std::vector<uint32_t> item_counts;   // global, n_items
+  std::vector<uint32_t> item_of_row;   // n_rows, ascending
+  std::vector<int32_t> row_of_item;    // n_items, -1 if no row
+  alignas(64) unsigned char tmap[128];
+  bool tmap_ready = false;
+  // counting workspace (grow-only)
+  gpa::DBuf<uint32_t> d_counts, d_prefix, d_ext, d_flat;
+  gpa::DBuf<gpa::PrefixTask> d_tasks;
+  cudaEvent_t ev0 = nullptr, ev1 = nullptr, ev2 = nullptr;
+  double build_ms[3] = {0, 0, 0};      // upload, histogram, bitset
+};
+
+namespace gpa {
+// Build the static bitset (histogram, rows, bitset) -- shared by gpa_bitset_create / gpa_mine.
+gpa_bitset* bitset_build(const gpa_tx_csr* db, uint64_t row_min_count, const gpa_dist* dist, const gpa_options* opt);
+void bitset_free(gpa_bitset* bs);
+// Count a grouped batch into bs->d_counts (device, M entries, summed over ranks).
+void count_grouped(gpa_bitset* bs, const GroupedBatch& b, uint32_t kernel, CountStats* st);
+// Count all pairs of rows (lexicographic pair order) into bs->d_counts (n(n-1)/2 entries).
+void count_all_pairs(gpa_bitset* bs, uint32_t kernel, CountStats* st);
+}  // namespace gpa

@@ -1,0 +1,242 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle, element by element.
+
+Bar: bit-exact -- supports are integers.  Inputs are the seeded
+generators of gen/; expected values come only from oracle/ (or, for the bit layout, from a
+numpy bit-packing written here).  Sizes span several tiles / stripes plus ragged tails.
+"""
+import os
+from itertools import combinations
+
+import numpy as np
+import pytest
+
+import gen
+import oracle
+import paper_conf_cluster_zhangzb11a_b200 as gpa
+
+pytestmark = pytest.mark.gpu
+
+KERNELS = [gpa.KERNEL_V0, gpa.KERNEL_PREFIX, gpa.KERNEL_PAIRS]
+
+
+def expected_bits(ds, item_of_row, pitch_words):
+    """Row r, transaction t -> word t//32, bit t%32 (LSB first), built with numpy."""
+    out = np.zeros((len(item_of_row), pitch_words), dtype=np.uint32)
+    pos = {int(it): r for r, it in enumerate(item_of_row)}
+    for t, tx in enumerate(ds.transactions()):
+        for it in set(int(x) for x in tx):
+            if it in pos:
+                out[pos[it], t // 32] |= np.uint32(1 << (t % 32))
+    return out
+
+
+def assert_mine_equal(res, ref):
+    assert len(res.levels) == len(ref.levels), ([lv.n_cand for lv in res.levels], [len(l.cand) for l in ref.levels])
+    for lv, rl in zip(res.levels, ref.levels):
+        assert lv.k == rl.k
+        assert np.array_equal(lv.cand, rl.cand), f"C_{lv.k} differs"
+        assert np.array_equal(lv.counts, rl.count), f"counts of C_{lv.k} differ"
+    assert res.frequent() == ref.frequent()
+
+
+# ---------------------------------------------------------------- Fig. 2 (P13@2637)
+
+def test_fig2_bitset_and_supports(fig2):
+    txs, vert = fig2
+    ds = gen.from_lists(txs, 8)
+    with gpa.Bitset(ds) as bs:
+        assert bs.n_tx == 4 and bs.n_rows == 7
+        assert list(bs.rows()) == [1, 2, 3, 4, 5, 6, 7]
+        words = bs.export()
+        for cand, tids, bits in vert:
+            if len(cand) == 1:
+                w = int(words[cand[0] - 1, 0])
+                assert "".join("1" if (w >> t) & 1 else "0" for t in range(4)) == bits  # T1 = bit 0
+            for kern in KERNELS:
+                assert bs.count(np.array([cand]), kernel=kern)[0] == bits.count("1")
+    for theta in (1, 2, 3, 4):
+        for kern in (gpa.KERNEL_AUTO, gpa.KERNEL_V0, gpa.KERNEL_PREFIX):
+            res = gpa.mine(ds, min_count=theta, options=gpa.Options(count_kernel=kern), keep_candidates=True)
+            assert_mine_equal(res, oracle.mine_ds(ds, theta))
+
+
+# ---------------------------------------------------------------- bitset layout
+
+@pytest.mark.parametrize("n_tx", [1, 31, 32, 33, 511, 512, 513, 1023, 1024, 1025, 4097])
+def test_bitset_layout_ragged_sizes(n_tx):
+    ds = gen.random_db(n_tx, n_tx, 40, max_len=12, duplicates=True, unsorted=True)
+    with gpa.Bitset(ds) as bs:
+        assert bs.row_pitch_bytes % 128 == 0 and bs.row_pitch_bytes * 8 >= n_tx
+        rows = bs.rows()
+        ref = oracle.mine_ds(ds, 1).levels[0].count
+        assert np.array_equal(bs.item_counts(), ref)
+        assert np.array_equal(rows, np.nonzero(ref)[0])
+        assert np.array_equal(bs.export(), expected_bits(ds, rows, bs.row_pitch_bytes // 4))
+
+
+def test_bitset_row_min_count_and_absent_items():
+    ds = gen.random_db(5, 3000, 64, max_len=10)
+    ref = oracle.mine_ds(ds, 1).levels[0].count
+    with gpa.Bitset(ds, row_min_count=60) as bs:
+        assert np.array_equal(bs.rows(), np.nonzero(ref >= 60)[0])
+        absent = [i for i in range(64) if ref[i] < 60]
+        if absent:
+            with pytest.raises(gpa.GpaError) as e:
+                bs.count(np.array([[absent[0]]]))
+            assert e.value.status == 2  # GPA_ERR_RANGE
+
+
+# ---------------------------------------------------------------- gpa_count vs the literal definition
+
+@pytest.mark.parametrize("kern", KERNELS)
+@pytest.mark.parametrize("k", [1, 2, 3, 5, 8, 12])
+def test_count_random_candidates(kern, k):
+    rng = np.random.default_rng(k * 7 + kern)
+    ds = gen.random_db(100 + k, 20_000 + 37 * k, 24, max_len=16)
+    with gpa.Bitset(ds) as bs:
+        rows = bs.rows()
+        cands = np.array(sorted({tuple(sorted(rng.choice(rows, size=k, replace=False))) for _ in range(300)}),
+                         dtype=np.uint32)
+        cands = cands[rng.permutation(len(cands))]  # any order
+        got = bs.count(cands, kernel=kern)
+        ref = oracle.support_batch(ds.offsets, ds.items, ds.n_items, cands)
+        assert np.array_equal(got, ref.astype(np.uint32))
+
+
+@pytest.mark.parametrize("n_items", [2, 3, 127, 128, 129, 200, 257])
+def test_pairs_kernel_tile_boundaries(n_items):
+    """All pairs of n rows through the tiled kernel, n around the 128-row tile edge."""
+    ds = gen.random_db(n_items, 3000, n_items, max_len=min(n_items, 40), p_empty=0.0)
+    with gpa.Bitset(ds) as bs:
+        rows = bs.rows()
+        pairs = np.array(list(combinations(rows.tolist(), 2)), dtype=np.uint32).reshape(-1, 2)
+        if len(pairs) == 0:
+            return
+        got = bs.count(pairs, kernel=gpa.KERNEL_PAIRS)
+        ref = oracle.support_batch(ds.offsets, ds.items, ds.n_items, pairs)
+        assert np.array_equal(got, ref.astype(np.uint32))
+
+
+def test_count_errors():
+    ds = gen.random_db(9, 500, 10, max_len=5, p_empty=0.0)
+    with gpa.Bitset(ds) as bs:
+        with pytest.raises(gpa.GpaError) as e:
+            bs.count(np.array([[3, 2]]))
+        assert e.value.status == 1
+        with pytest.raises(gpa.GpaError) as e:
+            bs.count(np.array([[1, 10]]))
+        assert e.value.status == 1
+        assert len(bs.count(np.zeros((0, 3), np.uint32))) == 0
+
+
+def test_invalid_csr_rejected():
+    with pytest.raises(gpa.GpaError) as e:
+        gpa.mine(np.array([0, 2, 1], np.uint64), np.array([1, 2], np.uint32), 4, min_count=1)
+    assert e.value.status == 1
+    with pytest.raises(gpa.GpaError) as e:
+        gpa.mine(np.array([0, 2], np.uint64), np.array([1, 9], np.uint32), 4, min_count=1)
+    assert e.value.status == 1
+    with pytest.raises(gpa.GpaError) as e:
+        gpa.mine(np.array([1, 2], np.uint64), np.array([1, 2], np.uint32), 4, min_count=1)
+    assert e.value.status == 1
+
+
+# ---------------------------------------------------------------- gpa_mine vs the oracle (every level)
+
+@pytest.mark.parametrize("seed", range(8))
+def test_mine_random(seed):
+    rng = np.random.default_rng(seed)
+    ds = gen.random_db(seed, int(rng.integers(1, 3000)), int(rng.integers(2, 30)), max_len=12,
+                       duplicates=seed % 2 == 1, unsorted=seed % 3 == 0)
+    theta = int(rng.integers(1, max(2, ds.n_tx // 8)))
+    ref = oracle.mine_ds(ds, theta)
+    for kern in (gpa.KERNEL_AUTO, gpa.KERNEL_V0, gpa.KERNEL_PREFIX):
+        res = gpa.mine(ds, min_count=theta, options=gpa.Options(count_kernel=kern), keep_candidates=True)
+        assert res.n_tx == ds.n_tx
+        assert_mine_equal(res, ref)
+
+
+@pytest.mark.parametrize("name", ["chess", "mushroom", "t40i10d100k", "accidents"])
+def test_mine_configs(name):
+    ds = gen.make(name)
+    theta = oracle.min_count(ds.n_tx, gen.CONFIGS[name].minsup)
+    assert gpa.min_count(ds.n_tx, gen.CONFIGS[name].minsup) == theta
+    ref = oracle.mine_ds(ds, theta)
+    kernels = [gpa.KERNEL_AUTO, gpa.KERNEL_PREFIX] + ([gpa.KERNEL_V0] if name in ("chess", "mushroom") else [])
+    for kern in kernels:
+        res = gpa.mine(ds, min_count=theta, options=gpa.Options(count_kernel=kern), keep_candidates=True)
+        assert_mine_equal(res, ref)
+
+
+def test_mine_device_input_equals_host_input():
+    import torch
+    ds = gen.make("mushroom")
+    theta = oracle.min_count(ds.n_tx, "0.20")
+    off = torch.from_numpy(ds.offsets.view(np.int64)).cuda()
+    it = torch.from_numpy(ds.items.view(np.int32)).cuda()
+    a = gpa.mine(off, it, ds.n_items, min_count=theta, keep_candidates=True)
+    b = gpa.mine(ds, min_count=theta, keep_candidates=True)
+    for la, lb in zip(a.levels, b.levels):
+        assert np.array_equal(la.cand, lb.cand) and np.array_equal(la.counts, lb.counts)
+    # and on a caller-provided torch stream
+    s = torch.cuda.Stream()
+    c = gpa.mine(off, it, ds.n_items, min_count=theta, options=gpa.Options(stream=s.cuda_stream))
+    assert c.frequent() == b.frequent()
+
+
+def test_mine_max_k_and_degenerate():
+    ds = gen.make("chess")
+    theta = oracle.min_count(ds.n_tx, "0.90")
+    res = gpa.mine(ds, min_count=theta, options=gpa.Options(max_k=3))
+    assert len(res.levels) == 3
+    ref = oracle.mine_ds(ds, theta)
+    for k in (1, 2, 3):
+        fi, fs = res.frequent(k)
+        keep = ref.levels[k - 1].count >= theta
+        assert np.array_equal(fi, ref.levels[k - 1].cand[keep]) and np.array_equal(fs, ref.levels[k - 1].count[keep])
+    # theta above every count: only generation 1, nothing frequent
+    res = gpa.mine(ds, min_count=ds.n_tx + 1)
+    assert len(res.levels) == 1 and res.frequent() == {}
+    # empty database
+    res = gpa.mine(np.zeros(1, np.uint64), np.zeros(0, np.uint32), 5, min_count=1)
+    assert res.frequent() == {} and res.n_tx == 0
+    # replicated transaction: all 2^L - 1 subsets, support N
+    T = [1, 4, 6, 9, 12, 13]
+    rep = gen.from_lists([T] * 700, 16)
+    F = gpa.mine(rep, min_count=700).frequent()
+    assert len(F) == 2 ** len(T) - 1 and set(F.values()) == {700}
+
+
+# ---------------------------------------------------------------- full-size bench configuration (sampled)
+
+def test_t40i10d10m_full_size_sampled():
+    """BASELINE.json's largest config at full size in the bench's launch configuration: every
+    level's counts on sampled candidates against the literal definition, level 1 against
+    numpy.bincount, and invariants (|C_2| = C(|L_1|, 2), downward closure of F)."""
+    name = "t40i10d10m"
+    ds = gen.make(name)
+    theta = oracle.min_count(ds.n_tx, gen.CONFIGS[name].minsup)
+    res = gpa.mine(ds, min_count=theta, keep_candidates=True)
+    c1 = np.bincount(ds.items, minlength=ds.n_items)
+    assert np.array_equal(res.levels[0].counts, c1)
+    n1 = int((c1 >= theta).sum())
+    assert res.levels[1].n_cand == n1 * (n1 - 1) // 2
+    F = res.frequent()
+    for X, s in F.items():
+        if len(X) > 1:
+            for Y in combinations(X, len(X) - 1):
+                assert F[Y] >= s
+    rng = np.random.default_rng(5)
+    sample, expect = [], []
+    for lv in res.levels[1:]:
+        # frequent and infrequent candidates alike, plus the extremes of the level
+        idx = set(rng.choice(lv.n_cand, size=min(6, lv.n_cand), replace=False).tolist())
+        idx |= {int(np.argmax(lv.counts)), int(np.argmin(lv.counts))}
+        for i in sorted(idx):
+            sample.append(lv.cand[i])
+            expect.append(lv.counts[i])
+    for k in sorted({len(c) for c in sample}):
+        cs = np.array([c for c in sample if len(c) == k], dtype=np.uint32)
+        ex = np.array([e for c, e in zip(sample, expect) if len(c) == k], dtype=np.uint64)
+        lit = oracle.support_batch(ds.offsets, ds.items, ds.n_items, cs)
+        assert np.array_equal(lit, ex), k
