@@ -94,10 +94,11 @@ typedef struct {
 } gpa_tx_csr;
 
 /* Counting kernel selection. */
-#define GPA_KERNEL_AUTO 0u     /* PAIRS for k = 2, PREFIX for k >= 3 */
+#define GPA_KERNEL_AUTO 0u     /* PAIRS for k = 2, TRIE for 3 <= k <= 16, PREFIX above */
 #define GPA_KERNEL_V0 1u       /* the paper's design: one CTA per candidate, AND of all k rows */
 #define GPA_KERNEL_PREFIX 2u   /* prefix-staged streaming: (k-1)-prefix AND held on chip, siblings streamed */
 #define GPA_KERNEL_PAIRS 3u    /* k = 2 only: TMA-tiled AND-popcount "Gram" tile kernel */
+#define GPA_KERNEL_TRIE 4u     /* 2 <= k <= 16: transaction-tiled trie walk, rows staged in shared memory */
 
 #define GPA_KEEP_CANDIDATES 1u /* gpa_mine: keep every generation's (C_k, counts), not only F */
 

@@ -38,6 +38,25 @@ uint64_t launch_count_prefix(const uint32_t* rows, uint64_t pitch_words, const u
                              const uint32_t* ext_rows, const PrefixTask* tasks, uint32_t n_tasks, uint32_t* counts,
                              cudaStream_t stream);
 
+// Transaction-tiled trie walk for generations k in [2, kTrieMaxK] (count_trie.cu).  Candidates
+// (lexicographic) are cut into blocks of <= kTrieMaxCand candidates touching <= kTrieMaxRows rows.
+constexpr uint32_t kTrieMaxK = 16;
+constexpr uint32_t kTrieMaxRows = 64;
+constexpr uint32_t kTrieMaxCand = 256;
+struct TrieBlock {
+  uint32_t cand_begin;   // first candidate (global index)
+  uint32_t n_cand;       // <= kTrieMaxCand
+  uint32_t row_begin;    // into block_rows
+  uint32_t n_rows;       // <= kTrieMaxRows
+};
+uint32_t trie_stripes(uint64_t pitch_words);
+// cand_lrows[c]: byte d = block-local row of item d; cand_lcp[c]: items shared with candidate c-1
+// (0 for the first candidate of every 32-candidate warp chunk).  counts must be zeroed.
+uint64_t launch_count_trie(uint32_t k, const uint32_t* rows, uint64_t pitch_words, const TrieBlock* blocks,
+                           const uint32_t* block_rows, const uint4* cand_lrows, const uint8_t* cand_lcp,
+                           uint32_t n_blocks, uint32_t max_rows, uint32_t n_parts, uint32_t* counts,
+                           cudaStream_t stream);
+
 // k = 2 TMA-tiled kernel: all pairs (a < b) of the n_rows rows; counts[pair_index] must be zeroed.
 // tmap: opaque 128-byte CUtensorMap built by make_pairs_tensor_map.
 bool make_pairs_tensor_map(void* tmap128, const uint32_t* rows, uint32_t n_rows, uint64_t pitch_words);

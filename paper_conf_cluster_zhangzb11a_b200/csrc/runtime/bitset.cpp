@@ -27,7 +27,7 @@ float event_ms(cudaEvent_t a, cudaEvent_t b) {
 }
 
 void validate_options(const gpa_options& o) {
-  GPA_REQUIRE(o.count_kernel <= GPA_KERNEL_PAIRS, GPA_ERR_INVALID, "unknown count_kernel %u", o.count_kernel);
+  GPA_REQUIRE(o.count_kernel <= GPA_KERNEL_TRIE, GPA_ERR_INVALID, "unknown count_kernel %u", o.count_kernel);
   GPA_REQUIRE(o.max_k <= GPA_MAX_K, GPA_ERR_INVALID, "max_k %u > GPA_MAX_K", o.max_k);
   GPA_REQUIRE(!o.reserved[0] && !o.reserved[1] && !o.reserved[2], GPA_ERR_INVALID, "reserved option fields must be 0");
 }
@@ -168,6 +168,10 @@ void bitset_free(gpa_bitset* bs) {
   bs->d_ext.reset();
   bs->d_flat.reset();
   bs->d_tasks.reset();
+  bs->d_tblocks.reset();
+  bs->d_trows.reset();
+  bs->d_lrows.reset();
+  bs->d_lcp.reset();
   if (bs->stream) cudaStreamSynchronize(bs->stream);
   if (bs->ev0) cudaEventDestroy(bs->ev0);
   if (bs->ev1) cudaEventDestroy(bs->ev1);
@@ -204,6 +208,86 @@ void count_flat_v0(gpa_bitset* bs, const std::vector<uint32_t>& flat, uint32_t k
   finish_counts(bs, M, st);
 }
 
+// Transaction-tiled trie walk: cut the lexicographic candidate list into blocks (<= kTrieMaxCand
+// candidates, <= kTrieMaxRows distinct rows), give every candidate its block-local row bytes and
+// its shared-prefix length with the previous candidate of the same 32-candidate warp chunk.
+void count_trie_batch(gpa_bitset* bs, const GroupedBatch& b, CountStats* st) {
+  cudaStream_t s = bs->stream;
+  const uint32_t k = b.k, km1 = k - 1;
+  const uint64_t M = b.size(), G = b.groups();
+  std::vector<TrieBlock> blocks;
+  std::vector<uint32_t> brows;
+  std::vector<uint4> lrows(M);
+  std::vector<uint8_t> lcp(M);
+  std::vector<uint32_t> stamp(bs->n_rows, UINT32_MAX);
+  std::vector<uint8_t> local(bs->n_rows, 0);
+  std::vector<uint32_t> cur(k), prev(k);
+  uint32_t max_rows = 0;
+  TrieBlock blk{0, 0, 0, 0};
+  auto close_block = [&]() {
+    if (blk.n_cand) {
+      blocks.push_back(blk);
+      max_rows = std::max(max_rows, blk.n_rows);
+    }
+    blk = TrieBlock{blk.cand_begin + blk.n_cand, 0, (uint32_t)brows.size(), 0};
+  };
+  uint64_t c = 0;
+  for (uint64_t g = 0; g < G; ++g) {
+    for (uint64_t j = b.ext_off[g]; j < b.ext_off[g + 1]; ++j, ++c) {
+      std::copy(b.prefix.begin() + g * km1, b.prefix.begin() + (g + 1) * km1, cur.begin());
+      cur[km1] = b.ext[j];
+      const uint32_t id = (uint32_t)blocks.size();
+      uint32_t fresh = 0;
+      for (uint32_t d = 0; d < k; ++d) fresh += stamp[cur[d]] != id;
+      // duplicate rows inside one candidate cannot happen (strictly increasing)
+      if (blk.n_cand == kTrieMaxCand || blk.n_rows + fresh > kTrieMaxRows) {
+        close_block();
+        fresh = k;
+      }
+      const uint32_t id2 = (uint32_t)blocks.size();
+      uint8_t bytes[16] = {0};
+      for (uint32_t d = 0; d < k; ++d) {
+        const uint32_t r = cur[d];
+        if (stamp[r] != id2) {
+          stamp[r] = id2;
+          local[r] = (uint8_t)blk.n_rows++;
+          brows.push_back(r);
+        }
+        bytes[d] = local[r];
+      }
+      memcpy(&lrows[c], bytes, 16);
+      uint32_t l = 0;
+      if (blk.n_cand % 32 != 0)
+        while (l < km1 && cur[l] == prev[l]) ++l;
+      lcp[c] = (uint8_t)l;
+      ++blk.n_cand;
+      std::swap(prev, cur);
+    }
+  }
+  close_block();
+  const uint32_t n_blocks = (uint32_t)blocks.size();
+  const uint32_t n_stripes = trie_stripes(bs->pitch_words);
+  uint32_t n_parts = std::max<uint32_t>(1, n_stripes / 64);
+  const uint32_t want = (uint32_t)bs->n_sms * 2 * 3;
+  if ((uint64_t)n_blocks * n_parts < want) n_parts = std::min<uint32_t>(n_stripes, (want + n_blocks - 1) / n_blocks);
+  bs->d_tblocks.ensure(n_blocks, s);
+  bs->d_trows.ensure(std::max<size_t>(brows.size(), 1), s);
+  bs->d_lrows.ensure(M, s);
+  bs->d_lcp.ensure(M, s);
+  bs->d_counts.ensure(M, s);
+  GPA_CUDA(cudaMemcpyAsync(bs->d_tblocks.p, blocks.data(), n_blocks * sizeof(TrieBlock), cudaMemcpyHostToDevice, s));
+  GPA_CUDA(cudaMemcpyAsync(bs->d_trows.p, brows.data(), brows.size() * sizeof(uint32_t), cudaMemcpyHostToDevice, s));
+  GPA_CUDA(cudaMemcpyAsync(bs->d_lrows.p, lrows.data(), M * sizeof(uint4), cudaMemcpyHostToDevice, s));
+  GPA_CUDA(cudaMemcpyAsync(bs->d_lcp.p, lcp.data(), M, cudaMemcpyHostToDevice, s));
+  GPA_CUDA(cudaMemsetAsync(bs->d_counts.p, 0, M * sizeof(uint32_t), s));
+  GPA_CUDA(cudaEventRecord(bs->ev0, s));
+  if (bs->n_rows)
+    launch_count_trie(k, bs->rows.p, bs->pitch_words, bs->d_tblocks.p, bs->d_trows.p, bs->d_lrows.p, bs->d_lcp.p,
+                      n_blocks, max_rows, n_parts, bs->d_counts.p, s);
+  if (st) { st->kernel = GPA_KERNEL_TRIE; st->launches = 1; }
+  finish_counts(bs, M, st);
+}
+
 }  // namespace
 
 void count_grouped(gpa_bitset* bs, const GroupedBatch& b, uint32_t kernel, CountStats* st) {
@@ -211,8 +295,15 @@ void count_grouped(gpa_bitset* bs, const GroupedBatch& b, uint32_t kernel, Count
   const uint64_t M = b.size(), G = b.groups();
   const uint32_t km1 = b.k - 1;
   if (M == 0) return;
-  if (kernel == GPA_KERNEL_AUTO) kernel = GPA_KERNEL_PREFIX;
-  if (kernel == GPA_KERNEL_PAIRS) kernel = GPA_KERNEL_PREFIX;  // grouped batches use the prefix kernel
+  if (kernel == GPA_KERNEL_AUTO || kernel == GPA_KERNEL_PAIRS)  // grouped batches: trie walk, else prefix
+    kernel = (b.k >= 2 && b.k <= kTrieMaxK) ? GPA_KERNEL_TRIE : GPA_KERNEL_PREFIX;
+  if (kernel == GPA_KERNEL_TRIE) {
+    if (b.k >= 2 && b.k <= kTrieMaxK) {
+      count_trie_batch(bs, b, st);
+      return;
+    }
+    kernel = GPA_KERNEL_PREFIX;
+  }
   if (kernel == GPA_KERNEL_V0 || km1 == 0) {
     std::vector<uint32_t> flat(M * b.k);
     for (uint64_t g = 0; g < G; ++g)
@@ -355,7 +446,7 @@ extern "C" gpa_status gpa_count(gpa_bitset* bs, const uint32_t* cand, uint32_t k
   return gpa::guard([&] {
     GPA_REQUIRE(bs, GPA_ERR_INVALID, "bitset is NULL");
     GPA_REQUIRE(k >= 1 && k <= GPA_MAX_K, GPA_ERR_INVALID, "k must be in [1, %u]", GPA_MAX_K);
-    GPA_REQUIRE(kernel <= GPA_KERNEL_PAIRS, GPA_ERR_INVALID, "unknown kernel %u", kernel);
+    GPA_REQUIRE(kernel <= GPA_KERNEL_TRIE, GPA_ERR_INVALID, "unknown kernel %u", kernel);
     if (M == 0) return;
     GPA_REQUIRE(cand && counts_out, GPA_ERR_INVALID, "NULL argument");
     GPA_REQUIRE(M <= (UINT64_MAX / 8) / k && M < (1ull << 32), GPA_ERR_INVALID, "M * k overflows");
@@ -377,8 +468,9 @@ extern "C" gpa_status gpa_count(gpa_bitset* bs, const uint32_t* cand, uint32_t k
     uint32_t kern = kernel == GPA_KERNEL_AUTO ? bs->opt.count_kernel : kernel;
     if (k == 1) kern = GPA_KERNEL_V0;
     if (kern == GPA_KERNEL_AUTO)
-      kern = (k == 2 && (double)M * 8 >= (double)bs->n_rows * bs->n_rows) ? GPA_KERNEL_PAIRS : GPA_KERNEL_PREFIX;
-    if (kern == GPA_KERNEL_PAIRS && k != 2) kern = GPA_KERNEL_PREFIX;
+      kern = (k == 2 && (double)M * 8 >= (double)bs->n_rows * bs->n_rows) ? GPA_KERNEL_PAIRS
+             : (k <= gpa::kTrieMaxK ? GPA_KERNEL_TRIE : GPA_KERNEL_PREFIX);
+    if (kern == GPA_KERNEL_PAIRS && k != 2) kern = k <= gpa::kTrieMaxK ? GPA_KERNEL_TRIE : GPA_KERNEL_PREFIX;
     if (kern == GPA_KERNEL_PAIRS) {
       gpa::count_all_pairs(bs, GPA_KERNEL_PAIRS, nullptr);
       const uint64_t n = bs->n_rows, P = n * (n - 1) / 2;
@@ -407,7 +499,7 @@ extern "C" gpa_status gpa_count(gpa_bitset* bs, const uint32_t* cand, uint32_t k
       GPA_CUDA(cudaStreamSynchronize(bs->stream));
       return;
     }
-    // PREFIX: group by (k-1)-prefix (sort candidate indices lexicographically)
+    // PREFIX / TRIE: group by (k-1)-prefix (sort candidate indices lexicographically)
     std::vector<uint64_t> order(M);
     std::iota(order.begin(), order.end(), 0);
     std::sort(order.begin(), order.end(), [&](uint64_t a, uint64_t b) {
@@ -428,7 +520,7 @@ extern "C" gpa_status gpa_count(gpa_bitset* bs, const uint32_t* cand, uint32_t k
       b.ext[i] = rows[m * k + k - 1];
     }
     b.ext_off.push_back(M);
-    gpa::count_grouped(bs, b, GPA_KERNEL_PREFIX, nullptr);
+    gpa::count_grouped(bs, b, kern, nullptr);
     std::vector<uint32_t> sorted(M);
     GPA_CUDA(cudaMemcpyAsync(sorted.data(), bs->d_counts.p, M * 4, cudaMemcpyDeviceToHost, bs->stream));
     GPA_CUDA(cudaStreamSynchronize(bs->stream));

@@ -140,6 +140,10 @@ struct gpa_bitset {
   // counting workspace (grow-only)
   gpa::DBuf<uint32_t> d_counts, d_prefix, d_ext, d_flat;
   gpa::DBuf<gpa::PrefixTask> d_tasks;
+  gpa::DBuf<gpa::TrieBlock> d_tblocks;
+  gpa::DBuf<uint32_t> d_trows;
+  gpa::DBuf<uint4> d_lrows;
+  gpa::DBuf<uint8_t> d_lcp;
   cudaEvent_t ev0 = nullptr, ev1 = nullptr, ev2 = nullptr;
   double build_ms[3] = {0, 0, 0};      // upload, histogram, bitset
 };

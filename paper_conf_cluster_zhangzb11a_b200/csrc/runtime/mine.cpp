@@ -38,38 +38,44 @@ double now_ms() {
   return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now().time_since_epoch()).count();
 }
 
-// Record generation k: candidates are given in ROW ids (M x k, lexicographic) or, for k = 2,
-// implicitly as all pairs of n rows.  Returns L_k in row ids.
-std::vector<uint32_t> record_level(gpa_result* R, const gpa_bitset* bs, uint32_t k, const std::vector<uint32_t>* cand_rows,
-                                   uint64_t M, const std::vector<uint32_t>& counts, bool keep, uint64_t* n_freq) {
+// Record generation k.  Candidates are the grouped batch b (k >= 3) or, for k = 2 (b == nullptr),
+// all pairs of the n rows in lexicographic order.  Returns L_k in row ids (lexicographic).
+std::vector<uint32_t> record_level(gpa_result* R, const gpa_bitset* bs, uint32_t k, const GroupedBatch* b, uint64_t M,
+                                   const std::vector<uint32_t>& counts, bool keep, uint64_t* n_freq) {
   gpa_level_data lv;
   lv.k = k;
   lv.n_cand = M;
   lv.kept = keep;
   std::vector<uint32_t> Lk;
   const auto& ior = bs->item_of_row;
-  auto row_of_cand = [&](uint64_t m, uint32_t j, uint64_t& a, uint64_t& b) -> uint32_t {
-    if (cand_rows) return (*cand_rows)[m * k + j];
-    return j == 0 ? (uint32_t)a : (uint32_t)b;
-  };
-  uint64_t a = 0, b = 1;  // pair cursor for the implicit k = 2 order
-  const uint64_t n = bs->n_rows;
+  const uint32_t theta = (uint32_t)R->min_count;
   if (keep) {
     lv.cand_items.resize(M * k);
     lv.cand_counts = counts;
   }
-  for (uint64_t m = 0; m < M; ++m) {
-    if (keep)
-      for (uint32_t j = 0; j < k; ++j) lv.cand_items[m * k + j] = ior[row_of_cand(m, j, a, b)];
-    if (counts[m] >= R->min_count) {
-      for (uint32_t j = 0; j < k; ++j) {
-        const uint32_t r = row_of_cand(m, j, a, b);
-        Lk.push_back(r);
-        lv.freq_items.push_back(ior[r]);
-      }
+  auto emit = [&](uint64_t m, const uint32_t* pre, uint32_t last) {
+    if (keep) {
+      uint32_t* dst = lv.cand_items.data() + m * k;
+      for (uint32_t j = 0; j + 1 < k; ++j) dst[j] = ior[pre[j]];
+      dst[k - 1] = ior[last];
+    }
+    if (counts[m] >= theta) {
+      Lk.insert(Lk.end(), pre, pre + (k - 1));
+      Lk.push_back(last);
+      for (uint32_t j = 0; j + 1 < k; ++j) lv.freq_items.push_back(ior[pre[j]]);
+      lv.freq_items.push_back(ior[last]);
       lv.freq_support.push_back(counts[m]);
     }
-    if (!cand_rows && ++b == n) { ++a; b = a + 1; }
+  };
+  if (b) {
+    const uint64_t G = b->groups();
+    for (uint64_t g = 0; g < G; ++g)
+      for (uint64_t j = b->ext_off[g]; j < b->ext_off[g + 1]; ++j) emit(j, b->prefix.data() + g * (k - 1), b->ext[j]);
+  } else {
+    const uint64_t n = bs->n_rows;
+    uint64_t m = 0;
+    for (uint32_t a = 0; a + 1 < n; ++a)
+      for (uint32_t c = a + 1; c < n; ++c, ++m) emit(m, &a, c);
   }
   lv.n_freq = lv.freq_support.size();
   *n_freq = lv.n_freq;
@@ -157,18 +163,8 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     double t2 = now_ms();
     R->phase_ms[GPA_PHASE_COUNT] += t2 - t1;
 
-    std::vector<uint32_t> cand_rows;
-    if (k > 2) {
-      cand_rows.resize(M * k);
-      for (uint64_t g = 0; g < G; ++g)
-        for (uint64_t j = batch.ext_off[g]; j < batch.ext_off[g + 1]; ++j) {
-          std::copy(batch.prefix.begin() + g * (k - 1), batch.prefix.begin() + (g + 1) * (k - 1),
-                    cand_rows.begin() + j * k);
-          cand_rows[j * k + k - 1] = batch.ext[j];
-        }
-    }
     uint64_t n_freq = 0;
-    L = record_level(R, bs, k, k > 2 ? &cand_rows : nullptr, M, counts, keep, &n_freq);
+    L = record_level(R, bs, k, k > 2 ? &batch : nullptr, M, counts, keep, &n_freq);
     nL = n_freq;
     gpa_level_stats& st = R->levels.back().stats;
     st.n_cand = M;

@@ -16,7 +16,7 @@ import paper_conf_cluster_zhangzb11a_b200 as gpa
 
 pytestmark = pytest.mark.gpu
 
-KERNELS = [gpa.KERNEL_V0, gpa.KERNEL_PREFIX, gpa.KERNEL_PAIRS]
+KERNELS = [gpa.KERNEL_V0, gpa.KERNEL_PREFIX, gpa.KERNEL_PAIRS, gpa.KERNEL_TRIE]
 
 
 def expected_bits(ds, item_of_row, pitch_words):
@@ -55,7 +55,7 @@ def test_fig2_bitset_and_supports(fig2):
             for kern in KERNELS:
                 assert bs.count(np.array([cand]), kernel=kern)[0] == bits.count("1")
     for theta in (1, 2, 3, 4):
-        for kern in (gpa.KERNEL_AUTO, gpa.KERNEL_V0, gpa.KERNEL_PREFIX):
+        for kern in (gpa.KERNEL_AUTO, gpa.KERNEL_V0, gpa.KERNEL_PREFIX, gpa.KERNEL_TRIE):
             res = gpa.mine(ds, min_count=theta, options=gpa.Options(count_kernel=kern), keep_candidates=True)
             assert_mine_equal(res, oracle.mine_ds(ds, theta))
 
@@ -89,7 +89,7 @@ def test_bitset_row_min_count_and_absent_items():
 # ---------------------------------------------------------------- gpa_count vs the literal definition
 
 @pytest.mark.parametrize("kern", KERNELS)
-@pytest.mark.parametrize("k", [1, 2, 3, 5, 8, 12])
+@pytest.mark.parametrize("k", [1, 2, 3, 5, 8, 12, 16, 20])
 def test_count_random_candidates(kern, k):
     rng = np.random.default_rng(k * 7 + kern)
     ds = gen.random_db(100 + k, 20_000 + 37 * k, 24, max_len=16)
@@ -98,6 +98,22 @@ def test_count_random_candidates(kern, k):
         cands = np.array(sorted({tuple(sorted(rng.choice(rows, size=k, replace=False))) for _ in range(300)}),
                          dtype=np.uint32)
         cands = cands[rng.permutation(len(cands))]  # any order
+        got = bs.count(cands, kernel=kern)
+        ref = oracle.support_batch(ds.offsets, ds.items, ds.n_items, cands)
+        assert np.array_equal(got, ref.astype(np.uint32))
+
+
+@pytest.mark.parametrize("kern", [gpa.KERNEL_TRIE, gpa.KERNEL_PREFIX])
+@pytest.mark.parametrize("k", [3, 4, 7])
+def test_count_many_rows_per_block(kern, k):
+    """Random candidates over 300 items: trie blocks are cut at 64 distinct rows / 256 candidates,
+    warps at 32 candidates; counts over a ragged 70,001-transaction axis (stripe tail)."""
+    rng = np.random.default_rng(k)
+    ds = gen.random_db(77 + k, 70_001, 300, max_len=60, p_empty=0.05)
+    with gpa.Bitset(ds) as bs:
+        rows = bs.rows()
+        cands = np.array(sorted({tuple(sorted(rng.choice(rows[:120] if i % 2 else rows, size=k, replace=False)))
+                                 for i in range(1500)}), dtype=np.uint32)
         got = bs.count(cands, kernel=kern)
         ref = oracle.support_batch(ds.offsets, ds.items, ds.n_items, cands)
         assert np.array_equal(got, ref.astype(np.uint32))
@@ -150,7 +166,7 @@ def test_mine_random(seed):
                        duplicates=seed % 2 == 1, unsorted=seed % 3 == 0)
     theta = int(rng.integers(1, max(2, ds.n_tx // 8)))
     ref = oracle.mine_ds(ds, theta)
-    for kern in (gpa.KERNEL_AUTO, gpa.KERNEL_V0, gpa.KERNEL_PREFIX):
+    for kern in (gpa.KERNEL_AUTO, gpa.KERNEL_V0, gpa.KERNEL_PREFIX, gpa.KERNEL_TRIE):
         res = gpa.mine(ds, min_count=theta, options=gpa.Options(count_kernel=kern), keep_candidates=True)
         assert res.n_tx == ds.n_tx
         assert_mine_equal(res, ref)
@@ -163,6 +179,7 @@ def test_mine_configs(name):
     assert gpa.min_count(ds.n_tx, gen.CONFIGS[name].minsup) == theta
     ref = oracle.mine_ds(ds, theta)
     kernels = [gpa.KERNEL_AUTO, gpa.KERNEL_PREFIX] + ([gpa.KERNEL_V0] if name in ("chess", "mushroom") else [])
+    # AUTO = pairs (k = 2) + trie (k >= 3); PREFIX = prefix kernel for every k
     for kern in kernels:
         res = gpa.mine(ds, min_count=theta, options=gpa.Options(count_kernel=kern), keep_candidates=True)
         assert_mine_equal(res, ref)

@@ -1,0 +1,93 @@
+"""Host-side logic of the GPU path, tested on CPU: the library's own join + prune candidate
+generation (runtime/candgen.cpp, compiled here into a test shim) against the oracle's
+independent implementation and against the definition; and the grouping invariants the counting
+kernels rely on (lexicographic order, groups = (k-1)-prefix runs)."""
+import ctypes
+import os
+import subprocess
+from itertools import combinations
+
+import numpy as np
+import pytest
+
+import gen
+import oracle
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+CSRC = os.path.join(ROOT, "paper_conf_cluster_zhangzb11a_b200", "csrc")
+
+
+@pytest.fixture(scope="module")
+def shim(tmp_path_factory):
+    import nvidia.nccl
+    nccl = list(nvidia.nccl.__path__)[0]
+    out = tmp_path_factory.mktemp("shim") / "libcandgen_shim.so"
+    subprocess.check_call(["g++", "-O2", "-std=c++17", "-shared", "-fPIC", "-pthread", "-I", CSRC, "-I",
+                           os.path.join(ROOT, "include"), "-I", "/usr/local/cuda/include", "-I",
+                           os.path.join(nccl, "include"), os.path.join(ROOT, "tests", "cpp", "candgen_shim.cpp"),
+                           os.path.join(CSRC, "runtime", "candgen.cpp"), "-o", str(out)])
+    lib = ctypes.CDLL(str(out))
+    lib.shim_candgen.restype = ctypes.c_int
+    return lib
+
+
+def run_shim(lib, L):
+    L = np.ascontiguousarray(L, dtype=np.uint32)
+    n, km1 = L.shape
+    cap = max(16, n * n)
+    pre = np.zeros(cap * km1 + 1, np.uint32)
+    off = np.zeros(cap + 2, np.uint64)
+    ext = np.zeros(cap + 1, np.uint32)
+    ng, nc = ctypes.c_uint64(), ctypes.c_uint64()
+    rc = lib.shim_candgen(L.ctypes.data_as(ctypes.c_void_p), ctypes.c_uint64(n), ctypes.c_uint32(km1),
+                          pre.ctypes.data_as(ctypes.c_void_p), off.ctypes.data_as(ctypes.c_void_p),
+                          ext.ctypes.data_as(ctypes.c_void_p), ctypes.c_uint64(cap), ctypes.byref(ng), ctypes.byref(nc))
+    assert rc == 0
+    G, M = ng.value, nc.value
+    pre = pre[: G * km1].reshape(G, km1)
+    off = off[: G + 1]
+    ext = ext[:M]
+    cands = []
+    for g in range(G):
+        assert off[g + 1] > off[g]  # groups are non-empty
+        for j in range(int(off[g]), int(off[g + 1])):
+            cands.append(tuple(int(x) for x in pre[g]) + (int(ext[j]),))
+    return cands, pre, off
+
+
+@pytest.mark.parametrize("seed", range(10))
+def test_candgen_matches_oracle_and_definition(shim, seed):
+    rng = np.random.default_rng(seed)
+    n, km1 = 10, int(rng.integers(1, 5))
+    allsets = list(combinations(range(n), km1))
+    L = sorted(s for s in allsets if rng.random() < 0.6)
+    if not L:
+        return
+    got, pre, off = run_shim(shim, np.array(L, dtype=np.uint32).reshape(-1, km1))
+    ref = [tuple(map(int, r)) for r in oracle.candgen(np.array(L, dtype=np.uint32).reshape(-1, km1))]
+    Ls = set(L)
+    defn = [X for X in combinations(range(n), km1 + 1) if all(S in Ls for S in combinations(X, km1))]
+    assert got == ref == defn
+    # groups are distinct (k-1)-prefixes in increasing order
+    assert [tuple(p) for p in pre.tolist()] == sorted(set(tuple(p) for p in pre.tolist()))
+
+
+@pytest.mark.parametrize("name", ["mushroom", "chess"])
+def test_candgen_real_levels(shim, name):
+    """Every generation of a real mining run, incl. the threaded path (large L)."""
+    ds = gen.make(name)
+    theta = oracle.min_count(ds.n_tx, gen.CONFIGS[name].minsup)
+    r = oracle.mine_ds(ds, theta)
+    for lv, nxt in zip(r.levels[1:], r.levels[2:]):
+        L = lv.cand[lv.count >= theta]
+        got, _, _ = run_shim(shim, L)
+        assert got == [tuple(map(int, x)) for x in nxt.cand]
+
+
+def test_candgen_threaded_large(shim):
+    """A large L_2 (~20k pairs) forces the multi-threaded split; result must equal the oracle's."""
+    rng = np.random.default_rng(3)
+    pairs = sorted({tuple(sorted(rng.choice(400, 2, replace=False))) for _ in range(20000)})
+    L = np.array(pairs, dtype=np.uint32)
+    got, _, _ = run_shim(shim, L)
+    assert got == [tuple(map(int, x)) for x in oracle.candgen(L)]
