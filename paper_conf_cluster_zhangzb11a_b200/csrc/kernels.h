@@ -41,7 +41,8 @@ uint64_t launch_count_prefix(const uint32_t* rows, uint64_t pitch_words, const u
 // Transaction-tiled trie walk for generations k in [2, kTrieMaxK] (count_trie.cu).  Candidates
 // (lexicographic) are cut into blocks of <= kTrieMaxCand candidates touching <= kTrieMaxRows rows.
 constexpr uint32_t kTrieMaxK = 16;
-constexpr uint32_t kTrieMaxRows = 64;
+constexpr uint32_t kTrieWideMaxK = 8;    // k <= 8: 8 words per lane (256-word stripes), <= 32 rows / block
+constexpr uint32_t kTrieMaxRows = 64;    // k > 8: 4 words per lane (128-word stripes), <= 64 rows / block
 constexpr uint32_t kTrieMaxCand = 256;
 struct TrieBlock {
   uint32_t cand_begin;   // first candidate (global index)
@@ -49,9 +50,11 @@ struct TrieBlock {
   uint32_t row_begin;    // into block_rows
   uint32_t n_rows;       // <= kTrieMaxRows
 };
-uint32_t trie_stripes(uint64_t pitch_words);
+uint32_t trie_max_rows(uint32_t k);
+uint32_t trie_stripes(uint32_t k, uint64_t pitch_words);
 // cand_lrows[c]: byte d = block-local row of item d; cand_lcp[c]: items shared with candidate c-1
-// (0 for the first candidate of every 32-candidate warp chunk).  counts must be zeroed.
+// (0 for the first candidate of every warp chunk: a block's n candidates are split into chunks of
+// ceil(n / 8)).  counts must be zeroed.
 uint64_t launch_count_trie(uint32_t k, const uint32_t* rows, uint64_t pitch_words, const TrieBlock* blocks,
                            const uint32_t* block_rows, const uint4* cand_lrows, const uint8_t* cand_lcp,
                            uint32_t n_blocks, uint32_t max_rows, uint32_t n_parts, uint32_t* counts,

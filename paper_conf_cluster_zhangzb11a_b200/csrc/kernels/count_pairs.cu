@@ -13,7 +13,10 @@
 //     complete_tx); a diagonal tile loads one box and uses it as both operands;
 //   * 8 consumer warps: thread (tx, ty) owns the 8 x 8 pairs (ty + 16 i, tx + 16 j); per
 //     16-byte slot it loads 8 A and 8 B fragments (LDS.128, conflict-free thanks to the
-//     swizzle) and does 64 x 4 AND + POPC + add into 64 register accumulators;
+//     swizzle) and does 64 x 4 AND + popcount + add into 64 register accumulators; the 4 words
+//     of a slot go through one carry-save adder so 3 POPC count 4 words (the XU pipe that runs
+//     POPC is 4x narrower than the ALU pipe that runs LOP3); diagonal tiles skip the
+//     micro-pairs that lie entirely below the diagonal;
 //   * epilogue: one atomicAdd per (CTA, pair a < b) into the lexicographic pair index.
 // Each loaded word feeds 128 pair-words, so the kernel is bound by the POPC pipe (16 / clk /
 // SM, measured: profiles/r01_microbench_popc.txt), not by HBM: DRAM traffic is about
@@ -141,8 +144,15 @@ __global__ void __launch_bounds__(kThreads, 1) count_pairs_kernel(const __grid_c
       for (int j = 0; j < 8; ++j) {
         const uint4 b = lds128(B + (tx + 16 * j) * 128 + ((q ^ swb) << 4));
 #pragma unroll
-        for (int i = 0; i < 8; ++i)
-          acc[i][j] += (__popc(a[i].x & b.x) + __popc(a[i].y & b.y)) + (__popc(a[i].z & b.z) + __popc(a[i].w & b.w));
+        for (int i = 0; i < 8; ++i) {
+          // diagonal tile: micro-pairs with i > j have a = ty + 16i > b = tx + 16j for every thread
+          if (diag && i > j) continue;
+          // carry-save adder over 3 of the 4 AND words: popc(x)+popc(y)+popc(z) = popc(x^y^z) + 2 popc(maj(x,y,z));
+          // 3 POPC (XU pipe, 16/clk/SM) instead of 4, paid with 2 LOP3 (ALU pipe, 64/clk/SM)
+          const uint32_t x = a[i].x & b.x, y = a[i].y & b.y, z = a[i].z & b.z, w = a[i].w & b.w;
+          const uint32_t sum = x ^ y ^ z, carry = (x & y) | (z & (x ^ y));
+          acc[i][j] += __popc(sum) + __popc(w) + (__popc(carry) << 1);
+        }
       }
     }
     __syncwarp();

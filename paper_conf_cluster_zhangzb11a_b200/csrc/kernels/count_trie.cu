@@ -9,14 +9,18 @@
 //
 //   * the host cuts the candidate list into BLOCKS of <= 256 lexicographically consecutive
 //     candidates touching <= 64 distinct rows; each of the 8 warps of a CTA owns 32 of them;
-//   * a CTA = (block, part of the transaction axis).  It streams its part in STRIPES of 128
-//     words (4,096 transactions): the block's rows' 512-byte segments are brought into shared
-//     memory by 1-D bulk async copies (cp.async.bulk + mbarrier complete_tx), double buffered;
-//   * every warp walks its 32 candidates for the stripe: lane = 4 consecutive words (LDS.128,
-//     conflict-free); a register stack V[d] = AND of the first d+1 rows is recomputed only from
-//     the first position where a candidate differs from its predecessor (lcp), the leaf is one
-//     LDS.128 + 4 AND + 4 POPC into a per-candidate REGISTER accumulator;
-//   * only after the whole part: warp reduction (redux.sync) + one atomicAdd per (CTA, candidate).
+//   * a CTA = (block, part of the transaction axis).  It streams its part in STRIPES of 128 x W
+//     words (W = 2 for k <= 8, else 1): a producer warp brings the block's rows' segments into a
+//     shared-memory ring with 1-D bulk async copies (cp.async.bulk + mbarrier complete_tx);
+//   * the 8 consumer warps split the block's candidates evenly and walk them for every stripe:
+//     lane = W x 4 words (W independent LDS.128 per row, conflict-free); a register stack V[d] = AND of the first d+1 rows is recomputed only from
+//     the first position where a candidate differs from its predecessor (lcp; a warp-uniform
+//     jump into an unrolled fall-through chain, so skipped levels cost nothing), the leaf is one
+//     LDS.128 + 4 AND + 4 POPC per 16 bytes, reduced across the warp with redux.sync into a
+//     per-candidate shared-memory counter (a compact, non-unrolled candidate loop: no I-cache
+//     thrash);  the bitset pitch is a
+//     multiple of the 128-word stripe, so there is no ragged stripe to mask;
+//   * only after the whole part: one atomicAdd per (CTA, candidate).
 // Work per cand x word: ~1 LDS word + 1 AND + 1 POPC + (lcp recompute); no per-stripe reductions,
 // no global traffic besides the row segments (DRAM ~ the bitset once per part-window, the grid is
 // part-major so concurrently running CTAs share the same stripes in L2).  Bound: POPC issue.
@@ -27,11 +31,10 @@
 namespace gpa {
 namespace {
 
-constexpr int kThreads = 256;
-constexpr int kWarps = kThreads / 32;
+constexpr int kWarps = 8;                          // consumer warps
+constexpr int kThreads = (kWarps + 1) * 32;        // + 1 producer warp (bulk copies)
 constexpr int kCandPerWarp = 32;
-constexpr int kStripeWords = 128;                 // 32 lanes x 4 words
-constexpr int kSegBytes = kStripeWords * 4;       // 512 B per row segment
+constexpr uint32_t kTrieMaxStages = 8;
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 
@@ -40,6 +43,9 @@ __device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
 }
 __device__ __forceinline__ void mbar_arrive_expect_tx(uint32_t bar, uint32_t bytes) {
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint32_t bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
 }
 __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
   asm volatile(
@@ -64,21 +70,46 @@ __device__ __forceinline__ uint4 lds128(uint32_t addr) {
   asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(addr));
   return v;
 }
-__device__ __forceinline__ uint32_t byte_of(const uint4& v, int d) {
-  const uint32_t w = d < 4 ? v.x : d < 8 ? v.y : d < 12 ? v.z : v.w;
-  return (w >> (8 * (d & 3))) & 0xffu;
+__device__ __forceinline__ uint4 and4(const uint4& a, const uint4& b) {
+  return make_uint4(a.x & b.x, a.y & b.y, a.z & b.z, a.w & b.w);
 }
 
-template <int K>
-__global__ void __launch_bounds__(kThreads, 2) count_trie_kernel(
+// byte offset (local row * segment bytes) of level d in the candidate's descriptor: 16-bit
+// fields, levels 0-7 in lo, 8-15 in hi
+__device__ __forceinline__ uint32_t off_of(const uint4& lo, const uint4& hi, int d) {
+  const uint4& v = d < 8 ? lo : hi;
+  const int e = d & 7;
+  const uint32_t w = e < 2 ? v.x : e < 4 ? v.y : e < 6 ? v.z : v.w;
+  return (e & 1) ? (w >> 16) : (w & 0xffffu);
+}
+
+// One trie level: V[D] = V[D-1] & row segment (V[0] = the row segment); W uint4 per lane.
+template <int K, int W, int D>
+__device__ __forceinline__ void trie_level(uint4 (&V)[K - 1][W], uint32_t base, const uint4& lo, const uint4& hi) {
+  if constexpr (D < K - 1) {
+    const uint32_t a = base + off_of(lo, hi, D);
+    uint4 v[W];
+#pragma unroll
+    for (int u = 0; u < W; ++u) v[u] = lds128(a + u * 512);
+#pragma unroll
+    for (int u = 0; u < W; ++u) V[D][u] = D == 0 ? v[u] : and4(V[D > 0 ? D - 1 : 0][u], v[u]);
+  }
+}
+
+template <int K, int W>
+__global__ void __maxnreg__(112) count_trie_kernel(
     const uint32_t* __restrict__ rows, uint64_t pitch_words, const TrieBlock* __restrict__ blocks,
     const uint32_t* __restrict__ block_rows, const uint4* __restrict__ cand_lrows, const uint8_t* __restrict__ cand_lcp,
-    uint32_t n_blocks, uint32_t n_parts, uint32_t n_stripes, uint32_t* __restrict__ counts) {
+    uint32_t n_blocks, uint32_t n_parts, uint32_t n_stripes, uint32_t n_stages, uint32_t* __restrict__ counts) {
+  constexpr uint32_t kStripeWords = 128 * W;
+  constexpr uint32_t kSegBytes = kStripeWords * 4;
   extern __shared__ __align__(16) uint8_t smem[];
-  __shared__ uint4 s_lrows[kWarps * kCandPerWarp];
+  __shared__ uint4 s_desc[kWarps * kCandPerWarp][2];
   __shared__ uint8_t s_lcp[kWarps * kCandPerWarp];
+  __shared__ uint32_t s_cnt[kWarps * kCandPerWarp];
   __shared__ uint32_t s_rowid[kTrieMaxRows];
-  __shared__ __align__(8) uint64_t s_full[2];
+  __shared__ __align__(8) uint64_t s_full[kTrieMaxStages];
+  __shared__ __align__(8) uint64_t s_empty[kTrieMaxStages];
 
   const uint32_t b = blockIdx.x % n_blocks;
   const uint32_t part = blockIdx.x / n_blocks;
@@ -87,15 +118,28 @@ __global__ void __launch_bounds__(kThreads, 2) count_trie_kernel(
   const uint32_t st1 = (uint32_t)((uint64_t)n_stripes * (part + 1) / n_parts);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
 
+  // descriptor: 16-bit shared-memory offsets of the candidate's rows (local row * segment bytes)
   for (uint32_t i = threadIdx.x; i < blk.n_cand; i += kThreads) {
-    s_lrows[i] = cand_lrows[blk.cand_begin + i];
+    const uint4 lr = cand_lrows[blk.cand_begin + i];
+    const uint32_t w[4] = {lr.x, lr.y, lr.z, lr.w};
+    uint32_t o[8];
+#pragma unroll
+    for (int q = 0; q < 8; ++q) {
+      const uint32_t b0 = (w[q >> 1] >> (16 * (q & 1))) & 0xffu, b1 = (w[q >> 1] >> (16 * (q & 1) + 8)) & 0xffu;
+      o[q] = (b0 * kSegBytes) | ((b1 * kSegBytes) << 16);
+    }
+    s_desc[i][0] = make_uint4(o[0], o[1], o[2], o[3]);
+    s_desc[i][1] = make_uint4(o[4], o[5], o[6], o[7]);
     s_lcp[i] = cand_lcp[blk.cand_begin + i];
   }
   for (uint32_t i = threadIdx.x; i < blk.n_rows; i += kThreads) s_rowid[i] = block_rows[blk.row_begin + i];
   const uint32_t full0 = smem_u32(&s_full[0]);
+  const uint32_t empty0 = smem_u32(&s_empty[0]);
   if (threadIdx.x == 0) {
-    mbar_init(full0, 1);
-    mbar_init(full0 + 8, 1);
+    for (uint32_t q = 0; q < n_stages; ++q) {
+      mbar_init(full0 + 8 * q, 1);
+      mbar_init(empty0 + 8 * q, kWarps);
+    }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
@@ -104,109 +148,130 @@ __global__ void __launch_bounds__(kThreads, 2) count_trie_kernel(
   const uint32_t buf0 = smem_u32(smem);
   const uint32_t buf_bytes = blk.n_rows * kSegBytes;
 
-  // warp 0 issues the bulk copies of stripe s into buffer (i & 1)
-  auto issue = [&](uint32_t s, uint32_t i) {
-    if (warp == 0) {
-      const uint32_t bar = full0 + 8 * (i & 1);
+  if (warp == kWarps) {
+    // ---------------- producer warp: stripe s -> ring slot i % n_stages, one bulk copy per row
+    for (uint32_t s = st0, i = 0; s < st1; ++s, ++i) {
+      const uint32_t slot = i % n_stages;
+      mbar_wait(empty0 + 8 * slot, ((i / n_stages) & 1) ^ 1);
+      const uint32_t bar = full0 + 8 * slot;
       const uint64_t w0 = (uint64_t)s * kStripeWords;
-      const uint32_t words = (uint32_t)((pitch_words - w0) < (uint64_t)kStripeWords ? (pitch_words - w0) : (uint64_t)kStripeWords);
-      if (lane == 0) mbar_arrive_expect_tx(bar, words * 4 * blk.n_rows);
+      if (lane == 0) mbar_arrive_expect_tx(bar, kSegBytes * blk.n_rows);
       __syncwarp();
-      const uint32_t dst = buf0 + (i & 1) * buf_bytes;
+      const uint32_t dst = buf0 + slot * buf_bytes;
       for (uint32_t r = lane; r < blk.n_rows; r += 32)
-        bulk_g2s(dst + r * kSegBytes, rows + (uint64_t)s_rowid[r] * pitch_words + w0, words * 4, bar);
+        bulk_g2s(dst + r * kSegBytes, rows + (uint64_t)s_rowid[r] * pitch_words + w0, kSegBytes, bar);
     }
-  };
+    return;
+  }
 
-  const int my0 = warp * kCandPerWarp;
-  const int n_mine = max(0, min(kCandPerWarp, (int)blk.n_cand - my0));
-  uint32_t acc[kCandPerWarp];
+  // ---------------- consumer warps: the block's candidates split evenly, <= 32 per warp
+  const int chunk = ((int)blk.n_cand + kWarps - 1) / kWarps;
+  const int my0 = warp * chunk;
+  const int n_mine = max(0, min(chunk, (int)blk.n_cand - my0));
+  uint32_t* cnt = s_cnt + warp * kCandPerWarp;   // per-candidate partial counts of this warp
+  if (lane < kCandPerWarp) cnt[lane] = 0;
+  __syncwarp();
+  uint4 V[K - 1][W];
 #pragma unroll
-  for (int j = 0; j < kCandPerWarp; ++j) acc[j] = 0;
-  uint4 V[K - 1];
+  for (int d = 0; d < K - 1; ++d)
 #pragma unroll
-  for (int d = 0; d < K - 1; ++d) V[d] = make_uint4(0, 0, 0, 0);
+    for (int u = 0; u < W; ++u) V[d][u] = make_uint4(0, 0, 0, 0);
 
-  issue(st0, 0);
   for (uint32_t s = st0, i = 0; s < st1; ++s, ++i) {
-    if (s + 1 < st1) issue(s + 1, i + 1);
-    mbar_wait(full0 + 8 * (i & 1), (i >> 1) & 1);
-    const uint64_t w0 = (uint64_t)s * kStripeWords;
-    const bool lane_ok = w0 + (uint64_t)lane * 4 < pitch_words;
-    const uint32_t base = buf0 + (i & 1) * buf_bytes + lane * 16;
-#pragma unroll
-    for (int j = 0; j < kCandPerWarp; ++j) {
-      if (j < n_mine) {
-        const uint4 lr = s_lrows[my0 + j];
-        const int l = s_lcp[my0 + j];
-#pragma unroll
-        for (int d = 0; d < K - 1; ++d) {
-          if (d >= l) {
-            const uint4 v = lds128(base + byte_of(lr, d) * kSegBytes);
-            if (d == 0) {
-              V[0] = v;
-            } else {
-              V[d].x = V[d - 1].x & v.x; V[d].y = V[d - 1].y & v.y;
-              V[d].z = V[d - 1].z & v.z; V[d].w = V[d - 1].w & v.w;
-            }
+    const uint32_t slot = i % n_stages;
+    mbar_wait(full0 + 8 * slot, (i / n_stages) & 1);
+    const uint32_t base = buf0 + slot * buf_bytes + lane * 16;
+#pragma unroll 1
+    for (int j = 0; j < n_mine; ++j) {
+      const uint4 lo = s_desc[my0 + j][0];
+      const uint4 hi = K > 8 ? s_desc[my0 + j][1] : make_uint4(0, 0, 0, 0);
+      // recompute the prefix stack from the first level that differs from the previous
+      // candidate (warp-uniform branches; only the needed levels execute).  Common cases first:
+      // a sibling (lcp = K-1) only needs the leaf, a cousin (lcp = K-2) one level.
+      const int l = s_lcp[my0 + j];
+      if (l <= K - 2) {
+        if (l <= K - 3) {
+          switch (l) {
+#define GPA_TRIE_LEVEL(D) \
+  case D:                 \
+    if constexpr (D <= K - 3) trie_level<K, W, D>(V, base, lo, hi); [[fallthrough]];
+            GPA_TRIE_LEVEL(0) GPA_TRIE_LEVEL(1) GPA_TRIE_LEVEL(2) GPA_TRIE_LEVEL(3) GPA_TRIE_LEVEL(4)
+            GPA_TRIE_LEVEL(5) GPA_TRIE_LEVEL(6) GPA_TRIE_LEVEL(7) GPA_TRIE_LEVEL(8) GPA_TRIE_LEVEL(9)
+            GPA_TRIE_LEVEL(10) GPA_TRIE_LEVEL(11) GPA_TRIE_LEVEL(12) GPA_TRIE_LEVEL(13)
+#undef GPA_TRIE_LEVEL
+            default:
+              break;
           }
         }
-        const uint4 v = lds128(base + byte_of(lr, K - 1) * kSegBytes);
-        const uint32_t c = (__popc(V[K - 2].x & v.x) + __popc(V[K - 2].y & v.y)) +
-                           (__popc(V[K - 2].z & v.z) + __popc(V[K - 2].w & v.w));
-        acc[j] += lane_ok ? c : 0u;
+        trie_level<K, W, K - 2>(V, base, lo, hi);
       }
-    }
-    __syncthreads();  // buffer (i & 1) may be refilled at iteration i + 2 (issued at the top of i + 1)
-  }
+      const uint32_t a = base + off_of(lo, hi, K - 1);
+      uint4 v[W];
 #pragma unroll
-  for (int j = 0; j < kCandPerWarp; ++j) {
-    if (j < n_mine) {
-      const uint32_t sum = __reduce_add_sync(0xffffffffu, acc[j]);
-      if (lane == 0 && sum) atomicAdd(&counts[blk.cand_begin + my0 + j], sum);
+      for (int u = 0; u < W; ++u) v[u] = lds128(a + u * 512);
+      uint32_t c = 0;
+#pragma unroll
+      for (int u = 0; u < W; ++u)
+        c += (__popc(V[K - 2][u].x & v[u].x) + __popc(V[K - 2][u].y & v[u].y)) +
+             (__popc(V[K - 2][u].z & v[u].z) + __popc(V[K - 2][u].w & v[u].w));
+      // warp-reduce this stripe's partial count (redux.sync) into the candidate's smem slot
+      c = __reduce_add_sync(0xffffffffu, c);
+      if (lane == 0) cnt[j] += c;
     }
+    __syncwarp();
+    if (lane == 0) mbar_arrive(empty0 + 8 * slot);
   }
+  __syncwarp();
+  if (lane < n_mine && cnt[lane]) atomicAdd(&counts[blk.cand_begin + my0 + lane], cnt[lane]);
 }
 
-template <int K>
+template <int K, int W>
 void launch_k(const uint32_t* rows, uint64_t pitch_words, const TrieBlock* blocks, const uint32_t* block_rows,
-              const uint4* lrows, const uint8_t* lcp, uint32_t n_blocks, uint32_t n_parts, uint32_t n_stripes,
-              uint32_t max_rows, uint32_t* counts, cudaStream_t stream) {
-  const size_t smem = (size_t)2 * max_rows * kSegBytes;
+              const uint4* lrows, const uint8_t* lcp, uint32_t n_blocks, uint32_t n_parts, uint32_t max_rows,
+              uint32_t* counts, cudaStream_t stream) {
+  constexpr uint32_t kSegBytes = 512 * W;
+  const uint32_t n_stripes = (uint32_t)(pitch_words / (128 * W));
+  if (n_parts > n_stripes) n_parts = n_stripes;
+  if (n_parts < 1) n_parts = 1;
+  // ring depth: as many stripes in flight as fit in ~96 KB (2 CTAs / SM), 2..kTrieMaxStages
+  uint32_t stages = (uint32_t)((96u * 1024u) / ((size_t)max_rows * kSegBytes));
+  stages = stages < 2 ? 2 : (stages > kTrieMaxStages ? kTrieMaxStages : stages);
+  const size_t smem = (size_t)stages * max_rows * kSegBytes;
   static bool attr = false;
   if (!attr) {
-    GPA_CUDA(cudaFuncSetAttribute(count_trie_kernel<K>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                  2 * kTrieMaxRows * kSegBytes));
+    GPA_CUDA(cudaFuncSetAttribute(count_trie_kernel<K, W>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024));
     attr = true;
   }
   const uint64_t grid = (uint64_t)n_blocks * n_parts;
   GPA_REQUIRE(grid < (1ull << 31), GPA_ERR_INVALID, "count_trie: grid too large");
-  count_trie_kernel<K><<<(unsigned)grid, kThreads, smem, stream>>>(rows, pitch_words, blocks, block_rows, lrows, lcp,
-                                                                   n_blocks, n_parts, n_stripes, counts);
+  count_trie_kernel<K, W><<<(unsigned)grid, kThreads, smem, stream>>>(rows, pitch_words, blocks, block_rows, lrows,
+                                                                      lcp, n_blocks, n_parts, n_stripes, stages, counts);
   GPA_CUDA(cudaGetLastError());
 }
 
 }  // namespace
 
-uint32_t trie_stripes(uint64_t pitch_words) { return (uint32_t)((pitch_words + kStripeWords - 1) / kStripeWords); }
+uint32_t trie_max_rows(uint32_t k) { return k <= kTrieWideMaxK ? kTrieMaxRows / 2 : kTrieMaxRows; }
+
+uint32_t trie_stripes(uint32_t k, uint64_t pitch_words) {
+  return (uint32_t)(pitch_words / (k <= kTrieWideMaxK ? 256 : 128));
+}
 
 uint64_t launch_count_trie(uint32_t k, const uint32_t* rows, uint64_t pitch_words, const TrieBlock* blocks,
                            const uint32_t* block_rows, const uint4* cand_lrows, const uint8_t* cand_lcp,
                            uint32_t n_blocks, uint32_t max_rows, uint32_t n_parts, uint32_t* counts,
                            cudaStream_t stream) {
   if (n_blocks == 0) return 0;
-  const uint32_t n_stripes = trie_stripes(pitch_words);
-  if (n_parts > n_stripes) n_parts = n_stripes;
-  if (n_parts < 1) n_parts = 1;
-#define GPA_TRIE_CASE(KK)                                                                                   \
-  case KK:                                                                                                  \
-    launch_k<KK>(rows, pitch_words, blocks, block_rows, cand_lrows, cand_lcp, n_blocks, n_parts, n_stripes, \
-                 max_rows, counts, stream);                                                                 \
+  GPA_REQUIRE(max_rows <= trie_max_rows(k), GPA_ERR_INVALID, "count_trie: block with %u rows", max_rows);
+#define GPA_TRIE_CASE(KK, WW)                                                                                     \
+  case KK:                                                                                                       \
+    launch_k<KK, WW>(rows, pitch_words, blocks, block_rows, cand_lrows, cand_lcp, n_blocks, n_parts, max_rows,   \
+                     counts, stream);                                                                            \
     break;
   switch (k) {
-    GPA_TRIE_CASE(2) GPA_TRIE_CASE(3) GPA_TRIE_CASE(4) GPA_TRIE_CASE(5) GPA_TRIE_CASE(6) GPA_TRIE_CASE(7)
-    GPA_TRIE_CASE(8) GPA_TRIE_CASE(9) GPA_TRIE_CASE(10) GPA_TRIE_CASE(11) GPA_TRIE_CASE(12) GPA_TRIE_CASE(13)
-    GPA_TRIE_CASE(14) GPA_TRIE_CASE(15) GPA_TRIE_CASE(16)
+    GPA_TRIE_CASE(2, 2) GPA_TRIE_CASE(3, 2) GPA_TRIE_CASE(4, 2) GPA_TRIE_CASE(5, 2) GPA_TRIE_CASE(6, 2)
+    GPA_TRIE_CASE(7, 2) GPA_TRIE_CASE(8, 2) GPA_TRIE_CASE(9, 1) GPA_TRIE_CASE(10, 1) GPA_TRIE_CASE(11, 1)
+    GPA_TRIE_CASE(12, 1) GPA_TRIE_CASE(13, 1) GPA_TRIE_CASE(14, 1) GPA_TRIE_CASE(15, 1) GPA_TRIE_CASE(16, 1)
     default:
       fail(GPA_ERR_INVALID, "count_trie: k = %u outside [2, %u]", k, kTrieMaxK);
   }

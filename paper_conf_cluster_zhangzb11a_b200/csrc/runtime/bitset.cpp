@@ -223,9 +223,14 @@ void count_trie_batch(gpa_bitset* bs, const GroupedBatch& b, CountStats* st) {
   std::vector<uint8_t> local(bs->n_rows, 0);
   std::vector<uint32_t> cur(k), prev(k);
   uint32_t max_rows = 0;
+  const uint32_t rmax = trie_max_rows(k);
   TrieBlock blk{0, 0, 0, 0};
   auto close_block = [&]() {
     if (blk.n_cand) {
+      // the kernel splits a block's candidates evenly over its 8 warps: every warp chunk starts
+      // with an empty prefix stack
+      const uint32_t chunk = (blk.n_cand + 7) / 8;
+      for (uint32_t c0 = 0; c0 < blk.n_cand; c0 += chunk) lcp[blk.cand_begin + c0] = 0;
       blocks.push_back(blk);
       max_rows = std::max(max_rows, blk.n_rows);
     }
@@ -240,7 +245,7 @@ void count_trie_batch(gpa_bitset* bs, const GroupedBatch& b, CountStats* st) {
       uint32_t fresh = 0;
       for (uint32_t d = 0; d < k; ++d) fresh += stamp[cur[d]] != id;
       // duplicate rows inside one candidate cannot happen (strictly increasing)
-      if (blk.n_cand == kTrieMaxCand || blk.n_rows + fresh > kTrieMaxRows) {
+      if (blk.n_cand == kTrieMaxCand || blk.n_rows + fresh > rmax) {
         close_block();
         fresh = k;
       }
@@ -257,7 +262,7 @@ void count_trie_batch(gpa_bitset* bs, const GroupedBatch& b, CountStats* st) {
       }
       memcpy(&lrows[c], bytes, 16);
       uint32_t l = 0;
-      if (blk.n_cand % 32 != 0)
+      if (c > 0)
         while (l < km1 && cur[l] == prev[l]) ++l;
       lcp[c] = (uint8_t)l;
       ++blk.n_cand;
@@ -266,7 +271,7 @@ void count_trie_batch(gpa_bitset* bs, const GroupedBatch& b, CountStats* st) {
   }
   close_block();
   const uint32_t n_blocks = (uint32_t)blocks.size();
-  const uint32_t n_stripes = trie_stripes(bs->pitch_words);
+  const uint32_t n_stripes = trie_stripes(k, bs->pitch_words);
   uint32_t n_parts = std::max<uint32_t>(1, n_stripes / 64);
   const uint32_t want = (uint32_t)bs->n_sms * 2 * 3;
   if ((uint64_t)n_blocks * n_parts < want) n_parts = std::min<uint32_t>(n_stripes, (want + n_blocks - 1) / n_blocks);
