@@ -222,11 +222,13 @@ def main():
     value = cand_tx / (step_ms * 1e-3)
     launches_per_step = 2 + sum(lv.stats["launches"] for lv in res.levels[1:])  # hist + bitset + counting
 
-    # ---- dominant kernel: largest count time per step (generation 2: the tiled pair kernel)
-    dom = max(res.levels[1:], key=lambda lv: float(np.mean(level_ms[lv.k])))
-    dom_ms = max_over_ranks(float(np.mean(level_ms[dom.k])))
-    dom_work = dom.n_cand * n_tx
-    kernel_name = dom.stats["kernel_name"]
+    # ---- rooflines.  All counting kernels are bound by the XU pipe that executes POPC (16 / clk /
+    # SM on sm_100a, profiles/r01_microbench_popc.txt), not by HBM (the bitset is re-read from L2
+    # / shared memory).  Peak in cand*tx/s = 148 SM x 16 POPC/clk / (POPC per word) x 32 tx/word x
+    # f_SM:  the pair kernel counts 4 words with 3 POPC (carry-save adder) -> 0.75 POPC / word;
+    # the trie / prefix / v0 kernels use 1 POPC / word.  "achieved" uses the algorithmic work
+    # |C_k| x N of the launch and its CUDA-event time inside the timed region.
+    sm_max = None
     peaks = {}
     try:
         peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
@@ -234,23 +236,30 @@ def main():
         pass
     clk = clocks.summary()
     sm_max = clk.get("sm_max_mhz") or peaks.get("sm_max_mhz", 1965.0)
-    if kernel_name == "pairs":
-        # ALU bound: 148 SMs x 16 POPC/clk/SM x 32 tx per word (profiles/r01_microbench_popc.txt)
-        peak = 148 * 16 * 32 * sm_max * 1e6 / 1e12
-        roof = {"bound": "alu", "achieved": dom_work / (dom_ms * 1e-3) / 1e12, "peak": peak, "unit": "Tcand*tx/s",
-                "peak_basis": f"148 SM x 16 POPC/clk x 32 tx/word x {sm_max:.0f} MHz (POPC rate measured)"}
-    else:
-        hbm = peaks.get("hbm_gbs", 6650.0)
-        rowbytes = dom.n_cand  # placeholder replaced below
-        groups = max(dom.stats["n_groups"], 1)
-        rowbytes = (groups * (dom.k - 1) + dom.n_cand) * (n_tx / 8)
-        roof = {"bound": "hbm", "achieved": rowbytes / (dom_ms * 1e-3) / 1e9, "peak": hbm, "unit": "GB/s",
-                "peak_basis": "MEASURED_PEAKS.json hbm_gbs"}
-    roof["frac"] = roof["achieved"] / roof["peak"]
+    popc_per_word = {"pairs": 0.75}
+
+    def roof_for(levels):
+        ms = max_over_ranks(sum(float(np.mean(level_ms[lv.k])) for lv in levels))
+        work = sum(lv.n_cand for lv in levels) * n_tx
+        name = levels[0].stats["kernel_name"]
+        ppw = popc_per_word.get(name, 1.0)
+        peak = 148 * 16 / ppw * 32 * sm_max * 1e6 / 1e12
+        ach = work / (ms * 1e-3) / 1e12
+        return {"bound": "alu", "achieved": ach, "peak": peak, "unit": "Tcand*tx/s", "frac": ach / peak,
+                "peak_basis": f"XU pipe: 148 SM x 16 POPC/clk / {ppw} POPC per 32-tx word x 32 x {sm_max:.0f} MHz "
+                              f"(POPC rate measured, profiles/r01_microbench_popc.txt)",
+                "kernel_ms": ms, "work": work}
+
+    by_kernel = {}
+    for lv in res.levels[1:]:
+        by_kernel.setdefault(lv.stats["kernel_name"], []).append(lv)
+    roof_all = {name: roof_for(lvs) for name, lvs in by_kernel.items()}
+    dom = max(res.levels[1:], key=lambda lv: float(np.mean(level_ms[lv.k])))   # single longest launch
+    roof = roof_for([dom])
+    roof["kernel"] = f"count_{dom.stats['kernel_name']} (generation {dom.k}, the longest launch)"
     roof["traffic"] = None
-    roof["kernel"] = f"count_{kernel_name} (generation {dom.k})"
-    roof["kernel_ms"] = dom_ms
-    roof["work_per_launch"] = dom_work
+    for r in roof_all.values():
+        r.pop("peak_basis", None)
 
     # ---- end to end: pinned host CSR, H2D + every D2H inside the timed region
     e2e = None
@@ -301,6 +310,7 @@ def main():
                        if cfg.name == "t40i10d10m" else "none (small config)",
                        "parallelism": f"tx-shard x{world}", "kernel": args.kernel},
             "roofline": roof,
+            "roofline_by_kernel": roof_all,
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": launches_per_step * args.steps,

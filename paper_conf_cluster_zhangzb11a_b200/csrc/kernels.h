@@ -50,8 +50,8 @@ struct TrieBlock {
   uint32_t row_begin;    // into block_rows
   uint32_t n_rows;       // <= kTrieMaxRows
 };
-uint32_t trie_max_rows(uint32_t k);
-uint32_t trie_stripes(uint32_t k, uint64_t pitch_words);
+inline uint32_t trie_max_rows(uint32_t k) { return k <= kTrieWideMaxK ? kTrieMaxRows / 2 : kTrieMaxRows; }
+inline uint32_t trie_stripe_words(uint32_t k) { return k <= kTrieWideMaxK ? 256 : 128; }
 // cand_lrows[c]: byte d = block-local row of item d; cand_lcp[c]: items shared with candidate c-1
 // (0 for the first candidate of every warp chunk: a block's n candidates are split into chunks of
 // ceil(n / 8)).  counts must be zeroed.

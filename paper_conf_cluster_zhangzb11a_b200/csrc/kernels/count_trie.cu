@@ -251,12 +251,6 @@ void launch_k(const uint32_t* rows, uint64_t pitch_words, const TrieBlock* block
 
 }  // namespace
 
-uint32_t trie_max_rows(uint32_t k) { return k <= kTrieWideMaxK ? kTrieMaxRows / 2 : kTrieMaxRows; }
-
-uint32_t trie_stripes(uint32_t k, uint64_t pitch_words) {
-  return (uint32_t)(pitch_words / (k <= kTrieWideMaxK ? 256 : 128));
-}
-
 uint64_t launch_count_trie(uint32_t k, const uint32_t* rows, uint64_t pitch_words, const TrieBlock* blocks,
                            const uint32_t* block_rows, const uint4* cand_lrows, const uint8_t* cand_lcp,
                            uint32_t n_blocks, uint32_t max_rows, uint32_t n_parts, uint32_t* counts,

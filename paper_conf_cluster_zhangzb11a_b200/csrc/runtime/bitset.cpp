@@ -213,65 +213,16 @@ void count_flat_v0(gpa_bitset* bs, const std::vector<uint32_t>& flat, uint32_t k
 // its shared-prefix length with the previous candidate of the same 32-candidate warp chunk.
 void count_trie_batch(gpa_bitset* bs, const GroupedBatch& b, CountStats* st) {
   cudaStream_t s = bs->stream;
-  const uint32_t k = b.k, km1 = k - 1;
-  const uint64_t M = b.size(), G = b.groups();
-  std::vector<TrieBlock> blocks;
-  std::vector<uint32_t> brows;
-  std::vector<uint4> lrows(M);
-  std::vector<uint8_t> lcp(M);
-  std::vector<uint32_t> stamp(bs->n_rows, UINT32_MAX);
-  std::vector<uint8_t> local(bs->n_rows, 0);
-  std::vector<uint32_t> cur(k), prev(k);
-  uint32_t max_rows = 0;
-  const uint32_t rmax = trie_max_rows(k);
-  TrieBlock blk{0, 0, 0, 0};
-  auto close_block = [&]() {
-    if (blk.n_cand) {
-      // the kernel splits a block's candidates evenly over its 8 warps: every warp chunk starts
-      // with an empty prefix stack
-      const uint32_t chunk = (blk.n_cand + 7) / 8;
-      for (uint32_t c0 = 0; c0 < blk.n_cand; c0 += chunk) lcp[blk.cand_begin + c0] = 0;
-      blocks.push_back(blk);
-      max_rows = std::max(max_rows, blk.n_rows);
-    }
-    blk = TrieBlock{blk.cand_begin + blk.n_cand, 0, (uint32_t)brows.size(), 0};
-  };
-  uint64_t c = 0;
-  for (uint64_t g = 0; g < G; ++g) {
-    for (uint64_t j = b.ext_off[g]; j < b.ext_off[g + 1]; ++j, ++c) {
-      std::copy(b.prefix.begin() + g * km1, b.prefix.begin() + (g + 1) * km1, cur.begin());
-      cur[km1] = b.ext[j];
-      const uint32_t id = (uint32_t)blocks.size();
-      uint32_t fresh = 0;
-      for (uint32_t d = 0; d < k; ++d) fresh += stamp[cur[d]] != id;
-      // duplicate rows inside one candidate cannot happen (strictly increasing)
-      if (blk.n_cand == kTrieMaxCand || blk.n_rows + fresh > rmax) {
-        close_block();
-        fresh = k;
-      }
-      const uint32_t id2 = (uint32_t)blocks.size();
-      uint8_t bytes[16] = {0};
-      for (uint32_t d = 0; d < k; ++d) {
-        const uint32_t r = cur[d];
-        if (stamp[r] != id2) {
-          stamp[r] = id2;
-          local[r] = (uint8_t)blk.n_rows++;
-          brows.push_back(r);
-        }
-        bytes[d] = local[r];
-      }
-      memcpy(&lrows[c], bytes, 16);
-      uint32_t l = 0;
-      if (c > 0)
-        while (l < km1 && cur[l] == prev[l]) ++l;
-      lcp[c] = (uint8_t)l;
-      ++blk.n_cand;
-      std::swap(prev, cur);
-    }
-  }
-  close_block();
+  const uint32_t k = b.k;
+  const uint64_t M = b.size();
+  TriePlan P = plan_trie(b, bs->n_rows);
+  const auto& blocks = P.blocks;
+  const auto& brows = P.rows;
+  const auto& lrows = P.lrows;
+  const auto& lcp = P.lcp;
+  const uint32_t max_rows = P.max_rows;
   const uint32_t n_blocks = (uint32_t)blocks.size();
-  const uint32_t n_stripes = trie_stripes(k, bs->pitch_words);
+  const uint32_t n_stripes = (uint32_t)(bs->pitch_words / trie_stripe_words(k));
   uint32_t n_parts = std::max<uint32_t>(1, n_stripes / 64);
   const uint32_t want = (uint32_t)bs->n_sms * 2 * 3;
   if ((uint64_t)n_blocks * n_parts < want) n_parts = std::min<uint32_t>(n_stripes, (want + n_blocks - 1) / n_blocks);

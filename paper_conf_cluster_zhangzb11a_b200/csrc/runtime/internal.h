@@ -88,6 +88,19 @@ struct GroupedBatch {
 // (k-1)-prefix; candidates come out in lexicographic order.
 GroupedBatch candgen_join_prune(const std::vector<uint32_t>& L, uint64_t n, uint32_t km1);
 
+// Work plan of the trie kernel for a grouped batch (host side; see count_trie.cu): blocks of
+// <= kTrieMaxCand lexicographically consecutive candidates touching <= trie_max_rows(k) rows, the
+// block-local row byte of every item of every candidate, and the shared-prefix length with the
+// previous candidate (0 at the start of every warp chunk of ceil(n_cand / 8) candidates).
+struct TriePlan {
+  std::vector<TrieBlock> blocks;
+  std::vector<uint32_t> rows;     // global row ids, concatenated per block
+  std::vector<uint4> lrows;       // M entries: byte d = local row of item d
+  std::vector<uint8_t> lcp;       // M entries
+  uint32_t max_rows = 0;
+};
+TriePlan plan_trie(const GroupedBatch& b, uint32_t n_rows);
+
 const char* last_error_cstr();
 
 // Run f() and translate exceptions into a gpa_status + thread-local message (no exception

@@ -28,6 +28,7 @@ def shim(tmp_path_factory):
                            os.path.join(CSRC, "runtime", "candgen.cpp"), "-o", str(out)])
     lib = ctypes.CDLL(str(out))
     lib.shim_candgen.restype = ctypes.c_int
+    lib.shim_plan_trie.restype = ctypes.c_int
     return lib
 
 
@@ -91,3 +92,66 @@ def test_candgen_threaded_large(shim):
     L = np.array(pairs, dtype=np.uint32)
     got, _, _ = run_shim(shim, L)
     assert got == [tuple(map(int, x)) for x in oracle.candgen(L)]
+
+
+def run_plan(lib, L, n_rows):
+    L = np.ascontiguousarray(L, dtype=np.uint32)
+    n, km1 = L.shape
+    k = km1 + 1
+    cap = max(64, n * n)
+    blocks = np.zeros(cap * 4, np.uint32)
+    rows = np.zeros(cap, np.uint32)
+    lrows = np.zeros(cap * 16, np.uint8)
+    lcp = np.zeros(cap, np.uint8)
+    cand = np.zeros(cap * k, np.uint32)
+    nb, nr, nc = ctypes.c_uint64(), ctypes.c_uint64(), ctypes.c_uint64()
+    P = lambda a: a.ctypes.data_as(ctypes.c_void_p)
+    rc = lib.shim_plan_trie(P(L), ctypes.c_uint64(n), ctypes.c_uint32(km1), ctypes.c_uint32(n_rows), P(blocks),
+                            ctypes.byref(nb), P(rows), ctypes.byref(nr), P(lrows), P(lcp), P(cand),
+                            ctypes.c_uint64(cap), ctypes.byref(nc))
+    assert rc == 0
+    M = nc.value
+    return (blocks[: nb.value * 4].reshape(-1, 4), rows[: nr.value], lrows[: M * 16].reshape(M, 16), lcp[:M],
+            cand[: M * k].reshape(M, k))
+
+
+@pytest.mark.parametrize("name,k", [("mushroom", 3), ("mushroom", 5), ("chess", 4), ("random", 3), ("random", 9)])
+def test_trie_plan_invariants(shim, name, k):
+    """Blocks tile the candidates in order with <= 256 candidates and <= trie_max_rows(k) rows;
+    local row bytes map back to each candidate's rows; lcp is the shared prefix with the previous
+    candidate, reset to 0 at every warp chunk (ceil(n/8)) start -- what count_trie assumes."""
+    if name == "random":
+        rng = np.random.default_rng(k)
+        L = np.array(sorted({tuple(sorted(rng.choice(300, k - 1, replace=False))) for _ in range(6000)}), np.uint32)
+        L = np.array(sorted({tuple(x) for x in L.tolist()} |
+                            {tuple([0, 1, 2, 3, 4, 5, 6, 7][: k - 2]) + (q,) for q in range(8, 200)}), np.uint32)
+        n_rows = 300
+    else:
+        ds = gen.make(name)
+        theta = oracle.min_count(ds.n_tx, gen.CONFIGS[name].minsup)
+        r = oracle.mine_ds(ds, theta)
+        lv = r.levels[k - 2]
+        L = lv.cand[lv.count >= theta]
+        n_rows = ds.n_items
+    blocks, rows, lrows, lcp, cand = run_plan(shim, L, n_rows)
+    M = len(cand)
+    if M == 0:
+        return
+    rmax = 32 if k <= 8 else 64
+    pos = 0
+    for cb, nc, rb, nr in blocks.tolist():
+        assert cb == pos and 0 < nc <= 256 and nr <= rmax
+        chunk = (nc + 7) // 8
+        for i in range(nc):
+            c = cb + i
+            assert [int(rows[rb + int(lrows[c, d])]) for d in range(k)] == cand[c].tolist()
+            assert all(lrows[c, d] < nr for d in range(k))
+            if i % chunk == 0:
+                assert lcp[c] == 0
+            else:
+                l = 0
+                while l < k - 1 and cand[c, l] == cand[c - 1, l]:
+                    l += 1
+                assert lcp[c] == l
+        pos += nc
+    assert pos == M
