@@ -41,8 +41,8 @@ uint64_t launch_count_prefix(const uint32_t* rows, uint64_t pitch_words, const u
 // Transaction-tiled trie walk for generations k in [2, kTrieMaxK] (count_trie.cu).  Candidates
 // (lexicographic) are cut into blocks of <= kTrieMaxCand candidates touching <= kTrieMaxRows rows.
 constexpr uint32_t kTrieMaxK = 16;
-constexpr uint32_t kTrieWideMaxK = 8;    // k <= 8: 8 words per lane (256-word stripes), <= 32 rows / block
-constexpr uint32_t kTrieMaxRows = 64;    // k > 8: 4 words per lane (128-word stripes), <= 64 rows / block
+constexpr uint32_t kTrieWideMaxK = 8;    // 4 <= k <= 8: 8 words per lane (256-word stripes), <= 32 rows / block
+constexpr uint32_t kTrieMaxRows = 64;    // otherwise: 4 words per lane (128-word stripes), <= 64 rows / block
 constexpr uint32_t kTrieMaxCand = 256;
 struct TrieBlock {
   uint32_t cand_begin;   // first candidate (global index)
@@ -50,8 +50,9 @@ struct TrieBlock {
   uint32_t row_begin;    // into block_rows
   uint32_t n_rows;       // <= kTrieMaxRows
 };
-inline uint32_t trie_max_rows(uint32_t k) { return k <= kTrieWideMaxK ? kTrieMaxRows / 2 : kTrieMaxRows; }
-inline uint32_t trie_stripe_words(uint32_t k) { return k <= kTrieWideMaxK ? 256 : 128; }
+inline bool trie_wide(uint32_t k) { return k >= 3 && k <= kTrieWideMaxK; }
+inline uint32_t trie_max_rows(uint32_t k) { return trie_wide(k) ? kTrieMaxRows / 2 : kTrieMaxRows; }
+inline uint32_t trie_stripe_words(uint32_t k) { return trie_wide(k) ? 256 : 128; }
 // cand_lrows[c]: byte d = block-local row of item d; cand_lcp[c]: items shared with candidate c-1
 // (0 for the first candidate of every warp chunk: a block's n candidates are split into chunks of
 // ceil(n / 8)).  counts must be zeroed.

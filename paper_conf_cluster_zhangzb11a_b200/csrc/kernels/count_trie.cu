@@ -263,7 +263,7 @@ uint64_t launch_count_trie(uint32_t k, const uint32_t* rows, uint64_t pitch_word
                      counts, stream);                                                                            \
     break;
   switch (k) {
-    GPA_TRIE_CASE(2, 2) GPA_TRIE_CASE(3, 2) GPA_TRIE_CASE(4, 2) GPA_TRIE_CASE(5, 2) GPA_TRIE_CASE(6, 2)
+    GPA_TRIE_CASE(2, 1) GPA_TRIE_CASE(3, 2) GPA_TRIE_CASE(4, 2) GPA_TRIE_CASE(5, 2) GPA_TRIE_CASE(6, 2)
     GPA_TRIE_CASE(7, 2) GPA_TRIE_CASE(8, 2) GPA_TRIE_CASE(9, 1) GPA_TRIE_CASE(10, 1) GPA_TRIE_CASE(11, 1)
     GPA_TRIE_CASE(12, 1) GPA_TRIE_CASE(13, 1) GPA_TRIE_CASE(14, 1) GPA_TRIE_CASE(15, 1) GPA_TRIE_CASE(16, 1)
     default:

@@ -215,7 +215,9 @@ void count_trie_batch(gpa_bitset* bs, const GroupedBatch& b, CountStats* st) {
   cudaStream_t s = bs->stream;
   const uint32_t k = b.k;
   const uint64_t M = b.size();
+  const double tp0 = wall_ms();
   TriePlan P = plan_trie(b, bs->n_rows);
+  const double tp1 = wall_ms();
   const auto& blocks = P.blocks;
   const auto& brows = P.rows;
   const auto& lrows = P.lrows;
@@ -241,7 +243,12 @@ void count_trie_batch(gpa_bitset* bs, const GroupedBatch& b, CountStats* st) {
     launch_count_trie(k, bs->rows.p, bs->pitch_words, bs->d_tblocks.p, bs->d_trows.p, bs->d_lrows.p, bs->d_lcp.p,
                       n_blocks, max_rows, n_parts, bs->d_counts.p, s);
   if (st) { st->kernel = GPA_KERNEL_TRIE; st->launches = 1; }
+  const double tp2 = wall_ms();
   finish_counts(bs, M, st);
+  if (trace_enabled())
+    fprintf(stderr, "[gpa] k=%u trie: M=%llu blocks=%u max_rows=%u parts=%u plan %.2f ms, h2d+launch %.2f ms, "
+            "kernel %.2f ms\n", k, (unsigned long long)M, n_blocks, max_rows, n_parts, tp1 - tp0, tp2 - tp1,
+            st ? st->count_ms : -1.0);
 }
 
 }  // namespace
@@ -251,8 +258,13 @@ void count_grouped(gpa_bitset* bs, const GroupedBatch& b, uint32_t kernel, Count
   const uint64_t M = b.size(), G = b.groups();
   const uint32_t km1 = b.k - 1;
   if (M == 0) return;
-  if (kernel == GPA_KERNEL_AUTO || kernel == GPA_KERNEL_PAIRS)  // grouped batches: trie walk, else prefix
-    kernel = (b.k >= 2 && b.k <= kTrieMaxK) ? GPA_KERNEL_TRIE : GPA_KERNEL_PREFIX;
+  if (kernel == GPA_KERNEL_AUTO || kernel == GPA_KERNEL_PAIRS) {
+    // grouped batches: large sibling groups amortise the (k-1)-row prefix well in the streaming
+    // prefix kernel (measured: T40I10D10M k = 3, 4.6 siblings / group); small groups (deep
+    // generations, ~2 siblings) need the trie walk's reuse across groups
+    const double sib = (double)M / (double)std::max<uint64_t>(G, 1);
+    kernel = (b.k >= 2 && b.k <= kTrieMaxK && sib < 4.0) ? GPA_KERNEL_TRIE : GPA_KERNEL_PREFIX;
+  }
   if (kernel == GPA_KERNEL_TRIE) {
     if (b.k >= 2 && b.k <= kTrieMaxK) {
       count_trie_batch(bs, b, st);

@@ -103,6 +103,11 @@ TriePlan plan_trie(const GroupedBatch& b, uint32_t n_rows);
 
 const char* last_error_cstr();
 
+// Host tracing (SURVEY.md §5 "Tracing"): GPA_TRACE=1 prints one line per mining phase / level
+// with host wall-clock splits to stderr.
+bool trace_enabled();
+double wall_ms();
+
 // Run f() and translate exceptions into a gpa_status + thread-local message (no exception
 // crosses the C ABI).
 template <class F>

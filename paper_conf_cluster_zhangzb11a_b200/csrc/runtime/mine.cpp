@@ -11,6 +11,7 @@
 #include <chrono>
 
 #include "internal.h"
+#include "pool.h"
 
 struct gpa_level_data {
   uint32_t k = 0;
@@ -40,45 +41,82 @@ double now_ms() {
 
 // Record generation k.  Candidates are the grouped batch b (k >= 3) or, for k = 2 (b == nullptr),
 // all pairs of the n rows in lexicographic order.  Returns L_k in row ids (lexicographic).
+// Two parallel passes over contiguous candidate ranges: count the frequent candidates of each
+// range, then write L_k, the frequent itemsets (original ids) and their supports at exact
+// offsets (no growing vectors, no concatenation).
 std::vector<uint32_t> record_level(gpa_result* R, const gpa_bitset* bs, uint32_t k, const GroupedBatch* b, uint64_t M,
                                    const std::vector<uint32_t>& counts, bool keep, uint64_t* n_freq) {
   gpa_level_data lv;
   lv.k = k;
   lv.n_cand = M;
   lv.kept = keep;
-  std::vector<uint32_t> Lk;
   const auto& ior = bs->item_of_row;
   const uint32_t theta = (uint32_t)R->min_count;
+  const uint64_t n = bs->n_rows;
+  // outer units: groups (k >= 3) or first items a (k = 2)
+  const uint64_t U = b ? b->groups() : (n ? n - 1 : 0);
+  auto unit_begin = [&](uint64_t u) -> uint64_t { return b ? b->ext_off[u] : pair_index(u, u + 1, n); };
   if (keep) {
     lv.cand_items.resize(M * k);
     lv.cand_counts = counts;
   }
-  auto emit = [&](uint64_t m, const uint32_t* pre, uint32_t last) {
-    if (keep) {
-      uint32_t* dst = lv.cand_items.data() + m * k;
-      for (uint32_t j = 0; j + 1 < k; ++j) dst[j] = ior[pre[j]];
-      dst[k - 1] = ior[last];
+  const size_t T = std::min<size_t>(pool_threads() * 4, std::max<uint64_t>(1, M / 4096));
+  std::vector<uint64_t> ucut(T + 1, U);
+  ucut[0] = 0;
+  for (size_t t = 1; t < T; ++t) {  // equal candidate counts per range
+    const uint64_t target = M * t / T;
+    uint64_t lo = ucut[t - 1], hi = U;
+    while (lo < hi) {
+      const uint64_t mid = (lo + hi) / 2;
+      if (unit_begin(mid) < target) lo = mid + 1; else hi = mid;
     }
-    if (counts[m] >= theta) {
-      Lk.insert(Lk.end(), pre, pre + (k - 1));
-      Lk.push_back(last);
-      for (uint32_t j = 0; j + 1 < k; ++j) lv.freq_items.push_back(ior[pre[j]]);
-      lv.freq_items.push_back(ior[last]);
-      lv.freq_support.push_back(counts[m]);
-    }
-  };
-  if (b) {
-    const uint64_t G = b->groups();
-    for (uint64_t g = 0; g < G; ++g)
-      for (uint64_t j = b->ext_off[g]; j < b->ext_off[g + 1]; ++j) emit(j, b->prefix.data() + g * (k - 1), b->ext[j]);
-  } else {
-    const uint64_t n = bs->n_rows;
-    uint64_t m = 0;
-    for (uint32_t a = 0; a + 1 < n; ++a)
-      for (uint32_t c = a + 1; c < n; ++c, ++m) emit(m, &a, c);
+    ucut[t] = lo;
   }
-  lv.n_freq = lv.freq_support.size();
-  *n_freq = lv.n_freq;
+  std::vector<uint64_t> nf(T + 1, 0);
+  parallel_for(T, [&](size_t t) {
+    const uint64_t c0 = ucut[t] < U ? unit_begin(ucut[t]) : M, c1 = ucut[t + 1] < U ? unit_begin(ucut[t + 1]) : M;
+    uint64_t c = 0;
+    for (uint64_t m = c0; m < c1; ++m) c += counts[m] >= theta;
+    nf[t + 1] = c;
+  });
+  for (size_t t = 0; t < T; ++t) nf[t + 1] += nf[t];
+  const uint64_t F = nf[T];
+  std::vector<uint32_t> Lk(F * k);
+  lv.freq_items.resize(F * k);
+  lv.freq_support.resize(F);
+  parallel_for(T, [&](size_t t) {
+    uint64_t f = nf[t];
+    auto emit = [&](uint64_t m, const uint32_t* pre, uint32_t last) {
+      if (keep) {
+        uint32_t* dst = lv.cand_items.data() + m * k;
+        for (uint32_t j = 0; j + 1 < k; ++j) dst[j] = ior[pre[j]];
+        dst[k - 1] = ior[last];
+      }
+      if (counts[m] >= theta) {
+        uint32_t* lrow = Lk.data() + f * k;
+        uint32_t* irow = lv.freq_items.data() + f * k;
+        for (uint32_t j = 0; j + 1 < k; ++j) {
+          lrow[j] = pre[j];
+          irow[j] = ior[pre[j]];
+        }
+        lrow[k - 1] = last;
+        irow[k - 1] = ior[last];
+        lv.freq_support[f] = counts[m];
+        ++f;
+      }
+    };
+    for (uint64_t u = ucut[t]; u < ucut[t + 1]; ++u) {
+      if (b) {
+        for (uint64_t j = b->ext_off[u]; j < b->ext_off[u + 1]; ++j) emit(j, b->prefix.data() + u * (k - 1), b->ext[j]);
+      } else {
+        const uint32_t a = (uint32_t)u;
+        uint64_t m = unit_begin(u);
+        for (uint32_t c = a + 1; c < n; ++c, ++m) emit(m, &a, c);
+      }
+    }
+  });
+  lv.n_freq = F;
+  *n_freq = F;
   R->levels.push_back(std::move(lv));
   return Lk;
 }
@@ -164,7 +202,12 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     R->phase_ms[GPA_PHASE_COUNT] += t2 - t1;
 
     uint64_t n_freq = 0;
+    const double tr0 = now_ms();
     L = record_level(R, bs, k, k > 2 ? &batch : nullptr, M, counts, keep, &n_freq);
+    if (trace_enabled())
+      fprintf(stderr, "[gpa] k=%u M=%llu G=%llu: candgen %.2f ms, count phase %.2f ms (kernel %.2f), "
+              "threshold %.2f ms -> |L|=%llu\n", k, (unsigned long long)M, (unsigned long long)G, t1 - t0, t2 - t1,
+              cs.count_ms, now_ms() - tr0, (unsigned long long)n_freq);
     nL = n_freq;
     gpa_level_stats& st = R->levels.back().stats;
     st.n_cand = M;

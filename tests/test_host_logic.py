@@ -25,7 +25,7 @@ def shim(tmp_path_factory):
     subprocess.check_call(["g++", "-O2", "-std=c++17", "-shared", "-fPIC", "-pthread", "-I", CSRC, "-I",
                            os.path.join(ROOT, "include"), "-I", "/usr/local/cuda/include", "-I",
                            os.path.join(nccl, "include"), os.path.join(ROOT, "tests", "cpp", "candgen_shim.cpp"),
-                           os.path.join(CSRC, "runtime", "candgen.cpp"), "-o", str(out)])
+                           os.path.join(CSRC, "runtime", "candgen.cpp"), os.path.join(CSRC, "runtime", "pool.cpp"), "-o", str(out)])
     lib = ctypes.CDLL(str(out))
     lib.shim_candgen.restype = ctypes.c_int
     lib.shim_plan_trie.restype = ctypes.c_int
@@ -115,12 +115,16 @@ def run_plan(lib, L, n_rows):
             cand[: M * k].reshape(M, k))
 
 
-@pytest.mark.parametrize("name,k", [("mushroom", 3), ("mushroom", 5), ("chess", 4), ("random", 3), ("random", 9)])
+@pytest.mark.parametrize("name,k", [("mushroom", 3), ("mushroom", 5), ("chess", 4), ("random", 3), ("random", 9),
+                                    ("dense", 3)])
 def test_trie_plan_invariants(shim, name, k):
     """Blocks tile the candidates in order with <= 256 candidates and <= trie_max_rows(k) rows;
     local row bytes map back to each candidate's rows; lcp is the shared prefix with the previous
     candidate, reset to 0 at every warp chunk (ceil(n/8)) start -- what count_trie assumes."""
-    if name == "random":
+    if name == "dense":  # all pairs of 80 rows: 82,160 candidates -> the parallel (multi-range) plan
+        L = np.array(list(combinations(range(80), 2)), np.uint32)
+        n_rows = 80
+    elif name == "random":
         rng = np.random.default_rng(k)
         L = np.array(sorted({tuple(sorted(rng.choice(300, k - 1, replace=False))) for _ in range(6000)}), np.uint32)
         L = np.array(sorted({tuple(x) for x in L.tolist()} |
@@ -137,7 +141,7 @@ def test_trie_plan_invariants(shim, name, k):
     M = len(cand)
     if M == 0:
         return
-    rmax = 32 if k <= 8 else 64
+    rmax = 32 if 3 <= k <= 8 else 64
     pos = 0
     for cb, nc, rb, nr in blocks.tolist():
         assert cb == pos and 0 < nc <= 256 and nr <= rmax
