@@ -41,7 +41,7 @@ uint64_t launch_count_prefix(const uint32_t* rows, uint64_t pitch_words, const u
 // Transaction-tiled trie walk for generations k in [2, kTrieMaxK] (count_trie.cu).  Candidates
 // (lexicographic) are cut into blocks of <= kTrieMaxCand candidates touching <= kTrieMaxRows rows.
 constexpr uint32_t kTrieMaxK = 16;
-constexpr uint32_t kTrieWideMaxK = 8;    // 4 <= k <= 8: 8 words per lane (256-word stripes), <= 32 rows / block
+constexpr uint32_t kTrieWideMaxK = 9;    // 3 <= k <= 9: 8 words per lane (256-word stripes), <= 32 rows / block
 constexpr uint32_t kTrieMaxRows = 64;    // otherwise: 4 words per lane (128-word stripes), <= 64 rows / block
 constexpr uint32_t kTrieMaxCand = 256;
 struct TrieBlock {

@@ -96,8 +96,14 @@ __device__ __forceinline__ void trie_level(uint4 (&V)[K - 1][W], uint32_t base, 
   }
 }
 
+// Register budget: 3 CTAs (27 warps) per SM when the prefix stack is small, else 2.
 template <int K, int W>
-__global__ void __maxnreg__(112) count_trie_kernel(
+constexpr int kTrieRegs = (K - 1) * W * 4 <= 40 ? 72 : 112;
+template <int K, int W>
+constexpr uint32_t kTrieRingBytes = kTrieRegs<K, W> == 72 ? 64u * 1024u : 96u * 1024u;
+
+template <int K, int W>
+__global__ void __maxnreg__((kTrieRegs<K, W>)) count_trie_kernel(
     const uint32_t* __restrict__ rows, uint64_t pitch_words, const TrieBlock* __restrict__ blocks,
     const uint32_t* __restrict__ block_rows, const uint4* __restrict__ cand_lrows, const uint8_t* __restrict__ cand_lcp,
     uint32_t n_blocks, uint32_t n_parts, uint32_t n_stripes, uint32_t n_stages, uint32_t* __restrict__ counts) {
@@ -233,8 +239,8 @@ void launch_k(const uint32_t* rows, uint64_t pitch_words, const TrieBlock* block
   const uint32_t n_stripes = (uint32_t)(pitch_words / (128 * W));
   if (n_parts > n_stripes) n_parts = n_stripes;
   if (n_parts < 1) n_parts = 1;
-  // ring depth: as many stripes in flight as fit in ~96 KB (2 CTAs / SM), 2..kTrieMaxStages
-  uint32_t stages = (uint32_t)((96u * 1024u) / ((size_t)max_rows * kSegBytes));
+  // ring depth: as many stripes in flight as fit the ring budget (3 or 2 CTAs / SM), 2..kTrieMaxStages
+  uint32_t stages = (uint32_t)(kTrieRingBytes<K, W> / ((size_t)max_rows * kSegBytes));
   stages = stages < 2 ? 2 : (stages > kTrieMaxStages ? kTrieMaxStages : stages);
   const size_t smem = (size_t)stages * max_rows * kSegBytes;
   static bool attr = false;
@@ -264,7 +270,7 @@ uint64_t launch_count_trie(uint32_t k, const uint32_t* rows, uint64_t pitch_word
     break;
   switch (k) {
     GPA_TRIE_CASE(2, 1) GPA_TRIE_CASE(3, 2) GPA_TRIE_CASE(4, 2) GPA_TRIE_CASE(5, 2) GPA_TRIE_CASE(6, 2)
-    GPA_TRIE_CASE(7, 2) GPA_TRIE_CASE(8, 2) GPA_TRIE_CASE(9, 1) GPA_TRIE_CASE(10, 1) GPA_TRIE_CASE(11, 1)
+    GPA_TRIE_CASE(7, 2) GPA_TRIE_CASE(8, 2) GPA_TRIE_CASE(9, 2) GPA_TRIE_CASE(10, 1) GPA_TRIE_CASE(11, 1)
     GPA_TRIE_CASE(12, 1) GPA_TRIE_CASE(13, 1) GPA_TRIE_CASE(14, 1) GPA_TRIE_CASE(15, 1) GPA_TRIE_CASE(16, 1)
     default:
       fail(GPA_ERR_INVALID, "count_trie: k = %u outside [2, %u]", k, kTrieMaxK);
