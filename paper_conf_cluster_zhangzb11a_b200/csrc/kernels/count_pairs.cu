@@ -13,9 +13,9 @@
 //     complete_tx); a diagonal tile loads one box and uses it as both operands;
 //   * 8 consumer warps: thread (tx, ty) owns the 8 x 8 pairs (ty + 16 i, tx + 16 j); per
 //     16-byte slot it loads 8 A and 8 B fragments (LDS.128, conflict-free thanks to the
-//     swizzle) and does 64 x 4 AND + popcount + add into 64 register accumulators; the 4 words
-//     of a slot go through one carry-save adder so 3 POPC count 4 words (the XU pipe that runs
-//     POPC is 4x narrower than the ALU pipe that runs LOP3); diagonal tiles skip the
+//     swizzle) and does 64 x 8 AND + popcount + add into 64 register accumulators; the 8 words
+//     of two slots go through a carry-save adder tree so 4 POPC count 8 words (the XU pipe that
+//     runs POPC is 4x narrower than the ALU pipe that runs LOP3); diagonal tiles skip the
 //     micro-pairs that lie entirely below the diagonal;
 //   * epilogue: one atomicAdd per (CTA, pair a < b) into the lexicographic pair index.
 // Each loaded word feeds 128 pair-words, so the kernel is bound by the POPC pipe (16 / clk /
@@ -33,6 +33,7 @@ namespace {
 constexpr int kTile = 128;                  // rows per tile side
 constexpr int kChunkWords = 32;             // words per TMA box row (128 B = swizzle span)
 constexpr int kStages = 3;
+constexpr int kTreeRows = 5;   // micro-tile rows 0..4 use the 8-word adder tree, rows 5..7 two 4-word adders
 constexpr int kConsumerWarps = 8;
 constexpr int kThreads = (kConsumerWarps + 1) * 32;
 constexpr uint32_t kBoxBytes = kTile * kChunkWords * 4;        // 16 KB
@@ -68,6 +69,11 @@ __device__ __forceinline__ void tma_load_2d(uint32_t dst, const void* tmap, int 
       "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(dst),
       "l"(tmap), "r"(c0), "r"(c1), "r"(bar)
       : "memory");
+}
+__device__ __forceinline__ uint32_t imad(uint32_t a, uint32_t b, uint32_t c) {
+  uint32_t d;
+  asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "r"(c));
+  return d;
 }
 __device__ __forceinline__ uint4 lds128(uint32_t addr) {
   uint4 v;
@@ -136,22 +142,52 @@ __global__ void __launch_bounds__(kThreads, 1) count_pairs_kernel(const __grid_c
     const uint32_t A = buf0 + stage * kStageBytes;
     const uint32_t B = diag ? A : A + kBoxBytes;
 #pragma unroll 1
-    for (uint32_t q = 0; q < 8; ++q) {
-      uint4 a[8];
+    for (uint32_t q = 0; q < 8; q += 2) {
+      // two 16-byte slots (8 words) per pair: a 7 -> 3 carry-save adder tree plus the 8th word
+      uint4 a0[8], a1[8];
 #pragma unroll
-      for (int i = 0; i < 8; ++i) a[i] = lds128(A + (ty + 16 * i) * 128 + ((q ^ swa) << 4));
+      for (int i = 0; i < 8; ++i) {
+        a0[i] = lds128(A + (ty + 16 * i) * 128 + ((q ^ swa) << 4));
+        a1[i] = lds128(A + (ty + 16 * i) * 128 + (((q + 1) ^ swa) << 4));
+      }
 #pragma unroll
       for (int j = 0; j < 8; ++j) {
-        const uint4 b = lds128(B + (tx + 16 * j) * 128 + ((q ^ swb) << 4));
+        const uint4 b0 = lds128(B + (tx + 16 * j) * 128 + ((q ^ swb) << 4));
+        const uint4 b1 = lds128(B + (tx + 16 * j) * 128 + (((q + 1) ^ swb) << 4));
 #pragma unroll
         for (int i = 0; i < 8; ++i) {
           // diagonal tile: micro-pairs with i > j have a = ty + 16i > b = tx + 16j for every thread
           if (diag && i > j) continue;
-          // carry-save adder over 3 of the 4 AND words: popc(x)+popc(y)+popc(z) = popc(x^y^z) + 2 popc(maj(x,y,z));
-          // 3 POPC (XU pipe, 16/clk/SM) instead of 4, paid with 2 LOP3 (ALU pipe, 64/clk/SM)
-          const uint32_t x = a[i].x & b.x, y = a[i].y & b.y, z = a[i].z & b.z, w = a[i].w & b.w;
-          const uint32_t sum = x ^ y ^ z, carry = (x & y) | (z & (x ^ y));
-          acc[i][j] += __popc(sum) + __popc(w) + (__popc(carry) << 1);
+          if (i < kTreeRows) {
+            // popcount of 8 AND words with 4 POPC (XU pipe, 16/clk/SM) instead of 8, paid with
+            // 8 LOP3 (ALU pipe, 64/clk/SM): full adders (x0,x1,x2) -> (s1,c1), (x3,x4,x5) ->
+            // (s2,c2), (s1,s2,x6) -> (ones,c3), (c1,c2,c3) -> (twos,fours);
+            // total = ones + x7 + 2 twos + 4 fours
+            const uint32_t x0 = a0[i].x & b0.x, x1 = a0[i].y & b0.y, x2 = a0[i].z & b0.z, x3 = a0[i].w & b0.w;
+            const uint32_t x4 = a1[i].x & b1.x, x5 = a1[i].y & b1.y, x6 = a1[i].z & b1.z, x7 = a1[i].w & b1.w;
+            const uint32_t s1 = x0 ^ x1 ^ x2, c1 = (x0 & x1) | (x2 & (x0 ^ x1));
+            const uint32_t s2 = x3 ^ x4 ^ x5, c2 = (x3 & x4) | (x5 & (x3 ^ x4));
+            const uint32_t ones = s1 ^ s2 ^ x6, c3 = (s1 & s2) | (x6 & (s1 ^ s2));
+            const uint32_t twos = c1 ^ c2 ^ c3, fours = (c1 & c2) | (c3 & (c1 ^ c2));
+            // the accumulation runs on the FMA pipe (IMAD), leaving the ALU pipe to the LOP3s
+            acc[i][j] = imad(__popc(ones), 1u, acc[i][j]);
+            acc[i][j] = imad(__popc(x7), 1u, acc[i][j]);
+            acc[i][j] = imad(__popc(twos), 2u, acc[i][j]);
+            acc[i][j] = imad(__popc(fours), 4u, acc[i][j]);
+          } else {
+            // the other rows: one full adder per 4 words (3 POPC / 4 words) -- fewer LOP3, more
+            // POPC, so that the ALU and XU pipes are loaded evenly
+            const uint32_t x0 = a0[i].x & b0.x, x1 = a0[i].y & b0.y, x2 = a0[i].z & b0.z, x3 = a0[i].w & b0.w;
+            const uint32_t x4 = a1[i].x & b1.x, x5 = a1[i].y & b1.y, x6 = a1[i].z & b1.z, x7 = a1[i].w & b1.w;
+            const uint32_t s1 = x0 ^ x1 ^ x2, c1 = (x0 & x1) | (x2 & (x0 ^ x1));
+            const uint32_t s2 = x4 ^ x5 ^ x6, c2 = (x4 & x5) | (x6 & (x4 ^ x5));
+            acc[i][j] = imad(__popc(s1), 1u, acc[i][j]);
+            acc[i][j] = imad(__popc(x3), 1u, acc[i][j]);
+            acc[i][j] = imad(__popc(c1), 2u, acc[i][j]);
+            acc[i][j] = imad(__popc(s2), 1u, acc[i][j]);
+            acc[i][j] = imad(__popc(x7), 1u, acc[i][j]);
+            acc[i][j] = imad(__popc(c2), 2u, acc[i][j]);
+          }
         }
       }
     }
