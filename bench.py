@@ -46,6 +46,7 @@ def parse():
     p.add_argument("--config", default="t40i10d10m", choices=list(gen.CONFIGS))
     p.add_argument("--kernel", default="auto", choices=["auto", "v0", "prefix", "pairs", "trie"])
     p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--dist", action="store_true", help="use the NCCL path even with one rank")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-sample-tx", type=int, default=0, help="oracle sample size (0 = auto)")
     return p.parse_args()
@@ -96,9 +97,10 @@ class ClockSampler:
                 "reasons": reasons, "samples": len(self.samples)}
 
 
-def shard_range(n_tx: int, rank: int, world: int):
-    """Contiguous rank ranges on generator-chunk boundaries (multiples of 512 transactions)."""
-    ch = gen.chunk_size()
+def shard_range(n_tx: int, rank: int, world: int, quest: bool = True):
+    """Contiguous rank ranges: Quest data on generator-chunk boundaries (102,400 transactions,
+    so each rank generates only its own chunks), other data on 512-transaction boundaries."""
+    ch = gen.chunk_size() if quest else 512
     n_chunks = (n_tx + ch - 1) // ch
     c0 = n_chunks * rank // world
     c1 = n_chunks * (rank + 1) // world
@@ -108,7 +110,7 @@ def shard_range(n_tx: int, rank: int, world: int):
 def cpu_sample_size(cfg, requested):
     if requested:
         return requested
-    return {"t40i10d10m": 409_600, "t40i10d100k": 25_000, "accidents": 100_000}.get(cfg.name, cfg.n_tx)
+    return {"t40i10d10m": 819_200, "t40i10d100k": 25_000, "accidents": 100_000}.get(cfg.name, cfg.n_tx)
 
 
 def run_oracle_sample(cfg, n_sample):
@@ -172,12 +174,15 @@ def main():
 
     torch.cuda.set_device(local)
     dist = None
-    if world > 1:
-        tdist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    if world > 1 or args.dist:
+        if not tdist.is_initialized():
+            os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+            os.environ.setdefault("MASTER_PORT", "29531")
+            tdist.init_process_group("nccl", device_id=torch.device("cuda", local), rank=rank, world_size=world)
         dist = gpa.Dist.from_torch(local)
 
     # ---- this rank's shard of the workload (synthetic, seeded)
-    b0, b1 = shard_range(cfg.n_tx, rank, world)
+    b0, b1 = shard_range(cfg.n_tx, rank, world, cfg.kind == "quest")
     ds = gen.make(cfg.name, tx_begin=b0, tx_end=b1)
     theta = gpa.min_count(cfg.n_tx, cfg.minsup)
     kern = {"auto": gpa.KERNEL_AUTO, "v0": gpa.KERNEL_V0, "prefix": gpa.KERNEL_PREFIX,
@@ -189,12 +194,12 @@ def main():
     torch.cuda.synchronize()
 
     def barrier():
-        if world > 1:
+        if dist is not None:
             tdist.barrier(device_ids=[local])
         torch.cuda.synchronize()
 
     def max_over_ranks(x: float) -> float:
-        if world == 1:
+        if dist is None:
             return x
         t = torch.tensor([x], dtype=torch.float64, device="cuda")
         tdist.all_reduce(t, op=tdist.ReduceOp.MAX)
@@ -257,7 +262,20 @@ def main():
     dom = max(res.levels[1:], key=lambda lv: float(np.mean(level_ms[lv.k])))   # single longest launch
     roof = roof_for([dom])
     roof["kernel"] = f"count_{dom.stats['kernel_name']} (generation {dom.k}, the longest launch)"
+    # DRAM traffic per launch of this kernel from the committed ncu --set full capture
+    # (profiles/traffic.json, written from profiles/r*_ncu_*.txt); null if not captured
     roof["traffic"] = None
+    try:
+        tr = json.load(open(os.path.join(ROOT, "profiles", "traffic.json")))
+        key = {"pairs": "count_pairs_kernel", "prefix": "count_prefix_kernel"}.get(
+            dom.stats["kernel_name"], f"count_trie_kernel<{dom.k}, {2 if 3 <= dom.k <= 9 else 1}>")
+        if key in tr:
+            roof["traffic"] = tr[key]["dram_bytes"]
+            roof["traffic_unit"] = "bytes per launch (ncu dram__bytes_read.sum + dram__bytes_write.sum)"
+            # algorithmic bytes of this launch: each of the n rows read once (streaming design)
+            roof["algorithmic_bytes"] = (dom.stats["n_groups"] + 1) * (n_tx / 8) if dom.k == 2 else None
+    except Exception:
+        pass
     for r in roof_all.values():
         r.pop("peak_basis", None)
 

@@ -257,3 +257,26 @@ def test_t40i10d10m_full_size_sampled():
         ex = np.array([e for c, e in zip(sample, expect) if len(c) == k], dtype=np.uint64)
         lit = oracle.support_batch(ds.offsets, ds.items, ds.n_items, cs)
         assert np.array_equal(lit, ex), k
+
+
+def test_nccl_single_rank_dist_matches_local():
+    """The NCCL path end to end on one GPU: unique id broadcast through torch.distributed, a
+    1-rank communicator, and every all-reduce of gpa_mine (flags, N, histogram, counts)."""
+    import torch
+    import torch.distributed as tdist
+    if not tdist.is_initialized():
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        os.environ.setdefault("MASTER_PORT", "29533")
+        tdist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+    d = gpa.Dist.from_torch(0)
+    try:
+        ds = gen.make("mushroom")
+        theta = oracle.min_count(ds.n_tx, "0.20")
+        a = gpa.mine(ds, min_count=theta, dist=d, options=gpa.Options(device=0), keep_candidates=True)
+        assert_mine_equal(a, oracle.mine_ds(ds, theta))
+        with gpa.Bitset(ds, dist=d, options=gpa.Options(device=0)) as bs:
+            c = oracle.mine_ds(ds, theta).levels[2].cand
+            assert np.array_equal(bs.count(c), oracle.support_batch(ds.offsets, ds.items, ds.n_items, c).astype(np.uint32))
+    finally:
+        d.close()
+        tdist.destroy_process_group()
