@@ -35,7 +35,21 @@ __global__ void __launch_bounds__(kHistThreads) hist_validate_kernel(const uint6
     const uint64_t o0 = __ldg(offsets + t), o1 = __ldg(offsets + t + 1);
     if (o1 < o0) { my_flags |= kFlagBadOffsets; continue; }
     uint32_t prev = 0;
-    for (uint64_t j = o0; j < o1; ++j) {
+    uint64_t j = o0;
+    for (; j + 4 <= o1; j += 4) {  // 4 independent loads in flight
+      uint32_t it[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) it[u] = __ldg(items + j + u);
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        if (it[u] >= n_items) { my_flags |= kFlagBadItem; continue; }
+        if ((j + u) > o0 && it[u] <= prev) my_flags |= kFlagNonCanonical;
+        prev = it[u];
+        if (kSmem) atomicAdd(&s_hist[it[u]], 1u);
+        else atomicAdd(&hist[it[u]], 1u);
+      }
+    }
+    for (; j < o1; ++j) {
       const uint32_t it = __ldg(items + j);
       if (it >= n_items) { my_flags |= kFlagBadItem; continue; }
       if (j > o0 && it <= prev) my_flags |= kFlagNonCanonical;

@@ -20,17 +20,7 @@ void set_last_error(gpa_status st, const std::string& msg) {
 
 const char* last_error_cstr() { return t_last_error.c_str(); }
 
-bool trace_enabled() {
-  static const bool on = [] {
-    const char* e = std::getenv("GPA_TRACE");
-    return e && *e && *e != '0';
-  }();
-  return on;
-}
 
-double wall_ms() {
-  return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now().time_since_epoch()).count();
-}
 
 void fail(gpa_status st, const char* fmt, ...) {
   char buf[1024];

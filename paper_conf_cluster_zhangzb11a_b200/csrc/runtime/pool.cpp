@@ -2,6 +2,7 @@
 
 #include <algorithm>
 #include <atomic>
+#include <chrono>
 #include <condition_variable>
 #include <cstdlib>
 #include <mutex>
@@ -100,6 +101,18 @@ Pool& pool() {
 }  // namespace
 
 size_t pool_threads() { return pool().size(); }
+
+bool trace_enabled() {
+  static const bool on = [] {
+    const char* e = std::getenv("GPA_TRACE");
+    return e && *e && *e != '0';
+  }();
+  return on;
+}
+
+double wall_ms() {
+  return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now().time_since_epoch()).count();
+}
 void parallel_for(size_t n, const std::function<void(size_t)>& f) { pool().run(n, f); }
 
 }  // namespace gpa

@@ -9,4 +9,7 @@
 namespace gpa {
 size_t pool_threads();
 void parallel_for(size_t n, const std::function<void(size_t)>& f);
+// host tracing (GPA_TRACE=1) and wall clock; declared for the runtime in internal.h as well
+bool trace_enabled();
+double wall_ms();
 }  // namespace gpa
