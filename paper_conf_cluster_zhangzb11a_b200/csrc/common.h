@@ -4,6 +4,7 @@
 #include <cstdint>
 #include <cstdio>
 #include <string>
+#include <utility>
 #include <cuda_runtime.h>
 #include "gpapriori.h"
 
@@ -45,6 +46,45 @@ inline uint64_t pitch_words_for(uint64_t n_tx) {
 __host__ __device__ inline uint64_t pair_index(uint64_t a, uint64_t b, uint64_t n) {
   return a * n - a * (a + 1) / 2 + (b - a - 1);
 }
+
+// Device buffer allocated from the device's stream-ordered pool (cudaMallocAsync).  The pool's
+// release threshold is raised once per device so repeated calls reuse memory without a
+// cudaMalloc / cudaFree round trip.
+template <class T>
+struct DBuf {
+  T* p = nullptr;
+  size_t n = 0;
+  cudaStream_t s = nullptr;
+  DBuf() = default;
+  DBuf(const DBuf&) = delete;
+  DBuf& operator=(const DBuf&) = delete;
+  DBuf(DBuf&& o) noexcept { swap(o); }
+  DBuf& operator=(DBuf&& o) noexcept { reset(); swap(o); return *this; }
+  ~DBuf() { reset(); }
+  void swap(DBuf& o) noexcept { std::swap(p, o.p); std::swap(n, o.n); std::swap(s, o.s); }
+  void reset() noexcept {
+    if (p) cudaFreeAsync(p, s);
+    p = nullptr; n = 0;
+  }
+  void alloc(size_t count, cudaStream_t stream) {
+    reset();
+    s = stream;
+    n = count;
+    if (count == 0) return;
+    cudaError_t e = cudaMallocAsync(reinterpret_cast<void**>(&p), count * sizeof(T), stream);
+    if (e != cudaSuccess) {
+      p = nullptr;
+      n = 0;
+      cudaGetLastError();
+      fail(e == cudaErrorMemoryAllocation ? GPA_ERR_OOM : GPA_ERR_CUDA, "device allocation of %zu bytes failed: %s",
+           count * sizeof(T), cudaGetErrorString(e));
+    }
+  }
+  // grow-only reuse
+  void ensure(size_t count, cudaStream_t stream) {
+    if (count > n || stream != s) alloc(count, stream);
+  }
+};
 
 // Flags written by the validation/histogram kernel.
 constexpr uint32_t kFlagBadOffsets = 1u;

@@ -4,6 +4,8 @@
 #include <cstdint>
 #include <cuda_runtime.h>
 
+#include "common.h"
+
 namespace gpa {
 
 // ---- generation 1 (P13@338: "test their frequencies by scanning the transaction database")
@@ -66,5 +68,41 @@ uint64_t launch_count_trie(uint32_t k, const uint32_t* rows, uint64_t pitch_word
 bool make_pairs_tensor_map(void* tmap128, const uint32_t* rows, uint32_t n_rows, uint64_t pitch_words);
 uint64_t launch_count_pairs(const void* tmap128, uint32_t n_rows, uint64_t pitch_words, uint32_t* counts,
                             int n_sms, cudaStream_t stream);
+
+// ---- device-side level transition (candgen.cu)
+struct DeviceScratch {
+  DBuf<uint32_t> a, b, c, d, e, f, g, h, i;
+  DBuf<uint8_t> tmp;
+  uint32_t* u32a(size_t n, cudaStream_t s) { a.ensure(n ? n : 1, s); return a.p; }
+  uint32_t* u32b(size_t n, cudaStream_t s) { b.ensure(n ? n : 1, s); return b.p; }
+  uint32_t* u32c(size_t n, cudaStream_t s) { c.ensure(n ? n : 1, s); return c.p; }
+  uint32_t* u32d(size_t n, cudaStream_t s) { d.ensure(n ? n : 1, s); return d.p; }
+  uint32_t* u32e(size_t n, cudaStream_t s) { e.ensure(n ? n : 1, s); return e.p; }
+  uint32_t* u32f(size_t n, cudaStream_t s) { f.ensure(n ? n : 1, s); return f.p; }
+  uint32_t* u32g(size_t n, cudaStream_t s) { g.ensure(n ? n : 1, s); return g.p; }
+  uint32_t* u32h(size_t n, cudaStream_t s) { h.ensure(n ? n : 1, s); return h.p; }
+  uint32_t* u32i(size_t n, cudaStream_t s) { i.ensure(n ? n : 1, s); return i.p; }
+  void* get(size_t bytes, cudaStream_t s) { tmp.ensure(bytes ? bytes : 1, s); return tmp.p; }
+};
+// L_k on the device: n rows of k row ids (lexicographic) and their supports
+struct DeviceLevel {
+  uint32_t k = 0, n = 0;
+  DBuf<uint32_t> rows, sup;
+};
+// C_k on the device, grouped by (k-1)-prefix: prefix[G][k-1], ext_off[G+1], ext[M]
+struct DeviceBatch {
+  uint32_t k = 0, M = 0, G = 0;
+  DBuf<uint32_t> prefix, ext_off, ext;
+};
+// L_k = candidates of C_k with count >= theta, in order (k = 2: all pairs of n_rows rows in
+// pair_index order; k >= 3: the grouped batch prefix/ext_off/ext).  Returns |L_k| (synchronises).
+uint32_t device_threshold(const uint32_t* counts, uint32_t M, uint32_t theta, uint32_t k, uint32_t n_rows,
+                          const uint32_t* prefix, const uint32_t* ext_off, const uint32_t* ext, uint32_t G,
+                          DeviceLevel& out, DeviceScratch& scratch, int n_sms, cudaStream_t s);
+// items[i] = item_of_row[rows[i]] (row ids -> original item ids)
+void device_map_items(const uint32_t* rows, uint64_t n, const uint32_t* item_of_row, uint32_t* items, int n_sms,
+                      cudaStream_t s);
+// C_{k+1} = join + prune of L (k >= 2), grouped by k-prefix (synchronises for the sizes).
+void device_candgen(const DeviceLevel& L, DeviceBatch& out, DeviceScratch& scratch, int n_sms, cudaStream_t s);
 
 }  // namespace gpa

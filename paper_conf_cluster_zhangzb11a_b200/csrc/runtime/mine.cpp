@@ -39,86 +39,47 @@ double now_ms() {
   return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now().time_since_epoch()).count();
 }
 
-// Record generation k.  Candidates are the grouped batch b (k >= 3) or, for k = 2 (b == nullptr),
-// all pairs of the n rows in lexicographic order.  Returns L_k in row ids (lexicographic).
-// Two parallel passes over contiguous candidate ranges: count the frequent candidates of each
-// range, then write L_k, the frequent itemsets (original ids) and their supports at exact
-// offsets (no growing vectors, no concatenation).
-std::vector<uint32_t> record_level(gpa_result* R, const gpa_bitset* bs, uint32_t k, const GroupedBatch* b, uint64_t M,
-                                   const std::vector<uint32_t>& counts, bool keep, uint64_t* n_freq) {
+// Record generation k from the device-side threshold: L_k (F rows of k row ids, lexicographic)
+// and supports come back from the GPU; they are mapped to original item ids in parallel.  With
+// GPA_KEEP_CANDIDATES the whole C_k (the host batch b, or all pairs for k = 2) and its counts
+// are recorded as well.
+void record_level(gpa_result* R, const gpa_bitset* bs, uint32_t k, const GroupedBatch* b, uint64_t M,
+                  std::vector<uint32_t>&& Litems, std::vector<uint32_t>&& Lsup, bool keep,
+                  const std::vector<uint32_t>* counts) {
   gpa_level_data lv;
   lv.k = k;
   lv.n_cand = M;
   lv.kept = keep;
   const auto& ior = bs->item_of_row;
-  const uint32_t theta = (uint32_t)R->min_count;
-  const uint64_t n = bs->n_rows;
-  // outer units: groups (k >= 3) or first items a (k = 2)
-  const uint64_t U = b ? b->groups() : (n ? n - 1 : 0);
-  auto unit_begin = [&](uint64_t u) -> uint64_t { return b ? b->ext_off[u] : pair_index(u, u + 1, n); };
+  const uint64_t F = Lsup.size();
+  lv.freq_items = std::move(Litems);   // already mapped to original item ids on the device
+  lv.freq_support = std::move(Lsup);
   if (keep) {
+    lv.cand_counts = *counts;
     lv.cand_items.resize(M * k);
-    lv.cand_counts = counts;
-  }
-  const size_t T = std::min<size_t>(pool_threads() * 4, std::max<uint64_t>(1, M / 4096));
-  std::vector<uint64_t> ucut(T + 1, U);
-  ucut[0] = 0;
-  for (size_t t = 1; t < T; ++t) {  // equal candidate counts per range
-    const uint64_t target = M * t / T;
-    uint64_t lo = ucut[t - 1], hi = U;
-    while (lo < hi) {
-      const uint64_t mid = (lo + hi) / 2;
-      if (unit_begin(mid) < target) lo = mid + 1; else hi = mid;
-    }
-    ucut[t] = lo;
-  }
-  std::vector<uint64_t> nf(T + 1, 0);
-  parallel_for(T, [&](size_t t) {
-    const uint64_t c0 = ucut[t] < U ? unit_begin(ucut[t]) : M, c1 = ucut[t + 1] < U ? unit_begin(ucut[t + 1]) : M;
-    uint64_t c = 0;
-    for (uint64_t m = c0; m < c1; ++m) c += counts[m] >= theta;
-    nf[t + 1] = c;
-  });
-  for (size_t t = 0; t < T; ++t) nf[t + 1] += nf[t];
-  const uint64_t F = nf[T];
-  std::vector<uint32_t> Lk(F * k);
-  lv.freq_items.resize(F * k);
-  lv.freq_support.resize(F);
-  parallel_for(T, [&](size_t t) {
-    uint64_t f = nf[t];
-    auto emit = [&](uint64_t m, const uint32_t* pre, uint32_t last) {
-      if (keep) {
-        uint32_t* dst = lv.cand_items.data() + m * k;
-        for (uint32_t j = 0; j + 1 < k; ++j) dst[j] = ior[pre[j]];
-        dst[k - 1] = ior[last];
-      }
-      if (counts[m] >= theta) {
-        uint32_t* lrow = Lk.data() + f * k;
-        uint32_t* irow = lv.freq_items.data() + f * k;
-        for (uint32_t j = 0; j + 1 < k; ++j) {
-          lrow[j] = pre[j];
-          irow[j] = ior[pre[j]];
+    if (b) {
+      const uint64_t G = b->groups();
+      parallel_for(std::min<size_t>(pool_threads() * 2, std::max<uint64_t>(1, G / 1024)), [&](size_t t) {
+        const size_t TT = std::min<size_t>(pool_threads() * 2, std::max<uint64_t>(1, G / 1024));
+        for (uint64_t g = G * t / TT; g < G * (t + 1) / TT; ++g)
+          for (uint64_t j = b->ext_off[g]; j < b->ext_off[g + 1]; ++j) {
+            uint32_t* dst = lv.cand_items.data() + j * k;
+            for (uint32_t d = 0; d + 1 < k; ++d) dst[d] = ior[b->prefix[g * (k - 1) + d]];
+            dst[k - 1] = ior[b->ext[j]];
+          }
+      });
+    } else {
+      const uint64_t n = bs->n_rows;
+      uint64_t m = 0;
+      for (uint64_t a = 0; a + 1 < n; ++a)
+        for (uint64_t c = a + 1; c < n; ++c, ++m) {
+          lv.cand_items[2 * m] = ior[a];
+          lv.cand_items[2 * m + 1] = ior[c];
         }
-        lrow[k - 1] = last;
-        irow[k - 1] = ior[last];
-        lv.freq_support[f] = counts[m];
-        ++f;
-      }
-    };
-    for (uint64_t u = ucut[t]; u < ucut[t + 1]; ++u) {
-      if (b) {
-        for (uint64_t j = b->ext_off[u]; j < b->ext_off[u + 1]; ++j) emit(j, b->prefix.data() + u * (k - 1), b->ext[j]);
-      } else {
-        const uint32_t a = (uint32_t)u;
-        uint64_t m = unit_begin(u);
-        for (uint32_t c = a + 1; c < n; ++c, ++m) emit(m, &a, c);
-      }
     }
-  });
+  }
   lv.n_freq = F;
-  *n_freq = F;
   R->levels.push_back(std::move(lv));
-  return Lk;
 }
 
 }  // namespace
@@ -173,10 +134,17 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     R->levels.push_back(std::move(l1));
   }
 
-  std::vector<uint32_t> L;  // L_{k-1} in row ids
+  // ---- the level loop stays on the device: threshold + compaction of the counts into L_k and
+  // join + prune of C_{k+1} run as kernels (candgen.cu); only the sizes, the candidate batch (for
+  // the trie kernel's host-side plan) and L_k (for the result) cross PCIe.
+  DeviceScratch scratch;
+  DeviceLevel Ld, Ln;   // L_{k-1}, L_k on the device
+  DeviceBatch Bd;       // C_k on the device (k >= 3)
+  DBuf<uint32_t> d_ior;  // row -> original item id
+  d_ior.alloc(std::max<uint32_t>(bs->n_rows, 1), s);
+  if (bs->n_rows)
+    GPA_CUDA(cudaMemcpyAsync(d_ior.p, bs->item_of_row.data(), bs->n_rows * 4, cudaMemcpyHostToDevice, s));
   uint64_t nL = bs->n_rows;
-  for (uint32_t r = 0; r < bs->n_rows; ++r) L.push_back(r);
-
   for (uint32_t k = 2; k <= max_k && nL > 0; ++k) {
     double t0 = now_ms();
     CountStats cs;
@@ -186,32 +154,56 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
       M = (uint64_t)bs->n_rows * (bs->n_rows - 1) / 2;
       G = bs->n_rows ? bs->n_rows - 1 : 0;
     } else {
-      batch = candgen_join_prune(L, nL, k - 1);
-      M = batch.size();
-      G = batch.groups();
+      device_candgen(Ld, Bd, scratch, bs->n_sms, s);
+      M = Bd.M;
+      G = Bd.G;
+      if (M) {
+        batch.k = k;
+        batch.prefix.resize(G * (k - 1));
+        batch.ext.resize(M);
+        std::vector<uint32_t> off32(G + 1);
+        GPA_CUDA(cudaMemcpyAsync(batch.prefix.data(), Bd.prefix.p, G * (k - 1) * 4, cudaMemcpyDeviceToHost, s));
+        GPA_CUDA(cudaMemcpyAsync(off32.data(), Bd.ext_off.p, (G + 1) * 4, cudaMemcpyDeviceToHost, s));
+        GPA_CUDA(cudaMemcpyAsync(batch.ext.data(), Bd.ext.p, M * 4, cudaMemcpyDeviceToHost, s));
+        GPA_CUDA(cudaStreamSynchronize(s));
+        batch.ext_off.assign(off32.begin(), off32.end());
+      }
     }
     double t1 = now_ms();
     R->phase_ms[GPA_PHASE_CANDGEN] += t1 - t0;
     if (M == 0) break;
+    GPA_REQUIRE(M < (1ull << 32), GPA_ERR_INVALID, "generation %u has too many candidates", k);
     if (k == 2) count_all_pairs(bs, opt.count_kernel, &cs);
     else count_grouped(bs, batch, opt.count_kernel, &cs);
-    std::vector<uint32_t> counts(M);
-    GPA_CUDA(cudaMemcpyAsync(counts.data(), bs->d_counts.p, M * sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
-    GPA_CUDA(cudaStreamSynchronize(s));
     double t2 = now_ms();
     R->phase_ms[GPA_PHASE_COUNT] += t2 - t1;
 
-    uint64_t n_freq = 0;
+    const uint32_t F = device_threshold(bs->d_counts.p, (uint32_t)M, (uint32_t)min_count, k, bs->n_rows, Bd.prefix.p,
+                                        Bd.ext_off.p, Bd.ext.p, (uint32_t)G, Ln, scratch, bs->n_sms, s);
+    std::vector<uint32_t> Litems((size_t)F * k), Lsup(F), counts;
+    if (F) {
+      uint32_t* d_items = scratch.u32a((size_t)F * k, s);
+      device_map_items(Ln.rows.p, (uint64_t)F * k, d_ior.p, d_items, bs->n_sms, s);
+      GPA_CUDA(cudaMemcpyAsync(Litems.data(), d_items, (size_t)F * k * 4, cudaMemcpyDeviceToHost, s));
+      GPA_CUDA(cudaMemcpyAsync(Lsup.data(), Ln.sup.p, (size_t)F * 4, cudaMemcpyDeviceToHost, s));
+    }
+    if (keep) {
+      counts.resize(M);
+      GPA_CUDA(cudaMemcpyAsync(counts.data(), bs->d_counts.p, M * 4, cudaMemcpyDeviceToHost, s));
+    }
+    GPA_CUDA(cudaStreamSynchronize(s));
     const double tr0 = now_ms();
-    L = record_level(R, bs, k, k > 2 ? &batch : nullptr, M, counts, keep, &n_freq);
+    record_level(R, bs, k, k > 2 ? &batch : nullptr, M, std::move(Litems), std::move(Lsup), keep,
+                 keep ? &counts : nullptr);
+    std::swap(Ld, Ln);
+    nL = F;
     if (trace_enabled())
       fprintf(stderr, "[gpa] k=%u M=%llu G=%llu: candgen %.2f ms, count phase %.2f ms (kernel %.2f), "
-              "threshold %.2f ms -> |L|=%llu\n", k, (unsigned long long)M, (unsigned long long)G, t1 - t0, t2 - t1,
-              cs.count_ms, now_ms() - tr0, (unsigned long long)n_freq);
-    nL = n_freq;
+              "threshold %.2f ms (record %.2f) -> |L|=%u\n", k, (unsigned long long)M, (unsigned long long)G,
+              t1 - t0, t2 - t1, cs.count_ms, now_ms() - t2, now_ms() - tr0, F);
     gpa_level_stats& st = R->levels.back().stats;
     st.n_cand = M;
-    st.n_freq = n_freq;
+    st.n_freq = F;
     st.n_groups = G;
     st.kernel = cs.kernel;
     st.launches = cs.launches;
