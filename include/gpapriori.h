@@ -101,6 +101,8 @@ typedef struct {
 #define GPA_KERNEL_TRIE 4u     /* 2 <= k <= 16: transaction-tiled trie walk, rows staged in shared memory */
 
 #define GPA_KEEP_CANDIDATES 1u /* gpa_mine: keep every generation's (C_k, counts), not only F */
+#define GPA_HOST_CANDGEN 2u    /* gpa_mine: join + prune on the host thread pool instead of the device
+                                  (reference path; the default keeps the level transition on the GPU) */
 
 typedef struct {
   uint32_t count_kernel;       /* GPA_KERNEL_*; default GPA_KERNEL_AUTO */

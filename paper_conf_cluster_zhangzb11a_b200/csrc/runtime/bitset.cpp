@@ -30,6 +30,8 @@ void validate_options(const gpa_options& o) {
   GPA_REQUIRE(o.count_kernel <= GPA_KERNEL_TRIE, GPA_ERR_INVALID, "unknown count_kernel %u", o.count_kernel);
   GPA_REQUIRE(o.max_k <= GPA_MAX_K, GPA_ERR_INVALID, "max_k %u > GPA_MAX_K", o.max_k);
   GPA_REQUIRE(!o.reserved[0] && !o.reserved[1] && !o.reserved[2], GPA_ERR_INVALID, "reserved option fields must be 0");
+  GPA_REQUIRE((o.flags & ~(GPA_KEEP_CANDIDATES | GPA_HOST_CANDGEN)) == 0, GPA_ERR_INVALID, "unknown option flags 0x%x",
+              o.flags);
 }
 
 }  // namespace

@@ -91,6 +91,7 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
   if (opt_in) opt = *opt_in;
   GPA_REQUIRE(min_count >= 1, GPA_ERR_INVALID, "min_count must be >= 1");
   const bool keep = (opt.flags & GPA_KEEP_CANDIDATES) != 0;
+  const bool host_candgen = (opt.flags & GPA_HOST_CANDGEN) != 0;
   const uint32_t max_k = opt.max_k ? opt.max_k : GPA_MAX_K;
   GPA_REQUIRE(min_count < (1ull << 32), GPA_ERR_INVALID, "min_count must be < 2^32");
 
@@ -153,6 +154,31 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     if (k == 2) {
       M = (uint64_t)bs->n_rows * (bs->n_rows - 1) / 2;
       G = bs->n_rows ? bs->n_rows - 1 : 0;
+    } else if (host_candgen) {
+      // reference path (GPA_HOST_CANDGEN): L_{k-1} back to the host, threaded join + prune
+      // (runtime/candgen.cpp), the batch up to the device for the device-side threshold
+      std::vector<uint32_t> Lh((size_t)Ld.n * (k - 1));
+      if (Ld.n) {
+        GPA_CUDA(cudaMemcpyAsync(Lh.data(), Ld.rows.p, Lh.size() * 4, cudaMemcpyDeviceToHost, s));
+        GPA_CUDA(cudaStreamSynchronize(s));
+      }
+      batch = candgen_join_prune(Lh, Ld.n, k - 1);
+      M = batch.size();
+      G = batch.groups();
+      GPA_REQUIRE(M < (1ull << 32), GPA_ERR_INVALID, "generation %u has too many candidates", k);
+      Bd.k = k;
+      Bd.M = (uint32_t)M;
+      Bd.G = (uint32_t)G;
+      if (M) {
+        std::vector<uint32_t> off32(batch.ext_off.begin(), batch.ext_off.end());
+        Bd.prefix.ensure(std::max<size_t>(batch.prefix.size(), 1), s);
+        Bd.ext_off.ensure(G + 1, s);
+        Bd.ext.ensure(M, s);
+        GPA_CUDA(cudaMemcpyAsync(Bd.prefix.p, batch.prefix.data(), batch.prefix.size() * 4, cudaMemcpyHostToDevice, s));
+        GPA_CUDA(cudaMemcpyAsync(Bd.ext_off.p, off32.data(), (G + 1) * 4, cudaMemcpyHostToDevice, s));
+        GPA_CUDA(cudaMemcpyAsync(Bd.ext.p, batch.ext.data(), M * 4, cudaMemcpyHostToDevice, s));
+        GPA_CUDA(cudaStreamSynchronize(s));
+      }
     } else {
       device_candgen(Ld, Bd, scratch, bs->n_sms, s);
       M = Bd.M;

@@ -167,9 +167,11 @@ def test_mine_random(seed):
     theta = int(rng.integers(1, max(2, ds.n_tx // 8)))
     ref = oracle.mine_ds(ds, theta)
     for kern in (gpa.KERNEL_AUTO, gpa.KERNEL_V0, gpa.KERNEL_PREFIX, gpa.KERNEL_TRIE):
-        res = gpa.mine(ds, min_count=theta, options=gpa.Options(count_kernel=kern), keep_candidates=True)
-        assert res.n_tx == ds.n_tx
-        assert_mine_equal(res, ref)
+        for host in (False, True):
+            res = gpa.mine(ds, min_count=theta, options=gpa.Options(count_kernel=kern, host_candgen=host),
+                           keep_candidates=True)
+            assert res.n_tx == ds.n_tx
+            assert_mine_equal(res, ref)
 
 
 @pytest.mark.parametrize("name", ["chess", "mushroom", "t40i10d100k", "accidents"])
@@ -178,11 +180,15 @@ def test_mine_configs(name):
     theta = oracle.min_count(ds.n_tx, gen.CONFIGS[name].minsup)
     assert gpa.min_count(ds.n_tx, gen.CONFIGS[name].minsup) == theta
     ref = oracle.mine_ds(ds, theta)
-    kernels = [gpa.KERNEL_AUTO, gpa.KERNEL_PREFIX] + ([gpa.KERNEL_V0] if name in ("chess", "mushroom") else [])
-    # AUTO = pairs (k = 2) + trie (k >= 3); PREFIX = prefix kernel for every k
+    kernels = [gpa.KERNEL_AUTO, gpa.KERNEL_PREFIX, gpa.KERNEL_TRIE] + (
+        [gpa.KERNEL_V0] if name in ("chess", "mushroom") else [])
+    # AUTO = pairs (k = 2) + trie / prefix (k >= 3); device-side candidate generation by default,
+    # the host thread-pool join + prune as the reference path
     for kern in kernels:
         res = gpa.mine(ds, min_count=theta, options=gpa.Options(count_kernel=kern), keep_candidates=True)
         assert_mine_equal(res, ref)
+    res = gpa.mine(ds, min_count=theta, options=gpa.Options(host_candgen=True), keep_candidates=True)
+    assert_mine_equal(res, ref)
 
 
 def test_mine_device_input_equals_host_input():
@@ -280,3 +286,15 @@ def test_nccl_single_rank_dist_matches_local():
     finally:
         d.close()
         tdist.destroy_process_group()
+
+
+@pytest.mark.parametrize("host", [False, True])
+def test_mine_dense_long_runs(host):
+    """Dense DB: L_2 is (nearly) all pairs, so the join runs are long (device hash-set prune under
+    load, groups of up to ~40 siblings) and generations go deep."""
+    ds = gen.random_db(42, 6000, 44, max_len=24, p_empty=0.02)   # 10 generations, |C_6| = 24,036
+    theta = 500
+    ref = oracle.mine_ds(ds, theta)
+    res = gpa.mine(ds, min_count=theta, options=gpa.Options(host_candgen=host), keep_candidates=True)
+    assert_mine_equal(res, ref)
+    assert max(len(lv.cand) for lv in ref.levels[1:]) > 20000
