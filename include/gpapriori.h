@@ -103,6 +103,9 @@ typedef struct {
 #define GPA_KEEP_CANDIDATES 1u /* gpa_mine: keep every generation's (C_k, counts), not only F */
 #define GPA_HOST_CANDGEN 2u    /* gpa_mine: join + prune on the host thread pool instead of the device
                                   (reference path; the default keeps the level transition on the GPU) */
+#define GPA_NO_OVERLAP_INGEST 4u /* gpa_mine, host input: upload the whole database before computing
+                                  (default: upload in chunks overlapped with histogram, bitset build and
+                                  generation-2 counting) */
 
 typedef struct {
   uint32_t count_kernel;       /* GPA_KERNEL_*; default GPA_KERNEL_AUTO */

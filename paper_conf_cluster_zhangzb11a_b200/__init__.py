@@ -37,6 +37,7 @@ KERNEL_AUTO, KERNEL_V0, KERNEL_PREFIX, KERNEL_PAIRS, KERNEL_TRIE = 0, 1, 2, 3, 4
 KERNEL_NAMES = {0: "auto", 1: "v0", 2: "prefix", 3: "pairs", 4: "trie"}
 KEEP_CANDIDATES = 1
 HOST_CANDGEN = 2
+NO_OVERLAP_INGEST = 4
 MEM_HOST, MEM_DEVICE = 0, 1
 PHASES = ["upload", "histogram", "bitset", "candgen", "count", "threshold", "total"]
 STATUS = {0: "GPA_OK", 1: "GPA_ERR_INVALID", 2: "GPA_ERR_RANGE", 3: "GPA_ERR_OOM", 4: "GPA_ERR_CUDA",
@@ -136,12 +137,14 @@ class Options:
     device: int = -1
     max_k: int = 0
     host_candgen: bool = False   # join + prune on the host (reference path) instead of the device
+    overlap_ingest: bool = True  # host input: chunked upload overlapped with histogram / bitset / pairs
 
     def _c(self) -> _Options:
         o = _Options()
         lib().gpa_options_default(ctypes.byref(o))
         o.count_kernel = self.count_kernel
-        o.flags = (KEEP_CANDIDATES if self.keep_candidates else 0) | (HOST_CANDGEN if self.host_candgen else 0)
+        o.flags = ((KEEP_CANDIDATES if self.keep_candidates else 0) | (HOST_CANDGEN if self.host_candgen else 0)
+                   | (0 if self.overlap_ingest else NO_OVERLAP_INGEST))
         o.stream = self.stream or None
         o.device = self.device
         o.max_k = self.max_k
@@ -340,7 +343,7 @@ def mine(db, items=None, n_items=None, min_count: int = 1, dist: Dist | None = N
     inp = _Input(off, it, ni)
     o = options or Options()
     if keep_candidates is not None:
-        o = Options(o.count_kernel, keep_candidates, o.stream, o.device, o.max_k, o.host_candgen)
+        o = Options(o.count_kernel, keep_candidates, o.stream, o.device, o.max_k, o.host_candgen, o.overlap_ingest)
     copt = o._c()
     L = lib()
     h = ctypes.c_void_p()

@@ -11,16 +11,22 @@ namespace gpa {
 // ---- generation 1 (P13@338: "test their frequencies by scanning the transaction database")
 // Validates the CSR (offsets monotone, items < n_items, canonical order) into *flags and
 // accumulates hist[item] += 1 per (transaction, item) incidence.  hist must be zeroed.
-void launch_hist_validate(const uint64_t* offsets, const uint32_t* items, uint64_t n_tx, uint32_t n_items,
-                          uint32_t* hist, uint32_t* flags, int n_sms, cudaStream_t stream);
+// nnz = offsets[n_tx]: a transaction whose offsets leave [0, nnz] is flagged, never read.
+void launch_hist_validate(const uint64_t* offsets, const uint32_t* items, uint64_t n_tx, uint64_t nnz,
+                          uint32_t n_items, uint32_t* hist, uint32_t* flags, int n_sms, cudaStream_t stream);
+// same over transactions [tx_begin, tx_end) (offsets / items are the whole arrays)
+void launch_hist_validate_range(const uint64_t* offsets, const uint32_t* items, uint64_t tx_begin, uint64_t tx_end,
+                                uint64_t nnz, uint32_t n_items, uint32_t* hist, uint32_t* flags, int n_sms,
+                                cudaStream_t stream);
 // Same histogram for non-canonical input: an item counts once per transaction (set semantics).
-void launch_hist_dedup(const uint64_t* offsets, const uint32_t* items, uint64_t n_tx, uint32_t n_items,
+void launch_hist_dedup(const uint64_t* offsets, const uint32_t* items, uint64_t n_tx, uint64_t nnz, uint32_t n_items,
                        uint32_t* hist, int n_sms, cudaStream_t stream);
 
 // ---- static bitset (P18@755): rows[r][t/32] bit t%32 = [item_of_row[r] in t]
-void launch_bitset_build(const uint64_t* offsets, const uint32_t* items, uint64_t n_tx,
-                         const int32_t* row_of_item, uint32_t n_rows, uint64_t pitch_words, uint32_t* rows,
-                         cudaStream_t stream);
+// Transactions [tx_begin, tx_end) only (tx_begin a multiple of 512); items >= n_items are skipped.
+void launch_bitset_build(const uint64_t* offsets, const uint32_t* items, uint64_t n_tx, uint64_t nnz,
+                         const int32_t* row_of_item, uint32_t n_items, uint32_t n_rows, uint64_t pitch_words,
+                         uint32_t* rows, uint64_t tx_begin, uint64_t tx_end, cudaStream_t stream);
 
 // ---- support counting (complete intersection, P18@394-2515)
 // Paper design: one CTA per candidate, AND of all k rows, popc, block reduction.
@@ -66,8 +72,15 @@ uint64_t launch_count_trie(uint32_t k, const uint32_t* rows, uint64_t pitch_word
 // k = 2 TMA-tiled kernel: all pairs (a < b) of the n_rows rows; counts[pair_index] must be zeroed.
 // tmap: opaque 128-byte CUtensorMap built by make_pairs_tensor_map.
 bool make_pairs_tensor_map(void* tmap128, const uint32_t* rows, uint32_t n_rows, uint64_t pitch_words);
-uint64_t launch_count_pairs(const void* tmap128, uint32_t n_rows, uint64_t pitch_words, uint32_t* counts,
-                            int n_sms, cudaStream_t stream);
+// Words [word_begin, word_end) of the rows (multiples of 32); counts accumulate (atomic adds).
+uint64_t launch_count_pairs(const void* tmap128, uint32_t n_rows, uint64_t word_begin, uint64_t word_end,
+                            uint32_t* counts, int n_sms, cudaStream_t stream);
+// counts_sub[pair_index(a, b, n_sub)] = counts_all[pair_index(sel[a], sel[b], n_all)] (sel ascending)
+void launch_pairs_subset(const uint32_t* counts_all, uint32_t n_all, const uint32_t* sel, uint32_t n_sub,
+                         uint32_t* counts_sub, int n_sms, cudaStream_t stream);
+// rows_sub[r] = rows_all[sel[r]] (whole rows of pitch_words words)
+void launch_gather_rows(const uint32_t* rows_all, const uint32_t* sel, uint32_t n_sub, uint64_t pitch_words,
+                        uint32_t* rows_sub, int n_sms, cudaStream_t stream);
 
 // ---- device-side level transition (candgen.cu)
 struct DeviceScratch {

@@ -12,6 +12,7 @@
 //   shared-memory atomicOr (duplicates are harmless: OR is idempotent, so non-canonical input
 //   needs no special case), then writes every row's 64-byte segment with coalesced stores.  Every word of the output is written (padding
 //   transactions contribute no bits, so padding is zero).
+#include <algorithm>
 #include <cstdint>
 #include "../common.h"
 #include "../kernels.h"
@@ -27,11 +28,13 @@ constexpr uint32_t kRowBlock = 1024;     // rows per CTA tile: 1024 * 17 * 4 = 6
 
 __global__ void __launch_bounds__(kBuildThreads) bitset_build_kernel(const uint64_t* __restrict__ offsets,
                                                                      const uint32_t* __restrict__ items,
-                                                                     uint64_t n_tx, const int32_t* __restrict__ row_of_item,
-                                                                     uint32_t n_rows, uint32_t row_block,
+                                                                     uint64_t n_tx, uint64_t nnz,
+                                                                     const int32_t* __restrict__ row_of_item,
+                                                                     uint32_t n_items, uint32_t n_rows, uint32_t row_block,
+                                                                     uint64_t chunk0,
                                                                      uint64_t pitch_words, uint32_t* __restrict__ rows) {
   extern __shared__ uint32_t tile[];
-  const uint64_t chunk = blockIdx.x;
+  const uint64_t chunk = chunk0 + blockIdx.x;
   const uint32_t rb0 = blockIdx.y * row_block;
   const uint32_t nr = min(row_block, n_rows - rb0);
   for (uint32_t i = threadIdx.x; i < nr * kTileStride; i += blockDim.x) tile[i] = 0;
@@ -41,6 +44,7 @@ __global__ void __launch_bounds__(kBuildThreads) bitset_build_kernel(const uint6
     const uint64_t t = t0 + tl;
     if (t >= n_tx) break;
     const uint64_t o0 = __ldg(offsets + t), o1 = __ldg(offsets + t + 1);
+    if (o1 > nnz) continue;  // invalid CSR (rejected by the validation pass); never read past the items
     const uint32_t bit = 1u << (tl & 31);
     const uint32_t wcol = tl >> 5;
     uint64_t j = o0;
@@ -50,7 +54,7 @@ __global__ void __launch_bounds__(kBuildThreads) bitset_build_kernel(const uint6
 #pragma unroll
       for (int u = 0; u < 4; ++u) it[u] = __ldg(items + j + u);
 #pragma unroll
-      for (int u = 0; u < 4; ++u) r[u] = __ldg(row_of_item + it[u]);
+      for (int u = 0; u < 4; ++u) r[u] = it[u] < n_items ? __ldg(row_of_item + it[u]) : -1;
 #pragma unroll
       for (int u = 0; u < 4; ++u) {
         const uint32_t rr = (uint32_t)r[u] - rb0;   // r < 0 wraps to a huge value: skipped
@@ -58,7 +62,8 @@ __global__ void __launch_bounds__(kBuildThreads) bitset_build_kernel(const uint6
       }
     }
     for (; j < o1; ++j) {
-      const int32_t r = __ldg(row_of_item + __ldg(items + j));
+      const uint32_t it = __ldg(items + j);
+      const int32_t r = it < n_items ? __ldg(row_of_item + it) : -1;
       const uint32_t rr = (uint32_t)r - rb0;
       if (r >= 0 && rr < nr) atomicOr(&tile[rr * kTileStride + wcol], bit);
     }
@@ -73,18 +78,65 @@ __global__ void __launch_bounds__(kBuildThreads) bitset_build_kernel(const uint6
 
 }  // namespace
 
-void launch_bitset_build(const uint64_t* offsets, const uint32_t* items, uint64_t n_tx, const int32_t* row_of_item,
-                         uint32_t n_rows, uint64_t pitch_words, uint32_t* rows, cudaStream_t stream) {
-  if (n_rows == 0) return;
-  const uint64_t n_chunks = pitch_words / kChunkWords;
+void launch_bitset_build(const uint64_t* offsets, const uint32_t* items, uint64_t n_tx, uint64_t nnz,
+                         const int32_t* row_of_item,
+                         uint32_t n_items, uint32_t n_rows, uint64_t pitch_words, uint32_t* rows, uint64_t tx_begin,
+                         uint64_t tx_end, cudaStream_t stream) {
+  if (n_rows == 0 || tx_end <= tx_begin) return;
+  GPA_REQUIRE(tx_begin % kChunkTx == 0, GPA_ERR_INVALID, "bitset: range start not aligned");
+  const uint64_t c0 = tx_begin / kChunkTx;
+  // the range that ends at n_tx also writes the (zero) padding chunks up to the pitch
+  const uint64_t c1 = tx_end >= n_tx ? pitch_words / kChunkWords
+                                     : std::min<uint64_t>((tx_end + kChunkTx - 1) / kChunkTx, pitch_words / kChunkWords);
   const uint32_t rb = n_rows < kRowBlock ? n_rows : kRowBlock;
   const uint32_t n_rb = (n_rows + rb - 1) / rb;
   const size_t smem = (size_t)rb * kTileStride * sizeof(uint32_t);
   GPA_CUDA(cudaFuncSetAttribute(bitset_build_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-  GPA_REQUIRE(n_chunks < (1ull << 31), GPA_ERR_INVALID, "bitset: too many transactions");
-  dim3 grid((unsigned)n_chunks, n_rb);
-  bitset_build_kernel<<<grid, kBuildThreads, smem, stream>>>(offsets, items, n_tx, row_of_item, n_rows, rb,
+  GPA_REQUIRE(c1 - c0 < (1ull << 31), GPA_ERR_INVALID, "bitset: too many transactions");
+  dim3 grid((unsigned)(c1 - c0), n_rb);
+  bitset_build_kernel<<<grid, kBuildThreads, smem, stream>>>(offsets, items, n_tx, nnz, row_of_item, n_items, n_rows, rb, c0,
                                                              pitch_words, rows);
+  GPA_CUDA(cudaGetLastError());
+}
+
+namespace {
+__global__ void pairs_subset_kernel(const uint32_t* __restrict__ all, uint32_t n_all, const uint32_t* __restrict__ sel,
+                                    uint32_t n_sub, uint32_t* __restrict__ sub) {
+  // one warp per a, lanes over b
+  const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+  const uint32_t n_warps = (gridDim.x * blockDim.x) >> 5;
+  for (uint32_t a = warp; a + 1 < n_sub; a += n_warps) {
+    const uint64_t src0 = pair_index(sel[a], sel[a] + 1, n_all) - (sel[a] + 1);
+    const uint64_t dst0 = pair_index(a, a + 1, n_sub) - (a + 1);
+    for (uint32_t b = a + 1 + lane; b < n_sub; b += 32) sub[dst0 + b] = all[src0 + sel[b]];
+  }
+}
+__global__ void gather_rows_kernel(const uint4* __restrict__ all, const uint32_t* __restrict__ sel, uint32_t n_sub,
+                                   uint64_t pitch4, uint4* __restrict__ sub) {
+  for (uint32_t r = blockIdx.y; r < n_sub; r += gridDim.y) {
+    const uint4* src = all + (uint64_t)sel[r] * pitch4;
+    uint4* dst = sub + (uint64_t)r * pitch4;
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < pitch4; i += (uint64_t)gridDim.x * blockDim.x)
+      dst[i] = __ldg(src + i);
+  }
+}
+}  // namespace
+
+void launch_pairs_subset(const uint32_t* counts_all, uint32_t n_all, const uint32_t* sel, uint32_t n_sub,
+                         uint32_t* counts_sub, int n_sms, cudaStream_t stream) {
+  if (n_sub < 2) return;
+  pairs_subset_kernel<<<n_sms * 4, 256, 0, stream>>>(counts_all, n_all, sel, n_sub, counts_sub);
+  GPA_CUDA(cudaGetLastError());
+}
+
+void launch_gather_rows(const uint32_t* rows_all, const uint32_t* sel, uint32_t n_sub, uint64_t pitch_words,
+                        uint32_t* rows_sub, int n_sms, cudaStream_t stream) {
+  if (n_sub == 0) return;
+  const uint64_t pitch4 = pitch_words / 4;
+  unsigned gx = (unsigned)std::min<uint64_t>((pitch4 + 255) / 256, 64);
+  dim3 grid(gx, std::min<uint32_t>(n_sub, 65535));
+  gather_rows_kernel<<<grid, 256, 0, stream>>>(reinterpret_cast<const uint4*>(rows_all), sel, n_sub, pitch4,
+                                               reinterpret_cast<uint4*>(rows_sub));
   GPA_CUDA(cudaGetLastError());
 }
 

@@ -83,7 +83,7 @@ __device__ __forceinline__ uint4 lds128(uint32_t addr) {
 
 __global__ void __launch_bounds__(kThreads, 1) count_pairs_kernel(const __grid_constant__ CUtensorMap tmap,
                                                                   uint32_t n_rows, uint32_t n_blocks_side,
-                                                                  uint32_t n_tiles, uint32_t n_chunks,
+                                                                  uint32_t n_tiles, uint32_t chunk0, uint32_t n_chunks,
                                                                   uint32_t chunks_per_split,
                                                                   uint32_t* __restrict__ counts) {
   extern __shared__ uint8_t smem_raw[];
@@ -97,8 +97,8 @@ __global__ void __launch_bounds__(kThreads, 1) count_pairs_kernel(const __grid_c
   while (rem >= n_blocks_side - bi) { rem -= n_blocks_side - bi; ++bi; }
   const uint32_t bj = bi + rem;
   const bool diag = bi == bj;
-  const uint32_t c_begin = split * chunks_per_split;
-  const uint32_t c_end = min(c_begin + chunks_per_split, n_chunks);
+  const uint32_t c_begin = chunk0 + split * chunks_per_split;
+  const uint32_t c_end = min(c_begin + chunks_per_split, chunk0 + n_chunks);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
 
   if (threadIdx.x == 0) {
@@ -235,13 +235,14 @@ bool make_pairs_tensor_map(void* tmap128, const uint32_t* rows, uint32_t n_rows,
   return true;
 }
 
-uint64_t launch_count_pairs(const void* tmap128, uint32_t n_rows, uint64_t pitch_words, uint32_t* counts, int n_sms,
-                            cudaStream_t stream) {
-  if (n_rows < 2) return 0;
+uint64_t launch_count_pairs(const void* tmap128, uint32_t n_rows, uint64_t word_begin, uint64_t word_end,
+                            uint32_t* counts, int n_sms, cudaStream_t stream) {
+  if (n_rows < 2 || word_end <= word_begin) return 0;
   const uint32_t nb = (n_rows + kTile - 1) / kTile;
   const uint32_t n_tiles = nb * (nb + 1) / 2;
-  const uint32_t n_chunks = (uint32_t)(pitch_words / kChunkWords);
-  // K-split: about 4 waves of 2 resident CTAs per SM, never more splits than chunks.
+  const uint32_t chunk0 = (uint32_t)(word_begin / kChunkWords);
+  const uint32_t n_chunks = (uint32_t)((word_end - word_begin) / kChunkWords);
+  // K-split: about 4 waves of resident CTAs, never more splits than chunks.
   const uint64_t target = (uint64_t)n_sms * 2 * 4;
   uint32_t splits = (uint32_t)(target / n_tiles);
   if (splits < 1) splits = 1;
@@ -257,7 +258,8 @@ uint64_t launch_count_pairs(const void* tmap128, uint32_t n_rows, uint64_t pitch
   }
   CUtensorMap map;
   memcpy(&map, tmap128, sizeof(map));
-  count_pairs_kernel<<<(unsigned)grid, kThreads, kSmemBytes, stream>>>(map, n_rows, nb, n_tiles, n_chunks, per, counts);
+  count_pairs_kernel<<<(unsigned)grid, kThreads, kSmemBytes, stream>>>(map, n_rows, nb, n_tiles, chunk0, n_chunks, per,
+                                                                       counts);
   GPA_CUDA(cudaGetLastError());
   return grid;
 }

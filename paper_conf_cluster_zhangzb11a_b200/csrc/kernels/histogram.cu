@@ -21,7 +21,8 @@ constexpr uint32_t kHistSmemMaxItems = 48 * 1024;  // 192 KB of u32 bins
 template <bool kSmem>
 __global__ void __launch_bounds__(kHistThreads) hist_validate_kernel(const uint64_t* __restrict__ offsets,
                                                                      const uint32_t* __restrict__ items,
-                                                                     uint64_t n_tx, uint32_t n_items,
+                                                                     uint64_t tx_begin, uint64_t n_tx, uint64_t nnz,
+                                                                     uint32_t n_items,
                                                                      uint32_t* __restrict__ hist,
                                                                      uint32_t* __restrict__ flags) {
   extern __shared__ uint32_t s_hist[];
@@ -31,9 +32,9 @@ __global__ void __launch_bounds__(kHistThreads) hist_validate_kernel(const uint6
   }
   uint32_t my_flags = 0;
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  for (uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; t < n_tx; t += stride) {
+  for (uint64_t t = tx_begin + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; t < n_tx; t += stride) {
     const uint64_t o0 = __ldg(offsets + t), o1 = __ldg(offsets + t + 1);
-    if (o1 < o0) { my_flags |= kFlagBadOffsets; continue; }
+    if (o1 < o0 || o1 > nnz) { my_flags |= kFlagBadOffsets; continue; }
     uint32_t prev = 0;
     uint64_t j = o0;
     for (; j + 4 <= o1; j += 4) {  // 4 independent loads in flight
@@ -70,11 +71,12 @@ __global__ void __launch_bounds__(kHistThreads) hist_validate_kernel(const uint6
 // holds the same item (O(len^2) per transaction; only used for non-canonical input).
 __global__ void __launch_bounds__(kHistThreads) hist_dedup_kernel(const uint64_t* __restrict__ offsets,
                                                                   const uint32_t* __restrict__ items,
-                                                                  uint64_t n_tx, uint32_t n_items,
+                                                                  uint64_t n_tx, uint64_t nnz, uint32_t n_items,
                                                                   uint32_t* __restrict__ hist) {
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
   for (uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; t < n_tx; t += stride) {
     const uint64_t o0 = offsets[t], o1 = offsets[t + 1];
+    if (o1 < o0 || o1 > nnz) continue;
     for (uint64_t j = o0; j < o1; ++j) {
       const uint32_t it = items[j];
       if (it >= n_items) continue;
@@ -94,25 +96,33 @@ int grid_for(uint64_t n_tx, int n_sms) {
 
 }  // namespace
 
-void launch_hist_validate(const uint64_t* offsets, const uint32_t* items, uint64_t n_tx, uint32_t n_items,
-                          uint32_t* hist, uint32_t* flags, int n_sms, cudaStream_t stream) {
-  if (n_tx == 0) return;
-  const int grid = grid_for(n_tx, n_sms);
+void launch_hist_validate_range(const uint64_t* offsets, const uint32_t* items, uint64_t tx_begin, uint64_t tx_end,
+                                uint64_t nnz, uint32_t n_items, uint32_t* hist, uint32_t* flags, int n_sms,
+                                cudaStream_t stream) {
+  if (tx_end <= tx_begin) return;
+  const int grid = grid_for(tx_end - tx_begin, n_sms);
   if (n_items <= kHistSmemMaxItems) {
     size_t smem = (size_t)n_items * sizeof(uint32_t);
     if (smem > 48 * 1024)
       GPA_CUDA(cudaFuncSetAttribute(hist_validate_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    hist_validate_kernel<true><<<grid, kHistThreads, smem, stream>>>(offsets, items, n_tx, n_items, hist, flags);
+    hist_validate_kernel<true><<<grid, kHistThreads, smem, stream>>>(offsets, items, tx_begin, tx_end, nnz, n_items,
+                                                                     hist, flags);
   } else {
-    hist_validate_kernel<false><<<grid, kHistThreads, 0, stream>>>(offsets, items, n_tx, n_items, hist, flags);
+    hist_validate_kernel<false><<<grid, kHistThreads, 0, stream>>>(offsets, items, tx_begin, tx_end, nnz, n_items,
+                                                                   hist, flags);
   }
   GPA_CUDA(cudaGetLastError());
 }
 
-void launch_hist_dedup(const uint64_t* offsets, const uint32_t* items, uint64_t n_tx, uint32_t n_items,
+void launch_hist_validate(const uint64_t* offsets, const uint32_t* items, uint64_t n_tx, uint64_t nnz,
+                          uint32_t n_items, uint32_t* hist, uint32_t* flags, int n_sms, cudaStream_t stream) {
+  launch_hist_validate_range(offsets, items, 0, n_tx, nnz, n_items, hist, flags, n_sms, stream);
+}
+
+void launch_hist_dedup(const uint64_t* offsets, const uint32_t* items, uint64_t n_tx, uint64_t nnz, uint32_t n_items,
                        uint32_t* hist, int n_sms, cudaStream_t stream) {
   if (n_tx == 0) return;
-  hist_dedup_kernel<<<grid_for(n_tx, n_sms), kHistThreads, 0, stream>>>(offsets, items, n_tx, n_items, hist);
+  hist_dedup_kernel<<<grid_for(n_tx, n_sms), kHistThreads, 0, stream>>>(offsets, items, n_tx, nnz, n_items, hist);
   GPA_CUDA(cudaGetLastError());
 }
 

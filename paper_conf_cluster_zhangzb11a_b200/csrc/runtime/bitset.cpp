@@ -30,7 +30,7 @@ void validate_options(const gpa_options& o) {
   GPA_REQUIRE(o.count_kernel <= GPA_KERNEL_TRIE, GPA_ERR_INVALID, "unknown count_kernel %u", o.count_kernel);
   GPA_REQUIRE(o.max_k <= GPA_MAX_K, GPA_ERR_INVALID, "max_k %u > GPA_MAX_K", o.max_k);
   GPA_REQUIRE(!o.reserved[0] && !o.reserved[1] && !o.reserved[2], GPA_ERR_INVALID, "reserved option fields must be 0");
-  GPA_REQUIRE((o.flags & ~(GPA_KEEP_CANDIDATES | GPA_HOST_CANDGEN)) == 0, GPA_ERR_INVALID, "unknown option flags 0x%x",
+  GPA_REQUIRE((o.flags & ~(GPA_KEEP_CANDIDATES | GPA_HOST_CANDGEN | GPA_NO_OVERLAP_INGEST)) == 0, GPA_ERR_INVALID, "unknown option flags 0x%x",
               o.flags);
 }
 
@@ -96,6 +96,7 @@ gpa_bitset* bitset_build(const gpa_tx_csr* db, uint64_t row_min_count, const gpa
     items_dev = d_items.p;
   } else if (n_tx) {
     GPA_CUDA(cudaMemcpyAsync(&first_off, db->offsets, sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+    GPA_CUDA(cudaMemcpyAsync(&nnz, db->offsets + n_tx, sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
     GPA_CUDA(cudaStreamSynchronize(s));
     GPA_REQUIRE(first_off == 0, GPA_ERR_INVALID, "offsets[0] must be 0");
   }
@@ -113,13 +114,13 @@ gpa_bitset* bitset_build(const gpa_tx_csr* db, uint64_t row_min_count, const gpa
   GPA_CUDA(cudaMemsetAsync(d_hist.p, 0, std::max<uint32_t>(n_items, 1) * sizeof(uint32_t), s));
   GPA_CUDA(cudaMemsetAsync(d_flags.p, 0, sizeof(uint32_t), s));
   GPA_CUDA(cudaMemcpyAsync(d_ntx.p, &bs->n_tx_local, sizeof(uint64_t), cudaMemcpyHostToDevice, s));
-  launch_hist_validate(off_dev, items_dev, n_tx, n_items, d_hist.p, d_flags.p, bs->n_sms, s);
+  launch_hist_validate(off_dev, items_dev, n_tx, nnz, n_items, d_hist.p, d_flags.p, bs->n_sms, s);
   uint32_t flags = 0;
   GPA_CUDA(cudaMemcpyAsync(&flags, d_flags.p, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
   GPA_CUDA(cudaStreamSynchronize(s));
   if ((flags & kFlagNonCanonical) && !(flags & (kFlagBadItem | kFlagBadOffsets))) {
     GPA_CUDA(cudaMemsetAsync(d_hist.p, 0, n_items * sizeof(uint32_t), s));
-    launch_hist_dedup(off_dev, items_dev, n_tx, n_items, d_hist.p, bs->n_sms, s);
+    launch_hist_dedup(off_dev, items_dev, n_tx, nnz, n_items, d_hist.p, bs->n_sms, s);
   }
   allreduce_max_u32(dist, d_flags.p, 1, s);   // every rank takes the same accept / reject decision
   allreduce_sum_u32(dist, d_hist.p, n_items, s);
@@ -153,7 +154,8 @@ gpa_bitset* bitset_build(const gpa_tx_csr* db, uint64_t row_min_count, const gpa
     d_map.alloc(n_items, s);
     GPA_CUDA(cudaMemcpyAsync(d_map.p, bs->row_of_item.data(), n_items * sizeof(int32_t), cudaMemcpyHostToDevice, s));
     bs->rows.alloc((size_t)bs->n_rows * bs->pitch_words, s);
-    launch_bitset_build(off_dev, items_dev, n_tx, d_map.p, bs->n_rows, bs->pitch_words, bs->rows.p, s);
+    launch_bitset_build(off_dev, items_dev, n_tx, nnz, d_map.p, n_items, bs->n_rows, bs->pitch_words, bs->rows.p, 0,
+                        n_tx, s);
   }
   GPA_CUDA(cudaStreamSynchronize(s));
   bs->build_ms[2] = now_ms() - t2;
@@ -340,7 +342,7 @@ void count_all_pairs(gpa_bitset* bs, uint32_t kernel, CountStats* st) {
   bs->d_counts.ensure(M, s);
   GPA_CUDA(cudaMemsetAsync(bs->d_counts.p, 0, M * sizeof(uint32_t), s));
   GPA_CUDA(cudaEventRecord(bs->ev0, s));
-  launch_count_pairs(bs->tmap, bs->n_rows, bs->pitch_words, bs->d_counts.p, bs->n_sms, s);
+  launch_count_pairs(bs->tmap, bs->n_rows, 0, bs->pitch_words, bs->d_counts.p, bs->n_sms, s);
   if (st) { st->kernel = GPA_KERNEL_PAIRS; st->launches = 1; }
   finish_counts(bs, M, st);
 }

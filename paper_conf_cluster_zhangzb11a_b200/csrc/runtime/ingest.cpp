@@ -1,0 +1,274 @@
+// Overlapped ingest for host-resident input (gpa_mine end to end).
+//
+// Copying the horizontal database to the GPU (the paper's "copied ... to graphic memory",
+// P18@451/P18@755) costs as much as a third of a mining pass over PCIe.  Support counting is a
+// sum over transactions, so generation 2 can be counted chunk by chunk WHILE the next chunk of
+// transactions is still in flight: the CSR is split into ~8 transaction chunks (multiples of 8,192
+// transactions = whole bitset stripes); a copy stream uploads chunk c+1 while the compute stream
+// runs, for chunk c, the validation + histogram kernel, the static-bitset build and the tiled pair
+// kernel over the chunk's words.
+//
+// The rows of the bitset must be chosen before the global item counts are known.  After chunk 0
+// the rows are the items whose chunk-0 frequency, extrapolated, reaches half the threshold
+// (R0 -- a superset of L_1 with high probability).  At the end: if L_1 is contained in R0, the L_1
+// rows are gathered out of the R0 bitset and the L_1 pairs out of the R0 pair counts (exact:
+// counts are sums over transactions, the extra rows only cost work); otherwise the bitset is
+// rebuilt for L_1 from the device copy of the CSR and generation 2 is counted afresh.  Either way
+// the result is identical to the sequential path (same counts, same rows).
+#include <algorithm>
+
+#include "internal.h"
+#include "pool.h"
+
+namespace gpa {
+
+namespace {
+constexpr uint64_t kIngestAlign = 8192;   // transactions: one bitset stripe (256 words)
+constexpr uint32_t kIngestChunks = 8;
+}  // namespace
+
+bool ingest_overlap_eligible(const gpa_tx_csr* db) {
+  return db && db->memory == GPA_MEM_HOST && db->n_tx >= kIngestChunks * 4 * kIngestAlign && db->n_items >= 2 &&
+         db->n_items <= 16384 && db->offsets && db->items;
+}
+
+gpa_bitset* bitset_build_overlapped(const gpa_tx_csr* db, uint64_t row_min_count, const gpa_dist* dist,
+                                    const gpa_options* opt_in, bool* pairs_ready, CountStats* pair_stats) {
+  *pairs_ready = false;
+  gpa_options opt;
+  gpa_options_default(&opt);
+  if (opt_in) opt = *opt_in;
+  dist_check(dist);
+  DeviceInfo di = use_device(dist ? dist->device : opt.device);
+  auto* bs = new gpa_bitset();
+  struct Guard {
+    gpa_bitset* b;
+    ~Guard() { if (b) bitset_free(b); }
+  } guard{bs};
+  bs->device = di.device;
+  bs->n_sms = di.n_sms;
+  bs->dist = dist;
+  bs->opt = opt;
+  bs->n_items = db->n_items;
+  bs->n_tx_local = db->n_tx;
+  if (opt.stream) {
+    bs->stream = static_cast<cudaStream_t>(opt.stream);
+  } else {
+    GPA_CUDA(cudaStreamCreateWithFlags(&bs->stream, cudaStreamNonBlocking));
+    bs->own_stream = true;
+  }
+  GPA_CUDA(cudaEventCreate(&bs->ev0));
+  GPA_CUDA(cudaEventCreate(&bs->ev1));
+  GPA_CUDA(cudaEventCreate(&bs->ev2));
+  cudaStream_t s = bs->stream;
+  cudaStream_t cs = nullptr;
+  GPA_CUDA(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
+  struct StreamGuard {
+    cudaStream_t st;
+    ~StreamGuard() { if (st) { cudaStreamSynchronize(st); cudaStreamDestroy(st); } }
+  } cs_guard{cs};
+
+  const double t0 = wall_ms();
+  const uint64_t n_tx = db->n_tx;
+  const uint32_t n_items = db->n_items;
+  GPA_REQUIRE(db->offsets[0] == 0, GPA_ERR_INVALID, "offsets[0] must be 0");
+  const uint64_t nnz = db->offsets[n_tx];
+  bs->pitch_words = pitch_words_for(n_tx);
+
+  // chunk plan
+  uint64_t ct = (n_tx + kIngestChunks - 1) / kIngestChunks;
+  ct = (ct + kIngestAlign - 1) / kIngestAlign * kIngestAlign;
+  std::vector<uint64_t> cut;
+  for (uint64_t t = 0; t < n_tx; t += ct) cut.push_back(t);
+  cut.push_back(n_tx);
+  const size_t C = cut.size() - 1;
+  for (size_t c = 0; c < C; ++c)
+    GPA_REQUIRE(db->offsets[cut[c + 1]] >= db->offsets[cut[c]], GPA_ERR_INVALID, "offsets are not non-decreasing");
+
+  DBuf<uint64_t> d_off;
+  DBuf<uint32_t> d_items, d_hist, d_flags;
+  DBuf<uint64_t> d_ntx;
+  d_off.alloc(n_tx + 1, s);
+  d_items.alloc(std::max<uint64_t>(nnz, 1), s);
+  d_hist.alloc(n_items, s);
+  d_flags.alloc(1, s);
+  d_ntx.alloc(1, s);
+  GPA_CUDA(cudaMemsetAsync(d_hist.p, 0, n_items * 4, s));
+  GPA_CUDA(cudaMemsetAsync(d_flags.p, 0, 4, s));
+  GPA_CUDA(cudaMemcpyAsync(d_ntx.p, &bs->n_tx_local, 8, cudaMemcpyHostToDevice, s));
+  GPA_CUDA(cudaStreamSynchronize(s));  // the copy stream writes into these allocations
+  std::vector<cudaEvent_t> up(C, nullptr);
+  struct EvGuard {
+    std::vector<cudaEvent_t>& v;
+    ~EvGuard() { for (auto e : v) if (e) cudaEventDestroy(e); }
+  } ev_guard{up};
+  auto upload = [&](size_t c) {
+    const uint64_t a = cut[c], b = cut[c + 1];
+    const uint64_t ia = db->offsets[a], ib = db->offsets[b];
+    GPA_CUDA(cudaMemcpyAsync(d_off.p + a, db->offsets + a, (b - a + 1) * 8, cudaMemcpyHostToDevice, cs));
+    if (ib > ia) GPA_CUDA(cudaMemcpyAsync(d_items.p + ia, db->items + ia, (ib - ia) * 4, cudaMemcpyHostToDevice, cs));
+    GPA_CUDA(cudaEventCreateWithFlags(&up[c], cudaEventDisableTiming));
+    GPA_CUDA(cudaEventRecord(up[c], cs));
+  };
+
+  // ---- chunk 0: upload, histogram, choose the rows R0
+  upload(0);
+  if (C > 1) upload(1);
+  GPA_CUDA(cudaStreamWaitEvent(s, up[0], 0));
+  launch_hist_validate_range(d_off.p, d_items.p, cut[0], cut[1], nnz, n_items, d_hist.p, d_flags.p, bs->n_sms, s);
+  DBuf<uint32_t> d_h0;
+  d_h0.alloc(n_items, s);
+  GPA_CUDA(cudaMemcpyAsync(d_h0.p, d_hist.p, n_items * 4, cudaMemcpyDeviceToDevice, s));
+  DBuf<uint64_t> d_n0;
+  d_n0.alloc(1, s);
+  const uint64_t n0_local = cut[1] - cut[0];
+  GPA_CUDA(cudaMemcpyAsync(d_n0.p, &n0_local, 8, cudaMemcpyHostToDevice, s));
+  allreduce_sum_u32(dist, d_h0.p, n_items, s);  // every rank chooses the same R0
+  allreduce_sum_u64(dist, d_n0.p, 1, s);
+  allreduce_sum_u64(dist, d_ntx.p, 1, s);
+  std::vector<uint32_t> h0(n_items);
+  uint64_t n0 = 0, n_global = 0;
+  GPA_CUDA(cudaMemcpyAsync(h0.data(), d_h0.p, n_items * 4, cudaMemcpyDeviceToHost, s));
+  GPA_CUDA(cudaMemcpyAsync(&n0, d_n0.p, 8, cudaMemcpyDeviceToHost, s));
+  GPA_CUDA(cudaMemcpyAsync(&n_global, d_ntx.p, 8, cudaMemcpyDeviceToHost, s));
+  GPA_CUDA(cudaStreamSynchronize(s));
+  // R0: chunk-0 count >= half the threshold scaled to the chunk (h0 * N * 2 >= theta * n0)
+  std::vector<uint32_t> r0_items;
+  std::vector<int32_t> r0_of_item(n_items, -1);
+  for (uint32_t i = 0; i < n_items; ++i)
+    if (h0[i] > 0 && (unsigned __int128)h0[i] * n_global * 2 >= (unsigned __int128)row_min_count * n0) {
+      r0_of_item[i] = (int32_t)r0_items.size();
+      r0_items.push_back(i);
+    }
+  const uint32_t nr0 = (uint32_t)r0_items.size();
+  DBuf<int32_t> d_r0map;
+  DBuf<uint32_t> d_r0rows, d_r0pairs;
+  d_r0map.alloc(n_items, s);
+  GPA_CUDA(cudaMemcpyAsync(d_r0map.p, r0_of_item.data(), n_items * 4, cudaMemcpyHostToDevice, s));
+  const uint64_t P0 = (uint64_t)nr0 * (nr0 ? nr0 - 1 : 0) / 2;
+  alignas(64) unsigned char tmap0[128];
+  if (nr0) {
+    d_r0rows.alloc((size_t)nr0 * bs->pitch_words, s);
+    d_r0pairs.alloc(std::max<uint64_t>(P0, 1), s);
+    GPA_CUDA(cudaMemsetAsync(d_r0pairs.p, 0, std::max<uint64_t>(P0, 1) * 4, s));
+    if (nr0 >= 2) make_pairs_tensor_map(tmap0, d_r0rows.p, nr0, bs->pitch_words);
+  }
+  double pairs_ms = 0;
+  uint32_t pair_launches = 0;
+  std::vector<cudaEvent_t> pe(2 * C, nullptr);
+  struct EvGuard2 {
+    std::vector<cudaEvent_t>& v;
+    ~EvGuard2() { for (auto e : v) if (e) cudaEventDestroy(e); }
+  } pe_guard{pe};
+
+  // ---- all chunks: (upload c+1 in flight) histogram, bitset build over R0, generation-2 pairs
+  for (size_t c = 0; c < C; ++c) {
+    if (c + 2 < C) upload(c + 2);
+    if (c > 0) {
+      GPA_CUDA(cudaStreamWaitEvent(s, up[c], 0));
+      launch_hist_validate_range(d_off.p, d_items.p, cut[c], cut[c + 1], nnz, n_items, d_hist.p, d_flags.p, bs->n_sms, s);
+    }
+    if (nr0) {
+      launch_bitset_build(d_off.p, d_items.p, n_tx, nnz, d_r0map.p, n_items, nr0, bs->pitch_words, d_r0rows.p, cut[c],
+                          cut[c + 1], s);
+      if (nr0 >= 2) {
+        GPA_CUDA(cudaEventCreate(&pe[2 * c]));
+        GPA_CUDA(cudaEventCreate(&pe[2 * c + 1]));
+        GPA_CUDA(cudaEventRecord(pe[2 * c], s));
+        const uint64_t w0 = cut[c] / 32, w1 = c + 1 == C ? bs->pitch_words : cut[c + 1] / 32;
+        launch_count_pairs(tmap0, nr0, w0, w1, d_r0pairs.p, bs->n_sms, s);
+        GPA_CUDA(cudaEventRecord(pe[2 * c + 1], s));
+        ++pair_launches;
+      }
+    }
+  }
+  uint32_t flags = 0;
+  GPA_CUDA(cudaMemcpyAsync(&flags, d_flags.p, 4, cudaMemcpyDeviceToHost, s));
+  GPA_CUDA(cudaStreamSynchronize(s));
+  for (size_t c = 0; c < C; ++c)
+    if (pe[2 * c]) {
+      float ms = 0;
+      GPA_CUDA(cudaEventElapsedTime(&ms, pe[2 * c], pe[2 * c + 1]));
+      pairs_ms += ms;
+    }
+  const double t1 = wall_ms();
+  bs->build_ms[0] = t1 - t0;   // upload (overlapped with the kernels below)
+
+  // ---- global counts, validation (same rules and collectives as bitset_build)
+  if ((flags & kFlagNonCanonical) && !(flags & (kFlagBadItem | kFlagBadOffsets))) {
+    GPA_CUDA(cudaMemsetAsync(d_hist.p, 0, n_items * 4, s));
+    launch_hist_dedup(d_off.p, d_items.p, n_tx, nnz, n_items, d_hist.p, bs->n_sms, s);
+  }
+  allreduce_max_u32(dist, d_flags.p, 1, s);
+  allreduce_sum_u32(dist, d_hist.p, n_items, s);
+  if (nr0 >= 2) allreduce_sum_u32(dist, d_r0pairs.p, P0, s);
+  bs->item_counts.assign(n_items, 0);
+  GPA_CUDA(cudaMemcpyAsync(bs->item_counts.data(), d_hist.p, n_items * 4, cudaMemcpyDeviceToHost, s));
+  GPA_CUDA(cudaMemcpyAsync(&flags, d_flags.p, 4, cudaMemcpyDeviceToHost, s));
+  GPA_CUDA(cudaStreamSynchronize(s));
+  bs->n_tx_global = n_global;
+  GPA_REQUIRE(!(flags & kFlagBadOffsets), GPA_ERR_INVALID, "offsets are not non-decreasing%s",
+              dist ? " (on some rank)" : "");
+  GPA_REQUIRE(!(flags & kFlagBadItem), GPA_ERR_INVALID, "an item id is >= n_items (%u)%s", n_items,
+              dist ? " (on some rank)" : "");
+  GPA_REQUIRE(bs->n_tx_global < (1ull << 32), GPA_ERR_INVALID, "n_tx must be < 2^32 (32-bit supports)");
+  const double t2 = wall_ms();
+  bs->build_ms[1] = t2 - t1;
+
+  // ---- rows = L_1 (count >= row_min_count), ascending id
+  bs->row_of_item.assign(n_items, -1);
+  bool subset = true;
+  std::vector<uint32_t> sel;  // position of each L_1 item among the R0 rows
+  for (uint32_t i = 0; i < n_items; ++i) {
+    if (bs->item_counts[i] >= row_min_count && bs->item_counts[i] > 0) {
+      bs->row_of_item[i] = (int32_t)bs->item_of_row.size();
+      bs->item_of_row.push_back(i);
+      if (r0_of_item[i] < 0) subset = false;
+      else sel.push_back((uint32_t)r0_of_item[i]);
+    }
+  }
+  bs->n_rows = (uint32_t)bs->item_of_row.size();
+  if (bs->n_rows) {
+    bs->rows.alloc((size_t)bs->n_rows * bs->pitch_words, s);
+    if (subset) {
+      DBuf<uint32_t> d_sel;
+      d_sel.alloc(bs->n_rows, s);
+      GPA_CUDA(cudaMemcpyAsync(d_sel.p, sel.data(), bs->n_rows * 4, cudaMemcpyHostToDevice, s));
+      launch_gather_rows(d_r0rows.p, d_sel.p, bs->n_rows, bs->pitch_words, bs->rows.p, bs->n_sms, s);
+      if (bs->n_rows >= 2) {
+        const uint64_t P = (uint64_t)bs->n_rows * (bs->n_rows - 1) / 2;
+        bs->d_counts.ensure(P, s);
+        GPA_CUDA(cudaEventRecord(bs->ev0, s));
+        launch_pairs_subset(d_r0pairs.p, nr0, d_sel.p, bs->n_rows, bs->d_counts.p, bs->n_sms, s);
+        GPA_CUDA(cudaEventRecord(bs->ev1, s));
+        GPA_CUDA(cudaEventSynchronize(bs->ev1));
+        float ms = 0;
+        GPA_CUDA(cudaEventElapsedTime(&ms, bs->ev0, bs->ev1));
+        *pairs_ready = true;
+        if (pair_stats) {
+          pair_stats->kernel = GPA_KERNEL_PAIRS;
+          pair_stats->launches = pair_launches + 1;
+          pair_stats->count_ms = pairs_ms + ms;
+          pair_stats->allreduce_ms = 0;
+        }
+      }
+    } else {
+      // R0 missed a frequent item: rebuild the L_1 bitset from the device CSR (exact fallback)
+      DBuf<int32_t> d_map;
+      d_map.alloc(n_items, s);
+      GPA_CUDA(cudaMemcpyAsync(d_map.p, bs->row_of_item.data(), n_items * 4, cudaMemcpyHostToDevice, s));
+      launch_bitset_build(d_off.p, d_items.p, n_tx, nnz, d_map.p, n_items, bs->n_rows, bs->pitch_words, bs->rows.p, 0,
+                          n_tx, s);
+    }
+  }
+  GPA_CUDA(cudaStreamSynchronize(s));
+  bs->build_ms[2] = wall_ms() - t2;
+  if (trace_enabled())
+    fprintf(stderr, "[gpa] overlapped ingest: %zu chunks, R0 = %u rows, L1 = %u rows (%s), upload+hist+build+pairs "
+            "%.2f ms (pairs kernels %.2f ms), finish %.2f ms\n", C, nr0, bs->n_rows, subset ? "subset" : "rebuilt",
+            t1 - t0, pairs_ms, wall_ms() - t1);
+  guard.b = nullptr;
+  return bs;
+}
+
+}  // namespace gpa

@@ -131,6 +131,12 @@ namespace gpa {
 // Build the static bitset (histogram, rows, bitset) -- shared by gpa_bitset_create / gpa_mine.
 gpa_bitset* bitset_build(const gpa_tx_csr* db, uint64_t row_min_count, const gpa_dist* dist, const gpa_options* opt);
 void bitset_free(gpa_bitset* bs);
+// Host input, end to end: upload in transaction chunks overlapped with histogram, bitset build and
+// generation-2 pair counting (runtime/ingest.cpp).  *pairs_ready: bs->d_counts holds the L_1 pair
+// counts (pair_stats describes the kernels).
+bool ingest_overlap_eligible(const gpa_tx_csr* db);
+gpa_bitset* bitset_build_overlapped(const gpa_tx_csr* db, uint64_t row_min_count, const gpa_dist* dist,
+                                    const gpa_options* opt, bool* pairs_ready, struct CountStats* pair_stats);
 // Count a grouped batch into bs->d_counts (device, M entries, summed over ranks).
 void count_grouped(gpa_bitset* bs, const GroupedBatch& b, uint32_t kernel, CountStats* st);
 // Count all pairs of rows (lexicographic pair order) into bs->d_counts (n(n-1)/2 entries).

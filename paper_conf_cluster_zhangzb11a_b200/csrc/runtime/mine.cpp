@@ -95,7 +95,11 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
   const uint32_t max_k = opt.max_k ? opt.max_k : GPA_MAX_K;
   GPA_REQUIRE(min_count < (1ull << 32), GPA_ERR_INVALID, "min_count must be < 2^32");
 
-  gpa_bitset* bs = bitset_build(db, min_count, dist, &opt);
+  bool pairs_ready = false;
+  CountStats pair_stats;
+  const bool overlap = !(opt.flags & GPA_NO_OVERLAP_INGEST) && ingest_overlap_eligible(db);
+  gpa_bitset* bs = overlap ? bitset_build_overlapped(db, min_count, dist, &opt, &pairs_ready, &pair_stats)
+                           : bitset_build(db, min_count, dist, &opt);
   struct BsGuard {
     gpa_bitset* b;
     ~BsGuard() { bitset_free(b); }
@@ -199,7 +203,9 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     R->phase_ms[GPA_PHASE_CANDGEN] += t1 - t0;
     if (M == 0) break;
     GPA_REQUIRE(M < (1ull << 32), GPA_ERR_INVALID, "generation %u has too many candidates", k);
-    if (k == 2) count_all_pairs(bs, opt.count_kernel, &cs);
+    if (k == 2 && pairs_ready && (opt.count_kernel == GPA_KERNEL_AUTO || opt.count_kernel == GPA_KERNEL_PAIRS))
+      cs = pair_stats;  // counted during the overlapped ingest
+    else if (k == 2) count_all_pairs(bs, opt.count_kernel, &cs);
     else count_grouped(bs, batch, opt.count_kernel, &cs);
     double t2 = now_ms();
     R->phase_ms[GPA_PHASE_COUNT] += t2 - t1;

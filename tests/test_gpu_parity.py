@@ -298,3 +298,36 @@ def test_mine_dense_long_runs(host):
     res = gpa.mine(ds, min_count=theta, options=gpa.Options(host_candgen=host), keep_candidates=True)
     assert_mine_equal(res, ref)
     assert max(len(lv.cand) for lv in ref.levels[1:]) > 20000
+
+
+def test_overlapped_ingest_equals_sequential():
+    """Host input >= 262,144 transactions takes the chunked upload overlapped with histogram,
+    bitset build and generation-2 counting; results equal the sequential path and the oracle."""
+    ds = gen.make("accidents")
+    theta = oracle.min_count(ds.n_tx, "0.30")
+    ref = oracle.mine_ds(ds, theta)
+    a = gpa.mine(ds, min_count=theta, keep_candidates=True)
+    b = gpa.mine(ds, min_count=theta, options=gpa.Options(overlap_ingest=False), keep_candidates=True)
+    assert_mine_equal(a, ref)
+    assert_mine_equal(b, ref)
+
+
+def test_overlapped_ingest_row_estimate_miss():
+    """An item absent from the first chunk but frequent overall is missing from the chunk-0 row
+    estimate R0: the ingest must fall back to rebuilding the bitset (exact result either way)."""
+    rng = np.random.default_rng(9)
+    n = 300_000
+    base = rng.random((n, 12)) < 0.3
+    late = np.zeros(n, dtype=bool)
+    late[n // 2:] = rng.random(n - n // 2) < 0.6   # item 12: only in the second half, 30 % overall
+    mat = np.concatenate([base, late[:, None]], axis=1)
+    lens = mat.sum(axis=1).astype(np.uint64)
+    offsets = np.zeros(n + 1, np.uint64)
+    np.cumsum(lens, out=offsets[1:])
+    items = np.nonzero(mat)[1].astype(np.uint32)
+    ds = gen.Dataset("late", offsets, items, 13, n)
+    theta = n // 10
+    ref = oracle.mine_ds(ds, theta)
+    res = gpa.mine(ds, min_count=theta, keep_candidates=True)
+    assert (12,) in res.frequent()
+    assert_mine_equal(res, ref)
