@@ -115,7 +115,25 @@ uint32_t device_threshold(const uint32_t* counts, uint32_t M, uint32_t theta, ui
 // items[i] = item_of_row[rows[i]] (row ids -> original item ids)
 void device_map_items(const uint32_t* rows, uint64_t n, const uint32_t* item_of_row, uint32_t* items, int n_sms,
                       cudaStream_t s);
+// exclusive scan of n u32 (CUB); the total is written to *tot (device) when tot != nullptr
+void device_exclusive_scan(const uint32_t* in, uint32_t* out, uint32_t n, uint32_t* tot, DeviceScratch& scratch,
+                           cudaStream_t s);
 // C_{k+1} = join + prune of L (k >= 2), grouped by k-prefix (synchronises for the sizes).
 void device_candgen(const DeviceLevel& L, DeviceBatch& out, DeviceScratch& scratch, int n_sms, cudaStream_t s);
+
+// ---- device-side work planning (plan.cu)
+constexpr uint32_t kPlanMaxRows = 65536;   // row bitmap of the planning kernels (8 KB of shared memory)
+void launch_cand_group(const uint32_t* ext_off, uint32_t G, uint32_t* cand_group, int n_sms, cudaStream_t s);
+// R[w] = distinct rows of the candidates [windows[w].x, windows[w].x + windows[w].y)
+void launch_window_rows(const uint32_t* prefix, const uint32_t* ext, const uint32_t* cand_group, uint32_t k,
+                        uint32_t n_rows, const uint2* windows, uint32_t n_windows, uint32_t* R, cudaStream_t s);
+// per block (row_begin set, n_rows an upper bound): row list, exact n_rows, candidates' local row
+// bytes and lcp (count_trie's format)
+void launch_build_blocks(const uint32_t* prefix, const uint32_t* ext, const uint32_t* cand_group, uint32_t k,
+                         uint32_t n_rows, TrieBlock* blocks, uint32_t n_blocks, uint32_t* trows, uint4* lrows,
+                         uint8_t* lcp, cudaStream_t s);
+// write == false: n_tasks[g] = ceil(|group g| / 32); write == true: tasks at task_off
+void launch_prefix_tasks(const uint32_t* ext_off, uint32_t G, uint32_t* n_tasks, const uint32_t* task_off,
+                         PrefixTask* tasks, int n_sms, cudaStream_t s, bool write);
 
 }  // namespace gpa

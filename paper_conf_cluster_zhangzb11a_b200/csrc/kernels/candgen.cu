@@ -260,6 +260,11 @@ uint32_t device_threshold(const uint32_t* counts, uint32_t M, uint32_t theta, ui
   return F;
 }
 
+void device_exclusive_scan(const uint32_t* in, uint32_t* out, uint32_t n, uint32_t* tot, DeviceScratch& scratch,
+                           cudaStream_t s) {
+  exclusive_scan(in, out, n, tot, scratch, s);
+}
+
 void device_map_items(const uint32_t* rows, uint64_t n, const uint32_t* item_of_row, uint32_t* items, int n_sms,
                       cudaStream_t s) {
   if (n == 0) return;

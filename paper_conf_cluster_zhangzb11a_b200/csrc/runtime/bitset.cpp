@@ -176,6 +176,7 @@ void bitset_free(gpa_bitset* bs) {
   bs->d_trows.reset();
   bs->d_lrows.reset();
   bs->d_lcp.reset();
+  bs->d_cgroup.reset();
   if (bs->stream) cudaStreamSynchronize(bs->stream);
   if (bs->ev0) cudaEventDestroy(bs->ev0);
   if (bs->ev1) cudaEventDestroy(bs->ev1);
@@ -256,6 +257,119 @@ void count_trie_batch(gpa_bitset* bs, const GroupedBatch& b, CountStats* st) {
 }
 
 }  // namespace
+
+// ------------------------------------------------------------------ counting a device-resident batch
+
+bool count_device_batch(gpa_bitset* bs, DeviceBatch& B, uint32_t kernel, DeviceScratch& scratch, CountStats* st) {
+  cudaStream_t s = bs->stream;
+  const uint32_t k = B.k, M = B.M, G = B.G;
+  if (M == 0) return true;
+  if (kernel == GPA_KERNEL_V0 || bs->n_rows > kPlanMaxRows || k < 2) return false;
+  if (kernel == GPA_KERNEL_AUTO || kernel == GPA_KERNEL_PAIRS) {
+    const double sib = (double)M / (double)std::max<uint32_t>(G, 1);
+    kernel = (k <= kTrieMaxK && sib < 4.0) ? GPA_KERNEL_TRIE : GPA_KERNEL_PREFIX;
+  }
+  if (kernel == GPA_KERNEL_TRIE && k > kTrieMaxK) kernel = GPA_KERNEL_PREFIX;
+  const double tp0 = wall_ms();
+  bs->d_counts.ensure(M, s);
+  if (kernel == GPA_KERNEL_PREFIX) {
+    uint32_t* n_tasks = scratch.u32a(G, s);
+    uint32_t* task_off = scratch.u32b(G, s);
+    uint32_t* tot = scratch.u32c(1, s);
+    launch_prefix_tasks(B.ext_off.p, G, n_tasks, nullptr, nullptr, bs->n_sms, s, false);
+    device_exclusive_scan(n_tasks, task_off, G, tot, scratch, s);
+    uint32_t T = 0;
+    GPA_CUDA(cudaMemcpyAsync(&T, tot, 4, cudaMemcpyDeviceToHost, s));
+    GPA_CUDA(cudaStreamSynchronize(s));
+    bs->d_tasks.ensure(T, s);
+    launch_prefix_tasks(B.ext_off.p, G, nullptr, task_off, bs->d_tasks.p, bs->n_sms, s, true);
+    GPA_CUDA(cudaMemsetAsync(bs->d_counts.p, 0, (size_t)M * 4, s));
+    GPA_CUDA(cudaEventRecord(bs->ev0, s));
+    const uint32_t max_tasks = 1u << 20;
+    uint32_t launches = 0;
+    for (uint32_t t0 = 0; t0 < T; t0 += max_tasks) {
+      launch_count_prefix(bs->rows.p, bs->pitch_words, B.prefix.p, k - 1, B.ext.p, bs->d_tasks.p + t0,
+                          std::min(max_tasks, T - t0), bs->d_counts.p, s);
+      ++launches;
+    }
+    if (st) { st->kernel = GPA_KERNEL_PREFIX; st->launches = launches; }
+    finish_counts(bs, M, st);
+    return true;
+  }
+  // trie: windows of 256 candidates, halved until each touches <= rmax rows
+  const uint32_t rmax = trie_max_rows(k);
+  bs->d_cgroup.ensure(M, s);
+  launch_cand_group(B.ext_off.p, G, bs->d_cgroup.p, bs->n_sms, s);
+  std::vector<uint2> pending, next;
+  std::vector<TrieBlock> blocks;
+  for (uint32_t a = 0; a < M; a += kTrieMaxCand) pending.push_back(make_uint2(a, std::min(kTrieMaxCand, M - a)));
+  DBuf<uint2> d_win;
+  uint32_t passes = 0;
+  while (!pending.empty()) {
+    d_win.ensure(pending.size(), s);
+    uint32_t* R = scratch.u32d(pending.size(), s);
+    GPA_CUDA(cudaMemcpyAsync(d_win.p, pending.data(), pending.size() * sizeof(uint2), cudaMemcpyHostToDevice, s));
+    launch_window_rows(B.prefix.p, B.ext.p, bs->d_cgroup.p, k, bs->n_rows, d_win.p, (uint32_t)pending.size(), R, s);
+    std::vector<uint32_t> Rh(pending.size());
+    GPA_CUDA(cudaMemcpyAsync(Rh.data(), R, Rh.size() * 4, cudaMemcpyDeviceToHost, s));
+    GPA_CUDA(cudaStreamSynchronize(s));
+    next.clear();
+    for (size_t i = 0; i < pending.size(); ++i) {
+      const uint2 w = pending[i];
+      if (Rh[i] <= rmax) {
+        blocks.push_back(TrieBlock{w.x, w.y, 0, Rh[i]});
+      } else {  // a single candidate touches k <= 16 <= rmax rows, so halving terminates
+        next.push_back(make_uint2(w.x, w.y / 2));
+        next.push_back(make_uint2(w.x + w.y / 2, w.y - w.y / 2));
+      }
+    }
+    pending.swap(next);
+    ++passes;
+  }
+  std::sort(blocks.begin(), blocks.end(), [](const TrieBlock& a, const TrieBlock& b) { return a.cand_begin < b.cand_begin; });
+  {  // re-merge neighbours whose row counts add up within the limit (their union can only be smaller);
+     // the exact union is recomputed by build_blocks (n_rows) below
+    std::vector<TrieBlock> merged;
+    for (const auto& b : blocks) {
+      if (!merged.empty() && merged.back().n_cand + b.n_cand <= kTrieMaxCand && merged.back().n_rows + b.n_rows <= rmax) {
+        merged.back().n_cand += b.n_cand;
+        merged.back().n_rows += b.n_rows;  // upper bound until the exact count
+      } else {
+        merged.push_back(b);
+      }
+    }
+    blocks.swap(merged);
+  }
+  uint32_t rows_total = 0, max_rows = 0;
+  for (auto& b : blocks) {
+    b.row_begin = rows_total;
+    rows_total += b.n_rows;
+    max_rows = std::max(max_rows, b.n_rows);
+  }
+  const uint32_t n_blocks = (uint32_t)blocks.size();
+  bs->d_tblocks.ensure(n_blocks, s);
+  bs->d_trows.ensure(std::max<uint32_t>(rows_total, 1), s);
+  bs->d_lrows.ensure(M, s);
+  bs->d_lcp.ensure(M, s);
+  GPA_CUDA(cudaMemcpyAsync(bs->d_tblocks.p, blocks.data(), n_blocks * sizeof(TrieBlock), cudaMemcpyHostToDevice, s));
+  launch_build_blocks(B.prefix.p, B.ext.p, bs->d_cgroup.p, k, bs->n_rows, bs->d_tblocks.p, n_blocks, bs->d_trows.p,
+                      bs->d_lrows.p, bs->d_lcp.p, s);
+  const uint32_t n_stripes = (uint32_t)(bs->pitch_words / trie_stripe_words(k));
+  uint32_t n_parts = std::max<uint32_t>(1, n_stripes / 64);
+  const uint32_t want = (uint32_t)bs->n_sms * 2 * 3;
+  if ((uint64_t)n_blocks * n_parts < want) n_parts = std::min<uint32_t>(n_stripes, (want + n_blocks - 1) / n_blocks);
+  GPA_CUDA(cudaMemsetAsync(bs->d_counts.p, 0, (size_t)M * 4, s));
+  const double tp1 = wall_ms();
+  GPA_CUDA(cudaEventRecord(bs->ev0, s));
+  launch_count_trie(k, bs->rows.p, bs->pitch_words, bs->d_tblocks.p, bs->d_trows.p, bs->d_lrows.p, bs->d_lcp.p,
+                    n_blocks, max_rows, n_parts, bs->d_counts.p, s);
+  if (st) { st->kernel = GPA_KERNEL_TRIE; st->launches = 1; }
+  finish_counts(bs, M, st);
+  if (trace_enabled())
+    fprintf(stderr, "[gpa] k=%u trie (device plan, %u passes): M=%u blocks=%u max_rows=%u parts=%u plan %.2f ms, "
+            "kernel %.2f ms\n", k, passes, M, n_blocks, max_rows, n_parts, tp1 - tp0, st ? st->count_ms : -1.0);
+  return true;
+}
 
 void count_grouped(gpa_bitset* bs, const GroupedBatch& b, uint32_t kernel, CountStats* st) {
   cudaStream_t s = bs->stream;

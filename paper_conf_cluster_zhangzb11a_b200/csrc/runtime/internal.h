@@ -123,6 +123,7 @@ struct gpa_bitset {
   gpa::DBuf<uint32_t> d_trows;
   gpa::DBuf<uint4> d_lrows;
   gpa::DBuf<uint8_t> d_lcp;
+  gpa::DBuf<uint32_t> d_cgroup;      // candidate -> group (device planning)
   cudaEvent_t ev0 = nullptr, ev1 = nullptr, ev2 = nullptr;
   double build_ms[3] = {0, 0, 0};      // upload, histogram, bitset
 };
@@ -139,6 +140,9 @@ gpa_bitset* bitset_build_overlapped(const gpa_tx_csr* db, uint64_t row_min_count
                                     const gpa_options* opt, bool* pairs_ready, struct CountStats* pair_stats);
 // Count a grouped batch into bs->d_counts (device, M entries, summed over ranks).
 void count_grouped(gpa_bitset* bs, const GroupedBatch& b, uint32_t kernel, CountStats* st);
+// Count a device-resident grouped batch with device-side planning (trie blocks / prefix tasks);
+// returns false when it cannot (kernel v0, too many rows) and the host path must be used.
+bool count_device_batch(gpa_bitset* bs, DeviceBatch& B, uint32_t kernel, DeviceScratch& scratch, CountStats* st);
 // Count all pairs of rows (lexicographic pair order) into bs->d_counts (n(n-1)/2 entries).
 void count_all_pairs(gpa_bitset* bs, uint32_t kernel, CountStats* st);
 }  // namespace gpa

@@ -187,26 +187,33 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
       device_candgen(Ld, Bd, scratch, bs->n_sms, s);
       M = Bd.M;
       G = Bd.G;
-      if (M) {
-        batch.k = k;
-        batch.prefix.resize(G * (k - 1));
-        batch.ext.resize(M);
-        std::vector<uint32_t> off32(G + 1);
-        GPA_CUDA(cudaMemcpyAsync(batch.prefix.data(), Bd.prefix.p, G * (k - 1) * 4, cudaMemcpyDeviceToHost, s));
-        GPA_CUDA(cudaMemcpyAsync(off32.data(), Bd.ext_off.p, (G + 1) * 4, cudaMemcpyDeviceToHost, s));
-        GPA_CUDA(cudaMemcpyAsync(batch.ext.data(), Bd.ext.p, M * 4, cudaMemcpyDeviceToHost, s));
-        GPA_CUDA(cudaStreamSynchronize(s));
-        batch.ext_off.assign(off32.begin(), off32.end());
-      }
     }
     double t1 = now_ms();
     R->phase_ms[GPA_PHASE_CANDGEN] += t1 - t0;
     if (M == 0) break;
     GPA_REQUIRE(M < (1ull << 32), GPA_ERR_INVALID, "generation %u has too many candidates", k);
-    if (k == 2 && pairs_ready && (opt.count_kernel == GPA_KERNEL_AUTO || opt.count_kernel == GPA_KERNEL_PAIRS))
+    // the host copy of C_k is needed only for the host-planned kernels and for GPA_KEEP_CANDIDATES
+    auto fetch_batch = [&]() {
+      if (host_candgen || batch.size() == M) return;
+      batch.k = k;
+      batch.prefix.resize(G * (k - 1));
+      batch.ext.resize(M);
+      std::vector<uint32_t> off32(G + 1);
+      GPA_CUDA(cudaMemcpyAsync(batch.prefix.data(), Bd.prefix.p, G * (k - 1) * 4, cudaMemcpyDeviceToHost, s));
+      GPA_CUDA(cudaMemcpyAsync(off32.data(), Bd.ext_off.p, (G + 1) * 4, cudaMemcpyDeviceToHost, s));
+      GPA_CUDA(cudaMemcpyAsync(batch.ext.data(), Bd.ext.p, M * 4, cudaMemcpyDeviceToHost, s));
+      GPA_CUDA(cudaStreamSynchronize(s));
+      batch.ext_off.assign(off32.begin(), off32.end());
+    };
+    if (k == 2 && pairs_ready && (opt.count_kernel == GPA_KERNEL_AUTO || opt.count_kernel == GPA_KERNEL_PAIRS)) {
       cs = pair_stats;  // counted during the overlapped ingest
-    else if (k == 2) count_all_pairs(bs, opt.count_kernel, &cs);
-    else count_grouped(bs, batch, opt.count_kernel, &cs);
+    } else if (k == 2) {
+      count_all_pairs(bs, opt.count_kernel, &cs);
+    } else if (!count_device_batch(bs, Bd, opt.count_kernel, scratch, &cs)) {
+      fetch_batch();
+      count_grouped(bs, batch, opt.count_kernel, &cs);
+    }
+    if (keep && k > 2) fetch_batch();
     double t2 = now_ms();
     R->phase_ms[GPA_PHASE_COUNT] += t2 - t1;
 
