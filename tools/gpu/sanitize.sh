@@ -10,6 +10,12 @@ for name in ["chess", "mushroom"]:
     for kern in (gpa.KERNEL_AUTO, gpa.KERNEL_V0, gpa.KERNEL_PREFIX, gpa.KERNEL_TRIE):
         r = gpa.mine(ds, min_count=th, options=gpa.Options(count_kernel=kern, max_k=6))
         print(name, kern, len(r.frequent()))
+# overlapped ingest (host input >= 262,144 transactions) and the device level transition
+ds = gen.random_db(5, 270000, 40, max_len=12)
+r = gpa.mine(ds, min_count=5000, keep_candidates=True)
+print("overlap", len(r.frequent()))
+r = gpa.mine(ds, min_count=5000, options=gpa.Options(host_candgen=True, overlap_ingest=False))
+print("host", len(r.frequent()))
 ds = gen.random_db(3, 20000, 300, max_len=40, duplicates=True, unsorted=True)
 with gpa.Bitset(ds) as bs:
     rows = bs.rows()
