@@ -127,6 +127,16 @@ void launch_cand_group(const uint32_t* ext_off, uint32_t G, uint32_t* cand_group
 // R[w] = distinct rows of the candidates [windows[w].x, windows[w].x + windows[w].y)
 void launch_window_rows(const uint32_t* prefix, const uint32_t* ext, const uint32_t* cand_group, uint32_t k,
                         uint32_t n_rows, const uint2* windows, uint32_t n_windows, uint32_t* R, cudaStream_t s);
+// greedy partition of each window of `window` candidates into blocks of <= rmax distinct rows:
+// recs[w * window + i] = {first candidate, count, rows}, n_recs[w] = number of blocks of window w
+void launch_window_greedy(const uint32_t* prefix, const uint32_t* ext, const uint32_t* cand_group, uint32_t k,
+                          uint32_t n_rows, uint32_t M, uint32_t window, uint32_t rmax, uint3* recs, uint32_t* n_recs,
+                          cudaStream_t s);
+// blocks[off[w] + i] = record i of window w (row_begin left 0), rows[] = their row counts,
+// stats[0] = max(rows) (must be zeroed); then row_begin[b] = row_off[b]
+void launch_compact_blocks(const uint3* recs, const uint32_t* n_recs, const uint32_t* off, uint32_t n_win,
+                           uint32_t window, TrieBlock* blocks, uint32_t* rows, uint32_t* stats, cudaStream_t s);
+void launch_row_begin(const uint32_t* row_off, uint32_t n_blocks, TrieBlock* blocks, int n_sms, cudaStream_t s);
 // per block (row_begin set, n_rows an upper bound): row list, exact n_rows, candidates' local row
 // bytes and lcp (count_trie's format)
 void launch_build_blocks(const uint32_t* prefix, const uint32_t* ext, const uint32_t* cand_group, uint32_t k,

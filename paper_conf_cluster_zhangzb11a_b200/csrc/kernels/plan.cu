@@ -55,6 +55,59 @@ __global__ void window_rows_kernel(const uint32_t* __restrict__ prefix, const ui
   if (threadIdx.x == 0) R[blockIdx.x] = s_cnt;
 }
 
+// Greedy block partition of each window of <= 256 consecutive candidates (one CTA per window; the
+// walk is sequential like the host plan_trie, rows tracked in a shared-memory bitmap): a block is
+// closed when the next candidate would bring it over rmax distinct rows.  Writes up to 256 block
+// records per window (x = first candidate, y = count, z = distinct rows) and their number.
+__global__ void window_greedy_kernel(const uint32_t* __restrict__ prefix, const uint32_t* __restrict__ ext,
+                                     const uint32_t* __restrict__ cand_group, uint32_t k, uint32_t n_rows, uint32_t M,
+                                     uint32_t window, uint32_t rmax, uint3* recs, uint32_t* n_recs) {
+  __shared__ uint32_t bm[kMaxBitmapWords];
+  __shared__ uint32_t items[kTrieMaxCand * kTrieMaxK];   // the window's candidates, staged cooperatively
+  const uint32_t nw = (n_rows + 31) / 32;
+  const uint32_t c0 = blockIdx.x * window, c1 = min(c0 + window, M);
+  for (uint32_t i = threadIdx.x; i < nw; i += blockDim.x) bm[i] = 0;
+  for (uint32_t i = threadIdx.x; i < (c1 - c0) * k; i += blockDim.x)
+    items[i] = cand_item(prefix, ext, cand_group, k - 1, c0 + i / k, i % k);
+  __syncthreads();
+  if (threadIdx.x != 0) return;
+  uint32_t n = 0, start = c0, rows = 0;
+  for (uint32_t m = c0; m < c1; ++m) {
+    const uint32_t* cur = items + (m - c0) * k;
+    uint32_t fresh = 0;
+    for (uint32_t d = 0; d < k; ++d) fresh += !((bm[cur[d] >> 5] >> (cur[d] & 31)) & 1u);
+    if (rows + fresh > rmax) {  // close [start, m)
+      recs[(uint64_t)blockIdx.x * window + n++] = make_uint3(start, m - start, rows);
+      for (uint32_t i = 0; i < nw; ++i) bm[i] = 0;
+      start = m;
+      rows = 0;
+      fresh = k;
+    }
+    for (uint32_t d = 0; d < k; ++d) bm[cur[d] >> 5] |= 1u << (cur[d] & 31);
+    rows += fresh;
+  }
+  if (c1 > start) recs[(uint64_t)blockIdx.x * window + n++] = make_uint3(start, c1 - start, rows);
+  n_recs[blockIdx.x] = n;
+}
+
+// Compact the per-window records into the block table (row_begin filled later); rows[b] = the
+// block's distinct rows; stats[0] = max rows over blocks (atomicMax)
+__global__ void compact_blocks_kernel(const uint3* __restrict__ recs, const uint32_t* __restrict__ n_recs,
+                                      const uint32_t* __restrict__ off, uint32_t n_win, uint32_t window,
+                                      TrieBlock* blocks, uint32_t* rows, uint32_t* stats) {
+  for (uint32_t w = blockIdx.x; w < n_win; w += gridDim.x)
+    for (uint32_t i = threadIdx.x; i < n_recs[w]; i += blockDim.x) {
+      const uint3 r = recs[(uint64_t)w * window + i];
+      blocks[off[w] + i] = TrieBlock{r.x, r.y, 0, r.z};
+      rows[off[w] + i] = r.z;
+      atomicMax(&stats[0], r.z);
+    }
+}
+__global__ void row_begin_kernel(const uint32_t* __restrict__ row_off, uint32_t n_blocks, TrieBlock* blocks) {
+  for (uint32_t b = blockIdx.x * blockDim.x + threadIdx.x; b < n_blocks; b += gridDim.x * blockDim.x)
+    blocks[b].row_begin = row_off[b];
+}
+
 // One CTA per final block: row list, local row bytes and lcp of its candidates.
 __global__ void build_blocks_kernel(const uint32_t* __restrict__ prefix, const uint32_t* __restrict__ ext,
                                     const uint32_t* __restrict__ cand_group, uint32_t k, uint32_t n_rows,
@@ -140,6 +193,28 @@ void launch_window_rows(const uint32_t* prefix, const uint32_t* ext, const uint3
                         uint32_t n_rows, const uint2* windows, uint32_t n_windows, uint32_t* R, cudaStream_t s) {
   if (n_windows == 0) return;
   window_rows_kernel<<<n_windows, kThreads, 0, s>>>(prefix, ext, cand_group, k, n_rows, windows, R);
+  GPA_CUDA(cudaGetLastError());
+}
+
+void launch_window_greedy(const uint32_t* prefix, const uint32_t* ext, const uint32_t* cand_group, uint32_t k,
+                          uint32_t n_rows, uint32_t M, uint32_t window, uint32_t rmax, uint3* recs, uint32_t* n_recs,
+                          cudaStream_t s) {
+  if (M == 0) return;
+  const uint32_t n_win = (M + window - 1) / window;
+  window_greedy_kernel<<<n_win, 64, 0, s>>>(prefix, ext, cand_group, k, n_rows, M, window, rmax, recs, n_recs);
+  GPA_CUDA(cudaGetLastError());
+}
+
+void launch_compact_blocks(const uint3* recs, const uint32_t* n_recs, const uint32_t* off, uint32_t n_win,
+                           uint32_t window, TrieBlock* blocks, uint32_t* rows, uint32_t* stats, cudaStream_t s) {
+  if (n_win == 0) return;
+  compact_blocks_kernel<<<n_win < 4096 ? n_win : 4096, 64, 0, s>>>(recs, n_recs, off, n_win, window, blocks, rows, stats);
+  GPA_CUDA(cudaGetLastError());
+}
+
+void launch_row_begin(const uint32_t* row_off, uint32_t n_blocks, TrieBlock* blocks, int n_sms, cudaStream_t s) {
+  if (n_blocks == 0) return;
+  row_begin_kernel<<<grid_for(n_blocks, n_sms), kThreads, 0, s>>>(row_off, n_blocks, blocks);
   GPA_CUDA(cudaGetLastError());
 }
 

@@ -296,62 +296,38 @@ bool count_device_batch(gpa_bitset* bs, DeviceBatch& B, uint32_t kernel, DeviceS
     finish_counts(bs, M, st);
     return true;
   }
-  // trie: windows of 256 candidates, halved until each touches <= rmax rows
+  // trie: greedy blocks inside windows of 256 candidates (one CTA per window), one sync
   const uint32_t rmax = trie_max_rows(k);
   bs->d_cgroup.ensure(M, s);
   launch_cand_group(B.ext_off.p, G, bs->d_cgroup.p, bs->n_sms, s);
-  std::vector<uint2> pending, next;
-  std::vector<TrieBlock> blocks;
-  for (uint32_t a = 0; a < M; a += kTrieMaxCand) pending.push_back(make_uint2(a, std::min(kTrieMaxCand, M - a)));
-  DBuf<uint2> d_win;
-  uint32_t passes = 0;
-  while (!pending.empty()) {
-    d_win.ensure(pending.size(), s);
-    uint32_t* R = scratch.u32d(pending.size(), s);
-    GPA_CUDA(cudaMemcpyAsync(d_win.p, pending.data(), pending.size() * sizeof(uint2), cudaMemcpyHostToDevice, s));
-    launch_window_rows(B.prefix.p, B.ext.p, bs->d_cgroup.p, k, bs->n_rows, d_win.p, (uint32_t)pending.size(), R, s);
-    std::vector<uint32_t> Rh(pending.size());
-    GPA_CUDA(cudaMemcpyAsync(Rh.data(), R, Rh.size() * 4, cudaMemcpyDeviceToHost, s));
-    GPA_CUDA(cudaStreamSynchronize(s));
-    next.clear();
-    for (size_t i = 0; i < pending.size(); ++i) {
-      const uint2 w = pending[i];
-      if (Rh[i] <= rmax) {
-        blocks.push_back(TrieBlock{w.x, w.y, 0, Rh[i]});
-      } else {  // a single candidate touches k <= 16 <= rmax rows, so halving terminates
-        next.push_back(make_uint2(w.x, w.y / 2));
-        next.push_back(make_uint2(w.x + w.y / 2, w.y - w.y / 2));
-      }
-    }
-    pending.swap(next);
-    ++passes;
-  }
-  std::sort(blocks.begin(), blocks.end(), [](const TrieBlock& a, const TrieBlock& b) { return a.cand_begin < b.cand_begin; });
-  {  // re-merge neighbours whose row counts add up within the limit (their union can only be smaller);
-     // the exact union is recomputed by build_blocks (n_rows) below
-    std::vector<TrieBlock> merged;
-    for (const auto& b : blocks) {
-      if (!merged.empty() && merged.back().n_cand + b.n_cand <= kTrieMaxCand && merged.back().n_rows + b.n_rows <= rmax) {
-        merged.back().n_cand += b.n_cand;
-        merged.back().n_rows += b.n_rows;  // upper bound until the exact count
-      } else {
-        merged.push_back(b);
-      }
-    }
-    blocks.swap(merged);
-  }
-  uint32_t rows_total = 0, max_rows = 0;
-  for (auto& b : blocks) {
-    b.row_begin = rows_total;
-    rows_total += b.n_rows;
-    max_rows = std::max(max_rows, b.n_rows);
-  }
-  const uint32_t n_blocks = (uint32_t)blocks.size();
-  bs->d_tblocks.ensure(n_blocks, s);
+  const uint32_t window = kTrieMaxCand;
+  const uint32_t n_win = (M + window - 1) / window;
+  DBuf<uint3> d_recs;
+  d_recs.alloc((size_t)n_win * window, s);
+  uint32_t* d_nrec = scratch.u32d(n_win, s);
+  launch_window_greedy(B.prefix.p, B.ext.p, bs->d_cgroup.p, k, bs->n_rows, M, window, rmax, d_recs.p, d_nrec, s);
+  // block table on the device: scan of blocks per window, compaction, scan of rows per block
+  uint32_t* d_woff = scratch.u32e(n_win, s);
+  uint32_t* d_stats = scratch.u32f(4, s);   // [0] max rows, [1] #blocks, [2] #rows
+  GPA_CUDA(cudaMemsetAsync(d_stats, 0, 16, s));
+  device_exclusive_scan(d_nrec, d_woff, n_win, d_stats + 1, scratch, s);
+  const uint32_t max_blocks = M;  // every block holds >= 1 candidate
+  bs->d_tblocks.ensure(max_blocks, s);
+  uint32_t* d_brows = scratch.u32g(max_blocks, s);
+  uint32_t* d_roff = scratch.u32h(max_blocks, s);
+  launch_compact_blocks(d_recs.p, d_nrec, d_woff, n_win, window, bs->d_tblocks.p, d_brows, d_stats, s);
+  uint32_t st3[3] = {0, 0, 0};
+  GPA_CUDA(cudaMemcpyAsync(st3, d_stats, 12, cudaMemcpyDeviceToHost, s));
+  GPA_CUDA(cudaStreamSynchronize(s));
+  const uint32_t n_blocks = st3[1], max_rows = st3[0];
+  device_exclusive_scan(d_brows, d_roff, n_blocks, d_stats + 2, scratch, s);
+  launch_row_begin(d_roff, n_blocks, bs->d_tblocks.p, bs->n_sms, s);
+  const uint32_t passes = 1;
+  // total rows <= n_blocks * rmax
+  const uint32_t rows_total = n_blocks * rmax;
   bs->d_trows.ensure(std::max<uint32_t>(rows_total, 1), s);
   bs->d_lrows.ensure(M, s);
   bs->d_lcp.ensure(M, s);
-  GPA_CUDA(cudaMemcpyAsync(bs->d_tblocks.p, blocks.data(), n_blocks * sizeof(TrieBlock), cudaMemcpyHostToDevice, s));
   launch_build_blocks(B.prefix.p, B.ext.p, bs->d_cgroup.p, k, bs->n_rows, bs->d_tblocks.p, n_blocks, bs->d_trows.p,
                       bs->d_lrows.p, bs->d_lcp.p, s);
   const uint32_t n_stripes = (uint32_t)(bs->pitch_words / trie_stripe_words(k));
