@@ -126,6 +126,9 @@ __global__ void run_bound_kernel(const uint32_t* __restrict__ flags, const uint3
 
 // join + prune of member x with its later run siblings; EMIT = false counts survivors, EMIT = true
 // writes group x (prefix = L[x]) and its extensions at the scanned offsets
+// Join + prune of member x with its later run siblings, one WARP per x: lane j tests sibling
+// y = x + 1 + j (+32 ...); EMIT = false counts survivors, EMIT = true writes group x (prefix = L[x])
+// and its extensions, in sibling order, at the scanned offsets (warp ballot ranks the survivors).
 template <bool EMIT>
 __global__ void join_kernel(const uint32_t* __restrict__ L, uint32_t n, uint32_t w, const uint32_t* __restrict__ flags,
                             const uint32_t* __restrict__ run_ex, const uint32_t* __restrict__ bound,
@@ -134,53 +137,61 @@ __global__ void join_kernel(const uint32_t* __restrict__ L, uint32_t n, uint32_t
                             uint32_t* prefix, uint32_t* ext_off, uint32_t* ext) {
   uint32_t probe[GPA_MAX_K];
   uint64_t A[GPA_MAX_K], B[GPA_MAX_K];
-  for (uint32_t x = blockIdx.x * blockDim.x + threadIdx.x; x < n; x += gridDim.x * blockDim.x) {
-    if (EMIT && cnt[x] == 0) continue;
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, n_warps = (gridDim.x * blockDim.x) >> 5;
+  for (uint32_t x = warp; x < n; x += n_warps) {
+    if (EMIT && cnt[x] == 0) continue;  // warp-uniform
     // run index of x = (#run starts <= x) - 1
     const uint32_t r = run_ex[x] + flags[x] - 1;
     const uint32_t end = bound[r + 1];  // bound[n_runs] = n (sentinel)
+    if (!EMIT && end == x + 1) {
+      if (lane == 0) cnt[x] = 0;
+      continue;
+    }
     const uint32_t* px = L + (uint64_t)x * w;
     // subset "px without item d, then b": A[d] = sum_{i<d} (x_i+1) P^i,
     // B[d] = sum_{i>d} (x_i+1) P^(i-1); b lands at position w-1
     uint64_t pw = 1, acc = 0;
-    for (uint32_t i = 0; i < w; ++i) {  // A[i] = sum_{t<i} (x_t+1) P^t ; B[i] temporarily holds P^i
+    for (uint32_t i = 0; i < w; ++i) {  // B[i] temporarily holds P^i
       A[i] = acc;
       B[i] = pw;
       acc += (uint64_t)(px[i] + 1) * pw;
       pw *= kHashP;
     }
     const uint64_t p_last = B[w - 1];  // P^(w-1)
-    uint64_t suf = 0;                  // B[d] = sum_{i>d} (x_i+1) P^(i-1), built from the top
+    uint64_t suf = 0;
     for (uint32_t d = w; d-- > 0;) {
-      const uint64_t pd = B[d];
+      const uint64_t pprev = d > 0 ? B[d - 1] : 0;
       B[d] = suf;
-      suf += (uint64_t)(px[d] + 1) * (d > 0 ? B[d - 1] : 0);  // term for i = d at position d-1
-      (void)pd;
+      suf += (uint64_t)(px[d] + 1) * pprev;  // term of item d at position d-1
     }
-    uint32_t here = 0;
-    for (uint32_t y = x + 1; y < end; ++y) {
-      const uint32_t b = L[(uint64_t)y * w + w - 1];
-      const uint64_t hb = (uint64_t)(b + 1) * p_last;
-      bool keep = true;
-      // subsets dropping item d of the shared prefix (dropping either of the last two items
-      // gives the parents x or y, members of L by construction)
-      for (uint32_t d = 0; d + 1 < w && keep; ++d) {
-        uint32_t q = 0;
-        for (uint32_t i = 0; i < w; ++i)
-          if (i != d) probe[q++] = px[i];
-        probe[q] = b;
-        keep = contains(L, w, slots, mask, probe, A[d] + B[d] + hb);
-      }
+    uint32_t here = 0;  // survivors so far (warp-uniform)
+    for (uint32_t y0 = x + 1; y0 < end; y0 += 32) {
+      const uint32_t y = y0 + lane;
+      bool keep = y < end;
+      uint32_t b = 0;
       if (keep) {
-        if (EMIT) ext[cand_off[x] + here] = b;
-        ++here;
+        b = L[(uint64_t)y * w + w - 1];
+        const uint64_t hb = (uint64_t)(b + 1) * p_last;
+        // subsets dropping item d of the shared prefix (dropping either of the last two items
+        // gives the parents x or y, members of L by construction)
+        for (uint32_t d = 0; d + 1 < w && keep; ++d) {
+          uint32_t q = 0;
+          for (uint32_t i = 0; i < w; ++i)
+            if (i != d) probe[q++] = px[i];
+          probe[q] = b;
+          keep = contains(L, w, slots, mask, probe, A[d] + B[d] + hb);
+        }
       }
+      const uint32_t ballot = __ballot_sync(0xffffffffu, keep);
+      if (EMIT && keep) ext[cand_off[x] + here + __popc(ballot & ((1u << lane) - 1u))] = b;
+      here += __popc(ballot);
     }
     if (EMIT) {
       const uint32_t g = gidx[x];
-      for (uint32_t i = 0; i < w; ++i) prefix[(uint64_t)g * w + i] = px[i];
-      ext_off[g] = cand_off[x];
-    } else {
+      for (uint32_t i = lane; i < w; i += 32) prefix[(uint64_t)g * w + i] = px[i];
+      if (lane == 0) ext_off[g] = cand_off[x];
+    } else if (lane == 0) {
       cnt[x] = here;
     }
   }
@@ -293,7 +304,7 @@ void device_candgen(const DeviceLevel& L, DeviceBatch& out, DeviceScratch& scrat
   uint32_t* slots = scratch.u32i(cap, s);
   GPA_CUDA(cudaMemsetAsync(slots, 0xff, (size_t)cap * 4, s));
   hash_build_kernel<<<grid_for(n, n_sms), kThreads, 0, s>>>(L.rows.p, n, w, slots, cap - 1);
-  join_kernel<false><<<grid_for(n, n_sms), kThreads, 0, s>>>(L.rows.p, n, w, flags, run_ex, bound, slots, cap - 1, cnt,
+  join_kernel<false><<<grid_for(32ull * n, n_sms), kThreads, 0, s>>>(L.rows.p, n, w, flags, run_ex, bound, slots, cap - 1, cnt,
                                                              nullptr, nullptr, nullptr, nullptr, nullptr);
   GPA_CUDA(cudaGetLastError());
   uint32_t* cand_off = scratch.u32e(n, s);
@@ -310,7 +321,7 @@ void device_candgen(const DeviceLevel& L, DeviceBatch& out, DeviceScratch& scrat
   out.prefix.ensure((size_t)G * w, s);
   out.ext_off.ensure(G + 1, s);
   out.ext.ensure(M, s);
-  join_kernel<true><<<grid_for(n, n_sms), kThreads, 0, s>>>(L.rows.p, n, w, flags, run_ex, bound, slots, cap - 1, cnt,
+  join_kernel<true><<<grid_for(32ull * n, n_sms), kThreads, 0, s>>>(L.rows.p, n, w, flags, run_ex, bound, slots, cap - 1, cnt,
                                                             cand_off, gidx, out.prefix.p, out.ext_off.p, out.ext.p);
   GPA_CUDA(cudaGetLastError());
   ext_end_kernel<<<1, 32, 0, s>>>(sizes, out.ext_off.p);
