@@ -47,6 +47,9 @@ def parse():
     p.add_argument("--kernel", default="auto", choices=["auto", "v0", "prefix", "pairs", "trie"])
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--dist", action="store_true", help="use the NCCL path even with one rank")
+    p.add_argument("--emulate-shard", type=int, default=0,
+                   help="scaling study on one GPU: mine the first 1/S of the transactions with min_count/S "
+                        "(about one rank's share of the work at S GPUs); not a bench line")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-sample-tx", type=int, default=0, help="oracle sample size (0 = auto)")
     return p.parse_args()
@@ -183,8 +186,11 @@ def main():
 
     # ---- this rank's shard of the workload (synthetic, seeded)
     b0, b1 = shard_range(cfg.n_tx, rank, world, cfg.kind == "quest")
-    ds = gen.make(cfg.name, tx_begin=b0, tx_end=b1)
     theta = gpa.min_count(cfg.n_tx, cfg.minsup)
+    if args.emulate_shard > 1:
+        b0, b1 = shard_range(cfg.n_tx, 0, args.emulate_shard, cfg.kind == "quest")
+        theta = max(1, theta * (b1 - b0) // cfg.n_tx)
+    ds = gen.make(cfg.name, tx_begin=b0, tx_end=b1)
     kern = {"auto": gpa.KERNEL_AUTO, "v0": gpa.KERNEL_V0, "prefix": gpa.KERNEL_PREFIX,
             "pairs": gpa.KERNEL_PAIRS, "trie": gpa.KERNEL_TRIE}[args.kernel]
     stream = torch.cuda.current_stream()

@@ -189,12 +189,18 @@ void bitset_free(gpa_bitset* bs) {
 
 namespace {
 
+// start / end events of a counting launch: the caller's (deferred timing, no sync) or the bitset's
+cudaEvent_t ev_start(gpa_bitset* bs, CountStats* st) { return st && st->e0 ? st->e0 : bs->ev0; }
+
 void finish_counts(gpa_bitset* bs, size_t M, CountStats* st) {
   cudaStream_t s = bs->stream;
-  GPA_CUDA(cudaEventRecord(bs->ev1, s));
+  const bool deferred = st && st->e0;
+  cudaEvent_t e1 = deferred ? st->e1 : bs->ev1, e2 = deferred ? st->e2 : bs->ev2;
+  GPA_CUDA(cudaEventRecord(e1, s));
   allreduce_sum_u32(bs->dist, bs->d_counts.p, M, s);
-  GPA_CUDA(cudaEventRecord(bs->ev2, s));
-  GPA_CUDA(cudaEventSynchronize(bs->ev2));
+  GPA_CUDA(cudaEventRecord(e2, s));
+  if (deferred) return;
+  GPA_CUDA(cudaEventSynchronize(e2));
   if (st) {
     st->count_ms = event_ms(bs->ev0, bs->ev1);
     st->allreduce_ms = bs->dist ? event_ms(bs->ev1, bs->ev2) : 0.0;
@@ -206,7 +212,7 @@ void count_flat_v0(gpa_bitset* bs, const std::vector<uint32_t>& flat, uint32_t k
   bs->d_flat.ensure(std::max<size_t>(flat.size(), 1), s);
   bs->d_counts.ensure(std::max<uint64_t>(M, 1), s);
   GPA_CUDA(cudaMemcpyAsync(bs->d_flat.p, flat.data(), flat.size() * sizeof(uint32_t), cudaMemcpyHostToDevice, s));
-  GPA_CUDA(cudaEventRecord(bs->ev0, s));
+  GPA_CUDA(cudaEventRecord(ev_start(bs, st), s));
   if (bs->n_rows) launch_count_v0(bs->rows.p, bs->pitch_words, bs->d_flat.p, k, M, bs->d_counts.p, s);
   else GPA_CUDA(cudaMemsetAsync(bs->d_counts.p, 0, M * sizeof(uint32_t), s));
   if (st) { st->kernel = GPA_KERNEL_V0; st->launches = 1; }
@@ -243,7 +249,7 @@ void count_trie_batch(gpa_bitset* bs, const GroupedBatch& b, CountStats* st) {
   GPA_CUDA(cudaMemcpyAsync(bs->d_lrows.p, lrows.data(), M * sizeof(uint4), cudaMemcpyHostToDevice, s));
   GPA_CUDA(cudaMemcpyAsync(bs->d_lcp.p, lcp.data(), M, cudaMemcpyHostToDevice, s));
   GPA_CUDA(cudaMemsetAsync(bs->d_counts.p, 0, M * sizeof(uint32_t), s));
-  GPA_CUDA(cudaEventRecord(bs->ev0, s));
+  GPA_CUDA(cudaEventRecord(ev_start(bs, st), s));
   if (bs->n_rows)
     launch_count_trie(k, bs->rows.p, bs->pitch_words, bs->d_tblocks.p, bs->d_trows.p, bs->d_lrows.p, bs->d_lcp.p,
                       n_blocks, max_rows, n_parts, bs->d_counts.p, s);
@@ -284,7 +290,7 @@ bool count_device_batch(gpa_bitset* bs, DeviceBatch& B, uint32_t kernel, DeviceS
     bs->d_tasks.ensure(T, s);
     launch_prefix_tasks(B.ext_off.p, G, nullptr, task_off, bs->d_tasks.p, bs->n_sms, s, true);
     GPA_CUDA(cudaMemsetAsync(bs->d_counts.p, 0, (size_t)M * 4, s));
-    GPA_CUDA(cudaEventRecord(bs->ev0, s));
+    GPA_CUDA(cudaEventRecord(ev_start(bs, st), s));
     const uint32_t max_tasks = 1u << 20;
     uint32_t launches = 0;
     for (uint32_t t0 = 0; t0 < T; t0 += max_tasks) {
@@ -336,7 +342,7 @@ bool count_device_batch(gpa_bitset* bs, DeviceBatch& B, uint32_t kernel, DeviceS
   if ((uint64_t)n_blocks * n_parts < want) n_parts = std::min<uint32_t>(n_stripes, (want + n_blocks - 1) / n_blocks);
   GPA_CUDA(cudaMemsetAsync(bs->d_counts.p, 0, (size_t)M * 4, s));
   const double tp1 = wall_ms();
-  GPA_CUDA(cudaEventRecord(bs->ev0, s));
+  GPA_CUDA(cudaEventRecord(ev_start(bs, st), s));
   launch_count_trie(k, bs->rows.p, bs->pitch_words, bs->d_tblocks.p, bs->d_trows.p, bs->d_lrows.p, bs->d_lcp.p,
                     n_blocks, max_rows, n_parts, bs->d_counts.p, s);
   if (st) { st->kernel = GPA_KERNEL_TRIE; st->launches = 1; }
@@ -393,7 +399,7 @@ void count_grouped(gpa_bitset* bs, const GroupedBatch& b, uint32_t kernel, Count
   GPA_CUDA(cudaMemcpyAsync(bs->d_ext.p, b.ext.data(), M * sizeof(uint32_t), cudaMemcpyHostToDevice, s));
   GPA_CUDA(cudaMemcpyAsync(bs->d_tasks.p, tasks.data(), tasks.size() * sizeof(PrefixTask), cudaMemcpyHostToDevice, s));
   GPA_CUDA(cudaMemsetAsync(bs->d_counts.p, 0, M * sizeof(uint32_t), s));
-  GPA_CUDA(cudaEventRecord(bs->ev0, s));
+  GPA_CUDA(cudaEventRecord(ev_start(bs, st), s));
   // a task index must fit the kernel's 32-bit grid decode: launch in slices of tasks if needed
   const uint64_t max_tasks = 1u << 20;
   uint32_t launches = 0;
@@ -431,7 +437,7 @@ void count_all_pairs(gpa_bitset* bs, uint32_t kernel, CountStats* st) {
   }
   bs->d_counts.ensure(M, s);
   GPA_CUDA(cudaMemsetAsync(bs->d_counts.p, 0, M * sizeof(uint32_t), s));
-  GPA_CUDA(cudaEventRecord(bs->ev0, s));
+  GPA_CUDA(cudaEventRecord(ev_start(bs, st), s));
   launch_count_pairs(bs->tmap, bs->n_rows, 0, bs->pitch_words, bs->d_counts.p, bs->n_sms, s);
   if (st) { st->kernel = GPA_KERNEL_PAIRS; st->launches = 1; }
   finish_counts(bs, M, st);

@@ -96,6 +96,9 @@ struct CountStats {
   uint32_t launches = 0;
   double count_ms = 0;
   double allreduce_ms = 0;
+  // optional caller-owned events: with them the counting functions do not synchronise; the
+  // caller reads count_ms / allreduce_ms from (e0, e1) / (e1, e2) later
+  cudaEvent_t e0 = nullptr, e1 = nullptr, e2 = nullptr;
 };
 
 }  // namespace gpa

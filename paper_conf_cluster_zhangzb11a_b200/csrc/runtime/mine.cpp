@@ -9,6 +9,7 @@
 // (P13@474, ">=" per DESIGN.md Q1).  Stops when L_k or C_{k+1} is empty (P13@652).
 #include <algorithm>
 #include <chrono>
+#include <deque>
 
 #include "internal.h"
 #include "pool.h"
@@ -146,6 +147,28 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
   DeviceLevel Ld, Ln;   // L_{k-1}, L_k on the device
   DeviceBatch Bd;       // C_k on the device (k >= 3)
   DBuf<uint32_t> d_ior;  // row -> original item id
+  struct Pending {       // a generation's frequent itemsets, still on the device
+    size_t level = 0;
+    uint32_t F = 0, k = 0;
+    DBuf<uint32_t> items, sup;
+  };
+  std::vector<Pending> pending;
+  struct EvTriple {      // deferred timing of a generation's counting launch(es) and all-reduce
+    cudaEvent_t e[3] = {nullptr, nullptr, nullptr};
+    EvTriple() {
+      for (auto& x : e) GPA_CUDA(cudaEventCreate(&x));
+    }
+    EvTriple(EvTriple&& o) noexcept {
+      for (int i = 0; i < 3; ++i) std::swap(e[i], o.e[i]);
+    }
+    EvTriple(const EvTriple&) = delete;
+    ~EvTriple() {
+      for (auto x : e)
+        if (x) cudaEventDestroy(x);
+    }
+  };
+  std::deque<EvTriple> events;
+  std::vector<size_t> event_level;
   d_ior.alloc(std::max<uint32_t>(bs->n_rows, 1), s);
   if (bs->n_rows)
     GPA_CUDA(cudaMemcpyAsync(d_ior.p, bs->item_of_row.data(), bs->n_rows * 4, cudaMemcpyHostToDevice, s));
@@ -191,6 +214,10 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     double t1 = now_ms();
     R->phase_ms[GPA_PHASE_CANDGEN] += t1 - t0;
     if (M == 0) break;
+    EvTriple& ev = events.emplace_back();
+    cs.e0 = ev.e[0];
+    cs.e1 = ev.e[1];
+    cs.e2 = ev.e[2];
     GPA_REQUIRE(M < (1ull << 32), GPA_ERR_INVALID, "generation %u has too many candidates", k);
     // the host copy of C_k is needed only for the host-planned kernels and for GPA_KEEP_CANDIDATES
     auto fetch_batch = [&]() {
@@ -207,6 +234,7 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     };
     if (k == 2 && pairs_ready && (opt.count_kernel == GPA_KERNEL_AUTO || opt.count_kernel == GPA_KERNEL_PAIRS)) {
       cs = pair_stats;  // counted during the overlapped ingest
+      events.pop_back();
     } else if (k == 2) {
       count_all_pairs(bs, opt.count_kernel, &cs);
     } else if (!count_device_batch(bs, Bd, opt.count_kernel, scratch, &cs)) {
@@ -219,27 +247,35 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
 
     const uint32_t F = device_threshold(bs->d_counts.p, (uint32_t)M, (uint32_t)min_count, k, bs->n_rows, Bd.prefix.p,
                                         Bd.ext_off.p, Bd.ext.p, (uint32_t)G, Ln, scratch, bs->n_sms, s);
-    std::vector<uint32_t> Litems((size_t)F * k), Lsup(F), counts;
+    // the frequent itemsets of this generation (item ids) and supports stay on the device until the
+    // end of the loop: one transfer for all generations instead of one synchronisation each
+    Pending pd;
+    pd.level = R->levels.size();
+    pd.F = F;
+    pd.k = k;
     if (F) {
-      uint32_t* d_items = scratch.u32a((size_t)F * k, s);
-      device_map_items(Ln.rows.p, (uint64_t)F * k, d_ior.p, d_items, bs->n_sms, s);
-      GPA_CUDA(cudaMemcpyAsync(Litems.data(), d_items, (size_t)F * k * 4, cudaMemcpyDeviceToHost, s));
-      GPA_CUDA(cudaMemcpyAsync(Lsup.data(), Ln.sup.p, (size_t)F * 4, cudaMemcpyDeviceToHost, s));
+      pd.items.alloc((size_t)F * k, s);
+      pd.sup.alloc(F, s);
+      device_map_items(Ln.rows.p, (uint64_t)F * k, d_ior.p, pd.items.p, bs->n_sms, s);
+      GPA_CUDA(cudaMemcpyAsync(pd.sup.p, Ln.sup.p, (size_t)F * 4, cudaMemcpyDeviceToDevice, s));
     }
+    std::vector<uint32_t> counts;
     if (keep) {
       counts.resize(M);
       GPA_CUDA(cudaMemcpyAsync(counts.data(), bs->d_counts.p, M * 4, cudaMemcpyDeviceToHost, s));
+      GPA_CUDA(cudaStreamSynchronize(s));
     }
-    GPA_CUDA(cudaStreamSynchronize(s));
     const double tr0 = now_ms();
-    record_level(R, bs, k, k > 2 ? &batch : nullptr, M, std::move(Litems), std::move(Lsup), keep,
-                 keep ? &counts : nullptr);
+    record_level(R, bs, k, k > 2 ? &batch : nullptr, M, {}, {}, keep, keep ? &counts : nullptr);
+    R->levels.back().n_freq = F;
+    pending.push_back(std::move(pd));
     std::swap(Ld, Ln);
     nL = F;
     if (trace_enabled())
-      fprintf(stderr, "[gpa] k=%u M=%llu G=%llu: candgen %.2f ms, count phase %.2f ms (kernel %.2f), "
-              "threshold %.2f ms (record %.2f) -> |L|=%u\n", k, (unsigned long long)M, (unsigned long long)G,
-              t1 - t0, t2 - t1, cs.count_ms, now_ms() - t2, now_ms() - tr0, F);
+      fprintf(stderr, "[gpa] k=%u M=%llu G=%llu: candgen %.2f ms, count phase %.2f ms, threshold %.2f ms (record %.2f) "
+              "-> |L|=%u\n", k, (unsigned long long)M, (unsigned long long)G, t1 - t0, t2 - t1, now_ms() - t2,
+              now_ms() - tr0, F);
+    if (cs.e0) event_level.push_back(R->levels.size() - 1);
     gpa_level_stats& st = R->levels.back().stats;
     st.n_cand = M;
     st.n_freq = F;
@@ -251,6 +287,28 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     st.candgen_ms = t1 - t0;
     R->phase_ms[GPA_PHASE_THRESHOLD] += now_ms() - t2;
   }
+
+  // ---- deferred: kernel times and the frequent itemsets of every generation
+  GPA_CUDA(cudaStreamSynchronize(s));
+  for (size_t i = 0; i < event_level.size(); ++i) {
+    float a = 0, b = 0;
+    GPA_CUDA(cudaEventElapsedTime(&a, events[i].e[0], events[i].e[1]));
+    GPA_CUDA(cudaEventElapsedTime(&b, events[i].e[1], events[i].e[2]));
+    gpa_level_stats& st = R->levels[event_level[i]].stats;
+    st.count_ms = a;
+    st.allreduce_ms = dist ? b : 0.0;
+  }
+  for (auto& pd : pending) {
+    gpa_level_data& lv = R->levels[pd.level];
+    lv.freq_items.resize((size_t)pd.F * pd.k);
+    lv.freq_support.resize(pd.F);
+    if (pd.F) {
+      GPA_CUDA(cudaMemcpyAsync(lv.freq_items.data(), pd.items.p, (size_t)pd.F * pd.k * 4, cudaMemcpyDeviceToHost, s));
+      GPA_CUDA(cudaMemcpyAsync(lv.freq_support.data(), pd.sup.p, (size_t)pd.F * 4, cudaMemcpyDeviceToHost, s));
+    }
+  }
+  GPA_CUDA(cudaStreamSynchronize(s));
+  pending.clear();
 
   uint64_t acc = 0;
   for (auto& lv : R->levels) {
