@@ -70,23 +70,32 @@ __global__ void window_greedy_kernel(const uint32_t* __restrict__ prefix, const 
   for (uint32_t i = threadIdx.x; i < (c1 - c0) * k; i += blockDim.x)
     items[i] = cand_item(prefix, ext, cand_group, k - 1, c0 + i / k, i % k);
   __syncthreads();
-  if (threadIdx.x != 0) return;
+  if (threadIdx.x >= 32) return;
+  // warp 0 walks the candidates; lane d < k tests / sets the bit of item d (items of one candidate
+  // are distinct, so the k bit updates never collide)
+  const uint32_t lane = threadIdx.x;
   uint32_t n = 0, start = c0, rows = 0;
   for (uint32_t m = c0; m < c1; ++m) {
-    const uint32_t* cur = items + (m - c0) * k;
-    uint32_t fresh = 0;
-    for (uint32_t d = 0; d < k; ++d) fresh += !((bm[cur[d] >> 5] >> (cur[d] & 31)) & 1u);
+    const uint32_t r = lane < k ? items[(m - c0) * k + lane] : 0;
+    const bool fresh_bit = lane < k && !((bm[r >> 5] >> (r & 31)) & 1u);
+    uint32_t fresh = __popc(__ballot_sync(0xffffffffu, fresh_bit));
     if (rows + fresh > rmax) {  // close [start, m)
-      recs[(uint64_t)blockIdx.x * window + n++] = make_uint3(start, m - start, rows);
-      for (uint32_t i = 0; i < nw; ++i) bm[i] = 0;
+      if (lane == 0) recs[(uint64_t)blockIdx.x * window + n] = make_uint3(start, m - start, rows);
+      ++n;
+      __syncwarp();
+      for (uint32_t i = lane; i < nw; i += 32) bm[i] = 0;
+      __syncwarp();
       start = m;
       rows = 0;
       fresh = k;
     }
-    for (uint32_t d = 0; d < k; ++d) bm[cur[d] >> 5] |= 1u << (cur[d] & 31);
+    if (lane < k) atomicOr(&bm[r >> 5], 1u << (r & 31));
+    __syncwarp();
     rows += fresh;
   }
-  if (c1 > start) recs[(uint64_t)blockIdx.x * window + n++] = make_uint3(start, c1 - start, rows);
+  if (lane == 0 && c1 > start) recs[(uint64_t)blockIdx.x * window + n] = make_uint3(start, c1 - start, rows);
+  if (c1 > start) ++n;
+  if (lane != 0) return;
   n_recs[blockIdx.x] = n;
 }
 
