@@ -47,6 +47,8 @@ def parse():
     p.add_argument("--kernel", default="auto", choices=["auto", "v0", "prefix", "pairs", "trie"])
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--dist", action="store_true", help="use the NCCL path even with one rank")
+    p.add_argument("--all-configs", action="store_true",
+                   help="table of every BASELINE.json config (GPU mine time vs the oracle); not a bench line")
     p.add_argument("--emulate-shard", type=int, default=0,
                    help="scaling study on one GPU: mine the first 1/S of the transactions with min_count/S "
                         "(about one rank's share of the work at S GPUs); not a bench line")
@@ -159,8 +161,49 @@ def reference_arm(args, cfg, rank, world):
     print(json.dumps(line), flush=True)
 
 
+def all_configs_table(args):
+    """Every BASELINE.json configuration: GPU mining time (device-resident and end to end) against
+    the CPU oracle on all host cores; checks the frequent itemsets are identical."""
+    import torch
+    import oracle
+    import paper_conf_cluster_zhangzb11a_b200 as gpa
+    threads = max(1, len(os.sched_getaffinity(0)))
+    rows = []
+    for name, cfg in gen.CONFIGS.items():
+        ds = gen.make(name)
+        theta = gpa.min_count(ds.n_tx, cfg.minsup)
+        d_off = torch.from_numpy(ds.offsets.view(np.int64)).cuda()
+        d_items = torch.from_numpy(ds.items.view(np.int32)).cuda()
+        h_off = torch.from_numpy(ds.offsets.view(np.int64)).pin_memory()
+        h_items = torch.from_numpy(ds.items.view(np.int32)).pin_memory()
+        for _ in range(2):
+            res = gpa.mine(d_off, d_items, ds.n_items, min_count=theta)
+        ts, te = [], []
+        for _ in range(5):
+            torch.cuda.synchronize()
+            t = time.perf_counter()
+            res = gpa.mine(d_off, d_items, ds.n_items, min_count=theta)
+            ts.append(time.perf_counter() - t)
+            t = time.perf_counter()
+            gpa.mine(h_off, h_items, ds.n_items, min_count=theta)
+            te.append(time.perf_counter() - t)
+        t = time.perf_counter()
+        ref = oracle.mine_ds(ds, theta, threads=threads)
+        to = time.perf_counter() - t
+        same = res.frequent() == ref.frequent()
+        ms, me = 1e3 * float(np.median(ts)), 1e3 * float(np.median(te))
+        rows.append({"config": name, "n_tx": ds.n_tx, "min_count": theta, "generations": len(res.levels),
+                     "frequent": len(res.frequent()), "cand_tx": res.cand_tx, "gpu_ms": ms, "gpu_e2e_ms": me,
+                     "oracle_ms": to * 1e3, "oracle_threads": threads, "speedup_e2e": to * 1e3 / me,
+                     "identical_F": same})
+        print(json.dumps(rows[-1]), flush=True)
+
+
 def main():
     args = parse()
+    if args.all_configs:
+        all_configs_table(args)
+        return
     cfg = gen.CONFIGS[args.config]
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
