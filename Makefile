@@ -19,7 +19,7 @@ CU_OBJS   := $(patsubst $(CSRC)/kernels/%.cu,$(BUILD)/k_%.o,$(CU_SRCS))
 CPP_OBJS  := $(patsubst $(CSRC)/runtime/%.cpp,$(BUILD)/r_%.o,$(CPP_SRCS))
 HDRS      := include/gpapriori.h $(CSRC)/common.h $(CSRC)/kernels.h $(CSRC)/runtime/internal.h $(CSRC)/runtime/pool.h
 
-all: $(LIB) oracle/liboracle.so gen/libgen.so
+all: $(LIB) oracle/liboracle.so gen/libgen.so examples/gpa_mine_fimi
 
 $(BUILD):
 	mkdir -p $(BUILD)
@@ -39,7 +39,10 @@ oracle/liboracle.so: oracle/apriori_oracle.c
 gen/libgen.so: gen/quest.c
 	$(CC) -O2 -shared -fPIC -Wall -o $@ $< -lm -lpthread
 
+examples/gpa_mine_fimi: examples/gpa_mine_fimi.c include/gpapriori.h $(LIB)
+	$(CC) -O2 -std=c11 -D_POSIX_C_SOURCE=200809L -Wall -Iinclude -o $@ $< -L$(PKG) -lgpapriori -Wl,-rpath,'$$ORIGIN/../$(PKG)'
+
 clean:
-	rm -rf $(BUILD) $(LIB) oracle/liboracle.so gen/libgen.so
+	rm -rf $(BUILD) $(LIB) oracle/liboracle.so gen/libgen.so examples/gpa_mine_fimi
 
 .PHONY: all clean

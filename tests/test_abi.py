@@ -92,3 +92,20 @@ def test_null_arguments_are_rejected():
     assert b"NULL" in L.gpa_last_error()
     for fn in ("gpa_bitset_destroy", "gpa_result_destroy", "gpa_dist_destroy"):
         assert getattr(L, fn)(None) == 0
+
+
+def test_c_example_builds_and_fails_loudly_without_gpu(tmp_path):
+    """examples/gpa_mine_fimi.c uses only the C ABI; without a GPU it must exit non-zero with the
+    library's CUDA error, not produce output."""
+    exe = os.path.join(ROOT, "examples", "gpa_mine_fimi")
+    subprocess.check_call(["make", "-C", ROOT, "-s", "examples/gpa_mine_fimi"])
+    try:
+        import torch
+        if torch.cuda.is_available():
+            pytest.skip("GPU present")
+    except ImportError:
+        pass
+    dat = tmp_path / "t.dat"
+    dat.write_text("1 2 3\n2 3\n")
+    r = subprocess.run([exe, str(dat), "0.5"], capture_output=True, text=True)
+    assert r.returncode != 0 and r.stdout == "" and "status 4" in r.stderr

@@ -331,3 +331,20 @@ def test_overlapped_ingest_row_estimate_miss():
     res = gpa.mine(ds, min_count=theta, keep_candidates=True)
     assert (12,) in res.frequent()
     assert_mine_equal(res, ref)
+
+
+def test_c_example_fimi_roundtrip(tmp_path, fig2):
+    """The C example (C ABI only) on the Fig. 2 database written as a FIMI file: every frequent
+    itemset and support as the oracle computes them."""
+    import subprocess
+    txs, _ = fig2
+    dat = tmp_path / "fig2.dat"
+    dat.write_text("\n".join(" ".join(map(str, t)) for t in txs) + "\n")
+    exe = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "examples", "gpa_mine_fimi")
+    out = subprocess.run([exe, str(dat), "0.5"], capture_output=True, text=True, check=True).stdout
+    got = {}
+    for line in out.strip().splitlines():
+        items, sup = line.rsplit(" (", 1)
+        got[tuple(int(x) for x in items.split())] = int(sup.rstrip(")"))
+    ref = oracle.mine_ds(gen.from_lists(txs, 8), 2).frequent()
+    assert got == ref
