@@ -49,17 +49,17 @@ uint64_t launch_count_prefix(const uint32_t* rows, uint64_t pitch_words, const u
 // Transaction-tiled trie walk for generations k in [2, kTrieMaxK] (count_trie.cu).  Candidates
 // (lexicographic) are cut into blocks of <= kTrieMaxCand candidates touching <= kTrieMaxRows rows.
 constexpr uint32_t kTrieMaxK = 16;
-constexpr uint32_t kTrieWideMaxK = 9;    // 3 <= k <= 9: 8 words per lane (256-word stripes), <= 32 rows / block
-constexpr uint32_t kTrieMaxRows = 64;    // otherwise: 4 words per lane (128-word stripes), <= 64 rows / block
+constexpr uint32_t kTrieMaxRows = 64;    // k = 2: 4 words per lane (128-word stripes), <= 64 rows / block
+constexpr uint32_t kTrieWideRows = 32;   // k >= 3: 8 words per lane (256-word stripes), <= 32 rows / block
 constexpr uint32_t kTrieMaxCand = 256;
 struct TrieBlock {
   uint32_t cand_begin;   // first candidate (global index)
   uint32_t n_cand;       // <= kTrieMaxCand
   uint32_t row_begin;    // into block_rows
-  uint32_t n_rows;       // <= kTrieMaxRows
+  uint32_t n_rows;       // <= trie_max_rows(k)
 };
-inline bool trie_wide(uint32_t k) { return k >= 3 && k <= kTrieWideMaxK; }
-inline uint32_t trie_max_rows(uint32_t k) { return trie_wide(k) ? kTrieMaxRows / 2 : kTrieMaxRows; }
+inline bool trie_wide(uint32_t k) { return k >= 3; }
+inline uint32_t trie_max_rows(uint32_t k) { return trie_wide(k) ? kTrieWideRows : kTrieMaxRows; }
 inline uint32_t trie_stripe_words(uint32_t k) { return trie_wide(k) ? 256 : 128; }
 // cand_lrows[c]: byte d = block-local row of item d; cand_lcp[c]: items shared with candidate c-1
 // (0 for the first candidate of every warp chunk: a block's n candidates are split into chunks of

@@ -8,22 +8,31 @@
 // reusing loaded words across MANY candidates, not only siblings:
 //
 //   * the host cuts the candidate list into BLOCKS of <= 256 lexicographically consecutive
-//     candidates touching <= 64 distinct rows; each of the 8 warps of a CTA owns 32 of them;
+//     candidates touching <= 32 distinct rows (64 for k = 2); each of the 8 warps of a CTA owns
+//     32 of them;
 //   * a CTA = (block, part of the transaction axis).  It streams its part in STRIPES of 128 x W
-//     words (W = 2 for k <= 8, else 1): a producer warp brings the block's rows' segments into a
+//     words (W = 2 for k >= 3, 1 for k = 2): a producer warp brings the block's rows' segments into a
 //     shared-memory ring with 1-D bulk async copies (cp.async.bulk + mbarrier complete_tx);
 //   * the 8 consumer warps split the block's candidates evenly and walk them for every stripe:
-//     lane = W x 4 words (W independent LDS.128 per row, conflict-free); a register stack V[d] = AND of the first d+1 rows is recomputed only from
-//     the first position where a candidate differs from its predecessor (lcp; a warp-uniform
-//     jump into an unrolled fall-through chain, so skipped levels cost nothing), the leaf is one
-//     LDS.128 + 4 AND + 4 POPC per 16 bytes, reduced across the warp with redux.sync into a
-//     per-candidate shared-memory counter (a compact, non-unrolled candidate loop: no I-cache
-//     thrash);  the bitset pitch is a
-//     multiple of the 128-word stripe, so there is no ragged stripe to mask;
+//     lane = 8 words (2 independent LDS.128 per row, conflict-free); the deepest three levels of
+//     the prefix stack V[d] = AND of the first d+1 rows live in registers and are recomputed only
+//     from the first position where a candidate differs from its predecessor (lcp; a warp-uniform
+//     jump into an unrolled fall-through chain, so skipped levels cost nothing); shallower levels
+//     are folded from shared memory when a candidate changes them (rare), which keeps the kernel
+//     at 72 registers = 3 CTAs (27 warps) per SM for every k;
+//   * the leaf is 2 LDS.128 + 8 AND + 8 POPC per lane, reduced across the warp with redux.sync;
+//     lane j keeps candidate j's running count in a register (the reduced value is added one
+//     candidate later, and the next candidate's descriptor is loaded one candidate ahead, so
+//     neither latency sits on the critical path).  Compact, non-unrolled candidate loop: no
+//     I-cache thrash.  The bitset pitch is a multiple of the 256-word stripe: no ragged stripe;
 //   * only after the whole part: one atomicAdd per (CTA, candidate).
-// Work per cand x word: ~1 LDS word + 1 AND + 1 POPC + (lcp recompute); no per-stripe reductions,
-// no global traffic besides the row segments (DRAM ~ the bitset once per part-window, the grid is
-// part-major so concurrently running CTAs share the same stripes in L2).  Bound: POPC issue.
+// Work per cand x word: ~1 LDS word + 1 AND + 1 POPC + (lcp recompute); no per-stripe reductions
+// to memory, no global traffic besides the row segments (DRAM ~ the bitset once per part-window;
+// the grid is part-major so concurrently running CTAs share the same stripes in L2).  Measured
+// bound (ncu, k = 6, 7): shared-memory bandwidth (~80%) with POPC issue at 62-68%.
+// Tried and rejected (slower): 16 words per lane at 2 CTAs/SM (k >= 7 +40%);
+// a per-class program keeping V_Q & R_a for 4 anchors in registers (half the row loads, but
+// +25% instructions and warp imbalance: +50%).
 #include <cstdint>
 #include "../common.h"
 #include "../kernels.h"
@@ -35,6 +44,7 @@ constexpr int kWarps = 8;                          // consumer warps
 constexpr int kThreads = (kWarps + 1) * 32;        // + 1 producer warp (bulk copies)
 constexpr int kCandPerWarp = 32;
 constexpr uint32_t kTrieMaxStages = 8;
+constexpr uint32_t kTrieRingBytes = 64u * 1024u;   // stripe ring per CTA (3 CTAs / SM)
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 
@@ -83,36 +93,56 @@ __device__ __forceinline__ uint32_t off_of(const uint4& lo, const uint4& hi, int
   return (e & 1) ? (w >> 16) : (w & 0xffffu);
 }
 
-// One trie level: V[D] = V[D-1] & row segment (V[0] = the row segment); W uint4 per lane.
+// Register-resident prefix levels: only the deepest kTrieRegLevels levels of the stack V live in
+// registers (V[i] = AND of rows 0..D0+i, D0 = K-1-kTrieRegLevels); a candidate whose shared prefix
+// with its predecessor is shorter than D0 (a new (K-3)-prefix: ~10-20% of candidates at deep
+// generations) folds rows 0..D0 from shared memory again.  This keeps the stack at 3 x W uint4 for
+// every K: 72 registers, 3 CTAs (27 warps) per SM, W = 2 up to K = 16.
+template <int K>
+constexpr int kTrieRegLevels = K - 1 < 3 ? K - 1 : 3;
+
+// Level D (>= D0) of the stack: V[D-D0] = V[D-D0-1] & row_D, or the fold of rows 0..D0 for D = D0.
 template <int K, int W, int D>
-__device__ __forceinline__ void trie_level(uint4 (&V)[K - 1][W], uint32_t base, const uint4& lo, const uint4& hi) {
-  if constexpr (D < K - 1) {
-    const uint32_t a = base + off_of(lo, hi, D);
-    uint4 v[W];
+__device__ __forceinline__ void trie_level(uint4 (&V)[kTrieRegLevels<K>][W], uint32_t base, const uint4& lo,
+                                           const uint4& hi) {
+  constexpr int D0 = K - 1 - kTrieRegLevels<K>;
+  if constexpr (D >= D0 && D < K - 1) {
+    if constexpr (D == D0) {
+      uint4 v[W];
+      const uint32_t a0 = base + off_of(lo, hi, 0);
 #pragma unroll
-    for (int u = 0; u < W; ++u) v[u] = lds128(a + u * 512);
+      for (int u = 0; u < W; ++u) v[u] = lds128(a0 + u * 512);
 #pragma unroll
-    for (int u = 0; u < W; ++u) V[D][u] = D == 0 ? v[u] : and4(V[D > 0 ? D - 1 : 0][u], v[u]);
+      for (int d = 1; d <= D0; ++d) {
+        const uint32_t a = base + off_of(lo, hi, d);
+#pragma unroll
+        for (int u = 0; u < W; ++u) v[u] = and4(v[u], lds128(a + u * 512));
+      }
+#pragma unroll
+      for (int u = 0; u < W; ++u) V[0][u] = v[u];
+    } else {
+      const uint32_t a = base + off_of(lo, hi, D);
+      uint4 v[W];
+#pragma unroll
+      for (int u = 0; u < W; ++u) v[u] = lds128(a + u * 512);
+#pragma unroll
+      for (int u = 0; u < W; ++u) V[D - D0][u] = and4(V[D - D0 - 1 >= 0 ? D - D0 - 1 : 0][u], v[u]);
+    }
   }
 }
 
-// Register budget: 3 CTAs (27 warps) per SM when the prefix stack is small, else 2.
 template <int K, int W>
-constexpr int kTrieRegs = (K - 1) * W * 4 <= 40 ? 72 : 112;
-template <int K, int W>
-constexpr uint32_t kTrieRingBytes = kTrieRegs<K, W> == 72 ? 64u * 1024u : 96u * 1024u;
-
-template <int K, int W>
-__global__ void __maxnreg__((kTrieRegs<K, W>)) count_trie_kernel(
+__global__ void __launch_bounds__(kThreads, 3) count_trie_kernel(
     const uint32_t* __restrict__ rows, uint64_t pitch_words, const TrieBlock* __restrict__ blocks,
     const uint32_t* __restrict__ block_rows, const uint4* __restrict__ cand_lrows, const uint8_t* __restrict__ cand_lcp,
     uint32_t n_blocks, uint32_t n_parts, uint32_t n_stripes, uint32_t n_stages, uint32_t* __restrict__ counts) {
   constexpr uint32_t kStripeWords = 128 * W;
   constexpr uint32_t kSegBytes = kStripeWords * 4;
+  constexpr int R = kTrieRegLevels<K>;
+  constexpr int D0 = K - 1 - R;
   extern __shared__ __align__(16) uint8_t smem[];
-  __shared__ uint4 s_desc[kWarps * kCandPerWarp][2];
+  __shared__ uint4 s_desc[kWarps * kCandPerWarp][K > 8 ? 2 : 1];
   __shared__ uint8_t s_lcp[kWarps * kCandPerWarp];
-  __shared__ uint32_t s_cnt[kWarps * kCandPerWarp];
   __shared__ uint32_t s_rowid[kTrieMaxRows];
   __shared__ __align__(8) uint64_t s_full[kTrieMaxStages];
   __shared__ __align__(8) uint64_t s_empty[kTrieMaxStages];
@@ -135,7 +165,7 @@ __global__ void __maxnreg__((kTrieRegs<K, W>)) count_trie_kernel(
       o[q] = (b0 * kSegBytes) | ((b1 * kSegBytes) << 16);
     }
     s_desc[i][0] = make_uint4(o[0], o[1], o[2], o[3]);
-    s_desc[i][1] = make_uint4(o[4], o[5], o[6], o[7]);
+    if constexpr (K > 8) s_desc[i][K > 8 ? 1 : 0] = make_uint4(o[4], o[5], o[6], o[7]);
     s_lcp[i] = cand_lcp[blk.cand_begin + i];
   }
   for (uint32_t i = threadIdx.x; i < blk.n_rows; i += kThreads) s_rowid[i] = block_rows[blk.row_begin + i];
@@ -170,16 +200,17 @@ __global__ void __maxnreg__((kTrieRegs<K, W>)) count_trie_kernel(
     return;
   }
 
-  // ---------------- consumer warps: the block's candidates split evenly, <= 32 per warp
+  // ---------------- consumer warps: the block's candidates split evenly, <= 32 per warp.
+  // Lane j accumulates candidate my0 + j over all stripes of the part (register, no shared-memory
+  // counters); the warp-reduced count of candidate j is added one iteration later, and the next
+  // candidate's descriptor is loaded one iteration ahead, so neither latency sits on the chain.
   const int chunk = ((int)blk.n_cand + kWarps - 1) / kWarps;
   const int my0 = warp * chunk;
   const int n_mine = max(0, min(chunk, (int)blk.n_cand - my0));
-  uint32_t* cnt = s_cnt + warp * kCandPerWarp;   // per-candidate partial counts of this warp
-  if (lane < kCandPerWarp) cnt[lane] = 0;
-  __syncwarp();
-  uint4 V[K - 1][W];
+  uint32_t acc = 0;
+  uint4 V[R][W];
 #pragma unroll
-  for (int d = 0; d < K - 1; ++d)
+  for (int d = 0; d < R; ++d)
 #pragma unroll
     for (int u = 0; u < W; ++u) V[d][u] = make_uint4(0, 0, 0, 0);
 
@@ -187,17 +218,22 @@ __global__ void __maxnreg__((kTrieRegs<K, W>)) count_trie_kernel(
     const uint32_t slot = i % n_stages;
     mbar_wait(full0 + 8 * slot, (i / n_stages) & 1);
     const uint32_t base = buf0 + slot * buf_bytes + lane * 16;
+    uint4 lo = s_desc[my0][0];
+    uint4 hi = K > 8 ? s_desc[my0][K > 8 ? 1 : 0] : make_uint4(0, 0, 0, 0);
+    int l = s_lcp[my0];
+    uint32_t c_prev = 0;
+    int j_prev = -1;
 #pragma unroll 1
     for (int j = 0; j < n_mine; ++j) {
-      const uint4 lo = s_desc[my0 + j][0];
-      const uint4 hi = K > 8 ? s_desc[my0 + j][1] : make_uint4(0, 0, 0, 0);
-      // recompute the prefix stack from the first level that differs from the previous
-      // candidate (warp-uniform branches; only the needed levels execute).  Common cases first:
-      // a sibling (lcp = K-1) only needs the leaf, a cousin (lcp = K-2) one level.
-      const int l = s_lcp[my0 + j];
+      const int jn = my0 + (j + 1 < n_mine ? j + 1 : j);
+      const uint4 lo_n = s_desc[jn][0];
+      const uint4 hi_n = K > 8 ? s_desc[jn][K > 8 ? 1 : 0] : make_uint4(0, 0, 0, 0);
+      const int l_n = s_lcp[jn];
+      // recompute the stack from the first level that differs from the previous candidate
+      // (warp-uniform; a sibling (lcp = K-1) only needs the leaf, a cousin (K-2) one level)
       if (l <= K - 2) {
         if (l <= K - 3) {
-          switch (l) {
+          switch (l < D0 ? D0 : l) {
 #define GPA_TRIE_LEVEL(D) \
   case D:                 \
     if constexpr (D <= K - 3) trie_level<K, W, D>(V, base, lo, hi); [[fallthrough]];
@@ -215,20 +251,23 @@ __global__ void __maxnreg__((kTrieRegs<K, W>)) count_trie_kernel(
       uint4 v[W];
 #pragma unroll
       for (int u = 0; u < W; ++u) v[u] = lds128(a + u * 512);
+      acc += lane == j_prev ? c_prev : 0u;
       uint32_t c = 0;
 #pragma unroll
       for (int u = 0; u < W; ++u)
-        c += (__popc(V[K - 2][u].x & v[u].x) + __popc(V[K - 2][u].y & v[u].y)) +
-             (__popc(V[K - 2][u].z & v[u].z) + __popc(V[K - 2][u].w & v[u].w));
-      // warp-reduce this stripe's partial count (redux.sync) into the candidate's smem slot
-      c = __reduce_add_sync(0xffffffffu, c);
-      if (lane == 0) cnt[j] += c;
+        c += (__popc(V[R - 1][u].x & v[u].x) + __popc(V[R - 1][u].y & v[u].y)) +
+             (__popc(V[R - 1][u].z & v[u].z) + __popc(V[R - 1][u].w & v[u].w));
+      c_prev = __reduce_add_sync(0xffffffffu, c);
+      j_prev = j;
+      lo = lo_n;
+      hi = hi_n;
+      l = l_n;
     }
+    acc += lane == j_prev ? c_prev : 0u;
     __syncwarp();
     if (lane == 0) mbar_arrive(empty0 + 8 * slot);
   }
-  __syncwarp();
-  if (lane < n_mine && cnt[lane]) atomicAdd(&counts[blk.cand_begin + my0 + lane], cnt[lane]);
+  if (lane < n_mine && acc) atomicAdd(&counts[blk.cand_begin + my0 + lane], acc);
 }
 
 template <int K, int W>
@@ -240,7 +279,7 @@ void launch_k(const uint32_t* rows, uint64_t pitch_words, const TrieBlock* block
   if (n_parts > n_stripes) n_parts = n_stripes;
   if (n_parts < 1) n_parts = 1;
   // ring depth: as many stripes in flight as fit the ring budget (3 or 2 CTAs / SM), 2..kTrieMaxStages
-  uint32_t stages = (uint32_t)(kTrieRingBytes<K, W> / ((size_t)max_rows * kSegBytes));
+  uint32_t stages = (uint32_t)(kTrieRingBytes / ((size_t)max_rows * kSegBytes));
   stages = stages < 2 ? 2 : (stages > kTrieMaxStages ? kTrieMaxStages : stages);
   const size_t smem = (size_t)stages * max_rows * kSegBytes;
   static bool attr = false;
@@ -270,8 +309,8 @@ uint64_t launch_count_trie(uint32_t k, const uint32_t* rows, uint64_t pitch_word
     break;
   switch (k) {
     GPA_TRIE_CASE(2, 1) GPA_TRIE_CASE(3, 2) GPA_TRIE_CASE(4, 2) GPA_TRIE_CASE(5, 2) GPA_TRIE_CASE(6, 2)
-    GPA_TRIE_CASE(7, 2) GPA_TRIE_CASE(8, 2) GPA_TRIE_CASE(9, 2) GPA_TRIE_CASE(10, 1) GPA_TRIE_CASE(11, 1)
-    GPA_TRIE_CASE(12, 1) GPA_TRIE_CASE(13, 1) GPA_TRIE_CASE(14, 1) GPA_TRIE_CASE(15, 1) GPA_TRIE_CASE(16, 1)
+    GPA_TRIE_CASE(7, 2) GPA_TRIE_CASE(8, 2) GPA_TRIE_CASE(9, 2) GPA_TRIE_CASE(10, 2) GPA_TRIE_CASE(11, 2)
+    GPA_TRIE_CASE(12, 2) GPA_TRIE_CASE(13, 2) GPA_TRIE_CASE(14, 2) GPA_TRIE_CASE(15, 2) GPA_TRIE_CASE(16, 2)
     default:
       fail(GPA_ERR_INVALID, "count_trie: k = %u outside [2, %u]", k, kTrieMaxK);
   }

@@ -141,7 +141,7 @@ def test_trie_plan_invariants(shim, name, k):
     M = len(cand)
     if M == 0:
         return
-    rmax = 32 if 3 <= k <= 9 else 64
+    rmax = 32 if k >= 3 else 64
     pos = 0
     for cb, nc, rb, nr in blocks.tolist():
         assert cb == pos and 0 < nc <= 256 and nr <= rmax
