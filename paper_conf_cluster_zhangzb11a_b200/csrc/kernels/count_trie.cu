@@ -85,12 +85,14 @@ __device__ __forceinline__ uint4 and4(const uint4& a, const uint4& b) {
 }
 
 // byte offset (local row * segment bytes) of level d in the candidate's descriptor: 16-bit
-// fields, levels 0-7 in lo, 8-15 in hi
+// fields, levels 0-7 in lo, 8-15 in hi.  Segments are >= 512 B, so the low 5 bits of level 0's
+// field are free: they carry the candidate's lcp (kLcpMask).
+constexpr uint32_t kLcpMask = 31u;
 __device__ __forceinline__ uint32_t off_of(const uint4& lo, const uint4& hi, int d) {
   const uint4& v = d < 8 ? lo : hi;
   const int e = d & 7;
   const uint32_t w = e < 2 ? v.x : e < 4 ? v.y : e < 6 ? v.z : v.w;
-  return (e & 1) ? (w >> 16) : (w & 0xffffu);
+  return (e & 1) ? (w >> 16) : (w & (d == 0 ? 0xffffu & ~kLcpMask : 0xffffu));
 }
 
 // Register-resident prefix levels: only the deepest kTrieRegLevels levels of the stack V live in
@@ -142,7 +144,6 @@ __global__ void __launch_bounds__(kThreads, 3) count_trie_kernel(
   constexpr int D0 = K - 1 - R;
   extern __shared__ __align__(16) uint8_t smem[];
   __shared__ uint4 s_desc[kWarps * kCandPerWarp][K > 8 ? 2 : 1];
-  __shared__ uint8_t s_lcp[kWarps * kCandPerWarp];
   __shared__ uint32_t s_rowid[kTrieMaxRows];
   __shared__ __align__(8) uint64_t s_full[kTrieMaxStages];
   __shared__ __align__(8) uint64_t s_empty[kTrieMaxStages];
@@ -164,9 +165,8 @@ __global__ void __launch_bounds__(kThreads, 3) count_trie_kernel(
       const uint32_t b0 = (w[q >> 1] >> (16 * (q & 1))) & 0xffu, b1 = (w[q >> 1] >> (16 * (q & 1) + 8)) & 0xffu;
       o[q] = (b0 * kSegBytes) | ((b1 * kSegBytes) << 16);
     }
-    s_desc[i][0] = make_uint4(o[0], o[1], o[2], o[3]);
+    s_desc[i][0] = make_uint4(o[0] | cand_lcp[blk.cand_begin + i], o[1], o[2], o[3]);
     if constexpr (K > 8) s_desc[i][K > 8 ? 1 : 0] = make_uint4(o[4], o[5], o[6], o[7]);
-    s_lcp[i] = cand_lcp[blk.cand_begin + i];
   }
   for (uint32_t i = threadIdx.x; i < blk.n_rows; i += kThreads) s_rowid[i] = block_rows[blk.row_begin + i];
   const uint32_t full0 = smem_u32(&s_full[0]);
@@ -202,8 +202,7 @@ __global__ void __launch_bounds__(kThreads, 3) count_trie_kernel(
 
   // ---------------- consumer warps: the block's candidates split evenly, <= 32 per warp.
   // Lane j accumulates candidate my0 + j over all stripes of the part (register, no shared-memory
-  // counters); the warp-reduced count of candidate j is added one iteration later, and the next
-  // candidate's descriptor is loaded one iteration ahead, so neither latency sits on the chain.
+  // counters).
   const int chunk = ((int)blk.n_cand + kWarps - 1) / kWarps;
   const int my0 = warp * chunk;
   const int n_mine = max(0, min(chunk, (int)blk.n_cand - my0));
@@ -214,56 +213,57 @@ __global__ void __launch_bounds__(kThreads, 3) count_trie_kernel(
 #pragma unroll
     for (int u = 0; u < W; ++u) V[d][u] = make_uint4(0, 0, 0, 0);
 
+  // one candidate: recompute the stack from the first level that differs from the previous
+  // candidate (warp-uniform; a sibling (lcp = K-1) only needs the leaf, a cousin (K-2) one
+  // level), then this lane's popcount of the leaf AND
+  auto candidate = [&](uint32_t base, const uint4& lo, const uint4& hi) -> uint32_t {
+    const int l = lo.x & kLcpMask;
+    if (l <= K - 2) {
+      if (l <= K - 3) {
+        switch (l < D0 ? D0 : l) {
+#define GPA_TRIE_LEVEL(D) \
+  case D:                 \
+    if constexpr (D <= K - 3) trie_level<K, W, D>(V, base, lo, hi); [[fallthrough]];
+          GPA_TRIE_LEVEL(0) GPA_TRIE_LEVEL(1) GPA_TRIE_LEVEL(2) GPA_TRIE_LEVEL(3) GPA_TRIE_LEVEL(4)
+          GPA_TRIE_LEVEL(5) GPA_TRIE_LEVEL(6) GPA_TRIE_LEVEL(7) GPA_TRIE_LEVEL(8) GPA_TRIE_LEVEL(9)
+          GPA_TRIE_LEVEL(10) GPA_TRIE_LEVEL(11) GPA_TRIE_LEVEL(12) GPA_TRIE_LEVEL(13)
+#undef GPA_TRIE_LEVEL
+          default:
+            break;
+        }
+      }
+      trie_level<K, W, K - 2>(V, base, lo, hi);
+    }
+    const uint32_t a = base + off_of(lo, hi, K - 1);
+    uint4 v[W];
+#pragma unroll
+    for (int u = 0; u < W; ++u) v[u] = lds128(a + u * 512);
+    uint32_t c = 0;
+#pragma unroll
+    for (int u = 0; u < W; ++u)
+      c += (__popc(V[R - 1][u].x & v[u].x) + __popc(V[R - 1][u].y & v[u].y)) +
+           (__popc(V[R - 1][u].z & v[u].z) + __popc(V[R - 1][u].w & v[u].w));
+    return c;
+  };
+
   for (uint32_t s = st0, i = 0; s < st1; ++s, ++i) {
     const uint32_t slot = i % n_stages;
     mbar_wait(full0 + 8 * slot, (i / n_stages) & 1);
     const uint32_t base = buf0 + slot * buf_bytes + lane * 16;
-    uint4 lo = s_desc[my0][0];
-    uint4 hi = K > 8 ? s_desc[my0][K > 8 ? 1 : 0] : make_uint4(0, 0, 0, 0);
-    int l = s_lcp[my0];
-    uint32_t c_prev = 0;
-    int j_prev = -1;
+    // candidates in pairs: both lane partials (<= 32 x 8 x 32 = 8,192 summed over the warp) share
+    // one redux.sync, packed into 16-bit halves
 #pragma unroll 1
-    for (int j = 0; j < n_mine; ++j) {
-      const int jn = my0 + (j + 1 < n_mine ? j + 1 : j);
-      const uint4 lo_n = s_desc[jn][0];
-      const uint4 hi_n = K > 8 ? s_desc[jn][K > 8 ? 1 : 0] : make_uint4(0, 0, 0, 0);
-      const int l_n = s_lcp[jn];
-      // recompute the stack from the first level that differs from the previous candidate
-      // (warp-uniform; a sibling (lcp = K-1) only needs the leaf, a cousin (K-2) one level)
-      if (l <= K - 2) {
-        if (l <= K - 3) {
-          switch (l < D0 ? D0 : l) {
-#define GPA_TRIE_LEVEL(D) \
-  case D:                 \
-    if constexpr (D <= K - 3) trie_level<K, W, D>(V, base, lo, hi); [[fallthrough]];
-            GPA_TRIE_LEVEL(0) GPA_TRIE_LEVEL(1) GPA_TRIE_LEVEL(2) GPA_TRIE_LEVEL(3) GPA_TRIE_LEVEL(4)
-            GPA_TRIE_LEVEL(5) GPA_TRIE_LEVEL(6) GPA_TRIE_LEVEL(7) GPA_TRIE_LEVEL(8) GPA_TRIE_LEVEL(9)
-            GPA_TRIE_LEVEL(10) GPA_TRIE_LEVEL(11) GPA_TRIE_LEVEL(12) GPA_TRIE_LEVEL(13)
-#undef GPA_TRIE_LEVEL
-            default:
-              break;
-          }
-        }
-        trie_level<K, W, K - 2>(V, base, lo, hi);
-      }
-      const uint32_t a = base + off_of(lo, hi, K - 1);
-      uint4 v[W];
-#pragma unroll
-      for (int u = 0; u < W; ++u) v[u] = lds128(a + u * 512);
-      acc += lane == j_prev ? c_prev : 0u;
-      uint32_t c = 0;
-#pragma unroll
-      for (int u = 0; u < W; ++u)
-        c += (__popc(V[R - 1][u].x & v[u].x) + __popc(V[R - 1][u].y & v[u].y)) +
-             (__popc(V[R - 1][u].z & v[u].z) + __popc(V[R - 1][u].w & v[u].w));
-      c_prev = __reduce_add_sync(0xffffffffu, c);
-      j_prev = j;
-      lo = lo_n;
-      hi = hi_n;
-      l = l_n;
+    for (int j = 0; j < n_mine; j += 2) {
+      const bool two = j + 1 < n_mine;
+      const uint4 lo0 = s_desc[my0 + j][0];
+      const uint4 hi0 = K > 8 ? s_desc[my0 + j][K > 8 ? 1 : 0] : make_uint4(0, 0, 0, 0);
+      const uint4 lo1 = s_desc[my0 + j + (two ? 1 : 0)][0];
+      const uint4 hi1 = K > 8 ? s_desc[my0 + j + (two ? 1 : 0)][K > 8 ? 1 : 0] : make_uint4(0, 0, 0, 0);
+      uint32_t c = candidate(base, lo0, hi0);
+      if (two) c |= candidate(base, lo1, hi1) << 16;
+      c = __reduce_add_sync(0xffffffffu, c);
+      acc += lane == j ? (c & 0xffffu) : (lane == j + 1 ? (c >> 16) : 0u);
     }
-    acc += lane == j_prev ? c_prev : 0u;
     __syncwarp();
     if (lane == 0) mbar_arrive(empty0 + 8 * slot);
   }

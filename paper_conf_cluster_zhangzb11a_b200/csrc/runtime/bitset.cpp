@@ -8,11 +8,22 @@
 // leave the (rank-summed) counts in bs->d_counts.
 #include <algorithm>
 #include <chrono>
+#include <cstdlib>
 #include <numeric>
 
 #include "internal.h"
 
 namespace gpa {
+
+// AUTO's choice between the streaming prefix kernel (mean sibling group >= cut) and the trie walk;
+// GPA_AUTO_SIBLINGS overrides the cut (experiments only)
+static double auto_sibling_cut() {
+  static const double cut = [] {
+    const char* e = getenv("GPA_AUTO_SIBLINGS");
+    return e ? atof(e) : 4.0;
+  }();
+  return cut;
+}
 
 namespace {
 
@@ -273,7 +284,7 @@ bool count_device_batch(gpa_bitset* bs, DeviceBatch& B, uint32_t kernel, DeviceS
   if (kernel == GPA_KERNEL_V0 || bs->n_rows > kPlanMaxRows || k < 2) return false;
   if (kernel == GPA_KERNEL_AUTO || kernel == GPA_KERNEL_PAIRS) {
     const double sib = (double)M / (double)std::max<uint32_t>(G, 1);
-    kernel = (k <= kTrieMaxK && sib < 4.0) ? GPA_KERNEL_TRIE : GPA_KERNEL_PREFIX;
+    kernel = (k <= kTrieMaxK && sib < auto_sibling_cut()) ? GPA_KERNEL_TRIE : GPA_KERNEL_PREFIX;
   }
   if (kernel == GPA_KERNEL_TRIE && k > kTrieMaxK) kernel = GPA_KERNEL_PREFIX;
   const double tp0 = wall_ms();
@@ -363,7 +374,7 @@ void count_grouped(gpa_bitset* bs, const GroupedBatch& b, uint32_t kernel, Count
     // prefix kernel (measured: T40I10D10M k = 3, 4.6 siblings / group); small groups (deep
     // generations, ~2 siblings) need the trie walk's reuse across groups
     const double sib = (double)M / (double)std::max<uint64_t>(G, 1);
-    kernel = (b.k >= 2 && b.k <= kTrieMaxK && sib < 4.0) ? GPA_KERNEL_TRIE : GPA_KERNEL_PREFIX;
+    kernel = (b.k >= 2 && b.k <= kTrieMaxK && sib < auto_sibling_cut()) ? GPA_KERNEL_TRIE : GPA_KERNEL_PREFIX;
   }
   if (kernel == GPA_KERNEL_TRIE) {
     if (b.k >= 2 && b.k <= kTrieMaxK) {
