@@ -75,6 +75,13 @@ bool make_pairs_tensor_map(void* tmap128, const uint32_t* rows, uint32_t n_rows,
 // Words [word_begin, word_end) of the rows (multiples of 32); counts accumulate (atomic adds).
 uint64_t launch_count_pairs(const void* tmap128, uint32_t n_rows, uint64_t word_begin, uint64_t word_end,
                             uint32_t* counts, int n_sms, cudaStream_t stream);
+// k = 2 on the tensor cores (count_pairs_tc.cu): C = B B^T over words [word_begin, word_end)
+// (multiples of 4) as a tcgen05 kind::i8 GEMM of the bit-expanded rows; counts accumulate.
+uint64_t launch_count_pairs_tc(const uint32_t* rows, uint64_t pitch_words, uint32_t n_rows, uint64_t word_begin,
+                               uint64_t word_end, uint32_t* counts, int n_sms, cudaStream_t stream);
+inline bool pairs_kernel_k2(uint32_t kernel) {
+  return kernel == GPA_KERNEL_AUTO || kernel == GPA_KERNEL_PAIRS || kernel == GPA_KERNEL_PAIRS_TC;
+}
 // counts_sub[pair_index(a, b, n_sub)] = counts_all[pair_index(sel[a], sel[b], n_all)] (sel ascending)
 void launch_pairs_subset(const uint32_t* counts_all, uint32_t n_all, const uint32_t* sel, uint32_t n_sub,
                          uint32_t* counts_sub, int n_sms, cudaStream_t stream);

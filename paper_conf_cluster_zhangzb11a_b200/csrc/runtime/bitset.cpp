@@ -38,7 +38,7 @@ float event_ms(cudaEvent_t a, cudaEvent_t b) {
 }
 
 void validate_options(const gpa_options& o) {
-  GPA_REQUIRE(o.count_kernel <= GPA_KERNEL_TRIE, GPA_ERR_INVALID, "unknown count_kernel %u", o.count_kernel);
+  GPA_REQUIRE(o.count_kernel <= GPA_KERNEL_PAIRS_TC, GPA_ERR_INVALID, "unknown count_kernel %u", o.count_kernel);
   GPA_REQUIRE(o.max_k <= GPA_MAX_K, GPA_ERR_INVALID, "max_k %u > GPA_MAX_K", o.max_k);
   GPA_REQUIRE(!o.reserved[0] && !o.reserved[1] && !o.reserved[2], GPA_ERR_INVALID, "reserved option fields must be 0");
   GPA_REQUIRE((o.flags & ~(GPA_KEEP_CANDIDATES | GPA_HOST_CANDGEN | GPA_NO_OVERLAP_INGEST)) == 0, GPA_ERR_INVALID, "unknown option flags 0x%x",
@@ -282,7 +282,7 @@ bool count_device_batch(gpa_bitset* bs, DeviceBatch& B, uint32_t kernel, DeviceS
   const uint32_t k = B.k, M = B.M, G = B.G;
   if (M == 0) return true;
   if (kernel == GPA_KERNEL_V0 || bs->n_rows > kPlanMaxRows || k < 2) return false;
-  if (kernel == GPA_KERNEL_AUTO || kernel == GPA_KERNEL_PAIRS) {
+  if (kernel == GPA_KERNEL_AUTO || kernel == GPA_KERNEL_PAIRS || kernel == GPA_KERNEL_PAIRS_TC) {
     const double sib = (double)M / (double)std::max<uint32_t>(G, 1);
     kernel = (k <= kTrieMaxK && sib < auto_sibling_cut()) ? GPA_KERNEL_TRIE : GPA_KERNEL_PREFIX;
   }
@@ -369,7 +369,7 @@ void count_grouped(gpa_bitset* bs, const GroupedBatch& b, uint32_t kernel, Count
   const uint64_t M = b.size(), G = b.groups();
   const uint32_t km1 = b.k - 1;
   if (M == 0) return;
-  if (kernel == GPA_KERNEL_AUTO || kernel == GPA_KERNEL_PAIRS) {
+  if (kernel == GPA_KERNEL_AUTO || kernel == GPA_KERNEL_PAIRS || kernel == GPA_KERNEL_PAIRS_TC) {
     // grouped batches: large sibling groups amortise the (k-1)-row prefix well in the streaming
     // prefix kernel (measured: T40I10D10M k = 3, 4.6 siblings / group); small groups (deep
     // generations, ~2 siblings) need the trie walk's reuse across groups
@@ -429,8 +429,8 @@ void count_all_pairs(gpa_bitset* bs, uint32_t kernel, CountStats* st) {
   const uint64_t n = bs->n_rows;
   const uint64_t M = n * (n - 1) / 2;
   if (n < 2) return;
-  if (kernel == GPA_KERNEL_AUTO) kernel = GPA_KERNEL_PAIRS;
-  if (kernel != GPA_KERNEL_PAIRS) {
+  if (kernel == GPA_KERNEL_AUTO) kernel = GPA_KERNEL_PAIRS_TC;
+  if (kernel != GPA_KERNEL_PAIRS && kernel != GPA_KERNEL_PAIRS_TC) {
     GroupedBatch b;
     b.k = 2;
     b.ext_off.push_back(0);
@@ -442,15 +442,18 @@ void count_all_pairs(gpa_bitset* bs, uint32_t kernel, CountStats* st) {
     count_grouped(bs, b, kernel, st);
     return;
   }
-  if (!bs->tmap_ready) {
+  if (kernel == GPA_KERNEL_PAIRS && !bs->tmap_ready) {
     make_pairs_tensor_map(bs->tmap, bs->rows.p, bs->n_rows, bs->pitch_words);
     bs->tmap_ready = true;
   }
   bs->d_counts.ensure(M, s);
   GPA_CUDA(cudaMemsetAsync(bs->d_counts.p, 0, M * sizeof(uint32_t), s));
   GPA_CUDA(cudaEventRecord(ev_start(bs, st), s));
-  launch_count_pairs(bs->tmap, bs->n_rows, 0, bs->pitch_words, bs->d_counts.p, bs->n_sms, s);
-  if (st) { st->kernel = GPA_KERNEL_PAIRS; st->launches = 1; }
+  if (kernel == GPA_KERNEL_PAIRS_TC)
+    launch_count_pairs_tc(bs->rows.p, bs->pitch_words, bs->n_rows, 0, bs->pitch_words, bs->d_counts.p, bs->n_sms, s);
+  else
+    launch_count_pairs(bs->tmap, bs->n_rows, 0, bs->pitch_words, bs->d_counts.p, bs->n_sms, s);
+  if (st) { st->kernel = kernel; st->launches = 1; }
   finish_counts(bs, M, st);
 }
 
@@ -525,7 +528,7 @@ extern "C" gpa_status gpa_count(gpa_bitset* bs, const uint32_t* cand, uint32_t k
   return gpa::guard([&] {
     GPA_REQUIRE(bs, GPA_ERR_INVALID, "bitset is NULL");
     GPA_REQUIRE(k >= 1 && k <= GPA_MAX_K, GPA_ERR_INVALID, "k must be in [1, %u]", GPA_MAX_K);
-    GPA_REQUIRE(kernel <= GPA_KERNEL_TRIE, GPA_ERR_INVALID, "unknown kernel %u", kernel);
+    GPA_REQUIRE(kernel <= GPA_KERNEL_PAIRS_TC, GPA_ERR_INVALID, "unknown kernel %u", kernel);
     if (M == 0) return;
     GPA_REQUIRE(cand && counts_out, GPA_ERR_INVALID, "NULL argument");
     GPA_REQUIRE(M <= (UINT64_MAX / 8) / k && M < (1ull << 32), GPA_ERR_INVALID, "M * k overflows");
@@ -547,11 +550,12 @@ extern "C" gpa_status gpa_count(gpa_bitset* bs, const uint32_t* cand, uint32_t k
     uint32_t kern = kernel == GPA_KERNEL_AUTO ? bs->opt.count_kernel : kernel;
     if (k == 1) kern = GPA_KERNEL_V0;
     if (kern == GPA_KERNEL_AUTO)
-      kern = (k == 2 && (double)M * 8 >= (double)bs->n_rows * bs->n_rows) ? GPA_KERNEL_PAIRS
+      kern = (k == 2 && (double)M * 8 >= (double)bs->n_rows * bs->n_rows) ? GPA_KERNEL_PAIRS_TC
              : (k <= gpa::kTrieMaxK ? GPA_KERNEL_TRIE : GPA_KERNEL_PREFIX);
-    if (kern == GPA_KERNEL_PAIRS && k != 2) kern = k <= gpa::kTrieMaxK ? GPA_KERNEL_TRIE : GPA_KERNEL_PREFIX;
-    if (kern == GPA_KERNEL_PAIRS) {
-      gpa::count_all_pairs(bs, GPA_KERNEL_PAIRS, nullptr);
+    if ((kern == GPA_KERNEL_PAIRS || kern == GPA_KERNEL_PAIRS_TC) && k != 2)
+      kern = k <= gpa::kTrieMaxK ? GPA_KERNEL_TRIE : GPA_KERNEL_PREFIX;
+    if (kern == GPA_KERNEL_PAIRS || kern == GPA_KERNEL_PAIRS_TC) {
+      gpa::count_all_pairs(bs, kern, nullptr);
       const uint64_t n = bs->n_rows, P = n * (n - 1) / 2;
       std::vector<uint32_t> all(P);
       if (P) {

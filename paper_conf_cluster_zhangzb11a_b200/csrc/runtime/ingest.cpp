@@ -147,11 +147,13 @@ gpa_bitset* bitset_build_overlapped(const gpa_tx_csr* db, uint64_t row_min_count
   GPA_CUDA(cudaMemcpyAsync(d_r0map.p, r0_of_item.data(), n_items * 4, cudaMemcpyHostToDevice, s));
   const uint64_t P0 = (uint64_t)nr0 * (nr0 ? nr0 - 1 : 0) / 2;
   alignas(64) unsigned char tmap0[128];
+  // generation 2 on the tensor cores unless the caller pinned the CUDA-core pair kernel
+  const bool pairs_tc = bs->opt.count_kernel != GPA_KERNEL_PAIRS;
   if (nr0) {
     d_r0rows.alloc((size_t)nr0 * bs->pitch_words, s);
     d_r0pairs.alloc(std::max<uint64_t>(P0, 1), s);
     GPA_CUDA(cudaMemsetAsync(d_r0pairs.p, 0, std::max<uint64_t>(P0, 1) * 4, s));
-    if (nr0 >= 2) make_pairs_tensor_map(tmap0, d_r0rows.p, nr0, bs->pitch_words);
+    if (nr0 >= 2 && !pairs_tc) make_pairs_tensor_map(tmap0, d_r0rows.p, nr0, bs->pitch_words);
   }
   double pairs_ms = 0;
   uint32_t pair_launches = 0;
@@ -176,7 +178,10 @@ gpa_bitset* bitset_build_overlapped(const gpa_tx_csr* db, uint64_t row_min_count
         GPA_CUDA(cudaEventCreate(&pe[2 * c + 1]));
         GPA_CUDA(cudaEventRecord(pe[2 * c], s));
         const uint64_t w0 = cut[c] / 32, w1 = c + 1 == C ? bs->pitch_words : cut[c + 1] / 32;
-        launch_count_pairs(tmap0, nr0, w0, w1, d_r0pairs.p, bs->n_sms, s);
+        if (pairs_tc)
+          launch_count_pairs_tc(d_r0rows.p, bs->pitch_words, nr0, w0, w1, d_r0pairs.p, bs->n_sms, s);
+        else
+          launch_count_pairs(tmap0, nr0, w0, w1, d_r0pairs.p, bs->n_sms, s);
         GPA_CUDA(cudaEventRecord(pe[2 * c + 1], s));
         ++pair_launches;
       }
@@ -246,7 +251,7 @@ gpa_bitset* bitset_build_overlapped(const gpa_tx_csr* db, uint64_t row_min_count
         GPA_CUDA(cudaEventElapsedTime(&ms, bs->ev0, bs->ev1));
         *pairs_ready = true;
         if (pair_stats) {
-          pair_stats->kernel = GPA_KERNEL_PAIRS;
+          pair_stats->kernel = pairs_tc ? GPA_KERNEL_PAIRS_TC : GPA_KERNEL_PAIRS;
           pair_stats->launches = pair_launches + 1;
           pair_stats->count_ms = pairs_ms + ms;
           pair_stats->allreduce_ms = 0;

@@ -232,7 +232,7 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
       GPA_CUDA(cudaStreamSynchronize(s));
       batch.ext_off.assign(off32.begin(), off32.end());
     };
-    if (k == 2 && pairs_ready && (opt.count_kernel == GPA_KERNEL_AUTO || opt.count_kernel == GPA_KERNEL_PAIRS)) {
+    if (k == 2 && pairs_ready && pairs_kernel_k2(opt.count_kernel)) {
       cs = pair_stats;  // counted during the overlapped ingest
       events.pop_back();
     } else if (k == 2) {

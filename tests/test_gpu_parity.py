@@ -16,7 +16,7 @@ import paper_conf_cluster_zhangzb11a_b200 as gpa
 
 pytestmark = pytest.mark.gpu
 
-KERNELS = [gpa.KERNEL_V0, gpa.KERNEL_PREFIX, gpa.KERNEL_PAIRS, gpa.KERNEL_TRIE]
+KERNELS = [gpa.KERNEL_V0, gpa.KERNEL_PREFIX, gpa.KERNEL_PAIRS, gpa.KERNEL_TRIE, gpa.KERNEL_PAIRS_TC]
 
 
 def expected_bits(ds, item_of_row, pitch_words):
@@ -119,18 +119,40 @@ def test_count_many_rows_per_block(kern, k):
         assert np.array_equal(got, ref.astype(np.uint32))
 
 
-@pytest.mark.parametrize("n_items", [2, 3, 127, 128, 129, 200, 257])
-def test_pairs_kernel_tile_boundaries(n_items):
-    """All pairs of n rows through the tiled kernel, n around the 128-row tile edge."""
+@pytest.mark.parametrize("kern", [gpa.KERNEL_PAIRS, gpa.KERNEL_PAIRS_TC])
+@pytest.mark.parametrize("n_items", [2, 3, 127, 128, 129, 200, 255, 256, 257, 385, 513])
+def test_pairs_kernel_tile_boundaries(kern, n_items):
+    """All pairs of n rows through the tiled kernels, n around the 128-row (CUDA-core kernel,
+    tensor-core A side) and 256-row (tensor-core B side) tile edges."""
     ds = gen.random_db(n_items, 3000, n_items, max_len=min(n_items, 40), p_empty=0.0)
     with gpa.Bitset(ds) as bs:
         rows = bs.rows()
         pairs = np.array(list(combinations(rows.tolist(), 2)), dtype=np.uint32).reshape(-1, 2)
         if len(pairs) == 0:
             return
-        got = bs.count(pairs, kernel=gpa.KERNEL_PAIRS)
+        got = bs.count(pairs, kernel=kern)
         ref = oracle.support_batch(ds.offsets, ds.items, ds.n_items, pairs)
         assert np.array_equal(got, ref.astype(np.uint32))
+
+
+@pytest.mark.parametrize("n_tx", [1, 127, 129, 8191, 8193, 100_003, 1_000_001])
+def test_pairs_tc_transaction_axis(n_tx):
+    """The tensor-core pair Gram over transaction counts that cut its 128-transaction stages and
+    its K-split anywhere (dense rows: counts far above one stage), equal to the CUDA-core kernel
+    and, on sampled pairs, to the literal definition."""
+    ds = gen.random_db(n_tx % 97 + 5, n_tx, 150, max_len=60, p_empty=0.02)
+    with gpa.Bitset(ds) as bs:
+        rows = bs.rows()
+        pairs = np.array(list(combinations(rows.tolist(), 2)), dtype=np.uint32).reshape(-1, 2)
+        if len(pairs) == 0:
+            return
+        tc = bs.count(pairs, kernel=gpa.KERNEL_PAIRS_TC)
+        cc = bs.count(pairs, kernel=gpa.KERNEL_PAIRS)
+        assert np.array_equal(tc, cc)
+        rng = np.random.default_rng(n_tx)
+        pick = rng.choice(len(pairs), size=min(len(pairs), 200), replace=False)
+        ref = oracle.support_batch(ds.offsets, ds.items, ds.n_items, pairs[pick])
+        assert np.array_equal(tc[pick], ref.astype(np.uint32))
 
 
 def test_count_errors():
@@ -180,7 +202,7 @@ def test_mine_configs(name):
     theta = oracle.min_count(ds.n_tx, gen.CONFIGS[name].minsup)
     assert gpa.min_count(ds.n_tx, gen.CONFIGS[name].minsup) == theta
     ref = oracle.mine_ds(ds, theta)
-    kernels = [gpa.KERNEL_AUTO, gpa.KERNEL_PREFIX, gpa.KERNEL_TRIE] + (
+    kernels = [gpa.KERNEL_AUTO, gpa.KERNEL_PAIRS, gpa.KERNEL_PREFIX, gpa.KERNEL_TRIE] + (
         [gpa.KERNEL_V0] if name in ("chess", "mushroom") else [])
     # AUTO = pairs (k = 2) + trie / prefix (k >= 3); device-side candidate generation by default,
     # the host thread-pool join + prune as the reference path
