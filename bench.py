@@ -262,6 +262,7 @@ def main():
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     level_ms = {}
     barrier()
+    launches0 = gpa.kernel_launches()
     with ClockSampler(local) as clocks:
         ev0.record(stream)
         for _ in range(args.steps):
@@ -270,18 +271,22 @@ def main():
                 level_ms.setdefault(lv.k, []).append(lv.stats["count_ms"])
         ev1.record(stream)
         barrier()
+    launches = gpa.kernel_launches() - launches0   # every kernel the library launched in the region
     step_ms = max_over_ranks(ev0.elapsed_time(ev1) / args.steps)
     n_tx = res.n_tx
     cand_tx = res.cand_tx
     value = cand_tx / (step_ms * 1e-3)
-    launches_per_step = 2 + sum(lv.stats["launches"] for lv in res.levels[1:])  # hist + bitset + counting
 
-    # ---- rooflines.  All counting kernels are bound by the XU pipe that executes POPC (16 / clk /
-    # SM on sm_100a, profiles/r01_microbench_popc.txt), not by HBM (the bitset is re-read from L2
-    # / shared memory).  Peak in cand*tx/s = 148 SM x 16 POPC/clk / (POPC per word) x 32 tx/word x
-    # f_SM:  the pair kernel counts 4 words with 3 POPC (carry-save adder) -> 0.75 POPC / word;
-    # the trie / prefix / v0 kernels use 1 POPC / word.  "achieved" uses the algorithmic work
-    # |C_k| x N of the launch and its CUDA-event time inside the timed region.
+    # ---- rooflines.  The CUDA-core counting kernels are bound by the XU pipe that executes POPC
+    # (16 / clk / SM on sm_100a, profiles/r01_microbench_popc.txt), not by HBM (the bitset is
+    # re-read from L2 / shared memory).  Peak in cand*tx/s = 148 SM x 16 POPC/clk / (POPC per
+    # word) x 32 tx/word x f_SM:  the pair kernel counts 4 words with 3 POPC (carry-save adder)
+    # -> 0.75 POPC / word; the trie / prefix / v0 kernels use 1 POPC / word.  The tensor-core pair
+    # kernel (pairs_tc) is a u8 GEMM: "tensor" bound, achieved = 2 x |C_2| x N integer ops (the
+    # algorithmic MACs; tile padding below the diagonal not counted) / time against the int8
+    # dense peak = 2 x the measured bf16 peak (MEASURED_PEAKS.json; int8 : bf16 = 4.5 : 2.25
+    # PFLOP/s nominal).  "achieved" uses the algorithmic work |C_k| x N of the launch and its
+    # CUDA-event time inside the timed region.
     sm_max = None
     peaks = {}
     try:
@@ -296,6 +301,16 @@ def main():
         ms = max_over_ranks(sum(float(np.mean(level_ms[lv.k])) for lv in levels))
         work = sum(lv.n_cand for lv in levels) * n_tx
         name = levels[0].stats["kernel_name"]
+        if name == "pairs_tc":
+            bf16 = float(peaks.get("bf16_tflops", 2250.0 * 1965 / 1965))
+            peak = 2.0 * bf16
+            ach = 2.0 * work / (ms * 1e-3) / 1e12
+            return {"bound": "tensor", "achieved": ach, "peak": peak, "unit": "TOPS (int8, 2 ops per cand*tx)",
+                    "frac": ach / peak,
+                    "peak_basis": f"int8 dense = 2 x measured bf16 {bf16:.1f} TFLOP/s (MEASURED_PEAKS.json)"
+                                  if "bf16_tflops" in peaks else "int8 dense = 2 x 2250 TFLOP/s nominal bf16 (no "
+                                  "MEASURED_PEAKS.json)",
+                    "kernel_ms": ms, "work": work, "cand_tx_per_s": work / (ms * 1e-3)}
         ppw = popc_per_word.get(name, 1.0)
         peak = 148 * 16 / ppw * 32 * sm_max * 1e6 / 1e12
         ach = work / (ms * 1e-3) / 1e12
@@ -316,8 +331,9 @@ def main():
     roof["traffic"] = None
     try:
         tr = json.load(open(os.path.join(ROOT, "profiles", "traffic.json")))
-        key = {"pairs": "count_pairs_kernel", "prefix": "count_prefix_kernel"}.get(
-            dom.stats["kernel_name"], f"count_trie_kernel<{dom.k}, {2 if 3 <= dom.k <= 9 else 1}>")
+        key = {"pairs": "count_pairs_kernel", "prefix": "count_prefix_kernel",
+               "pairs_tc": "count_pairs_tc_kernel"}.get(
+            dom.stats["kernel_name"], f"count_trie_kernel<{dom.k}, {1 if dom.k == 2 else 2}>")
         if key in tr:
             roof["traffic"] = tr[key]["dram_bytes"]
             roof["traffic_unit"] = "bytes per launch (ncu dram__bytes_read.sum + dram__bytes_write.sum)"
@@ -380,7 +396,7 @@ def main():
             "roofline_by_kernel": roof_all,
             "cpu_baseline": cpu,
             "e2e": e2e,
-            "gpu_launches": launches_per_step * args.steps,
+            "gpu_launches": launches,
             "clocks": clk,
             "kernel_time_ms": {f"k{k}": float(np.mean(v)) for k, v in sorted(level_ms.items())},
             "count_throughput": cand_tx / (sum(float(np.mean(v)) for v in level_ms.values()) * 1e-3),

@@ -67,6 +67,11 @@ const char* gpa_last_error(void);
 /* Library version string, e.g. "gpapriori-b200 0.1 sm_100a". */
 const char* gpa_version(void);
 
+/* Number of GPU kernels this library has launched in the process so far (all devices, all
+ * threads; includes the CUB scan kernels of the device level transition).  Instrumentation for
+ * benchmarks: the difference across a timed region is the kernel-launch count of that region. */
+uint64_t gpa_kernel_launches(void);
+
 /* ------------------------------------------------------------------ inputs */
 
 #define GPA_MEM_HOST 0u        /* offsets/items are host pointers (pinned or pageable) */

@@ -82,6 +82,7 @@ def lib() -> ctypes.CDLL:
     sig = {
         "gpa_last_error": (ctypes.c_char_p, []),
         "gpa_version": (ctypes.c_char_p, []),
+        "gpa_kernel_launches": (ctypes.c_uint64, []),
         "gpa_options_default": (None, [P(_Options)]),
         "gpa_min_count": (u64, [u64, u64, u64]),
         "gpa_dist_unique_id": (ctypes.c_int, [ctypes.c_char_p]),
@@ -121,6 +122,11 @@ def _check(status: int) -> None:
 
 def version() -> str:
     return lib().gpa_version().decode()
+
+
+def kernel_launches() -> int:
+    """Kernels this library has launched in the process so far (gpa_kernel_launches)."""
+    return int(lib().gpa_kernel_launches())
 
 
 def min_count(n_tx: int, minsup) -> int:

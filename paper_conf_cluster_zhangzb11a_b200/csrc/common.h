@@ -1,6 +1,7 @@
 // Internal helpers shared by the library's runtime (.cpp) and kernel (.cu) translation units.
 // Nothing here is part of the C ABI (include/gpapriori.h is).
 #pragma once
+#include <atomic>
 #include <cstdint>
 #include <cstdio>
 #include <string>
@@ -9,6 +10,11 @@
 #include "gpapriori.h"
 
 namespace gpa {
+
+// Process-wide count of the library's kernel launches (every <<<>>> site and CUB's scan kernels),
+// exported through gpa_kernel_launches() so a benchmark can state how many of its kernels ran.
+inline std::atomic<uint64_t> g_kernel_launches{0};
+inline void note_launch(uint64_t n = 1) { g_kernel_launches.fetch_add(n, std::memory_order_relaxed); }
 
 struct Error {
   gpa_status status;

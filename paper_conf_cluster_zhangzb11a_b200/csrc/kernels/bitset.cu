@@ -94,8 +94,8 @@ void launch_bitset_build(const uint64_t* offsets, const uint32_t* items, uint64_
   GPA_CUDA(cudaFuncSetAttribute(bitset_build_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   GPA_REQUIRE(c1 - c0 < (1ull << 31), GPA_ERR_INVALID, "bitset: too many transactions");
   dim3 grid((unsigned)(c1 - c0), n_rb);
-  bitset_build_kernel<<<grid, kBuildThreads, smem, stream>>>(offsets, items, n_tx, nnz, row_of_item, n_items, n_rows, rb, c0,
-                                                             pitch_words, rows);
+  { bitset_build_kernel<<<grid, kBuildThreads, smem, stream>>>(offsets, items, n_tx, nnz, row_of_item, n_items, n_rows, rb, c0,
+                                                             pitch_words, rows); note_launch(); }
   GPA_CUDA(cudaGetLastError());
 }
 
@@ -125,7 +125,7 @@ __global__ void gather_rows_kernel(const uint4* __restrict__ all, const uint32_t
 void launch_pairs_subset(const uint32_t* counts_all, uint32_t n_all, const uint32_t* sel, uint32_t n_sub,
                          uint32_t* counts_sub, int n_sms, cudaStream_t stream) {
   if (n_sub < 2) return;
-  pairs_subset_kernel<<<n_sms * 4, 256, 0, stream>>>(counts_all, n_all, sel, n_sub, counts_sub);
+  { pairs_subset_kernel<<<n_sms * 4, 256, 0, stream>>>(counts_all, n_all, sel, n_sub, counts_sub); note_launch(); }
   GPA_CUDA(cudaGetLastError());
 }
 
@@ -135,8 +135,8 @@ void launch_gather_rows(const uint32_t* rows_all, const uint32_t* sel, uint32_t 
   const uint64_t pitch4 = pitch_words / 4;
   unsigned gx = (unsigned)std::min<uint64_t>((pitch4 + 255) / 256, 64);
   dim3 grid(gx, std::min<uint32_t>(n_sub, 65535));
-  gather_rows_kernel<<<grid, 256, 0, stream>>>(reinterpret_cast<const uint4*>(rows_all), sel, n_sub, pitch4,
-                                               reinterpret_cast<uint4*>(rows_sub));
+  { gather_rows_kernel<<<grid, 256, 0, stream>>>(reinterpret_cast<const uint4*>(rows_all), sel, n_sub, pitch4,
+                                               reinterpret_cast<uint4*>(rows_sub)); note_launch(); }
   GPA_CUDA(cudaGetLastError());
 }
 

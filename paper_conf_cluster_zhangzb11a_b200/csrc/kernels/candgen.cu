@@ -236,7 +236,8 @@ void exclusive_scan(const uint32_t* in, uint32_t* out, uint32_t n, uint32_t* tot
   GPA_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, bytes, in, out, n, s));
   void* tmp = scratch.get(bytes, s);
   GPA_CUDA(cub::DeviceScan::ExclusiveSum(tmp, bytes, in, out, n, s));
-  if (tot) total_kernel<<<1, 32, 0, s>>>(in, out, n, tot);
+  note_launch(2);  // CUB: init + scan kernels
+  if (tot) { total_kernel<<<1, 32, 0, s>>>(in, out, n, tot); note_launch(); }
 }
 
 }  // namespace
@@ -249,7 +250,7 @@ uint32_t device_threshold(const uint32_t* counts, uint32_t M, uint32_t theta, ui
   if (M == 0) return 0;
   uint32_t* flags = scratch.u32a(M, s);
   uint32_t* pos = scratch.u32b(M, s);
-  flag_ge_kernel<<<grid_for(M, n_sms), kThreads, 0, s>>>(counts, M, theta, flags);
+  { flag_ge_kernel<<<grid_for(M, n_sms), kThreads, 0, s>>>(counts, M, theta, flags); note_launch(); }
   GPA_CUDA(cudaGetLastError());
   uint32_t* sizes = scratch.u32c(4, s);
   exclusive_scan(flags, pos, M, sizes, scratch, s);
@@ -260,11 +261,11 @@ uint32_t device_threshold(const uint32_t* counts, uint32_t M, uint32_t theta, ui
   out.sup.ensure(std::max<uint32_t>(F, 1), s);
   if (F) {
     if (k == 2)
-      scatter_pairs_kernel<<<grid_for(M, n_sms), kThreads, 0, s>>>(counts, flags, pos, M, n_rows, out.rows.p,
-                                                                  out.sup.p);
+      { scatter_pairs_kernel<<<grid_for(M, n_sms), kThreads, 0, s>>>(counts, flags, pos, M, n_rows, out.rows.p,
+                                                                  out.sup.p); note_launch(); }
     else
-      scatter_grouped_kernel<<<grid_for(M, n_sms), kThreads, 0, s>>>(counts, flags, pos, M, prefix, ext_off, ext, G,
-                                                                    k - 1, out.rows.p, out.sup.p);
+      { scatter_grouped_kernel<<<grid_for(M, n_sms), kThreads, 0, s>>>(counts, flags, pos, M, prefix, ext_off, ext, G,
+                                                                    k - 1, out.rows.p, out.sup.p); note_launch(); }
     GPA_CUDA(cudaGetLastError());
   }
   out.n = F;
@@ -279,7 +280,7 @@ void device_exclusive_scan(const uint32_t* in, uint32_t* out, uint32_t n, uint32
 void device_map_items(const uint32_t* rows, uint64_t n, const uint32_t* item_of_row, uint32_t* items, int n_sms,
                       cudaStream_t s) {
   if (n == 0) return;
-  map_items_kernel<<<grid_for(n, n_sms), kThreads, 0, s>>>(rows, n, item_of_row, items);
+  { map_items_kernel<<<grid_for(n, n_sms), kThreads, 0, s>>>(rows, n, item_of_row, items); note_launch(); }
   GPA_CUDA(cudaGetLastError());
 }
 
@@ -293,25 +294,25 @@ void device_candgen(const DeviceLevel& L, DeviceBatch& out, DeviceScratch& scrat
   uint32_t* cnt = scratch.u32c(n, s);
   uint32_t* bound = scratch.u32d(n + 1, s);
   uint32_t* sizes = scratch.u32h(4, s);  // [0] = M, [1] = G
-  run_start_kernel<<<grid_for(n, n_sms), kThreads, 0, s>>>(L.rows.p, n, w, flags);
+  { run_start_kernel<<<grid_for(n, n_sms), kThreads, 0, s>>>(L.rows.p, n, w, flags); note_launch(); }
   GPA_CUDA(cudaGetLastError());
   exclusive_scan(flags, run_ex, n, nullptr, scratch, s);
-  run_bound_kernel<<<grid_for(n, n_sms), kThreads, 0, s>>>(flags, run_ex, n, bound);
-  bound_sentinel_kernel<<<1, 32, 0, s>>>(flags, run_ex, n, bound);
+  { run_bound_kernel<<<grid_for(n, n_sms), kThreads, 0, s>>>(flags, run_ex, n, bound); note_launch(); }
+  { bound_sentinel_kernel<<<1, 32, 0, s>>>(flags, run_ex, n, bound); note_launch(); }
   // hash set over L for the prune probes
   uint32_t cap = 16;
   while (cap < 2 * n + 1) cap <<= 1;
   uint32_t* slots = scratch.u32i(cap, s);
   GPA_CUDA(cudaMemsetAsync(slots, 0xff, (size_t)cap * 4, s));
-  hash_build_kernel<<<grid_for(n, n_sms), kThreads, 0, s>>>(L.rows.p, n, w, slots, cap - 1);
-  join_kernel<false><<<grid_for(32ull * n, n_sms), kThreads, 0, s>>>(L.rows.p, n, w, flags, run_ex, bound, slots, cap - 1, cnt,
-                                                             nullptr, nullptr, nullptr, nullptr, nullptr);
+  { hash_build_kernel<<<grid_for(n, n_sms), kThreads, 0, s>>>(L.rows.p, n, w, slots, cap - 1); note_launch(); }
+  { join_kernel<false><<<grid_for(32ull * n, n_sms), kThreads, 0, s>>>(L.rows.p, n, w, flags, run_ex, bound, slots, cap - 1, cnt,
+                                                             nullptr, nullptr, nullptr, nullptr, nullptr); note_launch(); }
   GPA_CUDA(cudaGetLastError());
   uint32_t* cand_off = scratch.u32e(n, s);
   uint32_t* gflag = scratch.u32f(n, s);
   uint32_t* gidx = scratch.u32g(n, s);
   exclusive_scan(cnt, cand_off, n, sizes, scratch, s);
-  nonzero_kernel<<<grid_for(n, n_sms), kThreads, 0, s>>>(cnt, n, gflag);
+  { nonzero_kernel<<<grid_for(n, n_sms), kThreads, 0, s>>>(cnt, n, gflag); note_launch(); }
   exclusive_scan(gflag, gidx, n, sizes + 1, scratch, s);
   uint32_t MG[2] = {0, 0};
   GPA_CUDA(cudaMemcpyAsync(MG, sizes, 8, cudaMemcpyDeviceToHost, s));
@@ -321,10 +322,10 @@ void device_candgen(const DeviceLevel& L, DeviceBatch& out, DeviceScratch& scrat
   out.prefix.ensure((size_t)G * w, s);
   out.ext_off.ensure(G + 1, s);
   out.ext.ensure(M, s);
-  join_kernel<true><<<grid_for(32ull * n, n_sms), kThreads, 0, s>>>(L.rows.p, n, w, flags, run_ex, bound, slots, cap - 1, cnt,
-                                                            cand_off, gidx, out.prefix.p, out.ext_off.p, out.ext.p);
+  { join_kernel<true><<<grid_for(32ull * n, n_sms), kThreads, 0, s>>>(L.rows.p, n, w, flags, run_ex, bound, slots, cap - 1, cnt,
+                                                            cand_off, gidx, out.prefix.p, out.ext_off.p, out.ext.p); note_launch(); }
   GPA_CUDA(cudaGetLastError());
-  ext_end_kernel<<<1, 32, 0, s>>>(sizes, out.ext_off.p);
+  { ext_end_kernel<<<1, 32, 0, s>>>(sizes, out.ext_off.p); note_launch(); }
   out.M = M;
   out.G = G;
 }

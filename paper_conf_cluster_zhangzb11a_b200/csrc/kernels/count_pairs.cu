@@ -258,8 +258,8 @@ uint64_t launch_count_pairs(const void* tmap128, uint32_t n_rows, uint64_t word_
   }
   CUtensorMap map;
   memcpy(&map, tmap128, sizeof(map));
-  count_pairs_kernel<<<(unsigned)grid, kThreads, kSmemBytes, stream>>>(map, n_rows, nb, n_tiles, chunk0, n_chunks, per,
-                                                                       counts);
+  { count_pairs_kernel<<<(unsigned)grid, kThreads, kSmemBytes, stream>>>(map, n_rows, nb, n_tiles, chunk0, n_chunks, per,
+                                                                       counts); note_launch(); }
   GPA_CUDA(cudaGetLastError());
   return grid;
 }

@@ -93,8 +93,8 @@ uint64_t launch_count_prefix(const uint32_t* rows, uint64_t pitch_words, const u
   const uint64_t n_blocks = n_stripes * n_tasks;
   GPA_REQUIRE(n_blocks < (1ull << 31), GPA_ERR_INVALID, "count_prefix: grid too large (%llu CTAs)",
               (unsigned long long)n_blocks);
-  count_prefix_kernel<<<(unsigned)n_blocks, kPrefixThreads, 0, stream>>>(
-      reinterpret_cast<const uint4*>(rows), pitch4, prefix_rows, km1, ext_rows, tasks, n_tasks, counts);
+  { count_prefix_kernel<<<(unsigned)n_blocks, kPrefixThreads, 0, stream>>>(
+      reinterpret_cast<const uint4*>(rows), pitch4, prefix_rows, km1, ext_rows, tasks, n_tasks, counts); note_launch(); }
   GPA_CUDA(cudaGetLastError());
   return n_blocks;
 }

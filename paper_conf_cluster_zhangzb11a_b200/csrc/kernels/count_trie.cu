@@ -289,8 +289,8 @@ void launch_k(const uint32_t* rows, uint64_t pitch_words, const TrieBlock* block
   }
   const uint64_t grid = (uint64_t)n_blocks * n_parts;
   GPA_REQUIRE(grid < (1ull << 31), GPA_ERR_INVALID, "count_trie: grid too large");
-  count_trie_kernel<K, W><<<(unsigned)grid, kThreads, smem, stream>>>(rows, pitch_words, blocks, block_rows, lrows,
-                                                                      lcp, n_blocks, n_parts, n_stripes, stages, counts);
+  { count_trie_kernel<K, W><<<(unsigned)grid, kThreads, smem, stream>>>(rows, pitch_words, blocks, block_rows, lrows,
+                                                                      lcp, n_blocks, n_parts, n_stripes, stages, counts); note_launch(); }
   GPA_CUDA(cudaGetLastError());
 }
 

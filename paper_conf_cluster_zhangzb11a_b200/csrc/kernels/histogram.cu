@@ -105,11 +105,11 @@ void launch_hist_validate_range(const uint64_t* offsets, const uint32_t* items, 
     size_t smem = (size_t)n_items * sizeof(uint32_t);
     if (smem > 48 * 1024)
       GPA_CUDA(cudaFuncSetAttribute(hist_validate_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    hist_validate_kernel<true><<<grid, kHistThreads, smem, stream>>>(offsets, items, tx_begin, tx_end, nnz, n_items,
-                                                                     hist, flags);
+    { hist_validate_kernel<true><<<grid, kHistThreads, smem, stream>>>(offsets, items, tx_begin, tx_end, nnz, n_items,
+                                                                     hist, flags); note_launch(); }
   } else {
-    hist_validate_kernel<false><<<grid, kHistThreads, 0, stream>>>(offsets, items, tx_begin, tx_end, nnz, n_items,
-                                                                   hist, flags);
+    { hist_validate_kernel<false><<<grid, kHistThreads, 0, stream>>>(offsets, items, tx_begin, tx_end, nnz, n_items,
+                                                                   hist, flags); note_launch(); }
   }
   GPA_CUDA(cudaGetLastError());
 }
@@ -122,7 +122,7 @@ void launch_hist_validate(const uint64_t* offsets, const uint32_t* items, uint64
 void launch_hist_dedup(const uint64_t* offsets, const uint32_t* items, uint64_t n_tx, uint64_t nnz, uint32_t n_items,
                        uint32_t* hist, int n_sms, cudaStream_t stream) {
   if (n_tx == 0) return;
-  hist_dedup_kernel<<<grid_for(n_tx, n_sms), kHistThreads, 0, stream>>>(offsets, items, n_tx, nnz, n_items, hist);
+  { hist_dedup_kernel<<<grid_for(n_tx, n_sms), kHistThreads, 0, stream>>>(offsets, items, n_tx, nnz, n_items, hist); note_launch(); }
   GPA_CUDA(cudaGetLastError());
 }
 

@@ -194,14 +194,14 @@ unsigned grid_for(uint64_t n, int n_sms) {
 
 void launch_cand_group(const uint32_t* ext_off, uint32_t G, uint32_t* cand_group, int n_sms, cudaStream_t s) {
   if (G == 0) return;
-  cand_group_kernel<<<grid_for(G, n_sms), kThreads, 0, s>>>(ext_off, G, cand_group);
+  { cand_group_kernel<<<grid_for(G, n_sms), kThreads, 0, s>>>(ext_off, G, cand_group); note_launch(); }
   GPA_CUDA(cudaGetLastError());
 }
 
 void launch_window_rows(const uint32_t* prefix, const uint32_t* ext, const uint32_t* cand_group, uint32_t k,
                         uint32_t n_rows, const uint2* windows, uint32_t n_windows, uint32_t* R, cudaStream_t s) {
   if (n_windows == 0) return;
-  window_rows_kernel<<<n_windows, kThreads, 0, s>>>(prefix, ext, cand_group, k, n_rows, windows, R);
+  { window_rows_kernel<<<n_windows, kThreads, 0, s>>>(prefix, ext, cand_group, k, n_rows, windows, R); note_launch(); }
   GPA_CUDA(cudaGetLastError());
 }
 
@@ -210,20 +210,20 @@ void launch_window_greedy(const uint32_t* prefix, const uint32_t* ext, const uin
                           cudaStream_t s) {
   if (M == 0) return;
   const uint32_t n_win = (M + window - 1) / window;
-  window_greedy_kernel<<<n_win, 64, 0, s>>>(prefix, ext, cand_group, k, n_rows, M, window, rmax, recs, n_recs);
+  { window_greedy_kernel<<<n_win, 64, 0, s>>>(prefix, ext, cand_group, k, n_rows, M, window, rmax, recs, n_recs); note_launch(); }
   GPA_CUDA(cudaGetLastError());
 }
 
 void launch_compact_blocks(const uint3* recs, const uint32_t* n_recs, const uint32_t* off, uint32_t n_win,
                            uint32_t window, TrieBlock* blocks, uint32_t* rows, uint32_t* stats, cudaStream_t s) {
   if (n_win == 0) return;
-  compact_blocks_kernel<<<n_win < 4096 ? n_win : 4096, 64, 0, s>>>(recs, n_recs, off, n_win, window, blocks, rows, stats);
+  { compact_blocks_kernel<<<n_win < 4096 ? n_win : 4096, 64, 0, s>>>(recs, n_recs, off, n_win, window, blocks, rows, stats); note_launch(); }
   GPA_CUDA(cudaGetLastError());
 }
 
 void launch_row_begin(const uint32_t* row_off, uint32_t n_blocks, TrieBlock* blocks, int n_sms, cudaStream_t s) {
   if (n_blocks == 0) return;
-  row_begin_kernel<<<grid_for(n_blocks, n_sms), kThreads, 0, s>>>(row_off, n_blocks, blocks);
+  { row_begin_kernel<<<grid_for(n_blocks, n_sms), kThreads, 0, s>>>(row_off, n_blocks, blocks); note_launch(); }
   GPA_CUDA(cudaGetLastError());
 }
 
@@ -231,15 +231,15 @@ void launch_build_blocks(const uint32_t* prefix, const uint32_t* ext, const uint
                          uint32_t n_rows, TrieBlock* blocks, uint32_t n_blocks, uint32_t* trows, uint4* lrows,
                          uint8_t* lcp, cudaStream_t s) {
   if (n_blocks == 0) return;
-  build_blocks_kernel<<<n_blocks, kThreads, 0, s>>>(prefix, ext, cand_group, k, n_rows, blocks, trows, lrows, lcp);
+  { build_blocks_kernel<<<n_blocks, kThreads, 0, s>>>(prefix, ext, cand_group, k, n_rows, blocks, trows, lrows, lcp); note_launch(); }
   GPA_CUDA(cudaGetLastError());
 }
 
 void launch_prefix_tasks(const uint32_t* ext_off, uint32_t G, uint32_t* n_tasks, const uint32_t* task_off,
                          PrefixTask* tasks, int n_sms, cudaStream_t s, bool write) {
   if (G == 0) return;
-  if (!write) task_count_kernel<<<grid_for(G, n_sms), kThreads, 0, s>>>(ext_off, G, n_tasks);
-  else task_write_kernel<<<grid_for(G, n_sms), kThreads, 0, s>>>(ext_off, G, task_off, tasks);
+  if (!write) { task_count_kernel<<<grid_for(G, n_sms), kThreads, 0, s>>>(ext_off, G, n_tasks); note_launch(); }
+  else { task_write_kernel<<<grid_for(G, n_sms), kThreads, 0, s>>>(ext_off, G, task_off, tasks); note_launch(); }
   GPA_CUDA(cudaGetLastError());
 }
 

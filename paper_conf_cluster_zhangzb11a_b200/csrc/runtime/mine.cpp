@@ -428,3 +428,5 @@ extern "C" gpa_status gpa_result_destroy(gpa_result* r) {
 extern "C" const char* gpa_last_error(void) { return gpa::last_error_cstr(); }
 
 extern "C" const char* gpa_version(void) { return "gpapriori-b200 0.1 sm_100a"; }
+
+extern "C" uint64_t gpa_kernel_launches(void) { return gpa::g_kernel_launches.load(std::memory_order_relaxed); }
