@@ -37,10 +37,10 @@ void set_last_error(gpa_status st, const std::string& msg);
   } while (0)
 
 // Row layout of the static bitset: pitch (in 32-bit words) is a multiple of this many words
-// (1 KB = 8,192 transactions).  The paper aligns rows to 64 bytes (P18@1685); 1 KB is a whole
-// number of 128-B L2 lines / TMA 128B-swizzle spans (pair kernel) and of the trie kernel's
-// 128- and 256-word stripes, so no kernel ever handles a ragged row tail.
-constexpr uint64_t kPitchWords = 256;
+// (4 KB = 32,768 transactions).  The paper aligns rows to 64 bytes (P18@1685); 4 KB is a whole
+// number of 128-B L2 lines / TMA boxes (pair kernels) and of every trie stripe (128 / 256 words
+// in shared memory, 1,024 words in tensor memory), so no kernel ever handles a ragged row tail.
+constexpr uint64_t kPitchWords = 1024;
 
 inline uint64_t pitch_words_for(uint64_t n_tx) {
   uint64_t w = (n_tx + 31) / 32;

@@ -69,6 +69,13 @@ uint64_t launch_count_trie(uint32_t k, const uint32_t* rows, uint64_t pitch_word
                            uint32_t n_blocks, uint32_t max_rows, uint32_t n_parts, uint32_t* counts,
                            cudaStream_t stream);
 
+// Same walk with the stripe's rows staged in tensor memory (count_trie_tm.cu), 3 <= k <= 16,
+// blocks of <= kTrieWideRows rows; identical results.
+uint64_t launch_count_trie_tm(uint32_t k, const uint32_t* rows, uint64_t pitch_words, const TrieBlock* blocks,
+                              const uint32_t* block_rows, const uint4* cand_lrows, const uint8_t* cand_lcp,
+                              uint32_t n_blocks, uint32_t max_rows, uint32_t n_parts, uint32_t* counts,
+                              cudaStream_t stream);
+
 // k = 2 TMA-tiled kernel: all pairs (a < b) of the n_rows rows; counts[pair_index] must be zeroed.
 // tmap: opaque 128-byte CUtensorMap built by make_pairs_tensor_map.
 bool make_pairs_tensor_map(void* tmap128, const uint32_t* rows, uint32_t n_rows, uint64_t pitch_words);

@@ -28,6 +28,25 @@ static double auto_sibling_cut() {
 
 namespace {
 
+// k >= 3 trie walk: rows staged in shared memory (count_trie.cu); GPA_TRIE_TMEM=1 selects the
+// tensor-memory variant (count_trie_tm.cu) -- correct, but measured 1.6x slower on T40I10D10M
+// (DESIGN.md "Kernels"), so it is an experiment, not a default
+bool trie_tmem() {
+  static const bool v = [] {
+    const char* e = getenv("GPA_TRIE_TMEM");
+    return e && atoi(e) != 0;
+  }();
+  return v;
+}
+void launch_trie(uint32_t k, const uint32_t* rows, uint64_t pitch_words, const TrieBlock* blocks,
+                 const uint32_t* block_rows, const uint4* lrows, const uint8_t* lcp, uint32_t n_blocks,
+                 uint32_t max_rows, uint32_t n_parts, uint32_t* counts, cudaStream_t s) {
+  if (k >= 3 && max_rows <= kTrieWideRows && trie_tmem())
+    launch_count_trie_tm(k, rows, pitch_words, blocks, block_rows, lrows, lcp, n_blocks, max_rows, n_parts, counts, s);
+  else
+    launch_count_trie(k, rows, pitch_words, blocks, block_rows, lrows, lcp, n_blocks, max_rows, n_parts, counts, s);
+}
+
 double now_ms() {
   return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now().time_since_epoch()).count();
 }
@@ -263,8 +282,8 @@ void count_trie_batch(gpa_bitset* bs, const GroupedBatch& b, CountStats* st) {
   GPA_CUDA(cudaMemsetAsync(bs->d_counts.p, 0, M * sizeof(uint32_t), s));
   GPA_CUDA(cudaEventRecord(ev_start(bs, st), s));
   if (bs->n_rows)
-    launch_count_trie(k, bs->rows.p, bs->pitch_words, bs->d_tblocks.p, bs->d_trows.p, bs->d_lrows.p, bs->d_lcp.p,
-                      n_blocks, max_rows, n_parts, bs->d_counts.p, s);
+    launch_trie(k, bs->rows.p, bs->pitch_words, bs->d_tblocks.p, bs->d_trows.p, bs->d_lrows.p, bs->d_lcp.p,
+                n_blocks, max_rows, n_parts, bs->d_counts.p, s);
   if (st) { st->kernel = GPA_KERNEL_TRIE; st->launches = 1; }
   const double tp2 = wall_ms();
   finish_counts(bs, M, st);
@@ -355,8 +374,8 @@ bool count_device_batch(gpa_bitset* bs, DeviceBatch& B, uint32_t kernel, DeviceS
   GPA_CUDA(cudaMemsetAsync(bs->d_counts.p, 0, (size_t)M * 4, s));
   const double tp1 = wall_ms();
   GPA_CUDA(cudaEventRecord(ev_start(bs, st), s));
-  launch_count_trie(k, bs->rows.p, bs->pitch_words, bs->d_tblocks.p, bs->d_trows.p, bs->d_lrows.p, bs->d_lcp.p,
-                    n_blocks, max_rows, n_parts, bs->d_counts.p, s);
+  launch_trie(k, bs->rows.p, bs->pitch_words, bs->d_tblocks.p, bs->d_trows.p, bs->d_lrows.p, bs->d_lcp.p,
+              n_blocks, max_rows, n_parts, bs->d_counts.p, s);
   if (st) { st->kernel = GPA_KERNEL_TRIE; st->launches = 1; }
   finish_counts(bs, M, st);
   if (trace_enabled())
