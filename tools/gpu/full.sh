@@ -11,7 +11,8 @@ timeout 900 python bench.py --impl reference --steps 2 --warmup 1 > gpurun_out/b
 timeout 900 python bench.py --dist --steps 3 --warmup 1 --no-cpu-baseline > gpurun_out/bench_dist1.log 2>&1; echo "dist rc=$?" >> gpurun_out/bench_dist1.log
 B="python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu-baseline"
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches.csv $B > gpurun_out/ncu_launch.log 2>&1
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:count_pairs -c 1 -o gpurun_out/prof_pairs $B > gpurun_out/ncu_pairs.log 2>&1
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:count_trie -s 3 -c 1 -o gpurun_out/prof_trie $B > gpurun_out/ncu_trie.log 2>&1
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:count_prefix -c 1 -o gpurun_out/prof_prefix $B > gpurun_out/ncu_prefix.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:count_pairs_tc -c 1 -o gpurun_out/prof_pairs_tc $B > gpurun_out/ncu_pairs_tc.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:"count_pairs_kernel" -c 1 -o gpurun_out/prof_pairs $B --kernel pairs > gpurun_out/ncu_pairs.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:"count_trie_kernel<7" -c 1 -o gpurun_out/prof_trie $B > gpurun_out/ncu_trie.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:count_prefix -c 1 -o gpurun_out/prof_prefix $B --kernel prefix > gpurun_out/ncu_prefix.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:"bitset_build|hist_validate" -c 2 -o gpurun_out/prof_build $B > gpurun_out/ncu_build.log 2>&1
