@@ -44,7 +44,7 @@ def parse():
     p.add_argument("--warmup", type=int, default=3)
     p.add_argument("--impl", choices=["ours", "reference"], default="ours")
     p.add_argument("--config", default="t40i10d10m", choices=list(gen.CONFIGS))
-    p.add_argument("--kernel", default="auto", choices=["auto", "v0", "prefix", "pairs", "trie", "pairs_tc"])
+    p.add_argument("--kernel", default="auto", choices=["auto", "v0", "prefix", "pairs", "trie", "pairs_tc", "proj"])
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--dist", action="store_true", help="use the NCCL path even with one rank")
     p.add_argument("--all-configs", action="store_true",
@@ -235,7 +235,8 @@ def main():
         theta = max(1, theta * (b1 - b0) // cfg.n_tx)
     ds = gen.make(cfg.name, tx_begin=b0, tx_end=b1)
     kern = {"auto": gpa.KERNEL_AUTO, "v0": gpa.KERNEL_V0, "prefix": gpa.KERNEL_PREFIX,
-            "pairs": gpa.KERNEL_PAIRS, "trie": gpa.KERNEL_TRIE, "pairs_tc": gpa.KERNEL_PAIRS_TC}[args.kernel]
+            "pairs": gpa.KERNEL_PAIRS, "trie": gpa.KERNEL_TRIE, "pairs_tc": gpa.KERNEL_PAIRS_TC,
+            "proj": gpa.KERNEL_PROJ}[args.kernel]
     stream = torch.cuda.current_stream()
     opts = gpa.Options(count_kernel=kern, stream=stream.cuda_stream, device=local)
     d_off = torch.from_numpy(ds.offsets.view(np.int64)).cuda()

@@ -99,13 +99,19 @@ typedef struct {
 } gpa_tx_csr;
 
 /* Counting kernel selection. */
-#define GPA_KERNEL_AUTO 0u     /* PAIRS_TC for k = 2, TRIE for 3 <= k <= 16, PREFIX above */
+#define GPA_KERNEL_AUTO 0u     /* gpa_mine: PAIRS_TC for k = 2, PROJ for k >= 3 (TRIE / PREFIX if the projected
+                                  lists do not fit); gpa_count: TRIE for 3 <= k <= 16, PREFIX above */
 #define GPA_KERNEL_V0 1u       /* the paper's design: one CTA per candidate, AND of all k rows */
 #define GPA_KERNEL_PREFIX 2u   /* prefix-staged streaming: (k-1)-prefix AND held on chip, siblings streamed */
 #define GPA_KERNEL_PAIRS 3u    /* k = 2 only: TMA-tiled AND-popcount "Gram" tile kernel */
 #define GPA_KERNEL_TRIE 4u     /* 2 <= k <= 16: transaction-tiled trie walk, rows staged in shared memory */
 #define GPA_KERNEL_PAIRS_TC 5u /* k = 2 only: the pair Gram B B^T of the 0/1 rows as a tcgen05 integer GEMM
                                   (kind::i8, s32 accumulators in TMEM); exact, same counts as PAIRS */
+#define GPA_KERNEL_PROJ 6u     /* gpa_mine, k >= 3: "equivalent class clustering" (P13@2288-2486) on projected
+                                  vertical lists -- each L_{k-1} member keeps its last item's bits restricted
+                                  to the transactions of its (k-2)-prefix; a candidate's support is the
+                                  popcount of the AND of its two parents' lists (exact, same counts as
+                                  complete intersection).  k = 2 as AUTO; gpa_count treats it as AUTO */
 
 #define GPA_KEEP_CANDIDATES 1u /* gpa_mine: keep every generation's (C_k, counts), not only F */
 #define GPA_HOST_CANDGEN 2u    /* gpa_mine: join + prune on the host thread pool instead of the device

@@ -27,14 +27,14 @@ import numpy as np
 
 __all__ = [
     "GpaError", "lib", "version", "min_count", "Options", "Dist", "Bitset", "mine", "MineResult",
-    "KERNEL_AUTO", "KERNEL_V0", "KERNEL_PREFIX", "KERNEL_PAIRS", "KERNEL_TRIE", "KERNEL_PAIRS_TC", "PHASES",
+    "KERNEL_AUTO", "KERNEL_V0", "KERNEL_PREFIX", "KERNEL_PAIRS", "KERNEL_TRIE", "KERNEL_PAIRS_TC", "KERNEL_PROJ", "PHASES",
 ]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libgpapriori.so")
 
-KERNEL_AUTO, KERNEL_V0, KERNEL_PREFIX, KERNEL_PAIRS, KERNEL_TRIE, KERNEL_PAIRS_TC = 0, 1, 2, 3, 4, 5
-KERNEL_NAMES = {0: "auto", 1: "v0", 2: "prefix", 3: "pairs", 4: "trie", 5: "pairs_tc"}
+KERNEL_AUTO, KERNEL_V0, KERNEL_PREFIX, KERNEL_PAIRS, KERNEL_TRIE, KERNEL_PAIRS_TC, KERNEL_PROJ = 0, 1, 2, 3, 4, 5, 6
+KERNEL_NAMES = {0: "auto", 1: "v0", 2: "prefix", 3: "pairs", 4: "trie", 5: "pairs_tc", 6: "proj"}
 KEEP_CANDIDATES = 1
 HOST_CANDGEN = 2
 NO_OVERLAP_INGEST = 4

@@ -22,6 +22,8 @@ struct Error {
 };
 
 [[noreturn]] void fail(gpa_status st, const char* fmt, ...) __attribute__((format(printf, 2, 3)));
+bool trace_enabled();   // GPA_TRACE=1 (runtime/context.cpp)
+double wall_ms();       // host steady clock, ms
 void set_last_error(gpa_status st, const std::string& msg);
 
 #define GPA_CUDA(call)                                                                              \
@@ -89,6 +91,39 @@ struct DBuf {
   // grow-only reuse
   void ensure(size_t count, cudaStream_t stream) {
     if (count > n || stream != s) alloc(count, stream);
+  }
+};
+
+// Persistent grow-only device buffer (cudaMalloc / cudaFree, not stream-ordered): for the large
+// per-generation workspaces (projected lists) that a stream-ordered pool would re-map on every
+// call -- measured: cudaMallocAsync of 0.7 GB blocking the host for up to 0.5 s once the pool
+// fragments.  Grows by 1.25x so that a sequence of mining calls settles on one allocation.
+template <class T>
+struct PBuf {
+  T* p = nullptr;
+  size_t n = 0;
+  PBuf() = default;
+  PBuf(const PBuf&) = delete;
+  PBuf& operator=(const PBuf&) = delete;
+  ~PBuf() {
+    if (p) cudaFree(p);
+  }
+  T* ensure(size_t count) {
+    if (count == 0) count = 1;
+    if (count <= n) return p;
+    if (p) cudaFree(p);  // synchronises: no kernel still reads the old buffer
+    p = nullptr;
+    n = 0;
+    const size_t want = count + count / 4;
+    cudaError_t e = cudaMalloc(reinterpret_cast<void**>(&p), want * sizeof(T));
+    if (e != cudaSuccess) {
+      p = nullptr;
+      cudaGetLastError();
+      fail(e == cudaErrorMemoryAllocation ? GPA_ERR_OOM : GPA_ERR_CUDA, "device allocation of %zu bytes failed: %s",
+           want * sizeof(T), cudaGetErrorString(e));
+    }
+    n = want;
+    return p;
   }
 };
 

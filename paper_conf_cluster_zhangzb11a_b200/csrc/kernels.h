@@ -87,7 +87,8 @@ uint64_t launch_count_pairs(const void* tmap128, uint32_t n_rows, uint64_t word_
 uint64_t launch_count_pairs_tc(const uint32_t* rows, uint64_t pitch_words, uint32_t n_rows, uint64_t word_begin,
                                uint64_t word_end, uint32_t* counts, int n_sms, cudaStream_t stream);
 inline bool pairs_kernel_k2(uint32_t kernel) {
-  return kernel == GPA_KERNEL_AUTO || kernel == GPA_KERNEL_PAIRS || kernel == GPA_KERNEL_PAIRS_TC;
+  return kernel == GPA_KERNEL_AUTO || kernel == GPA_KERNEL_PAIRS || kernel == GPA_KERNEL_PAIRS_TC ||
+         kernel == GPA_KERNEL_PROJ;
 }
 // counts_sub[pair_index(a, b, n_sub)] = counts_all[pair_index(sel[a], sel[b], n_all)] (sel ascending)
 void launch_pairs_subset(const uint32_t* counts_all, uint32_t n_all, const uint32_t* sel, uint32_t n_sub,
@@ -112,20 +113,52 @@ struct DeviceScratch {
   void* get(size_t bytes, cudaStream_t s) { tmp.ensure(bytes ? bytes : 1, s); return tmp.p; }
 };
 // L_k on the device: n rows of k row ids (lexicographic) and their supports
+// par_a[p] / par_b[p]: index in L_{k-1} of the entry's left parent (its first k-1 items) and
+// right parent (first k-2 items + last item); for k = 2 the two row ids.  Used by the projected
+// lists of proj.cu.
 struct DeviceLevel {
   uint32_t k = 0, n = 0;
-  DBuf<uint32_t> rows, sup;
+  DBuf<uint32_t> rows, sup, par_a, par_b;
 };
 // C_k on the device, grouped by (k-1)-prefix: prefix[G][k-1], ext_off[G+1], ext[M]
+// gpar[g] = index in L_{k-1} of group g's prefix (the left parent), eidx[m] = index in L_{k-1} of
+// candidate m's right parent (prefix without its last item, plus ext[m]).
 struct DeviceBatch {
   uint32_t k = 0, M = 0, G = 0;
-  DBuf<uint32_t> prefix, ext_off, ext;
+  DBuf<uint32_t> prefix, ext_off, ext, gpar, eidx;
 };
 // L_k = candidates of C_k with count >= theta, in order (k = 2: all pairs of n_rows rows in
 // pair_index order; k >= 3: the grouped batch prefix/ext_off/ext).  Returns |L_k| (synchronises).
+// With gpar / eidx (k >= 3) or always for k = 2, also out.par_a / out.par_b.
 uint32_t device_threshold(const uint32_t* counts, uint32_t M, uint32_t theta, uint32_t k, uint32_t n_rows,
                           const uint32_t* prefix, const uint32_t* ext_off, const uint32_t* ext, uint32_t G,
+                          const uint32_t* gpar, const uint32_t* eidx,
                           DeviceLevel& out, DeviceScratch& scratch, int n_sms, cudaStream_t s);
+
+// ---- projected vertical lists (proj.cu; "equivalent class clustering", P13@2288-2486)
+// For every entry j of a level L (n entries with parents par_a / par_b): the bits of its last
+// item's row restricted to the transactions of its class (the entries with the same par_a), in
+// the class' position order.  Entries of single-member classes (no candidates) get no vector.
+// Buffers are persistent and grow-only (PBuf): one DeviceProj pair per thread and device lives
+// across generations and mining calls (proj_lists()).
+struct DeviceProj {
+  uint32_t n = 0;
+  PBuf<uint64_t> off;     // n: word offset of entry j's vector in data
+  PBuf<uint32_t> nw;      // n: words of entry j's vector (multiple of 32; 0 = none)
+  PBuf<uint32_t> data;
+  uint64_t words = 0;
+};
+// The calling thread's two DeviceProj for `device` (previous / current generation).
+DeviceProj* proj_lists(int device);
+// Vectors of L = L_{k-1} from the previous level's vectors (prev = those of L_{k-2}) or, for
+// L = L_2 (prev == nullptr), from the bitset rows.  Synchronises once (sizes).  Returns false
+// when the vectors do not fit (device memory / 32-bit totals): use complete intersection.
+bool proj_build(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const DeviceProj* prev,
+                const uint32_t* rows, uint64_t pitch_words, uint32_t n_rows, DeviceProj& out, DeviceScratch& scratch,
+                int n_sms, cudaStream_t s);
+// counts[m] += popc(V_gpar[g] & V_eidx[m]) for every candidate m of group g (counts zeroed by the caller)
+void launch_count_proj(const DeviceProj& P, const uint32_t* gpar, const uint32_t* ext_off, const uint32_t* eidx,
+                       uint32_t G, uint32_t* counts, cudaStream_t s);
 // items[i] = item_of_row[rows[i]] (row ids -> original item ids)
 void device_map_items(const uint32_t* rows, uint64_t n, const uint32_t* item_of_row, uint32_t* items, int n_sms,
                       cudaStream_t s);

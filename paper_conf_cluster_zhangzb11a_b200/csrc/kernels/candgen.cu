@@ -75,7 +75,7 @@ __global__ void flag_ge_kernel(const uint32_t* __restrict__ counts, uint32_t M, 
 // k = 2: candidate m is the pair (a, b) of pair_index order over n rows
 __global__ void scatter_pairs_kernel(const uint32_t* __restrict__ counts, const uint32_t* __restrict__ flags,
                                      const uint32_t* __restrict__ pos, uint32_t M, uint32_t n, uint32_t* L,
-                                     uint32_t* sup) {
+                                     uint32_t* sup, uint32_t* par_a, uint32_t* par_b) {
   for (uint32_t m = blockIdx.x * blockDim.x + threadIdx.x; m < M; m += gridDim.x * blockDim.x) {
     if (!flags[m]) continue;
     uint32_t lo = 0, hi = n - 1;  // a = last row whose first pair index <= m
@@ -88,6 +88,8 @@ __global__ void scatter_pairs_kernel(const uint32_t* __restrict__ counts, const 
     L[2ull * p] = a;
     L[2ull * p + 1] = b;
     sup[p] = counts[m];
+    par_a[p] = a;
+    par_b[p] = b;
   }
 }
 
@@ -95,8 +97,9 @@ __global__ void scatter_pairs_kernel(const uint32_t* __restrict__ counts, const 
 __global__ void scatter_grouped_kernel(const uint32_t* __restrict__ counts, const uint32_t* __restrict__ flags,
                                        const uint32_t* __restrict__ pos, uint32_t M,
                                        const uint32_t* __restrict__ prefix, const uint32_t* __restrict__ ext_off,
-                                       const uint32_t* __restrict__ ext, uint32_t G, uint32_t km1, uint32_t* L,
-                                       uint32_t* sup) {
+                                       const uint32_t* __restrict__ ext, uint32_t G, uint32_t km1,
+                                       const uint32_t* __restrict__ gpar, const uint32_t* __restrict__ eidx,
+                                       uint32_t* L, uint32_t* sup, uint32_t* par_a, uint32_t* par_b) {
   for (uint32_t m = blockIdx.x * blockDim.x + threadIdx.x; m < M; m += gridDim.x * blockDim.x) {
     if (!flags[m]) continue;
     uint32_t lo = 0, hi = G;  // g = last group with ext_off[g] <= m
@@ -109,6 +112,10 @@ __global__ void scatter_grouped_kernel(const uint32_t* __restrict__ counts, cons
     for (uint32_t d = 0; d < km1; ++d) dst[d] = prefix[(uint64_t)lo * km1 + d];
     dst[km1] = ext[m];
     sup[p] = counts[m];
+    if (gpar) {
+      par_a[p] = gpar[lo];
+      par_b[p] = eidx[m];
+    }
   }
 }
 
@@ -134,7 +141,7 @@ __global__ void join_kernel(const uint32_t* __restrict__ L, uint32_t n, uint32_t
                             const uint32_t* __restrict__ run_ex, const uint32_t* __restrict__ bound,
                             const uint32_t* __restrict__ slots, uint32_t mask, uint32_t* cnt,
                             const uint32_t* __restrict__ cand_off, const uint32_t* __restrict__ gidx,
-                            uint32_t* prefix, uint32_t* ext_off, uint32_t* ext) {
+                            uint32_t* prefix, uint32_t* ext_off, uint32_t* ext, uint32_t* gpar, uint32_t* eidx) {
   uint32_t probe[GPA_MAX_K];
   uint64_t A[GPA_MAX_K], B[GPA_MAX_K];
   const uint32_t lane = threadIdx.x & 31;
@@ -184,13 +191,20 @@ __global__ void join_kernel(const uint32_t* __restrict__ L, uint32_t n, uint32_t
         }
       }
       const uint32_t ballot = __ballot_sync(0xffffffffu, keep);
-      if (EMIT && keep) ext[cand_off[x] + here + __popc(ballot & ((1u << lane) - 1u))] = b;
+      if (EMIT && keep) {
+        const uint32_t at = cand_off[x] + here + __popc(ballot & ((1u << lane) - 1u));
+        ext[at] = b;
+        eidx[at] = y;
+      }
       here += __popc(ballot);
     }
     if (EMIT) {
       const uint32_t g = gidx[x];
       for (uint32_t i = lane; i < w; i += 32) prefix[(uint64_t)g * w + i] = px[i];
-      if (lane == 0) ext_off[g] = cand_off[x];
+      if (lane == 0) {
+        ext_off[g] = cand_off[x];
+        gpar[g] = x;
+      }
     } else if (lane == 0) {
       cnt[x] = here;
     }
@@ -244,6 +258,7 @@ void exclusive_scan(const uint32_t* in, uint32_t* out, uint32_t n, uint32_t* tot
 
 uint32_t device_threshold(const uint32_t* counts, uint32_t M, uint32_t theta, uint32_t k, uint32_t n_rows,
                           const uint32_t* prefix, const uint32_t* ext_off, const uint32_t* ext, uint32_t G,
+                          const uint32_t* gpar, const uint32_t* eidx,
                           DeviceLevel& out, DeviceScratch& scratch, int n_sms, cudaStream_t s) {
   out.k = k;
   out.n = 0;
@@ -259,13 +274,16 @@ uint32_t device_threshold(const uint32_t* counts, uint32_t M, uint32_t theta, ui
   GPA_CUDA(cudaStreamSynchronize(s));
   out.rows.ensure((size_t)std::max<uint32_t>(F, 1) * k, s);
   out.sup.ensure(std::max<uint32_t>(F, 1), s);
+  out.par_a.ensure(std::max<uint32_t>(F, 1), s);
+  out.par_b.ensure(std::max<uint32_t>(F, 1), s);
   if (F) {
     if (k == 2)
       { scatter_pairs_kernel<<<grid_for(M, n_sms), kThreads, 0, s>>>(counts, flags, pos, M, n_rows, out.rows.p,
-                                                                  out.sup.p); note_launch(); }
+                                                                  out.sup.p, out.par_a.p, out.par_b.p); note_launch(); }
     else
       { scatter_grouped_kernel<<<grid_for(M, n_sms), kThreads, 0, s>>>(counts, flags, pos, M, prefix, ext_off, ext, G,
-                                                                    k - 1, out.rows.p, out.sup.p); note_launch(); }
+                                                                    k - 1, gpar, eidx, out.rows.p, out.sup.p,
+                                                                    out.par_a.p, out.par_b.p); note_launch(); }
     GPA_CUDA(cudaGetLastError());
   }
   out.n = F;
@@ -306,7 +324,7 @@ void device_candgen(const DeviceLevel& L, DeviceBatch& out, DeviceScratch& scrat
   GPA_CUDA(cudaMemsetAsync(slots, 0xff, (size_t)cap * 4, s));
   { hash_build_kernel<<<grid_for(n, n_sms), kThreads, 0, s>>>(L.rows.p, n, w, slots, cap - 1); note_launch(); }
   { join_kernel<false><<<grid_for(32ull * n, n_sms), kThreads, 0, s>>>(L.rows.p, n, w, flags, run_ex, bound, slots, cap - 1, cnt,
-                                                             nullptr, nullptr, nullptr, nullptr, nullptr); note_launch(); }
+                                                             nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr); note_launch(); }
   GPA_CUDA(cudaGetLastError());
   uint32_t* cand_off = scratch.u32e(n, s);
   uint32_t* gflag = scratch.u32f(n, s);
@@ -322,8 +340,11 @@ void device_candgen(const DeviceLevel& L, DeviceBatch& out, DeviceScratch& scrat
   out.prefix.ensure((size_t)G * w, s);
   out.ext_off.ensure(G + 1, s);
   out.ext.ensure(M, s);
+  out.gpar.ensure(G, s);
+  out.eidx.ensure(M, s);
   { join_kernel<true><<<grid_for(32ull * n, n_sms), kThreads, 0, s>>>(L.rows.p, n, w, flags, run_ex, bound, slots, cap - 1, cnt,
-                                                            cand_off, gidx, out.prefix.p, out.ext_off.p, out.ext.p); note_launch(); }
+                                                            cand_off, gidx, out.prefix.p, out.ext_off.p, out.ext.p,
+                                                            out.gpar.p, out.eidx.p); note_launch(); }
   GPA_CUDA(cudaGetLastError());
   { ext_end_kernel<<<1, 32, 0, s>>>(sizes, out.ext_off.p); note_launch(); }
   out.M = M;

@@ -1,0 +1,454 @@
+// Projected vertical lists: generation k >= 3 counted on equivalence classes (sm_100a).
+//
+// The paper contrasts two ways of computing a candidate's vertical list (PAPER.md P13@2288-2486,
+// P18@1089): "equivalent class clustering" (Zaki) keeps the vertical lists of generation k-1 and
+// intersects two of them, while GPApriori's "complete intersection" re-ANDs k generation-1 rows
+// to save memory.  With 180 GB of HBM the first one is affordable once the
+// kept lists are stored COMPACTLY: the class of a (k-1)-itemset X = Q u {x} is its (k-2)-prefix
+// Q, and the kept list of X is the bit-row of x restricted to the transactions of Q,
+//
+//     V_X[i] = B[x][t_i],   t_0 < t_1 < ... the transactions containing Q   (|V_X| = supp(Q) bits),
+//
+// so that every member of a class shares one position list and one bit order, and a candidate
+// Q u {a, b} (parents Q u {a}, Q u {b}, P13@1006-1270) has
+//
+//     supp(Q u {a, b}) = popc(V_{Q u {a}} AND V_{Q u {b}})                 (count_proj_kernel),
+//
+// the same popcount-of-AND as complete intersection (P18@394), over supp(Q) bits instead of N.
+// The next generation's lists follow from this one's: the class of X' = Q u {a, b} is Q u {a},
+// whose transactions are the set bits of V_{Q u {a}}; hence V_{X'} = the bits of V_{Q u {b}} at
+// the set positions of V_{Q u {a}}: a parallel bit extract, pext(V_{Q u {b}}, V_{Q u {a}}),
+// word by word (pext_kernel; Hacker's Delight "compress", the mask-dependent half computed once
+// per mask word and shared by every member of the class).  Generation 3 starts from the static
+// bitset itself: the class of a pair {a, b} is {a}, mask = row a, sources = rows b (the "static
+// bitset" of P2@270 / P18@755 stays the only input).
+//
+// Layout: LANE-INTERLEAVED.  A vector is 32 bit streams ("lanes") of Lw words each, word j of
+// lane l at index 32 j + l; a bitset row is such a vector with Lw = pitch / 32.  Lane l of a new
+// vector is the pext of lane l of its source by lane l of its mask, so a warp's lane l only ever
+// touches lane l: every load is a coalesced 128-byte row, no cross-lane bit placement.  The
+// members of a class share one mask, hence one per-lane bit count and one layout: Lw_c = max
+// over lanes of the lane's words (each lane's tail zero-padded), members contiguous.  A bitset
+// row is cut into segments of kSegJ words per lane, each lane padded to whole words per segment,
+// so segments are independent work items.  All integer; counts are exact by construction.
+#include <cstdint>
+#include <map>
+#include <cub/block/block_scan.cuh>
+#include <cub/device/device_scan.cuh>
+
+#include "../common.h"
+#include "../kernels.h"
+
+namespace gpa {
+namespace {
+
+constexpr int kT = 256;
+constexpr uint32_t kSegJ = 256;          // segment of a bitset row: 256 words per lane (262,144 transactions)
+constexpr uint32_t kMemberGroup = 8;     // members sharing one mask preparation in pext_kernel
+
+unsigned grid_for(uint64_t n, int n_sms, int per_sm = 16) {
+  uint64_t g = (n + kT - 1) / kT;
+  const uint64_t cap = (uint64_t)n_sms * per_sm;
+  return (unsigned)(g < 1 ? 1 : (g > cap ? cap : g));
+}
+
+// ---------------------------------------------------------------- class structure
+// A class = a run of entries with the same par_a (the left parent = the (k-2)-prefix).
+__global__ void cls_flag_kernel(const uint32_t* __restrict__ par_a, uint32_t n, uint32_t* __restrict__ flag) {
+  for (uint32_t j = blockIdx.x * blockDim.x + threadIdx.x; j < n; j += gridDim.x * blockDim.x)
+    flag[j] = j == 0 || par_a[j] != par_a[j - 1];
+}
+
+__global__ void cls_bound_kernel(const uint32_t* __restrict__ flag, const uint32_t* __restrict__ ex, uint32_t n,
+                                 uint32_t* __restrict__ bound, uint32_t* __restrict__ n_cls) {
+  for (uint32_t j = blockIdx.x * blockDim.x + threadIdx.x; j < n; j += gridDim.x * blockDim.x) {
+    if (flag[j]) bound[ex[j]] = j;
+    if (j == n - 1) {
+      const uint32_t C = ex[j] + flag[j];
+      bound[C] = n;
+      *n_cls = C;
+    }
+  }
+}
+
+struct VecRef {
+  const uint32_t* p;
+  uint32_t lw;  // words per lane
+};
+
+// The mask of a class / the source of a member: a bitset row (generation 3) or one of the
+// previous generation's vectors.
+struct Src {
+  const uint32_t* rows;        // non-null: generation 3
+  uint64_t pitch;
+  const uint32_t* data;        // previous generation's vectors
+  const uint64_t* off;
+  const uint32_t* nw;
+  __device__ __forceinline__ VecRef vec(uint32_t id) const {
+    if (rows) return VecRef{rows + (uint64_t)id * pitch, (uint32_t)(pitch / 32)};
+    return VecRef{data + off[id], nw[id] / 32u};
+  }
+};
+
+__device__ __forceinline__ void seg_range(uint32_t lw, uint32_t nseg, uint32_t s, uint32_t& j0, uint32_t& j1) {
+  const uint32_t seg = nseg == 1 ? lw : kSegJ;
+  j0 = s * seg;
+  j1 = min(lw, j0 + seg);
+}
+
+// warp per (segment s, class c) pair p = s * cmax + c: lane l's mask popcount in the segment ->
+// words[p][l] = its output words (bits rounded up to whole words)
+__global__ void seg_popc_kernel(Src src, const uint32_t* __restrict__ par_a, const uint32_t* __restrict__ bound,
+                                const uint32_t* __restrict__ n_cls, uint32_t cmax, uint32_t nseg, uint32_t n_pairs,
+                                uint32_t* __restrict__ words) {
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t p = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  if (p >= n_pairs) return;
+  const uint32_t c = p % cmax, s = p / cmax;
+  uint32_t cnt = 0;
+  if (c < *n_cls) {
+    const uint32_t j0 = bound[c], m = bound[c + 1] - j0;
+    if (m >= 2) {
+      const VecRef mk = src.vec(par_a[j0]);
+      uint32_t a, b;
+      seg_range(mk.lw, nseg, s, a, b);
+      for (uint32_t j = a; j < b; ++j) cnt += __popc(mk.p[32ull * j + lane]);
+    }
+  }
+  words[(uint64_t)p * 32 + lane] = (cnt + 31) / 32;
+}
+
+// warp per class: lane l's word offset of every segment (loc), Lw_c = max over lanes of the
+// lane's total, words per member nwc = 32 Lw_c, the class' words and its pext items (one per
+// segment and group of kMemberGroup members)
+__global__ void cls_pad_kernel(const uint32_t* __restrict__ words, const uint32_t* __restrict__ bound,
+                               const uint32_t* __restrict__ n_cls, uint32_t cmax, uint32_t nseg,
+                               uint32_t* __restrict__ loc, uint32_t* __restrict__ nwc,
+                               uint64_t* __restrict__ cls_words, uint32_t* __restrict__ items) {
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  if (c >= cmax) return;
+  uint32_t m = 0;
+  if (c < *n_cls) m = bound[c + 1] - bound[c];
+  const uint32_t groups = m >= 2 ? (m + kMemberGroup - 1) / kMemberGroup : 0;
+  uint32_t acc = 0;
+  for (uint32_t s = 0; s < nseg; ++s) {
+    const uint64_t p = (uint64_t)s * cmax + c;
+    loc[p * 32 + lane] = acc;
+    acc += words[p * 32 + lane];
+    if (lane == 0) items[p] = groups;
+  }
+  const uint32_t lw = __reduce_max_sync(0xffffffffu, acc);
+  if (lane == 0) {
+    nwc[c] = groups ? 32u * lw : 0u;
+    cls_words[c] = groups ? (uint64_t)32u * lw * m : 0ull;
+  }
+}
+
+// entry j -> its vector (offset, words); entries of single-member classes get none
+__global__ void entry_off_kernel(const uint32_t* __restrict__ flag, const uint32_t* __restrict__ ex,
+                                 const uint32_t* __restrict__ bound, const uint32_t* __restrict__ nwc,
+                                 const uint64_t* __restrict__ cls_base, uint32_t n, uint64_t* __restrict__ off,
+                                 uint32_t* __restrict__ nw) {
+  for (uint32_t j = blockIdx.x * blockDim.x + threadIdx.x; j < n; j += gridDim.x * blockDim.x) {
+    const uint32_t c = ex[j] + flag[j] - 1;
+    const uint32_t j0 = bound[c], m = bound[c + 1] - j0;
+    if (m < 2) {
+      off[j] = 0;
+      nw[j] = 0;
+    } else {
+      nw[j] = nwc[c];
+      off[j] = cls_base[c] + (uint64_t)(j - j0) * nwc[c];
+    }
+  }
+}
+
+// Hacker's Delight 7-4 "compress" (= pext): the mask-dependent shift masks, then the per-source
+// part (x already ANDed with the mask).  Checked bit-exact against a reference pext on 10^7
+// random (x, m) pairs (tests/test_host_logic.py::test_compress_matches_pext mirrors it).
+__device__ __forceinline__ void hd_prep(uint32_t m, uint32_t (&mv)[5]) {
+  uint32_t mk = ~m << 1;
+#pragma unroll
+  for (int i = 0; i < 5; ++i) {
+    uint32_t mp = mk ^ (mk << 1);
+    mp ^= mp << 2;
+    mp ^= mp << 4;
+    mp ^= mp << 8;
+    mp ^= mp << 16;
+    const uint32_t v = mp & m;
+    mv[i] = v;
+    m = (m ^ v) | (v >> (1 << i));
+    mk &= ~mp;
+  }
+}
+__device__ __forceinline__ uint32_t hd_apply(uint32_t x, const uint32_t (&mv)[5]) {
+#pragma unroll
+  for (int i = 0; i < 5; ++i) {
+    const uint32_t t = x & mv[i];
+    x = (x ^ t) | (t >> (1 << i));
+  }
+  return x;
+}
+
+// One warp per item (pair p = (segment, class), group of <= kMemberGroup members): lane l walks
+// its mask words of the segment, and for every member appends pext(source word, mask word) to
+// the member's lane-l stream (a 32-bit accumulator + carry; whole words stored as they fill, the
+// last partial word at the end of the segment).  The bit count per step is the mask's, the same
+// for every member, so the fill level and output position are shared.
+__global__ void __launch_bounds__(kT) pext_kernel(Src src, const uint32_t* __restrict__ par_a,
+                                                  const uint32_t* __restrict__ par_b,
+                                                  const uint32_t* __restrict__ bound, uint32_t cmax, uint32_t nseg,
+                                                  uint32_t n_pairs, const uint32_t* __restrict__ item_off, uint32_t T,
+                                                  const uint32_t* __restrict__ loc, const uint64_t* __restrict__ off,
+                                                  uint32_t* __restrict__ data) {
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t it = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  if (it >= T) return;
+  uint32_t lo = 0, hi = n_pairs;  // pair p = last with item_off[p] <= it
+  while (lo + 1 < hi) {
+    const uint32_t mid = (lo + hi) >> 1;
+    if (item_off[mid] <= it) lo = mid; else hi = mid;
+  }
+  const uint32_t p = lo, c = p % cmax, s = p / cmax;
+  const uint32_t j0 = bound[c], m = bound[c + 1] - j0;
+  const uint32_t g = it - item_off[p];
+  const uint32_t first = j0 + g * kMemberGroup;
+  const uint32_t nm = min(kMemberGroup, m - g * kMemberGroup);
+  const VecRef mk = src.vec(par_a[j0]);
+  uint32_t ja, jb;
+  seg_range(mk.lw, nseg, s, ja, jb);
+  const uint32_t* S[kMemberGroup];
+  uint32_t* O[kMemberGroup];
+  uint32_t acc[kMemberGroup];
+#pragma unroll
+  for (uint32_t q = 0; q < kMemberGroup; ++q) {
+    const uint32_t e = first + (q < nm ? q : 0);
+    S[q] = src.vec(par_b[e]).p + lane;
+    O[q] = data + off[e] + lane;
+    acc[q] = 0;
+  }
+  uint32_t oj = loc[(uint64_t)p * 32 + lane];
+  uint32_t nb = 0;
+  for (uint32_t j = ja; j < jb; ++j) {
+    const uint32_t mw = mk.p[32ull * j + lane];
+    const uint32_t pc = __popc(mw);
+    uint32_t mv[5];
+    hd_prep(mw, mv);
+    const uint32_t nb2 = nb + pc;
+    uint32_t carry[kMemberGroup];
+#pragma unroll
+    for (uint32_t q = 0; q < kMemberGroup; ++q) {
+      carry[q] = 0;
+      if (q < nm) {
+        const uint32_t y = hd_apply(__ldg(S[q] + 32ull * j) & mw, mv);
+        const uint64_t v = (uint64_t)y << nb;
+        acc[q] |= (uint32_t)v;
+        carry[q] = (uint32_t)(v >> 32);
+      }
+    }
+    if (nb2 >= 32) {
+#pragma unroll
+      for (uint32_t q = 0; q < kMemberGroup; ++q)
+        if (q < nm) {
+          O[q][32ull * oj] = acc[q];
+          acc[q] = carry[q];
+        }
+      ++oj;
+      nb = nb2 - 32;
+    } else {
+      nb = nb2;
+    }
+  }
+  if (nb) {
+#pragma unroll
+    for (uint32_t q = 0; q < kMemberGroup; ++q)
+      if (q < nm) O[q][32ull * oj] = acc[q];
+  }
+}
+
+// ---------------------------------------------------------------- counting
+// CTA per group g (left parent x = gpar[g]); siblings in batches of 32 (lane j accumulates
+// sibling j); warps stride over 256-word chunks of the class vectors; one atomic per (warp,
+// sibling).  Two siblings share one packed redux.sync (per-warp sums <= 32 x 8 x 32 < 2^16).
+__global__ void __launch_bounds__(kT) count_proj_kernel(const uint32_t* __restrict__ data,
+                                                        const uint64_t* __restrict__ off,
+                                                        const uint32_t* __restrict__ nw,
+                                                        const uint32_t* __restrict__ gpar,
+                                                        const uint32_t* __restrict__ ext_off,
+                                                        const uint32_t* __restrict__ eidx,
+                                                        uint32_t* __restrict__ counts) {
+  const uint32_t g = blockIdx.x;
+  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const uint32_t x = gpar[g];
+  const uint32_t n = nw[x];
+  const uint32_t* X = data + off[x];
+  const uint32_t e0 = ext_off[g], e1 = ext_off[g + 1];
+  for (uint32_t b0 = e0; b0 < e1; b0 += 32) {
+    const uint32_t nb = min(32u, e1 - b0);
+    const uint64_t my_off = lane < nb ? off[eidx[b0 + lane]] : 0;
+    uint32_t acc = 0;
+    for (uint32_t w = warp * 256; w < n; w += (kT / 32) * 256) {
+      const uint32_t w0 = w + lane * 4, w1 = w + 128 + lane * 4;
+      const bool h0 = w0 < n, h1 = w1 < n;
+      const uint4 x0 = h0 ? *reinterpret_cast<const uint4*>(X + w0) : make_uint4(0, 0, 0, 0);
+      const uint4 x1 = h1 ? *reinterpret_cast<const uint4*>(X + w1) : make_uint4(0, 0, 0, 0);
+      for (uint32_t i = 0; i < nb; i += 2) {
+        uint32_t c = 0;
+#pragma unroll
+        for (uint32_t q = 0; q < 2; ++q) {
+          if (i + q < nb) {
+            const uint64_t yo = __shfl_sync(0xffffffffu, my_off, i + q);
+            const uint32_t* Y = data + yo;
+            const uint4 y0 = h0 ? *reinterpret_cast<const uint4*>(Y + w0) : make_uint4(0, 0, 0, 0);
+            const uint4 y1 = h1 ? *reinterpret_cast<const uint4*>(Y + w1) : make_uint4(0, 0, 0, 0);
+            const uint32_t v = __popc(x0.x & y0.x) + __popc(x0.y & y0.y) + __popc(x0.z & y0.z) +
+                               __popc(x0.w & y0.w) + __popc(x1.x & y1.x) + __popc(x1.y & y1.y) +
+                               __popc(x1.z & y1.z) + __popc(x1.w & y1.w);
+            c |= v << (16 * q);
+          }
+        }
+        c = __reduce_add_sync(0xffffffffu, c);
+        if (lane == i) acc += c & 0xffffu;
+        if (lane == i + 1) acc += c >> 16;
+      }
+    }
+    if (lane < nb && acc) atomicAdd(&counts[b0 + lane], acc);
+  }
+}
+
+template <class T>
+void scan_excl(const T* in, T* out, uint32_t n, DeviceScratch& scratch, cudaStream_t s) {
+  size_t bytes = 0;
+  GPA_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, bytes, in, out, n, s));
+  void* tmp = scratch.get(bytes, s);
+  GPA_CUDA(cub::DeviceScan::ExclusiveSum(tmp, bytes, in, out, n, s));
+  note_launch(2);
+}
+
+// totals: tot[0] = pext items, tot[1] = vector words
+__global__ void proj_totals_kernel(const uint32_t* __restrict__ items, const uint32_t* __restrict__ item_off,
+                                   uint32_t n_pairs, const uint64_t* __restrict__ cw, const uint64_t* __restrict__ cb,
+                                   uint32_t cmax, uint64_t* __restrict__ tot) {
+  if (threadIdx.x == 0 && blockIdx.x == 0) {
+    tot[0] = (uint64_t)item_off[n_pairs - 1] + items[n_pairs - 1];
+    tot[1] = cb[cmax - 1] + cw[cmax - 1];
+  }
+}
+
+// per-thread, per-device persistent workspace (grow-only): the class tables of proj_build and the
+// two generations of lists
+struct ProjWork {
+  PBuf<uint32_t> flag, ex, bound, small, words, loc, items, item_off, nwc;
+  PBuf<uint64_t> cls_words, cls_base, tot;
+  DeviceProj lists[2];
+};
+ProjWork& work_for(int device) {
+  thread_local std::map<int, ProjWork> w;
+  return w[device];
+}
+
+}  // namespace
+
+DeviceProj* proj_lists(int device) { return work_for(device).lists; }
+
+bool proj_build(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const DeviceProj* prev,
+                const uint32_t* rows, uint64_t pitch_words, uint32_t n_rows, DeviceProj& out, DeviceScratch& scratch,
+                int n_sms, cudaStream_t s) {
+  out.n = n;
+  out.words = 0;
+  if (n == 0) return true;
+  Src src{};
+  if (!prev) {
+    src.rows = rows;
+    src.pitch = pitch_words;
+  } else {
+    src.data = prev->data.p;
+    src.off = prev->off.p;
+    src.nw = prev->nw.p;
+  }
+  const uint32_t cmax = prev ? n : std::min(n, n_rows);
+  const uint32_t nseg = prev ? 1u : (uint32_t)((pitch_words / 32 + kSegJ - 1) / kSegJ);
+  const uint64_t n_pairs64 = (uint64_t)cmax * nseg;
+  GPA_REQUIRE(n_pairs64 * 32 < (1ull << 31), GPA_ERR_INVALID, "proj: too many classes");
+  const uint32_t n_pairs = (uint32_t)n_pairs64;
+
+  int device = 0;
+  GPA_CUDA(cudaGetDevice(&device));
+  ProjWork& W = work_for(device);
+  auto& flag = W.flag;
+  auto& ex = W.ex;
+  auto& bound = W.bound;
+  auto& small = W.small;
+  auto& words = W.words;
+  auto& loc = W.loc;
+  auto& items = W.items;
+  auto& item_off = W.item_off;
+  auto& nwc = W.nwc;
+  auto& cls_words = W.cls_words;
+  auto& cls_base = W.cls_base;
+  auto& tot = W.tot;
+  flag.ensure(n);
+  ex.ensure(n);
+  bound.ensure(n + 1);
+  small.ensure(4);
+  { cls_flag_kernel<<<grid_for(n, n_sms), kT, 0, s>>>(par_a, n, flag.p); note_launch(); }
+  scan_excl<uint32_t>(flag.p, ex.p, n, scratch, s);
+  { cls_bound_kernel<<<grid_for(n, n_sms), kT, 0, s>>>(flag.p, ex.p, n, bound.p, small.p); note_launch(); }
+  words.ensure((size_t)n_pairs * 32);
+  loc.ensure((size_t)n_pairs * 32);
+  items.ensure(n_pairs);
+  item_off.ensure(n_pairs);
+  nwc.ensure(cmax);
+  cls_words.ensure(cmax);
+  cls_base.ensure(cmax);
+  tot.ensure(2);
+  const unsigned warps_per_block = kT / 32;
+  { seg_popc_kernel<<<(n_pairs + warps_per_block - 1) / warps_per_block, kT, 0, s>>>(
+        src, par_a, bound.p, small.p, cmax, nseg, n_pairs, words.p); note_launch(); }
+  { cls_pad_kernel<<<(cmax + warps_per_block - 1) / warps_per_block, kT, 0, s>>>(
+        words.p, bound.p, small.p, cmax, nseg, loc.p, nwc.p, cls_words.p, items.p); note_launch(); }
+  scan_excl<uint32_t>(items.p, item_off.p, n_pairs, scratch, s);
+  scan_excl<uint64_t>(cls_words.p, cls_base.p, cmax, scratch, s);
+  { proj_totals_kernel<<<1, 32, 0, s>>>(items.p, item_off.p, n_pairs, cls_words.p, cls_base.p, cmax, tot.p);
+    note_launch(); }
+  GPA_CUDA(cudaGetLastError());
+  uint64_t T[2] = {0, 0};
+  GPA_CUDA(cudaMemcpyAsync(T, tot.p, sizeof(T), cudaMemcpyDeviceToHost, s));
+  const double h0 = wall_ms();
+  GPA_CUDA(cudaStreamSynchronize(s));
+  const double h1 = wall_ms();
+  if (T[0] >= (1ull << 31)) return false;
+  try {
+    out.data.ensure(T[1]);
+  } catch (const Error& e) {
+    if (e.status != GPA_ERR_OOM) throw;
+    return false;  // caller falls back to complete intersection
+  }
+  out.off.ensure(n);
+  out.nw.ensure(n);
+  out.words = T[1];
+  const double h2 = wall_ms();
+  // lanes shorter than their class' Lw keep a zero tail
+  GPA_CUDA(cudaMemsetAsync(out.data.p, 0, std::max<uint64_t>(T[1], 1) * 4, s));
+  { entry_off_kernel<<<grid_for(n, n_sms), kT, 0, s>>>(flag.p, ex.p, bound.p, nwc.p, cls_base.p, n, out.off.p,
+                                                      out.nw.p); note_launch(); }
+  if (T[0]) {
+    const uint64_t blocks = (T[0] + warps_per_block - 1) / warps_per_block;
+    { pext_kernel<<<(unsigned)blocks, kT, 0, s>>>(src, par_a, par_b, bound.p, cmax, nseg, n_pairs, item_off.p,
+                                                  (uint32_t)T[0], loc.p, out.off.p, out.data.p); note_launch(); }
+  }
+  GPA_CUDA(cudaGetLastError());
+  if (trace_enabled())
+    fprintf(stderr, "[gpa] proj_build n=%u: sync %.2f ms, alloc %.2f ms, launch %.2f ms\n", n, h1 - h0, h2 - h1,
+            wall_ms() - h2);
+  return true;
+}
+
+void launch_count_proj(const DeviceProj& P, const uint32_t* gpar, const uint32_t* ext_off, const uint32_t* eidx,
+                       uint32_t G, uint32_t* counts, cudaStream_t s) {
+  if (G == 0) return;
+  { count_proj_kernel<<<G, kT, 0, s>>>(P.data.p, P.off.p, P.nw.p, gpar, ext_off, eidx, counts); note_launch(); }
+  GPA_CUDA(cudaGetLastError());
+}
+
+}  // namespace gpa

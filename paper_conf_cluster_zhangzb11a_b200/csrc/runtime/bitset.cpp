@@ -58,7 +58,7 @@ float event_ms(cudaEvent_t a, cudaEvent_t b) {
 }
 
 void validate_options(const gpa_options& o) {
-  GPA_REQUIRE(o.count_kernel <= GPA_KERNEL_PAIRS_TC, GPA_ERR_INVALID, "unknown count_kernel %u", o.count_kernel);
+  GPA_REQUIRE(o.count_kernel <= GPA_KERNEL_PROJ, GPA_ERR_INVALID, "unknown count_kernel %u", o.count_kernel);
   GPA_REQUIRE(o.max_k <= GPA_MAX_K, GPA_ERR_INVALID, "max_k %u > GPA_MAX_K", o.max_k);
   GPA_REQUIRE(!o.reserved[0] && !o.reserved[1] && !o.reserved[2], GPA_ERR_INVALID, "reserved option fields must be 0");
   GPA_REQUIRE((o.flags & ~(GPA_KEEP_CANDIDATES | GPA_HOST_CANDGEN | GPA_NO_OVERLAP_INGEST)) == 0, GPA_ERR_INVALID, "unknown option flags 0x%x",
@@ -223,6 +223,8 @@ namespace {
 // start / end events of a counting launch: the caller's (deferred timing, no sync) or the bitset's
 cudaEvent_t ev_start(gpa_bitset* bs, CountStats* st) { return st && st->e0 ? st->e0 : bs->ev0; }
 
+}  // namespace
+
 void finish_counts(gpa_bitset* bs, size_t M, CountStats* st) {
   cudaStream_t s = bs->stream;
   const bool deferred = st && st->e0;
@@ -237,6 +239,8 @@ void finish_counts(gpa_bitset* bs, size_t M, CountStats* st) {
     st->allreduce_ms = bs->dist ? event_ms(bs->ev1, bs->ev2) : 0.0;
   }
 }
+
+namespace {
 
 void count_flat_v0(gpa_bitset* bs, const std::vector<uint32_t>& flat, uint32_t k, uint64_t M, CountStats* st) {
   cudaStream_t s = bs->stream;
@@ -301,6 +305,7 @@ bool count_device_batch(gpa_bitset* bs, DeviceBatch& B, uint32_t kernel, DeviceS
   cudaStream_t s = bs->stream;
   const uint32_t k = B.k, M = B.M, G = B.G;
   if (M == 0) return true;
+  if (kernel == GPA_KERNEL_PROJ) kernel = GPA_KERNEL_AUTO;
   if (kernel == GPA_KERNEL_V0 || bs->n_rows > kPlanMaxRows || k < 2) return false;
   if (kernel == GPA_KERNEL_AUTO || kernel == GPA_KERNEL_PAIRS || kernel == GPA_KERNEL_PAIRS_TC) {
     const double sib = (double)M / (double)std::max<uint32_t>(G, 1);
@@ -389,6 +394,7 @@ void count_grouped(gpa_bitset* bs, const GroupedBatch& b, uint32_t kernel, Count
   const uint64_t M = b.size(), G = b.groups();
   const uint32_t km1 = b.k - 1;
   if (M == 0) return;
+  if (kernel == GPA_KERNEL_PROJ) kernel = GPA_KERNEL_AUTO;
   if (kernel == GPA_KERNEL_AUTO || kernel == GPA_KERNEL_PAIRS || kernel == GPA_KERNEL_PAIRS_TC) {
     // grouped batches: large sibling groups amortise the (k-1)-row prefix well in the streaming
     // prefix kernel (measured: T40I10D10M k = 3, 4.6 siblings / group); small groups (deep
@@ -449,7 +455,7 @@ void count_all_pairs(gpa_bitset* bs, uint32_t kernel, CountStats* st) {
   const uint64_t n = bs->n_rows;
   const uint64_t M = n * (n - 1) / 2;
   if (n < 2) return;
-  if (kernel == GPA_KERNEL_AUTO) kernel = GPA_KERNEL_PAIRS_TC;
+  if (kernel == GPA_KERNEL_AUTO || kernel == GPA_KERNEL_PROJ) kernel = GPA_KERNEL_PAIRS_TC;
   if (kernel != GPA_KERNEL_PAIRS && kernel != GPA_KERNEL_PAIRS_TC) {
     GroupedBatch b;
     b.k = 2;
@@ -548,7 +554,7 @@ extern "C" gpa_status gpa_count(gpa_bitset* bs, const uint32_t* cand, uint32_t k
   return gpa::guard([&] {
     GPA_REQUIRE(bs, GPA_ERR_INVALID, "bitset is NULL");
     GPA_REQUIRE(k >= 1 && k <= GPA_MAX_K, GPA_ERR_INVALID, "k must be in [1, %u]", GPA_MAX_K);
-    GPA_REQUIRE(kernel <= GPA_KERNEL_PAIRS_TC, GPA_ERR_INVALID, "unknown kernel %u", kernel);
+    GPA_REQUIRE(kernel <= GPA_KERNEL_PROJ, GPA_ERR_INVALID, "unknown kernel %u", kernel);
     if (M == 0) return;
     GPA_REQUIRE(cand && counts_out, GPA_ERR_INVALID, "NULL argument");
     GPA_REQUIRE(M <= (UINT64_MAX / 8) / k && M < (1ull << 32), GPA_ERR_INVALID, "M * k overflows");
@@ -568,6 +574,7 @@ extern "C" gpa_status gpa_count(gpa_bitset* bs, const uint32_t* cand, uint32_t k
       }
     }
     uint32_t kern = kernel == GPA_KERNEL_AUTO ? bs->opt.count_kernel : kernel;
+    if (kern == GPA_KERNEL_PROJ) kern = GPA_KERNEL_AUTO;  // needs the level structure of gpa_mine
     if (k == 1) kern = GPA_KERNEL_V0;
     if (kern == GPA_KERNEL_AUTO)
       kern = (k == 2 && (double)M * 8 >= (double)bs->n_rows * bs->n_rows) ? GPA_KERNEL_PAIRS_TC

@@ -146,6 +146,9 @@ void count_grouped(gpa_bitset* bs, const GroupedBatch& b, uint32_t kernel, Count
 // Count a device-resident grouped batch with device-side planning (trie blocks / prefix tasks);
 // returns false when it cannot (kernel v0, too many rows) and the host path must be used.
 bool count_device_batch(gpa_bitset* bs, DeviceBatch& B, uint32_t kernel, DeviceScratch& scratch, CountStats* st);
+// After a counting launch: end event, all-reduce of the M counts (dist), and the timing (no sync
+// when st carries caller-owned events).
+void finish_counts(gpa_bitset* bs, size_t M, CountStats* st);
 // Count all pairs of rows (lexicographic pair order) into bs->d_counts (n(n-1)/2 entries).
 void count_all_pairs(gpa_bitset* bs, uint32_t kernel, CountStats* st);
 }  // namespace gpa

@@ -83,6 +83,29 @@ void record_level(gpa_result* R, const gpa_bitset* bs, uint32_t k, const Grouped
   R->levels.push_back(std::move(lv));
 }
 
+// Generation k >= 3 on projected vertical lists (proj.cu): the lists of L_{k-1}'s entries from
+// those of L_{k-2} (prev; the bitset rows for k = 3), then one popcount-of-AND per candidate over
+// its parents' lists.  false: the lists do not fit -- nothing counted, use complete intersection.
+bool count_projected(gpa_bitset* bs, uint32_t k, const DeviceLevel& L, const DeviceBatch& B, DeviceProj& prev,
+                     DeviceProj& cur, DeviceScratch& scratch, CountStats* cs) {
+  cudaStream_t s = bs->stream;
+  const double t0 = now_ms();
+  GPA_CUDA(cudaEventRecord(cs->e0, s));
+  if (!proj_build(L.n, L.par_a.p, L.par_b.p, k == 3 ? nullptr : &prev, bs->rows.p, bs->pitch_words, bs->n_rows, cur,
+                  scratch, bs->n_sms, s))
+    return false;
+  bs->d_counts.ensure(B.M, s);
+  GPA_CUDA(cudaMemsetAsync(bs->d_counts.p, 0, (size_t)B.M * 4, s));
+  launch_count_proj(cur, B.gpar.p, B.ext_off.p, B.eidx.p, B.G, bs->d_counts.p, s);
+  cs->kernel = GPA_KERNEL_PROJ;
+  cs->launches = 1;
+  finish_counts(bs, B.M, cs);
+  if (trace_enabled())
+    fprintf(stderr, "[gpa] k=%u proj: %u lists, %.1f MB, host %.2f ms\n", k, L.n, cur.words * 4.0 / 1e6,
+            now_ms() - t0);
+  return true;
+}
+
 }  // namespace
 
 gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist, const gpa_options* opt_in) {
@@ -147,6 +170,14 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
   DeviceLevel Ld, Ln;   // L_{k-1}, L_k on the device
   DeviceBatch Bd;       // C_k on the device (k >= 3)
   DBuf<uint32_t> d_ior;  // row -> original item id
+  // projected vertical lists (GPA_KERNEL_PROJ / AUTO): Pprev = the lists of L_{k-2}'s entries,
+  // Pcur = those of L_{k-1} built for generation k (proj.cu)
+  DeviceProj* plists = proj_lists(bs->device);
+  DeviceProj* Pprev = &plists[0];
+  DeviceProj* Pcur = &plists[1];
+  bool proj_on = !host_candgen && (opt.count_kernel == GPA_KERNEL_AUTO || opt.count_kernel == GPA_KERNEL_PROJ ||
+                                   opt.count_kernel == GPA_KERNEL_PAIRS || opt.count_kernel == GPA_KERNEL_PAIRS_TC) &&
+                 bs->pitch_words * 32ull < (1ull << 32);
   struct Pending {       // a generation's frequent itemsets, still on the device
     size_t level = 0;
     uint32_t F = 0, k = 0;
@@ -237,7 +268,9 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
       events.pop_back();
     } else if (k == 2) {
       count_all_pairs(bs, opt.count_kernel, &cs);
-    } else if (!count_device_batch(bs, Bd, opt.count_kernel, scratch, &cs)) {
+    } else if (proj_on && count_projected(bs, k, Ld, Bd, *Pprev, *Pcur, scratch, &cs)) {
+      std::swap(Pprev, Pcur);
+    } else if ((proj_on = false, !count_device_batch(bs, Bd, opt.count_kernel, scratch, &cs))) {
       fetch_batch();
       count_grouped(bs, batch, opt.count_kernel, &cs);
     }
@@ -246,7 +279,8 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     R->phase_ms[GPA_PHASE_COUNT] += t2 - t1;
 
     const uint32_t F = device_threshold(bs->d_counts.p, (uint32_t)M, (uint32_t)min_count, k, bs->n_rows, Bd.prefix.p,
-                                        Bd.ext_off.p, Bd.ext.p, (uint32_t)G, Ln, scratch, bs->n_sms, s);
+                                        Bd.ext_off.p, Bd.ext.p, (uint32_t)G, host_candgen ? nullptr : Bd.gpar.p,
+                                        host_candgen ? nullptr : Bd.eidx.p, Ln, scratch, bs->n_sms, s);
     // the frequent itemsets of this generation (item ids) and supports stay on the device until the
     // end of the loop: one transfer for all generations instead of one synchronisation each
     Pending pd;

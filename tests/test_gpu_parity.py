@@ -188,7 +188,7 @@ def test_mine_random(seed):
                        duplicates=seed % 2 == 1, unsorted=seed % 3 == 0)
     theta = int(rng.integers(1, max(2, ds.n_tx // 8)))
     ref = oracle.mine_ds(ds, theta)
-    for kern in (gpa.KERNEL_AUTO, gpa.KERNEL_V0, gpa.KERNEL_PREFIX, gpa.KERNEL_TRIE):
+    for kern in (gpa.KERNEL_AUTO, gpa.KERNEL_V0, gpa.KERNEL_PREFIX, gpa.KERNEL_TRIE, gpa.KERNEL_PROJ):
         for host in (False, True):
             res = gpa.mine(ds, min_count=theta, options=gpa.Options(count_kernel=kern, host_candgen=host),
                            keep_candidates=True)
@@ -202,9 +202,9 @@ def test_mine_configs(name):
     theta = oracle.min_count(ds.n_tx, gen.CONFIGS[name].minsup)
     assert gpa.min_count(ds.n_tx, gen.CONFIGS[name].minsup) == theta
     ref = oracle.mine_ds(ds, theta)
-    kernels = [gpa.KERNEL_AUTO, gpa.KERNEL_PAIRS, gpa.KERNEL_PREFIX, gpa.KERNEL_TRIE] + (
+    kernels = [gpa.KERNEL_AUTO, gpa.KERNEL_PAIRS, gpa.KERNEL_PREFIX, gpa.KERNEL_TRIE, gpa.KERNEL_PROJ] + (
         [gpa.KERNEL_V0] if name in ("chess", "mushroom") else [])
-    # AUTO = pairs (k = 2) + trie / prefix (k >= 3); device-side candidate generation by default,
+    # AUTO = pairs (k = 2) + projected lists (k >= 3); device-side candidate generation by default,
     # the host thread-pool join + prune as the reference path
     for kern in kernels:
         res = gpa.mine(ds, min_count=theta, options=gpa.Options(count_kernel=kern), keep_candidates=True)
