@@ -147,6 +147,7 @@ struct DeviceProj {
   PBuf<uint32_t> nw;      // n: words of entry j's vector (multiple of 32; 0 = none)
   PBuf<uint32_t> data;
   uint64_t words = 0;
+  uint32_t max_lw = 0;    // longest lane stream (words) of any class
 };
 // The calling thread's two DeviceProj for `device` (previous / current generation).
 DeviceProj* proj_lists(int device);

@@ -29,8 +29,8 @@
 // touches lane l: every load is a coalesced 128-byte row, no cross-lane bit placement.  The
 // members of a class share one mask, hence one per-lane bit count and one layout: Lw_c = max
 // over lanes of the lane's words (each lane's tail zero-padded), members contiguous.  A bitset
-// row is cut into segments of kSegJ words per lane, each lane padded to whole words per segment,
-// so segments are independent work items.  All integer; counts are exact by construction.
+// mask is cut into segments of kSegJ words per lane, each lane padded to whole words per
+// segment, so segments are independent work items.  All integer; counts are exact by construction.
 #include <cstdint>
 #include <map>
 #include <cub/block/block_scan.cuh>
@@ -43,8 +43,9 @@ namespace gpa {
 namespace {
 
 constexpr int kT = 256;
-constexpr uint32_t kSegJ = 256;          // segment of a bitset row: 256 words per lane (262,144 transactions)
+constexpr uint32_t kSegJ = 128;          // mask segment: 128 words per lane (a bitset row: 131,072 transactions)
 constexpr uint32_t kMemberGroup = 8;     // members sharing one mask preparation in pext_kernel
+constexpr uint32_t kItemsPerWarp = 4;    // pext items per warp (one binary search per run)
 
 unsigned grid_for(uint64_t n, int n_sms, int per_sm = 16) {
   uint64_t g = (n + kT - 1) / kT;
@@ -90,10 +91,9 @@ struct Src {
   }
 };
 
-__device__ __forceinline__ void seg_range(uint32_t lw, uint32_t nseg, uint32_t s, uint32_t& j0, uint32_t& j1) {
-  const uint32_t seg = nseg == 1 ? lw : kSegJ;
-  j0 = s * seg;
-  j1 = min(lw, j0 + seg);
+__device__ __forceinline__ void seg_range(uint32_t lw, uint32_t s, uint32_t& j0, uint32_t& j1) {
+  j0 = min(lw, s * kSegJ);
+  j1 = min(lw, j0 + kSegJ);
 }
 
 // warp per (segment s, class c) pair p = s * cmax + c: lane l's mask popcount in the segment ->
@@ -111,7 +111,7 @@ __global__ void seg_popc_kernel(Src src, const uint32_t* __restrict__ par_a, con
     if (m >= 2) {
       const VecRef mk = src.vec(par_a[j0]);
       uint32_t a, b;
-      seg_range(mk.lw, nseg, s, a, b);
+      seg_range(mk.lw, s, a, b);
       for (uint32_t j = a; j < b; ++j) cnt += __popc(mk.p[32ull * j + lane]);
     }
   }
@@ -124,7 +124,8 @@ __global__ void seg_popc_kernel(Src src, const uint32_t* __restrict__ par_a, con
 __global__ void cls_pad_kernel(const uint32_t* __restrict__ words, const uint32_t* __restrict__ bound,
                                const uint32_t* __restrict__ n_cls, uint32_t cmax, uint32_t nseg,
                                uint32_t* __restrict__ loc, uint32_t* __restrict__ nwc,
-                               uint64_t* __restrict__ cls_words, uint32_t* __restrict__ items) {
+                               uint64_t* __restrict__ cls_words, uint32_t* __restrict__ items,
+                               uint32_t* __restrict__ max_lw) {
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   if (c >= cmax) return;
@@ -135,13 +136,16 @@ __global__ void cls_pad_kernel(const uint32_t* __restrict__ words, const uint32_
   for (uint32_t s = 0; s < nseg; ++s) {
     const uint64_t p = (uint64_t)s * cmax + c;
     loc[p * 32 + lane] = acc;
-    acc += words[p * 32 + lane];
-    if (lane == 0) items[p] = groups;
+    const uint32_t w = words[p * 32 + lane];
+    acc += w;
+    const bool any = __any_sync(0xffffffffu, w != 0);
+    if (lane == 0) items[p] = any ? groups : 0;
   }
   const uint32_t lw = __reduce_max_sync(0xffffffffu, acc);
   if (lane == 0) {
     nwc[c] = groups ? 32u * lw : 0u;
     cls_words[c] = groups ? (uint64_t)32u * lw * m : 0ull;
+    if (groups && lw) atomicMax(max_lw, lw);
   }
 }
 
@@ -164,105 +168,151 @@ __global__ void entry_off_kernel(const uint32_t* __restrict__ flag, const uint32
 }
 
 // Hacker's Delight 7-4 "compress" (= pext): the mask-dependent shift masks, then the per-source
-// part (x already ANDed with the mask).  Checked bit-exact against a reference pext on 10^7
-// random (x, m) pairs (tests/test_host_logic.py::test_compress_matches_pext mirrors it).
+// part.  Right shifts by a constant are written as __umulhi(x, 2^(32-s)) and left shifts as
+// multiplies so that they issue on the FMA pipe next to the LOP3s on the ALU pipe (the kernel is
+// ALU-bound).  Checked bit-exact against a plain bit-by-bit pext (tests/test_host_logic.py
+// ::test_compress_matches_pext runs the same sequence of operations on the host).
+__device__ __forceinline__ uint32_t shr_c(uint32_t x, int s) { return __umulhi(x, 1u << (32 - s)); }
+__device__ __forceinline__ uint32_t shl_c(uint32_t x, int s) { return x * (1u << s); }
+
 __device__ __forceinline__ void hd_prep(uint32_t m, uint32_t (&mv)[5]) {
-  uint32_t mk = ~m << 1;
+  uint32_t mk = shl_c(~m, 1);
 #pragma unroll
   for (int i = 0; i < 5; ++i) {
-    uint32_t mp = mk ^ (mk << 1);
-    mp ^= mp << 2;
-    mp ^= mp << 4;
-    mp ^= mp << 8;
-    mp ^= mp << 16;
+    uint32_t mp = mk ^ shl_c(mk, 1);
+    mp ^= shl_c(mp, 2);
+    mp ^= shl_c(mp, 4);
+    mp ^= shl_c(mp, 8);
+    mp ^= shl_c(mp, 16);
     const uint32_t v = mp & m;
     mv[i] = v;
-    m = (m ^ v) | (v >> (1 << i));
+    m = (m ^ v) | shr_c(v, 1 << i);
     mk &= ~mp;
   }
 }
-__device__ __forceinline__ uint32_t hd_apply(uint32_t x, const uint32_t (&mv)[5]) {
+// pext(x, m) given m's shift masks (x need not be pre-masked: stage 0 folds the AND with m)
+__device__ __forceinline__ uint32_t hd_apply(uint32_t x, uint32_t m, const uint32_t (&mv)[5]) {
+  uint32_t t = x & mv[0];
+  x = (x & m & ~mv[0]) | shr_c(t, 1);
 #pragma unroll
-  for (int i = 0; i < 5; ++i) {
-    const uint32_t t = x & mv[i];
-    x = (x ^ t) | (t >> (1 << i));
+  for (int i = 1; i < 5; ++i) {
+    t = x & mv[i];
+    x = (x & ~mv[i]) | shr_c(t, 1 << i);
   }
   return x;
 }
 
-// One warp per item (pair p = (segment, class), group of <= kMemberGroup members): lane l walks
-// its mask words of the segment, and for every member appends pext(source word, mask word) to
-// the member's lane-l stream (a 32-bit accumulator + carry; whole words stored as they fill, the
-// last partial word at the end of the segment).  The bit count per step is the mask's, the same
-// for every member, so the fill level and output position are shared.
-__global__ void __launch_bounds__(kT) pext_kernel(Src src, const uint32_t* __restrict__ par_a,
-                                                  const uint32_t* __restrict__ par_b,
-                                                  const uint32_t* __restrict__ bound, uint32_t cmax, uint32_t nseg,
-                                                  uint32_t n_pairs, const uint32_t* __restrict__ item_off, uint32_t T,
-                                                  const uint32_t* __restrict__ loc, const uint64_t* __restrict__ off,
-                                                  uint32_t* __restrict__ data) {
-  const uint32_t lane = threadIdx.x & 31;
-  const uint32_t it = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  if (it >= T) return;
-  uint32_t lo = 0, hi = n_pairs;  // pair p = last with item_off[p] <= it
-  while (lo + 1 < hi) {
-    const uint32_t mid = (lo + hi) >> 1;
-    if (item_off[mid] <= it) lo = mid; else hi = mid;
-  }
-  const uint32_t p = lo, c = p % cmax, s = p / cmax;
-  const uint32_t j0 = bound[c], m = bound[c + 1] - j0;
-  const uint32_t g = it - item_off[p];
-  const uint32_t first = j0 + g * kMemberGroup;
-  const uint32_t nm = min(kMemberGroup, m - g * kMemberGroup);
-  const VecRef mk = src.vec(par_a[j0]);
-  uint32_t ja, jb;
-  seg_range(mk.lw, nseg, s, ja, jb);
-  const uint32_t* S[kMemberGroup];
-  uint32_t* O[kMemberGroup];
-  uint32_t acc[kMemberGroup];
-#pragma unroll
-  for (uint32_t q = 0; q < kMemberGroup; ++q) {
-    const uint32_t e = first + (q < nm ? q : 0);
-    S[q] = src.vec(par_b[e]).p + lane;
-    O[q] = data + off[e] + lane;
-    acc[q] = 0;
-  }
-  uint32_t oj = loc[(uint64_t)p * 32 + lane];
+// One item of pext_kernel for a group of nm <= G members (G = 2, 4, 8: the unrolled width, so a
+// class of 2 members does not pay for 8): lane l walks its mask words [ja, jb) and appends, for
+// every member, pext(source word, mask word) to the member's lane-l stream -- a 32-bit
+// accumulator, whole words stored as they fill, the last partial word at the segment's end.
+// The bit count per step is the mask's, the same for every member, so the fill level and the
+// output position are shared; the append is one 32x32->64 multiply by 2^fill.  The next step's
+// mask and source words are loaded one step ahead.
+template <uint32_t G>
+__device__ __forceinline__ void pext_item(const uint32_t* __restrict__ mp, const uint32_t* __restrict__ sbase,
+                                          const uint32_t (&so)[kMemberGroup], const uint32_t (&oo)[kMemberGroup],
+                                          uint32_t nm, uint32_t ja, uint32_t jb, uint32_t oj,
+                                          uint32_t* __restrict__ data) {
+  uint32_t acc[G], xn[G];
   uint32_t nb = 0;
+  uint32_t mn = __ldg(mp + 32u * ja);
+#pragma unroll
+  for (uint32_t q = 0; q < G; ++q) {
+    acc[q] = 0;
+    xn[q] = __ldg(sbase + (so[q] + 32u * ja));
+  }
   for (uint32_t j = ja; j < jb; ++j) {
-    const uint32_t mw = mk.p[32ull * j + lane];
-    const uint32_t pc = __popc(mw);
+    const uint32_t mw = mn;
+    uint32_t x[G];
+#pragma unroll
+    for (uint32_t q = 0; q < G; ++q) x[q] = xn[q];
+    const uint32_t jn = min(j + 1, jb - 1);
+    mn = __ldg(mp + 32u * jn);
+#pragma unroll
+    for (uint32_t q = 0; q < G; ++q) xn[q] = __ldg(sbase + (so[q] + 32u * jn));
     uint32_t mv[5];
     hd_prep(mw, mv);
-    const uint32_t nb2 = nb + pc;
-    uint32_t carry[kMemberGroup];
+    const uint32_t pw = 1u << nb;
+    nb += __popc(mw);
+    uint32_t carry[G];
 #pragma unroll
-    for (uint32_t q = 0; q < kMemberGroup; ++q) {
-      carry[q] = 0;
-      if (q < nm) {
-        const uint32_t y = hd_apply(__ldg(S[q] + 32ull * j) & mw, mv);
-        const uint64_t v = (uint64_t)y << nb;
-        acc[q] |= (uint32_t)v;
-        carry[q] = (uint32_t)(v >> 32);
-      }
+    for (uint32_t q = 0; q < G; ++q) {
+      const uint64_t v = (uint64_t)hd_apply(x[q], mw, mv) * pw;
+      acc[q] |= (uint32_t)v;
+      carry[q] = (uint32_t)(v >> 32);
     }
-    if (nb2 >= 32) {
+    if (nb >= 32) {
 #pragma unroll
-      for (uint32_t q = 0; q < kMemberGroup; ++q)
-        if (q < nm) {
-          O[q][32ull * oj] = acc[q];
-          acc[q] = carry[q];
-        }
+      for (uint32_t q = 0; q < G; ++q) {
+        if (q < nm) data[oo[q] + 32u * oj] = acc[q];
+        acc[q] = carry[q];
+      }
       ++oj;
-      nb = nb2 - 32;
-    } else {
-      nb = nb2;
+      nb -= 32;
     }
   }
   if (nb) {
 #pragma unroll
-    for (uint32_t q = 0; q < kMemberGroup; ++q)
-      if (q < nm) O[q][32ull * oj] = acc[q];
+    for (uint32_t q = 0; q < G; ++q)
+      if (q < nm) data[oo[q] + 32u * oj] = acc[q];
+  }
+}
+
+// Warp per run of kItemsPerWarp consecutive items; an item = (pair p = (segment, class), group of
+// <= kMemberGroup members -- the class' members split evenly over its groups).
+__global__ void __launch_bounds__(kT, 4) pext_kernel(Src src, const uint32_t* __restrict__ par_a,
+                                                     const uint32_t* __restrict__ par_b,
+                                                     const uint32_t* __restrict__ bound, uint32_t cmax,
+                                                     uint32_t n_pairs, const uint32_t* __restrict__ item_off,
+                                                     uint32_t T, const uint32_t* __restrict__ loc,
+                                                     const uint64_t* __restrict__ off, uint32_t* __restrict__ data) {
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t it0 = ((blockIdx.x * blockDim.x + threadIdx.x) >> 5) * kItemsPerWarp;
+  if (it0 >= T) return;
+  uint32_t p = 0;
+  {
+    uint32_t hi = n_pairs;  // pair = last with item_off[p] <= it0
+    while (p + 1 < hi) {
+      const uint32_t mid = (p + hi) >> 1;
+      if (item_off[mid] <= it0) p = mid; else hi = mid;
+    }
+  }
+  const uint32_t* base = src.rows ? src.rows : src.data;
+  for (uint32_t it = it0; it < min(T, it0 + kItemsPerWarp); ++it) {
+    if (p + 1 < n_pairs && item_off[p + 1] <= it) {  // next pair holding items: search [p + 1, n_pairs)
+      uint32_t hi = n_pairs;
+      ++p;
+      while (p + 1 < hi) {
+        const uint32_t mid = (p + hi) >> 1;
+        if (item_off[mid] <= it) p = mid; else hi = mid;
+      }
+    }
+    const uint32_t c = p % cmax, s = p / cmax;
+    const uint32_t j0 = bound[c], m = bound[c + 1] - j0;
+    const uint32_t groups = (m + kMemberGroup - 1) / kMemberGroup;
+    const uint32_t g = it - item_off[p];
+    const uint32_t first = j0 + (uint32_t)((uint64_t)m * g / groups);
+    const uint32_t nm = j0 + (uint32_t)((uint64_t)m * (g + 1) / groups) - first;
+    const VecRef mk = src.vec(par_a[j0]);
+    uint32_t ja, jb;
+    seg_range(mk.lw, s, ja, jb);
+    if (ja >= jb) continue;
+    uint32_t so[kMemberGroup], oo[kMemberGroup];
+#pragma unroll
+    for (uint32_t q = 0; q < kMemberGroup; ++q) {
+      const uint32_t e = first + (q < nm ? q : 0);  // surplus slots shadow member 0 (not stored)
+      so[q] = (uint32_t)(src.vec(par_b[e]).p - base);
+      oo[q] = (uint32_t)off[e] + lane;
+    }
+    const uint32_t oj = loc[(uint64_t)p * 32 + lane];
+    const uint32_t* mp = mk.p + lane;
+    if (nm <= 2)
+      pext_item<2>(mp, base + lane, so, oo, nm, ja, jb, oj, data);
+    else if (nm <= 4)
+      pext_item<4>(mp, base + lane, so, oo, nm, ja, jb, oj, data);
+    else
+      pext_item<8>(mp, base + lane, so, oo, nm, ja, jb, oj, data);
   }
 }
 
@@ -367,7 +417,10 @@ bool proj_build(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const 
     src.nw = prev->nw.p;
   }
   const uint32_t cmax = prev ? n : std::min(n, n_rows);
-  const uint32_t nseg = prev ? 1u : (uint32_t)((pitch_words / 32 + kSegJ - 1) / kSegJ);
+  const uint64_t lw_max = prev ? prev->max_lw : pitch_words / 32;
+  const uint32_t nseg = (uint32_t)std::max<uint64_t>(1, (lw_max + kSegJ - 1) / kSegJ);
+  // 32-bit word offsets inside pext_kernel
+  GPA_REQUIRE(prev || (uint64_t)n_rows * pitch_words < (1ull << 32), GPA_ERR_INVALID, "proj: bitset too large");
   const uint64_t n_pairs64 = (uint64_t)cmax * nseg;
   GPA_REQUIRE(n_pairs64 * 32 < (1ull << 31), GPA_ERR_INVALID, "proj: too many classes");
   const uint32_t n_pairs = (uint32_t)n_pairs64;
@@ -391,6 +444,7 @@ bool proj_build(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const 
   ex.ensure(n);
   bound.ensure(n + 1);
   small.ensure(4);
+  GPA_CUDA(cudaMemsetAsync(small.p, 0, 16, s));
   { cls_flag_kernel<<<grid_for(n, n_sms), kT, 0, s>>>(par_a, n, flag.p); note_launch(); }
   scan_excl<uint32_t>(flag.p, ex.p, n, scratch, s);
   { cls_bound_kernel<<<grid_for(n, n_sms), kT, 0, s>>>(flag.p, ex.p, n, bound.p, small.p); note_launch(); }
@@ -406,18 +460,20 @@ bool proj_build(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const 
   { seg_popc_kernel<<<(n_pairs + warps_per_block - 1) / warps_per_block, kT, 0, s>>>(
         src, par_a, bound.p, small.p, cmax, nseg, n_pairs, words.p); note_launch(); }
   { cls_pad_kernel<<<(cmax + warps_per_block - 1) / warps_per_block, kT, 0, s>>>(
-        words.p, bound.p, small.p, cmax, nseg, loc.p, nwc.p, cls_words.p, items.p); note_launch(); }
+        words.p, bound.p, small.p, cmax, nseg, loc.p, nwc.p, cls_words.p, items.p, small.p + 1); note_launch(); }
   scan_excl<uint32_t>(items.p, item_off.p, n_pairs, scratch, s);
   scan_excl<uint64_t>(cls_words.p, cls_base.p, cmax, scratch, s);
   { proj_totals_kernel<<<1, 32, 0, s>>>(items.p, item_off.p, n_pairs, cls_words.p, cls_base.p, cmax, tot.p);
     note_launch(); }
   GPA_CUDA(cudaGetLastError());
   uint64_t T[2] = {0, 0};
+  uint32_t mlw = 0;
   GPA_CUDA(cudaMemcpyAsync(T, tot.p, sizeof(T), cudaMemcpyDeviceToHost, s));
+  GPA_CUDA(cudaMemcpyAsync(&mlw, small.p + 1, 4, cudaMemcpyDeviceToHost, s));
   const double h0 = wall_ms();
   GPA_CUDA(cudaStreamSynchronize(s));
   const double h1 = wall_ms();
-  if (T[0] >= (1ull << 31)) return false;
+  if (T[0] >= (1ull << 31) || T[1] >= (1ull << 32)) return false;
   try {
     out.data.ensure(T[1]);
   } catch (const Error& e) {
@@ -427,14 +483,16 @@ bool proj_build(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const 
   out.off.ensure(n);
   out.nw.ensure(n);
   out.words = T[1];
+  out.max_lw = mlw;
   const double h2 = wall_ms();
   // lanes shorter than their class' Lw keep a zero tail
   GPA_CUDA(cudaMemsetAsync(out.data.p, 0, std::max<uint64_t>(T[1], 1) * 4, s));
   { entry_off_kernel<<<grid_for(n, n_sms), kT, 0, s>>>(flag.p, ex.p, bound.p, nwc.p, cls_base.p, n, out.off.p,
                                                       out.nw.p); note_launch(); }
   if (T[0]) {
-    const uint64_t blocks = (T[0] + warps_per_block - 1) / warps_per_block;
-    { pext_kernel<<<(unsigned)blocks, kT, 0, s>>>(src, par_a, par_b, bound.p, cmax, nseg, n_pairs, item_off.p,
+    const uint64_t warps = (T[0] + kItemsPerWarp - 1) / kItemsPerWarp;
+    const uint64_t blocks = (warps + warps_per_block - 1) / warps_per_block;
+    { pext_kernel<<<(unsigned)blocks, kT, 0, s>>>(src, par_a, par_b, bound.p, cmax, n_pairs, item_off.p,
                                                   (uint32_t)T[0], loc.p, out.off.p, out.data.p); note_launch(); }
   }
   GPA_CUDA(cudaGetLastError());

@@ -159,3 +159,62 @@ def test_trie_plan_invariants(shim, name, k):
                 assert lcp[c] == l
         pos += nc
     assert pos == M
+
+
+# ---------------------------------------------------------------- projected lists (proj.cu)
+
+def _hd_compress(x, m):
+    """The operation sequence of proj.cu's hd_prep / hd_apply (Hacker's Delight 7-4 compress,
+    right shifts as umulhi by 2^(32-s), left shifts as multiplies), vectorised over uint32."""
+    M32 = np.uint64(0xFFFFFFFF)
+    x = x.astype(np.uint64)
+    m = m.astype(np.uint64)
+
+    def shl(v, s):
+        return (v * np.uint64(1 << s)) & M32
+
+    def shr(v, s):
+        return (v * np.uint64(1 << (32 - s))) >> np.uint64(32)
+
+    mk = shl(~m & M32, 1)
+    mv = []
+    mm = m.copy()
+    for i in range(5):
+        mp = mk ^ shl(mk, 1)
+        for sh in (2, 4, 8, 16):
+            mp ^= shl(mp, sh)
+        v = mp & mm
+        mv.append(v)
+        mm = (mm ^ v) | shr(v, 1 << i)
+        mk &= ~mp & M32
+    t = x & mv[0]
+    y = (x & m & (~mv[0] & M32)) | shr(t, 1)
+    for i in range(1, 5):
+        t = y & mv[i]
+        y = (y & (~mv[i] & M32)) | shr(t, 1 << i)
+    return y.astype(np.uint32)
+
+
+def _pext_ref(x, m):
+    out = np.zeros_like(x)
+    k = np.zeros_like(x)
+    for i in range(32):
+        sel = (m >> np.uint32(i)) & np.uint32(1)
+        bit = (x >> np.uint32(i)) & np.uint32(1)
+        out |= (bit & sel) << k
+        k += sel
+    return out
+
+
+def test_compress_matches_pext():
+    """proj.cu's parallel bit extract equals the bit-by-bit definition (random, sparse, dense,
+    empty and full masks)."""
+    rng = np.random.default_rng(11)
+    n = 200_000
+    x = rng.integers(0, 2 ** 32, n, dtype=np.uint64).astype(np.uint32)
+    m = rng.integers(0, 2 ** 32, n, dtype=np.uint64).astype(np.uint32)
+    m[::3] &= rng.integers(0, 2 ** 32, len(m[::3]), dtype=np.uint64).astype(np.uint32)   # sparse
+    m[1::7] = 0xFFFFFFFF
+    m[2::11] = 0
+    m[3::13] = 0x80000001
+    assert np.array_equal(_hd_compress(x, m), _pext_ref(x, m))
