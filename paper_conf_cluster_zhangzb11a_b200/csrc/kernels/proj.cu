@@ -45,7 +45,6 @@ namespace {
 constexpr int kT = 256;
 constexpr uint32_t kSegJ = 128;          // mask segment: 128 words per lane (a bitset row: 131,072 transactions)
 constexpr uint32_t kMemberGroup = 8;     // members sharing one mask preparation in pext_kernel
-constexpr uint32_t kItemsPerWarp = 4;    // pext items per warp (one binary search per run)
 
 unsigned grid_for(uint64_t n, int n_sms, int per_sm = 16) {
   uint64_t g = (n + kT - 1) / kT;
@@ -215,22 +214,29 @@ __device__ __forceinline__ void pext_item(const uint32_t* __restrict__ mp, const
                                           uint32_t nm, uint32_t ja, uint32_t jb, uint32_t oj,
                                           uint32_t* __restrict__ data) {
   uint32_t acc[G], xn[G];
+  const uint32_t* P[G];
   uint32_t nb = 0;
-  uint32_t mn = __ldg(mp + 32u * ja);
+  mp += 32u * ja;
+  uint32_t mn = __ldg(mp);
 #pragma unroll
   for (uint32_t q = 0; q < G; ++q) {
     acc[q] = 0;
-    xn[q] = __ldg(sbase + (so[q] + 32u * ja));
+    P[q] = sbase + so[q] + 32u * ja;
+    xn[q] = __ldg(P[q]);
   }
   for (uint32_t j = ja; j < jb; ++j) {
     const uint32_t mw = mn;
     uint32_t x[G];
 #pragma unroll
     for (uint32_t q = 0; q < G; ++q) x[q] = xn[q];
-    const uint32_t jn = min(j + 1, jb - 1);
-    mn = __ldg(mp + 32u * jn);
+    const uint32_t step = j + 1 < jb ? 32u : 0u;
+    mp += step;
+    mn = __ldg(mp);
 #pragma unroll
-    for (uint32_t q = 0; q < G; ++q) xn[q] = __ldg(sbase + (so[q] + 32u * jn));
+    for (uint32_t q = 0; q < G; ++q) {
+      P[q] += step;
+      xn[q] = __ldg(P[q]);
+    }
     uint32_t mv[5];
     hd_prep(mw, mv);
     const uint32_t pw = 1u << nb;
@@ -261,33 +267,29 @@ __device__ __forceinline__ void pext_item(const uint32_t* __restrict__ mp, const
 
 // Warp per run of kItemsPerWarp consecutive items; an item = (pair p = (segment, class), group of
 // <= kMemberGroup members -- the class' members split evenly over its groups).
+// item -> its pair (items of pair p are item_off[p] .. + items[p])
+__global__ void item_pair_kernel(const uint32_t* __restrict__ items, const uint32_t* __restrict__ item_off,
+                                 uint32_t n_pairs, uint32_t* __restrict__ item_pair) {
+  for (uint32_t p = blockIdx.x * blockDim.x + threadIdx.x; p < n_pairs; p += gridDim.x * blockDim.x)
+    for (uint32_t i = 0; i < items[p]; ++i) item_pair[item_off[p] + i] = p;
+}
+
+// Warp per item = (pair p = (segment, class), group of <= kMemberGroup members -- the class'
+// members split evenly over its groups).  Items run pair-major = segment-major, so the warps in
+// flight share the same bitset segments in L2.
 __global__ void __launch_bounds__(kT, 4) pext_kernel(Src src, const uint32_t* __restrict__ par_a,
                                                      const uint32_t* __restrict__ par_b,
                                                      const uint32_t* __restrict__ bound, uint32_t cmax,
-                                                     uint32_t n_pairs, const uint32_t* __restrict__ item_off,
+                                                     const uint32_t* __restrict__ item_pair,
+                                                     const uint32_t* __restrict__ item_off,
                                                      uint32_t T, const uint32_t* __restrict__ loc,
                                                      const uint64_t* __restrict__ off, uint32_t* __restrict__ data) {
   const uint32_t lane = threadIdx.x & 31;
-  const uint32_t it0 = ((blockIdx.x * blockDim.x + threadIdx.x) >> 5) * kItemsPerWarp;
-  if (it0 >= T) return;
-  uint32_t p = 0;
-  {
-    uint32_t hi = n_pairs;  // pair = last with item_off[p] <= it0
-    while (p + 1 < hi) {
-      const uint32_t mid = (p + hi) >> 1;
-      if (item_off[mid] <= it0) p = mid; else hi = mid;
-    }
-  }
+  const uint32_t it = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  if (it >= T) return;
   const uint32_t* base = src.rows ? src.rows : src.data;
-  for (uint32_t it = it0; it < min(T, it0 + kItemsPerWarp); ++it) {
-    if (p + 1 < n_pairs && item_off[p + 1] <= it) {  // next pair holding items: search [p + 1, n_pairs)
-      uint32_t hi = n_pairs;
-      ++p;
-      while (p + 1 < hi) {
-        const uint32_t mid = (p + hi) >> 1;
-        if (item_off[mid] <= it) p = mid; else hi = mid;
-      }
-    }
+  {
+    const uint32_t p = item_pair[it];
     const uint32_t c = p % cmax, s = p / cmax;
     const uint32_t j0 = bound[c], m = bound[c + 1] - j0;
     const uint32_t groups = (m + kMemberGroup - 1) / kMemberGroup;
@@ -297,7 +299,7 @@ __global__ void __launch_bounds__(kT, 4) pext_kernel(Src src, const uint32_t* __
     const VecRef mk = src.vec(par_a[j0]);
     uint32_t ja, jb;
     seg_range(mk.lw, s, ja, jb);
-    if (ja >= jb) continue;
+    if (ja >= jb) return;
     uint32_t so[kMemberGroup], oo[kMemberGroup];
 #pragma unroll
     for (uint32_t q = 0; q < kMemberGroup; ++q) {
@@ -388,7 +390,7 @@ __global__ void proj_totals_kernel(const uint32_t* __restrict__ items, const uin
 // per-thread, per-device persistent workspace (grow-only): the class tables of proj_build and the
 // two generations of lists
 struct ProjWork {
-  PBuf<uint32_t> flag, ex, bound, small, words, loc, items, item_off, nwc;
+  PBuf<uint32_t> flag, ex, bound, small, words, loc, items, item_off, item_pair, nwc;
   PBuf<uint64_t> cls_words, cls_base, tot;
   DeviceProj lists[2];
 };
@@ -490,9 +492,11 @@ bool proj_build(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const 
   { entry_off_kernel<<<grid_for(n, n_sms), kT, 0, s>>>(flag.p, ex.p, bound.p, nwc.p, cls_base.p, n, out.off.p,
                                                       out.nw.p); note_launch(); }
   if (T[0]) {
-    const uint64_t warps = (T[0] + kItemsPerWarp - 1) / kItemsPerWarp;
-    const uint64_t blocks = (warps + warps_per_block - 1) / warps_per_block;
-    { pext_kernel<<<(unsigned)blocks, kT, 0, s>>>(src, par_a, par_b, bound.p, cmax, n_pairs, item_off.p,
+    W.item_pair.ensure(T[0]);
+    { item_pair_kernel<<<grid_for(n_pairs, n_sms), kT, 0, s>>>(items.p, item_off.p, n_pairs, W.item_pair.p);
+      note_launch(); }
+    const uint64_t blocks = (T[0] + warps_per_block - 1) / warps_per_block;
+    { pext_kernel<<<(unsigned)blocks, kT, 0, s>>>(src, par_a, par_b, bound.p, cmax, W.item_pair.p, item_off.p,
                                                   (uint32_t)T[0], loc.p, out.off.p, out.data.p); note_launch(); }
   }
   GPA_CUDA(cudaGetLastError());
