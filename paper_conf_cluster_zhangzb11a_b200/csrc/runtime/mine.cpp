@@ -106,6 +106,41 @@ bool count_projected(gpa_bitset* bs, uint32_t k, const DeviceLevel& L, const Dev
   return true;
 }
 
+// Page-locked staging for the frequent itemsets: each generation's L_k (item ids, supports) is
+// copied to the host right after its threshold, overlapping the next generations, into blocks
+// that persist per thread across calls (grow-only); the result vectors are filled from them at
+// the end (a pageable D2H of all of F took ~3 ms at the end of the loop on T40I10D10M).
+struct PinnedArena {
+  std::vector<std::pair<uint8_t*, size_t>> blocks;
+  size_t cur = 0, used = 0;
+  void reset() { cur = 0; used = 0; }
+  void* get(size_t bytes) {
+    bytes = (bytes + 255) & ~size_t(255);
+    while (cur < blocks.size() && used + bytes > blocks[cur].second) {
+      ++cur;
+      used = 0;
+    }
+    if (cur == blocks.size()) {
+      const size_t sz = std::max<size_t>(bytes, size_t(64) << 20);
+      void* p = nullptr;
+      GPA_CUDA(cudaHostAlloc(&p, sz, cudaHostAllocDefault));
+      blocks.emplace_back(static_cast<uint8_t*>(p), sz);
+      used = 0;
+    }
+    void* r = blocks[cur].first + used;
+    used += bytes;
+    return r;
+  }
+  ~PinnedArena() {
+    for (auto& b : blocks) cudaFreeHost(b.first);
+  }
+};
+
+PinnedArena& pinned_arena() {
+  thread_local PinnedArena a;
+  return a;
+}
+
 }  // namespace
 
 gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist, const gpa_options* opt_in) {
@@ -115,6 +150,7 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
   if (opt_in) opt = *opt_in;
   GPA_REQUIRE(min_count >= 1, GPA_ERR_INVALID, "min_count must be >= 1");
   const bool keep = (opt.flags & GPA_KEEP_CANDIDATES) != 0;
+  pinned_arena().reset();  // a previous call on this thread consumed its blocks before returning
   const bool host_candgen = (opt.flags & GPA_HOST_CANDGEN) != 0;
   const uint32_t max_k = opt.max_k ? opt.max_k : GPA_MAX_K;
   GPA_REQUIRE(min_count < (1ull << 32), GPA_ERR_INVALID, "min_count must be < 2^32");
@@ -182,8 +218,24 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     size_t level = 0;
     uint32_t F = 0, k = 0;
     DBuf<uint32_t> items, sup;
+    const uint32_t* h_items = nullptr;  // page-locked copies (pinned_arena)
+    const uint32_t* h_sup = nullptr;
   };
   std::vector<Pending> pending;
+  struct CopyStream {
+    cudaStream_t s = nullptr;
+    CopyStream() { GPA_CUDA(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking)); }
+    ~CopyStream() {
+      if (s) { cudaStreamSynchronize(s); cudaStreamDestroy(s); }
+    }
+  } copy_s;
+  constexpr int kCopyEvents = 4;   // re-recorded round robin: a wait captures the event's state at call time
+  struct Events {
+    cudaEvent_t e[kCopyEvents] = {};
+    Events() { for (auto& x : e) GPA_CUDA(cudaEventCreateWithFlags(&x, cudaEventDisableTiming)); }
+    ~Events() { for (auto x : e) if (x) cudaEventDestroy(x); }
+  } copy_evs;
+  cudaEvent_t* copy_ev = copy_evs.e;
   struct EvTriple {      // deferred timing of a generation's counting launch(es) and all-reduce
     cudaEvent_t e[3] = {nullptr, nullptr, nullptr};
     EvTriple() {
@@ -292,6 +344,15 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
       pd.sup.alloc(F, s);
       device_map_items(Ln.rows.p, (uint64_t)F * k, d_ior.p, pd.items.p, bs->n_sms, s);
       GPA_CUDA(cudaMemcpyAsync(pd.sup.p, Ln.sup.p, (size_t)F * 4, cudaMemcpyDeviceToDevice, s));
+      auto* hi = static_cast<uint32_t*>(pinned_arena().get((size_t)F * k * 4));
+      auto* hs = static_cast<uint32_t*>(pinned_arena().get((size_t)F * 4));
+      // D2H on the copy stream, overlapping the next generations on s
+      GPA_CUDA(cudaEventRecord(copy_ev[(k - 2) % kCopyEvents], s));
+      GPA_CUDA(cudaStreamWaitEvent(copy_s.s, copy_ev[(k - 2) % kCopyEvents], 0));
+      GPA_CUDA(cudaMemcpyAsync(hi, pd.items.p, (size_t)F * k * 4, cudaMemcpyDeviceToHost, copy_s.s));
+      GPA_CUDA(cudaMemcpyAsync(hs, pd.sup.p, (size_t)F * 4, cudaMemcpyDeviceToHost, copy_s.s));
+      pd.h_items = hi;
+      pd.h_sup = hs;
     }
     std::vector<uint32_t> counts;
     if (keep) {
@@ -323,7 +384,10 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
   }
 
   // ---- deferred: kernel times and the frequent itemsets of every generation
+  const double tf0 = now_ms();
   GPA_CUDA(cudaStreamSynchronize(s));
+  GPA_CUDA(cudaStreamSynchronize(copy_s.s));
+  const double tf1 = now_ms();
   for (size_t i = 0; i < event_level.size(); ++i) {
     float a = 0, b = 0;
     GPA_CUDA(cudaEventElapsedTime(&a, events[i].e[0], events[i].e[1]));
@@ -332,17 +396,15 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     st.count_ms = a;
     st.allreduce_ms = dist ? b : 0.0;
   }
-  for (auto& pd : pending) {
+  parallel_for(pending.size(), [&](size_t i) {
+    const Pending& pd = pending[i];
     gpa_level_data& lv = R->levels[pd.level];
-    lv.freq_items.resize((size_t)pd.F * pd.k);
-    lv.freq_support.resize(pd.F);
-    if (pd.F) {
-      GPA_CUDA(cudaMemcpyAsync(lv.freq_items.data(), pd.items.p, (size_t)pd.F * pd.k * 4, cudaMemcpyDeviceToHost, s));
-      GPA_CUDA(cudaMemcpyAsync(lv.freq_support.data(), pd.sup.p, (size_t)pd.F * 4, cudaMemcpyDeviceToHost, s));
-    }
-  }
-  GPA_CUDA(cudaStreamSynchronize(s));
+    lv.freq_items.assign(pd.h_items, pd.h_items + (size_t)pd.F * pd.k);
+    lv.freq_support.assign(pd.h_sup, pd.h_sup + pd.F);
+  });
   pending.clear();
+  if (trace_enabled())
+    fprintf(stderr, "[gpa] end of loop: drain %.2f ms, F transfer %.2f ms\n", tf1 - tf0, now_ms() - tf1);
 
   uint64_t acc = 0;
   for (auto& lv : R->levels) {

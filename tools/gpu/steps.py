@@ -14,5 +14,6 @@ for i in range(n):
     torch.cuda.synchronize(); t = time.perf_counter()
     r = gpa.mine(off, it, ds.n_items, min_count=theta, options=gpa.Options(count_kernel=kern))
     torch.cuda.synchronize(); dt = (time.perf_counter() - t) * 1e3
-    print(f"step {i}: {dt:.1f} ms  |F|={len(r.frequent())}  levels " +
+    print(f"step {i}: {dt:.1f} ms (C total {r.timing_ms['total']:.1f}, phases " +
+          " ".join(f"{k}:{v:.1f}" for k, v in r.timing_ms.items()) + f")  |F|={sum(lv.n_freq for lv in r.levels)}  levels " +
           " ".join(f"k{lv.k}:{lv.stats['count_ms']:.1f}" for lv in r.levels[1:]), flush=True)
