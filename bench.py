@@ -261,7 +261,7 @@ def main():
         res = gpa.mine(d_off, d_items, ds.n_items, min_count=theta, dist=dist, options=opts)
     # ---- timed: K steps, inputs resident in HBM
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    level_ms = {}
+    level_ms, build_ms = {}, {}
     barrier()
     launches0 = gpa.kernel_launches()
     with ClockSampler(local) as clocks:
@@ -270,6 +270,7 @@ def main():
             res = gpa.mine(d_off, d_items, ds.n_items, min_count=theta, dist=dist, options=opts)
             for lv in res.levels[1:]:
                 level_ms.setdefault(lv.k, []).append(lv.stats["count_ms"])
+                build_ms.setdefault(lv.k, []).append(lv.stats["build_ms"])
         ev1.record(stream)
         barrier()
     launches = gpa.kernel_launches() - launches0   # every kernel the library launched in the region
@@ -297,11 +298,26 @@ def main():
     clk = clocks.summary()
     sm_max = clk.get("sm_max_mhz") or peaks.get("sm_max_mhz", 1965.0)
     popc_per_word = {"pairs": 0.75}
+    # ALU and FMA pipes: 64 lanes / clk / SM each (rt_SMSP = 2 cycles per warp instruction on both,
+    # /opt/skills/guides/B300_MICROARCH.md "Pipe rates"), 148 SMs on B200
+    int_peak = 148 * 128 * sm_max * 1e6 / 1e12
+    PEXT_OPS = 17   # per member-word: HD compress 5 x (AND, shift, merge) + append (shift, OR)
 
-    def roof_for(levels):
-        ms = max_over_ranks(sum(float(np.mean(level_ms[lv.k])) for lv in levels))
-        work = sum(lv.n_cand for lv in levels) * n_tx
-        name = levels[0].stats["kernel_name"]
+    # one record per launch kind and generation: (name, k, ms per step, algorithmic work)
+    recs = []
+    for lv in res.levels[1:]:
+        ms = float(np.mean(level_ms[lv.k]))
+        if lv.stats["kernel_name"] == "proj":
+            bms = float(np.mean(build_ms[lv.k]))
+            recs.append(("pext", lv.k, bms, lv.stats["build_words"], lv))
+            recs.append(("count_proj", lv.k, ms - bms, lv.n_cand * n_tx, lv))
+        else:
+            recs.append((lv.stats["kernel_name"], lv.k, ms, lv.n_cand * n_tx, lv))
+
+    def roof_for(rs):
+        name = rs[0][0]
+        ms = max_over_ranks(sum(r[2] for r in rs))
+        work = sum(r[3] for r in rs)
         if name == "pairs_tc":
             bf16 = float(peaks.get("bf16_tflops", 2250.0 * 1965 / 1965))
             peak = 2.0 * bf16
@@ -312,6 +328,16 @@ def main():
                                   if "bf16_tflops" in peaks else "int8 dense = 2 x 2250 TFLOP/s nominal bf16 (no "
                                   "MEASURED_PEAKS.json)",
                     "kernel_ms": ms, "work": work, "cand_tx_per_s": work / (ms * 1e-3)}
+        if name == "pext":
+            ach = work * PEXT_OPS / (ms * 1e-3) / 1e12
+            return {"bound": "alu", "achieved": ach, "peak": int_peak, "unit": "T int ops/s", "frac": ach / int_peak,
+                    "peak_basis": f"ALU + FMA pipes, 2 x 64 lanes/clk/SM x 148 SM x {sm_max:.0f} MHz; "
+                                  f"{PEXT_OPS} algorithmic ops per compressed 32-bit mask word and member",
+                    "kernel_ms": ms, "work": work, "work_unit": "mask words x members"}
+        if name == "count_proj":
+            return {"bound": None, "achieved": work / (ms * 1e-3) / 1e12, "peak": None, "unit": "Tcand*tx/s "
+                    "(effective: supports of |C_k| x N cand*tx from the projected lists)", "frac": None,
+                    "kernel_ms": ms, "work": work}
         ppw = popc_per_word.get(name, 1.0)
         peak = 148 * 16 / ppw * 32 * sm_max * 1e6 / 1e12
         ach = work / (ms * 1e-3) / 1e12
@@ -321,25 +347,26 @@ def main():
                 "kernel_ms": ms, "work": work}
 
     by_kernel = {}
-    for lv in res.levels[1:]:
-        by_kernel.setdefault(lv.stats["kernel_name"], []).append(lv)
-    roof_all = {name: roof_for(lvs) for name, lvs in by_kernel.items()}
-    dom = max(res.levels[1:], key=lambda lv: float(np.mean(level_ms[lv.k])))   # single longest launch
+    for r in recs:
+        by_kernel.setdefault(r[0], []).append(r)
+    roof_all = {name: roof_for(rs) for name, rs in by_kernel.items()}
+    dom = max(recs, key=lambda r: r[2])   # single longest launch
     roof = roof_for([dom])
-    roof["kernel"] = f"count_{dom.stats['kernel_name']} (generation {dom.k}, the longest launch)"
+    roof["kernel"] = f"{dom[0] if dom[0] == 'pext' else 'count_' + dom[0]} (generation {dom[1]}, the longest launch)"
     # DRAM traffic per launch of this kernel from the committed ncu --set full capture
     # (profiles/traffic.json, written from profiles/r*_ncu_*.txt); null if not captured
     roof["traffic"] = None
     try:
         tr = json.load(open(os.path.join(ROOT, "profiles", "traffic.json")))
-        key = {"pairs": "count_pairs_kernel", "prefix": "count_prefix_kernel",
-               "pairs_tc": "count_pairs_tc_kernel"}.get(
-            dom.stats["kernel_name"], f"count_trie_kernel<{dom.k}, {1 if dom.k == 2 else 2}>")
+        key = {"pairs": "count_pairs_kernel", "prefix": "count_prefix_kernel", "pext": f"pext_kernel (k={dom[1]})",
+               "pairs_tc": "count_pairs_tc_kernel"}.get(dom[0], f"count_trie_kernel<{dom[1]}, 2>")
         if key in tr:
             roof["traffic"] = tr[key]["dram_bytes"]
             roof["traffic_unit"] = "bytes per launch (ncu dram__bytes_read.sum + dram__bytes_write.sum)"
-            # algorithmic bytes of this launch: each of the n rows read once (streaming design)
-            roof["algorithmic_bytes"] = (dom.stats["n_groups"] + 1) * (n_tx / 8) if dom.k == 2 else None
+            if dom[0] == "pext" and "algorithmic_bytes" in tr[key]:
+                roof["algorithmic_bytes"] = tr[key]["algorithmic_bytes"]
+            elif dom[1] == 2:   # each of the n rows read once (streaming design)
+                roof["algorithmic_bytes"] = (dom[4].stats["n_groups"] + 1) * (n_tx / 8)
     except Exception:
         pass
     for r in roof_all.values():
@@ -362,7 +389,8 @@ def main():
         e2e_ms = max_over_ranks(e0.elapsed_time(e1) / args.steps)
         assert r2.frequent() == res.frequent()
         h2d = int(ds.offsets.nbytes + ds.items.nbytes)
-        d2h = 4 * sum(lv.n_cand for lv in r2.levels)  # every generation's counts (+ the histogram)
+        # the histogram, and every generation's frequent itemsets (k item ids + support each)
+        d2h = 4 * ds.n_items + 4 * sum(lv.n_freq * (lv.k + 1) for lv in r2.levels[1:])
         e2e = {"value": cand_tx / (e2e_ms * 1e-3), "unit": "cand*tx/s", "ms_per_step": e2e_ms,
                "h2d_bytes_per_step": h2d * world, "d2h_bytes_per_step": d2h}
 

@@ -237,6 +237,10 @@ typedef struct {
   double count_ms;             /* CUDA-event time of the counting kernel(s), this rank */
   double allreduce_ms;         /* CUDA-event time of the count all-reduce (0 without dist) */
   double candgen_ms;           /* host join + prune + grouping */
+  double build_ms;             /* GPA_KERNEL_PROJ: CUDA-event time of the list-building kernel (pext) for
+                                  L_{k-1}'s projected lists (included in count_ms); 0 otherwise */
+  uint64_t build_words;        /* GPA_KERNEL_PROJ: 32-bit mask words x members the list build compressed
+                                  (its algorithmic work); 0 otherwise */
 } gpa_level_stats;
 gpa_status gpa_result_level_stats(const gpa_result* r, uint32_t k, gpa_level_stats* out);
 

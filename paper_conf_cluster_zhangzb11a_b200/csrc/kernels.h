@@ -148,6 +148,7 @@ struct DeviceProj {
   PBuf<uint32_t> data;
   uint64_t words = 0;
   uint32_t max_lw = 0;    // longest lane stream (words) of any class
+  uint64_t in_words = 0;  // mask words x members compressed to build these lists (algorithmic work)
 };
 // The calling thread's two DeviceProj for `device` (previous / current generation).
 DeviceProj* proj_lists(int device);
@@ -156,7 +157,7 @@ DeviceProj* proj_lists(int device);
 // when the vectors do not fit (device memory / 32-bit totals): use complete intersection.
 bool proj_build(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const DeviceProj* prev,
                 const uint32_t* rows, uint64_t pitch_words, uint32_t n_rows, DeviceProj& out, DeviceScratch& scratch,
-                int n_sms, cudaStream_t s);
+                int n_sms, cudaStream_t s, cudaEvent_t ev_build = nullptr);
 // counts[m] += popc(V_gpar[g] & V_eidx[m]) for every candidate m of group g (counts zeroed by the caller)
 void launch_count_proj(const DeviceProj& P, const uint32_t* gpar, const uint32_t* ext_off, const uint32_t* eidx,
                        uint32_t G, uint32_t* counts, cudaStream_t s);

@@ -99,7 +99,7 @@ __device__ __forceinline__ void seg_range(uint32_t lw, uint32_t s, uint32_t& j0,
 // words[p][l] = its output words (bits rounded up to whole words)
 __global__ void seg_popc_kernel(Src src, const uint32_t* __restrict__ par_a, const uint32_t* __restrict__ bound,
                                 const uint32_t* __restrict__ n_cls, uint32_t cmax, uint32_t nseg, uint32_t n_pairs,
-                                uint32_t* __restrict__ words) {
+                                uint32_t* __restrict__ words, unsigned long long* __restrict__ in_words) {
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t p = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   if (p >= n_pairs) return;
@@ -112,6 +112,7 @@ __global__ void seg_popc_kernel(Src src, const uint32_t* __restrict__ par_a, con
       uint32_t a, b;
       seg_range(mk.lw, s, a, b);
       for (uint32_t j = a; j < b; ++j) cnt += __popc(mk.p[32ull * j + lane]);
+      if (lane == 0 && b > a) atomicAdd(in_words, 32ull * (b - a) * m);
     }
   }
   words[(uint64_t)p * 32 + lane] = (cnt + 31) / 32;
@@ -405,10 +406,14 @@ DeviceProj* proj_lists(int device) { return work_for(device).lists; }
 
 bool proj_build(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const DeviceProj* prev,
                 const uint32_t* rows, uint64_t pitch_words, uint32_t n_rows, DeviceProj& out, DeviceScratch& scratch,
-                int n_sms, cudaStream_t s) {
+                int n_sms, cudaStream_t s, cudaEvent_t ev_build) {
   out.n = n;
   out.words = 0;
-  if (n == 0) return true;
+  out.in_words = 0;
+  if (n == 0) {
+    if (ev_build) GPA_CUDA(cudaEventRecord(ev_build, s));
+    return true;
+  }
   Src src{};
   if (!prev) {
     src.rows = rows;
@@ -460,7 +465,8 @@ bool proj_build(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const 
   tot.ensure(2);
   const unsigned warps_per_block = kT / 32;
   { seg_popc_kernel<<<(n_pairs + warps_per_block - 1) / warps_per_block, kT, 0, s>>>(
-        src, par_a, bound.p, small.p, cmax, nseg, n_pairs, words.p); note_launch(); }
+        src, par_a, bound.p, small.p, cmax, nseg, n_pairs, words.p,
+        reinterpret_cast<unsigned long long*>(small.p + 2)); note_launch(); }
   { cls_pad_kernel<<<(cmax + warps_per_block - 1) / warps_per_block, kT, 0, s>>>(
         words.p, bound.p, small.p, cmax, nseg, loc.p, nwc.p, cls_words.p, items.p, small.p + 1); note_launch(); }
   scan_excl<uint32_t>(items.p, item_off.p, n_pairs, scratch, s);
@@ -469,9 +475,9 @@ bool proj_build(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const 
     note_launch(); }
   GPA_CUDA(cudaGetLastError());
   uint64_t T[2] = {0, 0};
-  uint32_t mlw = 0;
+  uint32_t sm[4] = {0, 0, 0, 0};
   GPA_CUDA(cudaMemcpyAsync(T, tot.p, sizeof(T), cudaMemcpyDeviceToHost, s));
-  GPA_CUDA(cudaMemcpyAsync(&mlw, small.p + 1, 4, cudaMemcpyDeviceToHost, s));
+  GPA_CUDA(cudaMemcpyAsync(sm, small.p, sizeof(sm), cudaMemcpyDeviceToHost, s));
   const double h0 = wall_ms();
   GPA_CUDA(cudaStreamSynchronize(s));
   const double h1 = wall_ms();
@@ -485,12 +491,14 @@ bool proj_build(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const 
   out.off.ensure(n);
   out.nw.ensure(n);
   out.words = T[1];
-  out.max_lw = mlw;
+  out.max_lw = sm[1];
+  out.in_words = (uint64_t)sm[2] | ((uint64_t)sm[3] << 32);
   const double h2 = wall_ms();
   // lanes shorter than their class' Lw keep a zero tail
   GPA_CUDA(cudaMemsetAsync(out.data.p, 0, std::max<uint64_t>(T[1], 1) * 4, s));
   { entry_off_kernel<<<grid_for(n, n_sms), kT, 0, s>>>(flag.p, ex.p, bound.p, nwc.p, cls_base.p, n, out.off.p,
                                                       out.nw.p); note_launch(); }
+  if (ev_build) GPA_CUDA(cudaEventRecord(ev_build, s));  // start of the list build proper
   if (T[0]) {
     W.item_pair.ensure(T[0]);
     { item_pair_kernel<<<grid_for(n_pairs, n_sms), kT, 0, s>>>(items.p, item_off.p, n_pairs, W.item_pair.p);

@@ -99,6 +99,8 @@ struct CountStats {
   // optional caller-owned events: with them the counting functions do not synchronise; the
   // caller reads count_ms / allreduce_ms from (e0, e1) / (e1, e2) later
   cudaEvent_t e0 = nullptr, e1 = nullptr, e2 = nullptr;
+  cudaEvent_t ep = nullptr, eb = nullptr;  // GPA_KERNEL_PROJ: the list-building kernel (ep .. eb)
+  uint64_t build_words = 0;
 };
 
 }  // namespace gpa

@@ -92,10 +92,12 @@ bool count_projected(gpa_bitset* bs, uint32_t k, const DeviceLevel& L, const Dev
   const double t0 = now_ms();
   GPA_CUDA(cudaEventRecord(cs->e0, s));
   if (!proj_build(L.n, L.par_a.p, L.par_b.p, k == 3 ? nullptr : &prev, bs->rows.p, bs->pitch_words, bs->n_rows, cur,
-                  scratch, bs->n_sms, s))
+                  scratch, bs->n_sms, s, cs->ep))
     return false;
   bs->d_counts.ensure(B.M, s);
   GPA_CUDA(cudaMemsetAsync(bs->d_counts.p, 0, (size_t)B.M * 4, s));
+  GPA_CUDA(cudaEventRecord(cs->eb, s));
+  cs->build_words = cur.in_words;
   launch_count_proj(cur, B.gpar.p, B.ext_off.p, B.eidx.p, B.G, bs->d_counts.p, s);
   cs->kernel = GPA_KERNEL_PROJ;
   cs->launches = 1;
@@ -237,12 +239,12 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
   } copy_evs;
   cudaEvent_t* copy_ev = copy_evs.e;
   struct EvTriple {      // deferred timing of a generation's counting launch(es) and all-reduce
-    cudaEvent_t e[3] = {nullptr, nullptr, nullptr};
+    cudaEvent_t e[5] = {nullptr, nullptr, nullptr, nullptr, nullptr};  // + projected-list build [3, 4)
     EvTriple() {
       for (auto& x : e) GPA_CUDA(cudaEventCreate(&x));
     }
     EvTriple(EvTriple&& o) noexcept {
-      for (int i = 0; i < 3; ++i) std::swap(e[i], o.e[i]);
+      for (int i = 0; i < 5; ++i) std::swap(e[i], o.e[i]);
     }
     EvTriple(const EvTriple&) = delete;
     ~EvTriple() {
@@ -301,6 +303,8 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     cs.e0 = ev.e[0];
     cs.e1 = ev.e[1];
     cs.e2 = ev.e[2];
+    cs.ep = ev.e[3];
+    cs.eb = ev.e[4];
     GPA_REQUIRE(M < (1ull << 32), GPA_ERR_INVALID, "generation %u has too many candidates", k);
     // the host copy of C_k is needed only for the host-planned kernels and for GPA_KEEP_CANDIDATES
     auto fetch_batch = [&]() {
@@ -380,6 +384,7 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     st.count_ms = cs.count_ms;
     st.allreduce_ms = cs.allreduce_ms;
     st.candgen_ms = t1 - t0;
+    st.build_words = cs.build_words;
     R->phase_ms[GPA_PHASE_THRESHOLD] += now_ms() - t2;
   }
 
@@ -392,6 +397,12 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     float a = 0, b = 0;
     GPA_CUDA(cudaEventElapsedTime(&a, events[i].e[0], events[i].e[1]));
     GPA_CUDA(cudaEventElapsedTime(&b, events[i].e[1], events[i].e[2]));
+    gpa_level_stats& st0 = R->levels[event_level[i]].stats;
+    if (st0.kernel == GPA_KERNEL_PROJ) {
+      float c = 0;
+      GPA_CUDA(cudaEventElapsedTime(&c, events[i].e[3], events[i].e[4]));
+      st0.build_ms = c;
+    }
     gpa_level_stats& st = R->levels[event_level[i]].stats;
     st.count_ms = a;
     st.allreduce_ms = dist ? b : 0.0;

@@ -7,7 +7,7 @@ import gen, paper_conf_cluster_zhangzb11a_b200 as gpa
 for name in ["chess", "mushroom"]:
     ds = gen.make(name)
     th = gpa.min_count(ds.n_tx, gen.CONFIGS[name].minsup)
-    for kern in (gpa.KERNEL_AUTO, gpa.KERNEL_V0, gpa.KERNEL_PREFIX, gpa.KERNEL_TRIE):
+    for kern in (gpa.KERNEL_AUTO, gpa.KERNEL_V0, gpa.KERNEL_PREFIX, gpa.KERNEL_TRIE, gpa.KERNEL_PROJ):
         r = gpa.mine(ds, min_count=th, options=gpa.Options(count_kernel=kern, max_k=6))
         print(name, kern, len(r.frequent()))
 # overlapped ingest (host input >= 262,144 transactions) and the device level transition
