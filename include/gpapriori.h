@@ -241,6 +241,9 @@ typedef struct {
                                   L_{k-1}'s projected lists (included in count_ms); 0 otherwise */
   uint64_t build_words;        /* GPA_KERNEL_PROJ: 32-bit mask words x members the list build compressed
                                   (its algorithmic work); 0 otherwise */
+  double setup_ms;             /* GPA_KERNEL_PROJ: CUDA-event time from the start of the generation's
+                                  counting to the list-building kernel (class tables, sizes); the
+                                  support kernel is count_ms - setup_ms - build_ms */
 } gpa_level_stats;
 gpa_status gpa_result_level_stats(const gpa_result* r, uint32_t k, gpa_level_stats* out);
 

@@ -64,7 +64,7 @@ class _LevelStats(ctypes.Structure):
     _fields_ = [("n_cand", ctypes.c_uint64), ("n_freq", ctypes.c_uint64), ("n_groups", ctypes.c_uint64),
                 ("kernel", ctypes.c_uint32), ("launches", ctypes.c_uint32), ("count_ms", ctypes.c_double),
                 ("allreduce_ms", ctypes.c_double), ("candgen_ms", ctypes.c_double), ("build_ms", ctypes.c_double),
-                ("build_words", ctypes.c_uint64)]
+                ("build_words", ctypes.c_uint64), ("setup_ms", ctypes.c_double)]
 
 
 _LIB = None

@@ -402,6 +402,8 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
       float c = 0;
       GPA_CUDA(cudaEventElapsedTime(&c, events[i].e[3], events[i].e[4]));
       st0.build_ms = c;
+      GPA_CUDA(cudaEventElapsedTime(&c, events[i].e[0], events[i].e[3]));
+      st0.setup_ms = c;
     }
     gpa_level_stats& st = R->levels[event_level[i]].stats;
     st.count_ms = a;
