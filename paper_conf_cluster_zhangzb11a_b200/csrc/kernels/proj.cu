@@ -175,55 +175,70 @@ __global__ void entry_off_kernel(const uint32_t* __restrict__ flag, const uint32
 __device__ __forceinline__ uint32_t shr_c(uint32_t x, int s) { return __umulhi(x, 1u << (32 - s)); }
 __device__ __forceinline__ uint32_t shl_c(uint32_t x, int s) { return x * (1u << s); }
 
-__device__ __forceinline__ void hd_prep(uint32_t m, uint32_t (&mv)[5]) {
+__device__ __forceinline__ void hd_prep(uint32_t m, uint32_t (&mv)[5], uint32_t& m0) {
+  const uint32_t m_in = m;
   uint32_t mk = shl_c(~m, 1);
 #pragma unroll
   for (int i = 0; i < 5; ++i) {
-    uint32_t mp = mk ^ shl_c(mk, 1);
-    mp ^= shl_c(mp, 2);
-    mp ^= shl_c(mp, 4);
-    mp ^= shl_c(mp, 8);
-    mp ^= shl_c(mp, 16);
-    const uint32_t v = mp & m;
+    // parallel prefix XOR of mk (HD's 5 shift-xor steps) as 3-input XORs: windows 3, 9, 27, 54
+    uint32_t mp = mk ^ shl_c(mk, 1) ^ shl_c(mk, 2);
+    mp = mp ^ shl_c(mp, 3) ^ shl_c(mp, 6);
+    mp = mp ^ shl_c(mp, 9) ^ shl_c(mp, 18);
+    mp ^= shl_c(mp, 27);
+    uint32_t v;  // materialised (opaque AND), so hd_apply's merge is one LOP3 on (x, mv, shifted)
+    asm("and.b32 %0, %1, %2;" : "=r"(v) : "r"(mp), "r"(m));
     mv[i] = v;
     m = (m ^ v) | shr_c(v, 1 << i);
     mk &= ~mp;
   }
+  asm("lop3.b32 %0, %1, %2, 0, 0x30;" : "=r"(m0) : "r"(m_in), "r"(mv[0]));  // m & ~mv0: bits kept by stage 0
 }
-// pext(x, m) given m's shift masks (x need not be pre-masked: stage 0 folds the AND with m)
-__device__ __forceinline__ uint32_t hd_apply(uint32_t x, uint32_t m, const uint32_t (&mv)[5]) {
-  uint32_t t = x & mv[0];
-  x = (x & m & ~mv[0]) | shr_c(t, 1);
+// pext(x, m) given m's shift masks (x need not be pre-masked: stage 0 keeps x & m0 and moves x & mv0)
+// (each stage is two LOP3 -- the moving bits, then keep-or-moved in one 3-input op -- and one
+// IMAD.HI; written as PTX lop3 so that the compiler cannot split the merge into AND + OR)
+__device__ __forceinline__ uint32_t hd_apply(uint32_t x, uint32_t m0, const uint32_t (&mv)[5]) {
+  uint32_t t, y;
+  asm("and.b32 %0, %1, %2;" : "=r"(t) : "r"(x), "r"(mv[0]));
+  asm("lop3.b32 %0, %1, %2, %3, 0xEA;" : "=r"(y) : "r"(x), "r"(m0), "r"(shr_c(t, 1)));  // (x & m0) | ts
 #pragma unroll
   for (int i = 1; i < 5; ++i) {
-    t = x & mv[i];
-    x = (x & ~mv[i]) | shr_c(t, 1 << i);
+    asm("and.b32 %0, %1, %2;" : "=r"(t) : "r"(y), "r"(mv[i]));
+    asm("lop3.b32 %0, %1, %2, %3, 0xBA;" : "=r"(y) : "r"(y), "r"(mv[i]), "r"(shr_c(t, 1 << i)));  // (y & ~mv) | ts
   }
-  return x;
+  return y;
 }
 
-// One item of pext_kernel for a group of nm <= G members (G = 2, 4, 8: the unrolled width, so a
-// class of 2 members does not pay for 8): lane l walks its mask words [ja, jb) and appends, for
+// One item of pext_kernel for a group of nm <= G members (G = 2, 4, 6, 8: the unrolled width, so
+// a class of 2 members does not pay for 8): lane l walks its mask words [ja, jb) and appends, for
 // every member, pext(source word, mask word) to the member's lane-l stream -- a 32-bit
 // accumulator, whole words stored as they fill, the last partial word at the segment's end.
 // The bit count per step is the mask's, the same for every member, so the fill level and the
 // output position are shared; the append is one 32x32->64 multiply by 2^fill.  The next step's
 // mask and source words are loaded one step ahead.
+// base + idx words as one IMAD.WIDE.U32 on the FMA pipe: the scale (4) comes from a kernel
+// parameter, otherwise ptxas turns the multiply by a constant 4 into LEA + LEA.HI.X on the ALU pipe
+__device__ __forceinline__ const uint32_t* addr_of(const uint32_t* base, uint32_t idx, uint32_t wbytes) {
+  const uint32_t* r;
+  asm("mad.wide.u32 %0, %1, %2, %3;" : "=l"(r) : "r"(idx), "r"(wbytes), "l"(base));
+  return r;
+}
+
 template <uint32_t G>
 __device__ __forceinline__ void pext_item(const uint32_t* __restrict__ mp, const uint32_t* __restrict__ sbase,
-                                          const uint32_t (&so)[kMemberGroup], const uint32_t (&oo)[kMemberGroup],
+                                          const uint32_t (&so)[kMemberGroup], const uint32_t* __restrict__ s_oo,
                                           uint32_t nm, uint32_t ja, uint32_t jb, uint32_t oj,
-                                          uint32_t* __restrict__ data) {
+                                          uint32_t* __restrict__ data, uint32_t wbytes) {
+  // member q's word j of this lane: cur + so[q] with cur = sbase + 32 j (one 64-bit step per j, then
+  // one IMAD.WIDE per member); output base offsets in shared memory (read only when a word fills)
   uint32_t acc[G], xn[G];
-  const uint32_t* P[G];
   uint32_t nb = 0;
   mp += 32u * ja;
+  const uint32_t* cur = sbase + 32u * ja;
   uint32_t mn = __ldg(mp);
 #pragma unroll
   for (uint32_t q = 0; q < G; ++q) {
     acc[q] = 0;
-    P[q] = sbase + so[q] + 32u * ja;
-    xn[q] = __ldg(P[q]);
+    xn[q] = __ldg(addr_of(cur, so[q], wbytes));
   }
   for (uint32_t j = ja; j < jb; ++j) {
     const uint32_t mw = mn;
@@ -232,28 +247,28 @@ __device__ __forceinline__ void pext_item(const uint32_t* __restrict__ mp, const
     for (uint32_t q = 0; q < G; ++q) x[q] = xn[q];
     const uint32_t step = j + 1 < jb ? 32u : 0u;
     mp += step;
+    cur += step;
     mn = __ldg(mp);
 #pragma unroll
-    for (uint32_t q = 0; q < G; ++q) {
-      P[q] += step;
-      xn[q] = __ldg(P[q]);
-    }
-    uint32_t mv[5];
-    hd_prep(mw, mv);
+    for (uint32_t q = 0; q < G; ++q) xn[q] = __ldg(addr_of(cur, so[q], wbytes));
+    uint32_t mv[5], m0;
+    hd_prep(mw, mv, m0);
     const uint32_t pw = 1u << nb;
     nb += __popc(mw);
-    uint32_t carry[G];
 #pragma unroll
     for (uint32_t q = 0; q < G; ++q) {
-      const uint64_t v = (uint64_t)hd_apply(x[q], mw, mv) * pw;
-      acc[q] |= (uint32_t)v;
-      carry[q] = (uint32_t)(v >> 32);
+      // append at bit nb: one 32x32->64 multiply by 2^nb (FMA pipe); the low half is disjoint from
+      // the bits already in acc, so the OR is an add (FMA pipe as well); x[q] keeps the carry
+      uint64_t v;
+      asm("mul.wide.u32 %0, %1, %2;" : "=l"(v) : "r"(hd_apply(x[q], m0, mv)), "r"(pw));
+      asm("mad.lo.u32 %0, %1, 1, %0;" : "+r"(acc[q]) : "r"((uint32_t)v));
+      x[q] = (uint32_t)(v >> 32);
     }
     if (nb >= 32) {
 #pragma unroll
       for (uint32_t q = 0; q < G; ++q) {
-        if (q < nm) data[oo[q] + 32u * oj] = acc[q];
-        acc[q] = carry[q];
+        if (q < nm) data[s_oo[q] + 32u * oj] = acc[q];
+        acc[q] = x[q];
       }
       ++oj;
       nb -= 32;
@@ -262,12 +277,10 @@ __device__ __forceinline__ void pext_item(const uint32_t* __restrict__ mp, const
   if (nb) {
 #pragma unroll
     for (uint32_t q = 0; q < G; ++q)
-      if (q < nm) data[oo[q] + 32u * oj] = acc[q];
+      if (q < nm) data[s_oo[q] + 32u * oj] = acc[q];
   }
 }
 
-// Warp per run of kItemsPerWarp consecutive items; an item = (pair p = (segment, class), group of
-// <= kMemberGroup members -- the class' members split evenly over its groups).
 // item -> its pair (items of pair p are item_off[p] .. + items[p])
 __global__ void item_pair_kernel(const uint32_t* __restrict__ items, const uint32_t* __restrict__ item_off,
                                  uint32_t n_pairs, uint32_t* __restrict__ item_pair) {
@@ -275,8 +288,8 @@ __global__ void item_pair_kernel(const uint32_t* __restrict__ items, const uint3
     for (uint32_t i = 0; i < items[p]; ++i) item_pair[item_off[p] + i] = p;
 }
 
-// Warp per item = (pair p = (segment, class), group of <= kMemberGroup members -- the class'
-// members split evenly over its groups).  Items run pair-major = segment-major, so the warps in
+// Warp per item = (pair p = (segment, class), group of <= kMemberGroup members: full groups of 8,
+// the remainder in the class' last group).  Items run pair-major = segment-major, so the warps in
 // flight share the same bitset segments in L2.
 __global__ void __launch_bounds__(kT, 4) pext_kernel(Src src, const uint32_t* __restrict__ par_a,
                                                      const uint32_t* __restrict__ par_b,
@@ -284,7 +297,8 @@ __global__ void __launch_bounds__(kT, 4) pext_kernel(Src src, const uint32_t* __
                                                      const uint32_t* __restrict__ item_pair,
                                                      const uint32_t* __restrict__ item_off,
                                                      uint32_t T, const uint32_t* __restrict__ loc,
-                                                     const uint64_t* __restrict__ off, uint32_t* __restrict__ data) {
+                                                     const uint64_t* __restrict__ off, uint32_t* __restrict__ data,
+                                                     uint32_t wbytes) {
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t it = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   if (it >= T) return;
@@ -295,27 +309,33 @@ __global__ void __launch_bounds__(kT, 4) pext_kernel(Src src, const uint32_t* __
     const uint32_t j0 = bound[c], m = bound[c + 1] - j0;
     const uint32_t groups = (m + kMemberGroup - 1) / kMemberGroup;
     const uint32_t g = it - item_off[p];
-    const uint32_t first = j0 + (uint32_t)((uint64_t)m * g / groups);
-    const uint32_t nm = j0 + (uint32_t)((uint64_t)m * (g + 1) / groups) - first;
+    (void)groups;
+    const uint32_t first = j0 + g * kMemberGroup;  // full groups of 8, the remainder in the last
+    const uint32_t nm = min(kMemberGroup, m - g * kMemberGroup);
     const VecRef mk = src.vec(par_a[j0]);
     uint32_t ja, jb;
     seg_range(mk.lw, s, ja, jb);
     if (ja >= jb) return;
-    uint32_t so[kMemberGroup], oo[kMemberGroup];
+    __shared__ uint32_t s_oo[kT / 32][kMemberGroup];
+    uint32_t* oo = s_oo[threadIdx.x >> 5];
+    uint32_t so[kMemberGroup];
 #pragma unroll
     for (uint32_t q = 0; q < kMemberGroup; ++q) {
       const uint32_t e = first + (q < nm ? q : 0);  // surplus slots shadow member 0 (not stored)
       so[q] = (uint32_t)(src.vec(par_b[e]).p - base);
-      oo[q] = (uint32_t)off[e] + lane;
+      if (lane == q) oo[q] = (uint32_t)off[e] + 0u;
     }
+    __syncwarp();
     const uint32_t oj = loc[(uint64_t)p * 32 + lane];
     const uint32_t* mp = mk.p + lane;
     if (nm <= 2)
-      pext_item<2>(mp, base + lane, so, oo, nm, ja, jb, oj, data);
+      pext_item<2>(mp, base + lane, so, oo, nm, ja, jb, oj, data + lane, wbytes);
     else if (nm <= 4)
-      pext_item<4>(mp, base + lane, so, oo, nm, ja, jb, oj, data);
+      pext_item<4>(mp, base + lane, so, oo, nm, ja, jb, oj, data + lane, wbytes);
+    else if (nm <= 6)
+      pext_item<6>(mp, base + lane, so, oo, nm, ja, jb, oj, data + lane, wbytes);
     else
-      pext_item<8>(mp, base + lane, so, oo, nm, ja, jb, oj, data);
+      pext_item<8>(mp, base + lane, so, oo, nm, ja, jb, oj, data + lane, wbytes);
   }
 }
 
@@ -505,7 +525,7 @@ bool proj_build(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const 
       note_launch(); }
     const uint64_t blocks = (T[0] + warps_per_block - 1) / warps_per_block;
     { pext_kernel<<<(unsigned)blocks, kT, 0, s>>>(src, par_a, par_b, bound.p, cmax, W.item_pair.p, item_off.p,
-                                                  (uint32_t)T[0], loc.p, out.off.p, out.data.p); note_launch(); }
+                                                  (uint32_t)T[0], loc.p, out.off.p, out.data.p, 4u); note_launch(); }
   }
   GPA_CUDA(cudaGetLastError());
   if (trace_enabled())
