@@ -343,6 +343,30 @@ def _arr(ptr, n, shape):
     return np.ctypeslib.as_array(ptr, (n,)).copy().reshape(shape)
 
 
+class _ResultOwner:
+    """Owns a gpa_result handle; arrays viewing its memory keep it alive (freed with the last one)."""
+
+    def __init__(self, h):
+        self.h = h
+
+    def __del__(self):
+        if self.h:
+            try:
+                lib().gpa_result_destroy(self.h)
+            except Exception:   # interpreter shutdown
+                pass
+            self.h = None
+
+
+def _view(owner, ptr, n, shape):
+    """Zero-copy uint32 view of library-owned result memory (kept alive through ``owner``)."""
+    if n == 0 or not ptr:
+        return np.zeros(shape, dtype=np.uint32)
+    buf = (ctypes.c_uint32 * n).from_address(ctypes.addressof(ptr.contents))
+    buf._gpa_owner = owner
+    return np.frombuffer(buf, dtype=np.uint32).reshape(shape)
+
+
 def mine(db, items=None, n_items=None, min_count: int = 1, dist: Dist | None = None,
          options: Options | None = None, keep_candidates: bool | None = None) -> MineResult:
     """Level-wise mining with GPU support counting (gpa_mine)."""
@@ -356,6 +380,7 @@ def mine(db, items=None, n_items=None, min_count: int = 1, dist: Dist | None = N
     h = ctypes.c_void_p()
     _check(L.gpa_mine(ctypes.byref(inp.c), int(min_count), dist.h if dist else None, ctypes.byref(copt),
                       ctypes.byref(h)))
+    owner = _ResultOwner(h)   # the result's arrays below are views of its memory (no copy of F)
     try:
         nl = ctypes.c_uint32()
         _check(L.gpa_result_n_levels(h, ctypes.byref(nl)))
@@ -373,10 +398,10 @@ def mine(db, items=None, n_items=None, min_count: int = 1, dist: Dist | None = N
             stats = {f: getattr(st, f) for f, _ in _LevelStats._fields_}
             stats["kernel_name"] = KERNEL_NAMES.get(st.kernel, "?")
             kept = bool(cp)
-            levels.append(Level(k, nc.value, nf.value, _arr(fi, nf.value * k, (nf.value, k)),
-                                _arr(fs, nf.value, (nf.value,)),
-                                _arr(cp, nc.value * k, (nc.value, k)) if kept else None,
-                                _arr(cc, nc.value, (nc.value,)) if kept else None, stats))
+            levels.append(Level(k, nc.value, nf.value, _view(owner, fi, nf.value * k, (nf.value, k)),
+                                _view(owner, fs, nf.value, (nf.value,)),
+                                _view(owner, cp, nc.value * k, (nc.value, k)) if kept else None,
+                                _view(owner, cc, nc.value, (nc.value,)) if kept else None, stats))
         ntx, mc = ctypes.c_uint64(), ctypes.c_uint64()
         _check(L.gpa_result_info(h, ctypes.byref(ntx), ctypes.byref(mc)))
         n_tx = ntx.value
@@ -384,5 +409,5 @@ def mine(db, items=None, n_items=None, min_count: int = 1, dist: Dist | None = N
         _check(L.gpa_result_timing(h, tm))
         timing = {PHASES[i]: tm[i] for i in range(7)}
     finally:
-        L.gpa_result_destroy(h)
+        del owner   # destroyed here unless a level array still views it
     return MineResult(n_tx, int(min_count), levels, timing)
