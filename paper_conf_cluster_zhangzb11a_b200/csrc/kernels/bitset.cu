@@ -25,6 +25,7 @@ constexpr uint32_t kChunkTx = 512;       // transactions per CTA = 16 words (64-
 constexpr uint32_t kChunkWords = kChunkTx / 32;
 constexpr uint32_t kTileStride = 17;     // padded words per tile row (odd: conflict-free columns)
 constexpr uint32_t kRowBlock = 1024;     // rows per CTA tile: 1024 * 17 * 4 = 68 KB -> 3 CTAs / SM
+constexpr uint32_t kSmemRowMap = 1024;   // item -> row map in shared memory up to this many items (3 CTAs / SM)
 
 __global__ void __launch_bounds__(kBuildThreads) bitset_build_kernel(const uint64_t* __restrict__ offsets,
                                                                      const uint32_t* __restrict__ items,
@@ -34,38 +35,48 @@ __global__ void __launch_bounds__(kBuildThreads) bitset_build_kernel(const uint6
                                                                      uint64_t chunk0,
                                                                      uint64_t pitch_words, uint32_t* __restrict__ rows) {
   extern __shared__ uint32_t tile[];
+  __shared__ uint32_t soff[kChunkTx + 1];        // the chunk's offsets, relative to its first item
+  __shared__ int32_t srow[kSmemRowMap];          // row_of_item (n_items <= kSmemRowMap)
   const uint64_t chunk = chunk0 + blockIdx.x;
   const uint32_t rb0 = blockIdx.y * row_block;
   const uint32_t nr = min(row_block, n_rows - rb0);
+  const bool smap = n_items <= kSmemRowMap;
   for (uint32_t i = threadIdx.x; i < nr * kTileStride; i += blockDim.x) tile[i] = 0;
-  __syncthreads();
+  if (smap)
+    for (uint32_t i = threadIdx.x; i < n_items; i += blockDim.x) srow[i] = __ldg(row_of_item + i);
+  // item range of the chunk, clamped so that an invalid CSR (rejected by the validation pass)
+  // never reads past the items or out of the tile
   const uint64_t t0 = chunk * kChunkTx;
-  for (uint32_t tl = threadIdx.x; tl < kChunkTx; tl += blockDim.x) {
-    const uint64_t t = t0 + tl;
-    if (t >= n_tx) break;
-    const uint64_t o0 = __ldg(offsets + t), o1 = __ldg(offsets + t + 1);
-    if (o1 > nnz) continue;  // invalid CSR (rejected by the validation pass); never read past the items
-    const uint32_t bit = 1u << (tl & 31);
-    const uint32_t wcol = tl >> 5;
-    uint64_t j = o0;
-    for (; j + 4 <= o1; j += 4) {  // 4 independent item -> row gathers in flight
-      uint32_t it[4];
-      int32_t r[4];
+  const uint64_t te = t0 < n_tx ? t0 : n_tx;
+  const uint64_t A = min(__ldg(offsets + te), nnz);
+  for (uint32_t i = threadIdx.x; i <= kChunkTx; i += blockDim.x) {
+    const uint64_t t = t0 + i < n_tx ? t0 + i : n_tx;
+    const uint64_t o = min(max(__ldg(offsets + t), A), nnz);
+    soff[i] = (uint32_t)(o - A < 0xffffffffull ? o - A : 0xffffffffull);
+  }
+  __syncthreads();
+  // coalesced sweep over the chunk's items: thread k takes items 4k .. 4k+3 (+ 4 x 256 per round);
+  // the transaction of its first item by binary search in soff, then a forward walk
+  const uint32_t n_it = soff[kChunkTx];
+  for (uint32_t q = threadIdx.x * 4; q < n_it; q += blockDim.x * 4) {
+    uint32_t it[4];
 #pragma unroll
-      for (int u = 0; u < 4; ++u) it[u] = __ldg(items + j + u);
-#pragma unroll
-      for (int u = 0; u < 4; ++u) r[u] = it[u] < n_items ? __ldg(row_of_item + it[u]) : -1;
-#pragma unroll
-      for (int u = 0; u < 4; ++u) {
-        const uint32_t rr = (uint32_t)r[u] - rb0;   // r < 0 wraps to a huge value: skipped
-        if (r[u] >= 0 && rr < nr) atomicOr(&tile[rr * kTileStride + wcol], bit);
-      }
+    for (int u = 0; u < 4; ++u) it[u] = q + u < n_it ? __ldg(items + A + q + u) : 0xffffffffu;
+    uint32_t lo = 0, hi = kChunkTx;  // tx = last with soff[tx] <= q
+    while (lo + 1 < hi) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if (soff[mid] <= q) lo = mid; else hi = mid;
     }
-    for (; j < o1; ++j) {
-      const uint32_t it = __ldg(items + j);
-      const int32_t r = it < n_items ? __ldg(row_of_item + it) : -1;
-      const uint32_t rr = (uint32_t)r - rb0;
-      if (r >= 0 && rr < nr) atomicOr(&tile[rr * kTileStride + wcol], bit);
+    uint32_t tx = lo;
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const uint32_t j = q + u;
+      if (j >= n_it) break;
+      while (tx + 1 < kChunkTx && soff[tx + 1] <= j) ++tx;
+      const uint32_t x = it[u];
+      const int32_t r = x < n_items ? (smap ? srow[x] : __ldg(row_of_item + x)) : -1;
+      const uint32_t rr = (uint32_t)r - rb0;   // r < 0 wraps to a huge value: skipped
+      if (r >= 0 && rr < nr) atomicOr(&tile[rr * kTileStride + (tx >> 5)], 1u << (tx & 31));
     }
   }
   __syncthreads();
