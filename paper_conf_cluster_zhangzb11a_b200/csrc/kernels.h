@@ -158,6 +158,23 @@ DeviceProj* proj_lists(int device);
 bool proj_build(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const DeviceProj* prev,
                 const uint32_t* rows, uint64_t pitch_words, uint32_t n_rows, DeviceProj& out, DeviceScratch& scratch,
                 int n_sms, cudaStream_t s, cudaEvent_t ev_build = nullptr);
+// The same in two stages around one host read of the sizes: begin enqueues the class tables and
+// leaves the totals on the device (pp.d_tot: u64[2] = pext items, list words; pp.d_small: u32[4]),
+// finish (given those values) sizes the lists and launches the list build.
+struct ProjPending {
+  uint32_t n = 0, cmax = 0, nseg = 0, n_pairs = 0;
+  int device = 0;
+  const uint32_t *par_a = nullptr, *par_b = nullptr, *rows = nullptr;
+  const DeviceProj* prev = nullptr;
+  uint64_t pitch = 0;
+  const uint64_t* d_tot = nullptr;
+  const uint32_t* d_small = nullptr;
+};
+void proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const DeviceProj* prev,
+                      const uint32_t* rows, uint64_t pitch_words, uint32_t n_rows, DeviceScratch& scratch, int n_sms,
+                      cudaStream_t s, ProjPending& pp);
+bool proj_build_finish(const ProjPending& pp, const uint64_t T[2], const uint32_t sm[4], DeviceProj& out, int n_sms,
+                       cudaStream_t s, cudaEvent_t ev_build);
 // counts[m] += popc(V_gpar[g] & V_eidx[m]) for every candidate m of group g (counts zeroed by the caller)
 void launch_count_proj(const DeviceProj& P, const uint32_t* gpar, const uint32_t* ext_off, const uint32_t* eidx,
                        uint32_t G, uint32_t* counts, cudaStream_t s);
@@ -169,6 +186,14 @@ void device_exclusive_scan(const uint32_t* in, uint32_t* out, uint32_t n, uint32
                            cudaStream_t s);
 // C_{k+1} = join + prune of L (k >= 2), grouped by k-prefix (synchronises for the sizes).
 void device_candgen(const DeviceLevel& L, DeviceBatch& out, DeviceScratch& scratch, int n_sms, cudaStream_t s);
+// The same in two stages around one host read of the sizes (so that another stage-1 -- the
+// projected lists' class tables -- can share the synchronisation): begin leaves (M, G) at
+// *d_sizes on the device; finish sizes the batch on s and runs the emitting join on `run`
+// (waiting for s through ev when run != s).  begin returns false when |L| < 2 (no candidates).
+bool device_candgen_begin(const DeviceLevel& L, DeviceBatch& out, DeviceScratch& scratch, int n_sms, cudaStream_t s,
+                          const uint32_t** d_sizes);
+void device_candgen_finish(const DeviceLevel& L, DeviceBatch& out, DeviceScratch& scratch, int n_sms, cudaStream_t s,
+                           uint32_t M, uint32_t G, cudaStream_t run, cudaEvent_t ev);
 
 // ---- device-side work planning (plan.cu)
 constexpr uint32_t kPlanMaxRows = 65536;   // row bitmap of the planning kernels (8 KB of shared memory)

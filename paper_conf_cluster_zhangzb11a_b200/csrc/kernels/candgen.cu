@@ -302,11 +302,14 @@ void device_map_items(const uint32_t* rows, uint64_t n, const uint32_t* item_of_
   GPA_CUDA(cudaGetLastError());
 }
 
-void device_candgen(const DeviceLevel& L, DeviceBatch& out, DeviceScratch& scratch, int n_sms, cudaStream_t s) {
+// Stage 1: run detection, hash set, survivor counts and their scans; the sizes (M, G) are left on
+// the device (sizes[0], sizes[1]) -- no synchronisation.  Returns false when L has < 2 members.
+bool device_candgen_begin(const DeviceLevel& L, DeviceBatch& out, DeviceScratch& scratch, int n_sms, cudaStream_t s,
+                          const uint32_t** d_sizes) {
   const uint32_t n = L.n, w = L.k;
   out.k = w + 1;
   out.M = out.G = 0;
-  if (n < 2) return;
+  if (n < 2) return false;
   uint32_t* flags = scratch.u32a(n, s);
   uint32_t* run_ex = scratch.u32b(n, s);
   uint32_t* cnt = scratch.u32c(n, s);
@@ -332,23 +335,44 @@ void device_candgen(const DeviceLevel& L, DeviceBatch& out, DeviceScratch& scrat
   exclusive_scan(cnt, cand_off, n, sizes, scratch, s);
   { nonzero_kernel<<<grid_for(n, n_sms), kThreads, 0, s>>>(cnt, n, gflag); note_launch(); }
   exclusive_scan(gflag, gidx, n, sizes + 1, scratch, s);
-  uint32_t MG[2] = {0, 0};
-  GPA_CUDA(cudaMemcpyAsync(MG, sizes, 8, cudaMemcpyDeviceToHost, s));
-  GPA_CUDA(cudaStreamSynchronize(s));
-  const uint32_t M = MG[0], G = MG[1];
+  *d_sizes = sizes;
+  return true;
+}
+
+// Stage 2 (after the host has read M, G): the output buffers are sized on `s`, the emitting join
+// runs on `run` (which waits for `s` through `ev`; run == s for a single stream).
+void device_candgen_finish(const DeviceLevel& L, DeviceBatch& out, DeviceScratch& scratch, int n_sms, cudaStream_t s,
+                           uint32_t M, uint32_t G, cudaStream_t run, cudaEvent_t ev) {
+  const uint32_t n = L.n, w = L.k;
+  out.M = out.G = 0;
   if (M == 0) return;
   out.prefix.ensure((size_t)G * w, s);
   out.ext_off.ensure(G + 1, s);
   out.ext.ensure(M, s);
   out.gpar.ensure(G, s);
   out.eidx.ensure(M, s);
-  { join_kernel<true><<<grid_for(32ull * n, n_sms), kThreads, 0, s>>>(L.rows.p, n, w, flags, run_ex, bound, slots, cap - 1, cnt,
-                                                            cand_off, gidx, out.prefix.p, out.ext_off.p, out.ext.p,
-                                                            out.gpar.p, out.eidx.p); note_launch(); }
+  if (run != s) {
+    GPA_CUDA(cudaEventRecord(ev, s));
+    GPA_CUDA(cudaStreamWaitEvent(run, ev, 0));
+  }
+  uint32_t cap = 16;
+  while (cap < 2 * n + 1) cap <<= 1;
+  { join_kernel<true><<<grid_for(32ull * n, n_sms), kThreads, 0, run>>>(L.rows.p, n, w, scratch.a.p, scratch.b.p,
+        scratch.d.p, scratch.i.p, cap - 1, scratch.c.p, scratch.e.p, scratch.g.p, out.prefix.p, out.ext_off.p,
+        out.ext.p, out.gpar.p, out.eidx.p); note_launch(); }
   GPA_CUDA(cudaGetLastError());
-  { ext_end_kernel<<<1, 32, 0, s>>>(sizes, out.ext_off.p); note_launch(); }
+  { ext_end_kernel<<<1, 32, 0, run>>>(scratch.h.p, out.ext_off.p); note_launch(); }
   out.M = M;
   out.G = G;
+}
+
+void device_candgen(const DeviceLevel& L, DeviceBatch& out, DeviceScratch& scratch, int n_sms, cudaStream_t s) {
+  const uint32_t* sizes = nullptr;
+  if (!device_candgen_begin(L, out, scratch, n_sms, s, &sizes)) return;
+  uint32_t MG[2] = {0, 0};
+  GPA_CUDA(cudaMemcpyAsync(MG, sizes, 8, cudaMemcpyDeviceToHost, s));
+  GPA_CUDA(cudaStreamSynchronize(s));
+  device_candgen_finish(L, out, scratch, n_sms, s, MG[0], MG[1], s, nullptr);
 }
 
 }  // namespace gpa

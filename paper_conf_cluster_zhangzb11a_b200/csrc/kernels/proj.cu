@@ -424,25 +424,33 @@ ProjWork& work_for(int device) {
 
 DeviceProj* proj_lists(int device) { return work_for(device).lists; }
 
-bool proj_build(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const DeviceProj* prev,
-                const uint32_t* rows, uint64_t pitch_words, uint32_t n_rows, DeviceProj& out, DeviceScratch& scratch,
-                int n_sms, cudaStream_t s, cudaEvent_t ev_build) {
-  out.n = n;
-  out.words = 0;
-  out.in_words = 0;
-  if (n == 0) {
-    if (ev_build) GPA_CUDA(cudaEventRecord(ev_build, s));
-    return true;
-  }
+namespace {
+Src make_src(const ProjPending& pp) {
   Src src{};
-  if (!prev) {
-    src.rows = rows;
-    src.pitch = pitch_words;
+  if (!pp.prev) {
+    src.rows = pp.rows;
+    src.pitch = pp.pitch;
   } else {
-    src.data = prev->data.p;
-    src.off = prev->off.p;
-    src.nw = prev->nw.p;
+    src.data = pp.prev->data.p;
+    src.off = pp.prev->off.p;
+    src.nw = pp.prev->nw.p;
   }
+  return src;
+}
+}  // namespace
+
+void proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const DeviceProj* prev,
+                      const uint32_t* rows, uint64_t pitch_words, uint32_t n_rows, DeviceScratch& scratch, int n_sms,
+                      cudaStream_t s, ProjPending& pp) {
+  pp = ProjPending();
+  pp.n = n;
+  pp.par_a = par_a;
+  pp.par_b = par_b;
+  pp.prev = prev;
+  pp.rows = rows;
+  pp.pitch = pitch_words;
+  if (n == 0) return;
+  const Src src = make_src(pp);
   const uint32_t cmax = prev ? n : std::min(n, n_rows);
   const uint64_t lw_max = prev ? prev->max_lw : pitch_words / 32;
   const uint32_t nseg = (uint32_t)std::max<uint64_t>(1, (lw_max + kSegJ - 1) / kSegJ);
@@ -451,56 +459,53 @@ bool proj_build(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const 
   const uint64_t n_pairs64 = (uint64_t)cmax * nseg;
   GPA_REQUIRE(n_pairs64 * 32 < (1ull << 31), GPA_ERR_INVALID, "proj: too many classes");
   const uint32_t n_pairs = (uint32_t)n_pairs64;
-
-  int device = 0;
-  GPA_CUDA(cudaGetDevice(&device));
-  ProjWork& W = work_for(device);
-  auto& flag = W.flag;
-  auto& ex = W.ex;
-  auto& bound = W.bound;
-  auto& small = W.small;
-  auto& words = W.words;
-  auto& loc = W.loc;
-  auto& items = W.items;
-  auto& item_off = W.item_off;
-  auto& nwc = W.nwc;
-  auto& cls_words = W.cls_words;
-  auto& cls_base = W.cls_base;
-  auto& tot = W.tot;
-  flag.ensure(n);
-  ex.ensure(n);
-  bound.ensure(n + 1);
-  small.ensure(4);
-  GPA_CUDA(cudaMemsetAsync(small.p, 0, 16, s));
-  { cls_flag_kernel<<<grid_for(n, n_sms), kT, 0, s>>>(par_a, n, flag.p); note_launch(); }
-  scan_excl<uint32_t>(flag.p, ex.p, n, scratch, s);
-  { cls_bound_kernel<<<grid_for(n, n_sms), kT, 0, s>>>(flag.p, ex.p, n, bound.p, small.p); note_launch(); }
-  words.ensure((size_t)n_pairs * 32);
-  loc.ensure((size_t)n_pairs * 32);
-  items.ensure(n_pairs);
-  item_off.ensure(n_pairs);
-  nwc.ensure(cmax);
-  cls_words.ensure(cmax);
-  cls_base.ensure(cmax);
-  tot.ensure(2);
-  const unsigned warps_per_block = kT / 32;
-  { seg_popc_kernel<<<(n_pairs + warps_per_block - 1) / warps_per_block, kT, 0, s>>>(
-        src, par_a, bound.p, small.p, cmax, nseg, n_pairs, words.p,
-        reinterpret_cast<unsigned long long*>(small.p + 2)); note_launch(); }
-  { cls_pad_kernel<<<(cmax + warps_per_block - 1) / warps_per_block, kT, 0, s>>>(
-        words.p, bound.p, small.p, cmax, nseg, loc.p, nwc.p, cls_words.p, items.p, small.p + 1); note_launch(); }
-  scan_excl<uint32_t>(items.p, item_off.p, n_pairs, scratch, s);
-  scan_excl<uint64_t>(cls_words.p, cls_base.p, cmax, scratch, s);
-  { proj_totals_kernel<<<1, 32, 0, s>>>(items.p, item_off.p, n_pairs, cls_words.p, cls_base.p, cmax, tot.p);
+  pp.cmax = cmax;
+  pp.nseg = nseg;
+  pp.n_pairs = n_pairs;
+  GPA_CUDA(cudaGetDevice(&pp.device));
+  ProjWork& W = work_for(pp.device);
+  W.flag.ensure(n);
+  W.ex.ensure(n);
+  W.bound.ensure(n + 1);
+  W.small.ensure(4);
+  GPA_CUDA(cudaMemsetAsync(W.small.p, 0, 16, s));
+  { cls_flag_kernel<<<grid_for(n, n_sms), kT, 0, s>>>(par_a, n, W.flag.p); note_launch(); }
+  scan_excl<uint32_t>(W.flag.p, W.ex.p, n, scratch, s);
+  { cls_bound_kernel<<<grid_for(n, n_sms), kT, 0, s>>>(W.flag.p, W.ex.p, n, W.bound.p, W.small.p); note_launch(); }
+  W.words.ensure((size_t)n_pairs * 32);
+  W.loc.ensure((size_t)n_pairs * 32);
+  W.items.ensure(n_pairs);
+  W.item_off.ensure(n_pairs);
+  W.nwc.ensure(cmax);
+  W.cls_words.ensure(cmax);
+  W.cls_base.ensure(cmax);
+  W.tot.ensure(2);
+  const unsigned wpb = kT / 32;
+  { seg_popc_kernel<<<(n_pairs + wpb - 1) / wpb, kT, 0, s>>>(
+        src, par_a, W.bound.p, W.small.p, cmax, nseg, n_pairs, W.words.p,
+        reinterpret_cast<unsigned long long*>(W.small.p + 2)); note_launch(); }
+  { cls_pad_kernel<<<(cmax + wpb - 1) / wpb, kT, 0, s>>>(
+        W.words.p, W.bound.p, W.small.p, cmax, nseg, W.loc.p, W.nwc.p, W.cls_words.p, W.items.p, W.small.p + 1);
     note_launch(); }
+  scan_excl<uint32_t>(W.items.p, W.item_off.p, n_pairs, scratch, s);
+  scan_excl<uint64_t>(W.cls_words.p, W.cls_base.p, cmax, scratch, s);
+  { proj_totals_kernel<<<1, 32, 0, s>>>(W.items.p, W.item_off.p, n_pairs, W.cls_words.p, W.cls_base.p, cmax,
+                                        W.tot.p); note_launch(); }
   GPA_CUDA(cudaGetLastError());
-  uint64_t T[2] = {0, 0};
-  uint32_t sm[4] = {0, 0, 0, 0};
-  GPA_CUDA(cudaMemcpyAsync(T, tot.p, sizeof(T), cudaMemcpyDeviceToHost, s));
-  GPA_CUDA(cudaMemcpyAsync(sm, small.p, sizeof(sm), cudaMemcpyDeviceToHost, s));
-  const double h0 = wall_ms();
-  GPA_CUDA(cudaStreamSynchronize(s));
-  const double h1 = wall_ms();
+  pp.d_tot = W.tot.p;
+  pp.d_small = W.small.p;
+}
+
+bool proj_build_finish(const ProjPending& pp, const uint64_t T[2], const uint32_t sm[4], DeviceProj& out, int n_sms,
+                       cudaStream_t s, cudaEvent_t ev_build) {
+  const uint32_t n = pp.n;
+  out.n = n;
+  out.words = 0;
+  out.in_words = 0;
+  if (n == 0) {
+    if (ev_build) GPA_CUDA(cudaEventRecord(ev_build, s));
+    return true;
+  }
   if (T[0] >= (1ull << 31) || T[1] >= (1ull << 32)) return false;
   try {
     out.data.ensure(T[1]);
@@ -508,30 +513,44 @@ bool proj_build(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const 
     if (e.status != GPA_ERR_OOM) throw;
     return false;  // caller falls back to complete intersection
   }
+  ProjWork& W = work_for(pp.device);
+  const Src src = make_src(pp);
   out.off.ensure(n);
   out.nw.ensure(n);
   out.words = T[1];
   out.max_lw = sm[1];
   out.in_words = (uint64_t)sm[2] | ((uint64_t)sm[3] << 32);
-  const double h2 = wall_ms();
   // lanes shorter than their class' Lw keep a zero tail
   GPA_CUDA(cudaMemsetAsync(out.data.p, 0, std::max<uint64_t>(T[1], 1) * 4, s));
-  { entry_off_kernel<<<grid_for(n, n_sms), kT, 0, s>>>(flag.p, ex.p, bound.p, nwc.p, cls_base.p, n, out.off.p,
-                                                      out.nw.p); note_launch(); }
+  { entry_off_kernel<<<grid_for(n, n_sms), kT, 0, s>>>(W.flag.p, W.ex.p, W.bound.p, W.nwc.p, W.cls_base.p, n,
+                                                      out.off.p, out.nw.p); note_launch(); }
   if (ev_build) GPA_CUDA(cudaEventRecord(ev_build, s));  // start of the list build proper
   if (T[0]) {
     W.item_pair.ensure(T[0]);
-    { item_pair_kernel<<<grid_for(n_pairs, n_sms), kT, 0, s>>>(items.p, item_off.p, n_pairs, W.item_pair.p);
+    { item_pair_kernel<<<grid_for(pp.n_pairs, n_sms), kT, 0, s>>>(W.items.p, W.item_off.p, pp.n_pairs,
+                                                                 W.item_pair.p); note_launch(); }
+    const uint64_t blocks = (T[0] + kT / 32 - 1) / (kT / 32);
+    { pext_kernel<<<(unsigned)blocks, kT, 0, s>>>(src, pp.par_a, pp.par_b, W.bound.p, pp.cmax, W.item_pair.p,
+                                                  W.item_off.p, (uint32_t)T[0], W.loc.p, out.off.p, out.data.p, 4u);
       note_launch(); }
-    const uint64_t blocks = (T[0] + warps_per_block - 1) / warps_per_block;
-    { pext_kernel<<<(unsigned)blocks, kT, 0, s>>>(src, par_a, par_b, bound.p, cmax, W.item_pair.p, item_off.p,
-                                                  (uint32_t)T[0], loc.p, out.off.p, out.data.p, 4u); note_launch(); }
   }
   GPA_CUDA(cudaGetLastError());
-  if (trace_enabled())
-    fprintf(stderr, "[gpa] proj_build n=%u: sync %.2f ms, alloc %.2f ms, launch %.2f ms\n", n, h1 - h0, h2 - h1,
-            wall_ms() - h2);
   return true;
+}
+
+bool proj_build(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const DeviceProj* prev,
+                const uint32_t* rows, uint64_t pitch_words, uint32_t n_rows, DeviceProj& out, DeviceScratch& scratch,
+                int n_sms, cudaStream_t s, cudaEvent_t ev_build) {
+  ProjPending pp;
+  proj_build_begin(n, par_a, par_b, prev, rows, pitch_words, n_rows, scratch, n_sms, s, pp);
+  uint64_t T[2] = {0, 0};
+  uint32_t sm[4] = {0, 0, 0, 0};
+  if (n) {
+    GPA_CUDA(cudaMemcpyAsync(T, pp.d_tot, sizeof(T), cudaMemcpyDeviceToHost, s));
+    GPA_CUDA(cudaMemcpyAsync(sm, pp.d_small, sizeof(sm), cudaMemcpyDeviceToHost, s));
+    GPA_CUDA(cudaStreamSynchronize(s));
+  }
+  return proj_build_finish(pp, T, sm, out, n_sms, s, ev_build);
 }
 
 void launch_count_proj(const DeviceProj& P, const uint32_t* gpar, const uint32_t* ext_off, const uint32_t* eidx,

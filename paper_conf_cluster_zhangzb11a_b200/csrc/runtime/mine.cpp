@@ -9,6 +9,7 @@
 // (P13@474, ">=" per DESIGN.md Q1).  Stops when L_k or C_{k+1} is empty (P13@652).
 #include <algorithm>
 #include <chrono>
+#include <cstring>
 #include <deque>
 
 #include "internal.h"
@@ -84,16 +85,19 @@ void record_level(gpa_result* R, const gpa_bitset* bs, uint32_t k, const Grouped
 }
 
 // Generation k >= 3 on projected vertical lists (proj.cu): the lists of L_{k-1}'s entries from
-// those of L_{k-2} (prev; the bitset rows for k = 3), then one popcount-of-AND per candidate over
-// its parents' lists.  false: the lists do not fit -- nothing counted, use complete intersection.
-bool count_projected(gpa_bitset* bs, uint32_t k, const DeviceLevel& L, const DeviceBatch& B, DeviceProj& prev,
-                     DeviceProj& cur, DeviceScratch& scratch, CountStats* cs) {
+// those of L_{k-2} (the bitset rows for k = 3), then one popcount-of-AND per candidate over its
+// parents' lists.  false: the lists do not fit -- nothing counted, use complete intersection.
+// proj_build_begin shared the generation's one host synchronisation with the join
+// (the sizes T, sm came back with |C_k|): the list build (pext) on s, overlapping the emitting
+// join on the auxiliary stream; the supports wait for both (aux_done).
+bool count_projected_staged(gpa_bitset* bs, uint32_t k, const DeviceBatch& B, DeviceProj& cur, const ProjPending& pp,
+                            const uint64_t T[2], const uint32_t sm[4], cudaEvent_t aux_done, CountStats* cs) {
   cudaStream_t s = bs->stream;
   const double t0 = now_ms();
   GPA_CUDA(cudaEventRecord(cs->e0, s));
-  if (!proj_build(L.n, L.par_a.p, L.par_b.p, k == 3 ? nullptr : &prev, bs->rows.p, bs->pitch_words, bs->n_rows, cur,
-                  scratch, bs->n_sms, s, cs->ep))
-    return false;
+  const bool ok = proj_build_finish(pp, T, sm, cur, bs->n_sms, s, cs->ep);
+  GPA_CUDA(cudaStreamWaitEvent(s, aux_done, 0));
+  if (!ok) return false;
   bs->d_counts.ensure(B.M, s);
   GPA_CUDA(cudaMemsetAsync(bs->d_counts.p, 0, (size_t)B.M * 4, s));
   GPA_CUDA(cudaEventRecord(cs->eb, s));
@@ -103,9 +107,19 @@ bool count_projected(gpa_bitset* bs, uint32_t k, const DeviceLevel& L, const Dev
   cs->launches = 1;
   finish_counts(bs, B.M, cs);
   if (trace_enabled())
-    fprintf(stderr, "[gpa] k=%u proj: %u lists, %.1f MB, host %.2f ms\n", k, L.n, cur.words * 4.0 / 1e6,
+    fprintf(stderr, "[gpa] k=%u proj: %u lists, %.1f MB, host %.2f ms\n", k, pp.n, cur.words * 4.0 / 1e6,
             now_ms() - t0);
   return true;
+}
+
+// A few page-locked words per thread for the per-generation sizes (one D2H read per generation).
+uint32_t* host_sizes() {
+  thread_local struct H {
+    uint32_t* p = nullptr;
+    H() { GPA_CUDA(cudaHostAlloc(reinterpret_cast<void**>(&p), 64, cudaHostAllocDefault)); }
+    ~H() { if (p) cudaFreeHost(p); }
+  } h;
+  return h.p;
 }
 
 // Page-locked staging for the frequent itemsets: each generation's L_k (item ids, supports) is
@@ -238,6 +252,11 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     ~Events() { for (auto x : e) if (x) cudaEventDestroy(x); }
   } copy_evs;
   cudaEvent_t* copy_ev = copy_evs.e;
+  CopyStream aux_s;          // the emitting join of C_k, overlapping the list build on s
+  Events aux_evs;            // [0] s -> aux (batch buffers sized), [1] aux done
+  ProjPending ppend;
+  uint64_t pT[2] = {0, 0};
+  uint32_t psm[4] = {0, 0, 0, 0};
   struct EvTriple {      // deferred timing of a generation's counting launch(es) and all-reduce
     cudaEvent_t e[5] = {nullptr, nullptr, nullptr, nullptr, nullptr};  // + projected-list build [3, 4)
     EvTriple() {
@@ -291,6 +310,25 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
         GPA_CUDA(cudaMemcpyAsync(Bd.ext.p, batch.ext.data(), M * 4, cudaMemcpyHostToDevice, s));
         GPA_CUDA(cudaStreamSynchronize(s));
       }
+    } else if (proj_on) {
+      // join stage 1 and the projected lists' class tables share one synchronisation; then the
+      // emitting join runs on aux_s while the lists are built on s
+      const uint32_t* d_sizes = nullptr;
+      if (device_candgen_begin(Ld, Bd, scratch, bs->n_sms, s, &d_sizes)) {
+        proj_build_begin(Ld.n, Ld.par_a.p, Ld.par_b.p, k == 3 ? nullptr : Pprev, bs->rows.p, bs->pitch_words,
+                         bs->n_rows, scratch, bs->n_sms, s, ppend);
+        uint32_t* hs = host_sizes();
+        GPA_CUDA(cudaMemcpyAsync(hs, d_sizes, 8, cudaMemcpyDeviceToHost, s));
+        GPA_CUDA(cudaMemcpyAsync(hs + 2, ppend.d_tot, 16, cudaMemcpyDeviceToHost, s));
+        GPA_CUDA(cudaMemcpyAsync(hs + 6, ppend.d_small, 16, cudaMemcpyDeviceToHost, s));
+        GPA_CUDA(cudaStreamSynchronize(s));
+        M = hs[0];
+        G = hs[1];
+        std::memcpy(pT, hs + 2, 16);
+        std::memcpy(psm, hs + 6, 16);
+        device_candgen_finish(Ld, Bd, scratch, bs->n_sms, s, (uint32_t)M, (uint32_t)G, aux_s.s, aux_evs.e[0]);
+        GPA_CUDA(cudaEventRecord(aux_evs.e[1], aux_s.s));
+      }
     } else {
       device_candgen(Ld, Bd, scratch, bs->n_sms, s);
       M = Bd.M;
@@ -324,7 +362,7 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
       events.pop_back();
     } else if (k == 2) {
       count_all_pairs(bs, opt.count_kernel, &cs);
-    } else if (proj_on && count_projected(bs, k, Ld, Bd, *Pprev, *Pcur, scratch, &cs)) {
+    } else if (proj_on && count_projected_staged(bs, k, Bd, *Pcur, ppend, pT, psm, aux_evs.e[1], &cs)) {
       std::swap(Pprev, Pcur);
     } else if ((proj_on = false, !count_device_batch(bs, Bd, opt.count_kernel, scratch, &cs))) {
       fetch_batch();
