@@ -32,6 +32,7 @@
 // mask is cut into segments of kSegJ words per lane, each lane padded to whole words per
 // segment, so segments are independent work items.  All integer; counts are exact by construction.
 #include <cstdint>
+#include <cstdlib>
 #include <map>
 #include <cub/block/block_scan.cuh>
 #include <cub/device/device_scan.cuh>
@@ -507,6 +508,10 @@ bool proj_build_finish(const ProjPending& pp, const uint64_t T[2], const uint32_
     return true;
   }
   if (T[0] >= (1ull << 31) || T[1] >= (1ull << 32)) return false;
+  // GPA_PROJ_MAX_MB caps the lists of one generation (tests exercise the mid-run fallback to
+  // complete intersection with it; default: no cap beyond device memory)
+  if (const char* cap = getenv("GPA_PROJ_MAX_MB"))
+    if (T[1] * 4 > (uint64_t)atof(cap) * 1e6) return false;
   try {
     out.data.ensure(T[1]);
   } catch (const Error& e) {

@@ -9,6 +9,7 @@
 // (P13@474, ">=" per DESIGN.md Q1).  Stops when L_k or C_{k+1} is empty (P13@652).
 #include <algorithm>
 #include <chrono>
+#include <cstdlib>
 #include <cstring>
 #include <deque>
 
@@ -95,7 +96,10 @@ bool count_projected_staged(gpa_bitset* bs, uint32_t k, const DeviceBatch& B, De
   cudaStream_t s = bs->stream;
   const double t0 = now_ms();
   GPA_CUDA(cudaEventRecord(cs->e0, s));
-  const bool ok = proj_build_finish(pp, T, sm, cur, bs->n_sms, s, cs->ep);
+  // GPA_PROJ_TEST_MAX_K=k: behave as if the lists of generations > k did not fit (tests drive the
+  // mid-run fallback to complete intersection with it)
+  const char* tk = getenv("GPA_PROJ_TEST_MAX_K");
+  const bool ok = !(tk && k > (uint32_t)atoi(tk)) && proj_build_finish(pp, T, sm, cur, bs->n_sms, s, cs->ep);
   GPA_CUDA(cudaStreamWaitEvent(s, aux_done, 0));
   if (!ok) return false;
   bs->d_counts.ensure(B.M, s);

@@ -370,3 +370,24 @@ def test_c_example_fimi_roundtrip(tmp_path, fig2):
         got[tuple(int(x) for x in items.split())] = int(sup.rstrip(")"))
     ref = oracle.mine_ds(gen.from_lists(txs, 8), 2).frequent()
     assert got == ref
+
+
+# ---------------------------------------------------------------- projected lists: fallback
+
+@pytest.mark.parametrize("how", ["mb0", "k4", "k6"])
+def test_proj_fallback_to_complete_intersection(monkeypatch, how):
+    """When a generation's projected lists do not fit (forced with GPA_PROJ_MAX_MB=0 at generation 3,
+    or GPA_PROJ_TEST_MAX_K after generation 4 / 6), gpa_mine switches to complete intersection for
+    the remaining generations, with every (C_k, count) unchanged."""
+    ds = gen.make("mushroom")
+    theta = oracle.min_count(ds.n_tx, "0.20")
+    ref = oracle.mine_ds(ds, theta)
+    if how == "mb0":
+        monkeypatch.setenv("GPA_PROJ_MAX_MB", "0")
+    else:
+        monkeypatch.setenv("GPA_PROJ_TEST_MAX_K", how[1:])
+    res = gpa.mine(ds, min_count=theta, keep_candidates=True)
+    assert_mine_equal(res, ref)
+    kinds = {lv.k: lv.stats["kernel_name"] for lv in res.levels[2:]}
+    last = 2 if how == "mb0" else int(how[1:])
+    assert all((kinds[k] == "proj") == (k <= last) for k in kinds), kinds
