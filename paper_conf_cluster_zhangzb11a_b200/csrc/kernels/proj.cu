@@ -391,10 +391,10 @@ __global__ void __launch_bounds__(kT) count_proj_kernel(const uint32_t* __restri
 }
 
 template <class T>
-void scan_excl(const T* in, T* out, uint32_t n, DeviceScratch& scratch, cudaStream_t s) {
+void scan_excl(const T* in, T* out, uint32_t n, PBuf<uint8_t>& tmpbuf, cudaStream_t s) {
   size_t bytes = 0;
   GPA_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, bytes, in, out, n, s));
-  void* tmp = scratch.get(bytes, s);
+  void* tmp = tmpbuf.ensure(bytes);
   GPA_CUDA(cub::DeviceScan::ExclusiveSum(tmp, bytes, in, out, n, s));
   note_launch(2);
 }
@@ -414,6 +414,7 @@ __global__ void proj_totals_kernel(const uint32_t* __restrict__ items, const uin
 struct ProjWork {
   PBuf<uint32_t> flag, ex, bound, small, words, loc, items, item_off, item_pair, nwc;
   PBuf<uint64_t> cls_words, cls_base, tot;
+  PBuf<uint8_t> tmp;   // CUB temporary storage of its own: proj_build_begin may run beside the join's scans
   DeviceProj lists[2];
 };
 ProjWork& work_for(int device) {
@@ -471,7 +472,7 @@ void proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, 
   W.small.ensure(4);
   GPA_CUDA(cudaMemsetAsync(W.small.p, 0, 16, s));
   { cls_flag_kernel<<<grid_for(n, n_sms), kT, 0, s>>>(par_a, n, W.flag.p); note_launch(); }
-  scan_excl<uint32_t>(W.flag.p, W.ex.p, n, scratch, s);
+  scan_excl<uint32_t>(W.flag.p, W.ex.p, n, W.tmp, s);
   { cls_bound_kernel<<<grid_for(n, n_sms), kT, 0, s>>>(W.flag.p, W.ex.p, n, W.bound.p, W.small.p); note_launch(); }
   W.words.ensure((size_t)n_pairs * 32);
   W.loc.ensure((size_t)n_pairs * 32);
@@ -488,8 +489,8 @@ void proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, 
   { cls_pad_kernel<<<(cmax + wpb - 1) / wpb, kT, 0, s>>>(
         W.words.p, W.bound.p, W.small.p, cmax, nseg, W.loc.p, W.nwc.p, W.cls_words.p, W.items.p, W.small.p + 1);
     note_launch(); }
-  scan_excl<uint32_t>(W.items.p, W.item_off.p, n_pairs, scratch, s);
-  scan_excl<uint64_t>(W.cls_words.p, W.cls_base.p, cmax, scratch, s);
+  scan_excl<uint32_t>(W.items.p, W.item_off.p, n_pairs, W.tmp, s);
+  scan_excl<uint64_t>(W.cls_words.p, W.cls_base.p, cmax, W.tmp, s);
   { proj_totals_kernel<<<1, 32, 0, s>>>(W.items.p, W.item_off.p, n_pairs, W.cls_words.p, W.cls_base.p, cmax,
                                         W.tot.p); note_launch(); }
   GPA_CUDA(cudaGetLastError());

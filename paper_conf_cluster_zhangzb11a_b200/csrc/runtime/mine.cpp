@@ -318,14 +318,18 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
       // join stage 1 and the projected lists' class tables share one synchronisation; then the
       // emitting join runs on aux_s while the lists are built on s
       const uint32_t* d_sizes = nullptr;
+      // the class tables (aux_s) are independent of the join's stage 1 (s): both read L_{k-1}
+      GPA_CUDA(cudaEventRecord(aux_evs.e[2], s));
+      GPA_CUDA(cudaStreamWaitEvent(aux_s.s, aux_evs.e[2], 0));
       if (device_candgen_begin(Ld, Bd, scratch, bs->n_sms, s, &d_sizes)) {
         proj_build_begin(Ld.n, Ld.par_a.p, Ld.par_b.p, k == 3 ? nullptr : Pprev, bs->rows.p, bs->pitch_words,
-                         bs->n_rows, scratch, bs->n_sms, s, ppend);
+                         bs->n_rows, scratch, bs->n_sms, aux_s.s, ppend);
         uint32_t* hs = host_sizes();
         GPA_CUDA(cudaMemcpyAsync(hs, d_sizes, 8, cudaMemcpyDeviceToHost, s));
-        GPA_CUDA(cudaMemcpyAsync(hs + 2, ppend.d_tot, 16, cudaMemcpyDeviceToHost, s));
-        GPA_CUDA(cudaMemcpyAsync(hs + 6, ppend.d_small, 16, cudaMemcpyDeviceToHost, s));
+        GPA_CUDA(cudaMemcpyAsync(hs + 2, ppend.d_tot, 16, cudaMemcpyDeviceToHost, aux_s.s));
+        GPA_CUDA(cudaMemcpyAsync(hs + 6, ppend.d_small, 16, cudaMemcpyDeviceToHost, aux_s.s));
         GPA_CUDA(cudaStreamSynchronize(s));
+        GPA_CUDA(cudaStreamSynchronize(aux_s.s));
         M = hs[0];
         G = hs[1];
         std::memcpy(pT, hs + 2, 16);
