@@ -370,11 +370,18 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
       events.pop_back();
     } else if (k == 2) {
       count_all_pairs(bs, opt.count_kernel, &cs);
-    } else if (proj_on && count_projected_staged(bs, k, Bd, *Pcur, ppend, pT, psm, aux_evs.e[1], &cs)) {
-      std::swap(Pprev, Pcur);
-    } else if ((proj_on = false, !count_device_batch(bs, Bd, opt.count_kernel, scratch, &cs))) {
-      fetch_batch();
-      count_grouped(bs, batch, opt.count_kernel, &cs);
+    } else {
+      if (proj_on && count_projected_staged(bs, k, Bd, *Pcur, ppend, pT, psm, aux_evs.e[1], &cs)) {
+        std::swap(Pprev, Pcur);
+      } else {
+        // complete intersection from the static bitset (requested, or the projected lists did not
+        // fit: from here on for the remaining generations)
+        proj_on = false;
+        if (!count_device_batch(bs, Bd, opt.count_kernel, scratch, &cs)) {
+          fetch_batch();
+          count_grouped(bs, batch, opt.count_kernel, &cs);
+        }
+      }
     }
     if (keep && k > 2) fetch_batch();
     double t2 = now_ms();
