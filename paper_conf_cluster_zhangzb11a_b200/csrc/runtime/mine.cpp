@@ -234,6 +234,8 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
   bool proj_on = !host_candgen && (opt.count_kernel == GPA_KERNEL_AUTO || opt.count_kernel == GPA_KERNEL_PROJ ||
                                    opt.count_kernel == GPA_KERNEL_PAIRS || opt.count_kernel == GPA_KERNEL_PAIRS_TC) &&
                  bs->pitch_words * 32ull < (1ull << 32);
+  if (const char* e = getenv("GPA_PROJ"))   // GPA_PROJ=0: complete intersection for k >= 3 under AUTO (comparisons)
+    if (atoi(e) == 0 && opt.count_kernel != GPA_KERNEL_PROJ) proj_on = false;
   struct Pending {       // a generation's frequent itemsets, still on the device
     size_t level = 0;
     uint32_t F = 0, k = 0;
