@@ -19,7 +19,7 @@
 // whose transactions are the set bits of V_{Q u {a}}; hence V_{X'} = the bits of V_{Q u {b}} at
 // the set positions of V_{Q u {a}}: a parallel bit extract, pext(V_{Q u {b}}, V_{Q u {a}}),
 // word by word (pext_kernel; Hacker's Delight "compress", the mask-dependent half computed once
-// per mask word and shared by every member of the class).  Generation 3 starts from the static
+// per mask word and shared by a warp's group of up to 8 members of the class).  Generation 3 starts from the static
 // bitset itself: the class of a pair {a, b} is {a}, mask = row a, sources = rows b (the "static
 // bitset" of P2@270 / P18@755 stays the only input).
 //
@@ -29,12 +29,11 @@
 // touches lane l: every load is a coalesced 128-byte row, no cross-lane bit placement.  The
 // members of a class share one mask, hence one per-lane bit count and one layout: Lw_c = max
 // over lanes of the lane's words (each lane's tail zero-padded), members contiguous.  A bitset
-// mask is cut into segments of kSegJ words per lane, each lane padded to whole words per
-// segment, so segments are independent work items.  All integer; counts are exact by construction.
+// mask is cut into segments of kSegJ words per lane (every level), each lane padded to whole words
+// per segment, so segments are independent work items.  All integer; counts are exact by construction.
 #include <cstdint>
 #include <cstdlib>
 #include <map>
-#include <cub/block/block_scan.cuh>
 #include <cub/device/device_scan.cuh>
 
 #include "../common.h"
