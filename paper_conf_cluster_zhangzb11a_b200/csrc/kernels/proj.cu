@@ -208,7 +208,7 @@ __device__ __forceinline__ uint32_t hd_apply(uint32_t x, uint32_t m0, const uint
   return y;
 }
 
-// One item of pext_kernel for a group of nm <= G members (G = 2, 4, 6, 8: the unrolled width, so
+// One item of pext_kernel for a group of nm <= G members (G = 2, 3, 4, 6, 8: the unrolled width, so
 // a class of 2 members does not pay for 8): lane l walks its mask words [ja, jb) and appends, for
 // every member, pext(source word, mask word) to the member's lane-l stream -- a 32-bit
 // accumulator, whole words stored as they fill, the last partial word at the segment's end.
@@ -330,6 +330,8 @@ __global__ void __launch_bounds__(kT, 4) pext_kernel(Src src, const uint32_t* __
     const uint32_t* mp = mk.p + lane;
     if (nm <= 2)
       pext_item<2>(mp, base + lane, so, oo, nm, ja, jb, oj, data + lane, wbytes);
+    else if (nm == 3)
+      pext_item<3>(mp, base + lane, so, oo, nm, ja, jb, oj, data + lane, wbytes);
     else if (nm <= 4)
       pext_item<4>(mp, base + lane, so, oo, nm, ja, jb, oj, data + lane, wbytes);
     else if (nm <= 6)
