@@ -260,6 +260,30 @@ gpa_status gpa_result_timing(const gpa_result* r, double ms_by_phase[GPA_PHASE_C
 
 gpa_status gpa_result_destroy(gpa_result* r);
 
+/* ------------------------------------------------------------------ association rules (f4) */
+
+/*
+ * Association rules from a mining result -- the downstream use of frequent itemsets that the paper
+ * motivates (P4@338-720, "people who buy vegetables often also buy salad dressing"); the paper
+ * does not define them, the reading (Q19) is Agrawal & Srikant's (ref [2], P28@1007):
+ * for every frequent X with |X| >= 2 and every non-empty proper subset A of X, the rule
+ * A => X \ A is reported iff  supp(X) / supp(A) >= conf_num / conf_den, decided exactly as
+ * supp(X) * conf_den >= conf_num * supp(A) (64-bit integers).  Computed on the current CUDA device.
+ *
+ * Rule j: X = itemset number itemset[j] of the result (the index of gpa_result_get, canonical
+ * order), antecedent A = the items of X whose bit is set in antecedent_mask[j] (bit q = X's q-th
+ * item), consequent = the others; support of the rule = supp(X), antecedent_support[j] = supp(A).
+ * Rules come ordered by itemset index, then by mask.  Errors: GPA_ERR_INVALID (NULL, conf_den == 0),
+ * GPA_ERR_RANGE (an itemset longer than GPA_RULES_MAX_K, or more than 2^32 rules).  The arrays are
+ * owned by the gpa_rules handle (valid until gpa_rules_destroy; the result may be destroyed first).
+ */
+#define GPA_RULES_MAX_K 20u
+typedef struct gpa_rules gpa_rules;
+gpa_status gpa_rules_create(const gpa_result* r, uint64_t conf_num, uint64_t conf_den, gpa_rules** out);
+gpa_status gpa_rules_arrays(const gpa_rules* rules, uint64_t* n_rules, const uint32_t** itemset,
+                            const uint32_t** antecedent_mask, const uint32_t** antecedent_support);
+gpa_status gpa_rules_destroy(gpa_rules* rules);
+
 #ifdef __cplusplus
 }
 #endif

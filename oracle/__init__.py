@@ -188,3 +188,22 @@ def candgen(L: np.ndarray, prune: bool = True) -> np.ndarray:
     out = np.ctypeslib.as_array(cp, (max(m * k, 1),))[: m * k].copy().reshape(m, k) if m else np.zeros((0, k), np.uint32)
     ctypes.CDLL(None).free(ctypes.cast(cp, ctypes.c_void_p))
     return out
+
+
+def rules(F: dict, minconf) -> dict:
+    """Association rules from F ({itemset tuple: support}) by their definition (Q19,
+    Agrawal & Srikant ref [2]): for every X in F with |X| >= 2 and every non-empty proper subset A
+    of X, A => X \\ A when supp(X) / supp(A) >= minconf, compared exactly (Fraction).  Plain Python,
+    for small F.  Returns {(A, X \\ A): (supp(X), supp(A))}."""
+    from itertools import combinations
+    mc = Fraction(str(minconf)) if not isinstance(minconf, Fraction) else minconf
+    out = {}
+    for X, sx in F.items():
+        if len(X) < 2:
+            continue
+        for r in range(1, len(X)):
+            for A in combinations(X, r):
+                sa = F[A]
+                if Fraction(sx, sa) >= mc:
+                    out[(A, tuple(v for v in X if v not in A))] = (sx, sa)
+    return out

@@ -26,7 +26,7 @@ from fractions import Fraction
 import numpy as np
 
 __all__ = [
-    "GpaError", "lib", "version", "min_count", "Options", "Dist", "Bitset", "mine", "MineResult",
+    "GpaError", "lib", "version", "min_count", "Options", "Dist", "Bitset", "mine", "MineResult", "Rules",
     "KERNEL_AUTO", "KERNEL_V0", "KERNEL_PREFIX", "KERNEL_PAIRS", "KERNEL_TRIE", "KERNEL_PAIRS_TC", "KERNEL_PROJ", "PHASES",
 ]
 
@@ -107,6 +107,9 @@ def lib() -> ctypes.CDLL:
         "gpa_result_level_stats": (ctypes.c_int, [vp, u32, P(_LevelStats)]),
         "gpa_result_timing": (ctypes.c_int, [vp, ctypes.c_double * 7]),
         "gpa_result_destroy": (ctypes.c_int, [vp]),
+        "gpa_rules_create": (ctypes.c_int, [vp, u64, u64, P(vp)]),
+        "gpa_rules_arrays": (ctypes.c_int, [vp, P(u64), P(P(u32)), P(P(u32)), P(P(u32))]),
+        "gpa_rules_destroy": (ctypes.c_int, [vp]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)
@@ -309,6 +312,25 @@ class MineResult:
     min_count: int
     levels: list
     timing_ms: dict
+    _owner: object = None   # the library's result handle (kept for rules())
+
+    def rules(self, minconf: str | Fraction | float = "0.5") -> "Rules":
+        """Association rules A => X \\ A with supp(X) / supp(A) >= minconf (gpa_rules_create; exact
+        rational comparison: minconf is parsed as a decimal string / Fraction)."""
+        f = Fraction(str(minconf)) if not isinstance(minconf, Fraction) else minconf
+        L = lib()
+        h = ctypes.c_void_p()
+        _check(L.gpa_rules_create(self._owner.h, f.numerator, f.denominator, ctypes.byref(h)))
+        try:
+            n = ctypes.c_uint64()
+            px, pm, ps = (ctypes.POINTER(ctypes.c_uint32)() for _ in range(3))
+            _check(L.gpa_rules_arrays(h, ctypes.byref(n), ctypes.byref(px), ctypes.byref(pm), ctypes.byref(ps)))
+            x = _arr(px, n.value, (n.value,))
+            m = _arr(pm, n.value, (n.value,))
+            sa = _arr(ps, n.value, (n.value,))
+        finally:
+            L.gpa_rules_destroy(h)
+        return Rules(self, x, m, sa)
 
     def frequent(self, k: int | None = None):
         """F as {itemset tuple: support} (k=None), or the (items, supports) arrays of F_k."""
@@ -335,6 +357,32 @@ class MineResult:
     @property
     def count_ms(self) -> float:
         return sum(lv.stats.get("count_ms", 0.0) for lv in self.levels[1:])
+
+
+@dataclass
+class Rules:
+    """Association rules of a MineResult: rule j is (X = itemset number itemset[j] in canonical
+    order, antecedent = X's items selected by the bits of antecedent_mask[j], supp(A) =
+    antecedent_support[j])."""
+    result: "MineResult"
+    itemset: np.ndarray
+    antecedent_mask: np.ndarray
+    antecedent_support: np.ndarray
+
+    def __len__(self):
+        return len(self.itemset)
+
+    def as_dict(self) -> dict:
+        """{(antecedent tuple, consequent tuple): (supp(X), supp(A))}."""
+        flat = [(tuple(r), int(s)) for lv in self.result.levels for r, s in zip(lv.freq_items.tolist(),
+                                                                               lv.freq_support.tolist())]
+        out = {}
+        for x, m, sa in zip(self.itemset.tolist(), self.antecedent_mask.tolist(), self.antecedent_support.tolist()):
+            X, sx = flat[x]
+            A = tuple(v for q, v in enumerate(X) if m >> q & 1)
+            B = tuple(v for q, v in enumerate(X) if not m >> q & 1)
+            out[(A, B)] = (sx, sa)
+        return out
 
 
 def _arr(ptr, n, shape):
@@ -408,6 +456,7 @@ def mine(db, items=None, n_items=None, min_count: int = 1, dist: Dist | None = N
         tm = (ctypes.c_double * 7)()
         _check(L.gpa_result_timing(h, tm))
         timing = {PHASES[i]: tm[i] for i in range(7)}
-    finally:
-        del owner   # destroyed here unless a level array still views it
-    return MineResult(n_tx, int(min_count), levels, timing)
+    except BaseException:
+        del owner
+        raise
+    return MineResult(n_tx, int(min_count), levels, timing, owner)

@@ -5,6 +5,7 @@ generators of gen/; expected values come only from oracle/ (or, for the bit layo
 numpy bit-packing written here).  Sizes span several tiles / stripes plus ragged tails.
 """
 import os
+from fractions import Fraction
 from itertools import combinations
 
 import numpy as np
@@ -391,3 +392,39 @@ def test_proj_fallback_to_complete_intersection(monkeypatch, how):
     kinds = {lv.k: lv.stats["kernel_name"] for lv in res.levels[2:]}
     last = 2 if how == "mb0" else int(how[1:])
     assert all((kinds[k] == "proj") == (k <= last) for k in kinds), kinds
+
+
+# ---------------------------------------------------------------- association rules (f4)
+
+@pytest.mark.parametrize("name,minconf", [("fig2", "0.5"), ("fig2", "1"), ("chess", "0.95"), ("mushroom", "0.8"),
+                                          ("random", "0.3"), ("replicated", "1")])
+def test_rules_vs_oracle(fig2, name, minconf):
+    """gpa_rules_create on the device vs the definition (oracle.rules) on the same F: every rule,
+    supp(X) and supp(A) identical."""
+    if name == "fig2":
+        ds, theta = gen.from_lists(fig2[0], 8), 2
+    elif name == "random":
+        ds = gen.random_db(7, 3000, 24, max_len=12)
+        theta = 60
+    elif name == "replicated":
+        ds, theta = gen.from_lists([[0, 3, 4, 7, 9, 10, 12, 15]] * 40, 16), 40
+    else:
+        ds = gen.make(name)
+        theta = oracle.min_count(ds.n_tx, gen.CONFIGS[name].minsup)
+    res = gpa.mine(ds, min_count=theta)
+    F = res.frequent()
+    assert F == oracle.mine_ds(ds, theta).frequent()
+    got = res.rules(minconf).as_dict()
+    want = oracle.rules(F, minconf)
+    assert got == want
+    if name == "replicated":
+        assert len(got) == 3 ** 8 - 2 ** 9 + 1
+
+
+def test_rules_errors_and_empty():
+    ds = gen.random_db(8, 500, 12, max_len=5)
+    res = gpa.mine(ds, min_count=10 ** 6)   # nothing frequent
+    assert len(res.rules("0.5")) == 0
+    res = gpa.mine(ds, min_count=20)
+    with pytest.raises(gpa.GpaError):
+        res.rules(Fraction(1, 2 ** 33))   # conf_den >= 2^32

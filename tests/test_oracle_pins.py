@@ -235,3 +235,37 @@ def test_shard_invariance():
         parts = [gen.subset(d, a, b) for a, b in ((0, 512), (512, 4096), (4096, d.n_tx))]
         tot = sum(oracle.support_batch(p.offsets, p.items, p.n_items, lv.cand).astype(np.int64) for p in parts)
         assert np.array_equal(tot, lv.count.astype(np.int64))
+
+
+# ---------------------------------------------------------------- association rules (f4, Q19)
+
+def test_rules_fig2_confidences(fig2):
+    """Fig. 2 database at theta = 2: {1} => {3} has confidence supp{1,3} / supp{1} = 2/2, {3} => {1}
+    2/4 (supports printed in Fig. 2, P13@2637-2860)."""
+    txs, _ = fig2
+    ds = gen.from_lists(txs, 8)
+    F = oracle.mine_ds(ds, 2).frequent()
+    r1 = oracle.rules(F, "1")
+    assert r1[((1,), (3,))] == (2, 2)
+    assert ((3,), (1,)) not in r1
+    r5 = oracle.rules(F, "0.5")
+    assert r5[((3,), (1,))] == (2, 4)
+    assert all(Fraction(sx, sa) >= Fraction(1, 2) for sx, sa in r5.values())
+    # every rule's antecedent and consequent partition a frequent itemset
+    for (A, B), (sx, sa) in r5.items():
+        X = tuple(sorted(A + B))
+        assert F[X] == sx and F[A] == sa and not set(A) & set(B)
+
+
+def test_rules_closed_forms():
+    """Replicated transaction T (|T| = L, N copies): every rule has confidence 1, so at any minconf
+    <= 1 there are sum_{k>=2} C(L, k)(2^k - 2) = 3^L - 2^(L+1) + 1 of them; minconf 0 keeps all
+    sum_X (2^|X| - 2) candidates on any F; minconf above 1 keeps none."""
+    L = 6
+    ds = gen.from_lists([list(range(2, 2 + L))] * 50, 12)
+    F = oracle.mine_ds(ds, 50).frequent()
+    assert len(oracle.rules(F, "1")) == 3 ** L - 2 ** (L + 1) + 1
+    ds = gen.random_db(3, 200, 10, max_len=6)
+    F = oracle.mine_ds(ds, 5).frequent()
+    assert len(oracle.rules(F, "0")) == sum(2 ** len(X) - 2 for X in F if len(X) >= 2)
+    assert len(oracle.rules(F, "1.01")) == 0
