@@ -46,6 +46,7 @@ def parse():
     p.add_argument("--config", default="t40i10d10m", choices=list(gen.CONFIGS))
     p.add_argument("--kernel", default="auto", choices=["auto", "v0", "prefix", "pairs", "trie", "pairs_tc", "proj"])
     p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--no-rules", action="store_true", help="skip the association-rules measurement")
     p.add_argument("--dist", action="store_true", help="use the NCCL path even with one rank")
     p.add_argument("--all-configs", action="store_true",
                    help="table of every BASELINE.json config (GPU mine time vs the oracle); not a bench line")
@@ -396,6 +397,20 @@ def main():
         e2e = {"value": cand_tx / (e2e_ms * 1e-3), "unit": "cand*tx/s", "ms_per_step": e2e_ms,
                "h2d_bytes_per_step": h2d * world, "d2h_bytes_per_step": d2h}
 
+    # ---- association rules from this pass's F (outside the timed mining region): wall time
+    # of gpa_rules_create (F to the device, enumeration, rules back to the host)
+    rules = None
+    if rank == 0 and not args.no_rules:
+        minconf = "0.9"
+        res.rules(minconf)   # warm-up
+        torch.cuda.synchronize()
+        tr0 = time.perf_counter()
+        rl = res.rules(minconf)
+        tr = (time.perf_counter() - tr0) * 1e3
+        tested = sum(lv.n_freq * (2 ** lv.k - 2) for lv in res.levels[1:])
+        rules = {"minconf": minconf, "n_rules": len(rl), "antecedents_tested": tested, "ms": tr,
+                 "antecedents_per_s": tested / (tr * 1e-3)}
+
     # ---- CPU baseline: the oracle on a bounded sample (rank 0, N = 1 only)
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -426,6 +441,7 @@ def main():
             "roofline": roof,
             "roofline_by_kernel": roof_all,
             "cpu_baseline": cpu,
+            "rules": rules,
             "e2e": e2e,
             "gpu_launches": launches,
             "clocks": clk,

@@ -190,15 +190,16 @@ def candgen(L: np.ndarray, prune: bool = True) -> np.ndarray:
     return out
 
 
-def rules(F: dict, minconf) -> dict:
+def rules(F: dict, minconf, itemsets=None) -> dict:
     """Association rules from F ({itemset tuple: support}) by their definition (Q19,
     Agrawal & Srikant ref [2]): for every X in F with |X| >= 2 and every non-empty proper subset A
     of X, A => X \\ A when supp(X) / supp(A) >= minconf, compared exactly (Fraction).  Plain Python,
-    for small F.  Returns {(A, X \\ A): (supp(X), supp(A))}."""
+    for small F (or a few ``itemsets`` X of a large F).  Returns {(A, X \\ A): (supp(X), supp(A))}."""
     from itertools import combinations
     mc = Fraction(str(minconf)) if not isinstance(minconf, Fraction) else minconf
     out = {}
-    for X, sx in F.items():
+    for X in (F if itemsets is None else itemsets):
+        sx = F[X]
         if len(X) < 2:
             continue
         for r in range(1, len(X)):

@@ -286,6 +286,29 @@ def test_t40i10d10m_full_size_sampled():
         ex = np.array([e for c, e in zip(sample, expect) if len(c) == k], dtype=np.uint64)
         lit = oracle.support_batch(ds.offsets, ds.items, ds.n_items, cs)
         assert np.array_equal(lit, ex), k
+    # association rules at full size (150 M antecedents), a property check (the supports are this
+    # run's, already checked on samples above): for sampled itemsets X, the reported antecedent masks
+    # are exactly those with supp(X) / supp(A) >= 0.9 over F, with supp(A) as in F
+    rules = res.rules("0.9")
+    flat = [tuple(r) for lv in res.levels for r in lv.freq_items.tolist()]
+    first2 = res.levels[0].n_freq
+    pick = np.sort(rng.choice(np.arange(first2, len(flat)), size=300, replace=False))
+    sel = np.isin(rules.itemset, pick)
+    got = {}
+    for x, m, sa in zip(rules.itemset[sel].tolist(), rules.antecedent_mask[sel].tolist(),
+                        rules.antecedent_support[sel].tolist()):
+        got.setdefault(x, {})[m] = sa
+    n_rules = 0
+    for x in pick.tolist():
+        X = flat[x]
+        want = {}
+        for m in range(1, 2 ** len(X) - 1):
+            A = tuple(v for q, v in enumerate(X) if m >> q & 1)
+            if Fraction(F[X], F[A]) >= Fraction(9, 10):
+                want[m] = F[A]
+        assert got.get(x, {}) == want, X
+        n_rules += len(want)
+    assert n_rules > 0
 
 
 def test_nccl_single_rank_dist_matches_local():
