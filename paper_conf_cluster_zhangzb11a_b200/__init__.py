@@ -321,16 +321,12 @@ class MineResult:
         L = lib()
         h = ctypes.c_void_p()
         _check(L.gpa_rules_create(self._owner.h, f.numerator, f.denominator, ctypes.byref(h)))
-        try:
-            n = ctypes.c_uint64()
-            px, pm, ps = (ctypes.POINTER(ctypes.c_uint32)() for _ in range(3))
-            _check(L.gpa_rules_arrays(h, ctypes.byref(n), ctypes.byref(px), ctypes.byref(pm), ctypes.byref(ps)))
-            x = _arr(px, n.value, (n.value,))
-            m = _arr(pm, n.value, (n.value,))
-            sa = _arr(ps, n.value, (n.value,))
-        finally:
-            L.gpa_rules_destroy(h)
-        return Rules(self, x, m, sa)
+        owner = _ResultOwner(h, L.gpa_rules_destroy)   # the arrays below view the rules' memory
+        n = ctypes.c_uint64()
+        px, pm, ps = (ctypes.POINTER(ctypes.c_uint32)() for _ in range(3))
+        _check(L.gpa_rules_arrays(h, ctypes.byref(n), ctypes.byref(px), ctypes.byref(pm), ctypes.byref(ps)))
+        return Rules(self, _view(owner, px, n.value, (n.value,)), _view(owner, pm, n.value, (n.value,)),
+                     _view(owner, ps, n.value, (n.value,)))
 
     def frequent(self, k: int | None = None):
         """F as {itemset tuple: support} (k=None), or the (items, supports) arrays of F_k."""
@@ -392,15 +388,17 @@ def _arr(ptr, n, shape):
 
 
 class _ResultOwner:
-    """Owns a gpa_result handle; arrays viewing its memory keep it alive (freed with the last one)."""
+    """Owns a library handle (gpa_result, or gpa_rules with its destroy function); arrays viewing
+    its memory keep it alive (freed with the last one)."""
 
-    def __init__(self, h):
+    def __init__(self, h, destroy=None):
         self.h = h
+        self.destroy = destroy
 
     def __del__(self):
         if self.h:
             try:
-                lib().gpa_result_destroy(self.h)
+                (self.destroy or lib().gpa_result_destroy)(self.h)
             except Exception:   # interpreter shutdown
                 pass
             self.h = None

@@ -2,6 +2,7 @@
 // asynchronous on `stream`; all device pointers live on the current device.
 #pragma once
 #include <cstdint>
+#include <functional>
 #include <vector>
 #include <cuda_runtime.h>
 
@@ -139,10 +140,11 @@ uint32_t device_threshold(const uint32_t* counts, uint32_t M, uint32_t theta, ui
 // ---- association rules (rules.cu): F as n itemsets in canonical order (items at
 // items + item_off[i], len[i] items, support sup[i]); the rules A => X \ A of the itemsets x0 .. n-1
 // (those with |X| >= 2) with supp(X) * den >= num * supp(A), as (X index, antecedent mask, supp(A))
-// in (X, mask) order.  num, den < 2^32.  Synchronises.
-void device_rules(const uint32_t* items, const uint64_t* item_off, const uint32_t* len, const uint32_t* sup, uint32_t n,
-                  uint32_t x0, uint64_t num, uint64_t den, int n_sms, cudaStream_t s, std::vector<uint32_t>& rx,
-                  std::vector<uint32_t>& rmask, std::vector<uint32_t>& rsupa);
+// in (X, mask) order.  num, den < 2^32.  The rules land in host_alloc(n_rules): 3 x n_rules words
+// (X indices, masks, supports of A).  Returns n_rules.  Synchronises.
+uint64_t device_rules(const uint32_t* items, const uint64_t* item_off, const uint32_t* len, const uint32_t* sup,
+                      uint32_t n, uint32_t x0, uint64_t num, uint64_t den, int n_sms, cudaStream_t s,
+                      const std::function<uint32_t*(uint64_t)>& host_alloc);
 
 // ---- projected vertical lists (proj.cu; "equivalent class clustering", P13@2288-2486)
 // For every entry j of a level L (n entries with parents par_a / par_b): the bits of its last

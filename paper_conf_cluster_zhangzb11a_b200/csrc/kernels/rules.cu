@@ -11,6 +11,8 @@
 // masks 1 .. 2^k - 2 (bit i = X's i-th item in the antecedent), 32 at a time; pass 1 counts the
 // rules of every X, an exclusive scan places them, pass 2 writes them in (X, mask) order.
 #include <cstdint>
+#include <cstdio>
+#include <functional>
 #include <vector>
 
 #include "../common.h"
@@ -131,13 +133,11 @@ unsigned grid_for(uint64_t n, int n_sms) {
 
 }  // namespace
 
-void device_rules(const uint32_t* items, const uint64_t* item_off, const uint32_t* len, const uint32_t* sup, uint32_t n,
-                  uint32_t x0, uint64_t num, uint64_t den, int n_sms, cudaStream_t s, std::vector<uint32_t>& rx,
-                  std::vector<uint32_t>& rmask, std::vector<uint32_t>& rsupa) {
-  rx.clear();
-  rmask.clear();
-  rsupa.clear();
-  if (n == 0 || x0 >= n) return;
+uint64_t device_rules(const uint32_t* items, const uint64_t* item_off, const uint32_t* len, const uint32_t* sup,
+                      uint32_t n, uint32_t x0, uint64_t num, uint64_t den, int n_sms, cudaStream_t s,
+                      const std::function<uint32_t*(uint64_t)>& host_alloc) {
+  if (n == 0 || x0 >= n) return 0;
+  const double t0 = wall_ms();
   const FSet F{items, item_off, len, sup};
   uint32_t cap = 16;
   while (cap < 2 * n + 1) cap <<= 1;
@@ -155,6 +155,7 @@ void device_rules(const uint32_t* items, const uint64_t* item_off, const uint32_
   std::vector<uint32_t> hc(nx);
   GPA_CUDA(cudaMemcpyAsync(hc.data(), cnt.p, (size_t)nx * 4, cudaMemcpyDeviceToHost, s));
   GPA_CUDA(cudaStreamSynchronize(s));
+  const double t1 = wall_ms();
   std::vector<uint64_t> ho(nx);
   uint64_t tot = 0;
   for (uint32_t i = 0; i < nx; ++i) {
@@ -162,10 +163,9 @@ void device_rules(const uint32_t* items, const uint64_t* item_off, const uint32_
     tot += hc[i];
   }
   GPA_REQUIRE(tot < (1ull << 32), GPA_ERR_RANGE, "more than 2^32 rules");
-  rx.resize(tot);
-  rmask.resize(tot);
-  rsupa.resize(tot);
-  if (tot == 0) return;
+  if (tot == 0) return 0;
+  uint32_t* h = host_alloc(tot);   // 3 x tot words: X index, mask, supp(A)
+  const double t2 = wall_ms();
   off.alloc(nx, s);
   GPA_CUDA(cudaMemcpyAsync(off.p, ho.data(), (size_t)nx * 8, cudaMemcpyHostToDevice, s));
   DBuf<uint32_t> ox, om, os;
@@ -175,10 +175,14 @@ void device_rules(const uint32_t* items, const uint64_t* item_off, const uint32_
   { rules_kernel<true><<<grid, kT, 0, s>>>(F, x0, nx, slots.p, cap - 1, num, den, nullptr, off.p, ox.p, om.p, os.p);
     note_launch(); }
   GPA_CUDA(cudaGetLastError());
-  GPA_CUDA(cudaMemcpyAsync(rx.data(), ox.p, tot * 4, cudaMemcpyDeviceToHost, s));
-  GPA_CUDA(cudaMemcpyAsync(rmask.data(), om.p, tot * 4, cudaMemcpyDeviceToHost, s));
-  GPA_CUDA(cudaMemcpyAsync(rsupa.data(), os.p, tot * 4, cudaMemcpyDeviceToHost, s));
+  GPA_CUDA(cudaMemcpyAsync(h, ox.p, tot * 4, cudaMemcpyDeviceToHost, s));
+  GPA_CUDA(cudaMemcpyAsync(h + tot, om.p, tot * 4, cudaMemcpyDeviceToHost, s));
+  GPA_CUDA(cudaMemcpyAsync(h + 2 * tot, os.p, tot * 4, cudaMemcpyDeviceToHost, s));
   GPA_CUDA(cudaStreamSynchronize(s));
+  if (trace_enabled())
+    fprintf(stderr, "[gpa] rules: %u itemsets, %llu rules: hash + count pass %.2f ms, scan + alloc %.2f ms, emit + D2H "
+            "%.2f ms\n", n, (unsigned long long)tot, t1 - t0, t2 - t1, wall_ms() - t2);
+  return tot;
 }
 
 }  // namespace gpa

@@ -1,12 +1,42 @@
 // Association rules from a mining result (gpa_rules_*, Q19): the
 // result's frequent itemsets go to the device once, the rules are enumerated there (rules.cu)
 // and come back as three arrays owned by the gpa_rules handle.
+#include <sys/mman.h>
+
 #include <algorithm>
 
+
 #include "internal.h"
+#include "pool.h"
+
+// Host buffer for the rules (hundreds of MB): anonymous mapping with transparent huge pages, first
+// touched in parallel -- fresh 4 KB pages faulted in one by one by the D2H copy ran at ~2 GB/s.
+struct HostWords {
+  uint32_t* p = nullptr;
+  size_t bytes = 0;
+  ~HostWords() {
+    if (p) munmap(p, bytes);
+  }
+  uint32_t* alloc(uint64_t words) {
+    bytes = std::max<size_t>(words * 4, 4096);
+    void* m = mmap(nullptr, bytes, PROT_READ | PROT_WRITE, MAP_PRIVATE | MAP_ANONYMOUS, -1, 0);
+    GPA_REQUIRE(m != MAP_FAILED, GPA_ERR_OOM, "host allocation of %zu bytes failed", bytes);
+    p = static_cast<uint32_t*>(m);
+#ifdef MADV_HUGEPAGE
+    madvise(m, bytes, MADV_HUGEPAGE);
+#endif
+    const size_t T = std::max<size_t>(1, std::min<size_t>(gpa::pool_threads(), bytes >> 24));
+    auto* c = static_cast<volatile uint8_t*>(m);
+    gpa::parallel_for(T, [&](size_t t) {
+      for (size_t o = bytes * t / T; o < bytes * (t + 1) / T; o += 4096) c[o] = 0;
+    });
+    return p;
+  }
+};
 
 struct gpa_rules {
-  std::vector<uint32_t> itemset, mask, supp_a;
+  HostWords data;   // 3 x n words: X indices, masks, supports of A
+  uint64_t n = 0;
 };
 
 extern "C" gpa_status gpa_rules_create(const gpa_result* r, uint64_t conf_num, uint64_t conf_den, gpa_rules** out) {
@@ -67,8 +97,8 @@ extern "C" gpa_status gpa_rules_create(const gpa_result* r, uint64_t conf_num, u
       GPA_CUDA(cudaMemcpyAsync(d_len.p, len.data(), n * 4, cudaMemcpyHostToDevice, s));
       GPA_CUDA(cudaMemcpyAsync(d_sup.p, sup.data(), n * 4, cudaMemcpyHostToDevice, s));
       GPA_CUDA(cudaMemcpyAsync(d_off.p, off.data(), n * 8, cudaMemcpyHostToDevice, s));
-      device_rules(d_items.p, d_off.p, d_len.p, d_sup.p, (uint32_t)n, (uint32_t)x0, conf_num, conf_den, di.n_sms, s,
-                   R->itemset, R->mask, R->supp_a);
+      R->n = device_rules(d_items.p, d_off.p, d_len.p, d_sup.p, (uint32_t)n, (uint32_t)x0, conf_num, conf_den,
+                          di.n_sms, s, [&](uint64_t m) { return R->data.alloc(3 * m); });
     }
     *out = R;
     g.p = nullptr;
@@ -79,10 +109,11 @@ extern "C" gpa_status gpa_rules_arrays(const gpa_rules* rules, uint64_t* n_rules
                                        const uint32_t** antecedent_mask, const uint32_t** antecedent_support) {
   return gpa::guard([&] {
     GPA_REQUIRE(rules, GPA_ERR_INVALID, "rules is NULL");
-    if (n_rules) *n_rules = rules->itemset.size();
-    if (itemset) *itemset = rules->itemset.data();
-    if (antecedent_mask) *antecedent_mask = rules->mask.data();
-    if (antecedent_support) *antecedent_support = rules->supp_a.data();
+    const uint32_t* d = rules->data.p;
+    if (n_rules) *n_rules = rules->n;
+    if (itemset) *itemset = d;
+    if (antecedent_mask) *antecedent_mask = d ? d + rules->n : nullptr;
+    if (antecedent_support) *antecedent_support = d ? d + 2 * rules->n : nullptr;
   });
 }
 
