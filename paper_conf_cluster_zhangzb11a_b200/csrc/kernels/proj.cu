@@ -223,7 +223,7 @@ __device__ __forceinline__ const uint32_t* addr_of(const uint32_t* base, uint32_
   return r;
 }
 
-template <uint32_t G>
+template <uint32_t G, bool SPARSE>
 __device__ __forceinline__ void pext_item(const uint32_t* __restrict__ mp, const uint32_t* __restrict__ sbase,
                                           const uint32_t (&so)[kMemberGroup], const uint32_t* __restrict__ s_oo,
                                           uint32_t nm, uint32_t ja, uint32_t jb, uint32_t oj,
@@ -251,16 +251,47 @@ __device__ __forceinline__ void pext_item(const uint32_t* __restrict__ mp, const
     mn = __ldg(mp);
 #pragma unroll
     for (uint32_t q = 0; q < G; ++q) xn[q] = __ldg(addr_of(cur, so[q], wbytes));
-    uint32_t mv[5], m0;
-    hd_prep(mw, mv, m0);
     const uint32_t pw = 1u << nb;
-    nb += __popc(mw);
+    const uint32_t c = __popc(mw);
+    nb += c;
+    uint32_t y[G];
+    if constexpr (SPARSE) {
+      // sparse masks (bitset rows, ~5 % set): the mask's trailing ones stay in place; every further
+      // set bit p lands at position i = its rank: bit i of (x >> (p - i)), the shift as an IMAD.HI by
+      // 2^(32 - (p - i)) (p - i >= 1 past the trailing ones) shared by the group -- per member one
+      // IMAD.HI + one LOP3 per set bit; the loop runs to the warp's largest count
+      const uint32_t i0 = mw == 0xffffffffu ? 32u : (uint32_t)__ffs(~mw) - 1u;
+      const uint32_t idm = i0 >= 32 ? 0xffffffffu : (1u << i0) - 1u;
+#pragma unroll
+      for (uint32_t q = 0; q < G; ++q) y[q] = x[q] & idm;
+      uint32_t mm = mw & ~idm, i = i0;
+      const uint32_t T = __reduce_max_sync(0xffffffffu, c - min(i0, c));
+      for (uint32_t t = 0; t < T; ++t) {
+        const bool has = mm != 0;
+        const uint32_t pbit = has ? (uint32_t)__ffs(mm) - 1u : 0u;
+        mm &= mm - 1u;
+        const uint32_t M = has ? 1u << (32u - (pbit - i)) : 0u;
+        const uint32_t bi = has ? 1u << i : 0u;
+#pragma unroll
+        for (uint32_t q = 0; q < G; ++q) {
+          uint32_t r;
+          asm("lop3.b32 %0, %1, %2, %3, 0xF8;" : "=r"(r) : "r"(y[q]), "r"(__umulhi(x[q], M)), "r"(bi));  // y | (t & bi)
+          y[q] = r;
+        }
+        i += has ? 1u : 0u;
+      }
+    } else {
+      uint32_t mv[5], m0;
+      hd_prep(mw, mv, m0);
+#pragma unroll
+      for (uint32_t q = 0; q < G; ++q) y[q] = hd_apply(x[q], m0, mv);
+    }
 #pragma unroll
     for (uint32_t q = 0; q < G; ++q) {
       // append at bit nb: one 32x32->64 multiply by 2^nb (FMA pipe); the low half is disjoint from
       // the bits already in acc, so the OR is an add (FMA pipe as well); x[q] keeps the carry
       uint64_t v;
-      asm("mul.wide.u32 %0, %1, %2;" : "=l"(v) : "r"(hd_apply(x[q], m0, mv)), "r"(pw));
+      asm("mul.wide.u32 %0, %1, %2;" : "=l"(v) : "r"(y[q]), "r"(pw));
       asm("mad.lo.u32 %0, %1, 1, %0;" : "+r"(acc[q]) : "r"((uint32_t)v));
       x[q] = (uint32_t)(v >> 32);
     }
@@ -328,16 +359,24 @@ __global__ void __launch_bounds__(kT, 4) pext_kernel(Src src, const uint32_t* __
     __syncwarp();
     const uint32_t oj = loc[(uint64_t)p * 32 + lane];
     const uint32_t* mp = mk.p + lane;
-    if (nm <= 2)
-      pext_item<2>(mp, base + lane, so, oo, nm, ja, jb, oj, data + lane, wbytes);
-    else if (nm == 3)
-      pext_item<3>(mp, base + lane, so, oo, nm, ja, jb, oj, data + lane, wbytes);
-    else if (nm <= 4)
-      pext_item<4>(mp, base + lane, so, oo, nm, ja, jb, oj, data + lane, wbytes);
-    else if (nm <= 6)
-      pext_item<6>(mp, base + lane, so, oo, nm, ja, jb, oj, data + lane, wbytes);
-    else
-      pext_item<8>(mp, base + lane, so, oo, nm, ja, jb, oj, data + lane, wbytes);
+    if (src.rows) {  // generation 3: sparse bitset rows as masks
+      if (nm <= 2)
+        pext_item<2, true>(mp, base + lane, so, oo, nm, ja, jb, oj, data + lane, wbytes);
+      else if (nm <= 4)
+        pext_item<4, true>(mp, base + lane, so, oo, nm, ja, jb, oj, data + lane, wbytes);
+      else
+        pext_item<8, true>(mp, base + lane, so, oo, nm, ja, jb, oj, data + lane, wbytes);
+    } else if (nm <= 2) {
+      pext_item<2, false>(mp, base + lane, so, oo, nm, ja, jb, oj, data + lane, wbytes);
+    } else if (nm == 3) {
+      pext_item<3, false>(mp, base + lane, so, oo, nm, ja, jb, oj, data + lane, wbytes);
+    } else if (nm <= 4) {
+      pext_item<4, false>(mp, base + lane, so, oo, nm, ja, jb, oj, data + lane, wbytes);
+    } else if (nm <= 6) {
+      pext_item<6, false>(mp, base + lane, so, oo, nm, ja, jb, oj, data + lane, wbytes);
+    } else {
+      pext_item<8, false>(mp, base + lane, so, oo, nm, ja, jb, oj, data + lane, wbytes);
+    }
   }
 }
 

@@ -218,3 +218,32 @@ def test_compress_matches_pext():
     m[2::11] = 0
     m[3::13] = 0x80000001
     assert np.array_equal(_hd_compress(x, m), _pext_ref(x, m))
+
+
+def _sparse_compress(x, m):
+    """The sparse-mask sequence of proj.cu's pext_item<G, true> (generation 3): the mask's trailing
+    ones stay, every further set bit p of rank i comes from bit i of (x >> (p - i)), the shift as
+    umulhi(x, 2^(32 - (p - i)))."""
+    c = bin(m).count("1")
+    i0 = 32 if m == 0xFFFFFFFF else ((~m & 0xFFFFFFFF) & -(~m & 0xFFFFFFFF)).bit_length() - 1
+    idm = 0xFFFFFFFF if i0 >= 32 else (1 << i0) - 1
+    y, mm, i = x & idm, m & ~idm & 0xFFFFFFFF, i0
+    for _ in range(c - min(i0, c)):
+        p = (mm & -mm).bit_length() - 1
+        mm &= mm - 1
+        y |= ((x * (1 << (32 - (p - i)))) >> 32) & (1 << i)
+        i += 1
+    return y
+
+
+def test_sparse_compress_matches_pext():
+    rng = np.random.default_rng(12)
+    xs = rng.integers(0, 2 ** 32, 20000, dtype=np.uint64).tolist()
+    ms = rng.integers(0, 2 ** 32, 20000, dtype=np.uint64)
+    ms[::2] &= rng.integers(0, 2 ** 32, 10000, dtype=np.uint64) & rng.integers(0, 2 ** 32, 10000, dtype=np.uint64)
+    ms[1::9] = 0xFFFFFFFF
+    ms[2::11] = 0
+    ms[3::13] = 0x0000FFFF | 0x80000000
+    ms = ms.tolist()
+    ref = _pext_ref(np.array(xs, dtype=np.uint32), np.array(ms, dtype=np.uint32)).tolist()
+    assert [_sparse_compress(x, m) for x, m in zip(xs, ms)] == ref
