@@ -181,7 +181,9 @@ struct ProjPending {
   const uint64_t* d_tot = nullptr;
   const uint32_t* d_small = nullptr;
 };
-void proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const DeviceProj* prev,
+// begin returns false (nothing enqueued) when the lists cannot be addressed (bitset >= 2^32 words,
+// too many classes): use complete intersection.
+bool proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const DeviceProj* prev,
                       const uint32_t* rows, uint64_t pitch_words, uint32_t n_rows, DeviceScratch& scratch, int n_sms,
                       cudaStream_t s, ProjPending& pp);
 bool proj_build_finish(const ProjPending& pp, const uint64_t T[2], const uint32_t sm[4], DeviceProj& out, int n_sms,

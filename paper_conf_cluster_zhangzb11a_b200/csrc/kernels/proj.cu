@@ -481,7 +481,7 @@ Src make_src(const ProjPending& pp) {
 }
 }  // namespace
 
-void proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const DeviceProj* prev,
+bool proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const DeviceProj* prev,
                       const uint32_t* rows, uint64_t pitch_words, uint32_t n_rows, DeviceScratch& scratch, int n_sms,
                       cudaStream_t s, ProjPending& pp) {
   pp = ProjPending();
@@ -491,15 +491,17 @@ void proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, 
   pp.prev = prev;
   pp.rows = rows;
   pp.pitch = pitch_words;
-  if (n == 0) return;
+  if (n == 0) return true;
   const Src src = make_src(pp);
   const uint32_t cmax = prev ? n : std::min(n, n_rows);
   const uint64_t lw_max = prev ? prev->max_lw : pitch_words / 32;
   const uint32_t nseg = (uint32_t)std::max<uint64_t>(1, (lw_max + kSegJ - 1) / kSegJ);
   // 32-bit word offsets inside pext_kernel
-  GPA_REQUIRE(prev || (uint64_t)n_rows * pitch_words < (1ull << 32), GPA_ERR_INVALID, "proj: bitset too large");
+  // pext_kernel addresses sources with 32-bit word offsets, its tables with 31-bit indices: beyond
+  // that the caller uses complete intersection
+  if (!prev && (uint64_t)n_rows * pitch_words >= (1ull << 32)) return false;
   const uint64_t n_pairs64 = (uint64_t)cmax * nseg;
-  GPA_REQUIRE(n_pairs64 * 32 < (1ull << 31), GPA_ERR_INVALID, "proj: too many classes");
+  if (n_pairs64 * 32 >= (1ull << 31)) return false;
   const uint32_t n_pairs = (uint32_t)n_pairs64;
   pp.cmax = cmax;
   pp.nseg = nseg;
@@ -536,6 +538,7 @@ void proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, 
   GPA_CUDA(cudaGetLastError());
   pp.d_tot = W.tot.p;
   pp.d_small = W.small.p;
+  return true;
 }
 
 bool proj_build_finish(const ProjPending& pp, const uint64_t T[2], const uint32_t sm[4], DeviceProj& out, int n_sms,
@@ -588,7 +591,7 @@ bool proj_build(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const 
                 const uint32_t* rows, uint64_t pitch_words, uint32_t n_rows, DeviceProj& out, DeviceScratch& scratch,
                 int n_sms, cudaStream_t s, cudaEvent_t ev_build) {
   ProjPending pp;
-  proj_build_begin(n, par_a, par_b, prev, rows, pitch_words, n_rows, scratch, n_sms, s, pp);
+  if (!proj_build_begin(n, par_a, par_b, prev, rows, pitch_words, n_rows, scratch, n_sms, s, pp)) return false;
   uint64_t T[2] = {0, 0};
   uint32_t sm[4] = {0, 0, 0, 0};
   if (n) {

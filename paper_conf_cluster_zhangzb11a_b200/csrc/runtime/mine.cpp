@@ -261,6 +261,7 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
   CopyStream aux_s;          // the emitting join of C_k, overlapping the list build on s
   Events aux_evs;            // [0] s -> aux (batch buffers sized), [1] aux done
   ProjPending ppend;
+  bool aux_join = false;     // this generation's batch was emitted on aux_s
   uint64_t pT[2] = {0, 0};
   uint32_t psm[4] = {0, 0, 0, 0};
   struct EvTriple {      // deferred timing of a generation's counting launch(es) and all-reduce
@@ -317,6 +318,7 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
         GPA_CUDA(cudaStreamSynchronize(s));
       }
     } else if (proj_on) {
+      aux_join = false;
       // join stage 1 and the projected lists' class tables share one synchronisation; then the
       // emitting join runs on aux_s while the lists are built on s
       const uint32_t* d_sizes = nullptr;
@@ -324,12 +326,15 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
       GPA_CUDA(cudaEventRecord(aux_evs.e[2], s));
       GPA_CUDA(cudaStreamWaitEvent(aux_s.s, aux_evs.e[2], 0));
       if (device_candgen_begin(Ld, Bd, scratch, bs->n_sms, s, &d_sizes)) {
-        proj_build_begin(Ld.n, Ld.par_a.p, Ld.par_b.p, k == 3 ? nullptr : Pprev, bs->rows.p, bs->pitch_words,
-                         bs->n_rows, scratch, bs->n_sms, aux_s.s, ppend);
         uint32_t* hs = host_sizes();
+        if (proj_build_begin(Ld.n, Ld.par_a.p, Ld.par_b.p, k == 3 ? nullptr : Pprev, bs->rows.p, bs->pitch_words,
+                             bs->n_rows, scratch, bs->n_sms, aux_s.s, ppend)) {
+          GPA_CUDA(cudaMemcpyAsync(hs + 2, ppend.d_tot, 16, cudaMemcpyDeviceToHost, aux_s.s));
+          GPA_CUDA(cudaMemcpyAsync(hs + 6, ppend.d_small, 16, cudaMemcpyDeviceToHost, aux_s.s));
+        } else {
+          proj_on = false;   // lists not addressable: complete intersection from this generation on
+        }
         GPA_CUDA(cudaMemcpyAsync(hs, d_sizes, 8, cudaMemcpyDeviceToHost, s));
-        GPA_CUDA(cudaMemcpyAsync(hs + 2, ppend.d_tot, 16, cudaMemcpyDeviceToHost, aux_s.s));
-        GPA_CUDA(cudaMemcpyAsync(hs + 6, ppend.d_small, 16, cudaMemcpyDeviceToHost, aux_s.s));
         GPA_CUDA(cudaStreamSynchronize(s));
         GPA_CUDA(cudaStreamSynchronize(aux_s.s));
         M = hs[0];
@@ -338,6 +343,7 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
         std::memcpy(psm, hs + 6, 16);
         device_candgen_finish(Ld, Bd, scratch, bs->n_sms, s, (uint32_t)M, (uint32_t)G, aux_s.s, aux_evs.e[0]);
         GPA_CUDA(cudaEventRecord(aux_evs.e[1], aux_s.s));
+        aux_join = true;
       }
     } else {
       device_candgen(Ld, Bd, scratch, bs->n_sms, s);
@@ -379,6 +385,7 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
         // complete intersection from the static bitset (requested, or the projected lists did not
         // fit: from here on for the remaining generations)
         proj_on = false;
+        if (aux_join) GPA_CUDA(cudaStreamWaitEvent(s, aux_evs.e[1], 0));  // the batch came from aux_s
         if (!count_device_batch(bs, Bd, opt.count_kernel, scratch, &cs)) {
           fetch_batch();
           count_grouped(bs, batch, opt.count_kernel, &cs);
