@@ -381,18 +381,24 @@ __global__ void __launch_bounds__(kT, 4) pext_kernel(Src src, const uint32_t* __
 }
 
 // ---------------------------------------------------------------- counting
-// CTA per group g (left parent x = gpar[g]); siblings in batches of 32 (lane j accumulates
-// sibling j); warps stride over 256-word chunks of the class vectors; one atomic per (warp,
-// sibling).  Two siblings share one packed redux.sync (per-warp sums <= 32 x 8 x 32 < 2^16).
+// WARP = false: CTA per group g (left parent x = gpar[g]), its warps striding over 256-word chunks
+// of the class lists, one atomic per (warp, sibling) -- long lists (generation 3); WARP = true:
+// one warp per group walking the whole list, plain stores -- short lists (deep generations, where
+// a CTA per group would leave most of its warps idle).  Siblings in batches of 32 (lane j
+// accumulates sibling j); two siblings share one packed redux.sync (per-chunk warp sums
+// <= 32 x 8 x 32 < 2^16).
+template <bool WARP>
 __global__ void __launch_bounds__(kT) count_proj_kernel(const uint32_t* __restrict__ data,
                                                         const uint64_t* __restrict__ off,
                                                         const uint32_t* __restrict__ nw,
                                                         const uint32_t* __restrict__ gpar,
                                                         const uint32_t* __restrict__ ext_off,
                                                         const uint32_t* __restrict__ eidx,
-                                                        uint32_t* __restrict__ counts) {
-  const uint32_t g = blockIdx.x;
+                                                        uint32_t* __restrict__ counts, uint32_t G) {
   const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const uint32_t g = WARP ? blockIdx.x * (kT / 32) + warp : blockIdx.x;
+  if (WARP && g >= G) return;
+  constexpr uint32_t w_step = WARP ? 256u : (kT / 32) * 256u;
   const uint32_t x = gpar[g];
   const uint32_t n = nw[x];
   const uint32_t* X = data + off[x];
@@ -401,7 +407,7 @@ __global__ void __launch_bounds__(kT) count_proj_kernel(const uint32_t* __restri
     const uint32_t nb = min(32u, e1 - b0);
     const uint64_t my_off = lane < nb ? off[eidx[b0 + lane]] : 0;
     uint32_t acc = 0;
-    for (uint32_t w = warp * 256; w < n; w += (kT / 32) * 256) {
+    for (uint32_t w = WARP ? 0u : warp * 256u; w < n; w += w_step) {
       const uint32_t w0 = w + lane * 4, w1 = w + 128 + lane * 4;
       const bool h0 = w0 < n, h1 = w1 < n;
       const uint4 x0 = h0 ? *reinterpret_cast<const uint4*>(X + w0) : make_uint4(0, 0, 0, 0);
@@ -426,7 +432,11 @@ __global__ void __launch_bounds__(kT) count_proj_kernel(const uint32_t* __restri
         if (lane == i + 1) acc += c >> 16;
       }
     }
-    if (lane < nb && acc) atomicAdd(&counts[b0 + lane], acc);
+    if (WARP) {
+      if (lane < nb) counts[b0 + lane] = acc;
+    } else if (lane < nb && acc) {
+      atomicAdd(&counts[b0 + lane], acc);
+    }
   }
 }
 
@@ -605,7 +615,12 @@ bool proj_build(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const 
 void launch_count_proj(const DeviceProj& P, const uint32_t* gpar, const uint32_t* ext_off, const uint32_t* eidx,
                        uint32_t G, uint32_t* counts, cudaStream_t s) {
   if (G == 0) return;
-  { count_proj_kernel<<<G, kT, 0, s>>>(P.data.p, P.off.p, P.nw.p, gpar, ext_off, eidx, counts); note_launch(); }
+  if ((uint64_t)P.max_lw * 32 <= 8192)
+    { count_proj_kernel<true><<<(G + kT / 32 - 1) / (kT / 32), kT, 0, s>>>(P.data.p, P.off.p, P.nw.p, gpar, ext_off,
+                                                                          eidx, counts, G); note_launch(); }
+  else
+    { count_proj_kernel<false><<<G, kT, 0, s>>>(P.data.p, P.off.p, P.nw.p, gpar, ext_off, eidx, counts, G);
+      note_launch(); }
   GPA_CUDA(cudaGetLastError());
 }
 
