@@ -312,6 +312,177 @@ __device__ __forceinline__ void pext_item(const uint32_t* __restrict__ mp, const
   }
 }
 
+// ---------------------------------------------------------------- generation 3: bit gather
+// Generation 3's masks are bitset rows (~5 % set): instead of compressing every word per lane,
+// the warp gathers the ~C set bits of a 32-word chunk (row words 32 j .. 32 j + 31, one per lane)
+// in ceil(C / 32) ballots: lane l stages (l, bit) of its set bits in shared memory at its rank
+// (warp scan of the popcounts), then lane r of ballot t takes set bit 32 t + r, fetches the
+// member's word from its owner lane (shfl) and the ballot packs 32 of those bits into one output
+// word.  A member's list is the concatenation of these words (each chunk padded to whole words;
+// natural order, common to the class -- the next generation views it as 32 lane streams).
+// Work ~ output words, not input words.  (seg3 / cls3: sizes; pext3: the lists.)
+
+// warp per pair p = s * cmax + c: output words of row a's segment s (sum over its chunks)
+__global__ void seg3_kernel(const uint32_t* __restrict__ rows, uint64_t pitch, const uint32_t* __restrict__ par_a,
+                            const uint32_t* __restrict__ bound, const uint32_t* __restrict__ n_cls, uint32_t cmax,
+                            uint32_t n_pairs, uint32_t* __restrict__ w3, unsigned long long* __restrict__ in_words) {
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t p = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  if (p >= n_pairs) return;
+  const uint32_t c = p % cmax, s = p / cmax;
+  uint32_t words = 0;
+  if (c < *n_cls) {
+    const uint32_t j0 = bound[c], m = bound[c + 1] - j0;
+    if (m >= 2) {
+      const uint32_t* row = rows + (uint64_t)par_a[j0] * pitch + lane;
+      uint32_t a, b;
+      seg_range((uint32_t)(pitch / 32), s, a, b);
+      for (uint32_t j = a; j < b; ++j) {
+        const uint32_t C = __reduce_add_sync(0xffffffffu, (uint32_t)__popc(row[32ull * j]));
+        words += (C + 31) / 32;
+      }
+      if (lane == 0 && b > a) atomicAdd(in_words, 32ull * (b - a) * m);
+    }
+  }
+  if (lane == 0) w3[p] = words;
+}
+
+// thread per class: word offset of every segment in the class' lists, list words (a multiple of
+// 32), the class' words, pext3 items (one per segment with words and group of <= 8 members)
+__global__ void cls3_pad_kernel(const uint32_t* __restrict__ w3, const uint32_t* __restrict__ bound,
+                                const uint32_t* __restrict__ n_cls, uint32_t cmax, uint32_t nseg,
+                                uint32_t* __restrict__ loc3, uint32_t* __restrict__ nwc,
+                                uint64_t* __restrict__ cls_words, uint32_t* __restrict__ items,
+                                uint32_t* __restrict__ max_lw) {
+  const uint32_t C = *n_cls;
+  for (uint32_t c = blockIdx.x * blockDim.x + threadIdx.x; c < cmax; c += gridDim.x * blockDim.x) {
+    const uint32_t m = c < C ? bound[c + 1] - bound[c] : 0;
+    const uint32_t groups = m >= 2 ? (m + kMemberGroup - 1) / kMemberGroup : 0;
+    uint32_t acc = 0;
+    for (uint32_t s = 0; s < nseg; ++s) {
+      const uint64_t p = (uint64_t)s * cmax + c;
+      loc3[p] = acc;
+      acc += w3[p];
+      items[p] = w3[p] ? groups : 0;
+    }
+    const uint32_t words = groups ? (acc + 31u) & ~31u : 0u;
+    nwc[c] = words;
+    cls_words[c] = (uint64_t)words * m;
+    if (words) atomicMax(max_lw, words / 32u);
+  }
+}
+
+template <uint32_t G>
+__device__ __forceinline__ void pext3_item(const uint32_t* __restrict__ mrow, const uint32_t* __restrict__ sbase,
+                                           const uint32_t (&so)[kMemberGroup], const uint32_t* __restrict__ s_oo,
+                                           uint32_t nm, uint32_t ja, uint32_t jb, uint32_t ow0,
+                                           uint32_t* __restrict__ data, uint32_t wbytes, uint16_t* __restrict__ smap) {
+  const uint32_t lane = threadIdx.x & 31;
+  uint32_t keep[G], xn[G];
+  uint32_t wc = 0;  // words emitted in this segment (warp-uniform)
+  const uint32_t* mp = mrow + 32u * ja;
+  const uint32_t* cur = sbase + 32u * ja;
+  uint32_t mn = __ldg(mp);
+#pragma unroll
+  for (uint32_t q = 0; q < G; ++q) {
+    keep[q] = 0;
+    xn[q] = __ldg(addr_of(cur, so[q], wbytes));
+  }
+  for (uint32_t j = ja; j < jb; ++j) {
+    const uint32_t mw = mn;
+    uint32_t x[G];
+#pragma unroll
+    for (uint32_t q = 0; q < G; ++q) x[q] = xn[q];
+    const uint32_t step = j + 1 < jb ? 32u : 0u;
+    mp += step;
+    cur += step;
+    mn = __ldg(mp);
+#pragma unroll
+    for (uint32_t q = 0; q < G; ++q) xn[q] = __ldg(addr_of(cur, so[q], wbytes));
+    // ranks of this lane's set bits among the chunk's: warp scan of the popcounts
+    const uint32_t c = __popc(mw);
+    uint32_t o = c;
+#pragma unroll
+    for (uint32_t d = 1; d < 32; d <<= 1) {
+      const uint32_t t = __shfl_up_sync(0xffffffffu, o, d);
+      if (lane >= d) o += t;
+    }
+    const uint32_t C = __shfl_sync(0xffffffffu, o, 31);
+    o -= c;
+    for (uint32_t mm = mw; mm; mm &= mm - 1u) smap[o++] = (uint16_t)((lane << 5) | (uint32_t)(__ffs(mm) - 1));
+    __syncwarp();
+    for (uint32_t k0 = 0; k0 < C; k0 += 32) {
+      const uint32_t k = k0 + lane;
+      const bool ok = k < C;
+      const uint32_t v = ok ? smap[k] : 0u;
+      const uint32_t L = v >> 5, sh = v & 31u;
+#pragma unroll
+      for (uint32_t q = 0; q < G; ++q) {
+        const uint32_t xv = __shfl_sync(0xffffffffu, x[q], L);
+        const uint32_t b = __ballot_sync(0xffffffffu, ok && ((xv >> sh) & 1u));
+        if (lane == (wc & 31u)) keep[q] = b;
+      }
+      if ((wc & 31u) == 31u) {
+#pragma unroll
+        for (uint32_t q = 0; q < G; ++q)
+          if (q < nm) data[s_oo[q] + ow0 + (wc - 31u) + lane] = keep[q];
+      }
+      ++wc;
+    }
+    __syncwarp();  // smap is rewritten by the next chunk
+  }
+  if (wc & 31u) {
+    const uint32_t base = wc & ~31u;
+    if (lane < (wc & 31u)) {
+#pragma unroll
+      for (uint32_t q = 0; q < G; ++q)
+        if (q < nm) data[s_oo[q] + ow0 + base + lane] = keep[q];
+    }
+  }
+}
+
+__global__ void __launch_bounds__(kT, 4) pext3_kernel(const uint32_t* __restrict__ rows, uint64_t pitch,
+                                                      const uint32_t* __restrict__ par_a,
+                                                      const uint32_t* __restrict__ par_b,
+                                                      const uint32_t* __restrict__ bound, uint32_t cmax,
+                                                      const uint32_t* __restrict__ item_pair,
+                                                      const uint32_t* __restrict__ item_off, uint32_t T,
+                                                      const uint32_t* __restrict__ loc3,
+                                                      const uint64_t* __restrict__ off, uint32_t* __restrict__ data,
+                                                      uint32_t wbytes) {
+  __shared__ uint16_t s_map[kT / 32][1024];
+  __shared__ uint32_t s_oo[kT / 32][kMemberGroup];
+  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const uint32_t it = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  if (it >= T) return;
+  const uint32_t p = item_pair[it];
+  const uint32_t c = p % cmax, s = p / cmax;
+  const uint32_t j0 = bound[c], m = bound[c + 1] - j0;
+  const uint32_t g = it - item_off[p];
+  const uint32_t first = j0 + g * kMemberGroup;
+  const uint32_t nm = min(kMemberGroup, m - g * kMemberGroup);
+  uint32_t ja, jb;
+  seg_range((uint32_t)(pitch / 32), s, ja, jb);
+  if (ja >= jb) return;
+  uint32_t* oo = s_oo[warp];
+  uint32_t so[kMemberGroup];
+#pragma unroll
+  for (uint32_t q = 0; q < kMemberGroup; ++q) {
+    const uint32_t e = first + (q < nm ? q : 0);  // surplus slots shadow member 0 (not stored)
+    so[q] = (uint32_t)((uint64_t)par_b[e] * pitch);
+    if (lane == q) oo[q] = (uint32_t)off[e];
+  }
+  __syncwarp();
+  const uint32_t* mrow = rows + (uint64_t)par_a[j0] * pitch + lane;
+  const uint32_t ow0 = loc3[p];
+  if (nm <= 2)
+    pext3_item<2>(mrow, rows + lane, so, oo, nm, ja, jb, ow0, data, wbytes, s_map[warp]);
+  else if (nm <= 4)
+    pext3_item<4>(mrow, rows + lane, so, oo, nm, ja, jb, ow0, data, wbytes, s_map[warp]);
+  else
+    pext3_item<8>(mrow, rows + lane, so, oo, nm, ja, jb, ow0, data, wbytes, s_map[warp]);
+}
+
 // item -> its pair (items of pair p are item_off[p] .. + items[p])
 __global__ void item_pair_kernel(const uint32_t* __restrict__ items, const uint32_t* __restrict__ item_off,
                                  uint32_t n_pairs, uint32_t* __restrict__ item_pair) {
@@ -459,6 +630,15 @@ __global__ void proj_totals_kernel(const uint32_t* __restrict__ items, const uin
   }
 }
 
+// generation 3 by bit gather (pext3_kernel); GPA_PROJ_K3_PEXT=1 keeps the set-bit-walk pext (comparisons)
+bool gather3() {
+  static const bool v = [] {
+    const char* e = getenv("GPA_PROJ_K3_PEXT");
+    return !(e && atoi(e) != 0);
+  }();
+  return v;
+}
+
 // per-thread, per-device persistent workspace (grow-only): the class tables of proj_build and the
 // two generations of lists
 struct ProjWork {
@@ -535,12 +715,19 @@ bool proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, 
   W.cls_base.ensure(cmax);
   W.tot.ensure(2);
   const unsigned wpb = kT / 32;
-  { seg_popc_kernel<<<(n_pairs + wpb - 1) / wpb, kT, 0, s>>>(
-        src, par_a, W.bound.p, W.small.p, cmax, nseg, n_pairs, W.words.p,
-        reinterpret_cast<unsigned long long*>(W.small.p + 2)); note_launch(); }
-  { cls_pad_kernel<<<(cmax + wpb - 1) / wpb, kT, 0, s>>>(
-        W.words.p, W.bound.p, W.small.p, cmax, nseg, W.loc.p, W.nwc.p, W.cls_words.p, W.items.p, W.small.p + 1);
-    note_launch(); }
+  if (!prev && gather3()) {  // generation 3: bit gather (pext3_kernel), natural-order lists
+    { seg3_kernel<<<(n_pairs + wpb - 1) / wpb, kT, 0, s>>>(rows, pitch_words, par_a, W.bound.p, W.small.p, cmax, n_pairs,
+          W.words.p, reinterpret_cast<unsigned long long*>(W.small.p + 2)); note_launch(); }
+    { cls3_pad_kernel<<<grid_for(cmax, n_sms), kT, 0, s>>>(W.words.p, W.bound.p, W.small.p, cmax, nseg, W.loc.p,
+          W.nwc.p, W.cls_words.p, W.items.p, W.small.p + 1); note_launch(); }
+  } else {
+    { seg_popc_kernel<<<(n_pairs + wpb - 1) / wpb, kT, 0, s>>>(
+          src, par_a, W.bound.p, W.small.p, cmax, nseg, n_pairs, W.words.p,
+          reinterpret_cast<unsigned long long*>(W.small.p + 2)); note_launch(); }
+    { cls_pad_kernel<<<(cmax + wpb - 1) / wpb, kT, 0, s>>>(
+          W.words.p, W.bound.p, W.small.p, cmax, nseg, W.loc.p, W.nwc.p, W.cls_words.p, W.items.p, W.small.p + 1);
+      note_launch(); }
+  }
   scan_excl<uint32_t>(W.items.p, W.item_off.p, n_pairs, W.tmp, s);
   scan_excl<uint64_t>(W.cls_words.p, W.cls_base.p, cmax, W.tmp, s);
   { proj_totals_kernel<<<1, 32, 0, s>>>(W.items.p, W.item_off.p, n_pairs, W.cls_words.p, W.cls_base.p, cmax,
@@ -589,9 +776,14 @@ bool proj_build_finish(const ProjPending& pp, const uint64_t T[2], const uint32_
     { item_pair_kernel<<<grid_for(pp.n_pairs, n_sms), kT, 0, s>>>(W.items.p, W.item_off.p, pp.n_pairs,
                                                                  W.item_pair.p); note_launch(); }
     const uint64_t blocks = (T[0] + kT / 32 - 1) / (kT / 32);
-    { pext_kernel<<<(unsigned)blocks, kT, 0, s>>>(src, pp.par_a, pp.par_b, W.bound.p, pp.cmax, W.item_pair.p,
-                                                  W.item_off.p, (uint32_t)T[0], W.loc.p, out.off.p, out.data.p, 4u);
-      note_launch(); }
+    if (!pp.prev && gather3())
+      { pext3_kernel<<<(unsigned)blocks, kT, 0, s>>>(pp.rows, pp.pitch, pp.par_a, pp.par_b, W.bound.p, pp.cmax,
+                                                     W.item_pair.p, W.item_off.p, (uint32_t)T[0], W.loc.p, out.off.p,
+                                                     out.data.p, 4u); note_launch(); }
+    else
+      { pext_kernel<<<(unsigned)blocks, kT, 0, s>>>(src, pp.par_a, pp.par_b, W.bound.p, pp.cmax, W.item_pair.p,
+                                                    W.item_off.p, (uint32_t)T[0], W.loc.p, out.off.p, out.data.p, 4u);
+        note_launch(); }
   }
   GPA_CUDA(cudaGetLastError());
   return true;
