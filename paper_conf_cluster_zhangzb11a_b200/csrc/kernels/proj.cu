@@ -45,6 +45,7 @@ namespace {
 constexpr int kT = 256;
 constexpr uint32_t kSegJ = 128;          // mask segment: 128 words per lane (a bitset row: 131,072 transactions)
 constexpr uint32_t kMemberGroup = 8;     // members sharing one mask preparation in pext_kernel
+constexpr uint32_t kG3Group = 16;        // members sharing one chunk's bit ranks in pext3_kernel
 
 unsigned grid_for(uint64_t n, int n_sms, int per_sm = 16) {
   uint64_t g = (n + kT - 1) / kT;
@@ -357,7 +358,7 @@ __global__ void cls3_pad_kernel(const uint32_t* __restrict__ w3, const uint32_t*
   const uint32_t C = *n_cls;
   for (uint32_t c = blockIdx.x * blockDim.x + threadIdx.x; c < cmax; c += gridDim.x * blockDim.x) {
     const uint32_t m = c < C ? bound[c + 1] - bound[c] : 0;
-    const uint32_t groups = m >= 2 ? (m + kMemberGroup - 1) / kMemberGroup : 0;
+    const uint32_t groups = m >= 2 ? (m + kG3Group - 1) / kG3Group : 0;
     uint32_t acc = 0;
     for (uint32_t s = 0; s < nseg; ++s) {
       const uint64_t p = (uint64_t)s * cmax + c;
@@ -374,31 +375,43 @@ __global__ void cls3_pad_kernel(const uint32_t* __restrict__ w3, const uint32_t*
 
 template <uint32_t G>
 __device__ __forceinline__ void pext3_item(const uint32_t* __restrict__ mrow, const uint32_t* __restrict__ sbase,
-                                           const uint32_t (&so)[kMemberGroup], const uint32_t* __restrict__ s_oo,
+                                           const uint32_t (&so)[kG3Group], const uint32_t* __restrict__ s_oo,
                                            uint32_t nm, uint32_t ja, uint32_t jb, uint32_t ow0,
                                            uint32_t* __restrict__ data, uint32_t wbytes, uint16_t* __restrict__ smap) {
   const uint32_t lane = threadIdx.x & 31;
-  uint32_t keep[G], xn[G];
+  // groups of <= 8 load the next chunk's words one step ahead; 16-member groups have no registers
+  // left for that and rely on the other warps to hide the load latency
+  constexpr bool kPf = G <= 8;
+  constexpr uint32_t GP = kPf ? G : 1;
+  uint32_t keep[G], xn[GP];
   uint32_t wc = 0;  // words emitted in this segment (warp-uniform)
   const uint32_t* mp = mrow + 32u * ja;
   const uint32_t* cur = sbase + 32u * ja;
   uint32_t mn = __ldg(mp);
 #pragma unroll
-  for (uint32_t q = 0; q < G; ++q) {
-    keep[q] = 0;
-    xn[q] = __ldg(addr_of(cur, so[q], wbytes));
+  for (uint32_t q = 0; q < G; ++q) keep[q] = 0;
+  if constexpr (kPf) {
+#pragma unroll
+    for (uint32_t q = 0; q < GP; ++q) xn[q] = __ldg(addr_of(cur, so[q], wbytes));
   }
   for (uint32_t j = ja; j < jb; ++j) {
     const uint32_t mw = mn;
     uint32_t x[G];
+    if constexpr (kPf) {
 #pragma unroll
-    for (uint32_t q = 0; q < G; ++q) x[q] = xn[q];
+      for (uint32_t q = 0; q < GP; ++q) x[q] = xn[q];
+    } else {
+#pragma unroll
+      for (uint32_t q = 0; q < G; ++q) x[q] = __ldg(addr_of(cur, so[q], wbytes));
+    }
     const uint32_t step = j + 1 < jb ? 32u : 0u;
     mp += step;
     cur += step;
     mn = __ldg(mp);
+    if constexpr (kPf) {
 #pragma unroll
-    for (uint32_t q = 0; q < G; ++q) xn[q] = __ldg(addr_of(cur, so[q], wbytes));
+      for (uint32_t q = 0; q < GP; ++q) xn[q] = __ldg(addr_of(cur, so[q], wbytes));
+    }
     // ranks of this lane's set bits among the chunk's: warp scan of the popcounts
     const uint32_t c = __popc(mw);
     uint32_t o = c;
@@ -441,7 +454,7 @@ __device__ __forceinline__ void pext3_item(const uint32_t* __restrict__ mrow, co
   }
 }
 
-__global__ void __launch_bounds__(kT, 4) pext3_kernel(const uint32_t* __restrict__ rows, uint64_t pitch,
+__global__ void __launch_bounds__(kT, 3) pext3_kernel(const uint32_t* __restrict__ rows, uint64_t pitch,
                                                       const uint32_t* __restrict__ par_a,
                                                       const uint32_t* __restrict__ par_b,
                                                       const uint32_t* __restrict__ bound, uint32_t cmax,
@@ -451,7 +464,7 @@ __global__ void __launch_bounds__(kT, 4) pext3_kernel(const uint32_t* __restrict
                                                       const uint64_t* __restrict__ off, uint32_t* __restrict__ data,
                                                       uint32_t wbytes) {
   __shared__ uint16_t s_map[kT / 32][1024];
-  __shared__ uint32_t s_oo[kT / 32][kMemberGroup];
+  __shared__ uint32_t s_oo[kT / 32][kG3Group];
   const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const uint32_t it = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   if (it >= T) return;
@@ -459,15 +472,15 @@ __global__ void __launch_bounds__(kT, 4) pext3_kernel(const uint32_t* __restrict
   const uint32_t c = p % cmax, s = p / cmax;
   const uint32_t j0 = bound[c], m = bound[c + 1] - j0;
   const uint32_t g = it - item_off[p];
-  const uint32_t first = j0 + g * kMemberGroup;
-  const uint32_t nm = min(kMemberGroup, m - g * kMemberGroup);
+  const uint32_t first = j0 + g * kG3Group;
+  const uint32_t nm = min(kG3Group, m - g * kG3Group);
   uint32_t ja, jb;
   seg_range((uint32_t)(pitch / 32), s, ja, jb);
   if (ja >= jb) return;
   uint32_t* oo = s_oo[warp];
-  uint32_t so[kMemberGroup];
+  uint32_t so[kG3Group];
 #pragma unroll
-  for (uint32_t q = 0; q < kMemberGroup; ++q) {
+  for (uint32_t q = 0; q < kG3Group; ++q) {
     const uint32_t e = first + (q < nm ? q : 0);  // surplus slots shadow member 0 (not stored)
     so[q] = (uint32_t)((uint64_t)par_b[e] * pitch);
     if (lane == q) oo[q] = (uint32_t)off[e];
@@ -479,8 +492,10 @@ __global__ void __launch_bounds__(kT, 4) pext3_kernel(const uint32_t* __restrict
     pext3_item<2>(mrow, rows + lane, so, oo, nm, ja, jb, ow0, data, wbytes, s_map[warp]);
   else if (nm <= 4)
     pext3_item<4>(mrow, rows + lane, so, oo, nm, ja, jb, ow0, data, wbytes, s_map[warp]);
-  else
+  else if (nm <= 8)
     pext3_item<8>(mrow, rows + lane, so, oo, nm, ja, jb, ow0, data, wbytes, s_map[warp]);
+  else
+    pext3_item<16>(mrow, rows + lane, so, oo, nm, ja, jb, ow0, data, wbytes, s_map[warp]);
 }
 
 // item -> its pair (items of pair p are item_off[p] .. + items[p])
