@@ -336,7 +336,7 @@ def main():
             return {"bound": "alu", "achieved": ach, "peak": int_peak, "unit": "T int ops/s", "frac": ach / int_peak,
                     "peak_basis": f"ALU + FMA pipes, 2 x 64 lanes/clk/SM x 148 SM x {sm_max:.0f} MHz; "
                                   f"{PEXT_OPS} algorithmic ops per compressed 32-bit mask word and member (the HD "
-                                  f"compress formulation; generation 3 runs the set-bit walk on the same work unit)",
+                                  f"compress formulation as a work-normalised rate; generation 3 runs a warp bit gather on the same work unit)",
                     "kernel_ms": ms, "work": work, "work_unit": "mask words x members"}
         if name == "count_proj":
             return {"bound": None, "achieved": work / (ms * 1e-3) / 1e12, "peak": None, "unit": "Tcand*tx/s "
