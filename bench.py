@@ -362,7 +362,7 @@ def main():
     roof["traffic"] = None
     try:
         tr = json.load(open(os.path.join(ROOT, "profiles", "traffic.json")))
-        key = {"pairs": "count_pairs_kernel", "prefix": "count_prefix_kernel", "pext": f"pext_kernel (k={dom[1]})",
+        key = {"pairs": "count_pairs_kernel", "prefix": "count_prefix_kernel", "pext": "pext3_kernel (k=3)" if dom[1] == 3 else f"pext_kernel (k={dom[1]})",
                "pairs_tc": "count_pairs_tc_kernel"}.get(dom[0], f"count_trie_kernel<{dom[1]}, 2>")
         if key in tr:
             roof["traffic"] = tr[key]["dram_bytes"]

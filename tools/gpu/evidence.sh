@@ -6,5 +6,5 @@ timeout 600 python bench.py --steps 5 --warmup 3 > gpurun_out/bench.jsonl 2> gpu
 timeout 600 python bench.py --impl reference --steps 2 --warmup 1 > gpurun_out/bench_ref.jsonl 2> gpurun_out/bench_ref.err
 B="python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu-baseline --no-rules"
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches.csv $B > gpurun_out/ncu_launch.log 2>&1
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:"pext_kernel|count_pairs_tc_kernel|count_proj_kernel" -c 3 -o gpurun_out/prof_top $B > gpurun_out/ncu_top.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:"pext3_kernel|count_pairs_tc_kernel|count_proj_kernel" -c 3 -o gpurun_out/prof_top $B > gpurun_out/ncu_top.log 2>&1
 echo done
