@@ -417,6 +417,35 @@ def test_proj_fallback_to_complete_intersection(monkeypatch, how):
     assert all((kinds[k] == "proj") == (k <= last) for k in kinds), kinds
 
 
+@pytest.mark.parametrize("name", ["mushroom", "chess", "random"])
+def test_proj_k3_set_bit_walk_pext(name):
+    """Generation 3's lists by the set-bit-walk pext (GPA_PROJ_K3_PEXT=1, read once per process, so
+    a child process) instead of the default warp bit gather (pext3_kernel): every frequent itemset and
+    support equal to the oracle's."""
+    import json
+    import subprocess
+    import sys
+    if name == "random":
+        ds, theta = gen.random_db(11, 8000, 40, max_len=16), 80
+        spec = "gen.random_db(11, 8000, 40, max_len=16), 80"
+    else:
+        ds = gen.make(name)
+        theta = oracle.min_count(ds.n_tx, gen.CONFIGS[name].minsup)
+        spec = f"gen.make({name!r}), {theta}"
+    code = ("import json, gen, paper_conf_cluster_zhangzb11a_b200 as gpa\n"
+            f"ds, th = {spec}\n"
+            "r = gpa.mine(ds, min_count=th)\n"
+            "print(json.dumps(sorted([list(map(int, s)), int(c)] for s, c in r.frequent().items())))\n")
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, GPA_PROJ_K3_PEXT="1")
+    out = subprocess.run([sys.executable, "-c", code], cwd=root, env=env, capture_output=True, text=True,
+                         check=True, timeout=600).stdout
+    got = {tuple(s): c for s, c in json.loads(out.strip().splitlines()[-1])}
+    ref = oracle.mine_ds(ds, theta).frequent()
+    assert got == {tuple(map(int, s)): int(c) for s, c in ref.items()}
+    assert max(len(s) for s in got) >= 4
+
+
 # ---------------------------------------------------------------- association rules (f4)
 
 @pytest.mark.parametrize("name,minconf", [("fig2", "0.5"), ("fig2", "1"), ("chess", "0.95"), ("mushroom", "0.8"),
