@@ -349,7 +349,7 @@ __global__ void seg3_kernel(const uint32_t* __restrict__ rows, uint64_t pitch, c
 }
 
 // thread per class: word offset of every segment in the class' lists, list words (a multiple of
-// 32), the class' words, pext3 items (one per segment with words and group of <= 8 members)
+// 32), the class' words, pext3 items (one per segment with words and group of <= kG3Group members)
 __global__ void cls3_pad_kernel(const uint32_t* __restrict__ w3, const uint32_t* __restrict__ bound,
                                 const uint32_t* __restrict__ n_cls, uint32_t cmax, uint32_t nseg,
                                 uint32_t* __restrict__ loc3, uint32_t* __restrict__ nwc,
@@ -428,11 +428,12 @@ __device__ __forceinline__ void pext3_item(const uint32_t* __restrict__ mrow, co
       const uint32_t k = k0 + lane;
       const bool ok = k < C;
       const uint32_t v = ok ? smap[k] : 0u;
-      const uint32_t L = v >> 5, sh = v & 31u;
+      const uint32_t L = v >> 5;
+      const uint32_t bm = ok ? 1u << (v & 31u) : 0u;  // bit select, empty past the chunk's last set bit
 #pragma unroll
       for (uint32_t q = 0; q < G; ++q) {
         const uint32_t xv = __shfl_sync(0xffffffffu, x[q], L);
-        const uint32_t b = __ballot_sync(0xffffffffu, ok && ((xv >> sh) & 1u));
+        const uint32_t b = __ballot_sync(0xffffffffu, (xv & bm) != 0u);
         if (lane == (wc & 31u)) keep[q] = b;
       }
       if ((wc & 31u) == 31u) {
