@@ -369,6 +369,12 @@ def main():
             roof["traffic_unit"] = "bytes per launch (ncu dram__bytes_read.sum + dram__bytes_write.sum)"
             if dom[0] == "pext" and "algorithmic_bytes" in tr[key]:
                 roof["algorithmic_bytes"] = tr[key]["algorithmic_bytes"]
+                # the same launch against HBM: algorithmic bytes / its event time vs the measured copy bandwidth
+                # (far below 1: the build is issue-bound, not memory-bound)
+                if "hbm_gbs" in peaks:
+                    gbs = roof["algorithmic_bytes"] / (roof["kernel_ms"] * 1e-3) / 1e9
+                    roof["hbm_view"] = {"achieved": gbs, "peak": float(peaks["hbm_gbs"]), "unit": "GB/s",
+                                        "frac": gbs / float(peaks["hbm_gbs"])}
             elif dom[1] == 2:   # each of the n rows read once (streaming design)
                 roof["algorithmic_bytes"] = (dom[4].stats["n_groups"] + 1) * (n_tx / 8)
     except Exception:
