@@ -8,7 +8,7 @@
 //   of rows [rb*RB, rb*RB + RB).  It zeroes a shared-memory tile of RB rows x 16 words (row
 //   stride 17 words: lanes writing the same word column of different rows hit different
 //   banks; 68 KB for 1,024 rows -> 3 CTAs per SM to hide the gather latency), scans the chunk's
-//   transactions (one thread per transaction, 4 item -> row gathers in flight), sets bits with
+//   transactions (kPer consecutive items per thread, kPer item loads in flight), sets bits with
 //   shared-memory atomicOr (duplicates are harmless: OR is idempotent, so non-canonical input
 //   needs no special case), then writes every row's 64-byte segment with coalesced stores.  Every word of the output is written (padding
 //   transactions contribute no bits, so padding is zero).
@@ -25,6 +25,7 @@ constexpr uint32_t kChunkTx = 512;       // transactions per CTA = 16 words (64-
 constexpr uint32_t kChunkWords = kChunkTx / 32;
 constexpr uint32_t kTileStride = 17;     // padded words per tile row (odd: conflict-free columns)
 constexpr uint32_t kRowBlock = 1024;     // rows per CTA tile: 1024 * 17 * 4 = 68 KB -> 3 CTAs / SM
+constexpr uint32_t kPer = 8;             // items per thread and round of the sweep
 constexpr uint32_t kSmemRowMap = 1024;   // item -> row map in shared memory up to this many items (3 CTAs / SM)
 
 __global__ void __launch_bounds__(kBuildThreads) bitset_build_kernel(const uint64_t* __restrict__ offsets,
@@ -55,13 +56,14 @@ __global__ void __launch_bounds__(kBuildThreads) bitset_build_kernel(const uint6
     soff[i] = (uint32_t)(o - A < 0xffffffffull ? o - A : 0xffffffffull);
   }
   __syncthreads();
-  // coalesced sweep over the chunk's items: thread k takes items 4k .. 4k+3 (+ 4 x 256 per round);
-  // the transaction of its first item by binary search in soff, then a forward walk
+  // coalesced sweep over the chunk's items: thread k takes items kPer*k .. kPer*k + kPer-1 (+ kPer x 256
+  // per round; kPer loads in flight per thread); the transaction of its first item by binary search in
+  // soff, then a forward walk
   const uint32_t n_it = soff[kChunkTx];
-  for (uint32_t q = threadIdx.x * 4; q < n_it; q += blockDim.x * 4) {
-    uint32_t it[4];
+  for (uint32_t q = threadIdx.x * kPer; q < n_it; q += blockDim.x * kPer) {
+    uint32_t it[kPer];
 #pragma unroll
-    for (int u = 0; u < 4; ++u) it[u] = q + u < n_it ? __ldg(items + A + q + u) : 0xffffffffu;
+    for (int u = 0; u < (int)kPer; ++u) it[u] = q + u < n_it ? __ldg(items + A + q + u) : 0xffffffffu;
     uint32_t lo = 0, hi = kChunkTx;  // tx = last with soff[tx] <= q
     while (lo + 1 < hi) {
       const uint32_t mid = (lo + hi) >> 1;
@@ -69,7 +71,7 @@ __global__ void __launch_bounds__(kBuildThreads) bitset_build_kernel(const uint6
     }
     uint32_t tx = lo;
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {
+    for (int u = 0; u < (int)kPer; ++u) {
       const uint32_t j = q + u;
       if (j >= n_it) break;
       while (tx + 1 < kChunkTx && soff[tx + 1] <= j) ++tx;
