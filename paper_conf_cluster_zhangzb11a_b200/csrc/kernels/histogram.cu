@@ -37,12 +37,12 @@ __global__ void __launch_bounds__(kHistThreads) hist_validate_kernel(const uint6
     if (o1 < o0 || o1 > nnz) { my_flags |= kFlagBadOffsets; continue; }
     uint32_t prev = 0;
     uint64_t j = o0;
-    for (; j + 4 <= o1; j += 4) {  // 4 independent loads in flight
-      uint32_t it[4];
+    for (; j + 8 <= o1; j += 8) {  // 8 independent loads in flight
+      uint32_t it[8];
 #pragma unroll
-      for (int u = 0; u < 4; ++u) it[u] = __ldg(items + j + u);
+      for (int u = 0; u < 8; ++u) it[u] = __ldg(items + j + u);
 #pragma unroll
-      for (int u = 0; u < 4; ++u) {
+      for (int u = 0; u < 8; ++u) {
         if (it[u] >= n_items) { my_flags |= kFlagBadItem; continue; }
         if ((j + u) > o0 && it[u] <= prev) my_flags |= kFlagNonCanonical;
         prev = it[u];
