@@ -119,6 +119,10 @@ typedef struct {
 #define GPA_NO_OVERLAP_INGEST 4u /* gpa_mine, host input: upload the whole database before computing
                                   (default: upload in chunks overlapped with histogram, bitset build and
                                   generation-2 counting) */
+#define GPA_COMPLETE_INTERSECTION 8u /* gpa_mine: every generation k >= 3 by complete intersection from the
+                                  static bitset (the paper's method, P18@394; TRIE / PREFIX kernels), never
+                                  the projected lists of GPA_KERNEL_PROJ.  With count_kernel GPA_KERNEL_PAIRS
+                                  this is the north-star path without tensor cores */
 
 typedef struct {
   uint32_t count_kernel;       /* GPA_KERNEL_*; default GPA_KERNEL_AUTO */
@@ -151,12 +155,49 @@ gpa_status gpa_dist_destroy(gpa_dist* dist);
 /* rank / world of a communicator (for bindings and tests). */
 gpa_status gpa_dist_info(const gpa_dist* dist, int* rank, int* world);
 
+/*
+ * Host-staged collectives: the same sharded path (every all-reduce of gpa_bitset_create /
+ * gpa_count / gpa_mine, in the same order and sizes) over a caller-supplied in-place
+ * all-reduce of HOST memory -- for ranks that share one GPU (NCCL refuses two ranks on one
+ * device), for MPI / gloo users, and for tests of the sharded path.  Each collective copies
+ * the device buffer to a pinned host buffer, synchronises the stream, calls
+ *     fn(ctx, host_buf, n, dtype, op)   dtype: GPA_DT_U32 / GPA_DT_U64, op: GPA_OP_SUM / GPA_OP_MAX
+ * which must leave the element-wise reduction over all ranks in host_buf and return 0 (any
+ * other value fails the call with GPA_ERR_NCCL and marks the handle unusable, GPA_ERR_STATE),
+ * then copies the result back.  fn is called on the thread that called the library.
+ */
+#define GPA_DT_U32 0u
+#define GPA_DT_U64 1u
+#define GPA_OP_SUM 0u
+#define GPA_OP_MAX 1u
+typedef int (*gpa_host_allreduce_fn)(void* ctx, void* host_buf, uint64_t n, uint32_t dtype, uint32_t op);
+gpa_status gpa_dist_create_host(int rank, int world, int device, gpa_host_allreduce_fn fn, void* ctx,
+                                gpa_dist** out);
+
+/*
+ * Collective log: every all-reduce this handle has issued, in order, encoded as
+ * (op << 60) | (dtype << 56) | n.  *n_total = the number issued; min(cap, *n_total) entries are
+ * written to entries (may be NULL when cap == 0).  Every rank of a correct run issues the same
+ * sequence -- the library takes every path decision (overlapped ingest, fallbacks, input
+ * validation) collectively, so the sequences never diverge (tests compare them).
+ */
+gpa_status gpa_dist_log(const gpa_dist* dist, uint64_t* entries, uint64_t cap, uint64_t* n_total);
+
+/*
+ * Failure detection (NCCL): waits on the library's streams poll ncclCommGetAsyncError; an
+ * asynchronous NCCL error, or a wait longer than `seconds` (default 600; <= 0 disables), aborts the
+ * communicator (ncclCommAbort) and fails the call with GPA_ERR_NCCL; the handle then reports
+ * GPA_ERR_STATE.
+ */
+gpa_status gpa_dist_set_timeout(gpa_dist* dist, double seconds);
+
 /* ------------------------------------------------------------------ static bitset */
 
 /*
  * Build the static bitset of db on the device: one row per item whose (global) count is
  * >= row_min_count (row_min_count = 1: every occurring item; = min_count: the paper's
- * "vertical lists of first generation", P18@755).  Rows are ordered by ascending item id.
+ * "vertical lists of first generation", P18@755; = 0: every item id < n_items, absent items
+ * with an all-zero row).  Rows are ordered by ascending item id.
  * Row r, transaction t -> word t/32, bit t%32 (LSB first; Q9); padding bits are 0;
  * the row pitch is a multiple of 128 bytes (>= the paper's 64-byte alignment, P18@1685).
  * With dist, the call is collective; each rank holds the rows over its own transactions and
@@ -244,16 +285,23 @@ typedef struct {
   double setup_ms;             /* GPA_KERNEL_PROJ: CUDA-event time from the start of the generation's
                                   counting to the list-building kernel (class tables, sizes); the
                                   support kernel is count_ms - setup_ms - build_ms */
+  uint64_t build_bytes;        /* GPA_KERNEL_PROJ: algorithmic HBM bytes of the list build: every source
+                                  list (generation 3: bitset row) read once + the new lists written once */
+  uint64_t count_bytes;        /* GPA_KERNEL_PROJ: algorithmic HBM bytes of the support kernel: every list
+                                  of L_{k-1} read once + the counts written */
 } gpa_level_stats;
 gpa_status gpa_result_level_stats(const gpa_result* r, uint32_t k, gpa_level_stats* out);
 
-/* Phase times in milliseconds (host wall clock around each phase, device work included). */
-#define GPA_PHASE_UPLOAD 0     /* H2D of the CSR (host input only) */
+/* Phase times in milliseconds.  UPLOAD .. BITSET: host wall clock around each (synchronised)
+ * build phase; CANDGEN, COUNT, THRESHOLD: CUDA-event time on the mining stream, generation by
+ * generation (contiguous: their sum is the level loop's device timeline); TOTAL: wall clock. */
+#define GPA_PHASE_UPLOAD 0     /* H2D of the CSR (host input only; overlapped ingest: upload + histogram +
+                                  bitset + generation-2 counting of the chunks) */
 #define GPA_PHASE_HISTOGRAM 1  /* validation + generation-1 counts (+ all-reduce) */
 #define GPA_PHASE_BITSET 2     /* static bitset build */
-#define GPA_PHASE_CANDGEN 3    /* host join + prune + grouping + H2D of candidate groups */
-#define GPA_PHASE_COUNT 4      /* counting kernels (+ all-reduce) + D2H of counts */
-#define GPA_PHASE_THRESHOLD 5  /* L_k selection */
+#define GPA_PHASE_CANDGEN 3    /* join + prune of C_k (+ class tables of the projected lists) */
+#define GPA_PHASE_COUNT 4      /* list build + counting kernels + all-reduce */
+#define GPA_PHASE_THRESHOLD 5  /* L_k selection + compaction + item mapping */
 #define GPA_PHASE_TOTAL 6      /* whole gpa_mine call */
 #define GPA_PHASE_COUNT_ 7
 gpa_status gpa_result_timing(const gpa_result* r, double ms_by_phase[GPA_PHASE_COUNT_]);

@@ -38,6 +38,7 @@ KERNEL_NAMES = {0: "auto", 1: "v0", 2: "prefix", 3: "pairs", 4: "trie", 5: "pair
 KEEP_CANDIDATES = 1
 HOST_CANDGEN = 2
 NO_OVERLAP_INGEST = 4
+COMPLETE_INTERSECTION = 8
 MEM_HOST, MEM_DEVICE = 0, 1
 PHASES = ["upload", "histogram", "bitset", "candgen", "count", "threshold", "total"]
 STATUS = {0: "GPA_OK", 1: "GPA_ERR_INVALID", 2: "GPA_ERR_RANGE", 3: "GPA_ERR_OOM", 4: "GPA_ERR_CUDA",
@@ -64,10 +65,16 @@ class _LevelStats(ctypes.Structure):
     _fields_ = [("n_cand", ctypes.c_uint64), ("n_freq", ctypes.c_uint64), ("n_groups", ctypes.c_uint64),
                 ("kernel", ctypes.c_uint32), ("launches", ctypes.c_uint32), ("count_ms", ctypes.c_double),
                 ("allreduce_ms", ctypes.c_double), ("candgen_ms", ctypes.c_double), ("build_ms", ctypes.c_double),
-                ("build_words", ctypes.c_uint64), ("setup_ms", ctypes.c_double)]
+                ("build_words", ctypes.c_uint64), ("setup_ms", ctypes.c_double), ("build_bytes", ctypes.c_uint64),
+                ("count_bytes", ctypes.c_uint64)]
 
 
 _LIB = None
+# int fn(void* ctx, void* host_buf, uint64_t n, uint32_t dtype, uint32_t op)  (gpa_host_allreduce_fn)
+_HOST_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32,
+                            ctypes.c_uint32)
+DT_U32, DT_U64 = 0, 1
+OP_SUM, OP_MAX = 0, 1
 
 
 def lib() -> ctypes.CDLL:
@@ -90,6 +97,9 @@ def lib() -> ctypes.CDLL:
         "gpa_dist_create": (ctypes.c_int, [ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_char_p, P(vp)]),
         "gpa_dist_destroy": (ctypes.c_int, [vp]),
         "gpa_dist_info": (ctypes.c_int, [vp, P(ctypes.c_int), P(ctypes.c_int)]),
+        "gpa_dist_create_host": (ctypes.c_int, [ctypes.c_int, ctypes.c_int, ctypes.c_int, _HOST_FN, vp, P(vp)]),
+        "gpa_dist_log": (ctypes.c_int, [vp, P(u64), u64, P(u64)]),
+        "gpa_dist_set_timeout": (ctypes.c_int, [vp, ctypes.c_double]),
         "gpa_bitset_create": (ctypes.c_int, [P(_CSR), u32, vp, P(_Options), P(vp)]),
         "gpa_bitset_destroy": (ctypes.c_int, [vp]),
         "gpa_bitset_info": (ctypes.c_int, [vp, P(u64), P(u64), P(u32), P(u64)]),
@@ -148,13 +158,15 @@ class Options:
     max_k: int = 0
     host_candgen: bool = False   # join + prune on the host (reference path) instead of the device
     overlap_ingest: bool = True  # host input: chunked upload overlapped with histogram / bitset / pairs
+    complete_intersection: bool = False   # k >= 3 by complete intersection (the paper's method), no lists
 
     def _c(self) -> _Options:
         o = _Options()
         lib().gpa_options_default(ctypes.byref(o))
         o.count_kernel = self.count_kernel
         o.flags = ((KEEP_CANDIDATES if self.keep_candidates else 0) | (HOST_CANDGEN if self.host_candgen else 0)
-                   | (0 if self.overlap_ingest else NO_OVERLAP_INGEST))
+                   | (0 if self.overlap_ingest else NO_OVERLAP_INGEST)
+                   | (COMPLETE_INTERSECTION if self.complete_intersection else 0))
         o.stream = self.stream or None
         o.device = self.device
         o.max_k = self.max_k
@@ -195,13 +207,64 @@ def _args(db, items, n_items):
     return db, items, n_items
 
 
-class Dist:
-    """NCCL communicator over the ranks of a torch.distributed job (one process per GPU)."""
+def torch_host_allreduce(arr: np.ndarray, op: str) -> None:
+    """In-place all-reduce of a uint32 / uint64 host array over the current torch.distributed group
+    (the host-staged transport's callback).  Unsigned semantics through torch's signed tensors:
+    sums wrap in two's complement (bit-identical to the unsigned sum), max compares after flipping
+    the sign bit."""
+    import torch
+    import torch.distributed as tdist
+    t = torch.from_numpy(arr.view(np.int64) if arr.dtype == np.uint64 else arr.view(np.int32))
+    if op == "max":
+        sign = -2 ** 63 if arr.dtype == np.uint64 else -2 ** 31
+        t ^= sign
+        tdist.all_reduce(t, op=tdist.ReduceOp.MAX)
+        t ^= sign
+    else:
+        tdist.all_reduce(t, op=tdist.ReduceOp.SUM)
 
-    def __init__(self, rank: int, world: int, device: int, unique_id: bytes):
+
+class Dist:
+    """Communicator over the ranks of a torch.distributed job: NCCL (one process per GPU), or the
+    host-staged transport (gpa_dist_create_host) over any in-place host all-reduce."""
+
+    def __init__(self, rank: int, world: int, device: int, unique_id: bytes | None = None, host_allreduce=None):
         h = ctypes.c_void_p()
-        _check(lib().gpa_dist_create(rank, world, device, unique_id, ctypes.byref(h)))
+        self._fn = None
+        if host_allreduce is not None:
+            def fn(_ctx, buf, n, dtype, op):
+                try:
+                    ct = ctypes.c_uint32 if dtype == DT_U32 else ctypes.c_uint64
+                    arr = np.ctypeslib.as_array((ct * int(n)).from_address(buf))
+                    host_allreduce(arr, "max" if op == OP_MAX else "sum")
+                    return 0
+                except Exception:   # reported to the library as a failed collective
+                    import traceback
+                    traceback.print_exc()
+                    return 1
+            self._fn = _HOST_FN(fn)   # must outlive every library call on this handle
+            _check(lib().gpa_dist_create_host(rank, world, device, self._fn, None, ctypes.byref(h)))
+        else:
+            _check(lib().gpa_dist_create(rank, world, device, unique_id, ctypes.byref(h)))
         self.h, self.rank, self.world = h, rank, world
+
+    @classmethod
+    def host_from_torch(cls, device: int) -> "Dist":
+        """Host-staged transport over the current torch.distributed group (e.g. gloo): lets several
+        ranks share one GPU, which NCCL refuses."""
+        import torch.distributed as tdist
+        return cls(tdist.get_rank(), tdist.get_world_size(), device, host_allreduce=torch_host_allreduce)
+
+    def log(self) -> list:
+        """Every collective this handle issued, in order: (op, dtype, n) tuples (gpa_dist_log)."""
+        n = ctypes.c_uint64()
+        _check(lib().gpa_dist_log(self.h, None, 0, ctypes.byref(n)))
+        buf = (ctypes.c_uint64 * max(n.value, 1))()
+        _check(lib().gpa_dist_log(self.h, buf, n.value, ctypes.byref(n)))
+        return [(int(v) >> 60, (int(v) >> 56) & 15, int(v) & ((1 << 56) - 1)) for v in buf[: n.value]]
+
+    def set_timeout(self, seconds: float) -> None:
+        _check(lib().gpa_dist_set_timeout(self.h, float(seconds)))
 
     @staticmethod
     def unique_id() -> bytes:
@@ -420,7 +483,8 @@ def mine(db, items=None, n_items=None, min_count: int = 1, dist: Dist | None = N
     inp = _Input(off, it, ni)
     o = options or Options()
     if keep_candidates is not None:
-        o = Options(o.count_kernel, keep_candidates, o.stream, o.device, o.max_k, o.host_candgen, o.overlap_ingest)
+        import dataclasses
+        o = dataclasses.replace(o, keep_candidates=keep_candidates)
     copt = o._c()
     L = lib()
     h = ctypes.c_void_p()

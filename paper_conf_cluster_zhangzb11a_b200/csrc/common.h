@@ -2,6 +2,8 @@
 // Nothing here is part of the C ABI (include/gpapriori.h is).
 #pragma once
 #include <atomic>
+#include <mutex>
+#include <set>
 #include <cstdint>
 #include <cstdio>
 #include <string>
@@ -22,6 +24,9 @@ struct Error {
 };
 
 [[noreturn]] void fail(gpa_status st, const char* fmt, ...) __attribute__((format(printf, 2, 3)));
+// cudaStreamSynchronize, except inside a collective call (DistScope, runtime/context.cpp): then it
+// polls the communicator for asynchronous errors and times out instead of hanging on a lost peer.
+void stream_wait(cudaStream_t s);
 bool trace_enabled();   // GPA_TRACE=1 (runtime/context.cpp)
 double wall_ms();       // host steady clock, ms
 void set_last_error(gpa_status st, const std::string& msg);
@@ -126,6 +131,22 @@ struct PBuf {
     return p;
   }
 };
+
+// cudaFuncAttributeMaxDynamicSharedMemorySize is a per-DEVICE attribute of a kernel: raise it
+// once per (kernel, device) under a lock (a second device or a concurrent thread must not launch
+// without it).
+inline void ensure_smem_attr(const void* func, int bytes) {
+  static std::mutex mu;
+  static std::set<std::pair<std::pair<const void*, int>, int>> done;
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) fail(GPA_ERR_CUDA, "cudaGetDevice failed");
+  std::lock_guard<std::mutex> lk(mu);
+  auto key = std::make_pair(std::make_pair(func, dev), bytes);
+  if (done.count(key)) return;
+  cudaError_t e = cudaFuncSetAttribute(func, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+  if (e != cudaSuccess) fail(GPA_ERR_CUDA, "cudaFuncSetAttribute failed: %s", cudaGetErrorString(e));
+  done.insert(key);
+}
 
 // Flags written by the validation/histogram kernel.
 constexpr uint32_t kFlagBadOffsets = 1u;

@@ -271,7 +271,7 @@ uint32_t device_threshold(const uint32_t* counts, uint32_t M, uint32_t theta, ui
   exclusive_scan(flags, pos, M, sizes, scratch, s);
   uint32_t F = 0;
   GPA_CUDA(cudaMemcpyAsync(&F, sizes, 4, cudaMemcpyDeviceToHost, s));
-  GPA_CUDA(cudaStreamSynchronize(s));
+  stream_wait(s);
   out.rows.ensure((size_t)std::max<uint32_t>(F, 1) * k, s);
   out.sup.ensure(std::max<uint32_t>(F, 1), s);
   out.par_a.ensure(std::max<uint32_t>(F, 1), s);
@@ -371,7 +371,7 @@ void device_candgen(const DeviceLevel& L, DeviceBatch& out, DeviceScratch& scrat
   if (!device_candgen_begin(L, out, scratch, n_sms, s, &sizes)) return;
   uint32_t MG[2] = {0, 0};
   GPA_CUDA(cudaMemcpyAsync(MG, sizes, 8, cudaMemcpyDeviceToHost, s));
-  GPA_CUDA(cudaStreamSynchronize(s));
+  stream_wait(s);
   device_candgen_finish(L, out, scratch, n_sms, s, MG[0], MG[1], s, nullptr);
 }
 

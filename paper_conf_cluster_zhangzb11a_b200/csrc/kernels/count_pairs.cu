@@ -251,11 +251,7 @@ uint64_t launch_count_pairs(const void* tmap128, uint32_t n_rows, uint64_t word_
   splits = (n_chunks + per - 1) / per;
   const uint64_t grid = (uint64_t)n_tiles * splits;
   GPA_REQUIRE(grid < (1ull << 31), GPA_ERR_INVALID, "count_pairs: grid too large");
-  static bool attr_set = false;
-  if (!attr_set) {
-    GPA_CUDA(cudaFuncSetAttribute(count_pairs_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes));
-    attr_set = true;
-  }
+  ensure_smem_attr(reinterpret_cast<const void*>(count_pairs_kernel), (int)kSmemBytes);
   CUtensorMap map;
   memcpy(&map, tmap128, sizeof(map));
   { count_pairs_kernel<<<(unsigned)grid, kThreads, kSmemBytes, stream>>>(map, n_rows, nb, n_tiles, chunk0, n_chunks, per,

@@ -361,11 +361,7 @@ uint64_t launch_count_pairs_tc(const uint32_t* rows, uint64_t pitch_words, uint3
   if (grid < live) grid = live;
   if (grid > live * n_bst) grid = live * n_bst;
   GPA_REQUIRE(grid < (1ull << 31), GPA_ERR_INVALID, "count_pairs_tc: grid too large");
-  static bool attr = false;
-  if (!attr) {
-    GPA_CUDA(cudaFuncSetAttribute(count_pairs_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes));
-    attr = true;
-  }
+  ensure_smem_attr(reinterpret_cast<const void*>(count_pairs_tc_kernel), (int)kSmemBytes);
   {
     count_pairs_tc_kernel<<<(unsigned)grid, kThreads, kSmemBytes, stream>>>(tmap, n_rows, nbi, (uint32_t)live,
                                                                             word_begin, (uint32_t)n_bst, 1u, counts);

@@ -282,11 +282,7 @@ void launch_k(const uint32_t* rows, uint64_t pitch_words, const TrieBlock* block
   uint32_t stages = (uint32_t)(kTrieRingBytes / ((size_t)max_rows * kSegBytes));
   stages = stages < 2 ? 2 : (stages > kTrieMaxStages ? kTrieMaxStages : stages);
   const size_t smem = (size_t)stages * max_rows * kSegBytes;
-  static bool attr = false;
-  if (!attr) {
-    GPA_CUDA(cudaFuncSetAttribute(count_trie_kernel<K, W>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024));
-    attr = true;
-  }
+  ensure_smem_attr(reinterpret_cast<const void*>(count_trie_kernel<K, W>), 200 * 1024);
   const uint64_t grid = (uint64_t)n_blocks * n_parts;
   GPA_REQUIRE(grid < (1ull << 31), GPA_ERR_INVALID, "count_trie: grid too large");
   { count_trie_kernel<K, W><<<(unsigned)grid, kThreads, smem, stream>>>(rows, pitch_words, blocks, block_rows, lrows,

@@ -28,23 +28,10 @@ static double auto_sibling_cut() {
 
 namespace {
 
-// k >= 3 trie walk: rows staged in shared memory (count_trie.cu); GPA_TRIE_TMEM=1 selects the
-// tensor-memory variant (count_trie_tm.cu) -- correct, but measured 1.6x slower on T40I10D10M
-// (DESIGN.md "Kernels"), so it is an experiment, not a default
-bool trie_tmem() {
-  static const bool v = [] {
-    const char* e = getenv("GPA_TRIE_TMEM");
-    return e && atoi(e) != 0;
-  }();
-  return v;
-}
 void launch_trie(uint32_t k, const uint32_t* rows, uint64_t pitch_words, const TrieBlock* blocks,
                  const uint32_t* block_rows, const uint4* lrows, const uint8_t* lcp, uint32_t n_blocks,
                  uint32_t max_rows, uint32_t n_parts, uint32_t* counts, cudaStream_t s) {
-  if (k >= 3 && max_rows <= kTrieWideRows && trie_tmem())
-    launch_count_trie_tm(k, rows, pitch_words, blocks, block_rows, lrows, lcp, n_blocks, max_rows, n_parts, counts, s);
-  else
-    launch_count_trie(k, rows, pitch_words, blocks, block_rows, lrows, lcp, n_blocks, max_rows, n_parts, counts, s);
+  launch_count_trie(k, rows, pitch_words, blocks, block_rows, lrows, lcp, n_blocks, max_rows, n_parts, counts, s);
 }
 
 double now_ms() {
@@ -61,23 +48,22 @@ void validate_options(const gpa_options& o) {
   GPA_REQUIRE(o.count_kernel <= GPA_KERNEL_PROJ, GPA_ERR_INVALID, "unknown count_kernel %u", o.count_kernel);
   GPA_REQUIRE(o.max_k <= GPA_MAX_K, GPA_ERR_INVALID, "max_k %u > GPA_MAX_K", o.max_k);
   GPA_REQUIRE(!o.reserved[0] && !o.reserved[1] && !o.reserved[2], GPA_ERR_INVALID, "reserved option fields must be 0");
-  GPA_REQUIRE((o.flags & ~(GPA_KEEP_CANDIDATES | GPA_HOST_CANDGEN | GPA_NO_OVERLAP_INGEST)) == 0, GPA_ERR_INVALID, "unknown option flags 0x%x",
-              o.flags);
+  GPA_REQUIRE((o.flags & ~(GPA_KEEP_CANDIDATES | GPA_HOST_CANDGEN | GPA_NO_OVERLAP_INGEST | GPA_COMPLETE_INTERSECTION)) == 0,
+              GPA_ERR_INVALID, "unknown option flags 0x%x", o.flags);
 }
 
 }  // namespace
 
-gpa_bitset* bitset_build(const gpa_tx_csr* db, uint64_t row_min_count, const gpa_dist* dist, const gpa_options* opt_in) {
-  GPA_REQUIRE(db, GPA_ERR_INVALID, "db is NULL");
-  GPA_REQUIRE(db->memory == GPA_MEM_HOST || db->memory == GPA_MEM_DEVICE, GPA_ERR_INVALID, "db->memory must be "
-              "GPA_MEM_HOST or GPA_MEM_DEVICE");
-  GPA_REQUIRE(db->offsets || db->n_tx == 0, GPA_ERR_INVALID, "db->offsets is NULL");
+gpa_bitset* bitset_build(const gpa_tx_csr* db, uint64_t row_min_count, const gpa_dist* dist, const gpa_options* opt_in,
+                         bool prechecked) {
+  GPA_REQUIRE(db, GPA_ERR_INVALID, "db is NULL");   // a caller bug, not data: checked before any device work
   gpa_options opt;
   gpa_options_default(&opt);
   if (opt_in) opt = *opt_in;
   validate_options(opt);
   dist_check(dist);
   DeviceInfo di = use_device(dist ? dist->device : opt.device);
+  if (!prechecked) agree_input(db, dist, false);
 
   auto* bs = new gpa_bitset();
   struct Guard {
@@ -128,10 +114,10 @@ gpa_bitset* bitset_build(const gpa_tx_csr* db, uint64_t row_min_count, const gpa
   } else if (n_tx) {
     GPA_CUDA(cudaMemcpyAsync(&first_off, db->offsets, sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
     GPA_CUDA(cudaMemcpyAsync(&nnz, db->offsets + n_tx, sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
-    GPA_CUDA(cudaStreamSynchronize(s));
+    stream_wait(s);
     GPA_REQUIRE(first_off == 0, GPA_ERR_INVALID, "offsets[0] must be 0");
   }
-  GPA_CUDA(cudaStreamSynchronize(s));
+  stream_wait(s);
   double t1 = now_ms();
   bs->build_ms[0] = t1 - t0;
 
@@ -148,7 +134,7 @@ gpa_bitset* bitset_build(const gpa_tx_csr* db, uint64_t row_min_count, const gpa
   launch_hist_validate(off_dev, items_dev, n_tx, nnz, n_items, d_hist.p, d_flags.p, bs->n_sms, s);
   uint32_t flags = 0;
   GPA_CUDA(cudaMemcpyAsync(&flags, d_flags.p, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
-  GPA_CUDA(cudaStreamSynchronize(s));
+  stream_wait(s);
   if ((flags & kFlagNonCanonical) && !(flags & (kFlagBadItem | kFlagBadOffsets))) {
     GPA_CUDA(cudaMemsetAsync(d_hist.p, 0, n_items * sizeof(uint32_t), s));
     launch_hist_dedup(off_dev, items_dev, n_tx, nnz, n_items, d_hist.p, bs->n_sms, s);
@@ -161,7 +147,7 @@ gpa_bitset* bitset_build(const gpa_tx_csr* db, uint64_t row_min_count, const gpa
     GPA_CUDA(cudaMemcpyAsync(bs->item_counts.data(), d_hist.p, n_items * sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
   GPA_CUDA(cudaMemcpyAsync(&flags, d_flags.p, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
   GPA_CUDA(cudaMemcpyAsync(&bs->n_tx_global, d_ntx.p, sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
-  GPA_CUDA(cudaStreamSynchronize(s));
+  stream_wait(s);
   GPA_REQUIRE(!(flags & kFlagBadOffsets), GPA_ERR_INVALID, "offsets are not non-decreasing%s",
               dist ? " (on some rank)" : "");
   GPA_REQUIRE(!(flags & kFlagBadItem), GPA_ERR_INVALID, "an item id is >= n_items (%u)%s", n_items,
@@ -170,10 +156,12 @@ gpa_bitset* bitset_build(const gpa_tx_csr* db, uint64_t row_min_count, const gpa
   double t2 = now_ms();
   bs->build_ms[1] = t2 - t1;
 
-  // ---- rows: items with count >= row_min_count, ascending id (Q8, Q14)
+  // ---- rows: items with count >= row_min_count, ascending id (Q8, Q14); row_min_count
+  // 0: every item id owns a row, absent items an all-zero one (shards of one database then share
+  // one row set without a collective)
   bs->row_of_item.assign(n_items, -1);
   for (uint32_t i = 0; i < n_items; ++i) {
-    if (bs->item_counts[i] >= row_min_count && bs->item_counts[i] > 0) {
+    if (row_min_count == 0 || (bs->item_counts[i] >= row_min_count && bs->item_counts[i] > 0)) {
       bs->row_of_item[i] = (int32_t)bs->item_of_row.size();
       bs->item_of_row.push_back(i);
     }
@@ -188,7 +176,7 @@ gpa_bitset* bitset_build(const gpa_tx_csr* db, uint64_t row_min_count, const gpa
     launch_bitset_build(off_dev, items_dev, n_tx, nnz, d_map.p, n_items, bs->n_rows, bs->pitch_words, bs->rows.p, 0,
                         n_tx, s);
   }
-  GPA_CUDA(cudaStreamSynchronize(s));
+  stream_wait(s);
   bs->build_ms[2] = now_ms() - t2;
   guard.b = nullptr;
   return bs;
@@ -322,7 +310,7 @@ bool count_device_batch(gpa_bitset* bs, DeviceBatch& B, uint32_t kernel, DeviceS
     device_exclusive_scan(n_tasks, task_off, G, tot, scratch, s);
     uint32_t T = 0;
     GPA_CUDA(cudaMemcpyAsync(&T, tot, 4, cudaMemcpyDeviceToHost, s));
-    GPA_CUDA(cudaStreamSynchronize(s));
+    stream_wait(s);
     bs->d_tasks.ensure(T, s);
     launch_prefix_tasks(B.ext_off.p, G, nullptr, task_off, bs->d_tasks.p, bs->n_sms, s, true);
     GPA_CUDA(cudaMemsetAsync(bs->d_counts.p, 0, (size_t)M * 4, s));
@@ -360,7 +348,7 @@ bool count_device_batch(gpa_bitset* bs, DeviceBatch& B, uint32_t kernel, DeviceS
   launch_compact_blocks(d_recs.p, d_nrec, d_woff, n_win, window, bs->d_tblocks.p, d_brows, d_stats, s);
   uint32_t st3[3] = {0, 0, 0};
   GPA_CUDA(cudaMemcpyAsync(st3, d_stats, 12, cudaMemcpyDeviceToHost, s));
-  GPA_CUDA(cudaStreamSynchronize(s));
+  stream_wait(s);
   const uint32_t n_blocks = st3[1], max_rows = st3[0];
   device_exclusive_scan(d_brows, d_roff, n_blocks, d_stats + 2, scratch, s);
   launch_row_begin(d_roff, n_blocks, bs->d_tblocks.p, bs->n_sms, s);
@@ -505,6 +493,7 @@ extern "C" gpa_status gpa_bitset_create(const gpa_tx_csr* db, uint32_t row_min_c
                                         const gpa_options* opt, gpa_bitset** out) {
   return gpa::guard([&] {
     GPA_REQUIRE(out, GPA_ERR_INVALID, "out is NULL");
+    gpa::DistScope scope(dist);
     *out = gpa::bitset_build(db, row_min_count, dist, opt);
   });
 }
@@ -545,7 +534,7 @@ extern "C" gpa_status gpa_bitset_export(const gpa_bitset* bs, uint32_t* host_out
     gpa::use_device(bs->device);
     GPA_CUDA(cudaMemcpyAsync(host_out, bs->rows.p, (size_t)bs->n_rows * bs->pitch_words * 4, cudaMemcpyDeviceToHost,
                              bs->stream));
-    GPA_CUDA(cudaStreamSynchronize(bs->stream));
+    gpa::stream_wait(bs->stream);
   });
 }
 
@@ -560,18 +549,32 @@ extern "C" gpa_status gpa_count(gpa_bitset* bs, const uint32_t* cand, uint32_t k
     GPA_REQUIRE(M <= (UINT64_MAX / 8) / k && M < (1ull << 32), GPA_ERR_INVALID, "M * k overflows");
     gpa::dist_check(bs->dist);
     gpa::use_device(bs->device);
-    // validate + translate to row ids
+    gpa::DistScope scope(bs->dist);
+    // validate + translate to row ids; with dist the verdict is agreed across ranks before the
+    // counting collective (a rank-local rejection must not strand the others)
     std::vector<uint32_t> rows(M * k);
-    for (uint64_t m = 0; m < M; ++m) {
-      for (uint32_t j = 0; j < k; ++j) {
-        const uint32_t it = cand[m * k + j];
-        GPA_REQUIRE(it < bs->n_items, GPA_ERR_INVALID, "candidate %llu: item %u >= n_items", (unsigned long long)m, it);
-        GPA_REQUIRE(j == 0 || it > cand[m * k + j - 1], GPA_ERR_INVALID,
-                    "candidate %llu is not strictly increasing", (unsigned long long)m);
-        const int32_t r = bs->row_of_item[it];
-        GPA_REQUIRE(r >= 0, GPA_ERR_RANGE, "item %u has no bitset row", it);
-        rows[m * k + j] = (uint32_t)r;
+    uint32_t verdict[1] = {GPA_OK};
+    std::string why;
+    try {
+      for (uint64_t m = 0; m < M; ++m) {
+        for (uint32_t j = 0; j < k; ++j) {
+          const uint32_t it = cand[m * k + j];
+          GPA_REQUIRE(it < bs->n_items, GPA_ERR_INVALID, "candidate %llu: item %u >= n_items", (unsigned long long)m, it);
+          GPA_REQUIRE(j == 0 || it > cand[m * k + j - 1], GPA_ERR_INVALID,
+                      "candidate %llu is not strictly increasing", (unsigned long long)m);
+          const int32_t r = bs->row_of_item[it];
+          GPA_REQUIRE(r >= 0, GPA_ERR_RANGE, "item %u has no bitset row", it);
+          rows[m * k + j] = (uint32_t)r;
+        }
       }
+    } catch (const gpa::Error& e) {
+      verdict[0] = e.status;
+      why = e.msg;
+    }
+    gpa::dist_agree_max(bs->dist, verdict, 1);
+    if (verdict[0] != GPA_OK) {
+      if (!why.empty()) gpa::fail((gpa_status)verdict[0], "%s", why.c_str());
+      gpa::fail((gpa_status)verdict[0], "invalid candidates on another rank");
     }
     uint32_t kern = kernel == GPA_KERNEL_AUTO ? bs->opt.count_kernel : kernel;
     if (kern == GPA_KERNEL_PROJ) kern = GPA_KERNEL_AUTO;  // needs the level structure of gpa_mine
@@ -587,7 +590,7 @@ extern "C" gpa_status gpa_count(gpa_bitset* bs, const uint32_t* cand, uint32_t k
       std::vector<uint32_t> all(P);
       if (P) {
         GPA_CUDA(cudaMemcpyAsync(all.data(), bs->d_counts.p, P * 4, cudaMemcpyDeviceToHost, bs->stream));
-        GPA_CUDA(cudaStreamSynchronize(bs->stream));
+        gpa::stream_wait(bs->stream);
       }
       for (uint64_t m = 0; m < M; ++m) counts_out[m] = all[gpa::pair_index(rows[2 * m], rows[2 * m + 1], n)];
       return;
@@ -606,7 +609,7 @@ extern "C" gpa_status gpa_count(gpa_bitset* bs, const uint32_t* cand, uint32_t k
       b.ext_off[M] = M;
       gpa::count_grouped(bs, b, GPA_KERNEL_V0, nullptr);
       GPA_CUDA(cudaMemcpyAsync(counts_out, bs->d_counts.p, M * 4, cudaMemcpyDeviceToHost, bs->stream));
-      GPA_CUDA(cudaStreamSynchronize(bs->stream));
+      gpa::stream_wait(bs->stream);
       return;
     }
     // PREFIX / TRIE: group by (k-1)-prefix (sort candidate indices lexicographically)
@@ -633,7 +636,7 @@ extern "C" gpa_status gpa_count(gpa_bitset* bs, const uint32_t* cand, uint32_t k
     gpa::count_grouped(bs, b, kern, nullptr);
     std::vector<uint32_t> sorted(M);
     GPA_CUDA(cudaMemcpyAsync(sorted.data(), bs->d_counts.p, M * 4, cudaMemcpyDeviceToHost, bs->stream));
-    GPA_CUDA(cudaStreamSynchronize(bs->stream));
+    gpa::stream_wait(bs->stream);
     for (uint64_t i = 0; i < M; ++i) counts_out[order[i]] = sorted[i];
   });
 }

@@ -32,6 +32,55 @@ bool ingest_overlap_eligible(const gpa_tx_csr* db) {
          db->n_items <= 16384 && db->offsets && db->items;
 }
 
+std::vector<uint64_t> ingest_cuts(uint64_t n_tx) {
+  uint64_t ct = (n_tx + kIngestChunks - 1) / kIngestChunks;
+  ct = (ct + kIngestAlign - 1) / kIngestAlign * kIngestAlign;
+  std::vector<uint64_t> cut;
+  for (uint64_t t = 0; t < n_tx; t += ct) cut.push_back(t);
+  cut.push_back(n_tx);
+  return cut;
+}
+
+bool agree_input(const gpa_tx_csr* db, const gpa_dist* dist, bool want_overlap) {
+  enum : uint32_t { kBad = 1, kNoOverlap = 2 };
+  uint32_t flags = 0;
+  std::string why;
+  auto bad = [&](const char* m) {
+    if (!(flags & kBad)) why = m;
+    flags |= kBad;
+  };
+  if (!db) {
+    bad("db is NULL");
+  } else if (db->memory != GPA_MEM_HOST && db->memory != GPA_MEM_DEVICE) {
+    bad("db->memory must be GPA_MEM_HOST or GPA_MEM_DEVICE");
+  } else if (!db->offsets) {
+    bad("db->offsets is NULL");
+  } else if (db->memory == GPA_MEM_HOST) {
+    if (db->offsets[0] != 0) bad("offsets[0] must be 0");
+    else if (db->offsets[db->n_tx] > 0 && !db->items) bad("db->items is NULL");
+    else {
+      const std::vector<uint64_t> cut = ingest_cuts(db->n_tx);   // the upload sizes come from these
+      for (size_t c = 0; c + 1 < cut.size(); ++c)
+        if (db->offsets[cut[c + 1]] < db->offsets[cut[c]]) bad("offsets are not non-decreasing");
+    }
+  } else if (db->n_tx) {
+    uint64_t first = 0;
+    GPA_CUDA(cudaMemcpy(&first, db->offsets, sizeof(uint64_t), cudaMemcpyDeviceToHost));
+    if (first != 0) bad("offsets[0] must be 0");
+  }
+  if (!(want_overlap && ingest_overlap_eligible(db))) flags |= kNoOverlap;
+  const uint32_t n_items = db ? db->n_items : 0;
+  uint32_t v[3] = {flags, n_items, ~n_items};   // max of n_items and of its complement: max and min
+  dist_agree_max(dist, v, 3);
+  if (v[0] & kBad) {
+    if (flags & kBad) fail(GPA_ERR_INVALID, "%s", why.c_str());
+    fail(GPA_ERR_INVALID, "invalid input on another rank");
+  }
+  GPA_REQUIRE(v[1] == n_items && ~v[2] == n_items, GPA_ERR_INVALID, "ranks disagree on n_items (%u .. %u)", ~v[2],
+              v[1]);
+  return !(v[0] & kNoOverlap);
+}
+
 gpa_bitset* bitset_build_overlapped(const gpa_tx_csr* db, uint64_t row_min_count, const gpa_dist* dist,
                                     const gpa_options* opt_in, bool* pairs_ready, CountStats* pair_stats) {
   *pairs_ready = false;
@@ -71,19 +120,12 @@ gpa_bitset* bitset_build_overlapped(const gpa_tx_csr* db, uint64_t row_min_count
   const double t0 = wall_ms();
   const uint64_t n_tx = db->n_tx;
   const uint32_t n_items = db->n_items;
-  GPA_REQUIRE(db->offsets[0] == 0, GPA_ERR_INVALID, "offsets[0] must be 0");
   const uint64_t nnz = db->offsets[n_tx];
   bs->pitch_words = pitch_words_for(n_tx);
 
-  // chunk plan
-  uint64_t ct = (n_tx + kIngestChunks - 1) / kIngestChunks;
-  ct = (ct + kIngestAlign - 1) / kIngestAlign * kIngestAlign;
-  std::vector<uint64_t> cut;
-  for (uint64_t t = 0; t < n_tx; t += ct) cut.push_back(t);
-  cut.push_back(n_tx);
+  // chunk plan (agree_input checked offsets[0] and the monotonicity at the cuts on every rank)
+  const std::vector<uint64_t> cut = ingest_cuts(n_tx);
   const size_t C = cut.size() - 1;
-  for (size_t c = 0; c < C; ++c)
-    GPA_REQUIRE(db->offsets[cut[c + 1]] >= db->offsets[cut[c]], GPA_ERR_INVALID, "offsets are not non-decreasing");
 
   DBuf<uint64_t> d_off;
   DBuf<uint32_t> d_items, d_hist, d_flags;
@@ -96,7 +138,7 @@ gpa_bitset* bitset_build_overlapped(const gpa_tx_csr* db, uint64_t row_min_count
   GPA_CUDA(cudaMemsetAsync(d_hist.p, 0, n_items * 4, s));
   GPA_CUDA(cudaMemsetAsync(d_flags.p, 0, 4, s));
   GPA_CUDA(cudaMemcpyAsync(d_ntx.p, &bs->n_tx_local, 8, cudaMemcpyHostToDevice, s));
-  GPA_CUDA(cudaStreamSynchronize(s));  // the copy stream writes into these allocations
+  stream_wait(s);  // the copy stream writes into these allocations
   std::vector<cudaEvent_t> up(C, nullptr);
   struct EvGuard {
     std::vector<cudaEvent_t>& v;
@@ -131,7 +173,7 @@ gpa_bitset* bitset_build_overlapped(const gpa_tx_csr* db, uint64_t row_min_count
   GPA_CUDA(cudaMemcpyAsync(h0.data(), d_h0.p, n_items * 4, cudaMemcpyDeviceToHost, s));
   GPA_CUDA(cudaMemcpyAsync(&n0, d_n0.p, 8, cudaMemcpyDeviceToHost, s));
   GPA_CUDA(cudaMemcpyAsync(&n_global, d_ntx.p, 8, cudaMemcpyDeviceToHost, s));
-  GPA_CUDA(cudaStreamSynchronize(s));
+  stream_wait(s);
   // R0: chunk-0 count >= half the threshold scaled to the chunk (h0 * N * 2 >= theta * n0)
   std::vector<uint32_t> r0_items;
   std::vector<int32_t> r0_of_item(n_items, -1);
@@ -189,7 +231,7 @@ gpa_bitset* bitset_build_overlapped(const gpa_tx_csr* db, uint64_t row_min_count
   }
   uint32_t flags = 0;
   GPA_CUDA(cudaMemcpyAsync(&flags, d_flags.p, 4, cudaMemcpyDeviceToHost, s));
-  GPA_CUDA(cudaStreamSynchronize(s));
+  stream_wait(s);
   for (size_t c = 0; c < C; ++c)
     if (pe[2 * c]) {
       float ms = 0;
@@ -210,7 +252,7 @@ gpa_bitset* bitset_build_overlapped(const gpa_tx_csr* db, uint64_t row_min_count
   bs->item_counts.assign(n_items, 0);
   GPA_CUDA(cudaMemcpyAsync(bs->item_counts.data(), d_hist.p, n_items * 4, cudaMemcpyDeviceToHost, s));
   GPA_CUDA(cudaMemcpyAsync(&flags, d_flags.p, 4, cudaMemcpyDeviceToHost, s));
-  GPA_CUDA(cudaStreamSynchronize(s));
+  stream_wait(s);
   bs->n_tx_global = n_global;
   GPA_REQUIRE(!(flags & kFlagBadOffsets), GPA_ERR_INVALID, "offsets are not non-decreasing%s",
               dist ? " (on some rank)" : "");
@@ -266,7 +308,7 @@ gpa_bitset* bitset_build_overlapped(const gpa_tx_csr* db, uint64_t row_min_count
                           n_tx, s);
     }
   }
-  GPA_CUDA(cudaStreamSynchronize(s));
+  stream_wait(s);
   bs->build_ms[2] = wall_ms() - t2;
   if (trace_enabled())
     fprintf(stderr, "[gpa] overlapped ingest: %zu chunks, R0 = %u rows, L1 = %u rows (%s), upload+hist+build+pairs "

@@ -15,9 +15,15 @@
 #include "../kernels.h"
 
 struct gpa_dist {
-  ncclComm_t comm = nullptr;
+  ncclComm_t comm = nullptr;           // NCCL transport (gpa_dist_create)
+  gpa_host_allreduce_fn host_fn = nullptr;   // host-staged transport (gpa_dist_create_host)
+  void* host_ctx = nullptr;
   int rank = 0, world = 1, device = 0;
   bool failed = false;
+  double timeout_s = 600.0;
+  std::vector<uint64_t> log;           // (op << 60) | (dtype << 56) | n of every collective, in order
+  void* stage = nullptr;               // pinned staging of the host transport
+  size_t stage_bytes = 0;
 };
 
 namespace gpa {
@@ -28,11 +34,22 @@ struct DeviceInfo {
 };
 DeviceInfo use_device(int requested);   // cudaSetDevice + one-time pool setup
 
-// NCCL helpers (no-ops without dist)
+// Collective helpers (no-ops without dist; NCCL or the host-staged transport)
 void dist_check(const gpa_dist* d);
 void allreduce_sum_u32(const gpa_dist* d, uint32_t* buf, size_t n, cudaStream_t s);
 void allreduce_sum_u64(const gpa_dist* d, uint64_t* buf, size_t n, cudaStream_t s);
 void allreduce_max_u32(const gpa_dist* d, uint32_t* buf, size_t n, cudaStream_t s);
+// Element-wise max over ranks of a few host values (one small collective on a library stream of
+// the dist's device; identity without dist).  Every path decision that changes the collective
+// sequence goes through it so that all ranks take the same branch.
+void dist_agree_max(const gpa_dist* d, uint32_t* vals, size_t n);
+// While alive, waits on streams (stream_wait) of this thread poll d's NCCL communicator for
+// asynchronous errors and time out after d->timeout_s.
+struct DistScope {
+  const gpa_dist* prev;
+  explicit DistScope(const gpa_dist* d);
+  ~DistScope();
+};
 
 // Candidate batch grouped by (k-1)-prefix, in ROW ids.  Candidates are prefix + ext[j] for
 // j in [ext_off[g], ext_off[g+1]); global candidate index = position in ext.
@@ -101,6 +118,7 @@ struct CountStats {
   cudaEvent_t e0 = nullptr, e1 = nullptr, e2 = nullptr;
   cudaEvent_t ep = nullptr, eb = nullptr;  // GPA_KERNEL_PROJ: the list-building kernel (ep .. eb)
   uint64_t build_words = 0;
+  uint64_t build_bytes = 0, count_bytes = 0;   // GPA_KERNEL_PROJ: algorithmic bytes (gpa_level_stats)
 };
 
 }  // namespace gpa
@@ -135,12 +153,23 @@ struct gpa_bitset {
 
 namespace gpa {
 // Build the static bitset (histogram, rows, bitset) -- shared by gpa_bitset_create / gpa_mine.
-gpa_bitset* bitset_build(const gpa_tx_csr* db, uint64_t row_min_count, const gpa_dist* dist, const gpa_options* opt);
+// prechecked: the caller already ran agree_input for db (gpa_mine)
+gpa_bitset* bitset_build(const gpa_tx_csr* db, uint64_t row_min_count, const gpa_dist* dist, const gpa_options* opt,
+                         bool prechecked = false);
 void bitset_free(gpa_bitset* bs);
 // Host input, end to end: upload in transaction chunks overlapped with histogram, bitset build and
 // generation-2 pair counting (runtime/ingest.cpp).  *pairs_ready: bs->d_counts holds the L_1 pair
 // counts (pair_stats describes the kernels).
 bool ingest_overlap_eligible(const gpa_tx_csr* db);
+// transaction boundaries of the overlapped ingest's upload chunks: cut[0] = 0 .. cut.back() = n_tx
+std::vector<uint64_t> ingest_cuts(uint64_t n_tx);
+// Host-side input checks every rank runs BEFORE its first collective, agreed across ranks with one
+// small max all-reduce (a rank-local rejection must not strand the others inside a collective):
+// throws GPA_ERR_INVALID on every rank alike if any rank's input is malformed or the ranks disagree
+// on n_items.  Returns whether EVERY rank can take the overlapped ingest (want_overlap and
+// ingest_overlap_eligible on all ranks): a collective decision, so all ranks issue the same
+// collective sequence.
+bool agree_input(const gpa_tx_csr* db, const gpa_dist* dist, bool want_overlap);
 gpa_bitset* bitset_build_overlapped(const gpa_tx_csr* db, uint64_t row_min_count, const gpa_dist* dist,
                                     const gpa_options* opt, bool* pairs_ready, struct CountStats* pair_stats);
 // Count a grouped batch into bs->d_counts (device, M entries, summed over ranks).

@@ -92,7 +92,8 @@ void record_level(gpa_result* R, const gpa_bitset* bs, uint32_t k, const Grouped
 // (the sizes T, sm came back with |C_k|): the list build (pext) on s, overlapping the emitting
 // join on the auxiliary stream; the supports wait for both (aux_done).
 bool count_projected_staged(gpa_bitset* bs, uint32_t k, const DeviceBatch& B, DeviceProj& cur, const ProjPending& pp,
-                            const uint64_t T[2], const uint32_t sm[4], cudaEvent_t aux_done, CountStats* cs) {
+                            const uint64_t T[3], const uint32_t sm[4], cudaEvent_t aux_done, CountStats* cs,
+                            uint64_t src_words) {
   cudaStream_t s = bs->stream;
   const double t0 = now_ms();
   GPA_CUDA(cudaEventRecord(cs->e0, s));
@@ -106,6 +107,8 @@ bool count_projected_staged(gpa_bitset* bs, uint32_t k, const DeviceBatch& B, De
   GPA_CUDA(cudaMemsetAsync(bs->d_counts.p, 0, (size_t)B.M * 4, s));
   GPA_CUDA(cudaEventRecord(cs->eb, s));
   cs->build_words = cur.in_words;
+  cs->build_bytes = (src_words + cur.words) * 4;            // sources read once, lists written once
+  cs->count_bytes = cur.words * 4 + (uint64_t)B.M * 4;      // lists read once, counts written
   launch_count_proj(cur, B.gpar.p, B.ext_off.p, B.eidx.p, B.G, bs->d_counts.p, s);
   cs->kernel = GPA_KERNEL_PROJ;
   cs->launches = 1;
@@ -177,9 +180,13 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
 
   bool pairs_ready = false;
   CountStats pair_stats;
-  const bool overlap = !(opt.flags & GPA_NO_OVERLAP_INGEST) && ingest_overlap_eligible(db);
+  GPA_REQUIRE(db, GPA_ERR_INVALID, "db is NULL");   // a caller bug, not data: checked before any device work
+  dist_check(dist);
+  use_device(dist ? dist->device : opt.device);
+  // the ingest path is chosen collectively: every rank issues the same collective sequence
+  const bool overlap = agree_input(db, dist, !(opt.flags & GPA_NO_OVERLAP_INGEST));
   gpa_bitset* bs = overlap ? bitset_build_overlapped(db, min_count, dist, &opt, &pairs_ready, &pair_stats)
-                           : bitset_build(db, min_count, dist, &opt);
+                           : bitset_build(db, min_count, dist, &opt, true);
   struct BsGuard {
     gpa_bitset* b;
     ~BsGuard() { bitset_free(b); }
@@ -234,8 +241,7 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
   bool proj_on = !host_candgen && (opt.count_kernel == GPA_KERNEL_AUTO || opt.count_kernel == GPA_KERNEL_PROJ ||
                                    opt.count_kernel == GPA_KERNEL_PAIRS || opt.count_kernel == GPA_KERNEL_PAIRS_TC) &&
                  bs->pitch_words * 32ull < (1ull << 32);
-  if (const char* e = getenv("GPA_PROJ"))   // GPA_PROJ=0: complete intersection for k >= 3 under AUTO (comparisons)
-    if (atoi(e) == 0 && opt.count_kernel != GPA_KERNEL_PROJ) proj_on = false;
+  if (opt.flags & GPA_COMPLETE_INTERSECTION) proj_on = false;   // the paper's method for k >= 3
   struct Pending {       // a generation's frequent itemsets, still on the device
     size_t level = 0;
     uint32_t F = 0, k = 0;
@@ -262,15 +268,20 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
   Events aux_evs;            // [0] s -> aux (batch buffers sized), [1] aux done
   ProjPending ppend;
   bool aux_join = false;     // this generation's batch was emitted on aux_s
-  uint64_t pT[2] = {0, 0};
+  uint64_t pT[3] = {0, 0, 0};
   uint32_t psm[4] = {0, 0, 0, 0};
-  struct EvTriple {      // deferred timing of a generation's counting launch(es) and all-reduce
-    cudaEvent_t e[5] = {nullptr, nullptr, nullptr, nullptr, nullptr};  // + projected-list build [3, 4)
+  // deferred (device-side) timing of a generation on stream s: [5] generation start, [0] counting
+  // start, [1] counting end, [2] all-reduce end, [3, 4) projected-list build, [6] threshold end
+  struct EvTriple {
+    enum { kN = 7 };
+    cudaEvent_t e[kN] = {};
+    bool counted = false;   // e[0..2] recorded (not the generation counted during the overlapped ingest)
     EvTriple() {
       for (auto& x : e) GPA_CUDA(cudaEventCreate(&x));
     }
     EvTriple(EvTriple&& o) noexcept {
-      for (int i = 0; i < 5; ++i) std::swap(e[i], o.e[i]);
+      for (int i = 0; i < kN; ++i) std::swap(e[i], o.e[i]);
+      counted = o.counted;
     }
     EvTriple(const EvTriple&) = delete;
     ~EvTriple() {
@@ -286,6 +297,8 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
   uint64_t nL = bs->n_rows;
   for (uint32_t k = 2; k <= max_k && nL > 0; ++k) {
     double t0 = now_ms();
+    EvTriple& ev = events.emplace_back();
+    GPA_CUDA(cudaEventRecord(ev.e[5], s));
     CountStats cs;
     GroupedBatch batch;
     uint64_t M = 0, G = 0;
@@ -298,7 +311,7 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
       std::vector<uint32_t> Lh((size_t)Ld.n * (k - 1));
       if (Ld.n) {
         GPA_CUDA(cudaMemcpyAsync(Lh.data(), Ld.rows.p, Lh.size() * 4, cudaMemcpyDeviceToHost, s));
-        GPA_CUDA(cudaStreamSynchronize(s));
+        stream_wait(s);
       }
       batch = candgen_join_prune(Lh, Ld.n, k - 1);
       M = batch.size();
@@ -315,7 +328,7 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
         GPA_CUDA(cudaMemcpyAsync(Bd.prefix.p, batch.prefix.data(), batch.prefix.size() * 4, cudaMemcpyHostToDevice, s));
         GPA_CUDA(cudaMemcpyAsync(Bd.ext_off.p, off32.data(), (G + 1) * 4, cudaMemcpyHostToDevice, s));
         GPA_CUDA(cudaMemcpyAsync(Bd.ext.p, batch.ext.data(), M * 4, cudaMemcpyHostToDevice, s));
-        GPA_CUDA(cudaStreamSynchronize(s));
+        stream_wait(s);
       }
     } else if (proj_on) {
       aux_join = false;
@@ -329,18 +342,18 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
         uint32_t* hs = host_sizes();
         if (proj_build_begin(Ld.n, Ld.par_a.p, Ld.par_b.p, k == 3 ? nullptr : Pprev, bs->rows.p, bs->pitch_words,
                              bs->n_rows, scratch, bs->n_sms, aux_s.s, ppend)) {
-          GPA_CUDA(cudaMemcpyAsync(hs + 2, ppend.d_tot, 16, cudaMemcpyDeviceToHost, aux_s.s));
-          GPA_CUDA(cudaMemcpyAsync(hs + 6, ppend.d_small, 16, cudaMemcpyDeviceToHost, aux_s.s));
+          GPA_CUDA(cudaMemcpyAsync(hs + 2, ppend.d_tot, 24, cudaMemcpyDeviceToHost, aux_s.s));
+          GPA_CUDA(cudaMemcpyAsync(hs + 8, ppend.d_small, 16, cudaMemcpyDeviceToHost, aux_s.s));
         } else {
           proj_on = false;   // lists not addressable: complete intersection from this generation on
         }
         GPA_CUDA(cudaMemcpyAsync(hs, d_sizes, 8, cudaMemcpyDeviceToHost, s));
-        GPA_CUDA(cudaStreamSynchronize(s));
-        GPA_CUDA(cudaStreamSynchronize(aux_s.s));
+        stream_wait(s);
+        stream_wait(aux_s.s);
         M = hs[0];
         G = hs[1];
-        std::memcpy(pT, hs + 2, 16);
-        std::memcpy(psm, hs + 6, 16);
+        std::memcpy(pT, hs + 2, 24);
+        std::memcpy(psm, hs + 8, 16);
         device_candgen_finish(Ld, Bd, scratch, bs->n_sms, s, (uint32_t)M, (uint32_t)G, aux_s.s, aux_evs.e[0]);
         GPA_CUDA(cudaEventRecord(aux_evs.e[1], aux_s.s));
         aux_join = true;
@@ -351,9 +364,10 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
       G = Bd.G;
     }
     double t1 = now_ms();
-    R->phase_ms[GPA_PHASE_CANDGEN] += t1 - t0;
-    if (M == 0) break;
-    EvTriple& ev = events.emplace_back();
+    if (M == 0) {
+      events.pop_back();
+      break;
+    }
     cs.e0 = ev.e[0];
     cs.e1 = ev.e[1];
     cs.e2 = ev.e[2];
@@ -370,16 +384,16 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
       GPA_CUDA(cudaMemcpyAsync(batch.prefix.data(), Bd.prefix.p, G * (k - 1) * 4, cudaMemcpyDeviceToHost, s));
       GPA_CUDA(cudaMemcpyAsync(off32.data(), Bd.ext_off.p, (G + 1) * 4, cudaMemcpyDeviceToHost, s));
       GPA_CUDA(cudaMemcpyAsync(batch.ext.data(), Bd.ext.p, M * 4, cudaMemcpyDeviceToHost, s));
-      GPA_CUDA(cudaStreamSynchronize(s));
+      stream_wait(s);
       batch.ext_off.assign(off32.begin(), off32.end());
     };
     if (k == 2 && pairs_ready && pairs_kernel_k2(opt.count_kernel)) {
       cs = pair_stats;  // counted during the overlapped ingest
-      events.pop_back();
     } else if (k == 2) {
       count_all_pairs(bs, opt.count_kernel, &cs);
     } else {
-      if (proj_on && count_projected_staged(bs, k, Bd, *Pcur, ppend, pT, psm, aux_evs.e[1], &cs)) {
+      const uint64_t src_words = k == 3 ? (uint64_t)bs->n_rows * bs->pitch_words : Pprev->words;
+      if (proj_on && count_projected_staged(bs, k, Bd, *Pcur, ppend, pT, psm, aux_evs.e[1], &cs, src_words)) {
         std::swap(Pprev, Pcur);
       } else {
         // complete intersection from the static bitset (requested, or the projected lists did not
@@ -394,7 +408,6 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     }
     if (keep && k > 2) fetch_batch();
     double t2 = now_ms();
-    R->phase_ms[GPA_PHASE_COUNT] += t2 - t1;
 
     const uint32_t F = device_threshold(bs->d_counts.p, (uint32_t)M, (uint32_t)min_count, k, bs->n_rows, Bd.prefix.p,
                                         Bd.ext_off.p, Bd.ext.p, (uint32_t)G, host_candgen ? nullptr : Bd.gpar.p,
@@ -420,11 +433,13 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
       pd.h_items = hi;
       pd.h_sup = hs;
     }
+    ev.counted = cs.e0 != nullptr;
+    GPA_CUDA(cudaEventRecord(ev.e[6], s));
     std::vector<uint32_t> counts;
     if (keep) {
       counts.resize(M);
       GPA_CUDA(cudaMemcpyAsync(counts.data(), bs->d_counts.p, M * 4, cudaMemcpyDeviceToHost, s));
-      GPA_CUDA(cudaStreamSynchronize(s));
+      stream_wait(s);
     }
     const double tr0 = now_ms();
     record_level(R, bs, k, k > 2 ? &batch : nullptr, M, {}, {}, keep, keep ? &counts : nullptr);
@@ -436,7 +451,7 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
       fprintf(stderr, "[gpa] k=%u M=%llu G=%llu: candgen %.2f ms, count phase %.2f ms, threshold %.2f ms (record %.2f) "
               "-> |L|=%u\n", k, (unsigned long long)M, (unsigned long long)G, t1 - t0, t2 - t1, now_ms() - t2,
               now_ms() - tr0, F);
-    if (cs.e0) event_level.push_back(R->levels.size() - 1);
+    event_level.push_back(R->levels.size() - 1);
     gpa_level_stats& st = R->levels.back().stats;
     st.n_cand = M;
     st.n_freq = F;
@@ -447,29 +462,43 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     st.allreduce_ms = cs.allreduce_ms;
     st.candgen_ms = t1 - t0;
     st.build_words = cs.build_words;
-    R->phase_ms[GPA_PHASE_THRESHOLD] += now_ms() - t2;
+    st.build_bytes = cs.build_bytes;
+    st.count_bytes = cs.count_bytes;
   }
 
   // ---- deferred: kernel times and the frequent itemsets of every generation
   const double tf0 = now_ms();
-  GPA_CUDA(cudaStreamSynchronize(s));
-  GPA_CUDA(cudaStreamSynchronize(copy_s.s));
+  stream_wait(s);
+  stream_wait(copy_s.s);
   const double tf1 = now_ms();
+  // phases of the level loop from the events on s (device time, contiguous per generation):
+  // candidate generation = generation start -> counting start, counting (+ all-reduce) = counting
+  // start -> all-reduce end, threshold = all-reduce end -> threshold end
   for (size_t i = 0; i < event_level.size(); ++i) {
-    float a = 0, b = 0;
-    GPA_CUDA(cudaEventElapsedTime(&a, events[i].e[0], events[i].e[1]));
-    GPA_CUDA(cudaEventElapsedTime(&b, events[i].e[1], events[i].e[2]));
-    gpa_level_stats& st0 = R->levels[event_level[i]].stats;
-    if (st0.kernel == GPA_KERNEL_PROJ) {
-      float c = 0;
-      GPA_CUDA(cudaEventElapsedTime(&c, events[i].e[3], events[i].e[4]));
-      st0.build_ms = c;
-      GPA_CUDA(cudaEventElapsedTime(&c, events[i].e[0], events[i].e[3]));
-      st0.setup_ms = c;
-    }
+    const EvTriple& E = events[i];
     gpa_level_stats& st = R->levels[event_level[i]].stats;
+    float g = 0;
+    GPA_CUDA(cudaEventElapsedTime(&g, E.e[5], E.e[6]));
+    if (!E.counted) {   // generation 2 counted during the overlapped ingest: stats from the ingest
+      R->phase_ms[GPA_PHASE_THRESHOLD] += g;
+      continue;
+    }
+    float a = 0, b = 0, cg = 0;
+    GPA_CUDA(cudaEventElapsedTime(&a, E.e[0], E.e[1]));
+    GPA_CUDA(cudaEventElapsedTime(&b, E.e[1], E.e[2]));
+    GPA_CUDA(cudaEventElapsedTime(&cg, E.e[5], E.e[0]));
+    if (st.kernel == GPA_KERNEL_PROJ) {
+      float c = 0;
+      GPA_CUDA(cudaEventElapsedTime(&c, E.e[3], E.e[4]));
+      st.build_ms = c;
+      GPA_CUDA(cudaEventElapsedTime(&c, E.e[0], E.e[3]));
+      st.setup_ms = c;
+    }
     st.count_ms = a;
     st.allreduce_ms = dist ? b : 0.0;
+    R->phase_ms[GPA_PHASE_CANDGEN] += cg;
+    R->phase_ms[GPA_PHASE_COUNT] += a + b;
+    R->phase_ms[GPA_PHASE_THRESHOLD] += g - cg - a - b;
   }
   parallel_for(pending.size(), [&](size_t i) {
     const Pending& pd = pending[i];
@@ -500,6 +529,7 @@ extern "C" gpa_status gpa_mine(const gpa_tx_csr* db, uint64_t min_count, const g
                                gpa_result** out) {
   return gpa::guard([&] {
     GPA_REQUIRE(out, GPA_ERR_INVALID, "out is NULL");
+    gpa::DistScope scope(dist);
     *out = gpa::mine(db, min_count, dist, opt);
   });
 }

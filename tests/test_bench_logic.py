@@ -1,0 +1,52 @@
+"""bench.py's roofline arithmetic on a synthetic result (CPU): every reported fraction must be
+reproducible from the line's own fields (achieved = algorithmic work or bytes / event time,
+frac = achieved / peak), and the longest launch is the one reported."""
+import types
+
+import pytest
+
+import bench
+
+PEAKS = {"hbm_gbs": 6551.4, "bf16_tflops": 1641.7, "sm_max_mhz": 1965.0}
+
+
+def fake_result(n_tx):
+    L = lambda k, n_cand, n_freq, kern, **st: types.SimpleNamespace(
+        k=k, n_cand=n_cand, n_freq=n_freq, stats=dict(kernel_name=kern, **st))
+    levels = [L(1, 1000, 900, "v0"), L(2, 404_550, 5000, "pairs_tc"), L(3, 20_000, 9000, "proj"),
+              L(4, 15_000, 8000, "trie")]
+    return types.SimpleNamespace(levels=levels, n_tx=n_tx, cand_tx=sum(l.n_cand for l in levels[1:]) * n_tx)
+
+
+def test_roofline_records_reproducible():
+    n_tx = 10_000_000
+    res = fake_result(n_tx)
+    st = {2: dict(kernel_name="pairs_tc", count_ms=4.0, build_ms=0.0, setup_ms=0.0, allreduce_ms=0.0),
+          3: dict(kernel_name="proj", count_ms=6.0, build_ms=4.5, setup_ms=0.5, allreduce_ms=0.0,
+                  build_bytes=2_400_000_000, count_bytes=1_200_000_000),
+          4: dict(kernel_name="trie", count_ms=1.0, build_ms=0.0, setup_ms=0.0, allreduce_ms=0.0)}
+    recs = bench.roofline_records(res, st, n_tx, PEAKS, 1965.0)
+    by = {(r["kernel"], r["k"]): r for r in recs}
+    tc = by[("pairs_tc", 2)]
+    assert tc["bound"] == "tensor" and tc["peak"] == pytest.approx(2 * 1641.7)
+    assert tc["achieved"] == pytest.approx(2 * 404_550 * n_tx / 4e-3 / 1e12)
+    px = by[("lists", 3)]
+    assert px["bound"] == "hbm" and px["achieved"] == pytest.approx(2.4e9 / 4.5e-3 / 1e9)
+    cp = by[("count_proj", 3)]
+    assert cp["kernel_ms"] == pytest.approx(1.0) and cp["achieved"] == pytest.approx(1.2e9 / 1e-3 / 1e9)
+    tr = by[("trie", 4)]
+    assert tr["bound"] == "alu" and tr["peak"] == pytest.approx(148 * 16 * 32 * 1965e6 / 1e12)
+    for r in recs:
+        assert r["frac"] == pytest.approx(r["achieved"] / r["peak"])
+        x = dict(r)
+        bench.rescale(x)
+        assert x["frac"] == pytest.approx(r["frac"])
+    agg = bench.aggregate_by_kernel(recs)
+    assert agg["pairs_tc"]["kernel_ms"] == pytest.approx(4.0) and agg["lists"]["launches"] == 1
+
+
+def test_pitch_bytes_matches_library_rule():
+    assert bench.pitch_bytes(1) == 4096
+    assert bench.pitch_bytes(32768) == 4096
+    assert bench.pitch_bytes(32769) == 8192
+    assert bench.pitch_bytes(10_000_000) == 1_253_376

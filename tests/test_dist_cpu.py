@@ -91,3 +91,44 @@ def test_shard_ranges_many_worlds():
             assert r[0][0] == 0 and r[-1][1] == n_tx
             for (a, b), (c, d) in zip(r, r[1:]):
                 assert b == c and b % 512 == 0
+
+
+def _host_allreduce_worker(rank, world, port, out_q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    tdist.init_process_group("gloo", rank=rank, world_size=world)
+    import sys
+    sys.path.insert(0, ROOT)
+    import paper_conf_cluster_zhangzb11a_b200 as gpa
+    # the values the library sends: counts (u32 sums near / above 2^31), flags and n_items
+    # agreement (u32 max incl. complements ~n), N (u64 sums)
+    a = np.array([2 ** 31 + rank, 7 * rank, 0xFFFFFFFF - rank, 1], dtype=np.uint32)
+    b = np.array([5 + rank, 2 ** 32 - 10 * (rank + 1)], dtype=np.uint32)
+    c = np.array([2 ** 40 + rank, 2 ** 63 + rank], dtype=np.uint64)
+    d = np.array([2 ** 63 + rank, rank], dtype=np.uint64)
+    gpa.torch_host_allreduce(a, "max")
+    gpa.torch_host_allreduce(b, "sum")
+    gpa.torch_host_allreduce(c, "sum")
+    gpa.torch_host_allreduce(d, "max")
+    out_q.put((rank, a.tolist(), b.tolist(), c.tolist(), d.tolist()))
+    tdist.destroy_process_group()
+
+
+def test_host_transport_callback_unsigned_semantics():
+    """The host-staged transport's callback (gpa_dist_create_host over gloo, used by the world-2
+    GPU test): element-wise unsigned max and wrap-around sums of u32 / u64 arrays across 2 ranks."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = free_port()
+    ps = [ctx.Process(target=_host_allreduce_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in ps:
+        p.start()
+    res = [q.get(timeout=120) for _ in ps]
+    for p in ps:
+        p.join(60)
+        assert p.exitcode == 0
+    want_a = [2 ** 31 + 1, 7, 0xFFFFFFFF, 1]
+    want_b = [5 + 6, (2 ** 32 - 10 + 2 ** 32 - 20) % 2 ** 32]
+    want_c = [2 ** 41 + 1, (2 ** 64 + 1) % 2 ** 64]
+    want_d = [2 ** 63 + 1, 1]
+    for _, a, b, c, d in res:
+        assert a == want_a and b == want_b and c == want_c and d == want_d
