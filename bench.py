@@ -246,8 +246,8 @@ def roofline_records(res, stats_avg: dict, n_tx: int, peaks: dict, sm_max: float
     traffic, ...}.  achieved = ALGORITHMIC work / the launch's CUDA-event time:
       pairs_tc        tensor: 2 |C_2| N int8 ops against the int8 dense peak = 2 x the measured bf16
                       burst peak (MEASURED_PEAKS.json; nominal int8 : bf16 = 4.5 : 2.25)
-      lists           hbm: the projected-list build (positions + ballot gather): every source list read
-                      once + the new lists written once (build_bytes)
+      lists           hbm: the projected-list build (pext3 / pext): every source list read once + the
+                      new lists written once (build_bytes)
       count_proj      hbm: the lists of L_{k-1} read once + the counts written (count_bytes)
       pairs / trie / prefix / v0   alu: |C_k| N cand*tx against the POPC (XU) pipe: 148 SM x 16 /clk
                       (measured, profiles/r01_microbench_popc.txt) / POPC-per-word x 32 tx x f_SM
@@ -292,7 +292,8 @@ def roofline_records(res, stats_avg: dict, n_tx: int, peaks: dict, sm_max: float
                      "peak_basis": f"POPC (XU) pipe: 148 SM x 16 /clk / {ppw} POPC per 32-tx word x 32 x "
                                    f"{sm_max:.0f} MHz"})
     for r in recs:
-        t = traffic_entry("gather_kernel" if r["kernel"] == "lists" else r["kernel"], r["k"])
+        t = traffic_entry(("pext3_kernel" if r["k"] == 3 else "pext_kernel") if r["kernel"] == "lists" else r["kernel"],
+                          r["k"])
         r["traffic"] = t.get("dram_bytes") if t else None
         if t and "issue_active" in t:
             r["issue_active"] = t["issue_active"]

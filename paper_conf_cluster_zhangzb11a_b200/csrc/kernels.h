@@ -142,27 +142,29 @@ uint64_t device_rules(const uint32_t* items, const uint64_t* item_off, const uin
 // ---- projected vertical lists (proj.cu; "equivalent class clustering", P13@2288-2486)
 // For every entry j of a level L (n entries with parents par_a / par_b): the bits of its last
 // item's row restricted to the transactions of its class (the entries with the same par_a), in
-// the class' position order (natural bit order, segments of 2,048 words padded to whole words,
-// lists padded with zeros to a multiple of 4 words).  Entries of single-member classes (no
-// candidates) get no list.  Buffers are persistent and grow-only (PBuf): one DeviceProj pair per
-// thread and device lives across generations and mining calls (proj_lists()).
+// the class' position order.  Entries of single-member classes (no candidates) get no vector.
+// Buffers are persistent and grow-only (PBuf): one DeviceProj pair per thread and device lives
+// across generations and mining calls (proj_lists()).
 struct DeviceProj {
   uint32_t n = 0;
-  PBuf<uint64_t> off;     // n: word offset of entry j's list in data
-  PBuf<uint32_t> nw;      // n: words of entry j's list (multiple of 4; 0 = none)
+  PBuf<uint64_t> off;     // n: word offset of entry j's vector in data
+  PBuf<uint32_t> nw;      // n: words of entry j's vector (multiple of 32; 0 = none)
   PBuf<uint32_t> data;
   uint64_t words = 0;
-  uint32_t max_nw = 0;    // longest list (words)
-  uint32_t max_lw = 0;    // ceil(max_nw / 32)
-  uint64_t in_words = 0;  // mask words x members the build covered (algorithmic work of the old compress)
+  uint32_t max_lw = 0;    // longest lane stream (words) of any class
+  uint64_t in_words = 0;  // mask words x members compressed to build these lists (algorithmic work)
 };
 // The calling thread's two DeviceProj for `device` (previous / current generation).
 DeviceProj* proj_lists(int device);
-// Lists of L = L_{k-1} from the previous level's lists (prev = those of L_{k-2}) or, for L = L_2
-// (prev == nullptr), from the bitset rows -- in two stages around one host read of the sizes: begin
-// enqueues the class tables and leaves the totals on the device (pp.d_tot: u64[3] = gather items,
-// list words, mask positions; pp.d_small: u32[4] = classes, longest list, mask words x members lo /
-// hi), finish (given those values) sizes the lists and launches the position and gather kernels.
+// Vectors of L = L_{k-1} from the previous level's vectors (prev = those of L_{k-2}) or, for
+// L = L_2 (prev == nullptr), from the bitset rows.  Synchronises once (sizes).  Returns false
+// when the vectors do not fit (device memory / 32-bit totals): use complete intersection.
+bool proj_build(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const DeviceProj* prev,
+                const uint32_t* rows, uint64_t pitch_words, uint32_t n_rows, DeviceProj& out, DeviceScratch& scratch,
+                int n_sms, cudaStream_t s, cudaEvent_t ev_build = nullptr);
+// The same in two stages around one host read of the sizes: begin enqueues the class tables and
+// leaves the totals on the device (pp.d_tot: u64[2] = pext items, list words; pp.d_small: u32[4]),
+// finish (given those values) sizes the lists and launches the list build.
 struct ProjPending {
   uint32_t n = 0, cmax = 0, nseg = 0, n_pairs = 0;
   int device = 0;
@@ -172,13 +174,12 @@ struct ProjPending {
   const uint64_t* d_tot = nullptr;
   const uint32_t* d_small = nullptr;
 };
-// begin returns false (nothing enqueued) when the lists cannot be addressed (bitset or previous
-// lists >= 2^32 words, too many classes): use complete intersection.  finish returns false when
-// they do not fit (device memory, 32-bit totals).
+// begin returns false (nothing enqueued) when the lists cannot be addressed (bitset >= 2^32 words,
+// too many classes): use complete intersection.
 bool proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const DeviceProj* prev,
                       const uint32_t* rows, uint64_t pitch_words, uint32_t n_rows, DeviceScratch& scratch, int n_sms,
                       cudaStream_t s, ProjPending& pp);
-bool proj_build_finish(const ProjPending& pp, const uint64_t T[3], const uint32_t sm[4], DeviceProj& out, int n_sms,
+bool proj_build_finish(const ProjPending& pp, const uint64_t T[2], const uint32_t sm[4], DeviceProj& out, int n_sms,
                        cudaStream_t s, cudaEvent_t ev_build);
 // counts[m] += popc(V_gpar[g] & V_eidx[m]) for every candidate m of group g (counts zeroed by the caller)
 void launch_count_proj(const DeviceProj& P, const uint32_t* gpar, const uint32_t* ext_off, const uint32_t* eidx,

@@ -17,21 +17,20 @@
 // the same popcount-of-AND as complete intersection (P18@394), over supp(Q) bits instead of N.
 // The next generation's lists follow from this one's: the class of X' = Q u {a, b} is Q u {a},
 // whose transactions are the set bits of V_{Q u {a}}; hence V_{X'} = the bits of V_{Q u {b}} at
-// the set positions of V_{Q u {a}} (a parallel bit extract).  Generation 3 starts from the static
+// the set positions of V_{Q u {a}}: a parallel bit extract, pext(V_{Q u {b}}, V_{Q u {a}}),
+// word by word (pext_kernel; Hacker's Delight "compress", the mask-dependent half computed once
+// per mask word and shared by a warp's group of up to 8 members of the class).  Generation 3 starts from the static
 // bitset itself: the class of a pair {a, b} is {a}, mask = row a, sources = rows b (the "static
 // bitset" of P2@270 / P18@755 stays the only input).
 //
-// B200 design: POSITIONS ONCE PER CLASS, THEN A BALLOT GATHER PER MEMBER.  A class' mask is cut
-// into segments of kSegW words (65,536 bits); pos_kernel writes the set-bit positions of each
-// (class, segment) once (u16, segment-relative); gather_kernel then gives each warp a (class,
-// segment, group of <= 16 members) item: per round of 32 positions, lane l holds position 32r + l,
-// loads its word of each member's source list (L1 gather: the 32 positions of a round span a
-// few 128-byte lines) and one ballot packs the 32 selected bits into the member's next output
-// word.  Work ~ output words (~5 instructions per member and output word), independent of the
-// mask's density, with no per-word bit-compress network and no per-member re-ranking of the mask.
-// Lists are in natural order (bit i = word i/32, bit i%32), each segment padded to whole words
-// and each list to a multiple of 4 words (zero padding is common to the class, so it is never
-// selected and never counted).  All integer; counts are exact by construction.
+// Layout: LANE-INTERLEAVED.  A vector is 32 bit streams ("lanes") of Lw words each, word j of
+// lane l at index 32 j + l; a bitset row is such a vector with Lw = pitch / 32.  Lane l of a new
+// vector is the pext of lane l of its source by lane l of its mask, so a warp's lane l only ever
+// touches lane l: every load is a coalesced 128-byte row, no cross-lane bit placement.  The
+// members of a class share one mask, hence one per-lane bit count and one layout: Lw_c = max
+// over lanes of the lane's words (each lane's tail zero-padded), members contiguous.  A bitset
+// mask is cut into segments of kSegJ words per lane (every level), each lane padded to whole words
+// per segment, so segments are independent work items.  All integer; counts are exact by construction.
 #include <cstdint>
 #include <cstdlib>
 #include <map>
@@ -44,8 +43,9 @@ namespace gpa {
 namespace {
 
 constexpr int kT = 256;
-constexpr uint32_t kSegW = 2048;     // mask segment: 2,048 words = 65,536 bits (u16 positions)
-constexpr uint32_t kGroup = 16;      // members per gather item
+constexpr uint32_t kSegJ = 128;          // mask segment: 128 words per lane (a bitset row: 131,072 transactions)
+constexpr uint32_t kMemberGroup = 8;     // members sharing one mask preparation in pext_kernel
+constexpr uint32_t kG3Group = 16;        // members sharing one chunk's bit ranks in pext3_kernel
 
 unsigned grid_for(uint64_t n, int n_sms, int per_sm = 16) {
   uint64_t g = (n + kT - 1) / kT;
@@ -72,27 +72,35 @@ __global__ void cls_bound_kernel(const uint32_t* __restrict__ flag, const uint32
   }
 }
 
-// The mask of a class / the source of a member: a bitset row (generation 3) or one of the
-// previous generation's lists.  Word offsets are 32-bit (checked by proj_build_begin).
-struct Src {
-  const uint32_t* base;        // rows (generation 3) or the previous lists' data
-  uint64_t pitch;              // generation 3: row pitch (words); 0: lists
-  const uint64_t* off;         // lists: word offset of each list
-  const uint32_t* nw;          // lists: words of each list
-  __device__ __forceinline__ uint32_t offset(uint32_t id) const {
-    return pitch ? (uint32_t)(id * pitch) : (uint32_t)off[id];
-  }
-  __device__ __forceinline__ uint32_t words(uint32_t id) const { return pitch ? (uint32_t)pitch : nw[id]; }
+struct VecRef {
+  const uint32_t* p;
+  uint32_t lw;  // words per lane
 };
 
-__device__ __forceinline__ uint32_t n_segs(uint32_t words) { return (words + kSegW - 1) / kSegW; }
+// The mask of a class / the source of a member: a bitset row (generation 3) or one of the
+// previous generation's vectors.
+struct Src {
+  const uint32_t* rows;        // non-null: generation 3
+  uint64_t pitch;
+  const uint32_t* data;        // previous generation's vectors
+  const uint64_t* off;
+  const uint32_t* nw;
+  __device__ __forceinline__ VecRef vec(uint32_t id) const {
+    if (rows) return VecRef{rows + (uint64_t)id * pitch, (uint32_t)(pitch / 32)};
+    return VecRef{data + off[id], nw[id] / 32u};
+  }
+};
 
-// warp per (segment s, class c) pair p = s * cmax + c: set bits of the class mask in segment s
-// -> npos[p] and its output words wseg[p] = ceil(npos / 32); in_words += mask words x members
-__global__ void seg_count_kernel(Src src, const uint32_t* __restrict__ par_a, const uint32_t* __restrict__ bound,
-                                 const uint32_t* __restrict__ n_cls, uint32_t cmax, uint32_t n_pairs,
-                                 uint32_t* __restrict__ npos, uint32_t* __restrict__ wseg,
-                                 unsigned long long* __restrict__ in_words) {
+__device__ __forceinline__ void seg_range(uint32_t lw, uint32_t s, uint32_t& j0, uint32_t& j1) {
+  j0 = min(lw, s * kSegJ);
+  j1 = min(lw, j0 + kSegJ);
+}
+
+// warp per (segment s, class c) pair p = s * cmax + c: lane l's mask popcount in the segment ->
+// words[p][l] = its output words (bits rounded up to whole words)
+__global__ void seg_popc_kernel(Src src, const uint32_t* __restrict__ par_a, const uint32_t* __restrict__ bound,
+                                const uint32_t* __restrict__ n_cls, uint32_t cmax, uint32_t nseg, uint32_t n_pairs,
+                                uint32_t* __restrict__ words, unsigned long long* __restrict__ in_words) {
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t p = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   if (p >= n_pairs) return;
@@ -101,53 +109,48 @@ __global__ void seg_count_kernel(Src src, const uint32_t* __restrict__ par_a, co
   if (c < *n_cls) {
     const uint32_t j0 = bound[c], m = bound[c + 1] - j0;
     if (m >= 2) {
-      const uint32_t mid = par_a[j0];
-      const uint32_t W = src.words(mid);
-      const uint32_t w0 = s * kSegW, w1 = min(W, w0 + kSegW);
-      const uint32_t* mk = src.base + src.offset(mid);
-      for (uint32_t w = w0 + 4 * lane; w < w1; w += 128) {   // W is a multiple of 4
-        const uint4 v = __ldg(reinterpret_cast<const uint4*>(mk + w));
-        cnt += __popc(v.x) + __popc(v.y) + __popc(v.z) + __popc(v.w);
-      }
-      if (lane == 0 && w1 > w0) atomicAdd(in_words, (unsigned long long)(w1 - w0) * m);
+      const VecRef mk = src.vec(par_a[j0]);
+      uint32_t a, b;
+      seg_range(mk.lw, s, a, b);
+      for (uint32_t j = a; j < b; ++j) cnt += __popc(mk.p[32ull * j + lane]);
+      if (lane == 0 && b > a) atomicAdd(in_words, 32ull * (b - a) * m);
     }
   }
-  cnt = __reduce_add_sync(0xffffffffu, cnt);
+  words[(uint64_t)p * 32 + lane] = (cnt + 31) / 32;
+}
+
+// warp per class: lane l's word offset of every segment (loc), Lw_c = max over lanes of the
+// lane's total, words per member nwc = 32 Lw_c, the class' words and its pext items (one per
+// segment and group of kMemberGroup members)
+__global__ void cls_pad_kernel(const uint32_t* __restrict__ words, const uint32_t* __restrict__ bound,
+                               const uint32_t* __restrict__ n_cls, uint32_t cmax, uint32_t nseg,
+                               uint32_t* __restrict__ loc, uint32_t* __restrict__ nwc,
+                               uint64_t* __restrict__ cls_words, uint32_t* __restrict__ items,
+                               uint32_t* __restrict__ max_lw) {
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  if (c >= cmax) return;
+  uint32_t m = 0;
+  if (c < *n_cls) m = bound[c + 1] - bound[c];
+  const uint32_t groups = m >= 2 ? (m + kMemberGroup - 1) / kMemberGroup : 0;
+  uint32_t acc = 0;
+  for (uint32_t s = 0; s < nseg; ++s) {
+    const uint64_t p = (uint64_t)s * cmax + c;
+    loc[p * 32 + lane] = acc;
+    const uint32_t w = words[p * 32 + lane];
+    acc += w;
+    const bool any = __any_sync(0xffffffffu, w != 0);
+    if (lane == 0) items[p] = any ? groups : 0;
+  }
+  const uint32_t lw = __reduce_max_sync(0xffffffffu, acc);
   if (lane == 0) {
-    npos[p] = cnt;
-    wseg[p] = (cnt + 31) / 32;
+    nwc[c] = groups ? 32u * lw : 0u;
+    cls_words[c] = groups ? (uint64_t)32u * lw * m : 0ull;
+    if (groups && lw) atomicMax(max_lw, lw);
   }
 }
 
-// thread per class: the output word offset of every segment of the class (loc), words per member
-// nwc = the class total rounded up to 4 words (uint4 loads of count_proj), the class' words, its
-// segments and its gather items (one per segment of the mask and group of <= kGroup members)
-__global__ void cls_pad_kernel(Src src, const uint32_t* __restrict__ par_a, const uint32_t* __restrict__ wseg,
-                               const uint32_t* __restrict__ bound, const uint32_t* __restrict__ n_cls, uint32_t cmax,
-                               uint32_t nseg, uint32_t* __restrict__ loc, uint32_t* __restrict__ nwc,
-                               uint32_t* __restrict__ cls_nseg, uint64_t* __restrict__ cls_words,
-                               uint32_t* __restrict__ items, uint32_t* __restrict__ max_nw) {
-  const uint32_t C = *n_cls;
-  for (uint32_t c = blockIdx.x * blockDim.x + threadIdx.x; c < cmax; c += gridDim.x * blockDim.x) {
-    const uint32_t m = c < C ? bound[c + 1] - bound[c] : 0;
-    const uint32_t groups = m >= 2 ? (m + kGroup - 1) / kGroup : 0;
-    const uint32_t ns = groups ? n_segs(src.words(par_a[bound[c]])) : 0;
-    uint32_t acc = 0;
-    for (uint32_t s = 0; s < nseg; ++s) {
-      const uint64_t p = (uint64_t)s * cmax + c;
-      loc[p] = acc;
-      acc += wseg[p];
-      items[p] = s < ns ? groups : 0;
-    }
-    const uint32_t words = groups ? (acc + 3u) & ~3u : 0u;
-    nwc[c] = words;
-    cls_nseg[c] = ns;
-    cls_words[c] = (uint64_t)words * m;
-    if (words) atomicMax(max_nw, words);
-  }
-}
-
-// entry j -> its list (offset, words); entries of single-member classes get none
+// entry j -> its vector (offset, words); entries of single-member classes get none
 __global__ void entry_off_kernel(const uint32_t* __restrict__ flag, const uint32_t* __restrict__ ex,
                                  const uint32_t* __restrict__ bound, const uint32_t* __restrict__ nwc,
                                  const uint64_t* __restrict__ cls_base, uint32_t n, uint64_t* __restrict__ off,
@@ -165,40 +168,335 @@ __global__ void entry_off_kernel(const uint32_t* __restrict__ flag, const uint32
   }
 }
 
-// warp per pair p with set bits: the segment-relative positions (word << 5 | bit, u16) of the
-// class mask's set bits in segment s, in increasing order, at pos + pos_off[p].  128 words per
-// step (a uint4 per lane), ranks by a warp scan of the per-lane popcounts.
-__global__ void pos_kernel(Src src, const uint32_t* __restrict__ par_a, const uint32_t* __restrict__ bound,
-                           uint32_t cmax, uint32_t n_pairs, const uint32_t* __restrict__ npos,
-                           const uint64_t* __restrict__ pos_off, uint16_t* __restrict__ pos) {
+// Hacker's Delight 7-4 "compress" (= pext): the mask-dependent shift masks, then the per-source
+// part.  Right shifts by a constant are written as __umulhi(x, 2^(32-s)) and left shifts as
+// multiplies so that they issue on the FMA pipe next to the LOP3s on the ALU pipe (the kernel is
+// ALU-bound).  Checked bit-exact against a plain bit-by-bit pext (tests/test_host_logic.py
+// ::test_compress_matches_pext runs the same sequence of operations on the host).
+__device__ __forceinline__ uint32_t shr_c(uint32_t x, int s) { return __umulhi(x, 1u << (32 - s)); }
+__device__ __forceinline__ uint32_t shl_c(uint32_t x, int s) { return x * (1u << s); }
+
+__device__ __forceinline__ void hd_prep(uint32_t m, uint32_t (&mv)[5], uint32_t& m0) {
+  const uint32_t m_in = m;
+  uint32_t mk = shl_c(~m, 1);
+#pragma unroll
+  for (int i = 0; i < 5; ++i) {
+    // parallel prefix XOR of mk (HD's 5 shift-xor steps) as 3-input XORs: windows 3, 9, 27, 54
+    uint32_t mp = mk ^ shl_c(mk, 1) ^ shl_c(mk, 2);
+    mp = mp ^ shl_c(mp, 3) ^ shl_c(mp, 6);
+    mp = mp ^ shl_c(mp, 9) ^ shl_c(mp, 18);
+    mp ^= shl_c(mp, 27);
+    uint32_t v;  // materialised (opaque AND), so hd_apply's merge is one LOP3 on (x, mv, shifted)
+    asm("and.b32 %0, %1, %2;" : "=r"(v) : "r"(mp), "r"(m));
+    mv[i] = v;
+    m = (m ^ v) | shr_c(v, 1 << i);
+    mk &= ~mp;
+  }
+  asm("lop3.b32 %0, %1, %2, 0, 0x30;" : "=r"(m0) : "r"(m_in), "r"(mv[0]));  // m & ~mv0: bits kept by stage 0
+}
+// pext(x, m) given m's shift masks (x need not be pre-masked: stage 0 keeps x & m0 and moves x & mv0)
+// (each stage is two LOP3 -- the moving bits, then keep-or-moved in one 3-input op -- and one
+// IMAD.HI; written as PTX lop3 so that the compiler cannot split the merge into AND + OR)
+__device__ __forceinline__ uint32_t hd_apply(uint32_t x, uint32_t m0, const uint32_t (&mv)[5]) {
+  uint32_t t, y;
+  asm("and.b32 %0, %1, %2;" : "=r"(t) : "r"(x), "r"(mv[0]));
+  asm("lop3.b32 %0, %1, %2, %3, 0xEA;" : "=r"(y) : "r"(x), "r"(m0), "r"(shr_c(t, 1)));  // (x & m0) | ts
+#pragma unroll
+  for (int i = 1; i < 5; ++i) {
+    asm("and.b32 %0, %1, %2;" : "=r"(t) : "r"(y), "r"(mv[i]));
+    asm("lop3.b32 %0, %1, %2, %3, 0xBA;" : "=r"(y) : "r"(y), "r"(mv[i]), "r"(shr_c(t, 1 << i)));  // (y & ~mv) | ts
+  }
+  return y;
+}
+
+// One item of pext_kernel for a group of nm <= G members (G = 2, 3, 4, 6, 8: the unrolled width, so
+// a class of 2 members does not pay for 8): lane l walks its mask words [ja, jb) and appends, for
+// every member, pext(source word, mask word) to the member's lane-l stream -- a 32-bit
+// accumulator, whole words stored as they fill, the last partial word at the segment's end.
+// The bit count per step is the mask's, the same for every member, so the fill level and the
+// output position are shared; the append is one 32x32->64 multiply by 2^fill.  The next step's
+// mask and source words are loaded one step ahead.
+// base + idx words as one IMAD.WIDE.U32 on the FMA pipe: the scale (4) comes from a kernel
+// parameter, otherwise ptxas turns the multiply by a constant 4 into LEA + LEA.HI.X on the ALU pipe
+__device__ __forceinline__ const uint32_t* addr_of(const uint32_t* base, uint32_t idx, uint32_t wbytes) {
+  const uint32_t* r;
+  asm("mad.wide.u32 %0, %1, %2, %3;" : "=l"(r) : "r"(idx), "r"(wbytes), "l"(base));
+  return r;
+}
+
+template <uint32_t G, bool SPARSE>
+__device__ __forceinline__ void pext_item(const uint32_t* __restrict__ mp, const uint32_t* __restrict__ sbase,
+                                          const uint32_t (&so)[kMemberGroup], const uint32_t* __restrict__ s_oo,
+                                          uint32_t nm, uint32_t ja, uint32_t jb, uint32_t oj,
+                                          uint32_t* __restrict__ data, uint32_t wbytes) {
+  // member q's word j of this lane: cur + so[q] with cur = sbase + 32 j (one 64-bit step per j, then
+  // one IMAD.WIDE per member); output base offsets in shared memory (read only when a word fills)
+  uint32_t acc[G], xn[G];
+  uint32_t nb = 0;
+  mp += 32u * ja;
+  const uint32_t* cur = sbase + 32u * ja;
+  uint32_t mn = __ldg(mp);
+#pragma unroll
+  for (uint32_t q = 0; q < G; ++q) {
+    acc[q] = 0;
+    xn[q] = __ldg(addr_of(cur, so[q], wbytes));
+  }
+  for (uint32_t j = ja; j < jb; ++j) {
+    const uint32_t mw = mn;
+    uint32_t x[G];
+#pragma unroll
+    for (uint32_t q = 0; q < G; ++q) x[q] = xn[q];
+    const uint32_t step = j + 1 < jb ? 32u : 0u;
+    mp += step;
+    cur += step;
+    mn = __ldg(mp);
+#pragma unroll
+    for (uint32_t q = 0; q < G; ++q) xn[q] = __ldg(addr_of(cur, so[q], wbytes));
+    const uint32_t pw = 1u << nb;
+    const uint32_t c = __popc(mw);
+    nb += c;
+    uint32_t y[G];
+    if constexpr (SPARSE) {
+      // sparse masks (bitset rows, ~5 % set): the mask's trailing ones stay in place; every further
+      // set bit p lands at position i = its rank: bit i of (x >> (p - i)), the shift as an IMAD.HI by
+      // 2^(32 - (p - i)) (p - i >= 1 past the trailing ones) shared by the group -- per member one
+      // IMAD.HI + one LOP3 per set bit; the loop runs to the warp's largest count
+      const uint32_t i0 = mw == 0xffffffffu ? 32u : (uint32_t)__ffs(~mw) - 1u;
+      const uint32_t idm = i0 >= 32 ? 0xffffffffu : (1u << i0) - 1u;
+#pragma unroll
+      for (uint32_t q = 0; q < G; ++q) y[q] = x[q] & idm;
+      uint32_t mm = mw & ~idm, i = i0;
+      const uint32_t T = __reduce_max_sync(0xffffffffu, c - min(i0, c));
+      for (uint32_t t = 0; t < T; ++t) {
+        const bool has = mm != 0;
+        const uint32_t pbit = has ? (uint32_t)__ffs(mm) - 1u : 0u;
+        mm &= mm - 1u;
+        const uint32_t M = has ? 1u << (32u - (pbit - i)) : 0u;
+        const uint32_t bi = has ? 1u << i : 0u;
+#pragma unroll
+        for (uint32_t q = 0; q < G; ++q) {
+          uint32_t r;
+          asm("lop3.b32 %0, %1, %2, %3, 0xF8;" : "=r"(r) : "r"(y[q]), "r"(__umulhi(x[q], M)), "r"(bi));  // y | (t & bi)
+          y[q] = r;
+        }
+        i += has ? 1u : 0u;
+      }
+    } else {
+      uint32_t mv[5], m0;
+      hd_prep(mw, mv, m0);
+#pragma unroll
+      for (uint32_t q = 0; q < G; ++q) y[q] = hd_apply(x[q], m0, mv);
+    }
+#pragma unroll
+    for (uint32_t q = 0; q < G; ++q) {
+      // append at bit nb: one 32x32->64 multiply by 2^nb (FMA pipe); the low half is disjoint from
+      // the bits already in acc, so the OR is an add (FMA pipe as well); x[q] keeps the carry
+      uint64_t v;
+      asm("mul.wide.u32 %0, %1, %2;" : "=l"(v) : "r"(y[q]), "r"(pw));
+      asm("mad.lo.u32 %0, %1, 1, %0;" : "+r"(acc[q]) : "r"((uint32_t)v));
+      x[q] = (uint32_t)(v >> 32);
+    }
+    if (nb >= 32) {
+#pragma unroll
+      for (uint32_t q = 0; q < G; ++q) {
+        if (q < nm) data[s_oo[q] + 32u * oj] = acc[q];
+        acc[q] = x[q];
+      }
+      ++oj;
+      nb -= 32;
+    }
+  }
+  if (nb) {
+#pragma unroll
+    for (uint32_t q = 0; q < G; ++q)
+      if (q < nm) data[s_oo[q] + 32u * oj] = acc[q];
+  }
+}
+
+// ---------------------------------------------------------------- generation 3: bit gather
+// Generation 3's masks are bitset rows (~5 % set): instead of compressing every word per lane,
+// the warp gathers the ~C set bits of a 32-word chunk (row words 32 j .. 32 j + 31, one per lane)
+// in ceil(C / 32) ballots: lane l stages (l, bit) of its set bits in shared memory at its rank
+// (warp scan of the popcounts), then lane r of ballot t takes set bit 32 t + r, fetches the
+// member's word from its owner lane (shfl) and the ballot packs 32 of those bits into one output
+// word.  A member's list is the concatenation of these words (each chunk padded to whole words;
+// natural order, common to the class -- the next generation views it as 32 lane streams).
+// Work ~ output words, not input words.  (seg3 / cls3: sizes; pext3: the lists.)
+
+// warp per pair p = s * cmax + c: output words of row a's segment s (sum over its chunks)
+__global__ void seg3_kernel(const uint32_t* __restrict__ rows, uint64_t pitch, const uint32_t* __restrict__ par_a,
+                            const uint32_t* __restrict__ bound, const uint32_t* __restrict__ n_cls, uint32_t cmax,
+                            uint32_t n_pairs, uint32_t* __restrict__ w3, unsigned long long* __restrict__ in_words) {
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t p = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  if (p >= n_pairs || npos[p] == 0) return;
+  if (p >= n_pairs) return;
   const uint32_t c = p % cmax, s = p / cmax;
-  const uint32_t mid = par_a[bound[c]];
-  const uint32_t W = src.words(mid);
-  const uint32_t w0 = s * kSegW, w1 = min(W, w0 + kSegW);
-  const uint32_t* mk = src.base + src.offset(mid);
-  uint16_t* out = pos + pos_off[p];
-  uint32_t base = 0;
-  for (uint32_t w = w0; w < w1; w += 128) {
-    const uint32_t wl = w + 4 * lane;
-    const uint4 v = wl < w1 ? __ldg(reinterpret_cast<const uint4*>(mk + wl)) : make_uint4(0, 0, 0, 0);
-    const uint32_t t = __popc(v.x) + __popc(v.y) + __popc(v.z) + __popc(v.w);
-    uint32_t incl = t;
+  uint32_t words = 0;
+  if (c < *n_cls) {
+    const uint32_t j0 = bound[c], m = bound[c + 1] - j0;
+    if (m >= 2) {
+      const uint32_t* row = rows + (uint64_t)par_a[j0] * pitch + lane;
+      uint32_t a, b;
+      seg_range((uint32_t)(pitch / 32), s, a, b);
+      for (uint32_t j = a; j < b; ++j) {
+        const uint32_t C = __reduce_add_sync(0xffffffffu, (uint32_t)__popc(row[32ull * j]));
+        words += (C + 31) / 32;
+      }
+      if (lane == 0 && b > a) atomicAdd(in_words, 32ull * (b - a) * m);
+    }
+  }
+  if (lane == 0) w3[p] = words;
+}
+
+// thread per class: word offset of every segment in the class' lists, list words (a multiple of
+// 32), the class' words, pext3 items (one per segment with words and group of <= kG3Group members)
+__global__ void cls3_pad_kernel(const uint32_t* __restrict__ w3, const uint32_t* __restrict__ bound,
+                                const uint32_t* __restrict__ n_cls, uint32_t cmax, uint32_t nseg,
+                                uint32_t* __restrict__ loc3, uint32_t* __restrict__ nwc,
+                                uint64_t* __restrict__ cls_words, uint32_t* __restrict__ items,
+                                uint32_t* __restrict__ max_lw) {
+  const uint32_t C = *n_cls;
+  for (uint32_t c = blockIdx.x * blockDim.x + threadIdx.x; c < cmax; c += gridDim.x * blockDim.x) {
+    const uint32_t m = c < C ? bound[c + 1] - bound[c] : 0;
+    const uint32_t groups = m >= 2 ? (m + kG3Group - 1) / kG3Group : 0;
+    uint32_t acc = 0;
+    for (uint32_t s = 0; s < nseg; ++s) {
+      const uint64_t p = (uint64_t)s * cmax + c;
+      loc3[p] = acc;
+      acc += w3[p];
+      items[p] = w3[p] ? groups : 0;
+    }
+    const uint32_t words = groups ? (acc + 31u) & ~31u : 0u;
+    nwc[c] = words;
+    cls_words[c] = (uint64_t)words * m;
+    if (words) atomicMax(max_lw, words / 32u);
+  }
+}
+
+template <uint32_t G>
+__device__ __forceinline__ void pext3_item(const uint32_t* __restrict__ mrow, const uint32_t* __restrict__ sbase,
+                                           const uint32_t (&so)[kG3Group], const uint32_t* __restrict__ s_oo,
+                                           uint32_t nm, uint32_t ja, uint32_t jb, uint32_t ow0,
+                                           uint32_t* __restrict__ data, uint32_t wbytes, uint16_t* __restrict__ smap) {
+  const uint32_t lane = threadIdx.x & 31;
+  // groups of <= 8 load the next chunk's words one step ahead; 16-member groups have no registers
+  // left for that and rely on the other warps to hide the load latency
+  constexpr bool kPf = G <= 8;
+  constexpr uint32_t GP = kPf ? G : 1;
+  uint32_t keep[G], xn[GP];
+  uint32_t wc = 0;  // words emitted in this segment (warp-uniform)
+  const uint32_t* mp = mrow + 32u * ja;
+  const uint32_t* cur = sbase + 32u * ja;
+  uint32_t mn = __ldg(mp);
+#pragma unroll
+  for (uint32_t q = 0; q < G; ++q) keep[q] = 0;
+  if constexpr (kPf) {
+#pragma unroll
+    for (uint32_t q = 0; q < GP; ++q) xn[q] = __ldg(addr_of(cur, so[q], wbytes));
+  }
+  for (uint32_t j = ja; j < jb; ++j) {
+    const uint32_t mw = mn;
+    uint32_t x[G];
+    if constexpr (kPf) {
+#pragma unroll
+      for (uint32_t q = 0; q < GP; ++q) x[q] = xn[q];
+    } else {
+#pragma unroll
+      for (uint32_t q = 0; q < G; ++q) x[q] = __ldg(addr_of(cur, so[q], wbytes));
+    }
+    const uint32_t step = j + 1 < jb ? 32u : 0u;
+    mp += step;
+    cur += step;
+    mn = __ldg(mp);
+    if constexpr (kPf) {
+#pragma unroll
+      for (uint32_t q = 0; q < GP; ++q) xn[q] = __ldg(addr_of(cur, so[q], wbytes));
+    }
+    // ranks of this lane's set bits among the chunk's: warp scan of the popcounts
+    const uint32_t c = __popc(mw);
+    uint32_t o = c;
 #pragma unroll
     for (uint32_t d = 1; d < 32; d <<= 1) {
-      const uint32_t u = __shfl_up_sync(0xffffffffu, incl, d);
-      if (lane >= d) incl += u;
+      const uint32_t t = __shfl_up_sync(0xffffffffu, o, d);
+      if (lane >= d) o += t;
     }
-    uint32_t r = base + incl - t;
-    const uint32_t rel = (wl - w0) << 5;   // segment-relative bit index of word wl
-    const uint32_t x[4] = {v.x, v.y, v.z, v.w};
+    const uint32_t C = __shfl_sync(0xffffffffu, o, 31);
+    o -= c;
+    for (uint32_t mm = mw; mm; mm &= mm - 1u) smap[o++] = (uint16_t)((lane << 5) | (uint32_t)(__ffs(mm) - 1));
+    __syncwarp();
+    for (uint32_t k0 = 0; k0 < C; k0 += 32) {
+      const uint32_t k = k0 + lane;
+      const bool ok = k < C;
+      const uint32_t v = ok ? smap[k] : 0u;
+      const uint32_t L = v >> 5;
+      const uint32_t bm = ok ? 1u << (v & 31u) : 0u;  // bit select, empty past the chunk's last set bit
 #pragma unroll
-    for (uint32_t i = 0; i < 4; ++i)
-      for (uint32_t b = x[i]; b; b &= b - 1u) out[r++] = (uint16_t)(rel + 32u * i + (uint32_t)(__ffs(b) - 1));
-    base += __shfl_sync(0xffffffffu, incl, 31);
+      for (uint32_t q = 0; q < G; ++q) {
+        const uint32_t xv = __shfl_sync(0xffffffffu, x[q], L);
+        const uint32_t b = __ballot_sync(0xffffffffu, (xv & bm) != 0u);
+        if (lane == (wc & 31u)) keep[q] = b;
+      }
+      if ((wc & 31u) == 31u) {
+#pragma unroll
+        for (uint32_t q = 0; q < G; ++q)
+          if (q < nm) data[s_oo[q] + ow0 + (wc - 31u) + lane] = keep[q];
+      }
+      ++wc;
+    }
+    __syncwarp();  // smap is rewritten by the next chunk
   }
+  if (wc & 31u) {
+    const uint32_t base = wc & ~31u;
+    if (lane < (wc & 31u)) {
+#pragma unroll
+      for (uint32_t q = 0; q < G; ++q)
+        if (q < nm) data[s_oo[q] + ow0 + base + lane] = keep[q];
+    }
+  }
+}
+
+__global__ void __launch_bounds__(kT, 3) pext3_kernel(const uint32_t* __restrict__ rows, uint64_t pitch,
+                                                      const uint32_t* __restrict__ par_a,
+                                                      const uint32_t* __restrict__ par_b,
+                                                      const uint32_t* __restrict__ bound, uint32_t cmax,
+                                                      const uint32_t* __restrict__ item_pair,
+                                                      const uint32_t* __restrict__ item_off, uint32_t T,
+                                                      const uint32_t* __restrict__ loc3,
+                                                      const uint64_t* __restrict__ off, uint32_t* __restrict__ data,
+                                                      uint32_t wbytes) {
+  __shared__ uint16_t s_map[kT / 32][1024];
+  __shared__ uint32_t s_oo[kT / 32][kG3Group];
+  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const uint32_t it = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  if (it >= T) return;
+  const uint32_t p = item_pair[it];
+  const uint32_t c = p % cmax, s = p / cmax;
+  const uint32_t j0 = bound[c], m = bound[c + 1] - j0;
+  const uint32_t g = it - item_off[p];
+  const uint32_t first = j0 + g * kG3Group;
+  const uint32_t nm = min(kG3Group, m - g * kG3Group);
+  uint32_t ja, jb;
+  seg_range((uint32_t)(pitch / 32), s, ja, jb);
+  if (ja >= jb) return;
+  uint32_t* oo = s_oo[warp];
+  uint32_t so[kG3Group];
+#pragma unroll
+  for (uint32_t q = 0; q < kG3Group; ++q) {
+    const uint32_t e = first + (q < nm ? q : 0);  // surplus slots shadow member 0 (not stored)
+    so[q] = (uint32_t)((uint64_t)par_b[e] * pitch);
+    if (lane == q) oo[q] = (uint32_t)off[e];
+  }
+  __syncwarp();
+  const uint32_t* mrow = rows + (uint64_t)par_a[j0] * pitch + lane;
+  const uint32_t ow0 = loc3[p];
+  if (nm <= 2)
+    pext3_item<2>(mrow, rows + lane, so, oo, nm, ja, jb, ow0, data, wbytes, s_map[warp]);
+  else if (nm <= 4)
+    pext3_item<4>(mrow, rows + lane, so, oo, nm, ja, jb, ow0, data, wbytes, s_map[warp]);
+  else if (nm <= 8)
+    pext3_item<8>(mrow, rows + lane, so, oo, nm, ja, jb, ow0, data, wbytes, s_map[warp]);
+  else
+    pext3_item<16>(mrow, rows + lane, so, oo, nm, ja, jb, ow0, data, wbytes, s_map[warp]);
 }
 
 // item -> its pair (items of pair p are item_off[p] .. + items[p])
@@ -208,116 +506,63 @@ __global__ void item_pair_kernel(const uint32_t* __restrict__ items, const uint3
     for (uint32_t i = 0; i < items[p]; ++i) item_pair[item_off[p] + i] = p;
 }
 
-// base + idx words as one IMAD.WIDE.U32 (the scale comes from a kernel parameter so that ptxas
-// does not turn the multiply by 4 into LEA + LEA.HI.X on the ALU pipe)
-__device__ __forceinline__ const uint32_t* addr_of(const uint32_t* base, uint32_t idx, uint32_t wbytes) {
-  const uint32_t* r;
-  asm("mad.wide.u32 %0, %1, %2, %3;" : "=l"(r) : "r"(idx), "r"(wbytes), "l"(base));
-  return r;
-}
-
-// One gather item for G members (G = 2, 4, 8, 16: the unrolled width).  Round r: lane l takes
-// position 32 r + l of the segment (0 bits past the last), loads its word of every member's
-// source (an L1 gather), and ballot q packs the 32 selected bits of member q into one output word;
-// lane (r mod 32) keeps it, and every 32 rounds the lanes store 32 consecutive words per member
-// (coalesced).  The positions of the next round are loaded one round ahead.
-template <uint32_t G>
-__device__ __forceinline__ void gather_item(const uint16_t* __restrict__ P, uint32_t np,
-                                            const uint32_t* __restrict__ sb, const uint32_t (&so)[kGroup],
-                                            const uint32_t* __restrict__ oo, uint32_t nm,
-                                            uint32_t* __restrict__ data, uint32_t wbytes) {
+// Warp per item = (pair p = (segment, class), group of <= kMemberGroup members: full groups of 8,
+// the remainder in the class' last group).  Items run pair-major = segment-major, so the warps in
+// flight share the same bitset segments in L2.
+__global__ void __launch_bounds__(kT, 4) pext_kernel(Src src, const uint32_t* __restrict__ par_a,
+                                                     const uint32_t* __restrict__ par_b,
+                                                     const uint32_t* __restrict__ bound, uint32_t cmax,
+                                                     const uint32_t* __restrict__ item_pair,
+                                                     const uint32_t* __restrict__ item_off,
+                                                     uint32_t T, const uint32_t* __restrict__ loc,
+                                                     const uint64_t* __restrict__ off, uint32_t* __restrict__ data,
+                                                     uint32_t wbytes) {
   const uint32_t lane = threadIdx.x & 31;
-  uint32_t keep[G];
-#pragma unroll
-  for (uint32_t q = 0; q < G; ++q) keep[q] = 0;
-  const uint32_t rounds = (np + 31) / 32;
-  uint32_t vn = lane < np ? (uint32_t)__ldg(P + lane) : 0xffffffffu;
-  for (uint32_t r = 0; r < rounds; ++r) {
-    const uint32_t v = vn;
-    const uint32_t kn = 32u * (r + 1) + lane;
-    vn = kn < np ? (uint32_t)__ldg(P + kn) : 0xffffffffu;
-    const uint32_t bm = v != 0xffffffffu ? 1u << (v & 31u) : 0u;   // bit select, empty past the end
-    const uint32_t* lb = sb + (v != 0xffffffffu ? (v >> 5) : 0u);
-    uint32_t x[G];
-#pragma unroll
-    for (uint32_t q = 0; q < G; ++q) x[q] = __ldg(addr_of(lb, so[q], wbytes));
-    const bool mine = lane == (r & 31u);
-#pragma unroll
-    for (uint32_t q = 0; q < G; ++q) {
-      const uint32_t b = __ballot_sync(0xffffffffu, (x[q] & bm) != 0u);
-      keep[q] = mine ? b : keep[q];
-    }
-    if ((r & 31u) == 31u) {
-#pragma unroll
-      for (uint32_t q = 0; q < G; ++q)
-        if (q < nm) data[oo[q] + (r - 31u) + lane] = keep[q];
-    }
-  }
-  if (rounds & 31u) {
-    const uint32_t b0 = rounds & ~31u;
-    if (lane < (rounds & 31u)) {
-#pragma unroll
-      for (uint32_t q = 0; q < G; ++q)
-        if (q < nm) data[oo[q] + b0 + lane] = keep[q];
-    }
-  }
-}
-
-// Warp per item = (pair p = (segment s, class c), group of <= kGroup members).  Items run
-// pair-major = segment-major, so the warps in flight share the same source segments in L2.  The
-// item of a class' last segment also zeroes the list tails (words past the class' last segment, up
-// to the 4-word padding): every word of every list is written, no memset.
-__global__ void __launch_bounds__(kT, 3) gather_kernel(Src src, const uint32_t* __restrict__ par_a,
-                                                       const uint32_t* __restrict__ par_b,
-                                                       const uint32_t* __restrict__ bound, uint32_t cmax,
-                                                       const uint32_t* __restrict__ item_pair,
-                                                       const uint32_t* __restrict__ item_off, uint32_t T,
-                                                       const uint32_t* __restrict__ npos,
-                                                       const uint64_t* __restrict__ pos_off,
-                                                       const uint16_t* __restrict__ pos,
-                                                       const uint32_t* __restrict__ loc,
-                                                       const uint32_t* __restrict__ wseg,
-                                                       const uint32_t* __restrict__ nwc,
-                                                       const uint32_t* __restrict__ cls_nseg,
-                                                       const uint64_t* __restrict__ off,
-                                                       uint32_t* __restrict__ data, uint32_t wbytes) {
-  __shared__ uint32_t s_oo[kT / 32][kGroup];
-  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const uint32_t it = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   if (it >= T) return;
-  (void)par_a;
-  const uint32_t p = item_pair[it];
-  const uint32_t c = p % cmax, s = p / cmax;
-  const uint32_t j0 = bound[c], m = bound[c + 1] - j0;
-  const uint32_t g = it - item_off[p];
-  const uint32_t first = j0 + g * kGroup;
-  const uint32_t nm = min(kGroup, m - g * kGroup);
-  uint32_t* oo = s_oo[warp];
-  const uint32_t lp = loc[p];
-  uint32_t so[kGroup];
+  const uint32_t* base = src.rows ? src.rows : src.data;
+  {
+    const uint32_t p = item_pair[it];
+    const uint32_t c = p % cmax, s = p / cmax;
+    const uint32_t j0 = bound[c], m = bound[c + 1] - j0;
+    const uint32_t groups = (m + kMemberGroup - 1) / kMemberGroup;
+    const uint32_t g = it - item_off[p];
+    (void)groups;
+    const uint32_t first = j0 + g * kMemberGroup;  // full groups of 8, the remainder in the last
+    const uint32_t nm = min(kMemberGroup, m - g * kMemberGroup);
+    const VecRef mk = src.vec(par_a[j0]);
+    uint32_t ja, jb;
+    seg_range(mk.lw, s, ja, jb);
+    if (ja >= jb) return;
+    __shared__ uint32_t s_oo[kT / 32][kMemberGroup];
+    uint32_t* oo = s_oo[threadIdx.x >> 5];
+    uint32_t so[kMemberGroup];
 #pragma unroll
-  for (uint32_t q = 0; q < kGroup; ++q) {
-    const uint32_t e = first + (q < nm ? q : 0);  // surplus slots shadow member 0 (not stored)
-    so[q] = src.offset(par_b[e]);
-    if (lane == q) oo[q] = (uint32_t)off[e] + lp;
-  }
-  __syncwarp();
-  const uint32_t np = npos[p];
-  const uint32_t* sb = src.base + (uint64_t)s * kSegW;
-  const uint16_t* P = pos + pos_off[p];
-  if (nm <= 2)
-    gather_item<2>(P, np, sb, so, oo, nm, data, wbytes);
-  else if (nm <= 4)
-    gather_item<4>(P, np, sb, so, oo, nm, data, wbytes);
-  else if (nm <= 8)
-    gather_item<8>(P, np, sb, so, oo, nm, data, wbytes);
-  else
-    gather_item<16>(P, np, sb, so, oo, nm, data, wbytes);
-  if (s + 1 == cls_nseg[c]) {   // zero the tail of the members' lists
-    const uint32_t w_end = lp + wseg[p], W = nwc[c];
-    for (uint32_t q = 0; q < nm; ++q) {
-      const uint32_t base = oo[q] - lp;
-      for (uint32_t w = w_end + lane; w < W; w += 32) data[base + w] = 0u;
+    for (uint32_t q = 0; q < kMemberGroup; ++q) {
+      const uint32_t e = first + (q < nm ? q : 0);  // surplus slots shadow member 0 (not stored)
+      so[q] = (uint32_t)(src.vec(par_b[e]).p - base);
+      if (lane == q) oo[q] = (uint32_t)off[e] + 0u;
+    }
+    __syncwarp();
+    const uint32_t oj = loc[(uint64_t)p * 32 + lane];
+    const uint32_t* mp = mk.p + lane;
+    if (src.rows) {  // generation 3: sparse bitset rows as masks
+      if (nm <= 2)
+        pext_item<2, true>(mp, base + lane, so, oo, nm, ja, jb, oj, data + lane, wbytes);
+      else if (nm <= 4)
+        pext_item<4, true>(mp, base + lane, so, oo, nm, ja, jb, oj, data + lane, wbytes);
+      else
+        pext_item<8, true>(mp, base + lane, so, oo, nm, ja, jb, oj, data + lane, wbytes);
+    } else if (nm <= 2) {
+      pext_item<2, false>(mp, base + lane, so, oo, nm, ja, jb, oj, data + lane, wbytes);
+    } else if (nm == 3) {
+      pext_item<3, false>(mp, base + lane, so, oo, nm, ja, jb, oj, data + lane, wbytes);
+    } else if (nm <= 4) {
+      pext_item<4, false>(mp, base + lane, so, oo, nm, ja, jb, oj, data + lane, wbytes);
+    } else if (nm <= 6) {
+      pext_item<6, false>(mp, base + lane, so, oo, nm, ja, jb, oj, data + lane, wbytes);
+    } else {
+      pext_item<8, false>(mp, base + lane, so, oo, nm, ja, jb, oj, data + lane, wbytes);
     }
   }
 }
@@ -328,7 +573,7 @@ __global__ void __launch_bounds__(kT, 3) gather_kernel(Src src, const uint32_t* 
 // one warp per group walking the whole list, plain stores -- short lists (deep generations, where
 // a CTA per group would leave most of its warps idle).  Siblings in batches of 32 (lane j
 // accumulates sibling j); two siblings share one packed redux.sync (per-chunk warp sums
-// <= 32 x 8 x 32 < 2^16).  Lists hold a multiple of 4 words, zero-padded.
+// <= 32 x 8 x 32 < 2^16).
 template <bool WARP>
 __global__ void __launch_bounds__(kT) count_proj_kernel(const uint32_t* __restrict__ data,
                                                         const uint64_t* __restrict__ off,
@@ -391,29 +636,30 @@ void scan_excl(const T* in, T* out, uint32_t n, PBuf<uint8_t>& tmpbuf, cudaStrea
   note_launch(2);
 }
 
-// totals: tot[0] = gather items, tot[1] = list words, tot[2] = positions
+// totals: tot[0] = pext items, tot[1] = vector words
 __global__ void proj_totals_kernel(const uint32_t* __restrict__ items, const uint32_t* __restrict__ item_off,
                                    uint32_t n_pairs, const uint64_t* __restrict__ cw, const uint64_t* __restrict__ cb,
-                                   uint32_t cmax, const uint32_t* __restrict__ npos,
-                                   const uint64_t* __restrict__ pos_off, uint64_t* __restrict__ tot) {
+                                   uint32_t cmax, uint64_t* __restrict__ tot) {
   if (threadIdx.x == 0 && blockIdx.x == 0) {
     tot[0] = (uint64_t)item_off[n_pairs - 1] + items[n_pairs - 1];
     tot[1] = cb[cmax - 1] + cw[cmax - 1];
-    tot[2] = pos_off[n_pairs - 1] + npos[n_pairs - 1];
   }
 }
 
-// u32 -> u64 widening (the positions' offsets are scanned in 64 bits)
-__global__ void widen_kernel(const uint32_t* __restrict__ in, uint64_t* __restrict__ out, uint32_t n) {
-  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) out[i] = in[i];
+// generation 3 by bit gather (pext3_kernel); GPA_PROJ_K3_PEXT=1 keeps the set-bit-walk pext (comparisons)
+bool gather3() {
+  static const bool v = [] {
+    const char* e = getenv("GPA_PROJ_K3_PEXT");
+    return !(e && atoi(e) != 0);
+  }();
+  return v;
 }
 
 // per-thread, per-device persistent workspace (grow-only): the class tables of proj_build and the
 // two generations of lists
 struct ProjWork {
-  PBuf<uint32_t> flag, ex, bound, small, npos, wseg, loc, items, item_off, item_pair, nwc, cls_nseg;
-  PBuf<uint64_t> cls_words, cls_base, tot, npos64, pos_off;
-  PBuf<uint16_t> pos;
+  PBuf<uint32_t> flag, ex, bound, small, words, loc, items, item_off, item_pair, nwc;
+  PBuf<uint64_t> cls_words, cls_base, tot;
   PBuf<uint8_t> tmp;   // CUB temporary storage of its own: proj_build_begin may run beside the join's scans
   DeviceProj lists[2];
 };
@@ -422,27 +668,28 @@ ProjWork& work_for(int device) {
   return w[device];
 }
 
+}  // namespace
+
+DeviceProj* proj_lists(int device) { return work_for(device).lists; }
+
+namespace {
 Src make_src(const ProjPending& pp) {
   Src src{};
   if (!pp.prev) {
-    src.base = pp.rows;
+    src.rows = pp.rows;
     src.pitch = pp.pitch;
   } else {
-    src.base = pp.prev->data.p;
+    src.data = pp.prev->data.p;
     src.off = pp.prev->off.p;
     src.nw = pp.prev->nw.p;
   }
   return src;
 }
-
 }  // namespace
-
-DeviceProj* proj_lists(int device) { return work_for(device).lists; }
 
 bool proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const DeviceProj* prev,
                       const uint32_t* rows, uint64_t pitch_words, uint32_t n_rows, DeviceScratch& scratch, int n_sms,
                       cudaStream_t s, ProjPending& pp) {
-  (void)scratch;
   pp = ProjPending();
   pp.n = n;
   pp.par_a = par_a;
@@ -453,12 +700,12 @@ bool proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, 
   if (n == 0) return true;
   const Src src = make_src(pp);
   const uint32_t cmax = prev ? n : std::min(n, n_rows);
-  const uint64_t w_max = prev ? prev->max_nw : pitch_words;
-  const uint32_t nseg = (uint32_t)std::max<uint64_t>(1, (w_max + kSegW - 1) / kSegW);
-  // sources are addressed with 32-bit word offsets, the tables with 31-bit thread indices: beyond
+  const uint64_t lw_max = prev ? prev->max_lw : pitch_words / 32;
+  const uint32_t nseg = (uint32_t)std::max<uint64_t>(1, (lw_max + kSegJ - 1) / kSegJ);
+  // 32-bit word offsets inside pext_kernel
+  // pext_kernel addresses sources with 32-bit word offsets, its tables with 31-bit indices: beyond
   // that the caller uses complete intersection
   if (!prev && (uint64_t)n_rows * pitch_words >= (1ull << 32)) return false;
-  if (prev && prev->words >= (1ull << 32)) return false;
   const uint64_t n_pairs64 = (uint64_t)cmax * nseg;
   if (n_pairs64 * 32 >= (1ull << 31)) return false;
   const uint32_t n_pairs = (uint32_t)n_pairs64;
@@ -475,36 +722,39 @@ bool proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, 
   { cls_flag_kernel<<<grid_for(n, n_sms), kT, 0, s>>>(par_a, n, W.flag.p); note_launch(); }
   scan_excl<uint32_t>(W.flag.p, W.ex.p, n, W.tmp, s);
   { cls_bound_kernel<<<grid_for(n, n_sms), kT, 0, s>>>(W.flag.p, W.ex.p, n, W.bound.p, W.small.p); note_launch(); }
-  W.npos.ensure(n_pairs);
-  W.wseg.ensure(n_pairs);
-  W.loc.ensure(n_pairs);
+  W.words.ensure((size_t)n_pairs * 32);
+  W.loc.ensure((size_t)n_pairs * 32);
   W.items.ensure(n_pairs);
   W.item_off.ensure(n_pairs);
-  W.npos64.ensure(n_pairs);
-  W.pos_off.ensure(n_pairs);
   W.nwc.ensure(cmax);
-  W.cls_nseg.ensure(cmax);
   W.cls_words.ensure(cmax);
   W.cls_base.ensure(cmax);
-  W.tot.ensure(3);
+  W.tot.ensure(2);
   const unsigned wpb = kT / 32;
-  { seg_count_kernel<<<(n_pairs + wpb - 1) / wpb, kT, 0, s>>>(src, par_a, W.bound.p, W.small.p, cmax, n_pairs,
-        W.npos.p, W.wseg.p, reinterpret_cast<unsigned long long*>(W.small.p + 2)); note_launch(); }
-  { cls_pad_kernel<<<grid_for(cmax, n_sms), kT, 0, s>>>(src, par_a, W.wseg.p, W.bound.p, W.small.p, cmax, nseg,
-        W.loc.p, W.nwc.p, W.cls_nseg.p, W.cls_words.p, W.items.p, W.small.p + 1); note_launch(); }
-  { widen_kernel<<<grid_for(n_pairs, n_sms), kT, 0, s>>>(W.npos.p, W.npos64.p, n_pairs); note_launch(); }
+  if (!prev && gather3()) {  // generation 3: bit gather (pext3_kernel), natural-order lists
+    { seg3_kernel<<<(n_pairs + wpb - 1) / wpb, kT, 0, s>>>(rows, pitch_words, par_a, W.bound.p, W.small.p, cmax, n_pairs,
+          W.words.p, reinterpret_cast<unsigned long long*>(W.small.p + 2)); note_launch(); }
+    { cls3_pad_kernel<<<grid_for(cmax, n_sms), kT, 0, s>>>(W.words.p, W.bound.p, W.small.p, cmax, nseg, W.loc.p,
+          W.nwc.p, W.cls_words.p, W.items.p, W.small.p + 1); note_launch(); }
+  } else {
+    { seg_popc_kernel<<<(n_pairs + wpb - 1) / wpb, kT, 0, s>>>(
+          src, par_a, W.bound.p, W.small.p, cmax, nseg, n_pairs, W.words.p,
+          reinterpret_cast<unsigned long long*>(W.small.p + 2)); note_launch(); }
+    { cls_pad_kernel<<<(cmax + wpb - 1) / wpb, kT, 0, s>>>(
+          W.words.p, W.bound.p, W.small.p, cmax, nseg, W.loc.p, W.nwc.p, W.cls_words.p, W.items.p, W.small.p + 1);
+      note_launch(); }
+  }
   scan_excl<uint32_t>(W.items.p, W.item_off.p, n_pairs, W.tmp, s);
   scan_excl<uint64_t>(W.cls_words.p, W.cls_base.p, cmax, W.tmp, s);
-  scan_excl<uint64_t>(W.npos64.p, W.pos_off.p, n_pairs, W.tmp, s);
   { proj_totals_kernel<<<1, 32, 0, s>>>(W.items.p, W.item_off.p, n_pairs, W.cls_words.p, W.cls_base.p, cmax,
-                                        W.npos.p, W.pos_off.p, W.tot.p); note_launch(); }
+                                        W.tot.p); note_launch(); }
   GPA_CUDA(cudaGetLastError());
   pp.d_tot = W.tot.p;
   pp.d_small = W.small.p;
   return true;
 }
 
-bool proj_build_finish(const ProjPending& pp, const uint64_t T[3], const uint32_t sm[4], DeviceProj& out, int n_sms,
+bool proj_build_finish(const ProjPending& pp, const uint64_t T[2], const uint32_t sm[4], DeviceProj& out, int n_sms,
                        cudaStream_t s, cudaEvent_t ev_build) {
   const uint32_t n = pp.n;
   out.n = n;
@@ -519,22 +769,21 @@ bool proj_build_finish(const ProjPending& pp, const uint64_t T[3], const uint32_
   // complete intersection with it; default: no cap beyond device memory)
   if (const char* cap = getenv("GPA_PROJ_MAX_MB"))
     if (T[1] * 4 > (uint64_t)atof(cap) * 1e6) return false;
-  ProjWork& W = work_for(pp.device);
   try {
     out.data.ensure(T[1]);
-    W.pos.ensure(T[2]);
   } catch (const Error& e) {
     if (e.status != GPA_ERR_OOM) throw;
     return false;  // caller falls back to complete intersection
   }
+  ProjWork& W = work_for(pp.device);
   const Src src = make_src(pp);
   out.off.ensure(n);
   out.nw.ensure(n);
   out.words = T[1];
-  out.max_nw = sm[1];
-  out.max_lw = (sm[1] + 31) / 32;
+  out.max_lw = sm[1];
   out.in_words = (uint64_t)sm[2] | ((uint64_t)sm[3] << 32);
-  const unsigned wpb = kT / 32;
+  // lanes shorter than their class' Lw keep a zero tail
+  GPA_CUDA(cudaMemsetAsync(out.data.p, 0, std::max<uint64_t>(T[1], 1) * 4, s));
   { entry_off_kernel<<<grid_for(n, n_sms), kT, 0, s>>>(W.flag.p, W.ex.p, W.bound.p, W.nwc.p, W.cls_base.p, n,
                                                       out.off.p, out.nw.p); note_launch(); }
   if (ev_build) GPA_CUDA(cudaEventRecord(ev_build, s));  // start of the list build proper
@@ -542,23 +791,39 @@ bool proj_build_finish(const ProjPending& pp, const uint64_t T[3], const uint32_
     W.item_pair.ensure(T[0]);
     { item_pair_kernel<<<grid_for(pp.n_pairs, n_sms), kT, 0, s>>>(W.items.p, W.item_off.p, pp.n_pairs,
                                                                  W.item_pair.p); note_launch(); }
-    if (T[2])
-      { pos_kernel<<<(pp.n_pairs + wpb - 1) / wpb, kT, 0, s>>>(src, pp.par_a, W.bound.p, pp.cmax, pp.n_pairs,
-                                                               W.npos.p, W.pos_off.p, W.pos.p); note_launch(); }
-    const uint64_t blocks = (T[0] + wpb - 1) / wpb;
-    { gather_kernel<<<(unsigned)blocks, kT, 0, s>>>(src, pp.par_a, pp.par_b, W.bound.p, pp.cmax, W.item_pair.p,
-                                                    W.item_off.p, (uint32_t)T[0], W.npos.p, W.pos_off.p, W.pos.p,
-                                                    W.loc.p, W.wseg.p, W.nwc.p, W.cls_nseg.p, out.off.p, out.data.p,
-                                                    4u); note_launch(); }
+    const uint64_t blocks = (T[0] + kT / 32 - 1) / (kT / 32);
+    if (!pp.prev && gather3())
+      { pext3_kernel<<<(unsigned)blocks, kT, 0, s>>>(pp.rows, pp.pitch, pp.par_a, pp.par_b, W.bound.p, pp.cmax,
+                                                     W.item_pair.p, W.item_off.p, (uint32_t)T[0], W.loc.p, out.off.p,
+                                                     out.data.p, 4u); note_launch(); }
+    else
+      { pext_kernel<<<(unsigned)blocks, kT, 0, s>>>(src, pp.par_a, pp.par_b, W.bound.p, pp.cmax, W.item_pair.p,
+                                                    W.item_off.p, (uint32_t)T[0], W.loc.p, out.off.p, out.data.p, 4u);
+        note_launch(); }
   }
   GPA_CUDA(cudaGetLastError());
   return true;
 }
 
+bool proj_build(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const DeviceProj* prev,
+                const uint32_t* rows, uint64_t pitch_words, uint32_t n_rows, DeviceProj& out, DeviceScratch& scratch,
+                int n_sms, cudaStream_t s, cudaEvent_t ev_build) {
+  ProjPending pp;
+  if (!proj_build_begin(n, par_a, par_b, prev, rows, pitch_words, n_rows, scratch, n_sms, s, pp)) return false;
+  uint64_t T[2] = {0, 0};
+  uint32_t sm[4] = {0, 0, 0, 0};
+  if (n) {
+    GPA_CUDA(cudaMemcpyAsync(T, pp.d_tot, sizeof(T), cudaMemcpyDeviceToHost, s));
+    GPA_CUDA(cudaMemcpyAsync(sm, pp.d_small, sizeof(sm), cudaMemcpyDeviceToHost, s));
+    stream_wait(s);
+  }
+  return proj_build_finish(pp, T, sm, out, n_sms, s, ev_build);
+}
+
 void launch_count_proj(const DeviceProj& P, const uint32_t* gpar, const uint32_t* ext_off, const uint32_t* eidx,
                        uint32_t G, uint32_t* counts, cudaStream_t s) {
   if (G == 0) return;
-  if ((uint64_t)P.max_nw <= 8192)
+  if ((uint64_t)P.max_lw * 32 <= 8192)
     { count_proj_kernel<true><<<(G + kT / 32 - 1) / (kT / 32), kT, 0, s>>>(P.data.p, P.off.p, P.nw.p, gpar, ext_off,
                                                                           eidx, counts, G); note_launch(); }
   else

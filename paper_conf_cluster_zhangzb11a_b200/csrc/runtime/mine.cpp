@@ -92,7 +92,7 @@ void record_level(gpa_result* R, const gpa_bitset* bs, uint32_t k, const Grouped
 // (the sizes T, sm came back with |C_k|): the list build (pext) on s, overlapping the emitting
 // join on the auxiliary stream; the supports wait for both (aux_done).
 bool count_projected_staged(gpa_bitset* bs, uint32_t k, const DeviceBatch& B, DeviceProj& cur, const ProjPending& pp,
-                            const uint64_t T[3], const uint32_t sm[4], cudaEvent_t aux_done, CountStats* cs,
+                            const uint64_t T[2], const uint32_t sm[4], cudaEvent_t aux_done, CountStats* cs,
                             uint64_t src_words) {
   cudaStream_t s = bs->stream;
   const double t0 = now_ms();
@@ -268,7 +268,7 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
   Events aux_evs;            // [0] s -> aux (batch buffers sized), [1] aux done
   ProjPending ppend;
   bool aux_join = false;     // this generation's batch was emitted on aux_s
-  uint64_t pT[3] = {0, 0, 0};
+  uint64_t pT[2] = {0, 0};
   uint32_t psm[4] = {0, 0, 0, 0};
   // deferred (device-side) timing of a generation on stream s: [5] generation start, [0] counting
   // start, [1] counting end, [2] all-reduce end, [3, 4) projected-list build, [6] threshold end
@@ -342,8 +342,8 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
         uint32_t* hs = host_sizes();
         if (proj_build_begin(Ld.n, Ld.par_a.p, Ld.par_b.p, k == 3 ? nullptr : Pprev, bs->rows.p, bs->pitch_words,
                              bs->n_rows, scratch, bs->n_sms, aux_s.s, ppend)) {
-          GPA_CUDA(cudaMemcpyAsync(hs + 2, ppend.d_tot, 24, cudaMemcpyDeviceToHost, aux_s.s));
-          GPA_CUDA(cudaMemcpyAsync(hs + 8, ppend.d_small, 16, cudaMemcpyDeviceToHost, aux_s.s));
+          GPA_CUDA(cudaMemcpyAsync(hs + 2, ppend.d_tot, 16, cudaMemcpyDeviceToHost, aux_s.s));
+          GPA_CUDA(cudaMemcpyAsync(hs + 6, ppend.d_small, 16, cudaMemcpyDeviceToHost, aux_s.s));
         } else {
           proj_on = false;   // lists not addressable: complete intersection from this generation on
         }
@@ -352,8 +352,8 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
         stream_wait(aux_s.s);
         M = hs[0];
         G = hs[1];
-        std::memcpy(pT, hs + 2, 24);
-        std::memcpy(psm, hs + 8, 16);
+        std::memcpy(pT, hs + 2, 16);
+        std::memcpy(psm, hs + 6, 16);
         device_candgen_finish(Ld, Bd, scratch, bs->n_sms, s, (uint32_t)M, (uint32_t)G, aux_s.s, aux_evs.e[0]);
         GPA_CUDA(cudaEventRecord(aux_evs.e[1], aux_s.s));
         aux_join = true;

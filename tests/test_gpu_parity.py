@@ -296,7 +296,7 @@ def test_shard_sum_equals_oracle(name, request):
         levels = request.getfixturevalue("t40_full")[3]
     else:
         levels = [(lv.cand, lv.count) for lv in oracle.mine_ds(ds, theta).levels]
-    ch = gen.chunk_size() if gen.CONFIGS[name].kind == "quest" else 512
+    ch = gen.chunk_size() if gen.CONFIGS[name].kind == "quest" and ds.n_tx > 2 * gen.chunk_size() else 512
     cut = (ds.n_tx // 2 + ch - 1) // ch * ch
     assert 0 < cut < ds.n_tx
     acc = [np.zeros(len(c), np.uint64) for c, _ in levels]
@@ -473,17 +473,46 @@ def test_proj_fallback_to_complete_intersection(monkeypatch, how):
 
 @pytest.mark.parametrize("n_tx,n_items,max_len,theta", [(70_000, 40, 10, 1400), (140_000, 60, 12, 2800),
                                                           (9_000, 40, 12, 90)])
-def test_proj_gather_multi_segment_classes(n_tx, n_items, max_len, theta):
-    """Projected lists through the position + ballot-gather build (proj.cu): class masks spanning
-    several 65,536-bit segments (70,000 / 140,000 transactions), classes of more than 16 members
-    (several gather items per segment), ragged segment and list tails -- every (C_k, count) of
-    every generation equal to the oracle, and the generations k >= 3 really ran on the lists."""
+def test_proj_multi_segment_classes(n_tx, n_items, max_len, theta):
+    """Projected lists (proj.cu): class masks spanning several 131,072-transaction segments (70,000 /
+    140,000 transactions: bitset rows of 2,188 / 4,375 words), classes of more than 16 members
+    (several pext items per segment), ragged segment and list tails -- every (C_k, count) of every
+    generation equal to the oracle, and the generations k >= 3 really ran on the lists."""
     ds = gen.random_db(n_tx % 1000 + n_items, n_tx, n_items, max_len=max_len, p_empty=0.01)
     ref = oracle.mine_ds(ds, theta)
     res = gpa.mine(ds, min_count=theta, options=gpa.Options(count_kernel=gpa.KERNEL_PROJ), keep_candidates=True)
     assert_mine_equal(res, ref)
     assert len(res.levels) >= 4
     assert all(lv.stats["kernel_name"] == "proj" for lv in res.levels[2:])
+
+
+@pytest.mark.parametrize("name", ["mushroom", "chess", "random"])
+def test_proj_k3_set_bit_walk_pext(name):
+    """Generation 3's lists by the set-bit-walk pext (GPA_PROJ_K3_PEXT=1, read once per process, so
+    a child process) instead of the default warp bit gather (pext3_kernel): every frequent itemset and
+    support equal to the oracle's."""
+    import json
+    import subprocess
+    import sys
+    if name == "random":
+        ds, theta = gen.random_db(11, 8000, 40, max_len=16), 80
+        spec = "gen.random_db(11, 8000, 40, max_len=16), 80"
+    else:
+        ds = gen.make(name)
+        theta = oracle.min_count(ds.n_tx, gen.CONFIGS[name].minsup)
+        spec = f"gen.make({name!r}), {theta}"
+    code = ("import json, gen, paper_conf_cluster_zhangzb11a_b200 as gpa\n"
+            f"ds, th = {spec}\n"
+            "r = gpa.mine(ds, min_count=th)\n"
+            "print(json.dumps(sorted([list(map(int, s)), int(c)] for s, c in r.frequent().items())))\n")
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, GPA_PROJ_K3_PEXT="1")
+    out = subprocess.run([sys.executable, "-c", code], cwd=root, env=env, capture_output=True, text=True,
+                         check=True, timeout=600).stdout
+    got = {tuple(s): c for s, c in json.loads(out.strip().splitlines()[-1])}
+    ref = oracle.mine_ds(ds, theta).frequent()
+    assert got == {tuple(map(int, s)): int(c) for s, c in ref.items()}
+    assert max(len(s) for s in got) >= 4
 
 
 def test_complete_intersection_flag():

@@ -163,67 +163,87 @@ def test_trie_plan_invariants(shim, name, k):
 
 # ---------------------------------------------------------------- projected lists (proj.cu)
 
-SEG_W = 2048   # proj.cu kSegW: mask segment of 2,048 words (u16 positions)
+def _hd_compress(x, m):
+    """The operation sequence of proj.cu's hd_prep / hd_apply (Hacker's Delight 7-4 compress,
+    right shifts as umulhi by 2^(32-s), left shifts as multiplies), vectorised over uint32."""
+    M32 = np.uint64(0xFFFFFFFF)
+    x = x.astype(np.uint64)
+    m = m.astype(np.uint64)
+
+    def shl(v, s):
+        return (v * np.uint64(1 << s)) & M32
+
+    def shr(v, s):
+        return (v * np.uint64(1 << (32 - s))) >> np.uint64(32)
+
+    mk = shl(~m & M32, 1)
+    mv = []
+    mm = m.copy()
+    for i in range(5):
+        mp = mk ^ shl(mk, 1)
+        for sh in (2, 4, 8, 16):
+            mp ^= shl(mp, sh)
+        v = mp & mm
+        mv.append(v)
+        mm = (mm ^ v) | shr(v, 1 << i)
+        mk &= ~mp & M32
+    t = x & mv[0]
+    y = (x & m & (~mv[0] & M32)) | shr(t, 1)
+    for i in range(1, 5):
+        t = y & mv[i]
+        y = (y & (~mv[i] & M32)) | shr(t, 1 << i)
+    return y.astype(np.uint32)
 
 
-def _segment_positions(mask):
-    """proj.cu pos_kernel: per segment, the segment-relative positions (word << 5 | bit) of the
-    mask's set bits, in increasing order, as u16."""
-    out = []
-    for s0 in range(0, len(mask), SEG_W):
-        seg = mask[s0:s0 + SEG_W]
-        bits = np.unpackbits(seg.view(np.uint8), bitorder="little")
-        out.append(np.nonzero(bits)[0].astype(np.uint16))
+def _pext_ref(x, m):
+    out = np.zeros_like(x)
+    k = np.zeros_like(x)
+    for i in range(32):
+        sel = (m >> np.uint32(i)) & np.uint32(1)
+        bit = (x >> np.uint32(i)) & np.uint32(1)
+        out |= (bit & sel) << k
+        k += sel
     return out
 
 
-def _gather_list(mask, src):
-    """proj.cu gather_item: per segment, rounds of 32 positions; round r's word = ballot over lanes
-    l of bit (pos[32r + l] & 31) of src word (segment base + pos >> 5); words padded per segment,
-    the list padded to a multiple of 4 words with zeros."""
-    words = []
-    for s, pos in enumerate(_segment_positions(mask)):
-        for r in range(0, len(pos), 32):
-            w = 0
-            for lane, v in enumerate(pos[r:r + 32].tolist()):
-                x = int(src[s * SEG_W + (v >> 5)])
-                if x >> (v & 31) & 1:
-                    w |= 1 << lane
-            words.append(w)
-    words += [0] * (-len(words) % 4)
-    return np.array(words, dtype=np.uint32)
-
-
-def _bits(words):
-    return np.unpackbits(np.asarray(words, dtype=np.uint32).view(np.uint8), bitorder="little")
-
-
-def test_gather_lists_match_definition():
-    """The projected-list layout of proj.cu (segment positions + ballot gather, per-segment word
-    padding): dropping each segment's padding bits gives exactly the definition -- the bits of the
-    source at the set positions of the mask, in order (V_X[i] = B[x][t_i]); and the
-    padded lists of one class give the same popcount-of-AND supports as the unpadded definition."""
+def test_compress_matches_pext():
+    """proj.cu's parallel bit extract equals the bit-by-bit definition (random, sparse, dense,
+    empty and full masks)."""
     rng = np.random.default_rng(11)
-    for trial, (n_words, dens) in enumerate([(100, 0.05), (SEG_W, 0.3), (SEG_W + 37, 0.02), (2 * SEG_W + 4, 0.6),
-                                             (5000, 0.0), (64, 1.0)]):
-        mask = (rng.random(n_words * 32) < dens)
-        mk = np.packbits(mask, bitorder="little").view(np.uint32)
-        srcs = [np.packbits(rng.random(n_words * 32) < 0.4, bitorder="little").view(np.uint32) for _ in range(3)]
-        lists = [_gather_list(mk, s) for s in srcs]
-        segs = _segment_positions(mk)
-        for s, L in zip(srcs, lists):
-            assert len(L) % 4 == 0
-            b = _bits(L)
-            got, at = [], 0
-            for pos in segs:          # drop the per-segment padding bits
-                got.append(b[at:at + len(pos)])
-                at += (len(pos) + 31) // 32 * 32
-            assert not b[at:].any()
-            got = np.concatenate(got) if got else np.zeros(0, np.uint8)
-            want = _bits(s)[np.nonzero(mask)[0]]
-            assert np.array_equal(got, want), trial
-        # supports of {a, b} within the class = popc(AND) of the padded lists
-        for i in range(3):
-            for j in range(i + 1, 3):
-                want = int((_bits(srcs[i]) & _bits(srcs[j]) & mask).sum())
-                assert int((_bits(lists[i]) & _bits(lists[j])).sum()) == want
+    n = 200_000
+    x = rng.integers(0, 2 ** 32, n, dtype=np.uint64).astype(np.uint32)
+    m = rng.integers(0, 2 ** 32, n, dtype=np.uint64).astype(np.uint32)
+    m[::3] &= rng.integers(0, 2 ** 32, len(m[::3]), dtype=np.uint64).astype(np.uint32)   # sparse
+    m[1::7] = 0xFFFFFFFF
+    m[2::11] = 0
+    m[3::13] = 0x80000001
+    assert np.array_equal(_hd_compress(x, m), _pext_ref(x, m))
+
+
+def _sparse_compress(x, m):
+    """The sparse-mask sequence of proj.cu's pext_item<G, true> (generation 3): the mask's trailing
+    ones stay, every further set bit p of rank i comes from bit i of (x >> (p - i)), the shift as
+    umulhi(x, 2^(32 - (p - i)))."""
+    c = bin(m).count("1")
+    i0 = 32 if m == 0xFFFFFFFF else ((~m & 0xFFFFFFFF) & -(~m & 0xFFFFFFFF)).bit_length() - 1
+    idm = 0xFFFFFFFF if i0 >= 32 else (1 << i0) - 1
+    y, mm, i = x & idm, m & ~idm & 0xFFFFFFFF, i0
+    for _ in range(c - min(i0, c)):
+        p = (mm & -mm).bit_length() - 1
+        mm &= mm - 1
+        y |= ((x * (1 << (32 - (p - i)))) >> 32) & (1 << i)
+        i += 1
+    return y
+
+
+def test_sparse_compress_matches_pext():
+    rng = np.random.default_rng(12)
+    xs = rng.integers(0, 2 ** 32, 20000, dtype=np.uint64).tolist()
+    ms = rng.integers(0, 2 ** 32, 20000, dtype=np.uint64)
+    ms[::2] &= rng.integers(0, 2 ** 32, 10000, dtype=np.uint64) & rng.integers(0, 2 ** 32, 10000, dtype=np.uint64)
+    ms[1::9] = 0xFFFFFFFF
+    ms[2::11] = 0
+    ms[3::13] = 0x0000FFFF | 0x80000000
+    ms = ms.tolist()
+    ref = _pext_ref(np.array(xs, dtype=np.uint32), np.array(ms, dtype=np.uint32)).tolist()
+    assert [_sparse_compress(x, m) for x, m in zip(xs, ms)] == ref
