@@ -30,6 +30,17 @@ void launch_bitset_build(const uint64_t* offsets, const uint32_t* items, uint64_
                          const int32_t* row_of_item, uint32_t n_items, uint32_t n_rows, uint64_t pitch_words,
                          uint32_t* rows, uint64_t tx_begin, uint64_t tx_end, cudaStream_t stream);
 
+// Generation-1 counts AND the static bitset of ALL item ids (row = item id, n_items rows of
+// pitch_words) in one read of the CSR (bitset.cu scan_build_kernel): hist[i] += popcount of row i
+// over this range (set semantics), flags |= kFlagBad*.  hist, flags zeroed by the caller.  Needs
+// scan_build_supported(n_items, items) (n_items <= 1,024 and 16-byte aligned items).
+bool scan_build_supported(uint32_t n_items, const void* items);
+void launch_scan_build(const uint64_t* offsets, const uint32_t* items, uint64_t n_tx, uint64_t nnz, uint32_t n_items,
+                       uint64_t pitch_words, uint32_t* rows, uint32_t* hist, uint32_t* flags, cudaStream_t stream);
+// In place: row r <- row sel[r] for r in [r0, n_sel) (sel ascending, sel[r] >= r).
+void launch_compact_rows(uint32_t* rows, const uint32_t* sel, uint32_t r0, uint32_t n_sel, uint64_t pitch_words,
+                         int n_sms, cudaStream_t stream);
+
 // ---- support counting (complete intersection, P18@394-2515)
 // Paper design: one CTA per candidate, AND of all k rows, popc, block reduction.
 void launch_count_v0(const uint32_t* rows, uint64_t pitch_words, const uint32_t* cand_rows, uint32_t k,

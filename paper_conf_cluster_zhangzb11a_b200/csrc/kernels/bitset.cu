@@ -89,7 +89,168 @@ __global__ void __launch_bounds__(kBuildThreads) bitset_build_kernel(const uint6
   }
 }
 
+// ---------------------------------------------------------------- one pass: histogram + bitset
+// Generation 1 AND the static bitset from ONE read of the CSR (the database is read once, as
+// the paper copies it once, P18@755): CTA = one 512-transaction chunk, a shared-memory tile of
+// ALL n_items rows (identity row map; n_items <= kScanMaxItems), the chunk's items streamed into
+// shared memory by cp.async.bulk (double-buffered 16 KB pieces: bytes in flight without
+// registers), bits set with shared atomicOr, then every row's 64-byte segment written out and its
+// popcount added to hist[item] -- the generation-1 count with set semantics (a duplicate item
+// sets the same bit; P3@441), so non-canonical input needs no de-duplication pass.  Validation:
+// offsets monotone and <= nnz, items < n_items (flags).
+constexpr uint32_t kScanMaxItems = 1024;
+constexpr uint32_t kPiece = 4096;          // items per bulk-copy piece (16 KB)
+constexpr int kScanThreads = 256;
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
+}
+
+__global__ void __launch_bounds__(kScanThreads) scan_build_kernel(const uint64_t* __restrict__ offsets,
+                                                                  const uint32_t* __restrict__ items,
+                                                                  uint64_t n_tx, uint64_t nnz, uint32_t n_items,
+                                                                  uint64_t chunk0, uint64_t pitch_words,
+                                                                  uint32_t* __restrict__ rows,
+                                                                  uint32_t* __restrict__ hist,
+                                                                  uint32_t* __restrict__ flags) {
+  extern __shared__ __align__(16) uint32_t dyn[];
+  uint32_t* buf = dyn;                                   // 2 x (kPiece + 4) items (16-byte aligned pieces)
+  uint32_t* tile = dyn + 2 * (kPiece + 4);               // n_items x kTileStride words
+  __shared__ uint32_t soff[kChunkTx + 1];
+  __shared__ __align__(8) uint64_t bar[2];
+  __shared__ uint32_t s_flags;
+  const uint64_t chunk = chunk0 + blockIdx.x;
+  for (uint32_t i = threadIdx.x; i < n_items * kTileStride; i += blockDim.x) tile[i] = 0;
+  if (threadIdx.x == 0) {
+    s_flags = 0;
+    asm volatile("mbarrier.init.shared.b64 [%0], 1;" ::"r"(smem_u32(&bar[0])));
+    asm volatile("mbarrier.init.shared.b64 [%0], 1;" ::"r"(smem_u32(&bar[1])));
+    asm volatile("fence.mbarrier_init.release.cluster;");
+  }
+  const uint64_t t0 = chunk * kChunkTx;
+  const uint64_t te = t0 < n_tx ? t0 : n_tx;
+  const uint64_t A = min(__ldg(offsets + te), nnz);
+  uint32_t my_flags = 0;
+  for (uint32_t i = threadIdx.x; i <= kChunkTx; i += blockDim.x) {
+    const uint64_t t = t0 + i < n_tx ? t0 + i : n_tx;
+    const uint64_t o_raw = __ldg(offsets + t);
+    if (o_raw > nnz) my_flags |= kFlagBadOffsets;
+    if (i > 0 && t0 + i <= n_tx && o_raw < __ldg(offsets + t - 1)) my_flags |= kFlagBadOffsets;
+    const uint64_t o = min(max(o_raw, A), nnz);
+    soff[i] = (uint32_t)(o - A < 0xffffffffull ? o - A : 0xffffffffull);
+  }
+  __syncthreads();
+  const uint32_t n_it = soff[kChunkTx];
+  // pieces: items [A + p kPiece, ...) copied from the 16-byte aligned index at or below (the
+  // items pointer is 16-byte aligned, checked by the launcher), never past the last whole 16-byte
+  // group of the array: the last <= 3 items of the array are read from global memory directly
+  const uint64_t cend = nnz & ~3ull;
+  const uint32_t n_pieces = (n_it + kPiece - 1) / kPiece;
+  auto issue = [&](uint32_t p) {
+    const uint64_t first = A + (uint64_t)p * kPiece;
+    const uint64_t last = A + min(n_it, (p + 1) * kPiece);       // exclusive
+    const uint64_t a0 = first & ~3ull, a1 = ((last + 3) & ~3ull) < cend ? ((last + 3) & ~3ull) : cend;
+    if (a1 <= a0) {   // nothing copyable: complete the phase without a copy
+      asm volatile("mbarrier.arrive.shared.b64 _, [%0];" ::"r"(smem_u32(&bar[p & 1])) : "memory");
+      return;
+    }
+    const uint32_t bytes = (uint32_t)((a1 - a0) * 4);
+    const uint32_t b = smem_u32(&bar[p & 1]);
+    asm volatile("mbarrier.arrive.expect_tx.shared.b64 _, [%0], %1;" ::"r"(b), "r"(bytes) : "memory");
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                 ::"r"(smem_u32(buf + (p & 1) * (kPiece + 4))), "l"(items + a0), "r"(bytes), "r"(b) : "memory");
+  };
+  if (threadIdx.x == 0 && n_pieces > 0) {
+    issue(0);
+    if (n_pieces > 1) issue(1);
+  }
+  for (uint32_t p = 0; p < n_pieces; ++p) {
+    const uint32_t b = smem_u32(&bar[p & 1]);
+    const uint32_t parity = (p >> 1) & 1;
+    asm volatile("{ .reg .pred P; WAIT_%=: mbarrier.try_wait.parity.shared.b64 P, [%0], %1; @!P bra WAIT_%=; }"
+                 ::"r"(b), "r"(parity) : "memory");
+    const uint32_t q0 = p * kPiece, q1 = min(n_it, q0 + kPiece);
+    const uint32_t head = (uint32_t)((A + q0) & 3ull);
+    const uint32_t* pb = buf + (p & 1) * (kPiece + 4) + head;
+    // thread k: 16 consecutive items, the transaction of its first by binary search, then a walk
+    for (uint32_t q = q0 + threadIdx.x * 16; q < q1; q += blockDim.x * 16) {
+      uint32_t lo = 0, hi = kChunkTx;   // tx = last with soff[tx] <= q
+      while (lo + 1 < hi) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (soff[mid] <= q) lo = mid; else hi = mid;
+      }
+      uint32_t tx = lo;
+      const uint32_t qe = min(q1, q + 16);
+      for (uint32_t j = q; j < qe; ++j) {
+        while (tx + 1 < kChunkTx && soff[tx + 1] <= j) ++tx;
+        const uint32_t x = A + j < cend ? pb[j - q0] : __ldg(items + A + j);
+        if (x < n_items) atomicOr(&tile[x * kTileStride + (tx >> 5)], 1u << (tx & 31));
+        else my_flags |= kFlagBadItem;
+      }
+    }
+    __syncthreads();   // every thread is done with buffer p & 1
+    if (threadIdx.x == 0 && p + 2 < n_pieces) issue(p + 2);
+  }
+  // out: row segments (coalesced 64 B per row) and their popcounts into the histogram
+  uint32_t* out = rows + chunk * kChunkWords;
+  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  for (uint32_t r0 = warp * 2; r0 < n_items; r0 += 2 * (kScanThreads / 32)) {   // a warp: 2 rows of 16 words
+    const uint32_t r = r0 + (lane >> 4), w = lane & 15;
+    uint32_t v = 0;
+    if (r < n_items) {
+      v = tile[r * kTileStride + w];
+      out[(uint64_t)r * pitch_words + w] = v;
+    }
+    uint32_t c = __popc(v);
+#pragma unroll
+    for (uint32_t d = 8; d >= 1; d >>= 1) c += __shfl_xor_sync(0xffffffffu, c, d);
+    if ((lane & 15) == 0 && r < n_items && c) atomicAdd(&hist[r], c);
+  }
+  if (my_flags) atomicOr(&s_flags, my_flags);
+  __syncthreads();
+  if (threadIdx.x == 0 && s_flags) atomicOr(flags, s_flags);
+}
+
+// In-place compaction of a full bitset (row = item id) to the rows of the selected items
+// (sel ascending, sel[r] >= r): row r <- row sel[r] for r >= r0.  Each thread owns a column of
+// 16-byte words and walks the rows in increasing r; a row is only read at an iteration <= the one
+// that overwrites it (sel[r] >= r), so per-address program order makes it race-free.
+__global__ void compact_rows_kernel(uint4* __restrict__ rows, const uint32_t* __restrict__ sel, uint32_t r0,
+                                    uint32_t n_sel, uint64_t pitch4) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < pitch4; i += (uint64_t)gridDim.x * blockDim.x)
+    for (uint32_t r = r0; r < n_sel; ++r) rows[(uint64_t)r * pitch4 + i] = rows[(uint64_t)sel[r] * pitch4 + i];
+}
+
 }  // namespace
+
+bool scan_build_supported(uint32_t n_items, const void* items) {
+  return n_items >= 1 && n_items <= kScanMaxItems && ((uintptr_t)items & 15) == 0;
+}
+
+void launch_scan_build(const uint64_t* offsets, const uint32_t* items, uint64_t n_tx, uint64_t nnz, uint32_t n_items,
+                       uint64_t pitch_words, uint32_t* rows, uint32_t* hist, uint32_t* flags, cudaStream_t stream) {
+  GPA_REQUIRE(scan_build_supported(n_items, items), GPA_ERR_INVALID, "scan_build: n_items %u or items unaligned",
+              n_items);
+  const uint64_t n_chunks = pitch_words / kChunkWords;   // the padding chunks write zeros
+  GPA_REQUIRE(n_chunks < (1ull << 31), GPA_ERR_INVALID, "scan_build: too many transactions");
+  const size_t smem = (2 * (kPiece + 4) + (size_t)n_items * kTileStride) * sizeof(uint32_t);
+  ensure_smem_attr(reinterpret_cast<const void*>(scan_build_kernel), (int)smem);
+  { scan_build_kernel<<<(unsigned)n_chunks, kScanThreads, smem, stream>>>(offsets, items, n_tx, nnz, n_items, 0,
+                                                                         pitch_words, rows, hist, flags);
+    note_launch(); }
+  GPA_CUDA(cudaGetLastError());
+}
+
+void launch_compact_rows(uint32_t* rows, const uint32_t* sel, uint32_t r0, uint32_t n_sel, uint64_t pitch_words,
+                         int n_sms, cudaStream_t stream) {
+  if (r0 >= n_sel) return;
+  const uint64_t pitch4 = pitch_words / 4;
+  const uint64_t want = (pitch4 + 255) / 256;
+  const unsigned grid = (unsigned)std::min<uint64_t>(want, (uint64_t)n_sms * 8);
+  { compact_rows_kernel<<<grid, 256, 0, stream>>>(reinterpret_cast<uint4*>(rows), sel, r0, n_sel, pitch4);
+    note_launch(); }
+  GPA_CUDA(cudaGetLastError());
+}
 
 void launch_bitset_build(const uint64_t* offsets, const uint32_t* items, uint64_t n_tx, uint64_t nnz,
                          const int32_t* row_of_item,

@@ -131,13 +131,23 @@ gpa_bitset* bitset_build(const gpa_tx_csr* db, uint64_t row_min_count, const gpa
   GPA_CUDA(cudaMemsetAsync(d_hist.p, 0, std::max<uint32_t>(n_items, 1) * sizeof(uint32_t), s));
   GPA_CUDA(cudaMemsetAsync(d_flags.p, 0, sizeof(uint32_t), s));
   GPA_CUDA(cudaMemcpyAsync(d_ntx.p, &bs->n_tx_local, sizeof(uint64_t), cudaMemcpyHostToDevice, s));
-  launch_hist_validate(off_dev, items_dev, n_tx, nnz, n_items, d_hist.p, d_flags.p, bs->n_sms, s);
+  bs->pitch_words = pitch_words_for(n_tx);
+  // up to 1,024 item ids: ONE read of the CSR builds the rows of every item id and their popcounts
+  // are the generation-1 counts (scan_build); the L_1 rows are compacted afterwards.  Otherwise a
+  // histogram pass, then the build of the L_1 rows (a second read).
+  const bool scan = n_tx > 0 && scan_build_supported(n_items, items_dev);
   uint32_t flags = 0;
-  GPA_CUDA(cudaMemcpyAsync(&flags, d_flags.p, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
-  stream_wait(s);
-  if ((flags & kFlagNonCanonical) && !(flags & (kFlagBadItem | kFlagBadOffsets))) {
-    GPA_CUDA(cudaMemsetAsync(d_hist.p, 0, n_items * sizeof(uint32_t), s));
-    launch_hist_dedup(off_dev, items_dev, n_tx, nnz, n_items, d_hist.p, bs->n_sms, s);
+  if (scan) {
+    bs->rows.alloc((size_t)n_items * bs->pitch_words, s);
+    launch_scan_build(off_dev, items_dev, n_tx, nnz, n_items, bs->pitch_words, bs->rows.p, d_hist.p, d_flags.p, s);
+  } else {
+    launch_hist_validate(off_dev, items_dev, n_tx, nnz, n_items, d_hist.p, d_flags.p, bs->n_sms, s);
+    GPA_CUDA(cudaMemcpyAsync(&flags, d_flags.p, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+    stream_wait(s);
+    if ((flags & kFlagNonCanonical) && !(flags & (kFlagBadItem | kFlagBadOffsets))) {
+      GPA_CUDA(cudaMemsetAsync(d_hist.p, 0, n_items * sizeof(uint32_t), s));
+      launch_hist_dedup(off_dev, items_dev, n_tx, nnz, n_items, d_hist.p, bs->n_sms, s);
+    }
   }
   allreduce_max_u32(dist, d_flags.p, 1, s);   // every rank takes the same accept / reject decision
   allreduce_sum_u32(dist, d_hist.p, n_items, s);
@@ -167,8 +177,19 @@ gpa_bitset* bitset_build(const gpa_tx_csr* db, uint64_t row_min_count, const gpa
     }
   }
   bs->n_rows = (uint32_t)bs->item_of_row.size();
-  bs->pitch_words = pitch_words_for(n_tx);
-  if (bs->n_rows) {
+  if (scan) {
+    // row r <- row item_of_row[r] from the first row whose item differs (in place)
+    uint32_t r0 = 0;
+    while (r0 < bs->n_rows && bs->item_of_row[r0] == r0) ++r0;
+    if (r0 < bs->n_rows) {
+      DBuf<uint32_t> d_sel;
+      d_sel.alloc(bs->n_rows, s);
+      GPA_CUDA(cudaMemcpyAsync(d_sel.p, bs->item_of_row.data(), bs->n_rows * sizeof(uint32_t), cudaMemcpyHostToDevice,
+                               s));
+      launch_compact_rows(bs->rows.p, d_sel.p, r0, bs->n_rows, bs->pitch_words, bs->n_sms, s);
+      stream_wait(s);   // d_sel is freed at scope exit (stream-ordered, but keep the phase timing honest)
+    }
+  } else if (bs->n_rows) {
     DBuf<int32_t> d_map;
     d_map.alloc(n_items, s);
     GPA_CUDA(cudaMemcpyAsync(d_map.p, bs->row_of_item.data(), n_items * sizeof(int32_t), cudaMemcpyHostToDevice, s));
