@@ -3,7 +3,7 @@
 #pragma once
 #include <atomic>
 #include <mutex>
-#include <set>
+#include <map>
 #include <cstdint>
 #include <cstdio>
 #include <string>
@@ -133,19 +133,19 @@ struct PBuf {
 };
 
 // cudaFuncAttributeMaxDynamicSharedMemorySize is a per-DEVICE attribute of a kernel: raise it
-// once per (kernel, device) under a lock (a second device or a concurrent thread must not launch
-// without it).
+// per (kernel, device) to the largest size requested so far, under a lock (a second device or a
+// concurrent thread must not launch without it; a smaller request never lowers it).
 inline void ensure_smem_attr(const void* func, int bytes) {
   static std::mutex mu;
-  static std::set<std::pair<std::pair<const void*, int>, int>> done;
+  static std::map<std::pair<const void*, int>, int> set_to;
   int dev = 0;
   if (cudaGetDevice(&dev) != cudaSuccess) fail(GPA_ERR_CUDA, "cudaGetDevice failed");
   std::lock_guard<std::mutex> lk(mu);
-  auto key = std::make_pair(std::make_pair(func, dev), bytes);
-  if (done.count(key)) return;
+  int& cur = set_to[std::make_pair(func, dev)];
+  if (bytes <= cur) return;
   cudaError_t e = cudaFuncSetAttribute(func, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
   if (e != cudaSuccess) fail(GPA_ERR_CUDA, "cudaFuncSetAttribute failed: %s", cudaGetErrorString(e));
-  done.insert(key);
+  cur = bytes;
 }
 
 // Flags written by the validation/histogram kernel.

@@ -133,12 +133,13 @@ struct DeviceBatch {
   uint32_t k = 0, M = 0, G = 0;
   DBuf<uint32_t> prefix, ext_off, ext, gpar, eidx;
 };
-// L_k = candidates of C_k with count >= theta, in order (k = 2: all pairs of n_rows rows in
-// pair_index order; k >= 3: the grouped batch prefix/ext_off/ext).  Returns |L_k| (synchronises).
-// With gpar / eidx (k >= 3) or always for k = 2, also out.par_a / out.par_b.
+// L_k = candidates of C_k with count >= theta, in order (k = 2: all pairs of n_rows L_1 entries in
+// pair_index order, mapped to bitset rows through sel when non-null; k >= 3: the grouped batch
+// prefix/ext_off/ext).  Returns |L_k| (synchronises).  With gpar / eidx (k >= 3) or always for
+// k = 2, also out.par_a / out.par_b.
 uint32_t device_threshold(const uint32_t* counts, uint32_t M, uint32_t theta, uint32_t k, uint32_t n_rows,
-                          const uint32_t* prefix, const uint32_t* ext_off, const uint32_t* ext, uint32_t G,
-                          const uint32_t* gpar, const uint32_t* eidx,
+                          const uint32_t* sel, const uint32_t* prefix, const uint32_t* ext_off, const uint32_t* ext,
+                          uint32_t G, const uint32_t* gpar, const uint32_t* eidx,
                           DeviceLevel& out, DeviceScratch& scratch, int n_sms, cudaStream_t s);
 
 // ---- association rules (rules.cu): F as n itemsets in canonical order (items at

@@ -171,19 +171,31 @@ __global__ void __launch_bounds__(kScanThreads) scan_build_kernel(const uint64_t
                  ::"r"(b), "r"(parity) : "memory");
     const uint32_t q0 = p * kPiece, q1 = min(n_it, q0 + kPiece);
     const uint32_t head = (uint32_t)((A + q0) & 3ull);
-    const uint32_t* pb = buf + (p & 1) * (kPiece + 4) + head;
-    // thread k: 16 consecutive items, the transaction of its first by binary search, then a walk
-    for (uint32_t q = q0 + threadIdx.x * 16; q < q1; q += blockDim.x * 16) {
-      uint32_t lo = 0, hi = kChunkTx;   // tx = last with soff[tx] <= q
+    const uint4* pb = reinterpret_cast<const uint4*>(buf + (p & 1) * (kPiece + 4));   // 16-byte groups
+    // warp step = 32 aligned 16-byte groups of the buffer (128 items, one LDS.128 per lane:
+    // conflict-free); the transaction of the step's first item by a warp-uniform binary search,
+    // each lane's by a short walk from there
+    const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const uint32_t n_groups = (head + (q1 - q0) + 3) / 4;
+    for (uint32_t g0 = warp * 32; g0 < n_groups; g0 += (kScanThreads / 32) * 32) {
+      const uint32_t jw = q0 + (g0 * 4 > head ? g0 * 4 - head : 0u);   // first item of the step
+      uint32_t lo = 0, hi = kChunkTx;   // last tx with soff[tx] <= jw
       while (lo + 1 < hi) {
         const uint32_t mid = (lo + hi) >> 1;
-        if (soff[mid] <= q) lo = mid; else hi = mid;
+        if (soff[mid] <= jw) lo = mid; else hi = mid;
       }
+      const uint32_t g = g0 + lane;
+      if (g >= n_groups) continue;
+      const uint4 v = pb[g];
+      const uint32_t xs[4] = {v.x, v.y, v.z, v.w};
       uint32_t tx = lo;
-      const uint32_t qe = min(q1, q + 16);
-      for (uint32_t j = q; j < qe; ++j) {
+#pragma unroll
+      for (uint32_t i = 0; i < 4; ++i) {
+        const int64_t jj = (int64_t)q0 + (int64_t)(4 * g + i) - (int64_t)head;   // item index in the chunk
+        if (jj < (int64_t)q0 || jj >= (int64_t)q1) continue;
+        const uint32_t j = (uint32_t)jj;
         while (tx + 1 < kChunkTx && soff[tx + 1] <= j) ++tx;
-        const uint32_t x = A + j < cend ? pb[j - q0] : __ldg(items + A + j);
+        const uint32_t x = A + j < cend ? xs[i] : __ldg(items + A + j);
         if (x < n_items) atomicOr(&tile[x * kTileStride + (tx >> 5)], 1u << (tx & 31));
         else my_flags |= kFlagBadItem;
       }
@@ -193,7 +205,7 @@ __global__ void __launch_bounds__(kScanThreads) scan_build_kernel(const uint64_t
   }
   // out: row segments (coalesced 64 B per row) and their popcounts into the histogram
   uint32_t* out = rows + chunk * kChunkWords;
-  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;   // (as in the sweep)
   for (uint32_t r0 = warp * 2; r0 < n_items; r0 += 2 * (kScanThreads / 32)) {   // a warp: 2 rows of 16 words
     const uint32_t r = r0 + (lane >> 4), w = lane & 15;
     uint32_t v = 0;

@@ -74,7 +74,8 @@ __global__ void flag_ge_kernel(const uint32_t* __restrict__ counts, uint32_t M, 
 
 // k = 2: candidate m is the pair (a, b) of pair_index order over n rows
 __global__ void scatter_pairs_kernel(const uint32_t* __restrict__ counts, const uint32_t* __restrict__ flags,
-                                     const uint32_t* __restrict__ pos, uint32_t M, uint32_t n, uint32_t* L,
+                                     const uint32_t* __restrict__ pos, uint32_t M, uint32_t n,
+                                     const uint32_t* __restrict__ sel, uint32_t* L,
                                      uint32_t* sup, uint32_t* par_a, uint32_t* par_b) {
   for (uint32_t m = blockIdx.x * blockDim.x + threadIdx.x; m < M; m += gridDim.x * blockDim.x) {
     if (!flags[m]) continue;
@@ -83,7 +84,11 @@ __global__ void scatter_pairs_kernel(const uint32_t* __restrict__ counts, const 
       const uint32_t mid = (lo + hi) >> 1;
       if (pair_index(mid, mid + 1, n) <= m) lo = mid; else hi = mid;
     }
-    const uint32_t a = lo, b = (uint32_t)(m - pair_index(a, a + 1, n)) + a + 1;
+    uint32_t a = lo, b = (uint32_t)(m - pair_index(a, a + 1, n)) + a + 1;
+    if (sel) {   // logical L_1 indices -> bitset rows
+      a = sel[a];
+      b = sel[b];
+    }
     const uint32_t p = pos[m];
     L[2ull * p] = a;
     L[2ull * p + 1] = b;
@@ -257,8 +262,8 @@ void exclusive_scan(const uint32_t* in, uint32_t* out, uint32_t n, uint32_t* tot
 }  // namespace
 
 uint32_t device_threshold(const uint32_t* counts, uint32_t M, uint32_t theta, uint32_t k, uint32_t n_rows,
-                          const uint32_t* prefix, const uint32_t* ext_off, const uint32_t* ext, uint32_t G,
-                          const uint32_t* gpar, const uint32_t* eidx,
+                          const uint32_t* sel, const uint32_t* prefix, const uint32_t* ext_off, const uint32_t* ext,
+                          uint32_t G, const uint32_t* gpar, const uint32_t* eidx,
                           DeviceLevel& out, DeviceScratch& scratch, int n_sms, cudaStream_t s) {
   out.k = k;
   out.n = 0;
@@ -278,7 +283,7 @@ uint32_t device_threshold(const uint32_t* counts, uint32_t M, uint32_t theta, ui
   out.par_b.ensure(std::max<uint32_t>(F, 1), s);
   if (F) {
     if (k == 2)
-      { scatter_pairs_kernel<<<grid_for(M, n_sms), kThreads, 0, s>>>(counts, flags, pos, M, n_rows, out.rows.p,
+      { scatter_pairs_kernel<<<grid_for(M, n_sms), kThreads, 0, s>>>(counts, flags, pos, M, n_rows, sel, out.rows.p,
                                                                   out.sup.p, out.par_a.p, out.par_b.p); note_launch(); }
     else
       { scatter_grouped_kernel<<<grid_for(M, n_sms), kThreads, 0, s>>>(counts, flags, pos, M, prefix, ext_off, ext, G,

@@ -55,7 +55,7 @@ void validate_options(const gpa_options& o) {
 }  // namespace
 
 gpa_bitset* bitset_build(const gpa_tx_csr* db, uint64_t row_min_count, const gpa_dist* dist, const gpa_options* opt_in,
-                         bool prechecked) {
+                         bool prechecked, bool keep_all_rows) {
   GPA_REQUIRE(db, GPA_ERR_INVALID, "db is NULL");   // a caller bug, not data: checked before any device work
   gpa_options opt;
   gpa_options_default(&opt);
@@ -177,7 +177,17 @@ gpa_bitset* bitset_build(const gpa_tx_csr* db, uint64_t row_min_count, const gpa
     }
   }
   bs->n_rows = (uint32_t)bs->item_of_row.size();
-  if (scan) {
+  if (scan && keep_all_rows) {
+    // the one-pass build left a row for every item id: keep them (row = item id) and list L_1
+    bs->l1 = bs->item_of_row;
+    bs->item_of_row.resize(n_items);
+    for (uint32_t i = 0; i < n_items; ++i) {
+      bs->item_of_row[i] = i;
+      bs->row_of_item[i] = (int32_t)i;
+    }
+    bs->n_rows = n_items;
+    if (bs->l1.size() == n_items) bs->l1.clear();   // every row is in L_1
+  } else if (scan) {
     // row r <- row item_of_row[r] from the first row whose item differs (in place)
     uint32_t r0 = 0;
     while (r0 < bs->n_rows && bs->item_of_row[r0] == r0) ++r0;
@@ -217,6 +227,8 @@ void bitset_free(gpa_bitset* bs) {
   bs->d_lrows.reset();
   bs->d_lcp.reset();
   bs->d_cgroup.reset();
+  bs->d_l1.reset();
+  bs->d_pairs_all.reset();
   if (bs->stream) cudaStreamSynchronize(bs->stream);
   if (bs->ev0) cudaEventDestroy(bs->ev0);
   if (bs->ev1) cudaEventDestroy(bs->ev1);
@@ -461,17 +473,19 @@ void count_grouped(gpa_bitset* bs, const GroupedBatch& b, uint32_t kernel, Count
 
 void count_all_pairs(gpa_bitset* bs, uint32_t kernel, CountStats* st) {
   cudaStream_t s = bs->stream;
-  const uint64_t n = bs->n_rows;
+  const uint64_t n = l1_size(bs);
   const uint64_t M = n * (n - 1) / 2;
   if (n < 2) return;
+  const bool sub = !bs->l1.empty();   // L_1 is a subset of the rows
   if (kernel == GPA_KERNEL_AUTO || kernel == GPA_KERNEL_PROJ) kernel = GPA_KERNEL_PAIRS_TC;
   if (kernel != GPA_KERNEL_PAIRS && kernel != GPA_KERNEL_PAIRS_TC) {
     GroupedBatch b;
     b.k = 2;
     b.ext_off.push_back(0);
+    auto row = [&](uint64_t i) { return sub ? bs->l1[i] : (uint32_t)i; };
     for (uint64_t a = 0; a + 1 < n; ++a) {
-      b.prefix.push_back((uint32_t)a);
-      for (uint64_t c = a + 1; c < n; ++c) b.ext.push_back((uint32_t)c);
+      b.prefix.push_back(row(a));
+      for (uint64_t c = a + 1; c < n; ++c) b.ext.push_back(row(c));
       b.ext_off.push_back(b.ext.size());
     }
     count_grouped(bs, b, kernel, st);
@@ -481,14 +495,27 @@ void count_all_pairs(gpa_bitset* bs, uint32_t kernel, CountStats* st) {
     make_pairs_tensor_map(bs->tmap, bs->rows.p, bs->n_rows, bs->pitch_words);
     bs->tmap_ready = true;
   }
+  // the pair Gram over every row, then (L_1 a subset) the L_1 pairs gathered out of it
+  const uint64_t P = (uint64_t)bs->n_rows * (bs->n_rows - 1) / 2;
+  uint32_t* dst = bs->d_counts.p;
   bs->d_counts.ensure(M, s);
-  GPA_CUDA(cudaMemsetAsync(bs->d_counts.p, 0, M * sizeof(uint32_t), s));
+  dst = bs->d_counts.p;
+  if (sub) {
+    bs->d_pairs_all.ensure(P, s);
+    dst = bs->d_pairs_all.p;
+    if (bs->d_l1.n < n) {
+      bs->d_l1.alloc(n, s);
+      GPA_CUDA(cudaMemcpyAsync(bs->d_l1.p, bs->l1.data(), n * 4, cudaMemcpyHostToDevice, s));
+    }
+  }
+  GPA_CUDA(cudaMemsetAsync(dst, 0, (sub ? P : M) * sizeof(uint32_t), s));
   GPA_CUDA(cudaEventRecord(ev_start(bs, st), s));
   if (kernel == GPA_KERNEL_PAIRS_TC)
-    launch_count_pairs_tc(bs->rows.p, bs->pitch_words, bs->n_rows, 0, bs->pitch_words, bs->d_counts.p, bs->n_sms, s);
+    launch_count_pairs_tc(bs->rows.p, bs->pitch_words, bs->n_rows, 0, bs->pitch_words, dst, bs->n_sms, s);
   else
-    launch_count_pairs(bs->tmap, bs->n_rows, 0, bs->pitch_words, bs->d_counts.p, bs->n_sms, s);
-  if (st) { st->kernel = kernel; st->launches = 1; }
+    launch_count_pairs(bs->tmap, bs->n_rows, 0, bs->pitch_words, dst, bs->n_sms, s);
+  if (sub) launch_pairs_subset(dst, bs->n_rows, bs->d_l1.p, (uint32_t)n, bs->d_counts.p, bs->n_sms, s);
+  if (st) { st->kernel = kernel; st->launches = sub ? 2 : 1; }
   finish_counts(bs, M, st);
 }
 

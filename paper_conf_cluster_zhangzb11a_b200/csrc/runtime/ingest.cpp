@@ -276,17 +276,23 @@ gpa_bitset* bitset_build_overlapped(const gpa_tx_csr* db, uint64_t row_min_count
   }
   bs->n_rows = (uint32_t)bs->item_of_row.size();
   if (bs->n_rows) {
-    bs->rows.alloc((size_t)bs->n_rows * bs->pitch_words, s);
     if (subset) {
+      // L_1 within R0: the R0 bitset IS the static bitset (no row copy); L_1 is listed in bs->l1
+      // (R0 row ids) unless it is all of R0
+      const uint32_t n1 = bs->n_rows;
+      bs->rows = std::move(d_r0rows);
+      bs->item_of_row = r0_items;
+      bs->row_of_item = r0_of_item;
+      bs->n_rows = nr0;
+      if (n1 < nr0) bs->l1 = sel;
       DBuf<uint32_t> d_sel;
-      d_sel.alloc(bs->n_rows, s);
-      GPA_CUDA(cudaMemcpyAsync(d_sel.p, sel.data(), bs->n_rows * 4, cudaMemcpyHostToDevice, s));
-      launch_gather_rows(d_r0rows.p, d_sel.p, bs->n_rows, bs->pitch_words, bs->rows.p, bs->n_sms, s);
-      if (bs->n_rows >= 2) {
-        const uint64_t P = (uint64_t)bs->n_rows * (bs->n_rows - 1) / 2;
+      d_sel.alloc(n1, s);
+      GPA_CUDA(cudaMemcpyAsync(d_sel.p, sel.data(), n1 * 4, cudaMemcpyHostToDevice, s));
+      if (n1 >= 2) {
+        const uint64_t P = (uint64_t)n1 * (n1 - 1) / 2;
         bs->d_counts.ensure(P, s);
         GPA_CUDA(cudaEventRecord(bs->ev0, s));
-        launch_pairs_subset(d_r0pairs.p, nr0, d_sel.p, bs->n_rows, bs->d_counts.p, bs->n_sms, s);
+        launch_pairs_subset(d_r0pairs.p, nr0, d_sel.p, n1, bs->d_counts.p, bs->n_sms, s);
         GPA_CUDA(cudaEventRecord(bs->ev1, s));
         GPA_CUDA(cudaEventSynchronize(bs->ev1));
         float ms = 0;
@@ -301,6 +307,7 @@ gpa_bitset* bitset_build_overlapped(const gpa_tx_csr* db, uint64_t row_min_count
       }
     } else {
       // R0 missed a frequent item: rebuild the L_1 bitset from the device CSR (exact fallback)
+      bs->rows.alloc((size_t)bs->n_rows * bs->pitch_words, s);
       DBuf<int32_t> d_map;
       d_map.alloc(n_items, s);
       GPA_CUDA(cudaMemcpyAsync(d_map.p, bs->row_of_item.data(), n_items * 4, cudaMemcpyHostToDevice, s));

@@ -137,6 +137,11 @@ struct gpa_bitset {
   std::vector<uint32_t> item_counts;   // global, n_items
   std::vector<uint32_t> item_of_row;   // n_rows, ascending
   std::vector<int32_t> row_of_item;    // n_items, -1 if no row
+  // gpa_mine: the rows of L_1 when the bitset holds more rows than L_1 (all item ids after the
+  // one-pass build, the chunk-0 estimate R0 after the overlapped ingest): ascending row ids; empty =
+  // every row is in L_1.  Generation 2 counts pairs of these rows; L_k holds bitset row ids.
+  std::vector<uint32_t> l1;
+  gpa::DBuf<uint32_t> d_l1, d_pairs_all;
   alignas(64) unsigned char tmap[128];
   bool tmap_ready = false;
   // counting workspace (grow-only)
@@ -154,8 +159,12 @@ struct gpa_bitset {
 namespace gpa {
 // Build the static bitset (histogram, rows, bitset) -- shared by gpa_bitset_create / gpa_mine.
 // prechecked: the caller already ran agree_input for db (gpa_mine)
+// keep_all_rows (gpa_mine): with the one-pass build, keep the rows of every item id and list
+// L_1 in bs->l1 instead of compacting the rows.
 gpa_bitset* bitset_build(const gpa_tx_csr* db, uint64_t row_min_count, const gpa_dist* dist, const gpa_options* opt,
-                         bool prechecked = false);
+                         bool prechecked = false, bool keep_all_rows = false);
+// number of L_1 rows (bs->l1, or every row)
+inline uint32_t l1_size(const gpa_bitset* bs) { return bs->l1.empty() ? bs->n_rows : (uint32_t)bs->l1.size(); }
 void bitset_free(gpa_bitset* bs);
 // Host input, end to end: upload in transaction chunks overlapped with histogram, bitset build and
 // generation-2 pair counting (runtime/ingest.cpp).  *pairs_ready: bs->d_counts holds the L_1 pair
@@ -180,6 +189,7 @@ bool count_device_batch(gpa_bitset* bs, DeviceBatch& B, uint32_t kernel, DeviceS
 // After a counting launch: end event, all-reduce of the M counts (dist), and the timing (no sync
 // when st carries caller-owned events).
 void finish_counts(gpa_bitset* bs, size_t M, CountStats* st);
-// Count all pairs of rows (lexicographic pair order) into bs->d_counts (n(n-1)/2 entries).
+// Count all pairs of L_1 rows (bs->l1, or every row; lexicographic pair order) into bs->d_counts
+// (n(n-1)/2 entries, n = l1_size).
 void count_all_pairs(gpa_bitset* bs, uint32_t kernel, CountStats* st);
 }  // namespace gpa

@@ -71,13 +71,14 @@ void record_level(gpa_result* R, const gpa_bitset* bs, uint32_t k, const Grouped
             dst[k - 1] = ior[b->ext[j]];
           }
       });
-    } else {
-      const uint64_t n = bs->n_rows;
+    } else {   // generation 2: every pair of L_1 rows
+      const uint64_t n = l1_size(bs);
+      auto item = [&](uint64_t i) { return ior[bs->l1.empty() ? i : bs->l1[i]]; };
       uint64_t m = 0;
       for (uint64_t a = 0; a + 1 < n; ++a)
         for (uint64_t c = a + 1; c < n; ++c, ++m) {
-          lv.cand_items[2 * m] = ior[a];
-          lv.cand_items[2 * m + 1] = ior[c];
+          lv.cand_items[2 * m] = item(a);
+          lv.cand_items[2 * m + 1] = item(c);
         }
     }
   }
@@ -186,7 +187,7 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
   // the ingest path is chosen collectively: every rank issues the same collective sequence
   const bool overlap = agree_input(db, dist, !(opt.flags & GPA_NO_OVERLAP_INGEST));
   gpa_bitset* bs = overlap ? bitset_build_overlapped(db, min_count, dist, &opt, &pairs_ready, &pair_stats)
-                           : bitset_build(db, min_count, dist, &opt, true);
+                           : bitset_build(db, min_count, dist, &opt, true, true);
   struct BsGuard {
     gpa_bitset* b;
     ~BsGuard() { bitset_free(b); }
@@ -294,7 +295,11 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
   d_ior.alloc(std::max<uint32_t>(bs->n_rows, 1), s);
   if (bs->n_rows)
     GPA_CUDA(cudaMemcpyAsync(d_ior.p, bs->item_of_row.data(), bs->n_rows * 4, cudaMemcpyHostToDevice, s));
-  uint64_t nL = bs->n_rows;
+  uint64_t nL = l1_size(bs);
+  if (!bs->l1.empty() && (bs->d_l1.n < bs->l1.size())) {   // L_1 -> bitset rows (generation 2)
+    bs->d_l1.alloc(bs->l1.size(), s);
+    GPA_CUDA(cudaMemcpyAsync(bs->d_l1.p, bs->l1.data(), bs->l1.size() * 4, cudaMemcpyHostToDevice, s));
+  }
   for (uint32_t k = 2; k <= max_k && nL > 0; ++k) {
     double t0 = now_ms();
     EvTriple& ev = events.emplace_back();
@@ -303,8 +308,8 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     GroupedBatch batch;
     uint64_t M = 0, G = 0;
     if (k == 2) {
-      M = (uint64_t)bs->n_rows * (bs->n_rows - 1) / 2;
-      G = bs->n_rows ? bs->n_rows - 1 : 0;
+      M = nL * (nL - 1) / 2;
+      G = nL ? nL - 1 : 0;
     } else if (host_candgen) {
       // reference path (GPA_HOST_CANDGEN): L_{k-1} back to the host, threaded join + prune
       // (runtime/candgen.cpp), the batch up to the device for the device-side threshold
@@ -409,7 +414,8 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     if (keep && k > 2) fetch_batch();
     double t2 = now_ms();
 
-    const uint32_t F = device_threshold(bs->d_counts.p, (uint32_t)M, (uint32_t)min_count, k, bs->n_rows, Bd.prefix.p,
+    const uint32_t F = device_threshold(bs->d_counts.p, (uint32_t)M, (uint32_t)min_count, k, l1_size(bs),
+                                        k == 2 && !bs->l1.empty() ? bs->d_l1.p : nullptr, Bd.prefix.p,
                                         Bd.ext_off.p, Bd.ext.p, (uint32_t)G, host_candgen ? nullptr : Bd.gpar.p,
                                         host_candgen ? nullptr : Bd.eidx.p, Ln, scratch, bs->n_sms, s);
     // the frequent itemsets of this generation (item ids) and supports stay on the device until the
