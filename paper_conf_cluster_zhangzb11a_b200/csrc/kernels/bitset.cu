@@ -100,7 +100,8 @@ __global__ void __launch_bounds__(kBuildThreads) bitset_build_kernel(const uint6
 // offsets monotone and <= nnz, items < n_items (flags).
 constexpr uint32_t kScanMaxItems = 1024;
 constexpr uint32_t kPiece = 4096;          // items per bulk-copy piece (16 KB)
-constexpr int kScanThreads = 256;
+constexpr int kScanThreads = 512;          // 2 CTAs (112 KB of shared memory each) = 32 warps per SM
+constexpr uint32_t kScanStride = 20;       // tile row stride (words): 16-byte aligned rows for LDS/STS.128
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
   return (uint32_t)__cvta_generic_to_shared(p);
@@ -115,12 +116,14 @@ __global__ void __launch_bounds__(kScanThreads) scan_build_kernel(const uint64_t
                                                                   uint32_t* __restrict__ flags) {
   extern __shared__ __align__(16) uint32_t dyn[];
   uint32_t* buf = dyn;                                   // 2 x (kPiece + 4) items (16-byte aligned pieces)
-  uint32_t* tile = dyn + 2 * (kPiece + 4);               // n_items x kTileStride words
+  uint32_t* tile = dyn + 2 * (kPiece + 4);               // n_items x kScanStride words
   __shared__ uint32_t soff[kChunkTx + 1];
   __shared__ __align__(8) uint64_t bar[2];
   __shared__ uint32_t s_flags;
+  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const uint64_t chunk = chunk0 + blockIdx.x;
-  for (uint32_t i = threadIdx.x; i < n_items * kTileStride; i += blockDim.x) tile[i] = 0;
+  for (uint32_t i = threadIdx.x; i < n_items * (kScanStride / 4); i += blockDim.x)
+    reinterpret_cast<uint4*>(tile)[i] = make_uint4(0, 0, 0, 0);
   if (threadIdx.x == 0) {
     s_flags = 0;
     asm volatile("mbarrier.init.shared.b64 [%0], 1;" ::"r"(smem_u32(&bar[0])));
@@ -145,11 +148,13 @@ __global__ void __launch_bounds__(kScanThreads) scan_build_kernel(const uint64_t
   // items pointer is 16-byte aligned, checked by the launcher), never past the last whole 16-byte
   // group of the array: the last <= 3 items of the array are read from global memory directly
   const uint64_t cend = nnz & ~3ull;
+  const uint32_t n_copy = cend > A ? (cend - A < (uint64_t)n_it ? (uint32_t)(cend - A) : n_it) : 0u;   // items [0, n_copy) in smem
   const uint32_t n_pieces = (n_it + kPiece - 1) / kPiece;
   auto issue = [&](uint32_t p) {
     const uint64_t first = A + (uint64_t)p * kPiece;
     const uint64_t last = A + min(n_it, (p + 1) * kPiece);       // exclusive
-    const uint64_t a0 = first & ~3ull, a1 = ((last + 3) & ~3ull) < cend ? ((last + 3) & ~3ull) : cend;
+    const uint64_t a0 = first & ~3ull, a1r = (last + 3) & ~3ull;
+    const uint64_t a1 = a1r < cend ? a1r : cend;
     if (a1 <= a0) {   // nothing copyable: complete the phase without a copy
       asm volatile("mbarrier.arrive.shared.b64 _, [%0];" ::"r"(smem_u32(&bar[p & 1])) : "memory");
       return;
@@ -164,59 +169,62 @@ __global__ void __launch_bounds__(kScanThreads) scan_build_kernel(const uint64_t
     issue(0);
     if (n_pieces > 1) issue(1);
   }
+  const uint32_t head0 = (uint32_t)(A & 3ull);   // every piece starts at a multiple of kPiece: same head
   for (uint32_t p = 0; p < n_pieces; ++p) {
     const uint32_t b = smem_u32(&bar[p & 1]);
     const uint32_t parity = (p >> 1) & 1;
     asm volatile("{ .reg .pred P; WAIT_%=: mbarrier.try_wait.parity.shared.b64 P, [%0], %1; @!P bra WAIT_%=; }"
                  ::"r"(b), "r"(parity) : "memory");
     const uint32_t q0 = p * kPiece, q1 = min(n_it, q0 + kPiece);
-    const uint32_t head = (uint32_t)((A + q0) & 3ull);
     const uint4* pb = reinterpret_cast<const uint4*>(buf + (p & 1) * (kPiece + 4));   // 16-byte groups
-    // warp step = 32 aligned 16-byte groups of the buffer (128 items, one LDS.128 per lane:
-    // conflict-free); the transaction of the step's first item by a warp-uniform binary search,
-    // each lane's by a short walk from there
-    const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const uint32_t n_groups = (head + (q1 - q0) + 3) / 4;
+    // warp step = 32 aligned 16-byte groups of the buffer (128 items, one conflict-free LDS.128 per
+    // lane); group g holds items q0 - head0 + 4g .. + 3 (chunk-relative, 32-bit); the step's first
+    // transaction by a warp-uniform binary search, each lane's by a short walk from there
+    const uint32_t n_groups = (head0 + (q1 - q0) + 3) / 4;
     for (uint32_t g0 = warp * 32; g0 < n_groups; g0 += (kScanThreads / 32) * 32) {
-      const uint32_t jw = q0 + (g0 * 4 > head ? g0 * 4 - head : 0u);   // first item of the step
+      const uint32_t jw = q0 + (g0 * 4 > head0 ? g0 * 4 - head0 : 0u);   // first item of the step
       uint32_t lo = 0, hi = kChunkTx;   // last tx with soff[tx] <= jw
-      while (lo + 1 < hi) {
+#pragma unroll
+      for (int it = 0; it < 9; ++it) {
         const uint32_t mid = (lo + hi) >> 1;
-        if (soff[mid] <= jw) lo = mid; else hi = mid;
+        const bool le = soff[mid] <= jw;
+        lo = le ? mid : lo;
+        hi = le ? hi : mid;
       }
       const uint32_t g = g0 + lane;
       if (g >= n_groups) continue;
       const uint4 v = pb[g];
       const uint32_t xs[4] = {v.x, v.y, v.z, v.w};
       uint32_t tx = lo;
+      const int32_t jr0 = (int32_t)(q0 + 4 * g) - (int32_t)head0;   // chunk-relative index of xs[0]
 #pragma unroll
-      for (uint32_t i = 0; i < 4; ++i) {
-        const int64_t jj = (int64_t)q0 + (int64_t)(4 * g + i) - (int64_t)head;   // item index in the chunk
-        if (jj < (int64_t)q0 || jj >= (int64_t)q1) continue;
-        const uint32_t j = (uint32_t)jj;
-        while (tx + 1 < kChunkTx && soff[tx + 1] <= j) ++tx;
-        const uint32_t x = A + j < cend ? xs[i] : __ldg(items + A + j);
-        if (x < n_items) atomicOr(&tile[x * kTileStride + (tx >> 5)], 1u << (tx & 31));
+      for (int i = 0; i < 4; ++i) {
+        const int32_t jr = jr0 + i;
+        if (jr < (int32_t)q0 || jr >= (int32_t)q1) continue;
+        const uint32_t j = (uint32_t)jr;
+        while (soff[tx + 1] <= j) ++tx;   // soff[512] = n_it > j stops the walk
+        const uint32_t x = j < n_copy ? xs[i] : __ldg(items + A + j);
+        if (x < n_items) atomicOr(&tile[x * kScanStride + (tx >> 5)], 1u << (tx & 31));
         else my_flags |= kFlagBadItem;
       }
     }
     __syncthreads();   // every thread is done with buffer p & 1
     if (threadIdx.x == 0 && p + 2 < n_pieces) issue(p + 2);
   }
-  // out: row segments (coalesced 64 B per row) and their popcounts into the histogram
+  // out: a quad of lanes per row (4 x 16 bytes = the row's 64-byte segment, STG.128), the row's
+  // popcount into the histogram
   uint32_t* out = rows + chunk * kChunkWords;
-  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;   // (as in the sweep)
-  for (uint32_t r0 = warp * 2; r0 < n_items; r0 += 2 * (kScanThreads / 32)) {   // a warp: 2 rows of 16 words
-    const uint32_t r = r0 + (lane >> 4), w = lane & 15;
-    uint32_t v = 0;
+  const uint32_t quad = lane & 3;
+  for (uint32_t r = threadIdx.x >> 2; r < ((n_items + 7) & ~7u); r += kScanThreads / 4) {
+    uint4 v = make_uint4(0, 0, 0, 0);
     if (r < n_items) {
-      v = tile[r * kTileStride + w];
-      out[(uint64_t)r * pitch_words + w] = v;
+      v = *reinterpret_cast<const uint4*>(tile + r * kScanStride + 4 * quad);
+      *reinterpret_cast<uint4*>(out + (uint64_t)r * pitch_words + 4 * quad) = v;
     }
-    uint32_t c = __popc(v);
-#pragma unroll
-    for (uint32_t d = 8; d >= 1; d >>= 1) c += __shfl_xor_sync(0xffffffffu, c, d);
-    if ((lane & 15) == 0 && r < n_items && c) atomicAdd(&hist[r], c);
+    uint32_t c = __popc(v.x) + __popc(v.y) + __popc(v.z) + __popc(v.w);
+    c += __shfl_xor_sync(0xffffffffu, c, 1);
+    c += __shfl_xor_sync(0xffffffffu, c, 2);
+    if (quad == 0 && r < n_items && c) atomicAdd(&hist[r], c);
   }
   if (my_flags) atomicOr(&s_flags, my_flags);
   __syncthreads();
@@ -245,7 +253,7 @@ void launch_scan_build(const uint64_t* offsets, const uint32_t* items, uint64_t 
               n_items);
   const uint64_t n_chunks = pitch_words / kChunkWords;   // the padding chunks write zeros
   GPA_REQUIRE(n_chunks < (1ull << 31), GPA_ERR_INVALID, "scan_build: too many transactions");
-  const size_t smem = (2 * (kPiece + 4) + (size_t)n_items * kTileStride) * sizeof(uint32_t);
+  const size_t smem = (2 * (kPiece + 4) + (size_t)n_items * kScanStride) * sizeof(uint32_t);
   ensure_smem_attr(reinterpret_cast<const void*>(scan_build_kernel), (int)smem);
   { scan_build_kernel<<<(unsigned)n_chunks, kScanThreads, smem, stream>>>(offsets, items, n_tx, nnz, n_items, 0,
                                                                          pitch_words, rows, hist, flags);

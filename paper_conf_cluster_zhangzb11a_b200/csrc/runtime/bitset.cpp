@@ -186,7 +186,7 @@ gpa_bitset* bitset_build(const gpa_tx_csr* db, uint64_t row_min_count, const gpa
       bs->row_of_item[i] = (int32_t)i;
     }
     bs->n_rows = n_items;
-    if (bs->l1.size() == n_items) bs->l1.clear();   // every row is in L_1
+    bs->l1_sub = bs->l1.size() < n_items;   // else every row is in L_1
   } else if (scan) {
     // row r <- row item_of_row[r] from the first row whose item differs (in place)
     uint32_t r0 = 0;
@@ -476,7 +476,7 @@ void count_all_pairs(gpa_bitset* bs, uint32_t kernel, CountStats* st) {
   const uint64_t n = l1_size(bs);
   const uint64_t M = n * (n - 1) / 2;
   if (n < 2) return;
-  const bool sub = !bs->l1.empty();   // L_1 is a subset of the rows
+  const bool sub = bs->l1_sub;   // L_1 is a subset of the rows
   if (kernel == GPA_KERNEL_AUTO || kernel == GPA_KERNEL_PROJ) kernel = GPA_KERNEL_PAIRS_TC;
   if (kernel != GPA_KERNEL_PAIRS && kernel != GPA_KERNEL_PAIRS_TC) {
     GroupedBatch b;

@@ -284,7 +284,8 @@ gpa_bitset* bitset_build_overlapped(const gpa_tx_csr* db, uint64_t row_min_count
       bs->item_of_row = r0_items;
       bs->row_of_item = r0_of_item;
       bs->n_rows = nr0;
-      if (n1 < nr0) bs->l1 = sel;
+      bs->l1 = sel;
+      bs->l1_sub = n1 < nr0;
       DBuf<uint32_t> d_sel;
       d_sel.alloc(n1, s);
       GPA_CUDA(cudaMemcpyAsync(d_sel.p, sel.data(), n1 * 4, cudaMemcpyHostToDevice, s));

@@ -141,6 +141,7 @@ struct gpa_bitset {
   // one-pass build, the chunk-0 estimate R0 after the overlapped ingest): ascending row ids; empty =
   // every row is in L_1.  Generation 2 counts pairs of these rows; L_k holds bitset row ids.
   std::vector<uint32_t> l1;
+  bool l1_sub = false;                 // l1 is in use (possibly empty: nothing frequent)
   gpa::DBuf<uint32_t> d_l1, d_pairs_all;
   alignas(64) unsigned char tmap[128];
   bool tmap_ready = false;
@@ -164,7 +165,7 @@ namespace gpa {
 gpa_bitset* bitset_build(const gpa_tx_csr* db, uint64_t row_min_count, const gpa_dist* dist, const gpa_options* opt,
                          bool prechecked = false, bool keep_all_rows = false);
 // number of L_1 rows (bs->l1, or every row)
-inline uint32_t l1_size(const gpa_bitset* bs) { return bs->l1.empty() ? bs->n_rows : (uint32_t)bs->l1.size(); }
+inline uint32_t l1_size(const gpa_bitset* bs) { return bs->l1_sub ? (uint32_t)bs->l1.size() : bs->n_rows; }
 void bitset_free(gpa_bitset* bs);
 // Host input, end to end: upload in transaction chunks overlapped with histogram, bitset build and
 // generation-2 pair counting (runtime/ingest.cpp).  *pairs_ready: bs->d_counts holds the L_1 pair

@@ -73,7 +73,7 @@ void record_level(gpa_result* R, const gpa_bitset* bs, uint32_t k, const Grouped
       });
     } else {   // generation 2: every pair of L_1 rows
       const uint64_t n = l1_size(bs);
-      auto item = [&](uint64_t i) { return ior[bs->l1.empty() ? i : bs->l1[i]]; };
+      auto item = [&](uint64_t i) { return ior[bs->l1_sub ? bs->l1[i] : i]; };
       uint64_t m = 0;
       for (uint64_t a = 0; a + 1 < n; ++a)
         for (uint64_t c = a + 1; c < n; ++c, ++m) {
@@ -296,7 +296,7 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
   if (bs->n_rows)
     GPA_CUDA(cudaMemcpyAsync(d_ior.p, bs->item_of_row.data(), bs->n_rows * 4, cudaMemcpyHostToDevice, s));
   uint64_t nL = l1_size(bs);
-  if (!bs->l1.empty() && (bs->d_l1.n < bs->l1.size())) {   // L_1 -> bitset rows (generation 2)
+  if (bs->l1_sub && !bs->l1.empty() && bs->d_l1.n < bs->l1.size()) {   // L_1 -> bitset rows (generation 2)
     bs->d_l1.alloc(bs->l1.size(), s);
     GPA_CUDA(cudaMemcpyAsync(bs->d_l1.p, bs->l1.data(), bs->l1.size() * 4, cudaMemcpyHostToDevice, s));
   }
@@ -415,7 +415,7 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     double t2 = now_ms();
 
     const uint32_t F = device_threshold(bs->d_counts.p, (uint32_t)M, (uint32_t)min_count, k, l1_size(bs),
-                                        k == 2 && !bs->l1.empty() ? bs->d_l1.p : nullptr, Bd.prefix.p,
+                                        k == 2 && bs->l1_sub ? bs->d_l1.p : nullptr, Bd.prefix.p,
                                         Bd.ext_off.p, Bd.ext.p, (uint32_t)G, host_candgen ? nullptr : Bd.gpar.p,
                                         host_candgen ? nullptr : Bd.eidx.p, Ln, scratch, bs->n_sms, s);
     // the frequent itemsets of this generation (item ids) and supports stay on the device until the
