@@ -17,7 +17,7 @@ CU_SRCS   := $(wildcard $(CSRC)/kernels/*.cu)
 CPP_SRCS  := $(wildcard $(CSRC)/runtime/*.cpp)
 CU_OBJS   := $(patsubst $(CSRC)/kernels/%.cu,$(BUILD)/k_%.o,$(CU_SRCS))
 CPP_OBJS  := $(patsubst $(CSRC)/runtime/%.cpp,$(BUILD)/r_%.o,$(CPP_SRCS))
-HDRS      := include/gpapriori.h $(CSRC)/common.h $(CSRC)/kernels.h $(CSRC)/runtime/internal.h $(CSRC)/runtime/pool.h
+HDRS      := $(wildcard $(CSRC)/kernels/*.cuh) include/gpapriori.h $(CSRC)/common.h $(CSRC)/kernels.h $(CSRC)/runtime/internal.h $(CSRC)/runtime/pool.h
 
 all: $(LIB) oracle/liboracle.so gen/libgen.so examples/gpa_mine_fimi
 

@@ -107,6 +107,7 @@ void launch_gather_rows(const uint32_t* rows_all, const uint32_t* sel, uint32_t 
 struct DeviceScratch {
   DBuf<uint32_t> a, b, c, d, e, f, g, h, i;
   DBuf<uint8_t> tmp;
+  uint32_t hash_cap = 0;   // slots of the join's hash set (i), set by device_candgen_begin
   uint32_t* u32a(size_t n, cudaStream_t s) { a.ensure(n ? n : 1, s); return a.p; }
   uint32_t* u32b(size_t n, cudaStream_t s) { b.ensure(n ? n : 1, s); return b.p; }
   uint32_t* u32c(size_t n, cudaStream_t s) { c.ensure(n ? n : 1, s); return c.p; }
@@ -122,9 +123,14 @@ struct DeviceScratch {
 // par_a[p] / par_b[p]: index in L_{k-1} of the entry's left parent (its first k-1 items) and
 // right parent (first k-2 items + last item); for k = 2 the two row ids.  Used by the projected
 // lists of proj.cu.
+// Device-sized level (n_dev != nullptr): |L| is only on the device (*n_dev, = count.p) until the
+// next synchronisation, the arrays hold n_max (>= |L|) entries; the level-transition kernels read
+// the count from the device and run over the upper bound.
 struct DeviceLevel {
   uint32_t k = 0, n = 0;
-  DBuf<uint32_t> rows, sup, par_a, par_b;
+  DBuf<uint32_t> rows, sup, par_a, par_b, count;
+  const uint32_t* n_dev = nullptr;
+  uint32_t n_max = 0;
 };
 // C_k on the device, grouped by (k-1)-prefix: prefix[G][k-1], ext_off[G+1], ext[M]
 // gpar[g] = index in L_{k-1} of group g's prefix (the left parent), eidx[m] = index in L_{k-1} of
@@ -141,6 +147,11 @@ uint32_t device_threshold(const uint32_t* counts, uint32_t M, uint32_t theta, ui
                           const uint32_t* sel, const uint32_t* prefix, const uint32_t* ext_off, const uint32_t* ext,
                           uint32_t G, const uint32_t* gpar, const uint32_t* eidx,
                           DeviceLevel& out, DeviceScratch& scratch, int n_sms, cudaStream_t s);
+// The same without a synchronisation: out becomes device-sized (n_dev = &|L_k|, n_max = M).
+void device_threshold_async(const uint32_t* counts, uint32_t M, uint32_t theta, uint32_t k, uint32_t n_rows,
+                            const uint32_t* sel, const uint32_t* prefix, const uint32_t* ext_off, const uint32_t* ext,
+                            uint32_t G, const uint32_t* gpar, const uint32_t* eidx,
+                            DeviceLevel& out, DeviceScratch& scratch, int n_sms, cudaStream_t s);
 
 // ---- association rules (rules.cu): F as n itemsets in canonical order (items at
 // items + item_off[i], len[i] items, support sup[i]); the rules A => X \ A of the itemsets x0 .. n-1
@@ -188,17 +199,20 @@ struct ProjPending {
 };
 // begin returns false (nothing enqueued) when the lists cannot be addressed (bitset >= 2^32 words,
 // too many classes): use complete intersection.
+// n_dev: L is device-sized (n = its host upper bound, the count at *n_dev); set pp.n to the count
+// before proj_build_finish.
 bool proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const DeviceProj* prev,
                       const uint32_t* rows, uint64_t pitch_words, uint32_t n_rows, DeviceScratch& scratch, int n_sms,
-                      cudaStream_t s, ProjPending& pp);
+                      cudaStream_t s, ProjPending& pp, const uint32_t* n_dev = nullptr);
 bool proj_build_finish(const ProjPending& pp, const uint64_t T[2], const uint32_t sm[4], DeviceProj& out, int n_sms,
                        cudaStream_t s, cudaEvent_t ev_build);
 // counts[m] += popc(V_gpar[g] & V_eidx[m]) for every candidate m of group g (counts zeroed by the caller)
 void launch_count_proj(const DeviceProj& P, const uint32_t* gpar, const uint32_t* ext_off, const uint32_t* eidx,
                        uint32_t G, uint32_t* counts, cudaStream_t s);
-// items[i] = item_of_row[rows[i]] (row ids -> original item ids)
+// items[i] = item_of_row[rows[i]] (row ids -> original item ids) for i < n, or for i < *n_dev * k
+// when n_dev is given (n then an upper bound)
 void device_map_items(const uint32_t* rows, uint64_t n, const uint32_t* item_of_row, uint32_t* items, int n_sms,
-                      cudaStream_t s);
+                      cudaStream_t s, const uint32_t* n_dev = nullptr, uint32_t k = 1);
 // exclusive scan of n u32 (CUB); the total is written to *tot (device) when tot != nullptr
 void device_exclusive_scan(const uint32_t* in, uint32_t* out, uint32_t n, uint32_t* tot, DeviceScratch& scratch,
                            cudaStream_t s);

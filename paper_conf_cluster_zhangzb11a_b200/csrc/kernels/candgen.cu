@@ -13,57 +13,23 @@
 
 #include "../common.h"
 #include "../kernels.h"
+#include "level_dev.cuh"
 
 namespace gpa {
 namespace {
+using namespace lvl;
 
 constexpr int kThreads = 256;
 
-__device__ __forceinline__ int lex_cmp(const uint32_t* a, const uint32_t* b, uint32_t w) {
-  for (uint32_t i = 0; i < w; ++i)
-    if (a[i] != b[i]) return a[i] < b[i] ? -1 : 1;
-  return 0;
-}
-
-// Open-addressing hash set over the rows of L (slot = row index, 0xffffffff = empty), keyed by
-// the polynomial hash H = sum_i (x_i + 1) P^i (mod 2^64) finalised by a mixer.  H is linear in the
-// items, so the hash of "x without item d, plus b" is O(1) from per-x prefix / suffix sums.
-constexpr uint64_t kHashP = 0x9E3779B97F4A7C15ull | 1ull;
-constexpr uint32_t kEmpty = 0xffffffffu;
-
-__device__ __forceinline__ uint64_t hash_mix(uint64_t h) {
-  h ^= h >> 33;
-  h *= 0xFF51AFD7ED558CCDull;
-  h ^= h >> 33;
-  return h;
-}
-
-__device__ __forceinline__ uint64_t raw_hash(const uint32_t* key, uint32_t w) {
-  uint64_t h = 0, p = 1;
-  for (uint32_t i = 0; i < w; ++i) {
-    h += (uint64_t)(key[i] + 1) * p;
-    p *= kHashP;
-  }
-  return h;
-}
+// n_dev (device-sized levels): the member count lives on the device; n is its host upper bound
+__device__ __forceinline__ uint32_t eff_n(uint32_t n, const uint32_t* n_dev) { return n_dev ? min(*n_dev, n) : n; }
 
 __global__ void hash_build_kernel(const uint32_t* __restrict__ L, uint32_t n, uint32_t w, uint32_t* slots,
-                                  uint32_t mask) {
+                                  uint32_t mask, const uint32_t* __restrict__ n_dev) {
+  n = eff_n(n, n_dev);
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
     uint32_t h = (uint32_t)hash_mix(raw_hash(L + (uint64_t)i * w, w)) & mask;
     while (atomicCAS(&slots[h], kEmpty, i) != kEmpty) h = (h + 1) & mask;
-  }
-}
-
-// membership of key (w items, raw polynomial hash `raw`) in L
-__device__ __forceinline__ bool contains(const uint32_t* __restrict__ L, uint32_t w, const uint32_t* __restrict__ slots,
-                                         uint32_t mask, const uint32_t* key, uint64_t raw) {
-  uint32_t h = (uint32_t)hash_mix(raw) & mask;
-  for (;;) {
-    const uint32_t i = slots[h];
-    if (i == kEmpty) return false;
-    if (lex_cmp(L + (uint64_t)i * w, key, w) == 0) return true;
-    h = (h + 1) & mask;
   }
 }
 
@@ -125,9 +91,12 @@ __global__ void scatter_grouped_kernel(const uint32_t* __restrict__ counts, cons
 }
 
 // run starts: members whose first w-1 items differ from the previous member's
-__global__ void run_start_kernel(const uint32_t* __restrict__ L, uint32_t n, uint32_t w, uint32_t* flags) {
+// (zero past the device count: the scans run over the host upper bound)
+__global__ void run_start_kernel(const uint32_t* __restrict__ L, uint32_t n, uint32_t w, uint32_t* flags,
+                                 const uint32_t* __restrict__ n_dev) {
+  const uint32_t ne = eff_n(n, n_dev);
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x)
-    flags[i] = i == 0 || lex_cmp(L + (uint64_t)(i - 1) * w, L + (uint64_t)i * w, w - 1) != 0;
+    flags[i] = i < ne && (i == 0 || lex_cmp(L + (uint64_t)(i - 1) * w, L + (uint64_t)i * w, w - 1) != 0);
 }
 
 __global__ void run_bound_kernel(const uint32_t* __restrict__ flags, const uint32_t* __restrict__ run_ex,
@@ -136,83 +105,22 @@ __global__ void run_bound_kernel(const uint32_t* __restrict__ flags, const uint3
     if (flags[i]) bound[run_ex[i]] = i;
 }
 
-// join + prune of member x with its later run siblings; EMIT = false counts survivors, EMIT = true
-// writes group x (prefix = L[x]) and its extensions at the scanned offsets
-// Join + prune of member x with its later run siblings, one WARP per x: lane j tests sibling
-// y = x + 1 + j (+32 ...); EMIT = false counts survivors, EMIT = true writes group x (prefix = L[x])
-// and its extensions, in sibling order, at the scanned offsets (warp ballot ranks the survivors).
+// join + prune, one WARP per member x (lvl::join_warp)
 template <bool EMIT>
 __global__ void join_kernel(const uint32_t* __restrict__ L, uint32_t n, uint32_t w, const uint32_t* __restrict__ flags,
                             const uint32_t* __restrict__ run_ex, const uint32_t* __restrict__ bound,
                             const uint32_t* __restrict__ slots, uint32_t mask, uint32_t* cnt,
                             const uint32_t* __restrict__ cand_off, const uint32_t* __restrict__ gidx,
-                            uint32_t* prefix, uint32_t* ext_off, uint32_t* ext, uint32_t* gpar, uint32_t* eidx) {
-  uint32_t probe[GPA_MAX_K];
-  uint64_t A[GPA_MAX_K], B[GPA_MAX_K];
-  const uint32_t lane = threadIdx.x & 31;
+                            uint32_t* prefix, uint32_t* ext_off, uint32_t* ext, uint32_t* gpar, uint32_t* eidx,
+                            const uint32_t* __restrict__ n_dev) {
   const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, n_warps = (gridDim.x * blockDim.x) >> 5;
+  const uint32_t ne = eff_n(n, n_dev);
   for (uint32_t x = warp; x < n; x += n_warps) {
-    if (EMIT && cnt[x] == 0) continue;  // warp-uniform
-    // run index of x = (#run starts <= x) - 1
-    const uint32_t r = run_ex[x] + flags[x] - 1;
-    const uint32_t end = bound[r + 1];  // bound[n_runs] = n (sentinel)
-    if (!EMIT && end == x + 1) {
-      if (lane == 0) cnt[x] = 0;
-      continue;
-    }
-    const uint32_t* px = L + (uint64_t)x * w;
-    // subset "px without item d, then b": A[d] = sum_{i<d} (x_i+1) P^i,
-    // B[d] = sum_{i>d} (x_i+1) P^(i-1); b lands at position w-1
-    uint64_t pw = 1, acc = 0;
-    for (uint32_t i = 0; i < w; ++i) {  // B[i] temporarily holds P^i
-      A[i] = acc;
-      B[i] = pw;
-      acc += (uint64_t)(px[i] + 1) * pw;
-      pw *= kHashP;
-    }
-    const uint64_t p_last = B[w - 1];  // P^(w-1)
-    uint64_t suf = 0;
-    for (uint32_t d = w; d-- > 0;) {
-      const uint64_t pprev = d > 0 ? B[d - 1] : 0;
-      B[d] = suf;
-      suf += (uint64_t)(px[d] + 1) * pprev;  // term of item d at position d-1
-    }
-    uint32_t here = 0;  // survivors so far (warp-uniform)
-    for (uint32_t y0 = x + 1; y0 < end; y0 += 32) {
-      const uint32_t y = y0 + lane;
-      bool keep = y < end;
-      uint32_t b = 0;
-      if (keep) {
-        b = L[(uint64_t)y * w + w - 1];
-        const uint64_t hb = (uint64_t)(b + 1) * p_last;
-        // subsets dropping item d of the shared prefix (dropping either of the last two items
-        // gives the parents x or y, members of L by construction)
-        for (uint32_t d = 0; d + 1 < w && keep; ++d) {
-          uint32_t q = 0;
-          for (uint32_t i = 0; i < w; ++i)
-            if (i != d) probe[q++] = px[i];
-          probe[q] = b;
-          keep = contains(L, w, slots, mask, probe, A[d] + B[d] + hb);
-        }
-      }
-      const uint32_t ballot = __ballot_sync(0xffffffffu, keep);
-      if (EMIT && keep) {
-        const uint32_t at = cand_off[x] + here + __popc(ballot & ((1u << lane) - 1u));
-        ext[at] = b;
-        eidx[at] = y;
-      }
-      here += __popc(ballot);
-    }
-    if (EMIT) {
-      const uint32_t g = gidx[x];
-      for (uint32_t i = lane; i < w; i += 32) prefix[(uint64_t)g * w + i] = px[i];
-      if (lane == 0) {
-        ext_off[g] = cand_off[x];
-        gpar[g] = x;
-      }
-    } else if (lane == 0) {
-      cnt[x] = here;
-    }
+    if (x < ne)
+      lvl::join_warp<EMIT>(x, L, w, flags, run_ex, bound, slots, mask, cnt, cand_off, gidx, prefix, ext_off, ext,
+                           gpar, eidx);
+    else if (!EMIT && (threadIdx.x & 31) == 0)
+      cnt[x] = 0;   // past the device count: no survivors (the scans run over the upper bound)
   }
 }
 
@@ -223,8 +131,9 @@ __global__ void total_kernel(const uint32_t* __restrict__ in, const uint32_t* __
 }
 // bound[n_runs] = n (sentinel end of the last run)
 __global__ void bound_sentinel_kernel(const uint32_t* __restrict__ flags, const uint32_t* __restrict__ run_ex,
-                                      uint32_t n, uint32_t* bound) {
-  if (threadIdx.x == 0 && blockIdx.x == 0) bound[run_ex[n - 1] + flags[n - 1]] = n;
+                                      uint32_t n, uint32_t* bound, const uint32_t* __restrict__ n_dev) {
+  n = eff_n(n, n_dev);
+  if (threadIdx.x == 0 && blockIdx.x == 0) bound[n ? run_ex[n - 1] + flags[n - 1] : 0] = n;
 }
 // ext_off[G] = M
 __global__ void ext_end_kernel(const uint32_t* __restrict__ sizes, uint32_t* ext_off) {
@@ -237,7 +146,8 @@ __global__ void nonzero_kernel(const uint32_t* __restrict__ cnt, uint32_t n, uin
 }
 
 __global__ void map_items_kernel(const uint32_t* __restrict__ rows, uint64_t n, const uint32_t* __restrict__ ior,
-                                 uint32_t* items) {
+                                 uint32_t* items, const uint32_t* __restrict__ n_dev, uint32_t k) {
+  if (n_dev && (uint64_t)*n_dev * k < n) n = (uint64_t)*n_dev * k;
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
     items[i] = ior[rows[i]];
 }
@@ -261,38 +171,68 @@ void exclusive_scan(const uint32_t* in, uint32_t* out, uint32_t n, uint32_t* tot
 
 }  // namespace
 
+namespace {
+void threshold_impl(const uint32_t* counts, uint32_t M, uint32_t theta, uint32_t k, uint32_t n_rows, const uint32_t* sel,
+                    const uint32_t* prefix, const uint32_t* ext_off, const uint32_t* ext, uint32_t G,
+                    const uint32_t* gpar, const uint32_t* eidx, DeviceLevel& out, DeviceScratch& scratch, int n_sms,
+                    cudaStream_t s, uint32_t cap) {
+  uint32_t* flags = scratch.u32a(M, s);
+  uint32_t* pos = scratch.u32b(M, s);
+  { flag_ge_kernel<<<grid_for(M, n_sms), kThreads, 0, s>>>(counts, M, theta, flags); note_launch(); }
+  GPA_CUDA(cudaGetLastError());
+  out.count.ensure(1, s);
+  exclusive_scan(flags, pos, M, out.count.p, scratch, s);
+  out.rows.ensure((size_t)std::max<uint32_t>(cap, 1) * k, s);
+  out.sup.ensure(std::max<uint32_t>(cap, 1), s);
+  out.par_a.ensure(std::max<uint32_t>(cap, 1), s);
+  out.par_b.ensure(std::max<uint32_t>(cap, 1), s);
+  if (k == 2)
+    { scatter_pairs_kernel<<<grid_for(M, n_sms), kThreads, 0, s>>>(counts, flags, pos, M, n_rows, sel, out.rows.p,
+                                                                out.sup.p, out.par_a.p, out.par_b.p); note_launch(); }
+  else
+    { scatter_grouped_kernel<<<grid_for(M, n_sms), kThreads, 0, s>>>(counts, flags, pos, M, prefix, ext_off, ext, G,
+                                                                  k - 1, gpar, eidx, out.rows.p, out.sup.p,
+                                                                  out.par_a.p, out.par_b.p); note_launch(); }
+  GPA_CUDA(cudaGetLastError());
+}
+}  // namespace
+
 uint32_t device_threshold(const uint32_t* counts, uint32_t M, uint32_t theta, uint32_t k, uint32_t n_rows,
                           const uint32_t* sel, const uint32_t* prefix, const uint32_t* ext_off, const uint32_t* ext,
                           uint32_t G, const uint32_t* gpar, const uint32_t* eidx,
                           DeviceLevel& out, DeviceScratch& scratch, int n_sms, cudaStream_t s) {
   out.k = k;
   out.n = 0;
+  out.n_dev = nullptr;
+  out.n_max = 0;
   if (M == 0) return 0;
+  // |L_k| first (one synchronisation), then L_k at its exact size
   uint32_t* flags = scratch.u32a(M, s);
   uint32_t* pos = scratch.u32b(M, s);
   { flag_ge_kernel<<<grid_for(M, n_sms), kThreads, 0, s>>>(counts, M, theta, flags); note_launch(); }
-  GPA_CUDA(cudaGetLastError());
-  uint32_t* sizes = scratch.u32c(4, s);
-  exclusive_scan(flags, pos, M, sizes, scratch, s);
+  out.count.ensure(1, s);
+  exclusive_scan(flags, pos, M, out.count.p, scratch, s);
   uint32_t F = 0;
-  GPA_CUDA(cudaMemcpyAsync(&F, sizes, 4, cudaMemcpyDeviceToHost, s));
+  GPA_CUDA(cudaMemcpyAsync(&F, out.count.p, 4, cudaMemcpyDeviceToHost, s));
   stream_wait(s);
-  out.rows.ensure((size_t)std::max<uint32_t>(F, 1) * k, s);
-  out.sup.ensure(std::max<uint32_t>(F, 1), s);
-  out.par_a.ensure(std::max<uint32_t>(F, 1), s);
-  out.par_b.ensure(std::max<uint32_t>(F, 1), s);
-  if (F) {
-    if (k == 2)
-      { scatter_pairs_kernel<<<grid_for(M, n_sms), kThreads, 0, s>>>(counts, flags, pos, M, n_rows, sel, out.rows.p,
-                                                                  out.sup.p, out.par_a.p, out.par_b.p); note_launch(); }
-    else
-      { scatter_grouped_kernel<<<grid_for(M, n_sms), kThreads, 0, s>>>(counts, flags, pos, M, prefix, ext_off, ext, G,
-                                                                    k - 1, gpar, eidx, out.rows.p, out.sup.p,
-                                                                    out.par_a.p, out.par_b.p); note_launch(); }
-    GPA_CUDA(cudaGetLastError());
-  }
+  if (F) threshold_impl(counts, M, theta, k, n_rows, sel, prefix, ext_off, ext, G, gpar, eidx, out, scratch, n_sms, s,
+                        F);
   out.n = F;
   return F;
+}
+
+void device_threshold_async(const uint32_t* counts, uint32_t M, uint32_t theta, uint32_t k, uint32_t n_rows,
+                            const uint32_t* sel, const uint32_t* prefix, const uint32_t* ext_off, const uint32_t* ext,
+                            uint32_t G, const uint32_t* gpar, const uint32_t* eidx,
+                            DeviceLevel& out, DeviceScratch& scratch, int n_sms, cudaStream_t s) {
+  out.k = k;
+  out.n = 0;
+  out.n_dev = nullptr;
+  out.n_max = 0;
+  if (M == 0) return;
+  threshold_impl(counts, M, theta, k, n_rows, sel, prefix, ext_off, ext, G, gpar, eidx, out, scratch, n_sms, s, M);
+  out.n_dev = out.count.p;   // |L_k| stays on the device until the next generation's synchronisation
+  out.n_max = M;
 }
 
 void device_exclusive_scan(const uint32_t* in, uint32_t* out, uint32_t n, uint32_t* tot, DeviceScratch& scratch,
@@ -301,9 +241,9 @@ void device_exclusive_scan(const uint32_t* in, uint32_t* out, uint32_t n, uint32
 }
 
 void device_map_items(const uint32_t* rows, uint64_t n, const uint32_t* item_of_row, uint32_t* items, int n_sms,
-                      cudaStream_t s) {
+                      cudaStream_t s, const uint32_t* n_dev, uint32_t k) {
   if (n == 0) return;
-  { map_items_kernel<<<grid_for(n, n_sms), kThreads, 0, s>>>(rows, n, item_of_row, items); note_launch(); }
+  { map_items_kernel<<<grid_for(n, n_sms), kThreads, 0, s>>>(rows, n, item_of_row, items, n_dev, k); note_launch(); }
   GPA_CUDA(cudaGetLastError());
 }
 
@@ -311,7 +251,8 @@ void device_map_items(const uint32_t* rows, uint64_t n, const uint32_t* item_of_
 // the device (sizes[0], sizes[1]) -- no synchronisation.  Returns false when L has < 2 members.
 bool device_candgen_begin(const DeviceLevel& L, DeviceBatch& out, DeviceScratch& scratch, int n_sms, cudaStream_t s,
                           const uint32_t** d_sizes) {
-  const uint32_t n = L.n, w = L.k;
+  const uint32_t* n_dev = L.n_dev;
+  const uint32_t n = n_dev ? L.n_max : L.n, w = L.k;   // device-sized level: n = the host upper bound
   out.k = w + 1;
   out.M = out.G = 0;
   if (n < 2) return false;
@@ -320,19 +261,20 @@ bool device_candgen_begin(const DeviceLevel& L, DeviceBatch& out, DeviceScratch&
   uint32_t* cnt = scratch.u32c(n, s);
   uint32_t* bound = scratch.u32d(n + 1, s);
   uint32_t* sizes = scratch.u32h(4, s);  // [0] = M, [1] = G
-  { run_start_kernel<<<grid_for(n, n_sms), kThreads, 0, s>>>(L.rows.p, n, w, flags); note_launch(); }
+  { run_start_kernel<<<grid_for(n, n_sms), kThreads, 0, s>>>(L.rows.p, n, w, flags, n_dev); note_launch(); }
   GPA_CUDA(cudaGetLastError());
   exclusive_scan(flags, run_ex, n, nullptr, scratch, s);
   { run_bound_kernel<<<grid_for(n, n_sms), kThreads, 0, s>>>(flags, run_ex, n, bound); note_launch(); }
-  { bound_sentinel_kernel<<<1, 32, 0, s>>>(flags, run_ex, n, bound); note_launch(); }
+  { bound_sentinel_kernel<<<1, 32, 0, s>>>(flags, run_ex, n, bound, n_dev); note_launch(); }
   // hash set over L for the prune probes
   uint32_t cap = 16;
   while (cap < 2 * n + 1) cap <<= 1;
   uint32_t* slots = scratch.u32i(cap, s);
+  scratch.hash_cap = cap;   // the emitting join (stage 2) probes the same table
   GPA_CUDA(cudaMemsetAsync(slots, 0xff, (size_t)cap * 4, s));
-  { hash_build_kernel<<<grid_for(n, n_sms), kThreads, 0, s>>>(L.rows.p, n, w, slots, cap - 1); note_launch(); }
-  { join_kernel<false><<<grid_for(32ull * n, n_sms), kThreads, 0, s>>>(L.rows.p, n, w, flags, run_ex, bound, slots, cap - 1, cnt,
-                                                             nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr); note_launch(); }
+  { hash_build_kernel<<<grid_for(n, n_sms), kThreads, 0, s>>>(L.rows.p, n, w, slots, cap - 1, n_dev); note_launch(); }
+  { join_kernel<false><<<grid_for(32ull * n, n_sms), kThreads, 0, s>>>(L.rows.p, n, w, flags, run_ex, bound, slots,
+        cap - 1, cnt, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, n_dev); note_launch(); }
   GPA_CUDA(cudaGetLastError());
   uint32_t* cand_off = scratch.u32e(n, s);
   uint32_t* gflag = scratch.u32f(n, s);
@@ -360,11 +302,10 @@ void device_candgen_finish(const DeviceLevel& L, DeviceBatch& out, DeviceScratch
     GPA_CUDA(cudaEventRecord(ev, s));
     GPA_CUDA(cudaStreamWaitEvent(run, ev, 0));
   }
-  uint32_t cap = 16;
-  while (cap < 2 * n + 1) cap <<= 1;
+  const uint32_t cap = scratch.hash_cap;   // the table stage 1 built (sized for its upper bound)
   { join_kernel<true><<<grid_for(32ull * n, n_sms), kThreads, 0, run>>>(L.rows.p, n, w, scratch.a.p, scratch.b.p,
         scratch.d.p, scratch.i.p, cap - 1, scratch.c.p, scratch.e.p, scratch.g.p, out.prefix.p, out.ext_off.p,
-        out.ext.p, out.gpar.p, out.eidx.p); note_launch(); }
+        out.ext.p, out.gpar.p, out.eidx.p, nullptr); note_launch(); }
   GPA_CUDA(cudaGetLastError());
   { ext_end_kernel<<<1, 32, 0, run>>>(scratch.h.p, out.ext_off.p); note_launch(); }
   out.M = M;

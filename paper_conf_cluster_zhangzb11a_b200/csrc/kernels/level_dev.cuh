@@ -1,0 +1,129 @@
+// Device helpers of the level transition shared by candgen.cu (separate kernels) and
+// transition.cu (the fused cooperative kernel).  Internal; included by .cu files only.
+#pragma once
+#include <cstdint>
+#include "../common.h"
+
+namespace gpa {
+namespace lvl {
+
+__device__ __forceinline__ int lex_cmp(const uint32_t* a, const uint32_t* b, uint32_t w) {
+  for (uint32_t i = 0; i < w; ++i)
+    if (a[i] != b[i]) return a[i] < b[i] ? -1 : 1;
+  return 0;
+}
+
+// Open-addressing hash set over the rows of L (slot = row index, 0xffffffff = empty), keyed by
+// the polynomial hash H = sum_i (x_i + 1) P^i (mod 2^64) finalised by a mixer.  H is linear in the
+// items, so the hash of "x without item d, plus b" is O(1) from per-x prefix / suffix sums.
+constexpr uint64_t kHashP = 0x9E3779B97F4A7C15ull | 1ull;
+constexpr uint32_t kEmpty = 0xffffffffu;
+
+__device__ __forceinline__ uint64_t hash_mix(uint64_t h) {
+  h ^= h >> 33;
+  h *= 0xFF51AFD7ED558CCDull;
+  h ^= h >> 33;
+  return h;
+}
+
+__device__ __forceinline__ uint64_t raw_hash(const uint32_t* key, uint32_t w) {
+  uint64_t h = 0, p = 1;
+  for (uint32_t i = 0; i < w; ++i) {
+    h += (uint64_t)(key[i] + 1) * p;
+    p *= kHashP;
+  }
+  return h;
+}
+
+// membership of key (w items, raw polynomial hash `raw`) in L
+__device__ __forceinline__ bool contains(const uint32_t* __restrict__ L, uint32_t w, const uint32_t* __restrict__ slots,
+                                         uint32_t mask, const uint32_t* key, uint64_t raw) {
+  uint32_t h = (uint32_t)hash_mix(raw) & mask;
+  for (;;) {
+    const uint32_t i = slots[h];
+    if (i == kEmpty) return false;
+    if (lex_cmp(L + (uint64_t)i * w, key, w) == 0) return true;
+    h = (h + 1) & mask;
+  }
+}
+
+// Join + prune of member x of L (n members of w items, lexicographic) with its later run
+// siblings, by ONE WARP: lane j tests sibling y = x + 1 + j (+32 ...).  EMIT = false: cnt[x] =
+// survivors; EMIT = true: group gidx[x] (prefix = L[x]) and its extensions, in sibling order, at
+// cand_off[x] (warp ballot ranks the survivors).  flags / run_ex / bound: run starts, their
+// exclusive scan, run boundaries (bound[#runs] = n).
+template <bool EMIT>
+__device__ __forceinline__ void join_warp(uint32_t x, const uint32_t* __restrict__ L, uint32_t w,
+                                          const uint32_t* __restrict__ flags, const uint32_t* __restrict__ run_ex,
+                                          const uint32_t* __restrict__ bound, const uint32_t* __restrict__ slots,
+                                          uint32_t mask, uint32_t* cnt, const uint32_t* __restrict__ cand_off,
+                                          const uint32_t* __restrict__ gidx, uint32_t* prefix, uint32_t* ext_off,
+                                          uint32_t* ext, uint32_t* gpar, uint32_t* eidx) {
+  uint32_t probe[GPA_MAX_K];
+  uint64_t A[GPA_MAX_K], B[GPA_MAX_K];
+  const uint32_t lane = threadIdx.x & 31;
+  if (EMIT && cnt[x] == 0) return;  // warp-uniform
+  // run index of x = (#run starts <= x) - 1
+  const uint32_t r = run_ex[x] + flags[x] - 1;
+  const uint32_t end = bound[r + 1];  // bound[n_runs] = n (sentinel)
+  if (!EMIT && end == x + 1) {
+    if (lane == 0) cnt[x] = 0;
+    return;
+  }
+  const uint32_t* px = L + (uint64_t)x * w;
+  // subset "px without item d, then b": A[d] = sum_{i<d} (x_i+1) P^i,
+  // B[d] = sum_{i>d} (x_i+1) P^(i-1); b lands at position w-1
+  uint64_t pw = 1, acc = 0;
+  for (uint32_t i = 0; i < w; ++i) {  // B[i] temporarily holds P^i
+    A[i] = acc;
+    B[i] = pw;
+    acc += (uint64_t)(px[i] + 1) * pw;
+    pw *= kHashP;
+  }
+  const uint64_t p_last = B[w - 1];  // P^(w-1)
+  uint64_t suf = 0;
+  for (uint32_t d = w; d-- > 0;) {
+    const uint64_t pprev = d > 0 ? B[d - 1] : 0;
+    B[d] = suf;
+    suf += (uint64_t)(px[d] + 1) * pprev;  // term of item d at position d-1
+  }
+  uint32_t here = 0;  // survivors so far (warp-uniform)
+  for (uint32_t y0 = x + 1; y0 < end; y0 += 32) {
+    const uint32_t y = y0 + lane;
+    bool keep = y < end;
+    uint32_t b = 0;
+    if (keep) {
+      b = L[(uint64_t)y * w + w - 1];
+      const uint64_t hb = (uint64_t)(b + 1) * p_last;
+      // subsets dropping item d of the shared prefix (dropping either of the last two items
+      // gives the parents x or y, members of L by construction)
+      for (uint32_t d = 0; d + 1 < w && keep; ++d) {
+        uint32_t q = 0;
+        for (uint32_t i = 0; i < w; ++i)
+          if (i != d) probe[q++] = px[i];
+        probe[q] = b;
+        keep = contains(L, w, slots, mask, probe, A[d] + B[d] + hb);
+      }
+    }
+    const uint32_t ballot = __ballot_sync(0xffffffffu, keep);
+    if (EMIT && keep) {
+      const uint32_t at = cand_off[x] + here + __popc(ballot & ((1u << lane) - 1u));
+      ext[at] = b;
+      eidx[at] = y;
+    }
+    here += __popc(ballot);
+  }
+  if (EMIT) {
+    const uint32_t g = gidx[x];
+    for (uint32_t i = lane; i < w; i += 32) prefix[(uint64_t)g * w + i] = px[i];
+    if (lane == 0) {
+      ext_off[g] = cand_off[x];
+      gpar[g] = x;
+    }
+  } else if (lane == 0) {
+    cnt[x] = here;
+  }
+}
+
+}  // namespace lvl
+}  // namespace gpa

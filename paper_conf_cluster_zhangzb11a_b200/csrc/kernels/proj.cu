@@ -38,15 +38,13 @@
 
 #include "../common.h"
 #include "../kernels.h"
+#include "proj_dev.cuh"
 
 namespace gpa {
 namespace {
+using namespace pj;
 
 constexpr int kT = 256;
-constexpr uint32_t kSegJ = 128;          // mask segment: 128 words per lane (a bitset row: 131,072 transactions)
-constexpr uint32_t kMemberGroup = 8;     // members sharing one mask preparation in pext_kernel
-constexpr uint32_t kG3Group = 16;        // members sharing one chunk's bit ranks in pext3_kernel
-
 unsigned grid_for(uint64_t n, int n_sms, int per_sm = 16) {
   uint64_t g = (n + kT - 1) / kT;
   const uint64_t cap = (uint64_t)n_sms * per_sm;
@@ -55,13 +53,19 @@ unsigned grid_for(uint64_t n, int n_sms, int per_sm = 16) {
 
 // ---------------------------------------------------------------- class structure
 // A class = a run of entries with the same par_a (the left parent = the (k-2)-prefix).
-__global__ void cls_flag_kernel(const uint32_t* __restrict__ par_a, uint32_t n, uint32_t* __restrict__ flag) {
+// n_dev (device-sized level): the entry count lives on the device, n is its host upper bound; the
+// flags are zero past the count (the scans run over n)
+__global__ void cls_flag_kernel(const uint32_t* __restrict__ par_a, uint32_t n, uint32_t* __restrict__ flag,
+                                const uint32_t* __restrict__ n_dev) {
+  const uint32_t ne = n_dev ? min(*n_dev, n) : n;
   for (uint32_t j = blockIdx.x * blockDim.x + threadIdx.x; j < n; j += gridDim.x * blockDim.x)
-    flag[j] = j == 0 || par_a[j] != par_a[j - 1];
+    flag[j] = j < ne && (j == 0 || par_a[j] != par_a[j - 1]);
 }
 
 __global__ void cls_bound_kernel(const uint32_t* __restrict__ flag, const uint32_t* __restrict__ ex, uint32_t n,
-                                 uint32_t* __restrict__ bound, uint32_t* __restrict__ n_cls) {
+                                 uint32_t* __restrict__ bound, uint32_t* __restrict__ n_cls,
+                                 const uint32_t* __restrict__ n_dev) {
+  n = n_dev ? min(*n_dev, n) : n;   // n_cls stays 0 (zeroed by the caller) when the level is empty
   for (uint32_t j = blockIdx.x * blockDim.x + threadIdx.x; j < n; j += gridDim.x * blockDim.x) {
     if (flag[j]) bound[ex[j]] = j;
     if (j == n - 1) {
@@ -72,82 +76,20 @@ __global__ void cls_bound_kernel(const uint32_t* __restrict__ flag, const uint32
   }
 }
 
-struct VecRef {
-  const uint32_t* p;
-  uint32_t lw;  // words per lane
-};
-
-// The mask of a class / the source of a member: a bitset row (generation 3) or one of the
-// previous generation's vectors.
-struct Src {
-  const uint32_t* rows;        // non-null: generation 3
-  uint64_t pitch;
-  const uint32_t* data;        // previous generation's vectors
-  const uint64_t* off;
-  const uint32_t* nw;
-  __device__ __forceinline__ VecRef vec(uint32_t id) const {
-    if (rows) return VecRef{rows + (uint64_t)id * pitch, (uint32_t)(pitch / 32)};
-    return VecRef{data + off[id], nw[id] / 32u};
-  }
-};
-
-__device__ __forceinline__ void seg_range(uint32_t lw, uint32_t s, uint32_t& j0, uint32_t& j1) {
-  j0 = min(lw, s * kSegJ);
-  j1 = min(lw, j0 + kSegJ);
-}
-
-// warp per (segment s, class c) pair p = s * cmax + c: lane l's mask popcount in the segment ->
-// words[p][l] = its output words (bits rounded up to whole words)
 __global__ void seg_popc_kernel(Src src, const uint32_t* __restrict__ par_a, const uint32_t* __restrict__ bound,
                                 const uint32_t* __restrict__ n_cls, uint32_t cmax, uint32_t nseg, uint32_t n_pairs,
                                 uint32_t* __restrict__ words, unsigned long long* __restrict__ in_words) {
-  const uint32_t lane = threadIdx.x & 31;
   const uint32_t p = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  if (p >= n_pairs) return;
-  const uint32_t c = p % cmax, s = p / cmax;
-  uint32_t cnt = 0;
-  if (c < *n_cls) {
-    const uint32_t j0 = bound[c], m = bound[c + 1] - j0;
-    if (m >= 2) {
-      const VecRef mk = src.vec(par_a[j0]);
-      uint32_t a, b;
-      seg_range(mk.lw, s, a, b);
-      for (uint32_t j = a; j < b; ++j) cnt += __popc(mk.p[32ull * j + lane]);
-      if (lane == 0 && b > a) atomicAdd(in_words, 32ull * (b - a) * m);
-    }
-  }
-  words[(uint64_t)p * 32 + lane] = (cnt + 31) / 32;
+  if (p < n_pairs) seg_popc_warp(p, src, par_a, bound, *n_cls, cmax, words, in_words);
 }
 
-// warp per class: lane l's word offset of every segment (loc), Lw_c = max over lanes of the
-// lane's total, words per member nwc = 32 Lw_c, the class' words and its pext items (one per
-// segment and group of kMemberGroup members)
 __global__ void cls_pad_kernel(const uint32_t* __restrict__ words, const uint32_t* __restrict__ bound,
                                const uint32_t* __restrict__ n_cls, uint32_t cmax, uint32_t nseg,
                                uint32_t* __restrict__ loc, uint32_t* __restrict__ nwc,
                                uint64_t* __restrict__ cls_words, uint32_t* __restrict__ items,
                                uint32_t* __restrict__ max_lw) {
-  const uint32_t lane = threadIdx.x & 31;
   const uint32_t c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  if (c >= cmax) return;
-  uint32_t m = 0;
-  if (c < *n_cls) m = bound[c + 1] - bound[c];
-  const uint32_t groups = m >= 2 ? (m + kMemberGroup - 1) / kMemberGroup : 0;
-  uint32_t acc = 0;
-  for (uint32_t s = 0; s < nseg; ++s) {
-    const uint64_t p = (uint64_t)s * cmax + c;
-    loc[p * 32 + lane] = acc;
-    const uint32_t w = words[p * 32 + lane];
-    acc += w;
-    const bool any = __any_sync(0xffffffffu, w != 0);
-    if (lane == 0) items[p] = any ? groups : 0;
-  }
-  const uint32_t lw = __reduce_max_sync(0xffffffffu, acc);
-  if (lane == 0) {
-    nwc[c] = groups ? 32u * lw : 0u;
-    cls_words[c] = groups ? (uint64_t)32u * lw * m : 0ull;
-    if (groups && lw) atomicMax(max_lw, lw);
-  }
+  if (c < cmax) cls_pad_warp(c, words, bound, *n_cls, cmax, nseg, loc, nwc, cls_words, items, max_lw);
 }
 
 // entry j -> its vector (offset, words); entries of single-member classes get none
@@ -323,54 +265,21 @@ __device__ __forceinline__ void pext_item(const uint32_t* __restrict__ mp, const
 // natural order, common to the class -- the next generation views it as 32 lane streams).
 // Work ~ output words, not input words.  (seg3 / cls3: sizes; pext3: the lists.)
 
-// warp per pair p = s * cmax + c: output words of row a's segment s (sum over its chunks)
 __global__ void seg3_kernel(const uint32_t* __restrict__ rows, uint64_t pitch, const uint32_t* __restrict__ par_a,
                             const uint32_t* __restrict__ bound, const uint32_t* __restrict__ n_cls, uint32_t cmax,
                             uint32_t n_pairs, uint32_t* __restrict__ w3, unsigned long long* __restrict__ in_words) {
-  const uint32_t lane = threadIdx.x & 31;
   const uint32_t p = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  if (p >= n_pairs) return;
-  const uint32_t c = p % cmax, s = p / cmax;
-  uint32_t words = 0;
-  if (c < *n_cls) {
-    const uint32_t j0 = bound[c], m = bound[c + 1] - j0;
-    if (m >= 2) {
-      const uint32_t* row = rows + (uint64_t)par_a[j0] * pitch + lane;
-      uint32_t a, b;
-      seg_range((uint32_t)(pitch / 32), s, a, b);
-      for (uint32_t j = a; j < b; ++j) {
-        const uint32_t C = __reduce_add_sync(0xffffffffu, (uint32_t)__popc(row[32ull * j]));
-        words += (C + 31) / 32;
-      }
-      if (lane == 0 && b > a) atomicAdd(in_words, 32ull * (b - a) * m);
-    }
-  }
-  if (lane == 0) w3[p] = words;
+  if (p < n_pairs) seg3_warp(p, rows, pitch, par_a, bound, *n_cls, cmax, w3, in_words);
 }
 
-// thread per class: word offset of every segment in the class' lists, list words (a multiple of
-// 32), the class' words, pext3 items (one per segment with words and group of <= kG3Group members)
 __global__ void cls3_pad_kernel(const uint32_t* __restrict__ w3, const uint32_t* __restrict__ bound,
                                 const uint32_t* __restrict__ n_cls, uint32_t cmax, uint32_t nseg,
                                 uint32_t* __restrict__ loc3, uint32_t* __restrict__ nwc,
                                 uint64_t* __restrict__ cls_words, uint32_t* __restrict__ items,
                                 uint32_t* __restrict__ max_lw) {
   const uint32_t C = *n_cls;
-  for (uint32_t c = blockIdx.x * blockDim.x + threadIdx.x; c < cmax; c += gridDim.x * blockDim.x) {
-    const uint32_t m = c < C ? bound[c + 1] - bound[c] : 0;
-    const uint32_t groups = m >= 2 ? (m + kG3Group - 1) / kG3Group : 0;
-    uint32_t acc = 0;
-    for (uint32_t s = 0; s < nseg; ++s) {
-      const uint64_t p = (uint64_t)s * cmax + c;
-      loc3[p] = acc;
-      acc += w3[p];
-      items[p] = w3[p] ? groups : 0;
-    }
-    const uint32_t words = groups ? (acc + 31u) & ~31u : 0u;
-    nwc[c] = words;
-    cls_words[c] = (uint64_t)words * m;
-    if (words) atomicMax(max_lw, words / 32u);
-  }
+  for (uint32_t c = blockIdx.x * blockDim.x + threadIdx.x; c < cmax; c += gridDim.x * blockDim.x)
+    cls3_pad_thread(c, w3, bound, C, cmax, nseg, loc3, nwc, cls_words, items, max_lw);
 }
 
 template <uint32_t G>
@@ -689,7 +598,7 @@ Src make_src(const ProjPending& pp) {
 
 bool proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const DeviceProj* prev,
                       const uint32_t* rows, uint64_t pitch_words, uint32_t n_rows, DeviceScratch& scratch, int n_sms,
-                      cudaStream_t s, ProjPending& pp) {
+                      cudaStream_t s, ProjPending& pp, const uint32_t* n_dev) {
   pp = ProjPending();
   pp.n = n;
   pp.par_a = par_a;
@@ -719,9 +628,10 @@ bool proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, 
   W.bound.ensure(n + 1);
   W.small.ensure(4);
   GPA_CUDA(cudaMemsetAsync(W.small.p, 0, 16, s));
-  { cls_flag_kernel<<<grid_for(n, n_sms), kT, 0, s>>>(par_a, n, W.flag.p); note_launch(); }
+  { cls_flag_kernel<<<grid_for(n, n_sms), kT, 0, s>>>(par_a, n, W.flag.p, n_dev); note_launch(); }
   scan_excl<uint32_t>(W.flag.p, W.ex.p, n, W.tmp, s);
-  { cls_bound_kernel<<<grid_for(n, n_sms), kT, 0, s>>>(W.flag.p, W.ex.p, n, W.bound.p, W.small.p); note_launch(); }
+  { cls_bound_kernel<<<grid_for(n, n_sms), kT, 0, s>>>(W.flag.p, W.ex.p, n, W.bound.p, W.small.p, n_dev);
+    note_launch(); }
   W.words.ensure((size_t)n_pairs * 32);
   W.loc.ensure((size_t)n_pairs * 32);
   W.items.ensure(n_pairs);
@@ -809,7 +719,7 @@ bool proj_build(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const 
                 const uint32_t* rows, uint64_t pitch_words, uint32_t n_rows, DeviceProj& out, DeviceScratch& scratch,
                 int n_sms, cudaStream_t s, cudaEvent_t ev_build) {
   ProjPending pp;
-  if (!proj_build_begin(n, par_a, par_b, prev, rows, pitch_words, n_rows, scratch, n_sms, s, pp)) return false;
+  if (!proj_build_begin(n, par_a, par_b, prev, rows, pitch_words, n_rows, scratch, n_sms, s, pp, nullptr)) return false;
   uint64_t T[2] = {0, 0};
   uint32_t sm[4] = {0, 0, 0, 0};
   if (n) {

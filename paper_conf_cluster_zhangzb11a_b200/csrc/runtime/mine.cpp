@@ -246,6 +246,7 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
   struct Pending {       // a generation's frequent itemsets, still on the device
     size_t level = 0;
     uint32_t F = 0, k = 0;
+    bool open = false;                  // |L_k| not yet read back (device-sized level)
     DBuf<uint32_t> items, sup;
     const uint32_t* h_items = nullptr;  // page-locked copies (pinned_arena)
     const uint32_t* h_sup = nullptr;
@@ -265,6 +266,34 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     ~Events() { for (auto x : e) if (x) cudaEventDestroy(x); }
   } copy_evs;
   cudaEvent_t* copy_ev = copy_evs.e;
+  // |L_k| known on the host: record it and start the D2H of L_k (item ids, supports) on the copy
+  // stream -- s has just been synchronised, so everything that produced L_k is complete
+  auto finalize = [&](Pending& pd, uint32_t F) {
+    pd.F = F;
+    pd.open = false;
+    R->levels[pd.level].n_freq = F;
+    R->levels[pd.level].stats.n_freq = F;
+    if (F) {
+      auto* hi = static_cast<uint32_t*>(pinned_arena().get((size_t)F * pd.k * 4));
+      auto* hs = static_cast<uint32_t*>(pinned_arena().get((size_t)F * 4));
+      GPA_CUDA(cudaEventRecord(copy_ev[pd.k % kCopyEvents], s));
+      GPA_CUDA(cudaStreamWaitEvent(copy_s.s, copy_ev[pd.k % kCopyEvents], 0));
+      GPA_CUDA(cudaMemcpyAsync(hi, pd.items.p, (size_t)F * pd.k * 4, cudaMemcpyDeviceToHost, copy_s.s));
+      GPA_CUDA(cudaMemcpyAsync(hs, pd.sup.p, (size_t)F * 4, cudaMemcpyDeviceToHost, copy_s.s));
+      pd.h_items = hi;
+      pd.h_sup = hs;
+    }
+  };
+  // a device-sized L_{k-1}: read |L_{k-1}| now (a synchronisation of its own)
+  auto settle = [&](DeviceLevel& L) {
+    if (!L.n_dev) return;
+    uint32_t* hs = host_sizes();
+    GPA_CUDA(cudaMemcpyAsync(hs + 15, L.n_dev, 4, cudaMemcpyDeviceToHost, s));
+    stream_wait(s);
+    L.n = hs[15];
+    L.n_dev = nullptr;
+    finalize(pending.back(), L.n);
+  };
   CopyStream aux_s;          // the emitting join of C_k, overlapping the list build on s
   Events aux_evs;            // [0] s -> aux (batch buffers sized), [1] aux done
   ProjPending ppend;
@@ -313,6 +342,7 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     } else if (host_candgen) {
       // reference path (GPA_HOST_CANDGEN): L_{k-1} back to the host, threaded join + prune
       // (runtime/candgen.cpp), the batch up to the device for the device-side threshold
+      settle(Ld);
       std::vector<uint32_t> Lh((size_t)Ld.n * (k - 1));
       if (Ld.n) {
         GPA_CUDA(cudaMemcpyAsync(Lh.data(), Ld.rows.p, Lh.size() * 4, cudaMemcpyDeviceToHost, s));
@@ -343,31 +373,55 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
       // the class tables (aux_s) are independent of the join's stage 1 (s): both read L_{k-1}
       GPA_CUDA(cudaEventRecord(aux_evs.e[2], s));
       GPA_CUDA(cudaStreamWaitEvent(aux_s.s, aux_evs.e[2], 0));
+      // L_{k-1} is device-sized: |L_{k-1}| comes back with the sizes of C_k and of the lists -- ONE
+      // synchronisation per generation
+      const uint32_t n_up = Ld.n_dev ? Ld.n_max : Ld.n;
       if (device_candgen_begin(Ld, Bd, scratch, bs->n_sms, s, &d_sizes)) {
         uint32_t* hs = host_sizes();
-        if (proj_build_begin(Ld.n, Ld.par_a.p, Ld.par_b.p, k == 3 ? nullptr : Pprev, bs->rows.p, bs->pitch_words,
-                             bs->n_rows, scratch, bs->n_sms, aux_s.s, ppend)) {
+        if (proj_build_begin(n_up, Ld.par_a.p, Ld.par_b.p, k == 3 ? nullptr : Pprev, bs->rows.p, bs->pitch_words,
+                             bs->n_rows, scratch, bs->n_sms, aux_s.s, ppend, Ld.n_dev)) {
           GPA_CUDA(cudaMemcpyAsync(hs + 2, ppend.d_tot, 16, cudaMemcpyDeviceToHost, aux_s.s));
           GPA_CUDA(cudaMemcpyAsync(hs + 6, ppend.d_small, 16, cudaMemcpyDeviceToHost, aux_s.s));
         } else {
           proj_on = false;   // lists not addressable: complete intersection from this generation on
         }
         GPA_CUDA(cudaMemcpyAsync(hs, d_sizes, 8, cudaMemcpyDeviceToHost, s));
+        if (Ld.n_dev) GPA_CUDA(cudaMemcpyAsync(hs + 10, Ld.n_dev, 4, cudaMemcpyDeviceToHost, s));
         stream_wait(s);
         stream_wait(aux_s.s);
         M = hs[0];
         G = hs[1];
         std::memcpy(pT, hs + 2, 16);
         std::memcpy(psm, hs + 6, 16);
+        if (Ld.n_dev) {
+          Ld.n = hs[10];
+          Ld.n_dev = nullptr;
+          finalize(pending.back(), Ld.n);
+        }
+        ppend.n = Ld.n;   // the class tables ran over the upper bound; the lists are for |L_{k-1}| entries
         device_candgen_finish(Ld, Bd, scratch, bs->n_sms, s, (uint32_t)M, (uint32_t)G, aux_s.s, aux_evs.e[0]);
         GPA_CUDA(cudaEventRecord(aux_evs.e[1], aux_s.s));
         aux_join = true;
       }
     } else {
-      device_candgen(Ld, Bd, scratch, bs->n_sms, s);
+      // complete intersection: join + prune on the device, |L_{k-1}| read with the sizes of C_k
+      const uint32_t* d_sizes = nullptr;
+      if (device_candgen_begin(Ld, Bd, scratch, bs->n_sms, s, &d_sizes)) {
+        uint32_t* hs = host_sizes();
+        GPA_CUDA(cudaMemcpyAsync(hs, d_sizes, 8, cudaMemcpyDeviceToHost, s));
+        if (Ld.n_dev) GPA_CUDA(cudaMemcpyAsync(hs + 10, Ld.n_dev, 4, cudaMemcpyDeviceToHost, s));
+        stream_wait(s);
+        if (Ld.n_dev) {
+          Ld.n = hs[10];
+          Ld.n_dev = nullptr;
+          finalize(pending.back(), Ld.n);
+        }
+        device_candgen_finish(Ld, Bd, scratch, bs->n_sms, s, hs[0], hs[1], s, nullptr);
+      }
       M = Bd.M;
       G = Bd.G;
     }
+    settle(Ld);   // (candidate generation skipped: fewer than 2 members at most)
     double t1 = now_ms();
     if (M == 0) {
       events.pop_back();
@@ -414,31 +468,22 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     if (keep && k > 2) fetch_batch();
     double t2 = now_ms();
 
-    const uint32_t F = device_threshold(bs->d_counts.p, (uint32_t)M, (uint32_t)min_count, k, l1_size(bs),
-                                        k == 2 && bs->l1_sub ? bs->d_l1.p : nullptr, Bd.prefix.p,
-                                        Bd.ext_off.p, Bd.ext.p, (uint32_t)G, host_candgen ? nullptr : Bd.gpar.p,
-                                        host_candgen ? nullptr : Bd.eidx.p, Ln, scratch, bs->n_sms, s);
-    // the frequent itemsets of this generation (item ids) and supports stay on the device until the
-    // end of the loop: one transfer for all generations instead of one synchronisation each
+    // L_k = { c in C_k : count >= min_count } on the device WITHOUT a synchronisation: |L_k| stays on
+    // the device (Ln is device-sized) and comes back with the next generation's sizes (or settle())
+    device_threshold_async(bs->d_counts.p, (uint32_t)M, (uint32_t)min_count, k, l1_size(bs),
+                           k == 2 && bs->l1_sub ? bs->d_l1.p : nullptr, Bd.prefix.p, Bd.ext_off.p, Bd.ext.p,
+                           (uint32_t)G, host_candgen ? nullptr : Bd.gpar.p, host_candgen ? nullptr : Bd.eidx.p, Ln,
+                           scratch, bs->n_sms, s);
+    // the frequent itemsets of this generation (item ids) and supports, mapped on the device (over
+    // the upper bound M; the kernel stops at |L_k|); their D2H starts once |L_k| is known (finalize)
     Pending pd;
     pd.level = R->levels.size();
-    pd.F = F;
     pd.k = k;
-    if (F) {
-      pd.items.alloc((size_t)F * k, s);
-      pd.sup.alloc(F, s);
-      device_map_items(Ln.rows.p, (uint64_t)F * k, d_ior.p, pd.items.p, bs->n_sms, s);
-      GPA_CUDA(cudaMemcpyAsync(pd.sup.p, Ln.sup.p, (size_t)F * 4, cudaMemcpyDeviceToDevice, s));
-      auto* hi = static_cast<uint32_t*>(pinned_arena().get((size_t)F * k * 4));
-      auto* hs = static_cast<uint32_t*>(pinned_arena().get((size_t)F * 4));
-      // D2H on the copy stream, overlapping the next generations on s
-      GPA_CUDA(cudaEventRecord(copy_ev[(k - 2) % kCopyEvents], s));
-      GPA_CUDA(cudaStreamWaitEvent(copy_s.s, copy_ev[(k - 2) % kCopyEvents], 0));
-      GPA_CUDA(cudaMemcpyAsync(hi, pd.items.p, (size_t)F * k * 4, cudaMemcpyDeviceToHost, copy_s.s));
-      GPA_CUDA(cudaMemcpyAsync(hs, pd.sup.p, (size_t)F * 4, cudaMemcpyDeviceToHost, copy_s.s));
-      pd.h_items = hi;
-      pd.h_sup = hs;
-    }
+    pd.open = true;
+    pd.items.alloc((size_t)M * k, s);
+    pd.sup.alloc(M, s);
+    device_map_items(Ln.rows.p, (uint64_t)M * k, d_ior.p, pd.items.p, bs->n_sms, s, Ln.n_dev, k);
+    GPA_CUDA(cudaMemcpyAsync(pd.sup.p, Ln.sup.p, (size_t)M * 4, cudaMemcpyDeviceToDevice, s));
     ev.counted = cs.e0 != nullptr;
     GPA_CUDA(cudaEventRecord(ev.e[6], s));
     std::vector<uint32_t> counts;
@@ -449,18 +494,17 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     }
     const double tr0 = now_ms();
     record_level(R, bs, k, k > 2 ? &batch : nullptr, M, {}, {}, keep, keep ? &counts : nullptr);
-    R->levels.back().n_freq = F;
+    R->levels.back().n_freq = 0;   // set by finalize()
     pending.push_back(std::move(pd));
     std::swap(Ld, Ln);
-    nL = F;
+    nL = M;   // an upper bound of |L_k|: the next generation's candidate count decides
     if (trace_enabled())
-      fprintf(stderr, "[gpa] k=%u M=%llu G=%llu: candgen %.2f ms, count phase %.2f ms, threshold %.2f ms (record %.2f) "
-              "-> |L|=%u\n", k, (unsigned long long)M, (unsigned long long)G, t1 - t0, t2 - t1, now_ms() - t2,
-              now_ms() - tr0, F);
+      fprintf(stderr, "[gpa] k=%u M=%llu G=%llu: candgen %.2f ms, count phase %.2f ms, threshold enqueue %.2f ms "
+              "(record %.2f)\n", k, (unsigned long long)M, (unsigned long long)G, t1 - t0, t2 - t1, now_ms() - t2,
+              now_ms() - tr0);
     event_level.push_back(R->levels.size() - 1);
     gpa_level_stats& st = R->levels.back().stats;
     st.n_cand = M;
-    st.n_freq = F;
     st.n_groups = G;
     st.kernel = cs.kernel;
     st.launches = cs.launches;
@@ -472,6 +516,7 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     st.count_bytes = cs.count_bytes;
   }
 
+  settle(Ld);   // the last generation's |L_k| (when the loop ended on max_k)
   // ---- deferred: kernel times and the frequent itemsets of every generation
   const double tf0 = now_ms();
   stream_wait(s);
