@@ -551,11 +551,24 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     R->phase_ms[GPA_PHASE_COUNT] += a + b;
     R->phase_ms[GPA_PHASE_THRESHOLD] += g - cg - a - b;
   }
-  parallel_for(pending.size(), [&](size_t i) {
+  // pinned staging -> the result's vectors: sized first, then copied in ~256 KB pieces over the pool
+  // (one generation can hold most of F)
+  struct Piece { size_t i; uint64_t a, b; };
+  std::vector<Piece> pieces;
+  for (size_t i = 0; i < pending.size(); ++i) {
     const Pending& pd = pending[i];
     gpa_level_data& lv = R->levels[pd.level];
-    lv.freq_items.assign(pd.h_items, pd.h_items + (size_t)pd.F * pd.k);
-    lv.freq_support.assign(pd.h_sup, pd.h_sup + pd.F);
+    lv.freq_items.resize((size_t)pd.F * pd.k);
+    lv.freq_support.resize(pd.F);
+    const uint64_t step = std::max<uint64_t>(1, (uint64_t)65536 / std::max<uint32_t>(pd.k, 1));
+    for (uint64_t a = 0; a < pd.F; a += step) pieces.push_back({i, a, std::min<uint64_t>(pd.F, a + step)});
+  }
+  parallel_for(pieces.size(), [&](size_t j) {
+    const Piece& pc = pieces[j];
+    const Pending& pd = pending[pc.i];
+    gpa_level_data& lv = R->levels[pd.level];
+    std::memcpy(lv.freq_items.data() + pc.a * pd.k, pd.h_items + pc.a * pd.k, (pc.b - pc.a) * pd.k * 4);
+    std::memcpy(lv.freq_support.data() + pc.a, pd.h_sup + pc.a, (pc.b - pc.a) * 4);
   });
   pending.clear();
   if (trace_enabled())
