@@ -112,6 +112,11 @@ typedef struct {
                                   to the transactions of its (k-2)-prefix; a candidate's support is the
                                   popcount of the AND of its two parents' lists (exact, same counts as
                                   complete intersection).  k = 2 as AUTO; gpa_count treats it as AUTO */
+#define GPA_KERNEL_FUSED 7u    /* gpa_mine: every generation k >= 2 in ONE cooperative launch (grid-wide phases:
+                                  complete-intersection counting, threshold, join + prune; no per-level launch or
+                                  host round trip) when |L_1| <= 256 and the L_1 rows fit 64 MB; AUTO picks it for
+                                  such problems on one GPU.  Otherwise (or on a capacity overflow) AUTO's kernels.
+                                  gpa_count treats it as AUTO */
 
 #define GPA_KEEP_CANDIDATES 1u /* gpa_mine: keep every generation's (C_k, counts), not only F */
 #define GPA_HOST_CANDGEN 2u    /* gpa_mine: join + prune on the host thread pool instead of the device
@@ -119,6 +124,7 @@ typedef struct {
 #define GPA_NO_OVERLAP_INGEST 4u /* gpa_mine, host input: upload the whole database before computing
                                   (default: upload in chunks overlapped with histogram, bitset build and
                                   generation-2 counting) */
+#define GPA_MULTI_KERNEL 16u    /* gpa_mine: never the single-launch path of GPA_KERNEL_FUSED under AUTO */
 #define GPA_COMPLETE_INTERSECTION 8u /* gpa_mine: every generation k >= 3 by complete intersection from the
                                   static bitset (the paper's method, P18@394; TRIE / PREFIX kernels), never
                                   the projected lists of GPA_KERNEL_PROJ.  With count_kernel GPA_KERNEL_PAIRS

@@ -27,18 +27,20 @@ import numpy as np
 
 __all__ = [
     "GpaError", "lib", "version", "min_count", "Options", "Dist", "Bitset", "mine", "MineResult", "Rules",
-    "KERNEL_AUTO", "KERNEL_V0", "KERNEL_PREFIX", "KERNEL_PAIRS", "KERNEL_TRIE", "KERNEL_PAIRS_TC", "KERNEL_PROJ", "PHASES",
+    "KERNEL_AUTO", "KERNEL_V0", "KERNEL_PREFIX", "KERNEL_PAIRS", "KERNEL_TRIE", "KERNEL_PAIRS_TC", "KERNEL_PROJ",
+    "KERNEL_FUSED", "PHASES",
 ]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libgpapriori.so")
 
-KERNEL_AUTO, KERNEL_V0, KERNEL_PREFIX, KERNEL_PAIRS, KERNEL_TRIE, KERNEL_PAIRS_TC, KERNEL_PROJ = 0, 1, 2, 3, 4, 5, 6
-KERNEL_NAMES = {0: "auto", 1: "v0", 2: "prefix", 3: "pairs", 4: "trie", 5: "pairs_tc", 6: "proj"}
+KERNEL_AUTO, KERNEL_V0, KERNEL_PREFIX, KERNEL_PAIRS, KERNEL_TRIE, KERNEL_PAIRS_TC, KERNEL_PROJ, KERNEL_FUSED = range(8)
+KERNEL_NAMES = {0: "auto", 1: "v0", 2: "prefix", 3: "pairs", 4: "trie", 5: "pairs_tc", 6: "proj", 7: "fused"}
 KEEP_CANDIDATES = 1
 HOST_CANDGEN = 2
 NO_OVERLAP_INGEST = 4
 COMPLETE_INTERSECTION = 8
+MULTI_KERNEL = 16
 MEM_HOST, MEM_DEVICE = 0, 1
 PHASES = ["upload", "histogram", "bitset", "candgen", "count", "threshold", "total"]
 STATUS = {0: "GPA_OK", 1: "GPA_ERR_INVALID", 2: "GPA_ERR_RANGE", 3: "GPA_ERR_OOM", 4: "GPA_ERR_CUDA",
@@ -159,6 +161,7 @@ class Options:
     host_candgen: bool = False   # join + prune on the host (reference path) instead of the device
     overlap_ingest: bool = True  # host input: chunked upload overlapped with histogram / bitset / pairs
     complete_intersection: bool = False   # k >= 3 by complete intersection (the paper's method), no lists
+    multi_kernel: bool = False   # never the single-launch small-problem path (KERNEL_FUSED) under AUTO
 
     def _c(self) -> _Options:
         o = _Options()
@@ -166,7 +169,8 @@ class Options:
         o.count_kernel = self.count_kernel
         o.flags = ((KEEP_CANDIDATES if self.keep_candidates else 0) | (HOST_CANDGEN if self.host_candgen else 0)
                    | (0 if self.overlap_ingest else NO_OVERLAP_INGEST)
-                   | (COMPLETE_INTERSECTION if self.complete_intersection else 0))
+                   | (COMPLETE_INTERSECTION if self.complete_intersection else 0)
+                   | (MULTI_KERNEL if self.multi_kernel else 0))
         o.stream = self.stream or None
         o.device = self.device
         o.max_k = self.max_k

@@ -227,6 +227,25 @@ bool device_candgen_begin(const DeviceLevel& L, DeviceBatch& out, DeviceScratch&
 void device_candgen_finish(const DeviceLevel& L, DeviceBatch& out, DeviceScratch& scratch, int n_sms, cudaStream_t s,
                            uint32_t M, uint32_t G, cudaStream_t run, cudaEvent_t ev);
 
+// ---- the whole level loop in one cooperative launch for small problems (mine_fused.cu)
+constexpr uint32_t kFusedMaxRows = 256;                       // |L_1|
+constexpr uint64_t kFusedMaxBitsetBytes = 64ull << 20;        // L_1 rows (L2-resident)
+bool fused_eligible(uint32_t n1, uint64_t pitch_words);
+struct FusedOut {
+  struct Level {
+    uint32_t k = 0, M = 0, F = 0, G = 0;
+    uint64_t freq_word = 0, freq_entry = 0, cand_word = 0, cand_entry = 0;   // offsets into the arrays below
+  };
+  std::vector<Level> levels;               // generations 2 .. last
+  std::vector<uint32_t> items, sup;        // L_k item ids (F x k per generation) and supports, in order
+  std::vector<uint32_t> cand_items, cand_counts;   // keep: every C_k (M x k) and its counts
+};
+// Levels k >= 2 of gpa_mine over the L_1 rows (n1 entries; d_sel: entry -> bitset row or nullptr;
+// d_ior: bitset row -> item id).  false: a capacity was exceeded (nothing usable in out).
+bool mine_fused(const uint32_t* rows, uint64_t pitch_words, uint64_t n_tx, uint32_t n1, const uint32_t* d_sel,
+                const uint32_t* d_ior, uint32_t theta, uint32_t max_k, bool keep, int n_sms, cudaStream_t s,
+                FusedOut& out);
+
 // ---- device-side work planning (plan.cu)
 constexpr uint32_t kPlanMaxRows = 65536;   // row bitmap of the planning kernels (8 KB of shared memory)
 void launch_cand_group(const uint32_t* ext_off, uint32_t G, uint32_t* cand_group, int n_sms, cudaStream_t s);

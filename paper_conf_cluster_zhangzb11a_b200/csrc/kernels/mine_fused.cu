@@ -1,0 +1,439 @@
+// The whole level-wise loop in ONE cooperative launch, for problems whose L_1 bitset sits in L2
+// (sm_100a).  SURVEY.md §8(f) f1: "a fully device-resident level loop (CUDA graph or persistent
+// kernel, no per-level D2H)".
+//
+// Small databases (the chess-, mushroom- and accidents-shaped configurations: <= 256 frequent
+// items, a few MB of bitset) are latency-bound: the multi-kernel path spends ~30 launches and a
+// host synchronisation per generation on a few microseconds of counting.  Here every generation is
+// a sequence of grid-wide phases separated by grid.sync() -- no launch, no host round trip:
+//
+//   count    supp(c) = popc(AND of the k rows of c) -- the paper's complete intersection (P18@394),
+//            a warp per (prefix group, <= 32 extensions): the (k-1)-row prefix AND per 32-word
+//            chunk in registers, one AND + POPC per extension word, per-lane accumulators reduced
+//            once per batch (redux.sync)
+//   threshold L_k = { c : count >= theta } (P13@474, ">=" per DESIGN.md Q1): flag, grid scan,
+//            scatter of the rows in candidate (= lexicographic) order, the frequent itemsets and
+//            supports appended to the output arena in original item ids
+//   join     C_{k+1} = join of run siblings + prune by a hash set of L_k (P13@1006-1270, P13@178),
+//            grouped by k-prefix: run starts, grid scan, run bounds, hash insert, survivor counts,
+//            grid scans of the counts and of the non-empty groups, emit
+//
+// Termination when L_k or C_{k+1} is empty (P13@652) or after max_k.  Capacities are fixed at
+// launch; an overflow sets a status bit and the host reruns the problem on the multi-kernel path
+// (never a CPU path).  Integer only; the same sets and counts as every other path.
+#include <cooperative_groups.h>
+#include <algorithm>
+#include <map>
+#include <vector>
+#include <cstdint>
+#include <cstdlib>
+
+#include "../common.h"
+#include "../kernels.h"
+#include "level_dev.cuh"
+
+namespace cg = cooperative_groups;
+
+namespace gpa {
+namespace {
+
+constexpr int kFT = 256;                 // threads per CTA
+constexpr uint32_t kWarps = kFT / 32;
+
+// --- grid-wide exclusive scan of get(i), i < n -> out[i]; returns the total on every thread.
+// Two grid syncs: block sums, then (after every CTA read them) the next user may reuse bsum.
+template <class F>
+__device__ uint32_t grid_scan(F get, uint32_t* out, uint32_t n, uint32_t* bsum, cg::grid_group& grid) {
+  __shared__ uint32_t sh[kWarps + 1];
+  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const uint32_t per = ((n + gridDim.x - 1) / gridDim.x + kFT - 1) / kFT * kFT;
+  const uint32_t b0 = min(n, blockIdx.x * per), b1 = min(n, b0 + per);
+  uint32_t s = 0;
+  for (uint32_t i = b0 + threadIdx.x; i < b1; i += kFT) s += get(i);
+  s = __reduce_add_sync(0xffffffffu, s);
+  if (lane == 0) sh[warp] = s;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    uint32_t t = 0;
+    for (uint32_t w = 0; w < kWarps; ++w) t += sh[w];
+    bsum[blockIdx.x] = t;
+  }
+  __syncthreads();
+  grid.sync();
+  uint32_t off = 0, tot = 0;
+  for (uint32_t b = threadIdx.x; b < gridDim.x; b += kFT) {
+    const uint32_t v = bsum[b];
+    tot += v;
+    if (b < blockIdx.x) off += v;
+  }
+  off = __reduce_add_sync(0xffffffffu, off);
+  tot = __reduce_add_sync(0xffffffffu, tot);
+  __syncthreads();
+  if (lane == 0) sh[warp] = off;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    uint32_t a = 0;
+    for (uint32_t w = 0; w < kWarps; ++w) a += sh[w];
+    sh[kWarps] = a;
+  }
+  __syncthreads();
+  off = sh[kWarps];
+  __syncthreads();
+  if (lane == 0) sh[warp] = tot;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    uint32_t a = 0;
+    for (uint32_t w = 0; w < kWarps; ++w) a += sh[w];
+    sh[kWarps] = a;
+  }
+  __syncthreads();
+  tot = sh[kWarps];
+  __syncthreads();
+  // block-level scan of the CTA's range in chunks of kFT, offset by the earlier CTAs' sums
+  for (uint32_t base = b0; base < b1; base += kFT) {
+    const uint32_t i = base + threadIdx.x;
+    const uint32_t v = i < b1 ? get(i) : 0u;
+    uint32_t x = v;
+#pragma unroll
+    for (uint32_t d = 1; d < 32; d <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xffffffffu, x, d);
+      if (lane >= d) x += y;
+    }
+    if (lane == 31) sh[warp] = x;
+    __syncthreads();
+    uint32_t woff = 0, ctot = 0;
+    for (uint32_t w = 0; w < kWarps; ++w) {
+      const uint32_t t = sh[w];
+      if (w < warp) woff += t;
+      ctot += t;
+    }
+    if (i < b1) out[i] = off + woff + x - v;
+    off += ctot;
+    __syncthreads();
+  }
+  grid.sync();
+  return tot;
+}
+
+struct FusedParams {
+  const uint32_t* rows;      // bitset rows
+  uint64_t pitch;            // words per row
+  uint32_t W;                // words in use (ceil(n_tx / 32), multiple of 32 not required)
+  uint32_t n1;               // |L_1|
+  const uint32_t* sel;       // L_1 entry -> bitset row (nullptr: identity)
+  const uint32_t* ior;       // bitset row -> item id
+  uint32_t theta, max_k;
+  // capacities
+  uint32_t cap_cand;         // candidates per generation (M)
+  uint32_t cap_words;        // words of an L_k / C_k prefix table (entries x k)
+  uint32_t cap_hash;         // power of two
+  uint64_t cap_out;          // words of the output arenas (items; supports / counts separately)
+  int keep;                  // record every (C_k, counts)
+  // candidate buffers (C_k): grouped by (k-1)-prefix
+  uint32_t *prefix, *ext_off, *ext, *counts, *pos;
+  // levels: L rows (ping-pong), join scratch
+  uint32_t *L[2];
+  uint32_t *rs, *run_ex, *bound, *cnt, *cand_off, *gidx, *slots[2];
+  uint32_t* bsum;
+  // outputs: per generation k (index k): {M_k, F_k, G_k, freq arena offset (lo, hi), cand arena offset (lo, hi)}
+  uint32_t* level_tab;       // 8 words per generation, GPA_MAX_K + 1 generations
+  uint32_t *out_items, *out_sup, *cand_items, *cand_counts;
+  uint32_t* status;          // [0] bit 1: overflow, [1] generations done
+};
+
+__device__ __forceinline__ const uint32_t* row_ptr(const FusedParams& P, uint32_t r) {
+  return P.rows + (uint64_t)(P.sel ? P.sel[r] : r) * P.pitch;
+}
+
+// counts[m] for the grouped batch (G groups, prefix width km1) -- warp per (group, batch of <= 32
+// extensions), lanes over 32-word chunks of the rows
+__device__ void count_phase(const FusedParams& P, uint32_t G, uint32_t km1) {
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, n_warps = (gridDim.x * blockDim.x) >> 5;
+  // work items: (group, batch); batches per group = ceil(n_ext / 32); enumerate groups, then batches
+  for (uint32_t g = gw; g < G; g += n_warps) {
+    const uint32_t e0 = P.ext_off[g], e1 = P.ext_off[g + 1];
+    const uint32_t* pr = P.prefix + (uint64_t)g * km1;
+    for (uint32_t b0 = e0; b0 < e1; b0 += 32) {
+      const uint32_t nb = min(32u, e1 - b0);
+      // lane j: the row of extension j (word offset)
+      const uint64_t my_row = lane < nb ? (uint64_t)(P.sel ? P.sel[P.ext[b0 + lane]] : P.ext[b0 + lane]) * P.pitch : 0;
+      uint32_t acc[32];
+#pragma unroll
+      for (int j = 0; j < 32; ++j) acc[j] = 0;
+      for (uint32_t base = 0; base < P.W; base += 32) {   // lane = word of the chunk
+        const uint32_t w = base + lane;
+        const bool in = w < P.W;
+        uint32_t pw = in ? 0xffffffffu : 0u;
+        for (uint32_t d = 0; d < km1; ++d) pw &= in ? __ldg(row_ptr(P, pr[d]) + w) : 0u;
+#pragma unroll
+        for (int j = 0; j < 32; ++j) {
+          if (j < (int)nb) {
+            const uint64_t ro = __shfl_sync(0xffffffffu, my_row, j);
+            acc[j] += __popc(pw & (in ? __ldg(P.rows + ro + w) : 0u));
+          }
+        }
+      }
+#pragma unroll
+      for (int j = 0; j < 32; ++j) {
+        if (j < (int)nb) {
+          const uint32_t t = __reduce_add_sync(0xffffffffu, acc[j]);
+          if (lane == j) P.counts[b0 + j] = t;
+        }
+      }
+    }
+  }
+}
+
+__global__ void __launch_bounds__(kFT) mine_fused_kernel(FusedParams P) {
+  cg::grid_group grid = cg::this_grid();
+  const uint32_t tid = blockIdx.x * blockDim.x + threadIdx.x, n_threads = gridDim.x * blockDim.x;
+  const uint32_t gw = tid >> 5, n_warps = n_threads >> 5;
+  const uint32_t lane = threadIdx.x & 31;
+  // ---- C_2 = every pair of L_1 entries, grouped by the first: group a = {a} x (a, n1)
+  const uint32_t n1 = P.n1;
+  uint32_t G = n1 > 1 ? n1 - 1 : 0;
+  uint32_t M = n1 > 1 ? n1 * (n1 - 1) / 2 : 0;
+  for (uint32_t a = tid; a < G; a += n_threads) {
+    P.prefix[a] = a;
+    const uint32_t off = a * n1 - a * (a + 1) / 2;   // pair_index(a, a + 1, n1)
+    P.ext_off[a] = off;
+    for (uint32_t b = a + 1; b < n1; ++b) P.ext[off + (b - a - 1)] = b;
+  }
+  if (tid == 0) P.ext_off[G] = M;
+  for (uint32_t i = tid; i < P.cap_hash; i += n_threads) P.slots[0][i] = P.slots[1][i] = lvl::kEmpty;
+  uint64_t fw = 0, fn = 0, cw = 0, cn = 0;   // output arenas: words / entries so far (frequent, candidates)
+  uint32_t k = 2;
+  grid.sync();
+  for (; k <= P.max_k && M > 0; ++k) {
+    const uint32_t km1 = k - 1;
+    // ---- count C_k
+    count_phase(P, G, km1);
+    grid.sync();
+    // ---- threshold: L_k in candidate (lexicographic) order
+    const uint32_t theta = P.theta;
+    const uint32_t* counts = P.counts;
+    const uint32_t F = grid_scan([&](uint32_t m) { return counts[m] >= theta ? 1u : 0u; }, P.pos, M, P.bsum, grid);
+    uint32_t* Lk = P.L[k & 1];
+    const bool fit = (uint64_t)F * k <= P.cap_words && fw + (uint64_t)F * k <= P.cap_out &&
+                     (!P.keep || cw + (uint64_t)M * k <= P.cap_out);
+    if (!fit) {
+      if (tid == 0) P.status[0] |= 1u;
+      break;   // uniform: every thread computed the same F
+    }
+    for (uint32_t m = tid; m < M; m += n_threads) {
+      const uint32_t c = counts[m];
+      const bool freq = c >= theta;
+      if (!freq && !P.keep) continue;
+      uint32_t lo = 0, hi = G;   // g = last group with ext_off[g] <= m
+      while (lo + 1 < hi) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (P.ext_off[mid] <= m) lo = mid; else hi = mid;
+      }
+      const uint32_t* pr = P.prefix + (uint64_t)lo * km1;
+      const uint32_t e = P.ext[m];
+      if (freq) {
+        const uint32_t p = P.pos[m];
+        uint32_t* dst = Lk + (uint64_t)p * k;
+        uint32_t* od = P.out_items + fw + (uint64_t)p * k;
+        for (uint32_t d = 0; d < km1; ++d) {
+          dst[d] = pr[d];
+          od[d] = P.ior[P.sel ? P.sel[pr[d]] : pr[d]];
+        }
+        dst[km1] = e;
+        od[km1] = P.ior[P.sel ? P.sel[e] : e];
+        P.out_sup[fn + p] = c;
+      }
+      if (P.keep) {
+        uint32_t* cd = P.cand_items + cw + (uint64_t)m * k;
+        for (uint32_t d = 0; d < km1; ++d) cd[d] = P.ior[P.sel ? P.sel[pr[d]] : pr[d]];
+        cd[km1] = P.ior[P.sel ? P.sel[e] : e];
+        P.cand_counts[cn + m] = c;
+      }
+    }
+    if (tid == 0) {
+      uint32_t* t = P.level_tab + 8 * k;
+      t[0] = M;
+      t[1] = F;
+      t[2] = G;
+      P.status[1] = k;
+    }
+    grid.sync();
+    fw += (uint64_t)F * k;
+    fn += F;
+    if (P.keep) {
+      cw += (uint64_t)M * k;
+      cn += M;
+    }
+    if (F < 2 || k == P.max_k) {
+      ++k;
+      break;
+    }
+    // ---- C_{k+1} from L_k: run starts (same first k-1 items), bounds, hash set
+    const uint32_t w = k;
+    uint32_t* slots = P.slots[k & 1];
+    const uint32_t mask = P.cap_hash - 1;
+    const uint32_t R = grid_scan(
+        [&](uint32_t i) {
+          return (i == 0 || lvl::lex_cmp(Lk + (uint64_t)(i - 1) * w, Lk + (uint64_t)i * w, w - 1) != 0) ? 1u : 0u;
+        },
+        P.run_ex, F, P.bsum, grid);
+    for (uint32_t i = tid; i < F; i += n_threads) {
+      const bool st = i == 0 || lvl::lex_cmp(Lk + (uint64_t)(i - 1) * w, Lk + (uint64_t)i * w, w - 1) != 0;
+      P.rs[i] = st ? 1u : 0u;
+      if (st) P.bound[P.run_ex[i]] = i;
+      uint32_t h = (uint32_t)lvl::hash_mix(lvl::raw_hash(Lk + (uint64_t)i * w, w)) & mask;
+      while (atomicCAS(&slots[h], lvl::kEmpty, i) != lvl::kEmpty) h = (h + 1) & mask;
+    }
+    if (tid == 0) P.bound[R] = F;
+    // the other table (used by generation k - 1) is cleared for generation k + 1
+    uint32_t* other = P.slots[(k + 1) & 1];
+    for (uint32_t i = tid; i < P.cap_hash; i += n_threads) other[i] = lvl::kEmpty;
+    grid.sync();
+    for (uint32_t x = gw; x < F; x += n_warps)
+      lvl::join_warp<false>(x, Lk, w, P.rs, P.run_ex, P.bound, slots, mask, P.cnt, nullptr, nullptr, nullptr, nullptr,
+                            nullptr, nullptr, nullptr);
+    grid.sync();
+    const uint32_t* cntp = P.cnt;
+    const uint32_t M2 = grid_scan([&](uint32_t x) { return cntp[x]; }, P.cand_off, F, P.bsum, grid);
+    const uint32_t G2 = grid_scan([&](uint32_t x) { return cntp[x] ? 1u : 0u; }, P.gidx, F, P.bsum, grid);
+    if (M2 > P.cap_cand || (uint64_t)G2 * w > P.cap_words) {
+      if (tid == 0) P.status[0] |= 1u;
+      break;
+    }
+    for (uint32_t x = gw; x < F; x += n_warps)
+      lvl::join_warp<true>(x, Lk, w, P.rs, P.run_ex, P.bound, slots, mask, P.cnt, P.cand_off, P.gidx, P.prefix,
+                           P.ext_off, P.ext, P.pos, P.counts);   // gpar / eidx land in scratch (pos, counts)
+    if (tid == 0) P.ext_off[G2] = M2;
+    grid.sync();
+    M = M2;
+    G = G2;
+    (void)lane;
+  }
+}
+
+}  // namespace
+}  // namespace gpa
+
+namespace gpa {
+namespace {
+
+// per-thread, per-device persistent workspace of the fused loop (grow-only; sized once)
+struct FusedWork {
+  PBuf<uint32_t> prefix, ext_off, ext, counts, pos, L0, L1, rs, run_ex, bound, cnt, cand_off, gidx, s0, s1, bsum;
+  PBuf<uint32_t> level_tab, status, out_items, out_sup, cand_items, cand_counts;
+  int grid = 0;
+};
+FusedWork& fused_work(int device) {
+  thread_local std::map<int, FusedWork> w;
+  return w[device];
+}
+
+constexpr uint32_t kCapCand = 1u << 20;     // candidates of one generation
+constexpr uint32_t kCapWords = 1u << 24;    // words of an L_k / prefix table
+constexpr uint32_t kCapHash = 1u << 21;     // >= 2 x kCapCand slots
+constexpr uint64_t kCapOut = 1ull << 25;    // words of each output arena
+
+}  // namespace
+
+bool fused_eligible(uint32_t n1, uint64_t pitch_words) {
+  return n1 >= 1 && n1 <= kFusedMaxRows && (uint64_t)n1 * pitch_words * 4 <= kFusedMaxBitsetBytes;
+}
+
+bool mine_fused(const uint32_t* rows, uint64_t pitch_words, uint64_t n_tx, uint32_t n1, const uint32_t* d_sel,
+                const uint32_t* d_ior, uint32_t theta, uint32_t max_k, bool keep, int n_sms, cudaStream_t s,
+                FusedOut& out) {
+  int device = 0;
+  GPA_CUDA(cudaGetDevice(&device));
+  FusedWork& W = fused_work(device);
+  if (!W.grid) {
+    int per_sm = 0;
+    GPA_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, mine_fused_kernel, kFT, 0));
+    GPA_REQUIRE(per_sm > 0, GPA_ERR_CUDA, "mine_fused: kernel does not fit an SM");
+    W.grid = per_sm * n_sms;
+  }
+  FusedParams P{};
+  P.rows = rows;
+  P.pitch = pitch_words;
+  P.W = (uint32_t)((n_tx + 31) / 32);
+  P.n1 = n1;
+  P.sel = d_sel;
+  P.ior = d_ior;
+  P.theta = theta;
+  P.max_k = std::min<uint32_t>(max_k, GPA_MAX_K);
+  P.cap_cand = kCapCand;
+  // GPA_FUSED_TEST_CAP=n: pretend a generation holds at most n candidates (tests drive the overflow
+  // fallback to the multi-kernel path with it)
+  if (const char* e = getenv("GPA_FUSED_TEST_CAP")) P.cap_cand = std::min<uint32_t>(kCapCand, (uint32_t)atoi(e));
+  P.cap_words = kCapWords;
+  P.cap_hash = kCapHash;
+  P.cap_out = kCapOut;
+  P.keep = keep ? 1 : 0;
+  P.prefix = W.prefix.ensure(kCapWords);
+  P.ext_off = W.ext_off.ensure(kCapCand + 1);
+  P.ext = W.ext.ensure(kCapCand);
+  P.counts = W.counts.ensure(kCapCand);
+  P.pos = W.pos.ensure(kCapCand);
+  P.L[0] = W.L0.ensure(kCapWords);
+  P.L[1] = W.L1.ensure(kCapWords);
+  P.rs = W.rs.ensure(kCapCand);
+  P.run_ex = W.run_ex.ensure(kCapCand);
+  P.bound = W.bound.ensure(kCapCand + 1);
+  P.cnt = W.cnt.ensure(kCapCand);
+  P.cand_off = W.cand_off.ensure(kCapCand);
+  P.gidx = W.gidx.ensure(kCapCand);
+  P.slots[0] = W.s0.ensure(kCapHash);
+  P.slots[1] = W.s1.ensure(kCapHash);
+  P.bsum = W.bsum.ensure((size_t)W.grid);
+  P.level_tab = W.level_tab.ensure(8 * (GPA_MAX_K + 2));
+  P.status = W.status.ensure(4);
+  P.out_items = W.out_items.ensure(kCapOut);
+  P.out_sup = W.out_sup.ensure(kCapOut);
+  if (keep) {
+    P.cand_items = W.cand_items.ensure(kCapOut);
+    P.cand_counts = W.cand_counts.ensure(kCapOut);
+  }
+  GPA_CUDA(cudaMemsetAsync(P.status, 0, 16, s));
+  GPA_CUDA(cudaMemsetAsync(P.level_tab, 0, 8 * (GPA_MAX_K + 2) * 4, s));
+  void* args[] = {&P};
+  GPA_CUDA(cudaLaunchCooperativeKernel(reinterpret_cast<const void*>(mine_fused_kernel), W.grid, kFT, args, 0, s));
+  note_launch();
+  // sizes: status + per-generation (M, F, G)
+  std::vector<uint32_t> tab(8 * (GPA_MAX_K + 2)), st(4);
+  GPA_CUDA(cudaMemcpyAsync(st.data(), P.status, 16, cudaMemcpyDeviceToHost, s));
+  GPA_CUDA(cudaMemcpyAsync(tab.data(), P.level_tab, tab.size() * 4, cudaMemcpyDeviceToHost, s));
+  stream_wait(s);
+  if (st[0] & 1u) return false;   // a capacity was exceeded: the caller runs the multi-kernel path
+  out.levels.clear();
+  uint64_t fw = 0, fn = 0, cw = 0, cn = 0;
+  for (uint32_t k = 2; k <= st[1]; ++k) {
+    FusedOut::Level lv;
+    lv.k = k;
+    lv.M = tab[8 * k];
+    lv.F = tab[8 * k + 1];
+    lv.G = tab[8 * k + 2];
+    lv.freq_word = fw;
+    lv.freq_entry = fn;
+    lv.cand_word = cw;
+    lv.cand_entry = cn;
+    fw += (uint64_t)lv.F * k;
+    fn += lv.F;
+    if (keep) {
+      cw += (uint64_t)lv.M * k;
+      cn += lv.M;
+    }
+    out.levels.push_back(lv);
+  }
+  out.items.resize(fw);
+  out.sup.resize(fn);
+  out.cand_items.resize(cw);
+  out.cand_counts.resize(cn);
+  if (fw) GPA_CUDA(cudaMemcpyAsync(out.items.data(), P.out_items, fw * 4, cudaMemcpyDeviceToHost, s));
+  if (fn) GPA_CUDA(cudaMemcpyAsync(out.sup.data(), P.out_sup, fn * 4, cudaMemcpyDeviceToHost, s));
+  if (cw) GPA_CUDA(cudaMemcpyAsync(out.cand_items.data(), P.cand_items, cw * 4, cudaMemcpyDeviceToHost, s));
+  if (cn) GPA_CUDA(cudaMemcpyAsync(out.cand_counts.data(), P.cand_counts, cn * 4, cudaMemcpyDeviceToHost, s));
+  stream_wait(s);
+  return true;
+}
+
+}  // namespace gpa

@@ -45,10 +45,11 @@ float event_ms(cudaEvent_t a, cudaEvent_t b) {
 }
 
 void validate_options(const gpa_options& o) {
-  GPA_REQUIRE(o.count_kernel <= GPA_KERNEL_PROJ, GPA_ERR_INVALID, "unknown count_kernel %u", o.count_kernel);
+  GPA_REQUIRE(o.count_kernel <= GPA_KERNEL_FUSED, GPA_ERR_INVALID, "unknown count_kernel %u", o.count_kernel);
   GPA_REQUIRE(o.max_k <= GPA_MAX_K, GPA_ERR_INVALID, "max_k %u > GPA_MAX_K", o.max_k);
   GPA_REQUIRE(!o.reserved[0] && !o.reserved[1] && !o.reserved[2], GPA_ERR_INVALID, "reserved option fields must be 0");
-  GPA_REQUIRE((o.flags & ~(GPA_KEEP_CANDIDATES | GPA_HOST_CANDGEN | GPA_NO_OVERLAP_INGEST | GPA_COMPLETE_INTERSECTION)) == 0,
+  GPA_REQUIRE((o.flags & ~(GPA_KEEP_CANDIDATES | GPA_HOST_CANDGEN | GPA_NO_OVERLAP_INGEST | GPA_COMPLETE_INTERSECTION |
+                           GPA_MULTI_KERNEL)) == 0,
               GPA_ERR_INVALID, "unknown option flags 0x%x", o.flags);
 }
 
@@ -326,7 +327,7 @@ bool count_device_batch(gpa_bitset* bs, DeviceBatch& B, uint32_t kernel, DeviceS
   cudaStream_t s = bs->stream;
   const uint32_t k = B.k, M = B.M, G = B.G;
   if (M == 0) return true;
-  if (kernel == GPA_KERNEL_PROJ) kernel = GPA_KERNEL_AUTO;
+  if (kernel == GPA_KERNEL_PROJ || kernel == GPA_KERNEL_FUSED) kernel = GPA_KERNEL_AUTO;
   if (kernel == GPA_KERNEL_V0 || bs->n_rows > kPlanMaxRows || k < 2) return false;
   if (kernel == GPA_KERNEL_AUTO || kernel == GPA_KERNEL_PAIRS || kernel == GPA_KERNEL_PAIRS_TC) {
     const double sib = (double)M / (double)std::max<uint32_t>(G, 1);
@@ -415,7 +416,7 @@ void count_grouped(gpa_bitset* bs, const GroupedBatch& b, uint32_t kernel, Count
   const uint64_t M = b.size(), G = b.groups();
   const uint32_t km1 = b.k - 1;
   if (M == 0) return;
-  if (kernel == GPA_KERNEL_PROJ) kernel = GPA_KERNEL_AUTO;
+  if (kernel == GPA_KERNEL_PROJ || kernel == GPA_KERNEL_FUSED) kernel = GPA_KERNEL_AUTO;
   if (kernel == GPA_KERNEL_AUTO || kernel == GPA_KERNEL_PAIRS || kernel == GPA_KERNEL_PAIRS_TC) {
     // grouped batches: large sibling groups amortise the (k-1)-row prefix well in the streaming
     // prefix kernel (measured: T40I10D10M k = 3, 4.6 siblings / group); small groups (deep
@@ -477,7 +478,7 @@ void count_all_pairs(gpa_bitset* bs, uint32_t kernel, CountStats* st) {
   const uint64_t M = n * (n - 1) / 2;
   if (n < 2) return;
   const bool sub = bs->l1_sub;   // L_1 is a subset of the rows
-  if (kernel == GPA_KERNEL_AUTO || kernel == GPA_KERNEL_PROJ) kernel = GPA_KERNEL_PAIRS_TC;
+  if (kernel == GPA_KERNEL_AUTO || kernel == GPA_KERNEL_PROJ || kernel == GPA_KERNEL_FUSED) kernel = GPA_KERNEL_PAIRS_TC;
   if (kernel != GPA_KERNEL_PAIRS && kernel != GPA_KERNEL_PAIRS_TC) {
     GroupedBatch b;
     b.k = 2;
@@ -591,7 +592,7 @@ extern "C" gpa_status gpa_count(gpa_bitset* bs, const uint32_t* cand, uint32_t k
   return gpa::guard([&] {
     GPA_REQUIRE(bs, GPA_ERR_INVALID, "bitset is NULL");
     GPA_REQUIRE(k >= 1 && k <= GPA_MAX_K, GPA_ERR_INVALID, "k must be in [1, %u]", GPA_MAX_K);
-    GPA_REQUIRE(kernel <= GPA_KERNEL_PROJ, GPA_ERR_INVALID, "unknown kernel %u", kernel);
+    GPA_REQUIRE(kernel <= GPA_KERNEL_FUSED, GPA_ERR_INVALID, "unknown kernel %u", kernel);
     if (M == 0) return;
     GPA_REQUIRE(cand && counts_out, GPA_ERR_INVALID, "NULL argument");
     GPA_REQUIRE(M <= (UINT64_MAX / 8) / k && M < (1ull << 32), GPA_ERR_INVALID, "M * k overflows");
@@ -625,7 +626,7 @@ extern "C" gpa_status gpa_count(gpa_bitset* bs, const uint32_t* cand, uint32_t k
       gpa::fail((gpa_status)verdict[0], "invalid candidates on another rank");
     }
     uint32_t kern = kernel == GPA_KERNEL_AUTO ? bs->opt.count_kernel : kernel;
-    if (kern == GPA_KERNEL_PROJ) kern = GPA_KERNEL_AUTO;  // needs the level structure of gpa_mine
+    if (kern == GPA_KERNEL_PROJ || kern == GPA_KERNEL_FUSED) kern = GPA_KERNEL_AUTO;  // gpa_mine's level structure
     if (k == 1) kern = GPA_KERNEL_V0;
     if (kern == GPA_KERNEL_AUTO)
       kern = (k == 2 && (double)M * 8 >= (double)bs->n_rows * bs->n_rows) ? GPA_KERNEL_PAIRS_TC

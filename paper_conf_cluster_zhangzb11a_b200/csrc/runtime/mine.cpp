@@ -174,6 +174,7 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
   if (opt_in) opt = *opt_in;
   GPA_REQUIRE(min_count >= 1, GPA_ERR_INVALID, "min_count must be >= 1");
   const bool keep = (opt.flags & GPA_KEEP_CANDIDATES) != 0;
+  const bool fused_requested = opt.count_kernel == GPA_KERNEL_FUSED;
   pinned_arena().reset();  // a previous call on this thread consumed its blocks before returning
   const bool host_candgen = (opt.flags & GPA_HOST_CANDGEN) != 0;
   const uint32_t max_k = opt.max_k ? opt.max_k : GPA_MAX_K;
@@ -239,6 +240,7 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
   DeviceProj* plists = proj_lists(bs->device);
   DeviceProj* Pprev = &plists[0];
   DeviceProj* Pcur = &plists[1];
+  if (opt.count_kernel == GPA_KERNEL_FUSED) opt.count_kernel = GPA_KERNEL_AUTO;   // (the multi-kernel fallback)
   bool proj_on = !host_candgen && (opt.count_kernel == GPA_KERNEL_AUTO || opt.count_kernel == GPA_KERNEL_PROJ ||
                                    opt.count_kernel == GPA_KERNEL_PAIRS || opt.count_kernel == GPA_KERNEL_PAIRS_TC) &&
                  bs->pitch_words * 32ull < (1ull << 32);
@@ -328,6 +330,51 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
   if (bs->l1_sub && !bs->l1.empty() && bs->d_l1.n < bs->l1.size()) {   // L_1 -> bitset rows (generation 2)
     bs->d_l1.alloc(bs->l1.size(), s);
     GPA_CUDA(cudaMemcpyAsync(bs->d_l1.p, bs->l1.data(), bs->l1.size() * 4, cudaMemcpyHostToDevice, s));
+  }
+  // ---- small problems: every generation in one cooperative launch (mine_fused.cu); a capacity
+  // overflow falls through to the multi-kernel loop below
+  const bool want_fused = !dist && !host_candgen && !(opt.flags & GPA_MULTI_KERNEL) && nL >= 2 &&
+                          (fused_requested || opt.count_kernel == GPA_KERNEL_AUTO) &&
+                          fused_eligible((uint32_t)nL, bs->pitch_words);
+  if (want_fused) {
+    FusedOut fo;
+    EvTriple& ev = events.emplace_back();
+    GPA_CUDA(cudaEventRecord(ev.e[5], s));
+    GPA_CUDA(cudaEventRecord(ev.e[0], s));
+    const bool ok = mine_fused(bs->rows.p, bs->pitch_words, bs->n_tx_local, (uint32_t)nL,
+                               bs->l1_sub ? bs->d_l1.p : nullptr, d_ior.p, (uint32_t)min_count, max_k, keep,
+                               bs->n_sms, s, fo);
+    GPA_CUDA(cudaEventRecord(ev.e[1], s));
+    GPA_CUDA(cudaEventRecord(ev.e[2], s));
+    GPA_CUDA(cudaEventRecord(ev.e[6], s));
+    if (ok) {
+      ev.counted = true;
+      for (const auto& f : fo.levels) {
+        gpa_level_data lv;
+        lv.k = f.k;
+        lv.n_cand = f.M;
+        lv.n_freq = f.F;
+        lv.n_groups = f.G;
+        lv.kept = keep;
+        lv.freq_items.assign(fo.items.begin() + f.freq_word, fo.items.begin() + f.freq_word + (uint64_t)f.F * f.k);
+        lv.freq_support.assign(fo.sup.begin() + f.freq_entry, fo.sup.begin() + f.freq_entry + f.F);
+        if (keep) {
+          lv.cand_items.assign(fo.cand_items.begin() + f.cand_word,
+                               fo.cand_items.begin() + f.cand_word + (uint64_t)f.M * f.k);
+          lv.cand_counts.assign(fo.cand_counts.begin() + f.cand_entry, fo.cand_counts.begin() + f.cand_entry + f.M);
+        }
+        lv.stats.n_cand = f.M;
+        lv.stats.n_freq = f.F;
+        lv.stats.n_groups = f.G;
+        lv.stats.kernel = GPA_KERNEL_FUSED;
+        lv.stats.launches = R->levels.size() == 1 ? 1 : 0;   // one launch for all generations
+        R->levels.push_back(std::move(lv));
+      }
+      if (R->levels.size() > 1) event_level.push_back(1);   // the whole loop's time on generation 2
+      nL = 0;   // skip the multi-kernel loop
+    } else {
+      events.pop_back();
+    }
   }
   for (uint32_t k = 2; k <= max_k && nL > 0; ++k) {
     double t0 = now_ms();

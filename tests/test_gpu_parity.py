@@ -515,6 +515,55 @@ def test_proj_k3_set_bit_walk_pext(name):
     assert max(len(s) for s in got) >= 4
 
 
+@pytest.mark.parametrize("name", ["chess", "mushroom", "accidents", "fig2", "dense", "random"])
+def test_fused_single_launch_equals_oracle(fig2, name):
+    """GPA_KERNEL_FUSED (the whole level loop in one cooperative launch: complete-intersection
+    counting, threshold, join + prune as grid-wide phases) against the oracle on every (C_k, count)
+    and F, and against the multi-kernel path; exactly one library launch for all generations."""
+    if name == "fig2":
+        ds, theta = gen.from_lists(fig2[0], 8), 2
+    elif name == "dense":
+        ds, theta = gen.random_db(42, 6000, 44, max_len=24, p_empty=0.02), 500
+    elif name == "random":
+        ds, theta = gen.random_db(5, 2500, 28, max_len=12, duplicates=True, unsorted=True), 40
+    else:
+        ds = gen.make(name)
+        theta = oracle.min_count(ds.n_tx, gen.CONFIGS[name].minsup)
+    ref = oracle.mine_ds(ds, theta)
+    l0 = gpa.kernel_launches()
+    res = gpa.mine(ds, min_count=theta, options=gpa.Options(count_kernel=gpa.KERNEL_FUSED), keep_candidates=True)
+    assert_mine_equal(res, ref)
+    assert all(lv.stats["kernel_name"] == "fused" for lv in res.levels[1:])
+    multi = gpa.mine(ds, min_count=theta, options=gpa.Options(multi_kernel=True), keep_candidates=True)
+    assert_mine_equal(multi, ref)
+    assert all(lv.stats["kernel_name"] != "fused" for lv in multi.levels[1:])
+    # default options pick the fused path for these small problems
+    l1 = gpa.kernel_launches()
+    auto = gpa.mine(ds, min_count=theta, options=gpa.Options(overlap_ingest=False))
+    assert auto.frequent() == ref.frequent()
+    assert all(lv.stats["kernel_name"] == "fused" for lv in auto.levels[1:])
+    assert gpa.kernel_launches() - l1 <= 4   # one-pass build (+ row compaction) + the fused loop
+
+
+def test_fused_capacity_overflow_falls_back(monkeypatch):
+    """A generation larger than the fused path's capacity (forced with GPA_FUSED_TEST_CAP) reruns on the
+    multi-kernel path: every (C_k, count) unchanged."""
+    import json
+    import subprocess
+    import sys
+    code = ("import json, gen, oracle, paper_conf_cluster_zhangzb11a_b200 as gpa\n"
+            "ds = gen.make('mushroom'); th = oracle.min_count(ds.n_tx, '0.20')\n"
+            "r = gpa.mine(ds, min_count=th, keep_candidates=True)\n"
+            "ref = oracle.mine_ds(ds, th)\n"
+            "ok = all((lv.cand == rl.cand).all() and (lv.counts == rl.count).all() for lv, rl in zip(r.levels, ref.levels))\n"
+            "print(json.dumps([bool(ok and len(r.levels) == len(ref.levels)), sorted({lv.stats['kernel_name'] for lv in r.levels[1:]})]))\n")
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    out = subprocess.run([sys.executable, "-c", code], cwd=root, env=dict(os.environ, GPA_FUSED_TEST_CAP="100"),
+                         capture_output=True, text=True, check=True, timeout=600).stdout
+    ok, kinds = json.loads(out.strip().splitlines()[-1])
+    assert ok and "fused" not in kinds, kinds
+
+
 def test_complete_intersection_flag():
     """GPA_COMPLETE_INTERSECTION: k >= 3 by the paper's complete intersection (trie / prefix over the
     static bitset), k = 2 on the CUDA-core pair Gram with count_kernel PAIRS -- the north-star path
