@@ -37,42 +37,49 @@ namespace cg = cooperative_groups;
 namespace gpa {
 namespace {
 
-constexpr int kFT = 256;                 // threads per CTA
+constexpr int kFT = 512;                 // threads per CTA (one CTA per SM: cheap grid syncs)
 constexpr uint32_t kWarps = kFT / 32;
 
-// --- grid-wide exclusive scan of get(i), i < n -> out[i]; returns the total on every thread.
+template <class T>
+__device__ __forceinline__ T warp_sum(T v) {
+#pragma unroll
+  for (uint32_t d = 16; d >= 1; d >>= 1) v += __shfl_xor_sync(0xffffffffu, v, d);
+  return v;
+}
+
+// --- grid-wide exclusive scan of get(i), i < n -> put(i, prefix); returns the total on every thread.
 // Two grid syncs: block sums, then (after every CTA read them) the next user may reuse bsum.
-template <class F>
-__device__ uint32_t grid_scan(F get, uint32_t* out, uint32_t n, uint32_t* bsum, cg::grid_group& grid) {
-  __shared__ uint32_t sh[kWarps + 1];
+template <class T, class F, class Put>
+__device__ T grid_scan(F get, Put put, uint32_t n, T* bsum, cg::grid_group& grid) {
+  __shared__ T sh[kWarps + 1];
   const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const uint32_t per = ((n + gridDim.x - 1) / gridDim.x + kFT - 1) / kFT * kFT;
   const uint32_t b0 = min(n, blockIdx.x * per), b1 = min(n, b0 + per);
-  uint32_t s = 0;
+  T s = 0;
   for (uint32_t i = b0 + threadIdx.x; i < b1; i += kFT) s += get(i);
-  s = __reduce_add_sync(0xffffffffu, s);
+  s = warp_sum(s);
   if (lane == 0) sh[warp] = s;
   __syncthreads();
   if (threadIdx.x == 0) {
-    uint32_t t = 0;
+    T t = 0;
     for (uint32_t w = 0; w < kWarps; ++w) t += sh[w];
     bsum[blockIdx.x] = t;
   }
   __syncthreads();
   grid.sync();
-  uint32_t off = 0, tot = 0;
+  T off = 0, tot = 0;
   for (uint32_t b = threadIdx.x; b < gridDim.x; b += kFT) {
-    const uint32_t v = bsum[b];
+    const T v = bsum[b];
     tot += v;
     if (b < blockIdx.x) off += v;
   }
-  off = __reduce_add_sync(0xffffffffu, off);
-  tot = __reduce_add_sync(0xffffffffu, tot);
+  off = warp_sum(off);
+  tot = warp_sum(tot);
   __syncthreads();
   if (lane == 0) sh[warp] = off;
   __syncthreads();
   if (threadIdx.x == 0) {
-    uint32_t a = 0;
+    T a = 0;
     for (uint32_t w = 0; w < kWarps; ++w) a += sh[w];
     sh[kWarps] = a;
   }
@@ -82,7 +89,7 @@ __device__ uint32_t grid_scan(F get, uint32_t* out, uint32_t n, uint32_t* bsum, 
   if (lane == 0) sh[warp] = tot;
   __syncthreads();
   if (threadIdx.x == 0) {
-    uint32_t a = 0;
+    T a = 0;
     for (uint32_t w = 0; w < kWarps; ++w) a += sh[w];
     sh[kWarps] = a;
   }
@@ -92,22 +99,22 @@ __device__ uint32_t grid_scan(F get, uint32_t* out, uint32_t n, uint32_t* bsum, 
   // block-level scan of the CTA's range in chunks of kFT, offset by the earlier CTAs' sums
   for (uint32_t base = b0; base < b1; base += kFT) {
     const uint32_t i = base + threadIdx.x;
-    const uint32_t v = i < b1 ? get(i) : 0u;
-    uint32_t x = v;
+    const T v = i < b1 ? get(i) : T(0);
+    T x = v;
 #pragma unroll
     for (uint32_t d = 1; d < 32; d <<= 1) {
-      const uint32_t y = __shfl_up_sync(0xffffffffu, x, d);
+      const T y = __shfl_up_sync(0xffffffffu, x, d);
       if (lane >= d) x += y;
     }
     if (lane == 31) sh[warp] = x;
     __syncthreads();
-    uint32_t woff = 0, ctot = 0;
+    T woff = 0, ctot = 0;
     for (uint32_t w = 0; w < kWarps; ++w) {
-      const uint32_t t = sh[w];
+      const T t = sh[w];
       if (w < warp) woff += t;
       ctot += t;
     }
-    if (i < b1) out[i] = off + woff + x - v;
+    if (i < b1) put(i, off + woff + x - v);
     off += ctot;
     __syncthreads();
   }
@@ -134,7 +141,11 @@ struct FusedParams {
   // levels: L rows (ping-pong), join scratch
   uint32_t *L[2];
   uint32_t *rs, *run_ex, *bound, *cnt, *cand_off, *gidx, *slots[2];
-  uint32_t* bsum;
+  uint32_t* bsum;            // grid_scan block sums (u32)
+  uint64_t* bsum64;          // (u64)
+  uint32_t* sink;            // join outputs nobody reads here (the group's left parent, the right parent)
+  uint64_t* state;           // GenState handed from CTA 0 to the grid after a single-CTA generation
+  uint32_t zsplit;           // word slices per group in the counting phase (>= 1)
   // outputs: per generation k (index k): {M_k, F_k, G_k, freq arena offset (lo, hi), cand arena offset (lo, hi)}
   uint32_t* level_tab;       // 8 words per generation, GPA_MAX_K + 1 generations
   uint32_t *out_items, *out_sup, *cand_items, *cand_counts;
@@ -145,171 +156,263 @@ __device__ __forceinline__ const uint32_t* row_ptr(const FusedParams& P, uint32_
   return P.rows + (uint64_t)(P.sel ? P.sel[r] : r) * P.pitch;
 }
 
-// counts[m] for the grouped batch (G groups, prefix width km1) -- warp per (group, batch of <= 32
-// extensions), lanes over 32-word chunks of the rows
-__device__ void count_phase(const FusedParams& P, uint32_t G, uint32_t km1) {
-  const uint32_t lane = threadIdx.x & 31;
-  const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, n_warps = (gridDim.x * blockDim.x) >> 5;
-  // work items: (group, batch); batches per group = ceil(n_ext / 32); enumerate groups, then batches
-  for (uint32_t g = gw; g < G; g += n_warps) {
+// ---- teams: the whole grid (grid.sync, grid-wide scans) or CTA 0 alone (__syncthreads, block
+// scans) for generations too small to amortise grid-wide synchronisation
+struct GridTeam {
+  cg::grid_group& grid;
+  __device__ uint32_t tid() const { return blockIdx.x * blockDim.x + threadIdx.x; }
+  __device__ uint32_t nthreads() const { return gridDim.x * blockDim.x; }
+  __device__ void sync() const { grid.sync(); }
+  template <class T, class F, class Put>
+  __device__ T scan(F get, Put put, uint32_t n, T* bsum) const { return grid_scan<T>(get, put, n, bsum, grid); }
+};
+struct BlockTeam {
+  __device__ uint32_t tid() const { return threadIdx.x; }
+  __device__ uint32_t nthreads() const { return blockDim.x; }
+  __device__ void sync() const { __syncthreads(); }
+  template <class T, class F, class Put>
+  __device__ T scan(F get, Put put, uint32_t n, T*) const {   // exclusive, one CTA
+    __shared__ T sh[kWarps];
+    const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    T off = 0;
+    for (uint32_t base = 0; base < n; base += kFT) {
+      const uint32_t i = base + threadIdx.x;
+      const T v = i < n ? get(i) : T(0);
+      T x = v;
+#pragma unroll
+      for (uint32_t d = 1; d < 32; d <<= 1) {
+        const T y = __shfl_up_sync(0xffffffffu, x, d);
+        if (lane >= d) x += y;
+      }
+      if (lane == 31) sh[warp] = x;
+      __syncthreads();
+      T woff = 0, ctot = 0;
+      for (uint32_t w = 0; w < kWarps; ++w) {
+        const T t = sh[w];
+        if (w < warp) woff += t;
+        ctot += t;
+      }
+      if (i < n) put(i, off + woff + x - v);
+      off += ctot;
+      __syncthreads();
+    }
+    return off;
+  }
+};
+
+// counts[m] += popcount over a word slice -- warp per (group, slice of the words): per 32-word
+// chunk (lane = word) the prefix AND, then one AND + POPC per extension, warp-reduced (redux.sync)
+// into the extension's count; prefix rows' offsets staged in shared memory.  counts must be zero
+// (atomic adds when the words are split into slices).
+template <class Team>
+__device__ void count_phase(const Team& T, const FusedParams& P, uint32_t G, uint32_t km1, uint32_t Z) {
+  __shared__ uint64_t s_pre[kWarps][64];
+  const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  const uint32_t gw = T.tid() >> 5, n_warps = T.nthreads() >> 5;
+  const uint32_t n_chunks = (P.W + 31) / 32;
+  const uint32_t per = (n_chunks + Z - 1) / Z;
+  for (uint32_t it = gw; it < G * Z; it += n_warps) {
+    const uint32_t g = it / Z, z = it % Z;
+    const uint32_t c0 = z * per, c1 = min(n_chunks, c0 + per);
     const uint32_t e0 = P.ext_off[g], e1 = P.ext_off[g + 1];
     const uint32_t* pr = P.prefix + (uint64_t)g * km1;
+    for (uint32_t d = lane; d < km1; d += 32) s_pre[wib][d] = (uint64_t)(P.sel ? P.sel[pr[d]] : pr[d]) * P.pitch;
+    __syncwarp();
     for (uint32_t b0 = e0; b0 < e1; b0 += 32) {
       const uint32_t nb = min(32u, e1 - b0);
-      // lane j: the row of extension j (word offset)
       const uint64_t my_row = lane < nb ? (uint64_t)(P.sel ? P.sel[P.ext[b0 + lane]] : P.ext[b0 + lane]) * P.pitch : 0;
-      uint32_t acc[32];
-#pragma unroll
-      for (int j = 0; j < 32; ++j) acc[j] = 0;
-      for (uint32_t base = 0; base < P.W; base += 32) {   // lane = word of the chunk
-        const uint32_t w = base + lane;
+      uint32_t mine = 0;   // lane j: the count of extension j over this slice
+      for (uint32_t c = c0; c < c1; ++c) {
+        const uint32_t w = 32 * c + lane;
         const bool in = w < P.W;
         uint32_t pw = in ? 0xffffffffu : 0u;
-        for (uint32_t d = 0; d < km1; ++d) pw &= in ? __ldg(row_ptr(P, pr[d]) + w) : 0u;
-#pragma unroll
-        for (int j = 0; j < 32; ++j) {
-          if (j < (int)nb) {
-            const uint64_t ro = __shfl_sync(0xffffffffu, my_row, j);
-            acc[j] += __popc(pw & (in ? __ldg(P.rows + ro + w) : 0u));
-          }
+        for (uint32_t d = 0; d < km1; ++d) pw &= in ? __ldg(P.rows + s_pre[wib][d] + w) : 0u;
+        for (uint32_t j = 0; j < nb; ++j) {
+          const uint64_t ro = __shfl_sync(0xffffffffu, my_row, j);
+          const uint32_t t = __reduce_add_sync(0xffffffffu, (uint32_t)__popc(pw & (in ? __ldg(P.rows + ro + w) : 0u)));
+          mine += lane == j ? t : 0u;
         }
       }
-#pragma unroll
-      for (int j = 0; j < 32; ++j) {
-        if (j < (int)nb) {
-          const uint32_t t = __reduce_add_sync(0xffffffffu, acc[j]);
-          if (lane == j) P.counts[b0 + j] = t;
-        }
+      if (lane < nb && mine) {
+        if (Z == 1) P.counts[b0 + lane] = mine;
+        else atomicAdd(&P.counts[b0 + lane], mine);
       }
     }
+    __syncwarp();
   }
 }
+
+struct GenState {
+  uint32_t k, M, G;
+  uint64_t fw, fn, cw, cn;   // output arenas: words / entries so far (frequent, candidates)
+  uint32_t done;             // 0: next generation; 1: finished; 2: overflow
+};
+
+// One generation by a team: count C_k, threshold into L_k (+ outputs), join + prune into C_{k+1}.
+// Every team thread returns the same state.
+template <class Team>
+__device__ GenState generation(const Team& T, const FusedParams& P, GenState S) {
+  const uint32_t tid = T.tid(), n_threads = T.nthreads();
+  const uint32_t gw = tid >> 5, n_warps = n_threads >> 5;
+  const uint32_t k = S.k, km1 = k - 1, M = S.M, G = S.G;
+  // ---- count C_k: enough (group, word slice) items to occupy every warp
+  const uint32_t n_chunks = (P.W + 31) / 32;
+  uint32_t Z = G ? (4 * n_warps + G - 1) / G : 1;
+  Z = max(1u, min(Z, (n_chunks + 7) / 8));   // >= 8 chunks of 32 words per slice
+  count_phase(T, P, G, km1, Z);
+  T.sync();
+  // ---- threshold: L_k in candidate (lexicographic) order
+  const uint32_t theta = P.theta;
+  const uint32_t* counts = P.counts;
+  uint32_t* posp = P.pos;
+  const uint32_t F = T.template scan<uint32_t>([&](uint32_t m) { return counts[m] >= theta ? 1u : 0u; },
+                                              [&](uint32_t i, uint32_t v) { posp[i] = v; }, M, P.bsum);
+  T.sync();
+  uint32_t* Lk = P.L[k & 1];
+  if ((uint64_t)F * k > P.cap_words || S.fw + (uint64_t)F * k > P.cap_out ||
+      (P.keep && S.cw + (uint64_t)M * k > P.cap_out)) {
+    S.done = 2;
+    return S;
+  }
+  for (uint32_t m = tid; m < M; m += n_threads) {
+    const uint32_t c = counts[m];
+    const bool freq = c >= theta;
+    if (!freq && !P.keep) continue;
+    uint32_t lo = 0, hi = G;   // g = last group with ext_off[g] <= m
+    while (lo + 1 < hi) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if (P.ext_off[mid] <= m) lo = mid; else hi = mid;
+    }
+    const uint32_t* pr = P.prefix + (uint64_t)lo * km1;
+    const uint32_t e = P.ext[m];
+    if (freq) {
+      const uint32_t p = posp[m];
+      uint32_t* dst = Lk + (uint64_t)p * k;
+      uint32_t* od = P.out_items + S.fw + (uint64_t)p * k;
+      for (uint32_t d = 0; d < km1; ++d) {
+        dst[d] = pr[d];
+        od[d] = P.ior[P.sel ? P.sel[pr[d]] : pr[d]];
+      }
+      dst[km1] = e;
+      od[km1] = P.ior[P.sel ? P.sel[e] : e];
+      P.out_sup[S.fn + p] = c;
+    }
+    if (P.keep) {
+      uint32_t* cd = P.cand_items + S.cw + (uint64_t)m * k;
+      for (uint32_t d = 0; d < km1; ++d) cd[d] = P.ior[P.sel ? P.sel[pr[d]] : pr[d]];
+      cd[km1] = P.ior[P.sel ? P.sel[e] : e];
+      P.cand_counts[S.cn + m] = c;
+    }
+  }
+  if (tid == 0) {
+    uint32_t* t = P.level_tab + 8 * k;
+    t[0] = M;
+    t[1] = F;
+    t[2] = G;
+    P.status[1] = k;
+  }
+  S.fw += (uint64_t)F * k;
+  S.fn += F;
+  if (P.keep) {
+    S.cw += (uint64_t)M * k;
+    S.cn += M;
+  }
+  if (F < 2 || k == P.max_k) {
+    S.done = 1;
+    return S;
+  }
+  T.sync();
+  // ---- C_{k+1} from L_k: run starts (same first k-1 items), bounds, hash set
+  const uint32_t w = k;
+  uint32_t* slots = P.slots[k & 1];
+  const uint32_t mask = P.cap_hash - 1;
+  uint32_t* rexp = P.run_ex;
+  const uint32_t R = T.template scan<uint32_t>(
+      [&](uint32_t i) {
+        return (i == 0 || lvl::lex_cmp(Lk + (uint64_t)(i - 1) * w, Lk + (uint64_t)i * w, w - 1) != 0) ? 1u : 0u;
+      },
+      [&](uint32_t i, uint32_t v) { rexp[i] = v; }, F, P.bsum);
+  T.sync();
+  for (uint32_t i = tid; i < F; i += n_threads) {
+    const bool st = i == 0 || lvl::lex_cmp(Lk + (uint64_t)(i - 1) * w, Lk + (uint64_t)i * w, w - 1) != 0;
+    P.rs[i] = st ? 1u : 0u;
+    if (st) P.bound[rexp[i]] = i;
+    uint32_t h = (uint32_t)lvl::hash_mix(lvl::raw_hash(Lk + (uint64_t)i * w, w)) & mask;
+    while (atomicCAS(&slots[h], lvl::kEmpty, i) != lvl::kEmpty) h = (h + 1) & mask;
+  }
+  if (tid == 0) P.bound[R] = F;
+  // the other table (used by generation k - 1) is cleared for generation k + 1
+  uint32_t* other = P.slots[(k + 1) & 1];
+  for (uint32_t i = tid; i < P.cap_hash; i += n_threads) other[i] = lvl::kEmpty;
+  T.sync();
+  for (uint32_t x = gw; x < F; x += n_warps)
+    lvl::join_warp<false>(x, Lk, w, P.rs, P.run_ex, P.bound, slots, mask, P.cnt, nullptr, nullptr, nullptr, nullptr,
+                          nullptr, nullptr, nullptr);
+  T.sync();
+  // survivors and non-empty groups in ONE scan: (count << 32) | (count != 0)
+  const uint32_t* cntp = P.cnt;
+  uint32_t *cop = P.cand_off, *gip = P.gidx;
+  const uint64_t MG = T.template scan<uint64_t>(
+      [&](uint32_t x) { return ((uint64_t)cntp[x] << 32) | (cntp[x] ? 1ull : 0ull); },
+      [&](uint32_t i, uint64_t v) {
+        cop[i] = (uint32_t)(v >> 32);
+        gip[i] = (uint32_t)v;
+      },
+      F, P.bsum64);
+  T.sync();
+  const uint32_t M2 = (uint32_t)(MG >> 32), G2 = (uint32_t)MG;
+  if (M2 > P.cap_cand || (uint64_t)G2 * w > P.cap_words) {
+    S.done = 2;
+    return S;
+  }
+  for (uint32_t x = gw; x < F; x += n_warps)
+    lvl::join_warp<true>(x, Lk, w, P.rs, P.run_ex, P.bound, slots, mask, P.cnt, P.cand_off, P.gidx, P.prefix,
+                         P.ext_off, P.ext, P.sink, P.sink + P.cap_cand);   // parents: unused here
+  if (tid == 0) P.ext_off[G2] = M2;
+  for (uint32_t i = tid; i < M2; i += n_threads) P.counts[i] = 0;
+  S.k = k + 1;
+  S.M = M2;
+  S.G = G2;
+  S.done = M2 ? 0 : 1;
+  return S;
+}
+
+// a generation is run by CTA 0 alone below this many word operations (M x words x k)
+constexpr uint64_t kSmallGenWork = 4ull << 20;
 
 __global__ void __launch_bounds__(kFT) mine_fused_kernel(FusedParams P) {
   cg::grid_group grid = cg::this_grid();
   const uint32_t tid = blockIdx.x * blockDim.x + threadIdx.x, n_threads = gridDim.x * blockDim.x;
-  const uint32_t gw = tid >> 5, n_warps = n_threads >> 5;
-  const uint32_t lane = threadIdx.x & 31;
   // ---- C_2 = every pair of L_1 entries, grouped by the first: group a = {a} x (a, n1)
   const uint32_t n1 = P.n1;
-  uint32_t G = n1 > 1 ? n1 - 1 : 0;
-  uint32_t M = n1 > 1 ? n1 * (n1 - 1) / 2 : 0;
-  for (uint32_t a = tid; a < G; a += n_threads) {
+  GenState S{2, n1 > 1 ? n1 * (n1 - 1) / 2 : 0, n1 > 1 ? n1 - 1 : 0, 0, 0, 0, 0, 0};
+  for (uint32_t a = tid; a < S.G; a += n_threads) {
     P.prefix[a] = a;
     const uint32_t off = a * n1 - a * (a + 1) / 2;   // pair_index(a, a + 1, n1)
     P.ext_off[a] = off;
     for (uint32_t b = a + 1; b < n1; ++b) P.ext[off + (b - a - 1)] = b;
   }
-  if (tid == 0) P.ext_off[G] = M;
+  if (tid == 0) P.ext_off[S.G] = S.M;
+  for (uint32_t i = tid; i < S.M; i += n_threads) P.counts[i] = 0;
   for (uint32_t i = tid; i < P.cap_hash; i += n_threads) P.slots[0][i] = P.slots[1][i] = lvl::kEmpty;
-  uint64_t fw = 0, fn = 0, cw = 0, cn = 0;   // output arenas: words / entries so far (frequent, candidates)
-  uint32_t k = 2;
   grid.sync();
-  for (; k <= P.max_k && M > 0; ++k) {
-    const uint32_t km1 = k - 1;
-    // ---- count C_k
-    count_phase(P, G, km1);
-    grid.sync();
-    // ---- threshold: L_k in candidate (lexicographic) order
-    const uint32_t theta = P.theta;
-    const uint32_t* counts = P.counts;
-    const uint32_t F = grid_scan([&](uint32_t m) { return counts[m] >= theta ? 1u : 0u; }, P.pos, M, P.bsum, grid);
-    uint32_t* Lk = P.L[k & 1];
-    const bool fit = (uint64_t)F * k <= P.cap_words && fw + (uint64_t)F * k <= P.cap_out &&
-                     (!P.keep || cw + (uint64_t)M * k <= P.cap_out);
-    if (!fit) {
-      if (tid == 0) P.status[0] |= 1u;
-      break;   // uniform: every thread computed the same F
-    }
-    for (uint32_t m = tid; m < M; m += n_threads) {
-      const uint32_t c = counts[m];
-      const bool freq = c >= theta;
-      if (!freq && !P.keep) continue;
-      uint32_t lo = 0, hi = G;   // g = last group with ext_off[g] <= m
-      while (lo + 1 < hi) {
-        const uint32_t mid = (lo + hi) >> 1;
-        if (P.ext_off[mid] <= m) lo = mid; else hi = mid;
+  GridTeam GT{grid};
+  while (S.k <= P.max_k && S.M > 0 && S.done == 0) {
+    if ((uint64_t)S.M * P.W * S.k < kSmallGenWork) {
+      // CTA 0 runs the generation; everyone picks its state up after one grid-wide barrier
+      if (blockIdx.x == 0) {
+        const GenState N = generation(BlockTeam{}, P, S);
+        if (threadIdx.x == 0) *reinterpret_cast<GenState*>(P.state) = N;
+        __syncthreads();
       }
-      const uint32_t* pr = P.prefix + (uint64_t)lo * km1;
-      const uint32_t e = P.ext[m];
-      if (freq) {
-        const uint32_t p = P.pos[m];
-        uint32_t* dst = Lk + (uint64_t)p * k;
-        uint32_t* od = P.out_items + fw + (uint64_t)p * k;
-        for (uint32_t d = 0; d < km1; ++d) {
-          dst[d] = pr[d];
-          od[d] = P.ior[P.sel ? P.sel[pr[d]] : pr[d]];
-        }
-        dst[km1] = e;
-        od[km1] = P.ior[P.sel ? P.sel[e] : e];
-        P.out_sup[fn + p] = c;
-      }
-      if (P.keep) {
-        uint32_t* cd = P.cand_items + cw + (uint64_t)m * k;
-        for (uint32_t d = 0; d < km1; ++d) cd[d] = P.ior[P.sel ? P.sel[pr[d]] : pr[d]];
-        cd[km1] = P.ior[P.sel ? P.sel[e] : e];
-        P.cand_counts[cn + m] = c;
-      }
+      grid.sync();
+      S = *reinterpret_cast<const GenState*>(P.state);   // grid.sync() orders the write before the read
+    } else {
+      S = generation(GT, P, S);
+      grid.sync();
     }
-    if (tid == 0) {
-      uint32_t* t = P.level_tab + 8 * k;
-      t[0] = M;
-      t[1] = F;
-      t[2] = G;
-      P.status[1] = k;
-    }
-    grid.sync();
-    fw += (uint64_t)F * k;
-    fn += F;
-    if (P.keep) {
-      cw += (uint64_t)M * k;
-      cn += M;
-    }
-    if (F < 2 || k == P.max_k) {
-      ++k;
-      break;
-    }
-    // ---- C_{k+1} from L_k: run starts (same first k-1 items), bounds, hash set
-    const uint32_t w = k;
-    uint32_t* slots = P.slots[k & 1];
-    const uint32_t mask = P.cap_hash - 1;
-    const uint32_t R = grid_scan(
-        [&](uint32_t i) {
-          return (i == 0 || lvl::lex_cmp(Lk + (uint64_t)(i - 1) * w, Lk + (uint64_t)i * w, w - 1) != 0) ? 1u : 0u;
-        },
-        P.run_ex, F, P.bsum, grid);
-    for (uint32_t i = tid; i < F; i += n_threads) {
-      const bool st = i == 0 || lvl::lex_cmp(Lk + (uint64_t)(i - 1) * w, Lk + (uint64_t)i * w, w - 1) != 0;
-      P.rs[i] = st ? 1u : 0u;
-      if (st) P.bound[P.run_ex[i]] = i;
-      uint32_t h = (uint32_t)lvl::hash_mix(lvl::raw_hash(Lk + (uint64_t)i * w, w)) & mask;
-      while (atomicCAS(&slots[h], lvl::kEmpty, i) != lvl::kEmpty) h = (h + 1) & mask;
-    }
-    if (tid == 0) P.bound[R] = F;
-    // the other table (used by generation k - 1) is cleared for generation k + 1
-    uint32_t* other = P.slots[(k + 1) & 1];
-    for (uint32_t i = tid; i < P.cap_hash; i += n_threads) other[i] = lvl::kEmpty;
-    grid.sync();
-    for (uint32_t x = gw; x < F; x += n_warps)
-      lvl::join_warp<false>(x, Lk, w, P.rs, P.run_ex, P.bound, slots, mask, P.cnt, nullptr, nullptr, nullptr, nullptr,
-                            nullptr, nullptr, nullptr);
-    grid.sync();
-    const uint32_t* cntp = P.cnt;
-    const uint32_t M2 = grid_scan([&](uint32_t x) { return cntp[x]; }, P.cand_off, F, P.bsum, grid);
-    const uint32_t G2 = grid_scan([&](uint32_t x) { return cntp[x] ? 1u : 0u; }, P.gidx, F, P.bsum, grid);
-    if (M2 > P.cap_cand || (uint64_t)G2 * w > P.cap_words) {
-      if (tid == 0) P.status[0] |= 1u;
-      break;
-    }
-    for (uint32_t x = gw; x < F; x += n_warps)
-      lvl::join_warp<true>(x, Lk, w, P.rs, P.run_ex, P.bound, slots, mask, P.cnt, P.cand_off, P.gidx, P.prefix,
-                           P.ext_off, P.ext, P.pos, P.counts);   // gpar / eidx land in scratch (pos, counts)
-    if (tid == 0) P.ext_off[G2] = M2;
-    grid.sync();
-    M = M2;
-    G = G2;
-    (void)lane;
   }
+  if (S.done == 2 && tid == 0) P.status[0] |= 1u;
 }
 
 }  // namespace
@@ -320,7 +423,8 @@ namespace {
 
 // per-thread, per-device persistent workspace of the fused loop (grow-only; sized once)
 struct FusedWork {
-  PBuf<uint32_t> prefix, ext_off, ext, counts, pos, L0, L1, rs, run_ex, bound, cnt, cand_off, gidx, s0, s1, bsum;
+  PBuf<uint32_t> prefix, ext_off, ext, counts, pos, L0, L1, rs, run_ex, bound, cnt, cand_off, gidx, s0, s1, bsum, sink;
+  PBuf<uint64_t> bsum64, state;
   PBuf<uint32_t> level_tab, status, out_items, out_sup, cand_items, cand_counts;
   int grid = 0;
 };
@@ -385,6 +489,9 @@ bool mine_fused(const uint32_t* rows, uint64_t pitch_words, uint64_t n_tx, uint3
   P.slots[0] = W.s0.ensure(kCapHash);
   P.slots[1] = W.s1.ensure(kCapHash);
   P.bsum = W.bsum.ensure((size_t)W.grid);
+  P.bsum64 = W.bsum64.ensure((size_t)W.grid);
+  P.sink = W.sink.ensure(2 * (size_t)kCapCand);
+  P.state = W.state.ensure(8);
   P.level_tab = W.level_tab.ensure(8 * (GPA_MAX_K + 2));
   P.status = W.status.ensure(4);
   P.out_items = W.out_items.ensure(kCapOut);
