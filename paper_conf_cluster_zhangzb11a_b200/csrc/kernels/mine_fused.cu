@@ -141,10 +141,11 @@ struct FusedParams {
   // levels: L rows (ping-pong), join scratch
   uint32_t *L[2];
   uint32_t *rs, *run_ex, *bound, *cnt, *cand_off, *gidx, *slots[2];
+  uint32_t* erun;            // per L_k entry: exclusive run-start count (join_warp's run_ex)
   uint32_t* bsum;            // grid_scan block sums (u32)
   uint64_t* bsum64;          // (u64)
   uint32_t* sink;            // join outputs nobody reads here (the group's left parent, the right parent)
-  uint64_t* state;           // GenState handed from CTA 0 to the grid after a single-CTA generation
+  uint64_t* tstamp;          // GPA_FUSED_TRACE: %globaltimer at every phase boundary (64 x 16)
   uint32_t zsplit;           // word slices per group in the counting phase (>= 1)
   // outputs: per generation k (index k): {M_k, F_k, G_k, freq arena offset (lo, hi), cand arena offset (lo, hi)}
   uint32_t* level_tab;       // 8 words per generation, GPA_MAX_K + 1 generations
@@ -156,8 +157,7 @@ __device__ __forceinline__ const uint32_t* row_ptr(const FusedParams& P, uint32_
   return P.rows + (uint64_t)(P.sel ? P.sel[r] : r) * P.pitch;
 }
 
-// ---- teams: the whole grid (grid.sync, grid-wide scans) or CTA 0 alone (__syncthreads, block
-// scans) for generations too small to amortise grid-wide synchronisation
+// ---- the team running a generation: the whole grid (grid.sync, grid-wide scans)
 struct GridTeam {
   cg::grid_group& grid;
   __device__ uint32_t tid() const { return blockIdx.x * blockDim.x + threadIdx.x; }
@@ -166,79 +166,44 @@ struct GridTeam {
   template <class T, class F, class Put>
   __device__ T scan(F get, Put put, uint32_t n, T* bsum) const { return grid_scan<T>(get, put, n, bsum, grid); }
 };
-struct BlockTeam {
-  __device__ uint32_t tid() const { return threadIdx.x; }
-  __device__ uint32_t nthreads() const { return blockDim.x; }
-  __device__ void sync() const { __syncthreads(); }
-  template <class T, class F, class Put>
-  __device__ T scan(F get, Put put, uint32_t n, T*) const {   // exclusive, one CTA
-    __shared__ T sh[kWarps];
-    const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    T off = 0;
-    for (uint32_t base = 0; base < n; base += kFT) {
-      const uint32_t i = base + threadIdx.x;
-      const T v = i < n ? get(i) : T(0);
-      T x = v;
-#pragma unroll
-      for (uint32_t d = 1; d < 32; d <<= 1) {
-        const T y = __shfl_up_sync(0xffffffffu, x, d);
-        if (lane >= d) x += y;
-      }
-      if (lane == 31) sh[warp] = x;
-      __syncthreads();
-      T woff = 0, ctot = 0;
-      for (uint32_t w = 0; w < kWarps; ++w) {
-        const T t = sh[w];
-        if (w < warp) woff += t;
-        ctot += t;
-      }
-      if (i < n) put(i, off + woff + x - v);
-      off += ctot;
-      __syncthreads();
-    }
-    return off;
-  }
-};
-
-// counts[m] += popcount over a word slice -- warp per (group, slice of the words): per 32-word
-// chunk (lane = word) the prefix AND, then one AND + POPC per extension, warp-reduced (redux.sync)
-// into the extension's count; prefix rows' offsets staged in shared memory.  counts must be zero
-// (atomic adds when the words are split into slices).
+// counts[m] += popcount of the AND of candidate m's rows over one 32-word tile, for every tile:
+// work item = (tile t, range of prefix groups); the CTA stages the tile of EVERY L_1 row in
+// shared memory (<= 256 rows x 128 B), then a warp per group: the prefix AND from shared memory
+// (lane = word), one AND + POPC per extension, warp-reduced (redux.sync), one atomic per
+// (candidate, tile) with a non-zero count.  counts must be zero.
 template <class Team>
-__device__ void count_phase(const Team& T, const FusedParams& P, uint32_t G, uint32_t km1, uint32_t Z) {
-  __shared__ uint64_t s_pre[kWarps][64];
+__device__ void count_phase(const Team& T, const FusedParams& P, uint32_t G, uint32_t km1, uint32_t n_ranges) {
+  __shared__ uint32_t s_tile[kFusedMaxRows * 32];
   const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
-  const uint32_t gw = T.tid() >> 5, n_warps = T.nthreads() >> 5;
-  const uint32_t n_chunks = (P.W + 31) / 32;
-  const uint32_t per = (n_chunks + Z - 1) / Z;
-  for (uint32_t it = gw; it < G * Z; it += n_warps) {
-    const uint32_t g = it / Z, z = it % Z;
-    const uint32_t c0 = z * per, c1 = min(n_chunks, c0 + per);
-    const uint32_t e0 = P.ext_off[g], e1 = P.ext_off[g + 1];
-    const uint32_t* pr = P.prefix + (uint64_t)g * km1;
-    for (uint32_t d = lane; d < km1; d += 32) s_pre[wib][d] = (uint64_t)(P.sel ? P.sel[pr[d]] : pr[d]) * P.pitch;
-    __syncwarp();
-    for (uint32_t b0 = e0; b0 < e1; b0 += 32) {
-      const uint32_t nb = min(32u, e1 - b0);
-      const uint64_t my_row = lane < nb ? (uint64_t)(P.sel ? P.sel[P.ext[b0 + lane]] : P.ext[b0 + lane]) * P.pitch : 0;
-      uint32_t mine = 0;   // lane j: the count of extension j over this slice
-      for (uint32_t c = c0; c < c1; ++c) {
-        const uint32_t w = 32 * c + lane;
-        const bool in = w < P.W;
-        uint32_t pw = in ? 0xffffffffu : 0u;
-        for (uint32_t d = 0; d < km1; ++d) pw &= in ? __ldg(P.rows + s_pre[wib][d] + w) : 0u;
-        for (uint32_t j = 0; j < nb; ++j) {
-          const uint64_t ro = __shfl_sync(0xffffffffu, my_row, j);
-          const uint32_t t = __reduce_add_sync(0xffffffffu, (uint32_t)__popc(pw & (in ? __ldg(P.rows + ro + w) : 0u)));
-          mine += lane == j ? t : 0u;
-        }
-      }
-      if (lane < nb && mine) {
-        if (Z == 1) P.counts[b0 + lane] = mine;
-        else atomicAdd(&P.counts[b0 + lane], mine);
+  const uint32_t n_tiles = (P.W + 31) / 32;
+  const uint32_t gpr = (G + n_ranges - 1) / n_ranges;   // groups per range
+  const uint32_t cta = T.tid() / kFT, n_cta = T.nthreads() / kFT;
+  for (uint32_t it = cta; it < n_tiles * n_ranges; it += n_cta) {
+    const uint32_t t = it % n_tiles, r = it / n_tiles;   // consecutive CTAs: same range, next tile
+    const uint32_t w = 32 * t + lane;
+    __syncthreads();   // the previous item's readers are done with s_tile
+    for (uint32_t row = wib; row < P.n1; row += kWarps)
+      s_tile[row * 32 + lane] = w < P.W ? __ldg(P.rows + (uint64_t)(P.sel ? P.sel[row] : row) * P.pitch + w) : 0u;
+    __syncthreads();
+    const uint32_t g1 = min(G, (r + 1) * gpr);
+    for (uint32_t g = r * gpr + wib; g < g1; g += kWarps) {
+      const uint32_t* pr = P.prefix + (uint64_t)g * km1;
+      uint32_t pw = 0xffffffffu;
+      for (uint32_t d = 0; d < km1; ++d) pw &= s_tile[pr[d] * 32 + lane];
+      const uint32_t e0 = P.ext_off[g], e1 = P.ext_off[g + 1];
+      for (uint32_t m = e0; m < e1; ++m) {
+        const uint32_t c = __reduce_add_sync(0xffffffffu, (uint32_t)__popc(pw & s_tile[P.ext[m] * 32 + lane]));
+        if (lane == 0 && c) atomicAdd(&P.counts[m], c);
       }
     }
-    __syncwarp();
+  }
+}
+
+__device__ __forceinline__ void stamp(const FusedParams& P, uint32_t k, uint32_t ph) {
+  if (P.tstamp && blockIdx.x == 0 && threadIdx.x == 0) {
+    uint64_t t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    P.tstamp[(k % 64) * 16 + ph] = t;
   }
 }
 
@@ -255,62 +220,100 @@ __device__ GenState generation(const Team& T, const FusedParams& P, GenState S) 
   const uint32_t tid = T.tid(), n_threads = T.nthreads();
   const uint32_t gw = tid >> 5, n_warps = n_threads >> 5;
   const uint32_t k = S.k, km1 = k - 1, M = S.M, G = S.G;
-  // ---- count C_k: enough (group, word slice) items to occupy every warp
-  const uint32_t n_chunks = (P.W + 31) / 32;
-  uint32_t Z = G ? (4 * n_warps + G - 1) / G : 1;
-  Z = max(1u, min(Z, (n_chunks + 7) / 8));   // >= 8 chunks of 32 words per slice
-  count_phase(T, P, G, km1, Z);
+  // ---- count C_k: (tile, group range) items, about two per CTA
+  const uint32_t n_tiles = (P.W + 31) / 32;
+  const uint32_t n_cta = n_threads / kFT;
+  const uint32_t n_ranges = max(1u, min(G, (2 * n_cta + n_tiles - 1) / n_tiles));
+  stamp(P, k, 0);
+  count_phase(T, P, G, km1, n_ranges);
   T.sync();
-  // ---- threshold: L_k in candidate (lexicographic) order
+  stamp(P, k, 1);
+  // ---- threshold, run structure and hash set of L_k in ONE scan over the groups: group g holds
+  // nf_g frequent candidates (consecutive in L_k, lexicographic) and is a run of L_k when nf_g > 0
+  // (its members share the group's k-1 prefix) -> (L_k offset, run index) = scan of
+  // (nf_g << 32 | nf_g > 0)
   const uint32_t theta = P.theta;
   const uint32_t* counts = P.counts;
-  uint32_t* posp = P.pos;
-  const uint32_t F = T.template scan<uint32_t>([&](uint32_t m) { return counts[m] >= theta ? 1u : 0u; },
-                                              [&](uint32_t i, uint32_t v) { posp[i] = v; }, M, P.bsum);
-  T.sync();
+  const uint32_t* xo = P.ext_off;
+  uint32_t *loff = P.pos, *rrun = P.run_ex;   // per group: L_k offset, run index
+  auto nf = [&](uint32_t g) {
+    uint32_t c = 0;
+    for (uint32_t m = xo[g]; m < xo[g + 1]; ++m) c += counts[m] >= theta;
+    return c;
+  };
+  const uint64_t FR = T.template scan<uint64_t>(
+      [&](uint32_t g) {
+        const uint32_t c = nf(g);
+        return ((uint64_t)c << 32) | (c ? 1ull : 0ull);
+      },
+      [&](uint32_t g, uint64_t v) {
+        loff[g] = (uint32_t)(v >> 32);
+        rrun[g] = (uint32_t)v;
+      },
+      G, P.bsum64);
+  const uint32_t F = (uint32_t)(FR >> 32), R = (uint32_t)FR;
+  stamp(P, k, 2);
   uint32_t* Lk = P.L[k & 1];
   if ((uint64_t)F * k > P.cap_words || S.fw + (uint64_t)F * k > P.cap_out ||
       (P.keep && S.cw + (uint64_t)M * k > P.cap_out)) {
     S.done = 2;
     return S;
   }
-  for (uint32_t m = tid; m < M; m += n_threads) {
-    const uint32_t c = counts[m];
-    const bool freq = c >= theta;
-    if (!freq && !P.keep) continue;
-    uint32_t lo = 0, hi = G;   // g = last group with ext_off[g] <= m
-    while (lo + 1 < hi) {
-      const uint32_t mid = (lo + hi) >> 1;
-      if (P.ext_off[mid] <= m) lo = mid; else hi = mid;
-    }
-    const uint32_t* pr = P.prefix + (uint64_t)lo * km1;
-    const uint32_t e = P.ext[m];
-    if (freq) {
-      const uint32_t p = posp[m];
-      uint32_t* dst = Lk + (uint64_t)p * k;
-      uint32_t* od = P.out_items + S.fw + (uint64_t)p * k;
-      for (uint32_t d = 0; d < km1; ++d) {
-        dst[d] = pr[d];
-        od[d] = P.ior[P.sel ? P.sel[pr[d]] : pr[d]];
+  const uint32_t w = k;
+  uint32_t* slots = P.slots[k & 1];
+  const uint32_t mask = P.cap_hash - 1;
+  // warp per group: its frequent candidates at loff[g] + rank (ballot), their rows, outputs, run
+  // starts, run bounds and hash entries; every candidate to the keep arena
+  const uint32_t lane = threadIdx.x & 31;
+  for (uint32_t g = gw; g < G; g += n_warps) {
+    const uint32_t* pr = P.prefix + (uint64_t)g * km1;
+    const uint32_t e0 = xo[g], e1 = xo[g + 1];
+    uint32_t base = loff[g];
+    for (uint32_t m0 = e0; m0 < e1; m0 += 32) {
+      const uint32_t m = m0 + lane;
+      const bool valid = m < e1;
+      const uint32_t c = valid ? counts[m] : 0u;
+      const bool freq = valid && c >= theta;
+      const uint32_t bal = __ballot_sync(0xffffffffu, freq);
+      const uint32_t e = valid ? P.ext[m] : 0u;
+      if (freq) {
+        const uint32_t rank = __popc(bal & ((1u << lane) - 1u));
+        const uint32_t p = base + rank;
+        uint32_t* dst = Lk + (uint64_t)p * k;
+        uint32_t* od = P.out_items + S.fw + (uint64_t)p * k;
+        for (uint32_t d = 0; d < km1; ++d) {
+          dst[d] = pr[d];
+          od[d] = P.ior[P.sel ? P.sel[pr[d]] : pr[d]];
+        }
+        dst[km1] = e;
+        od[km1] = P.ior[P.sel ? P.sel[e] : e];
+        P.out_sup[S.fn + p] = c;
+        const bool start = p == loff[g];
+        P.rs[p] = start ? 1u : 0u;
+        if (start) P.bound[rrun[g]] = p;
+        uint32_t h = (uint32_t)lvl::hash_mix(lvl::raw_hash(dst, w)) & mask;
+        while (atomicCAS(&slots[h], lvl::kEmpty, p) != lvl::kEmpty) h = (h + 1) & mask;
       }
-      dst[km1] = e;
-      od[km1] = P.ior[P.sel ? P.sel[e] : e];
-      P.out_sup[S.fn + p] = c;
-    }
-    if (P.keep) {
-      uint32_t* cd = P.cand_items + S.cw + (uint64_t)m * k;
-      for (uint32_t d = 0; d < km1; ++d) cd[d] = P.ior[P.sel ? P.sel[pr[d]] : pr[d]];
-      cd[km1] = P.ior[P.sel ? P.sel[e] : e];
-      P.cand_counts[S.cn + m] = c;
+      if (P.keep && valid) {
+        uint32_t* cd = P.cand_items + S.cw + (uint64_t)m * k;
+        for (uint32_t d = 0; d < km1; ++d) cd[d] = P.ior[P.sel ? P.sel[pr[d]] : pr[d]];
+        cd[km1] = P.ior[P.sel ? P.sel[e] : e];
+        P.cand_counts[S.cn + m] = c;
+      }
+      base += __popc(bal);
     }
   }
   if (tid == 0) {
+    P.bound[R] = F;
     uint32_t* t = P.level_tab + 8 * k;
     t[0] = M;
     t[1] = F;
     t[2] = G;
     P.status[1] = k;
   }
+  // the other table (used by generation k - 1) is cleared for generation k + 1
+  uint32_t* other = P.slots[(k + 1) & 1];
+  for (uint32_t i = tid; i < P.cap_hash; i += n_threads) other[i] = lvl::kEmpty;
   S.fw += (uint64_t)F * k;
   S.fn += F;
   if (P.keep) {
@@ -322,33 +325,19 @@ __device__ GenState generation(const Team& T, const FusedParams& P, GenState S) 
     return S;
   }
   T.sync();
-  // ---- C_{k+1} from L_k: run starts (same first k-1 items), bounds, hash set
-  const uint32_t w = k;
-  uint32_t* slots = P.slots[k & 1];
-  const uint32_t mask = P.cap_hash - 1;
-  uint32_t* rexp = P.run_ex;
-  const uint32_t R = T.template scan<uint32_t>(
-      [&](uint32_t i) {
-        return (i == 0 || lvl::lex_cmp(Lk + (uint64_t)(i - 1) * w, Lk + (uint64_t)i * w, w - 1) != 0) ? 1u : 0u;
-      },
-      [&](uint32_t i, uint32_t v) { rexp[i] = v; }, F, P.bsum);
+  stamp(P, k, 3);
+  // per-entry exclusive run index for join_warp (run of entry p = #run starts <= p, minus 1):
+  // from the bounds -- entry p is in run r with bound[r] <= p < bound[r + 1]
+  uint32_t* rexp = P.erun;
+  for (uint32_t r = gw; r < R; r += n_warps)
+    for (uint32_t p = P.bound[r] + lane; p < P.bound[r + 1]; p += 32) rexp[p] = r + 1 - P.rs[p];
   T.sync();
-  for (uint32_t i = tid; i < F; i += n_threads) {
-    const bool st = i == 0 || lvl::lex_cmp(Lk + (uint64_t)(i - 1) * w, Lk + (uint64_t)i * w, w - 1) != 0;
-    P.rs[i] = st ? 1u : 0u;
-    if (st) P.bound[rexp[i]] = i;
-    uint32_t h = (uint32_t)lvl::hash_mix(lvl::raw_hash(Lk + (uint64_t)i * w, w)) & mask;
-    while (atomicCAS(&slots[h], lvl::kEmpty, i) != lvl::kEmpty) h = (h + 1) & mask;
-  }
-  if (tid == 0) P.bound[R] = F;
-  // the other table (used by generation k - 1) is cleared for generation k + 1
-  uint32_t* other = P.slots[(k + 1) & 1];
-  for (uint32_t i = tid; i < P.cap_hash; i += n_threads) other[i] = lvl::kEmpty;
-  T.sync();
+  stamp(P, k, 5);
   for (uint32_t x = gw; x < F; x += n_warps)
-    lvl::join_warp<false>(x, Lk, w, P.rs, P.run_ex, P.bound, slots, mask, P.cnt, nullptr, nullptr, nullptr, nullptr,
+    lvl::join_warp<false>(x, Lk, w, P.rs, rexp, P.bound, slots, mask, P.cnt, nullptr, nullptr, nullptr, nullptr,
                           nullptr, nullptr, nullptr);
   T.sync();
+  stamp(P, k, 6);
   // survivors and non-empty groups in ONE scan: (count << 32) | (count != 0)
   const uint32_t* cntp = P.cnt;
   uint32_t *cop = P.cand_off, *gip = P.gidx;
@@ -360,13 +349,14 @@ __device__ GenState generation(const Team& T, const FusedParams& P, GenState S) 
       },
       F, P.bsum64);
   T.sync();
+  stamp(P, k, 7);
   const uint32_t M2 = (uint32_t)(MG >> 32), G2 = (uint32_t)MG;
   if (M2 > P.cap_cand || (uint64_t)G2 * w > P.cap_words) {
     S.done = 2;
     return S;
   }
   for (uint32_t x = gw; x < F; x += n_warps)
-    lvl::join_warp<true>(x, Lk, w, P.rs, P.run_ex, P.bound, slots, mask, P.cnt, P.cand_off, P.gidx, P.prefix,
+    lvl::join_warp<true>(x, Lk, w, P.rs, P.erun, P.bound, slots, mask, P.cnt, P.cand_off, P.gidx, P.prefix,
                          P.ext_off, P.ext, P.sink, P.sink + P.cap_cand);   // parents: unused here
   if (tid == 0) P.ext_off[G2] = M2;
   for (uint32_t i = tid; i < M2; i += n_threads) P.counts[i] = 0;
@@ -377,8 +367,6 @@ __device__ GenState generation(const Team& T, const FusedParams& P, GenState S) 
   return S;
 }
 
-// a generation is run by CTA 0 alone below this many word operations (M x words x k)
-constexpr uint64_t kSmallGenWork = 4ull << 20;
 
 __global__ void __launch_bounds__(kFT) mine_fused_kernel(FusedParams P) {
   cg::grid_group grid = cg::this_grid();
@@ -398,19 +386,10 @@ __global__ void __launch_bounds__(kFT) mine_fused_kernel(FusedParams P) {
   grid.sync();
   GridTeam GT{grid};
   while (S.k <= P.max_k && S.M > 0 && S.done == 0) {
-    if ((uint64_t)S.M * P.W * S.k < kSmallGenWork) {
-      // CTA 0 runs the generation; everyone picks its state up after one grid-wide barrier
-      if (blockIdx.x == 0) {
-        const GenState N = generation(BlockTeam{}, P, S);
-        if (threadIdx.x == 0) *reinterpret_cast<GenState*>(P.state) = N;
-        __syncthreads();
-      }
-      grid.sync();
-      S = *reinterpret_cast<const GenState*>(P.state);   // grid.sync() orders the write before the read
-    } else {
-      S = generation(GT, P, S);
-      grid.sync();
-    }
+    const uint32_t kk = S.k;
+    S = generation(GT, P, S);
+    grid.sync();
+    stamp(P, kk, 8);
   }
   if (S.done == 2 && tid == 0) P.status[0] |= 1u;
 }
@@ -424,7 +403,8 @@ namespace {
 // per-thread, per-device persistent workspace of the fused loop (grow-only; sized once)
 struct FusedWork {
   PBuf<uint32_t> prefix, ext_off, ext, counts, pos, L0, L1, rs, run_ex, bound, cnt, cand_off, gidx, s0, s1, bsum, sink;
-  PBuf<uint64_t> bsum64, state;
+  PBuf<uint64_t> bsum64;
+  PBuf<uint32_t> erun;
   PBuf<uint32_t> level_tab, status, out_items, out_sup, cand_items, cand_counts;
   int grid = 0;
 };
@@ -491,7 +471,12 @@ bool mine_fused(const uint32_t* rows, uint64_t pitch_words, uint64_t n_tx, uint3
   P.bsum = W.bsum.ensure((size_t)W.grid);
   P.bsum64 = W.bsum64.ensure((size_t)W.grid);
   P.sink = W.sink.ensure(2 * (size_t)kCapCand);
-  P.state = W.state.ensure(8);
+  P.erun = W.erun.ensure(kCapCand);
+
+  static thread_local PBuf<uint64_t> tsb;
+  const bool trace = getenv("GPA_FUSED_TRACE") != nullptr;
+  P.tstamp = trace ? tsb.ensure(64 * 16) : nullptr;
+  if (trace) GPA_CUDA(cudaMemsetAsync(P.tstamp, 0, 64 * 16 * 8, s));
   P.level_tab = W.level_tab.ensure(8 * (GPA_MAX_K + 2));
   P.status = W.status.ensure(4);
   P.out_items = W.out_items.ensure(kCapOut);
@@ -510,6 +495,16 @@ bool mine_fused(const uint32_t* rows, uint64_t pitch_words, uint64_t n_tx, uint3
   GPA_CUDA(cudaMemcpyAsync(st.data(), P.status, 16, cudaMemcpyDeviceToHost, s));
   GPA_CUDA(cudaMemcpyAsync(tab.data(), P.level_tab, tab.size() * 4, cudaMemcpyDeviceToHost, s));
   stream_wait(s);
+  if (trace) {
+    std::vector<uint64_t> ts(64 * 16);
+    GPA_CUDA(cudaMemcpy(ts.data(), P.tstamp, ts.size() * 8, cudaMemcpyDeviceToHost));
+    for (uint32_t k = 2; k <= st[1]; ++k) {
+      fprintf(stderr, "[gpa] fused k=%u M=%u:", k, tab[8 * k]);
+      for (int ph = 1; ph <= 8; ++ph)
+        if (ts[k * 16 + ph] && ts[k * 16 + ph - 1]) fprintf(stderr, " %d:%.1fus", ph, (ts[k * 16 + ph] - ts[k * 16 + ph - 1]) * 1e-3);
+      fprintf(stderr, "\n");
+    }
+  }
   if (st[0] & 1u) return false;   // a capacity was exceeded: the caller runs the multi-kernel path
   out.levels.clear();
   uint64_t fw = 0, fn = 0, cw = 0, cn = 0;
