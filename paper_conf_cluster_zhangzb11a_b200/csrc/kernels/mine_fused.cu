@@ -166,34 +166,52 @@ struct GridTeam {
   template <class T, class F, class Put>
   __device__ T scan(F get, Put put, uint32_t n, T* bsum) const { return grid_scan<T>(get, put, n, bsum, grid); }
 };
-// counts[m] += popcount of the AND of candidate m's rows over one 32-word tile, for every tile:
-// work item = (tile t, range of prefix groups); the CTA stages the tile of EVERY L_1 row in
-// shared memory (<= 256 rows x 128 B), then a warp per group: the prefix AND from shared memory
-// (lane = word), one AND + POPC per extension, warp-reduced (redux.sync), one atomic per
-// (candidate, tile) with a non-zero count.  counts must be zero.
+// counts[m] += popcount of the AND of candidate m's rows over a batch of 32-word tiles: work item
+// = (tile batch, range of prefix groups); the CTA stages the batch of EVERY L_1 row in shared
+// memory (<= 8,192 words: 256 / |L_1| tiles), then a warp per group: its structure (prefix rows,
+// extensions) loaded once into lanes, per tile the prefix AND from shared memory (lane = word),
+// one AND + POPC per extension, warp-reduced (redux.sync), accumulated per extension in the lane
+// of that extension; one atomic per (candidate, item).  counts must be zero.
 template <class Team>
-__device__ void count_phase(const Team& T, const FusedParams& P, uint32_t G, uint32_t km1, uint32_t n_ranges) {
+__device__ void count_phase(const Team& T, const FusedParams& P, uint32_t G, uint32_t km1, uint32_t n_ranges,
+                            uint32_t tb) {
   __shared__ uint32_t s_tile[kFusedMaxRows * 32];
   const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
-  const uint32_t n_tiles = (P.W + 31) / 32;
+  const uint32_t n1 = P.n1;
+  const uint32_t n_tiles = (P.W + 31) / 32, n_batches = (n_tiles + tb - 1) / tb;
   const uint32_t gpr = (G + n_ranges - 1) / n_ranges;   // groups per range
   const uint32_t cta = T.tid() / kFT, n_cta = T.nthreads() / kFT;
-  for (uint32_t it = cta; it < n_tiles * n_ranges; it += n_cta) {
-    const uint32_t t = it % n_tiles, r = it / n_tiles;   // consecutive CTAs: same range, next tile
-    const uint32_t w = 32 * t + lane;
+  for (uint32_t it = cta; it < n_batches * n_ranges; it += n_cta) {
+    const uint32_t bt = it % n_batches, r = it / n_batches;   // consecutive CTAs: same range, next batch
+    const uint32_t t0 = bt * tb, nt = min(tb, n_tiles - t0);
     __syncthreads();   // the previous item's readers are done with s_tile
-    for (uint32_t row = wib; row < P.n1; row += kWarps)
-      s_tile[row * 32 + lane] = w < P.W ? __ldg(P.rows + (uint64_t)(P.sel ? P.sel[row] : row) * P.pitch + w) : 0u;
+    // s_tile[(tile * n1 + row) * 32 + word]
+    for (uint32_t x = wib; x < nt * n1; x += kWarps) {
+      const uint32_t tl = x / n1, row = x % n1;
+      const uint32_t w = 32 * (t0 + tl) + lane;
+      s_tile[x * 32 + lane] = w < P.W ? __ldg(P.rows + (uint64_t)(P.sel ? P.sel[row] : row) * P.pitch + w) : 0u;
+    }
     __syncthreads();
     const uint32_t g1 = min(G, (r + 1) * gpr);
     for (uint32_t g = r * gpr + wib; g < g1; g += kWarps) {
-      const uint32_t* pr = P.prefix + (uint64_t)g * km1;
-      uint32_t pw = 0xffffffffu;
-      for (uint32_t d = 0; d < km1; ++d) pw &= s_tile[pr[d] * 32 + lane];
       const uint32_t e0 = P.ext_off[g], e1 = P.ext_off[g + 1];
-      for (uint32_t m = e0; m < e1; ++m) {
-        const uint32_t c = __reduce_add_sync(0xffffffffu, (uint32_t)__popc(pw & s_tile[P.ext[m] * 32 + lane]));
-        if (lane == 0 && c) atomicAdd(&P.counts[m], c);
+      const uint32_t* prg = P.prefix + (uint64_t)g * km1;
+      const uint32_t my_pre = lane < km1 ? prg[lane] : 0u;   // prefix rows 0..31 in lanes, later ones loaded
+      for (uint32_t b0 = e0; b0 < e1; b0 += 32) {
+        const uint32_t nb = min(32u, e1 - b0);
+        const uint32_t my_ext = lane < nb ? P.ext[b0 + lane] : 0u;
+        uint32_t mine = 0;   // lane j: extension j's count over this item
+        for (uint32_t tl = 0; tl < nt; ++tl) {
+          const uint32_t* st = s_tile + tl * n1 * 32 + lane;
+          uint32_t pw = 0xffffffffu;
+          for (uint32_t d = 0; d < km1; ++d) pw &= st[(d < 32 ? __shfl_sync(0xffffffffu, my_pre, d) : prg[d]) * 32];
+          for (uint32_t j = 0; j < nb; ++j) {
+            const uint32_t c = __reduce_add_sync(0xffffffffu,
+                                                 (uint32_t)__popc(pw & st[__shfl_sync(0xffffffffu, my_ext, j) * 32]));
+            mine += lane == j ? c : 0u;
+          }
+        }
+        if (lane < nb && mine) atomicAdd(&P.counts[b0 + lane], mine);
       }
     }
   }
@@ -220,12 +238,14 @@ __device__ GenState generation(const Team& T, const FusedParams& P, GenState S) 
   const uint32_t tid = T.tid(), n_threads = T.nthreads();
   const uint32_t gw = tid >> 5, n_warps = n_threads >> 5;
   const uint32_t k = S.k, km1 = k - 1, M = S.M, G = S.G;
-  // ---- count C_k: (tile, group range) items, about two per CTA
+  // ---- count C_k: (tile batch, group range) items, about two per CTA
   const uint32_t n_tiles = (P.W + 31) / 32;
+  const uint32_t tb = max(1u, kFusedMaxRows / P.n1);        // tiles per batch (8,192 staged words)
+  const uint32_t n_batches = (n_tiles + tb - 1) / tb;
   const uint32_t n_cta = n_threads / kFT;
-  const uint32_t n_ranges = max(1u, min(G, (2 * n_cta + n_tiles - 1) / n_tiles));
+  const uint32_t n_ranges = max(1u, min(G, (2 * n_cta + n_batches - 1) / n_batches));
   stamp(P, k, 0);
-  count_phase(T, P, G, km1, n_ranges);
+  count_phase(T, P, G, km1, n_ranges, tb);
   T.sync();
   stamp(P, k, 1);
   // ---- threshold, run structure and hash set of L_k in ONE scan over the groups: group g holds
