@@ -37,7 +37,7 @@ namespace cg = cooperative_groups;
 namespace gpa {
 namespace {
 
-constexpr int kFT = 512;                 // threads per CTA (one CTA per SM: cheap grid syncs)
+constexpr int kFT = 1024;                // threads per CTA (one CTA per SM: cheap grid syncs)
 constexpr uint32_t kWarps = kFT / 32;
 
 template <class T>
@@ -229,6 +229,7 @@ struct GenState {
   uint32_t k, M, G;
   uint64_t fw, fn, cw, cn;   // output arenas: words / entries so far (frequent, candidates)
   uint32_t done;             // 0: next generation; 1: finished; 2: overflow
+  uint32_t hcap_prev;        // slots the previous generation's hash set used (dirty)
 };
 
 // One generation by a team: count C_k, threshold into L_k (+ outputs), join + prune into C_{k+1}.
@@ -281,7 +282,10 @@ __device__ GenState generation(const Team& T, const FusedParams& P, GenState S) 
   }
   const uint32_t w = k;
   uint32_t* slots = P.slots[k & 1];
-  const uint32_t mask = P.cap_hash - 1;
+  // hash set of L_k sized to it (>= 2|L_k| + 1 slots, >= 1,024): small tables stay in L1 / L2
+  uint32_t hcap = 1024;
+  while (hcap < 2 * F + 1 && hcap < P.cap_hash) hcap <<= 1;
+  const uint32_t mask = hcap - 1;
   // warp per group: its frequent candidates at loff[g] + rank (ballot), their rows, outputs, run
   // starts, run bounds and hash entries; every candidate to the keep arena
   const uint32_t lane = threadIdx.x & 31;
@@ -332,8 +336,10 @@ __device__ GenState generation(const Team& T, const FusedParams& P, GenState S) 
     P.status[1] = k;
   }
   // the other table (used by generation k - 1) is cleared for generation k + 1
+  // the other table (dirty in the region generation k - 1 used) is cleared for generation k + 1
   uint32_t* other = P.slots[(k + 1) & 1];
-  for (uint32_t i = tid; i < P.cap_hash; i += n_threads) other[i] = lvl::kEmpty;
+  for (uint32_t i = tid; i < S.hcap_prev; i += n_threads) other[i] = lvl::kEmpty;
+  S.hcap_prev = hcap;
   S.fw += (uint64_t)F * k;
   S.fn += F;
   if (P.keep) {
@@ -393,7 +399,7 @@ __global__ void __launch_bounds__(kFT) mine_fused_kernel(FusedParams P) {
   const uint32_t tid = blockIdx.x * blockDim.x + threadIdx.x, n_threads = gridDim.x * blockDim.x;
   // ---- C_2 = every pair of L_1 entries, grouped by the first: group a = {a} x (a, n1)
   const uint32_t n1 = P.n1;
-  GenState S{2, n1 > 1 ? n1 * (n1 - 1) / 2 : 0, n1 > 1 ? n1 - 1 : 0, 0, 0, 0, 0, 0};
+  GenState S{2, n1 > 1 ? n1 * (n1 - 1) / 2 : 0, n1 > 1 ? n1 - 1 : 0, 0, 0, 0, 0, 0, 0};
   for (uint32_t a = tid; a < S.G; a += n_threads) {
     P.prefix[a] = a;
     const uint32_t off = a * n1 - a * (a + 1) / 2;   // pair_index(a, a + 1, n1)
