@@ -114,7 +114,7 @@ typedef struct {
                                   complete intersection).  k = 2 as AUTO; gpa_count treats it as AUTO */
 #define GPA_KERNEL_FUSED 7u    /* gpa_mine: every generation k >= 2 in ONE cooperative launch (grid-wide phases:
                                   complete-intersection counting, threshold, join + prune; no per-level launch or
-                                  host round trip) when |L_1| <= 256 and the L_1 rows fit 64 MB; AUTO picks it for
+                                  host round trip) when |L_1| <= 1,024 and the L_1 rows fit 48 MB; AUTO picks it for
                                   such problems on one GPU.  Otherwise (or on a capacity overflow) AUTO's kernels.
                                   gpa_count treats it as AUTO */
 

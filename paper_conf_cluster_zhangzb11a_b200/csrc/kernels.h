@@ -228,8 +228,8 @@ void device_candgen_finish(const DeviceLevel& L, DeviceBatch& out, DeviceScratch
                            uint32_t M, uint32_t G, cudaStream_t run, cudaEvent_t ev);
 
 // ---- the whole level loop in one cooperative launch for small problems (mine_fused.cu)
-constexpr uint32_t kFusedMaxRows = 256;                       // |L_1|
-constexpr uint64_t kFusedMaxBitsetBytes = 64ull << 20;        // L_1 rows (L2-resident)
+constexpr uint32_t kFusedMaxRows = 1024;                      // |L_1| (a 32-word tile of every row: 128 KB)
+constexpr uint64_t kFusedMaxBitsetBytes = 48ull << 20;        // L_1 rows (L2-resident)
 bool fused_eligible(uint32_t n1, uint64_t pitch_words);
 struct FusedOut {
   struct Level {
@@ -242,9 +242,12 @@ struct FusedOut {
 };
 // Levels k >= 2 of gpa_mine over the L_1 rows (n1 entries; d_sel: entry -> bitset row or nullptr;
 // d_ior: bitset row -> item id).  false: a capacity was exceeded (nothing usable in out).
+// c2_counts: generation 2's counts (pair order over the n1 entries) already on the device, or
+// nullptr to count them in the fused loop.
 bool mine_fused(const uint32_t* rows, uint64_t pitch_words, uint64_t n_tx, uint32_t n1, const uint32_t* d_sel,
                 const uint32_t* d_ior, uint32_t theta, uint32_t max_k, bool keep, int n_sms, cudaStream_t s,
-                FusedOut& out);
+                FusedOut& out, const uint32_t* c2_counts = nullptr);
+constexpr uint32_t kFusedPairsTcRows = 128;   // above this |L_1|, generation 2 runs on the tensor cores first
 
 // ---- device-side work planning (plan.cu)
 constexpr uint32_t kPlanMaxRows = 65536;   // row bitmap of the planning kernels (8 KB of shared memory)

@@ -2,7 +2,7 @@
 // (sm_100a).  SURVEY.md §8(f) f1: "a fully device-resident level loop (CUDA graph or persistent
 // kernel, no per-level D2H)".
 //
-// Small databases (the chess-, mushroom- and accidents-shaped configurations: <= 256 frequent
+// Small databases (the chess-, mushroom-, accidents-shaped and T40I10D100K configurations: <= 1,024 frequent
 // items, a few MB of bitset) are latency-bound: the multi-kernel path spends ~30 launches and a
 // host synchronisation per generation on a few microseconds of counting.  Here every generation is
 // a sequence of grid-wide phases separated by grid.sync() -- no launch, no host round trip:
@@ -38,6 +38,8 @@ namespace gpa {
 namespace {
 
 constexpr int kFT = 1024;                // threads per CTA (one CTA per SM: cheap grid syncs)
+constexpr uint32_t kFusedStageWords = 8192;   // staged tile words per CTA when |L_1| <= 256
+constexpr uint32_t kNoSlot = 0xffffffffu, kClaimed = 0xfffffffeu;
 constexpr uint32_t kWarps = kFT / 32;
 
 template <class T>
@@ -142,6 +144,10 @@ struct FusedParams {
   uint32_t *L[2];
   uint32_t *rs, *run_ex, *bound, *cnt, *cand_off, *gidx, *slots[2];
   uint32_t* erun;            // per L_k entry: exclusive run-start count (join_warp's run_ex)
+  const uint32_t* c2_counts; // generation 2's counts in pair order, computed before the launch (or nullptr)
+  uint32_t *slot, *rowof;    // staging slot of each L_1 entry's row (kNoSlot: unused) and its inverse
+  uint32_t* n_used;          // slots assigned
+  uint32_t *pslot, *eslot;   // C_k's prefix / extension rows as staging slots
   uint32_t* bsum;            // grid_scan block sums (u32)
   uint64_t* bsum64;          // (u64)
   uint32_t* sink;            // join outputs nobody reads here (the group's left parent, the right parent)
@@ -168,16 +174,15 @@ struct GridTeam {
 };
 // counts[m] += popcount of the AND of candidate m's rows over a batch of 32-word tiles: work item
 // = (tile batch, range of prefix groups); the CTA stages the batch of EVERY L_1 row in shared
-// memory (<= 8,192 words: 256 / |L_1| tiles), then a warp per group: its structure (prefix rows,
+// memory (8,192 words: 256 / |L_1| tiles, or one tile of |L_1| x 32 words), then a warp per group: its structure (prefix rows,
 // extensions) loaded once into lanes, per tile the prefix AND from shared memory (lane = word),
 // one AND + POPC per extension, warp-reduced (redux.sync), accumulated per extension in the lane
 // of that extension; one atomic per (candidate, item).  counts must be zero.
 template <class Team>
 __device__ void count_phase(const Team& T, const FusedParams& P, uint32_t G, uint32_t km1, uint32_t n_ranges,
-                            uint32_t tb) {
-  __shared__ uint32_t s_tile[kFusedMaxRows * 32];
+                            uint32_t tb, uint32_t nu) {
+  extern __shared__ uint32_t s_tile[];   // max(8,192, |L_1| x 32) words (dynamic)
   const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
-  const uint32_t n1 = P.n1;
   const uint32_t n_tiles = (P.W + 31) / 32, n_batches = (n_tiles + tb - 1) / tb;
   const uint32_t gpr = (G + n_ranges - 1) / n_ranges;   // groups per range
   const uint32_t cta = T.tid() / kFT, n_cta = T.nthreads() / kFT;
@@ -185,9 +190,10 @@ __device__ void count_phase(const Team& T, const FusedParams& P, uint32_t G, uin
     const uint32_t bt = it % n_batches, r = it / n_batches;   // consecutive CTAs: same range, next batch
     const uint32_t t0 = bt * tb, nt = min(tb, n_tiles - t0);
     __syncthreads();   // the previous item's readers are done with s_tile
-    // s_tile[(tile * n1 + row) * 32 + word]
-    for (uint32_t x = wib; x < nt * n1; x += kWarps) {
-      const uint32_t tl = x / n1, row = x % n1;
+    // s_tile[(tile * nu + slot) * 32 + word]: only the rows this generation's candidates use
+    for (uint32_t x = wib; x < nt * nu; x += kWarps) {
+      const uint32_t tl = x / nu, sl = x % nu;
+      const uint32_t row = P.rowof[sl];
       const uint32_t w = 32 * (t0 + tl) + lane;
       s_tile[x * 32 + lane] = w < P.W ? __ldg(P.rows + (uint64_t)(P.sel ? P.sel[row] : row) * P.pitch + w) : 0u;
     }
@@ -195,16 +201,17 @@ __device__ void count_phase(const Team& T, const FusedParams& P, uint32_t G, uin
     const uint32_t g1 = min(G, (r + 1) * gpr);
     for (uint32_t g = r * gpr + wib; g < g1; g += kWarps) {
       const uint32_t e0 = P.ext_off[g], e1 = P.ext_off[g + 1];
-      const uint32_t* prg = P.prefix + (uint64_t)g * km1;
-      const uint32_t my_pre = lane < km1 ? prg[lane] : 0u;   // prefix rows 0..31 in lanes, later ones loaded
+      const uint32_t* prg = P.pslot + (uint64_t)g * km1;   // the candidates' rows as staging slots
+      const uint32_t my_pre = lane < km1 ? prg[lane] : 0u;  // prefix slots 0..31 in lanes, later ones loaded
       for (uint32_t b0 = e0; b0 < e1; b0 += 32) {
         const uint32_t nb = min(32u, e1 - b0);
-        const uint32_t my_ext = lane < nb ? P.ext[b0 + lane] : 0u;
+        const uint32_t my_ext = lane < nb ? P.eslot[b0 + lane] : 0u;
         uint32_t mine = 0;   // lane j: extension j's count over this item
         for (uint32_t tl = 0; tl < nt; ++tl) {
-          const uint32_t* st = s_tile + tl * n1 * 32 + lane;
+          const uint32_t* st = s_tile + tl * nu * 32 + lane;
           uint32_t pw = 0xffffffffu;
-          for (uint32_t d = 0; d < km1; ++d) pw &= st[(d < 32 ? __shfl_sync(0xffffffffu, my_pre, d) : prg[d]) * 32];
+          for (uint32_t d = 0; d < km1; ++d)
+            pw &= st[(d < 32 ? __shfl_sync(0xffffffffu, my_pre, d) : prg[d]) * 32];
           for (uint32_t j = 0; j < nb; ++j) {
             const uint32_t c = __reduce_add_sync(0xffffffffu,
                                                  (uint32_t)__popc(pw & st[__shfl_sync(0xffffffffu, my_ext, j) * 32]));
@@ -230,6 +237,7 @@ struct GenState {
   uint64_t fw, fn, cw, cn;   // output arenas: words / entries so far (frequent, candidates)
   uint32_t done;             // 0: next generation; 1: finished; 2: overflow
   uint32_t hcap_prev;        // slots the previous generation's hash set used (dirty)
+  uint32_t n_used;           // rows with a staging slot (the rows of L_{k-1})
 };
 
 // One generation by a team: count C_k, threshold into L_k (+ outputs), join + prune into C_{k+1}.
@@ -241,13 +249,16 @@ __device__ GenState generation(const Team& T, const FusedParams& P, GenState S) 
   const uint32_t k = S.k, km1 = k - 1, M = S.M, G = S.G;
   // ---- count C_k: (tile batch, group range) items, about two per CTA
   const uint32_t n_tiles = (P.W + 31) / 32;
-  const uint32_t tb = max(1u, kFusedMaxRows / P.n1);        // tiles per batch (8,192 staged words)
+  const uint32_t nu = S.n_used;   // rows C_k uses (slots assigned while L_{k-1} was scattered)
+  const uint32_t tb = max(1u, kFusedStageWords / (32 * max(nu, 1u)));   // tiles per batch (>= 8,192 staged words)
   const uint32_t n_batches = (n_tiles + tb - 1) / tb;
   const uint32_t n_cta = n_threads / kFT;
   const uint32_t n_ranges = max(1u, min(G, (2 * n_cta + n_batches - 1) / n_batches));
   stamp(P, k, 0);
-  count_phase(T, P, G, km1, n_ranges, tb);
-  T.sync();
+  if (!(k == 2 && P.c2_counts)) {   // (generation 2 counted by the tensor-core pair Gram before the launch)
+    count_phase(T, P, G, km1, n_ranges, tb, nu);
+    T.sync();
+  }
   stamp(P, k, 1);
   // ---- threshold, run structure and hash set of L_k in ONE scan over the groups: group g holds
   // nf_g frequent candidates (consecutive in L_k, lexicographic) and is a run of L_k when nf_g > 0
@@ -257,14 +268,23 @@ __device__ GenState generation(const Team& T, const FusedParams& P, GenState S) 
   const uint32_t* counts = P.counts;
   const uint32_t* xo = P.ext_off;
   uint32_t *loff = P.pos, *rrun = P.run_ex;   // per group: L_k offset, run index
-  auto nf = [&](uint32_t g) {
-    uint32_t c = 0;
-    for (uint32_t m = xo[g]; m < xo[g + 1]; ++m) c += counts[m] >= theta;
-    return c;
-  };
+  uint32_t* nfg = P.cnt;   // scratch: frequent candidates per group (warp per group)
+  // row slots are reassigned for the rows L_k uses (the next generation's candidates)
+  for (uint32_t i = tid; i < nu; i += n_threads) P.slot[P.rowof[i]] = kNoSlot;
+  if (tid == 0) *P.n_used = 0;
+  {
+    const uint32_t ln = threadIdx.x & 31;
+    for (uint32_t g = gw; g < G; g += n_warps) {
+      uint32_t c = 0;
+      for (uint32_t m = xo[g] + ln; m < xo[g + 1]; m += 32) c += counts[m] >= theta;
+      c = __reduce_add_sync(0xffffffffu, c);
+      if (ln == 0) nfg[g] = c;
+    }
+  }
+  T.sync();
   const uint64_t FR = T.template scan<uint64_t>(
       [&](uint32_t g) {
-        const uint32_t c = nf(g);
+        const uint32_t c = nfg[g];
         return ((uint64_t)c << 32) | (c ? 1ull : 0ull);
       },
       [&](uint32_t g, uint64_t v) {
@@ -312,6 +332,14 @@ __device__ GenState generation(const Team& T, const FusedParams& P, GenState S) 
         dst[km1] = e;
         od[km1] = P.ior[P.sel ? P.sel[e] : e];
         P.out_sup[S.fn + p] = c;
+        for (uint32_t d = 0; d < k; ++d) {   // the rows the next generation's candidates can use
+          const uint32_t rw = dst[d];
+          if (P.slot[rw] == kNoSlot && atomicCAS(&P.slot[rw], kNoSlot, kClaimed) == kNoSlot) {
+            const uint32_t sl = atomicAdd(P.n_used, 1u);
+            P.rowof[sl] = rw;
+            P.slot[rw] = sl;
+          }
+        }
         const bool start = p == loff[g];
         P.rs[p] = start ? 1u : 0u;
         if (start) P.bound[rrun[g]] = p;
@@ -386,20 +414,34 @@ __device__ GenState generation(const Team& T, const FusedParams& P, GenState S) 
                          P.ext_off, P.ext, P.sink, P.sink + P.cap_cand);   // parents: unused here
   if (tid == 0) P.ext_off[G2] = M2;
   for (uint32_t i = tid; i < M2; i += n_threads) P.counts[i] = 0;
+  T.sync();
+  // C_{k+1}'s rows as staging slots (assigned while L_k was scattered) for the counting phase
+  for (uint32_t i = tid; i < M2; i += n_threads) P.eslot[i] = P.slot[P.ext[i]];
+  for (uint32_t i = tid; i < G2 * w; i += n_threads) P.pslot[i] = P.slot[P.prefix[i]];
   S.k = k + 1;
   S.M = M2;
   S.G = G2;
+  S.n_used = *reinterpret_cast<volatile uint32_t*>(P.n_used);   // complete: phase C was followed by grid syncs
   S.done = M2 ? 0 : 1;
   return S;
 }
 
 
-__global__ void __launch_bounds__(kFT) mine_fused_kernel(FusedParams P) {
+__global__ void __launch_bounds__(kFT, 1) mine_fused_kernel(FusedParams P) {
   cg::grid_group grid = cg::this_grid();
   const uint32_t tid = blockIdx.x * blockDim.x + threadIdx.x, n_threads = gridDim.x * blockDim.x;
   // ---- C_2 = every pair of L_1 entries, grouped by the first: group a = {a} x (a, n1)
   const uint32_t n1 = P.n1;
-  GenState S{2, n1 > 1 ? n1 * (n1 - 1) / 2 : 0, n1 > 1 ? n1 - 1 : 0, 0, 0, 0, 0, 0, 0};
+  GenState S{2, n1 > 1 ? n1 * (n1 - 1) / 2 : 0, n1 > 1 ? n1 - 1 : 0, 0, 0, 0, 0, 0, 0, n1};
+  for (uint32_t r = tid; r < n1; r += n_threads) {   // generation 2: every row, slot = row
+    P.slot[r] = r;
+    P.rowof[r] = r;
+  }
+  for (uint32_t a = tid; a < S.G; a += n_threads) {
+    P.pslot[a] = a;
+    const uint32_t off = a * n1 - a * (a + 1) / 2;
+    for (uint32_t b = a + 1; b < n1; ++b) P.eslot[off + (b - a - 1)] = b;
+  }
   for (uint32_t a = tid; a < S.G; a += n_threads) {
     P.prefix[a] = a;
     const uint32_t off = a * n1 - a * (a + 1) / 2;   // pair_index(a, a + 1, n1)
@@ -407,7 +449,7 @@ __global__ void __launch_bounds__(kFT) mine_fused_kernel(FusedParams P) {
     for (uint32_t b = a + 1; b < n1; ++b) P.ext[off + (b - a - 1)] = b;
   }
   if (tid == 0) P.ext_off[S.G] = S.M;
-  for (uint32_t i = tid; i < S.M; i += n_threads) P.counts[i] = 0;
+  for (uint32_t i = tid; i < S.M; i += n_threads) P.counts[i] = P.c2_counts ? P.c2_counts[i] : 0u;
   for (uint32_t i = tid; i < P.cap_hash; i += n_threads) P.slots[0][i] = P.slots[1][i] = lvl::kEmpty;
   grid.sync();
   GridTeam GT{grid};
@@ -430,7 +472,7 @@ namespace {
 struct FusedWork {
   PBuf<uint32_t> prefix, ext_off, ext, counts, pos, L0, L1, rs, run_ex, bound, cnt, cand_off, gidx, s0, s1, bsum, sink;
   PBuf<uint64_t> bsum64;
-  PBuf<uint32_t> erun;
+  PBuf<uint32_t> erun, slot, rowof, n_used, pslot, eslot;
   PBuf<uint32_t> level_tab, status, out_items, out_sup, cand_items, cand_counts;
   int grid = 0;
 };
@@ -452,15 +494,17 @@ bool fused_eligible(uint32_t n1, uint64_t pitch_words) {
 
 bool mine_fused(const uint32_t* rows, uint64_t pitch_words, uint64_t n_tx, uint32_t n1, const uint32_t* d_sel,
                 const uint32_t* d_ior, uint32_t theta, uint32_t max_k, bool keep, int n_sms, cudaStream_t s,
-                FusedOut& out) {
+                FusedOut& out, const uint32_t* c2_counts) {
   int device = 0;
   GPA_CUDA(cudaGetDevice(&device));
   FusedWork& W = fused_work(device);
+  const size_t dsmem = (size_t)std::max<uint32_t>(kFusedStageWords, 32u * n1) * 4;
+  ensure_smem_attr(reinterpret_cast<const void*>(mine_fused_kernel), (int)(kFusedMaxRows * 32 * 4));
   if (!W.grid) {
     int per_sm = 0;
-    GPA_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, mine_fused_kernel, kFT, 0));
+    GPA_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, mine_fused_kernel, kFT, kFusedMaxRows * 32 * 4));
     GPA_REQUIRE(per_sm > 0, GPA_ERR_CUDA, "mine_fused: kernel does not fit an SM");
-    W.grid = per_sm * n_sms;
+    W.grid = per_sm * n_sms;   // one CTA per SM at the largest staging size: valid for every launch
   }
   FusedParams P{};
   P.rows = rows;
@@ -498,6 +542,12 @@ bool mine_fused(const uint32_t* rows, uint64_t pitch_words, uint64_t n_tx, uint3
   P.bsum64 = W.bsum64.ensure((size_t)W.grid);
   P.sink = W.sink.ensure(2 * (size_t)kCapCand);
   P.erun = W.erun.ensure(kCapCand);
+  P.c2_counts = c2_counts;
+  P.slot = W.slot.ensure(kFusedMaxRows);
+  P.rowof = W.rowof.ensure(kFusedMaxRows);
+  P.n_used = W.n_used.ensure(4);
+  P.pslot = W.pslot.ensure(kCapWords);
+  P.eslot = W.eslot.ensure(kCapCand);
 
   static thread_local PBuf<uint64_t> tsb;
   const bool trace = getenv("GPA_FUSED_TRACE") != nullptr;
@@ -514,7 +564,7 @@ bool mine_fused(const uint32_t* rows, uint64_t pitch_words, uint64_t n_tx, uint3
   GPA_CUDA(cudaMemsetAsync(P.status, 0, 16, s));
   GPA_CUDA(cudaMemsetAsync(P.level_tab, 0, 8 * (GPA_MAX_K + 2) * 4, s));
   void* args[] = {&P};
-  GPA_CUDA(cudaLaunchCooperativeKernel(reinterpret_cast<const void*>(mine_fused_kernel), W.grid, kFT, args, 0, s));
+  GPA_CUDA(cudaLaunchCooperativeKernel(reinterpret_cast<const void*>(mine_fused_kernel), W.grid, kFT, args, dsmem, s));
   note_launch();
   // sizes: status + per-generation (M, F, G)
   std::vector<uint32_t> tab(8 * (GPA_MAX_K + 2)), st(4);

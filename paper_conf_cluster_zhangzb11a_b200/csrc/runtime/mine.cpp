@@ -341,9 +341,16 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     EvTriple& ev = events.emplace_back();
     GPA_CUDA(cudaEventRecord(ev.e[5], s));
     GPA_CUDA(cudaEventRecord(ev.e[0], s));
+    // many L_1 rows: generation 2 (a dense contraction) on the tensor cores first, unless the
+    // overlapped ingest already counted it
+    const uint32_t* c2 = nullptr;
+    if (nL > kFusedPairsTcRows) {
+      if (!pairs_ready) count_all_pairs(bs, GPA_KERNEL_PAIRS_TC, nullptr);
+      c2 = bs->d_counts.p;
+    }
     const bool ok = mine_fused(bs->rows.p, bs->pitch_words, bs->n_tx_local, (uint32_t)nL,
                                bs->l1_sub ? bs->d_l1.p : nullptr, d_ior.p, (uint32_t)min_count, max_k, keep,
-                               bs->n_sms, s, fo);
+                               bs->n_sms, s, fo, c2);
     GPA_CUDA(cudaEventRecord(ev.e[1], s));
     GPA_CUDA(cudaEventRecord(ev.e[2], s));
     GPA_CUDA(cudaEventRecord(ev.e[6], s));
