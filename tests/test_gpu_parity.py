@@ -464,7 +464,7 @@ def test_proj_fallback_to_complete_intersection(monkeypatch, how):
         monkeypatch.setenv("GPA_PROJ_MAX_MB", "0")
     else:
         monkeypatch.setenv("GPA_PROJ_TEST_MAX_K", how[1:])
-    res = gpa.mine(ds, min_count=theta, keep_candidates=True)
+    res = gpa.mine(ds, min_count=theta, keep_candidates=True, options=gpa.Options(multi_kernel=True))
     assert_mine_equal(res, ref)
     kinds = {lv.k: lv.stats["kernel_name"] for lv in res.levels[2:]}
     last = 2 if how == "mb0" else int(how[1:])
@@ -503,7 +503,7 @@ def test_proj_k3_set_bit_walk_pext(name):
         spec = f"gen.make({name!r}), {theta}"
     code = ("import json, gen, paper_conf_cluster_zhangzb11a_b200 as gpa\n"
             f"ds, th = {spec}\n"
-            "r = gpa.mine(ds, min_count=th)\n"
+            "r = gpa.mine(ds, min_count=th, options=gpa.Options(multi_kernel=True))\n"
             "print(json.dumps(sorted([list(map(int, s)), int(c)] for s, c in r.frequent().items())))\n")
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
     env = dict(os.environ, GPA_PROJ_K3_PEXT="1")
