@@ -166,6 +166,13 @@ __device__ __forceinline__ const uint32_t* addr_of(const uint32_t* base, uint32_
   return r;
 }
 
+// base + 4 idx in one IMAD.WIDE (immediate scale: ptxas keeps the 64-bit addend in the multiply-add)
+__device__ __forceinline__ const uint32_t* addr4(const uint32_t* base, uint32_t idx) {
+  const uint32_t* r;
+  asm("mad.wide.u32 %0, %1, 4, %2;" : "=l"(r) : "r"(idx), "l"(base));
+  return r;
+}
+
 template <uint32_t G, bool SPARSE>
 __device__ __forceinline__ void pext_item(const uint32_t* __restrict__ mp, const uint32_t* __restrict__ sbase,
                                           const uint32_t (&so)[kMemberGroup], const uint32_t* __restrict__ s_oo,
@@ -282,44 +289,63 @@ __global__ void cls3_pad_kernel(const uint32_t* __restrict__ w3, const uint32_t*
     cls3_pad_thread(c, w3, bound, C, cmax, nseg, loc3, nwc, cls_words, items, max_lw);
 }
 
+// pext3 per-warp shared memory: a ring of three chunk slots of member words (set bits carried over
+// from chunk j - 1 still read its slot while chunk j's are packed and chunk j + 1's are stored),
+// the members' row / list offsets and the staged set bits not yet packed.
+constexpr uint32_t kP3Warps = 4;
+constexpr uint32_t kP3Blocks = kG3Group <= 16 ? 6 : 4;  // blocks/SM (shared memory)
+// A staged set bit is (word index in xs) << 5 | bit.  Member rows are 33 words apart: column 32 of
+// every row stays zero, so kP3None (slot 0, column 32, bit 0) packs a 0 for every member.
+constexpr uint32_t kP3Row = 33;
+constexpr uint16_t kP3None = 32u << 5;
+struct P3Warp {
+  uint32_t xs[3][kG3Group][kP3Row];
+  uint32_t so[kG3Group];    // member row: word offset of its bitset row
+  uint32_t oo[kG3Group];    // member list: word offset in data
+  uint16_t pos[1024 + 32];  // staged set bits not yet packed
+};
+
 template <uint32_t G>
-__device__ __forceinline__ void pext3_item(const uint32_t* __restrict__ mrow, const uint32_t* __restrict__ sbase,
-                                           const uint32_t (&so)[kG3Group], const uint32_t* __restrict__ s_oo,
-                                           uint32_t nm, uint32_t ja, uint32_t jb, uint32_t ow0,
-                                           uint32_t* __restrict__ data, uint32_t wbytes, uint16_t* __restrict__ smap) {
+__device__ __forceinline__ void pext3_item(P3Warp& w, const uint32_t* __restrict__ mrow,
+                                           const uint32_t* __restrict__ rows, uint32_t nm, uint32_t ja,
+                                           uint32_t jb, uint32_t ow0, uint32_t* __restrict__ data) {
   const uint32_t lane = threadIdx.x & 31;
-  // groups of <= 8 load the next chunk's words one step ahead; 16-member groups have no registers
-  // left for that and rely on the other warps to hide the load latency
-  constexpr bool kPf = G <= 8;
-  constexpr uint32_t GP = kPf ? G : 1;
-  uint32_t keep[G], xn[GP];
-  uint32_t wc = 0;  // words emitted in this segment (warp-uniform)
-  const uint32_t* mp = mrow + 32u * ja;
-  const uint32_t* cur = sbase + 32u * ja;
-  uint32_t mn = __ldg(mp);
+  uint32_t* xsl = &w.xs[0][0][lane];
+  if (lane < G) w.xs[0][lane][32] = 0u;  // the zero column kP3None reads
+  uint32_t xn[G], keep[G];
 #pragma unroll
   for (uint32_t q = 0; q < G; ++q) keep[q] = 0;
-  if constexpr (kPf) {
+  uint32_t wc = 0;      // words packed in this segment (warp-uniform)
+  uint32_t pend = 0;    // staged set bits not yet packed, < 32 between chunks (P3Carry)
+  bool old = false;     // some of them are from the chunk before the last one
+
+  const uint32_t* mp = mrow + 32u * ja;
+  const uint32_t* cur = rows + 32u * ja;
+  uint32_t mn = __ldg(mp);
 #pragma unroll
-    for (uint32_t q = 0; q < GP; ++q) xn[q] = __ldg(addr_of(cur, so[q], wbytes));
-  }
-  for (uint32_t j = ja; j < jb; ++j) {
-    const uint32_t mw = mn;
-    uint32_t x[G];
-    if constexpr (kPf) {
+  for (uint32_t q = 0; q < G; ++q) xn[q] = __ldg(addr4(cur, w.so[q]));  // slots >= nm: member 0 again
+  uint32_t slot = 0;
+  // j == jb: a last step that only flushes the set bits still pending
+  for (uint32_t j = ja; j <= jb; ++j) {
+    const bool real = j < jb;
+    uint32_t mw = 0;
+    if (real) {
 #pragma unroll
-      for (uint32_t q = 0; q < GP; ++q) x[q] = xn[q];
-    } else {
+      for (uint32_t q = 0; q < G; ++q) xsl[(slot * kG3Group + q) * kP3Row] = xn[q];
+      mw = mn;
+      if (j + 1 < jb) {  // chunk j + 1's words in flight while chunk j is packed
+        mp += 32;
+        cur += 32;
+        mn = __ldg(mp);
 #pragma unroll
-      for (uint32_t q = 0; q < G; ++q) x[q] = __ldg(addr_of(cur, so[q], wbytes));
+        for (uint32_t q = 0; q < G; ++q) xn[q] = __ldg(addr4(cur, w.so[q]));
+      }
     }
-    const uint32_t step = j + 1 < jb ? 32u : 0u;
-    mp += step;
-    cur += step;
-    mn = __ldg(mp);
-    if constexpr (kPf) {
-#pragma unroll
-      for (uint32_t q = 0; q < GP; ++q) xn[q] = __ldg(addr_of(cur, so[q], wbytes));
+    // pending bits of chunk j - 2 (their slot takes chunk j + 1), or at the end: one partial word
+    uint32_t base = pend;
+    if (pend && (old || !real)) {
+      if (lane >= pend) w.pos[lane] = kP3None;
+      base = 32;
     }
     // ranks of this lane's set bits among the chunk's: warp scan of the popcounts
     const uint32_t c = __popc(mw);
@@ -330,52 +356,61 @@ __device__ __forceinline__ void pext3_item(const uint32_t* __restrict__ mrow, co
       if (lane >= d) o += t;
     }
     const uint32_t C = __shfl_sync(0xffffffffu, o, 31);
-    o -= c;
-    for (uint32_t mm = mw; mm; mm &= mm - 1u) smap[o++] = (uint16_t)((lane << 5) | (uint32_t)(__ffs(mm) - 1));
-    __syncwarp();
-    for (uint32_t k0 = 0; k0 < C; k0 += 32) {
-      const uint32_t k = k0 + lane;
-      const bool ok = k < C;
-      const uint32_t v = ok ? smap[k] : 0u;
-      const uint32_t L = v >> 5;
-      const uint32_t bm = ok ? 1u << (v & 31u) : 0u;  // bit select, empty past the chunk's last set bit
+    o += base - c;
+    const uint32_t tag = (slot * kG3Group * kP3Row + lane) << 5;
+    uint16_t* pp = &w.pos[o];
+    for (uint32_t mm = mw; mm; mm &= mm - 1u) *pp++ = (uint16_t)(tag | (uint32_t)(__ffs(mm) - 1));
+    __syncwarp();  // chunk j's member words and set bits visible to the warp
+    const uint32_t t = base + C, nr = t >> 5;
+    for (uint32_t r = 0; r < nr; ++r) {  // one output word per member from set bits 32 r .. 32 r + 31
+      const uint32_t v = w.pos[32u * r + lane];
+      const uint32_t* xb = &w.xs[0][0][0] + (v >> 5);
+      const uint32_t bm = 1u << (v & 31u);
+      const bool mine = lane == (wc & 31u);
 #pragma unroll
       for (uint32_t q = 0; q < G; ++q) {
-        const uint32_t xv = __shfl_sync(0xffffffffu, x[q], L);
-        const uint32_t b = __ballot_sync(0xffffffffu, (xv & bm) != 0u);
-        if (lane == (wc & 31u)) keep[q] = b;
+        const uint32_t b = __ballot_sync(0xffffffffu, (xb[q * kP3Row] & bm) != 0u);
+        if (mine) keep[q] = b;
       }
       if ((wc & 31u) == 31u) {
 #pragma unroll
         for (uint32_t q = 0; q < G; ++q)
-          if (q < nm) data[s_oo[q] + ow0 + (wc - 31u) + lane] = keep[q];
+          if (q < nm) data[w.oo[q] + ow0 + (wc - 31u) + lane] = keep[q];
       }
       ++wc;
     }
-    __syncwarp();  // smap is rewritten by the next chunk
+    pend = t & 31u;
+    old = pend > C;
+    if (nr && pend) {
+      const uint32_t v = lane < pend ? w.pos[32u * nr + lane] : 0u;
+      __syncwarp();
+      if (lane < pend) w.pos[lane] = (uint16_t)v;
+    }
+    __syncwarp();
+    slot = slot == 2u ? 0u : slot + 1u;
   }
   if (wc & 31u) {
     const uint32_t base = wc & ~31u;
     if (lane < (wc & 31u)) {
 #pragma unroll
       for (uint32_t q = 0; q < G; ++q)
-        if (q < nm) data[s_oo[q] + ow0 + base + lane] = keep[q];
+        if (q < nm) data[w.oo[q] + ow0 + base + lane] = keep[q];
     }
   }
 }
 
-__global__ void __launch_bounds__(kT, 3) pext3_kernel(const uint32_t* __restrict__ rows, uint64_t pitch,
-                                                      const uint32_t* __restrict__ par_a,
-                                                      const uint32_t* __restrict__ par_b,
-                                                      const uint32_t* __restrict__ bound, uint32_t cmax,
-                                                      const uint32_t* __restrict__ item_pair,
-                                                      const uint32_t* __restrict__ item_off, uint32_t T,
-                                                      const uint32_t* __restrict__ loc3,
-                                                      const uint64_t* __restrict__ off, uint32_t* __restrict__ data,
-                                                      uint32_t wbytes) {
-  __shared__ uint16_t s_map[kT / 32][1024];
-  __shared__ uint32_t s_oo[kT / 32][kG3Group];
-  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+__global__ void __launch_bounds__(kP3Warps * 32, kP3Blocks) pext3_kernel(const uint32_t* __restrict__ rows, uint64_t pitch,
+                                                                 const uint32_t* __restrict__ par_a,
+                                                                 const uint32_t* __restrict__ par_b,
+                                                                 const uint32_t* __restrict__ bound, uint32_t cmax,
+                                                                 const uint32_t* __restrict__ item_pair,
+                                                                 const uint32_t* __restrict__ item_off, uint32_t T,
+                                                                 const uint32_t* __restrict__ loc3,
+                                                                 const uint64_t* __restrict__ off,
+                                                                 uint32_t* __restrict__ data) {
+  extern __shared__ __align__(16) unsigned char p3_smem[];
+  P3Warp& w = reinterpret_cast<P3Warp*>(p3_smem)[threadIdx.x >> 5];
+  const uint32_t lane = threadIdx.x & 31;
   const uint32_t it = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   if (it >= T) return;
   const uint32_t p = item_pair[it];
@@ -387,25 +422,26 @@ __global__ void __launch_bounds__(kT, 3) pext3_kernel(const uint32_t* __restrict
   uint32_t ja, jb;
   seg_range((uint32_t)(pitch / 32), s, ja, jb);
   if (ja >= jb) return;
-  uint32_t* oo = s_oo[warp];
-  uint32_t so[kG3Group];
-#pragma unroll
-  for (uint32_t q = 0; q < kG3Group; ++q) {
-    const uint32_t e = first + (q < nm ? q : 0);  // surplus slots shadow member 0 (not stored)
-    so[q] = (uint32_t)((uint64_t)par_b[e] * pitch);
-    if (lane == q) oo[q] = (uint32_t)off[e];
+  if (lane < kG3Group) {
+    const uint32_t e = first + (lane < nm ? lane : 0u);
+    w.so[lane] = (uint32_t)((uint64_t)par_b[e] * pitch);
+    w.oo[lane] = (uint32_t)off[e];
   }
   __syncwarp();
   const uint32_t* mrow = rows + (uint64_t)par_a[j0] * pitch + lane;
   const uint32_t ow0 = loc3[p];
-  if (nm <= 2)
-    pext3_item<2>(mrow, rows + lane, so, oo, nm, ja, jb, ow0, data, wbytes, s_map[warp]);
-  else if (nm <= 4)
-    pext3_item<4>(mrow, rows + lane, so, oo, nm, ja, jb, ow0, data, wbytes, s_map[warp]);
+  if (nm <= 4)
+    pext3_item<4>(w, mrow, rows + lane, nm, ja, jb, ow0, data);
   else if (nm <= 8)
-    pext3_item<8>(mrow, rows + lane, so, oo, nm, ja, jb, ow0, data, wbytes, s_map[warp]);
+    pext3_item<8>(w, mrow, rows + lane, nm, ja, jb, ow0, data);
+  else if (nm <= 12)
+    pext3_item<12>(w, mrow, rows + lane, nm, ja, jb, ow0, data);
+  else if (kG3Group > 16 && nm <= 16)
+    pext3_item<16>(w, mrow, rows + lane, nm, ja, jb, ow0, data);
+  else if (kG3Group > 24 && nm <= 24)
+    pext3_item<24>(w, mrow, rows + lane, nm, ja, jb, ow0, data);
   else
-    pext3_item<16>(mrow, rows + lane, so, oo, nm, ja, jb, ow0, data, wbytes, s_map[warp]);
+    pext3_item<kG3Group>(w, mrow, rows + lane, nm, ja, jb, ow0, data);
 }
 
 // item -> its pair (items of pair p are item_off[p] .. + items[p])
@@ -702,11 +738,14 @@ bool proj_build_finish(const ProjPending& pp, const uint64_t T[2], const uint32_
     { item_pair_kernel<<<grid_for(pp.n_pairs, n_sms), kT, 0, s>>>(W.items.p, W.item_off.p, pp.n_pairs,
                                                                  W.item_pair.p); note_launch(); }
     const uint64_t blocks = (T[0] + kT / 32 - 1) / (kT / 32);
-    if (!pp.prev && gather3())
-      { pext3_kernel<<<(unsigned)blocks, kT, 0, s>>>(pp.rows, pp.pitch, pp.par_a, pp.par_b, W.bound.p, pp.cmax,
-                                                     W.item_pair.p, W.item_off.p, (uint32_t)T[0], W.loc.p, out.off.p,
-                                                     out.data.p, 4u); note_launch(); }
-    else
+    if (!pp.prev && gather3()) {
+      const int smem = (int)(kP3Warps * sizeof(P3Warp));
+      ensure_smem_attr((const void*)pext3_kernel, smem);
+      pext3_kernel<<<(unsigned)((T[0] + kP3Warps - 1) / kP3Warps), kP3Warps * 32, smem, s>>>(
+          pp.rows, pp.pitch, pp.par_a, pp.par_b, W.bound.p, pp.cmax, W.item_pair.p, W.item_off.p, (uint32_t)T[0],
+          W.loc.p, out.off.p, out.data.p);
+      note_launch();
+    } else
       { pext_kernel<<<(unsigned)blocks, kT, 0, s>>>(src, pp.par_a, pp.par_b, W.bound.p, pp.cmax, W.item_pair.p,
                                                     W.item_off.p, (uint32_t)T[0], W.loc.p, out.off.p, out.data.p, 4u);
         note_launch(); }
