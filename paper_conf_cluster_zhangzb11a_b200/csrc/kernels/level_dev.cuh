@@ -52,6 +52,14 @@ __device__ __forceinline__ bool contains(const uint32_t* __restrict__ L, uint32_
 // survivors; EMIT = true: group gidx[x] (prefix = L[x]) and its extensions, in sibling order, at
 // cand_off[x] (warp ballot ranks the survivors).  flags / run_ex / bound: run starts, their
 // exclusive scan, run boundaries (bound[#runs] = n).
+// "px without item d, then b" == L row q?  (no key array: the items are read in place)
+__device__ __forceinline__ bool row_is_sub(const uint32_t* __restrict__ row, const uint32_t* __restrict__ px,
+                                           uint32_t w, uint32_t d, uint32_t b) {
+  for (uint32_t i = 0; i + 1 < w; ++i)
+    if (row[i] != px[i < d ? i : i + 1]) return false;
+  return row[w - 1] == b;
+}
+
 template <bool EMIT>
 __device__ __forceinline__ void join_warp(uint32_t x, const uint32_t* __restrict__ L, uint32_t w,
                                           const uint32_t* __restrict__ flags, const uint32_t* __restrict__ run_ex,
@@ -59,34 +67,24 @@ __device__ __forceinline__ void join_warp(uint32_t x, const uint32_t* __restrict
                                           uint32_t mask, uint32_t* cnt, const uint32_t* __restrict__ cand_off,
                                           const uint32_t* __restrict__ gidx, uint32_t* prefix, uint32_t* ext_off,
                                           uint32_t* ext, uint32_t* gpar, uint32_t* eidx) {
-  uint32_t probe[GPA_MAX_K];
-  uint64_t A[GPA_MAX_K], B[GPA_MAX_K];
   const uint32_t lane = threadIdx.x & 31;
   if (EMIT && cnt[x] == 0) return;  // warp-uniform
   // run index of x = (#run starts <= x) - 1
   const uint32_t r = run_ex[x] + flags[x] - 1;
-  const uint32_t end = bound[r + 1];  // bound[n_runs] = n (sentinel)
+  const uint32_t end = bound[r + 1];  // bound[n_runs] = n (sentinel end of the last run)
   if (!EMIT && end == x + 1) {
     if (lane == 0) cnt[x] = 0;
     return;
   }
   const uint32_t* px = L + (uint64_t)x * w;
-  // subset "px without item d, then b": A[d] = sum_{i<d} (x_i+1) P^i,
-  // B[d] = sum_{i>d} (x_i+1) P^(i-1); b lands at position w-1
-  uint64_t pw = 1, acc = 0;
-  for (uint32_t i = 0; i < w; ++i) {  // B[i] temporarily holds P^i
-    A[i] = acc;
-    B[i] = pw;
-    acc += (uint64_t)(px[i] + 1) * pw;
+  // hash of the subset "px without item d, then b" = A_d + B_d + (b + 1) P^(w-1) with
+  // A_d = sum_{i<d} (x_i+1) P^i, B_d = sum_{i>d} (x_i+1) P^(i-1): both walked with d below
+  uint64_t B0 = 0, pw = 1;
+  for (uint32_t i = 1; i < w; ++i) {
+    B0 += (uint64_t)(px[i] + 1) * pw;
     pw *= kHashP;
   }
-  const uint64_t p_last = B[w - 1];  // P^(w-1)
-  uint64_t suf = 0;
-  for (uint32_t d = w; d-- > 0;) {
-    const uint64_t pprev = d > 0 ? B[d - 1] : 0;
-    B[d] = suf;
-    suf += (uint64_t)(px[d] + 1) * pprev;  // term of item d at position d-1
-  }
+  const uint64_t p_last = pw;  // P^(w-1)
   uint32_t here = 0;  // survivors so far (warp-uniform)
   for (uint32_t y0 = x + 1; y0 < end; y0 += 32) {
     const uint32_t y = y0 + lane;
@@ -94,15 +92,25 @@ __device__ __forceinline__ void join_warp(uint32_t x, const uint32_t* __restrict
     uint32_t b = 0;
     if (keep) {
       b = L[(uint64_t)y * w + w - 1];
+      uint64_t A = 0, B = B0, pd = 1;
       const uint64_t hb = (uint64_t)(b + 1) * p_last;
       // subsets dropping item d of the shared prefix (dropping either of the last two items
       // gives the parents x or y, members of L by construction)
       for (uint32_t d = 0; d + 1 < w && keep; ++d) {
-        uint32_t q = 0;
-        for (uint32_t i = 0; i < w; ++i)
-          if (i != d) probe[q++] = px[i];
-        probe[q] = b;
-        keep = contains(L, w, slots, mask, probe, A[d] + B[d] + hb);
+        uint32_t h = (uint32_t)hash_mix(A + B + hb) & mask;
+        for (;;) {
+          const uint32_t i = slots[h];
+          if (i == kEmpty) {
+            keep = false;
+            break;
+          }
+          if (row_is_sub(L + (uint64_t)i * w, px, w, d, b)) break;
+          h = (h + 1) & mask;
+        }
+        const uint64_t xd = (uint64_t)(px[d] + 1) * pd, xd1 = (uint64_t)(px[d + 1] + 1) * pd;
+        A += xd;
+        B -= xd1;
+        pd *= kHashP;
       }
     }
     const uint32_t ballot = __ballot_sync(0xffffffffu, keep);

@@ -322,6 +322,8 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     }
   };
   std::deque<EvTriple> events;
+  EvTriple trace_evs;        // GPA_TRACE: [0] end of join stage 1 (s), [1] of the class tables (aux_s)
+  cudaEvent_t* trace_ev = trace_evs.e;
   std::vector<size_t> event_level;
   d_ior.alloc(std::max<uint32_t>(bs->n_rows, 1), s);
   if (bs->n_rows)
@@ -431,6 +433,7 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
       // synchronisation per generation
       const uint32_t n_up = Ld.n_dev ? Ld.n_max : Ld.n;
       if (device_candgen_begin(Ld, Bd, scratch, bs->n_sms, s, &d_sizes)) {
+        if (trace_enabled()) GPA_CUDA(cudaEventRecord(trace_ev[0], s));
         uint32_t* hs = host_sizes();
         if (proj_build_begin(n_up, Ld.par_a.p, Ld.par_b.p, k == 3 ? nullptr : Pprev, bs->rows.p, bs->pitch_words,
                              bs->n_rows, scratch, bs->n_sms, aux_s.s, ppend, Ld.n_dev)) {
@@ -439,10 +442,13 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
         } else {
           proj_on = false;   // lists not addressable: complete intersection from this generation on
         }
+        if (trace_enabled()) GPA_CUDA(cudaEventRecord(trace_ev[1], aux_s.s));
         GPA_CUDA(cudaMemcpyAsync(hs, d_sizes, 8, cudaMemcpyDeviceToHost, s));
         if (Ld.n_dev) GPA_CUDA(cudaMemcpyAsync(hs + 10, Ld.n_dev, 4, cudaMemcpyDeviceToHost, s));
+        const double tw0 = now_ms();
         stream_wait(s);
         stream_wait(aux_s.s);
+        const double tw1 = now_ms();
         M = hs[0];
         G = hs[1];
         std::memcpy(pT, hs + 2, 16);
@@ -456,6 +462,13 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
         device_candgen_finish(Ld, Bd, scratch, bs->n_sms, s, (uint32_t)M, (uint32_t)G, aux_s.s, aux_evs.e[0]);
         GPA_CUDA(cudaEventRecord(aux_evs.e[1], aux_s.s));
         aux_join = true;
+        if (trace_enabled()) {
+          float ja = 0, jb = 0;
+          GPA_CUDA(cudaEventElapsedTime(&ja, ev.e[5], trace_ev[0]));
+          GPA_CUDA(cudaEventElapsedTime(&jb, ev.e[5], trace_ev[1]));
+          fprintf(stderr, "[gpa] k=%u host: enqueue %.3f, wait %.3f, after wait %.3f ms; device: join stage 1 %.3f, "
+                  "class tables %.3f ms\n", k, tw0 - t0, tw1 - tw0, now_ms() - tw1, ja, jb);
+        }
       }
     } else {
       // complete intersection: join + prune on the device, |L_{k-1}| read with the sizes of C_k
@@ -601,6 +614,13 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     }
     st.count_ms = a;
     st.allreduce_ms = dist ? b : 0.0;
+    if (trace_enabled()) {   // device timeline of the generation (ms from the previous one's end)
+      float gap = 0;
+      if (i > 0) GPA_CUDA(cudaEventElapsedTime(&gap, events[i - 1].e[6], E.e[5]));
+      fprintf(stderr, "[gpa] gen %u: gap %.3f candgen %.3f setup %.3f build %.3f count %.3f threshold %.3f\n",
+              R->levels[event_level[i]].k, gap, cg, st.kernel == GPA_KERNEL_PROJ ? st.setup_ms : 0.0,
+              st.kernel == GPA_KERNEL_PROJ ? st.build_ms : 0.0, a, g - cg - a - b);
+    }
     R->phase_ms[GPA_PHASE_CANDGEN] += cg;
     R->phase_ms[GPA_PHASE_COUNT] += a + b;
     R->phase_ms[GPA_PHASE_THRESHOLD] += g - cg - a - b;
