@@ -292,11 +292,14 @@ def roofline_records(res, stats_avg: dict, n_tx: int, peaks: dict, sm_max: float
                      "peak_basis": f"POPC (XU) pipe: 148 SM x 16 /clk / {ppw} POPC per 32-tx word x 32 x "
                                    f"{sm_max:.0f} MHz"})
     for r in recs:
-        t = traffic_entry(("pext3_kernel" if r["k"] == 3 else "pext_kernel") if r["kernel"] == "lists" else r["kernel"],
-                          r["k"])
+        kern = {"lists": "pext3_kernel" if r["k"] == 3 else "pext_kernel",
+                "count_proj": "count_proj_kernel<0>" if r["k"] == 3 else "count_proj_kernel<1>"}.get(r["kernel"],
+                                                                                                   r["kernel"])
+        t = traffic_entry(kern, r["k"])
         r["traffic"] = t.get("dram_bytes") if t else None
-        if t and "issue_active" in t:
-            r["issue_active"] = t["issue_active"]
+        for key in ("issue_active", "tensor_pipe_active", "alu_pipe_active"):
+            if t and key in t:
+                r[key] = t[key]
     return recs
 
 
