@@ -212,7 +212,8 @@ void launch_count_proj(const DeviceProj& P, const uint32_t* gpar, const uint32_t
 // items[i] = item_of_row[rows[i]] (row ids -> original item ids) for i < n, or for i < *n_dev * k
 // when n_dev is given (n then an upper bound)
 void device_map_items(const uint32_t* rows, uint64_t n, const uint32_t* item_of_row, uint32_t* items, int n_sms,
-                      cudaStream_t s, const uint32_t* n_dev = nullptr, uint32_t k = 1);
+                      cudaStream_t s, const uint32_t* n_dev = nullptr, uint32_t k = 1,
+                      const uint32_t* sup_in = nullptr, uint32_t* sup_out = nullptr);
 // exclusive scan of n u32 (CUB); the total is written to *tot (device) when tot != nullptr
 void device_exclusive_scan(const uint32_t* in, uint32_t* out, uint32_t n, uint32_t* tot, DeviceScratch& scratch,
                            cudaStream_t s);

@@ -145,11 +145,16 @@ __global__ void nonzero_kernel(const uint32_t* __restrict__ cnt, uint32_t n, uin
     flags[i] = cnt[i] != 0;
 }
 
+// L_k's rows -> item ids (n = entries x k words) and, with sup_in, its supports copied to sup_out;
+// a device-sized level stops at its count
 __global__ void map_items_kernel(const uint32_t* __restrict__ rows, uint64_t n, const uint32_t* __restrict__ ior,
-                                 uint32_t* items, const uint32_t* __restrict__ n_dev, uint32_t k) {
+                                 uint32_t* items, const uint32_t* __restrict__ n_dev, uint32_t k,
+                                 const uint32_t* __restrict__ sup_in, uint32_t* sup_out) {
   if (n_dev && (uint64_t)*n_dev * k < n) n = (uint64_t)*n_dev * k;
-  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
     items[i] = ior[rows[i]];
+    if (sup_in && i % k == 0) sup_out[i / k] = sup_in[i / k];
+  }
 }
 
 unsigned grid_for(uint64_t n, int n_sms) {
@@ -241,9 +246,10 @@ void device_exclusive_scan(const uint32_t* in, uint32_t* out, uint32_t n, uint32
 }
 
 void device_map_items(const uint32_t* rows, uint64_t n, const uint32_t* item_of_row, uint32_t* items, int n_sms,
-                      cudaStream_t s, const uint32_t* n_dev, uint32_t k) {
+                      cudaStream_t s, const uint32_t* n_dev, uint32_t k, const uint32_t* sup_in, uint32_t* sup_out) {
   if (n == 0) return;
-  { map_items_kernel<<<grid_for(n, n_sms), kThreads, 0, s>>>(rows, n, item_of_row, items, n_dev, k); note_launch(); }
+  { map_items_kernel<<<grid_for(n, n_sms), kThreads, 0, s>>>(rows, n, item_of_row, items, n_dev, k, sup_in, sup_out);
+    note_launch(); }
   GPA_CUDA(cudaGetLastError());
 }
 

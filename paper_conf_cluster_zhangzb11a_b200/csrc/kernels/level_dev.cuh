@@ -1,5 +1,5 @@
 // Device helpers of the level transition shared by candgen.cu (separate kernels) and
-// transition.cu (the fused cooperative kernel).  Internal; included by .cu files only.
+// mine_fused.cu (the whole loop in one cooperative launch).  Internal; included by .cu files only.
 #pragma once
 #include <cstdint>
 #include "../common.h"

@@ -1,5 +1,5 @@
-// Device pieces of the projected-list class tables (proj.cu) shared with the fused level
-// transition (transition.cu).  Internal; included by .cu files only.
+// Device pieces of the projected-list builds (proj.cu): segments, class tables, generation 3's
+// word counts.  Internal; included by .cu files only.
 #pragma once
 #include <cstdint>
 #include "../common.h"

@@ -549,8 +549,7 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     pd.open = true;
     pd.items.alloc((size_t)M * k, s);
     pd.sup.alloc(M, s);
-    device_map_items(Ln.rows.p, (uint64_t)M * k, d_ior.p, pd.items.p, bs->n_sms, s, Ln.n_dev, k);
-    GPA_CUDA(cudaMemcpyAsync(pd.sup.p, Ln.sup.p, (size_t)M * 4, cudaMemcpyDeviceToDevice, s));
+    device_map_items(Ln.rows.p, (uint64_t)M * k, d_ior.p, pd.items.p, bs->n_sms, s, Ln.n_dev, k, Ln.sup.p, pd.sup.p);
     ev.counted = cs.e0 != nullptr;
     GPA_CUDA(cudaEventRecord(ev.e[6], s));
     std::vector<uint32_t> counts;

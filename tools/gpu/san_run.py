@@ -12,4 +12,6 @@ with gpa.Bitset(ds, row_min_count=th) as bs:                                    
     assert len(bs.count(a.levels[2].cand)) == a.levels[2].n_cand
 t = gen.make("t40i10d100k")
 d = gpa.mine(t, min_count=gpa.min_count(t.n_tx, "0.01"))                                # fused with the tc pair Gram
+e = gpa.mine(t, min_count=gpa.min_count(t.n_tx, "0.01"), options=gpa.Options(multi_kernel=True))  # pext3, pext, joins
+assert d.frequent() == e.frequent()
 print("san_run ok", len(a.frequent()), len(d.frequent()))
