@@ -104,10 +104,29 @@ void launch_gather_rows(const uint32_t* rows_all, const uint32_t* sel, uint32_t 
                         uint32_t* rows_sub, int n_sms, cudaStream_t stream);
 
 // ---- device-side level transition (candgen.cu)
+// Status words of the single-launch scans (scan.cu): per tile a flag (epoch << 2 | 1 aggregate /
+// 2 inclusive) and the two values; the epoch advances per scan, so nothing is cleared between
+// scans.  One per stream at a time (scans on one state must be stream-ordered).
+struct ScanState {
+  PBuf<uint32_t> flags;
+  PBuf<uint64_t> agg, inc;
+  uint32_t epoch = 0;
+};
+// fused scans (scan_dev.cuh): tiles of a scan of n values, and the epoch of the next scan on st
+uint32_t scan_tiles(uint32_t n);
+uint32_t scan_epoch(ScanState& st, uint32_t tiles, cudaStream_t s);
+void scan_excl_u32(const uint32_t* in, uint32_t* out, uint32_t n, uint32_t* tot, ScanState& st, cudaStream_t s);
+void scan_excl_u32(const uint32_t* in, uint32_t* out, uint32_t n, uint64_t* tot, ScanState& st, cudaStream_t s);
+void scan_excl_u64(const uint64_t* in, uint64_t* out, uint32_t n, uint64_t* tot, ScanState& st, cudaStream_t s);
+// (cnt << 32 | cnt != 0) scanned as one: off = exclusive sums of cnt, idx = exclusive count of the
+// non-zero cnt, tot2 = {sum, non-zero count}
+void scan_excl_split(const uint32_t* cnt, uint32_t* off, uint32_t* idx, uint32_t n, uint32_t* tot2, ScanState& st,
+                     cudaStream_t s);
+
 struct DeviceScratch {
   DBuf<uint32_t> a, b, c, d, e, f, g, h, i;
-  DBuf<uint8_t> tmp;
   uint32_t hash_cap = 0;   // slots of the join's hash set (i), set by device_candgen_begin
+  ScanState scan;
   uint32_t* u32a(size_t n, cudaStream_t s) { a.ensure(n ? n : 1, s); return a.p; }
   uint32_t* u32b(size_t n, cudaStream_t s) { b.ensure(n ? n : 1, s); return b.p; }
   uint32_t* u32c(size_t n, cudaStream_t s) { c.ensure(n ? n : 1, s); return c.p; }
@@ -117,7 +136,6 @@ struct DeviceScratch {
   uint32_t* u32g(size_t n, cudaStream_t s) { g.ensure(n ? n : 1, s); return g.p; }
   uint32_t* u32h(size_t n, cudaStream_t s) { h.ensure(n ? n : 1, s); return h.p; }
   uint32_t* u32i(size_t n, cudaStream_t s) { i.ensure(n ? n : 1, s); return i.p; }
-  void* get(size_t bytes, cudaStream_t s) { tmp.ensure(bytes ? bytes : 1, s); return tmp.p; }
 };
 // L_k on the device: n rows of k row ids (lexicographic) and their supports
 // par_a[p] / par_b[p]: index in L_{k-1} of the entry's left parent (its first k-1 items) and

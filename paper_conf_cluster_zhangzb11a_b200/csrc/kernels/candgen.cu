@@ -7,13 +7,14 @@
 //             Fig. 4 P18@863) + prune: every k-subset must be in L_k (P13@178; Q7),
 //             emitted grouped by k-prefix (group prefix = the left parent), lexicographic.
 // The same definitions as the host implementation in runtime/candgen.cpp, written for the GPU:
-// flags + exclusive scans (CUB) + scatters; prune probes are binary searches in the sorted L_k.
+// single-launch scans with fused flags / bounds (scan_dev.cuh) + scatters; prune probes hit a
+// device hash set over L_k (level_dev.cuh).
 #include <cstdint>
-#include <cub/device/device_scan.cuh>
 
 #include "../common.h"
 #include "../kernels.h"
 #include "level_dev.cuh"
+#include "scan_dev.cuh"
 
 namespace gpa {
 namespace {
@@ -33,18 +34,23 @@ __global__ void hash_build_kernel(const uint32_t* __restrict__ L, uint32_t n, ui
   }
 }
 
-__global__ void flag_ge_kernel(const uint32_t* __restrict__ counts, uint32_t M, uint32_t theta, uint32_t* flags) {
-  for (uint32_t m = blockIdx.x * blockDim.x + threadIdx.x; m < M; m += gridDim.x * blockDim.x)
-    flags[m] = counts[m] >= theta;
+// L_k's positions: pos[m] = #{m' < m : count >= theta}, *count = |L_k| (one launch)
+__global__ void __launch_bounds__(sd::kScanThreads, 1) ge_scan_kernel(const uint32_t* __restrict__ counts, uint32_t M,
+                                                                      uint32_t theta, uint32_t* __restrict__ pos,
+                                                                      uint32_t* count, uint32_t* sflags, uint64_t* agg,
+                                                                      uint64_t* inc, uint32_t epoch) {
+  sd::scan_tile<uint32_t>(
+      M, [&](uint32_t m) { return counts[m] >= theta ? 1u : 0u; }, [&](uint32_t m, uint32_t e, uint32_t) { pos[m] = e; },
+      [&](uint32_t t) { *count = t; }, sflags, agg, inc, epoch);
 }
 
 // k = 2: candidate m is the pair (a, b) of pair_index order over n rows
-__global__ void scatter_pairs_kernel(const uint32_t* __restrict__ counts, const uint32_t* __restrict__ flags,
+__global__ void scatter_pairs_kernel(const uint32_t* __restrict__ counts, uint32_t theta,
                                      const uint32_t* __restrict__ pos, uint32_t M, uint32_t n,
                                      const uint32_t* __restrict__ sel, uint32_t* L,
                                      uint32_t* sup, uint32_t* par_a, uint32_t* par_b) {
   for (uint32_t m = blockIdx.x * blockDim.x + threadIdx.x; m < M; m += gridDim.x * blockDim.x) {
-    if (!flags[m]) continue;
+    if (counts[m] < theta) continue;
     uint32_t lo = 0, hi = n - 1;  // a = last row whose first pair index <= m
     while (lo + 1 < hi) {
       const uint32_t mid = (lo + hi) >> 1;
@@ -65,14 +71,14 @@ __global__ void scatter_pairs_kernel(const uint32_t* __restrict__ counts, const 
 }
 
 // k >= 3: candidate m = prefix[g] ++ ext[m] with g the group holding m
-__global__ void scatter_grouped_kernel(const uint32_t* __restrict__ counts, const uint32_t* __restrict__ flags,
+__global__ void scatter_grouped_kernel(const uint32_t* __restrict__ counts, uint32_t theta,
                                        const uint32_t* __restrict__ pos, uint32_t M,
                                        const uint32_t* __restrict__ prefix, const uint32_t* __restrict__ ext_off,
                                        const uint32_t* __restrict__ ext, uint32_t G, uint32_t km1,
                                        const uint32_t* __restrict__ gpar, const uint32_t* __restrict__ eidx,
                                        uint32_t* L, uint32_t* sup, uint32_t* par_a, uint32_t* par_b) {
   for (uint32_t m = blockIdx.x * blockDim.x + threadIdx.x; m < M; m += gridDim.x * blockDim.x) {
-    if (!flags[m]) continue;
+    if (counts[m] < theta) continue;
     uint32_t lo = 0, hi = G;  // g = last group with ext_off[g] <= m
     while (lo + 1 < hi) {
       const uint32_t mid = (lo + hi) >> 1;
@@ -90,19 +96,29 @@ __global__ void scatter_grouped_kernel(const uint32_t* __restrict__ counts, cons
   }
 }
 
-// run starts: members whose first w-1 items differ from the previous member's
-// (zero past the device count: the scans run over the host upper bound)
-__global__ void run_start_kernel(const uint32_t* __restrict__ L, uint32_t n, uint32_t w, uint32_t* flags,
-                                 const uint32_t* __restrict__ n_dev) {
+// run starts (members whose first w-1 items differ from the previous member's; zero past the
+// device count: the scans run over the host upper bound) in one launch: flags, their exclusive
+// scan run_ex, bound[r] = the first member of run r and bound[#runs] = |L| (the sentinel)
+__global__ void __launch_bounds__(sd::kScanThreads, 1) run_scan_kernel(const uint32_t* __restrict__ L, uint32_t n,
+                                                                       uint32_t w, uint32_t* __restrict__ flags,
+                                                                       uint32_t* __restrict__ run_ex,
+                                                                       uint32_t* __restrict__ bound,
+                                                                       const uint32_t* __restrict__ n_dev,
+                                                                       uint32_t* sflags, uint64_t* agg, uint64_t* inc,
+                                                                       uint32_t epoch) {
   const uint32_t ne = eff_n(n, n_dev);
-  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x)
-    flags[i] = i < ne && (i == 0 || lex_cmp(L + (uint64_t)(i - 1) * w, L + (uint64_t)i * w, w - 1) != 0);
-}
-
-__global__ void run_bound_kernel(const uint32_t* __restrict__ flags, const uint32_t* __restrict__ run_ex,
-                                 uint32_t n, uint32_t* bound) {
-  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x)
-    if (flags[i]) bound[run_ex[i]] = i;
+  sd::scan_tile<uint32_t>(
+      n,
+      [&](uint32_t i) {
+        const uint32_t f = i < ne && (i == 0 || lex_cmp(L + (uint64_t)(i - 1) * w, L + (uint64_t)i * w, w - 1) != 0);
+        flags[i] = f;
+        return f;
+      },
+      [&](uint32_t i, uint32_t e, uint32_t f) {
+        run_ex[i] = e;
+        if (f) bound[e] = i;
+      },
+      [&](uint32_t runs) { bound[runs] = ne; }, sflags, agg, inc, epoch);
 }
 
 // join + prune, one WARP per member x (lvl::join_warp)
@@ -124,26 +140,11 @@ __global__ void join_kernel(const uint32_t* __restrict__ L, uint32_t n, uint32_t
   }
 }
 
-// sizes on the device: tot[0] = sum of an exclusive scan (last scanned + last input)
-__global__ void total_kernel(const uint32_t* __restrict__ in, const uint32_t* __restrict__ ex, uint32_t n,
-                             uint32_t* tot) {
-  if (threadIdx.x == 0 && blockIdx.x == 0) *tot = ex[n - 1] + in[n - 1];
-}
-// bound[n_runs] = n (sentinel end of the last run)
-__global__ void bound_sentinel_kernel(const uint32_t* __restrict__ flags, const uint32_t* __restrict__ run_ex,
-                                      uint32_t n, uint32_t* bound, const uint32_t* __restrict__ n_dev) {
-  n = eff_n(n, n_dev);
-  if (threadIdx.x == 0 && blockIdx.x == 0) bound[n ? run_ex[n - 1] + flags[n - 1] : 0] = n;
-}
 // ext_off[G] = M
 __global__ void ext_end_kernel(const uint32_t* __restrict__ sizes, uint32_t* ext_off) {
   if (threadIdx.x == 0 && blockIdx.x == 0) ext_off[sizes[1]] = sizes[0];
 }
 
-__global__ void nonzero_kernel(const uint32_t* __restrict__ cnt, uint32_t n, uint32_t* flags) {
-  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x)
-    flags[i] = cnt[i] != 0;
-}
 
 // L_k's rows -> item ids (n = entries x k words) and, with sup_in, its supports copied to sup_out;
 // a device-sized level stops at its count
@@ -166,12 +167,16 @@ unsigned grid_for(uint64_t n, int n_sms) {
 // exclusive scan of n u32 into out, total written to *tot on the device (no host sync)
 void exclusive_scan(const uint32_t* in, uint32_t* out, uint32_t n, uint32_t* tot, DeviceScratch& scratch,
                     cudaStream_t s) {
-  size_t bytes = 0;
-  GPA_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, bytes, in, out, n, s));
-  void* tmp = scratch.get(bytes, s);
-  GPA_CUDA(cub::DeviceScan::ExclusiveSum(tmp, bytes, in, out, n, s));
-  note_launch(2);  // CUB: init + scan kernels
-  if (tot) { total_kernel<<<1, 32, 0, s>>>(in, out, n, tot); note_launch(); }
+  scan_excl_u32(in, out, n, tot, scratch.scan, s);   // one launch, total included (scan.cu)
+}
+
+void ge_scan(const uint32_t* counts, uint32_t M, uint32_t theta, uint32_t* pos, uint32_t* count, DeviceScratch& scratch,
+             cudaStream_t s) {
+  const uint32_t tiles = scan_tiles(M);
+  const uint32_t ep = scan_epoch(scratch.scan, tiles, s);
+  { ge_scan_kernel<<<tiles, sd::kScanThreads, 0, s>>>(counts, M, theta, pos, count, scratch.scan.flags.p,
+                                                      scratch.scan.agg.p, scratch.scan.inc.p, ep); note_launch(); }
+  GPA_CUDA(cudaGetLastError());
 }
 
 }  // namespace
@@ -181,21 +186,18 @@ void threshold_impl(const uint32_t* counts, uint32_t M, uint32_t theta, uint32_t
                     const uint32_t* prefix, const uint32_t* ext_off, const uint32_t* ext, uint32_t G,
                     const uint32_t* gpar, const uint32_t* eidx, DeviceLevel& out, DeviceScratch& scratch, int n_sms,
                     cudaStream_t s, uint32_t cap) {
-  uint32_t* flags = scratch.u32a(M, s);
   uint32_t* pos = scratch.u32b(M, s);
-  { flag_ge_kernel<<<grid_for(M, n_sms), kThreads, 0, s>>>(counts, M, theta, flags); note_launch(); }
-  GPA_CUDA(cudaGetLastError());
   out.count.ensure(1, s);
-  exclusive_scan(flags, pos, M, out.count.p, scratch, s);
+  ge_scan(counts, M, theta, pos, out.count.p, scratch, s);
   out.rows.ensure((size_t)std::max<uint32_t>(cap, 1) * k, s);
   out.sup.ensure(std::max<uint32_t>(cap, 1), s);
   out.par_a.ensure(std::max<uint32_t>(cap, 1), s);
   out.par_b.ensure(std::max<uint32_t>(cap, 1), s);
   if (k == 2)
-    { scatter_pairs_kernel<<<grid_for(M, n_sms), kThreads, 0, s>>>(counts, flags, pos, M, n_rows, sel, out.rows.p,
+    { scatter_pairs_kernel<<<grid_for(M, n_sms), kThreads, 0, s>>>(counts, theta, pos, M, n_rows, sel, out.rows.p,
                                                                 out.sup.p, out.par_a.p, out.par_b.p); note_launch(); }
   else
-    { scatter_grouped_kernel<<<grid_for(M, n_sms), kThreads, 0, s>>>(counts, flags, pos, M, prefix, ext_off, ext, G,
+    { scatter_grouped_kernel<<<grid_for(M, n_sms), kThreads, 0, s>>>(counts, theta, pos, M, prefix, ext_off, ext, G,
                                                                   k - 1, gpar, eidx, out.rows.p, out.sup.p,
                                                                   out.par_a.p, out.par_b.p); note_launch(); }
   GPA_CUDA(cudaGetLastError());
@@ -212,11 +214,9 @@ uint32_t device_threshold(const uint32_t* counts, uint32_t M, uint32_t theta, ui
   out.n_max = 0;
   if (M == 0) return 0;
   // |L_k| first (one synchronisation), then L_k at its exact size
-  uint32_t* flags = scratch.u32a(M, s);
   uint32_t* pos = scratch.u32b(M, s);
-  { flag_ge_kernel<<<grid_for(M, n_sms), kThreads, 0, s>>>(counts, M, theta, flags); note_launch(); }
   out.count.ensure(1, s);
-  exclusive_scan(flags, pos, M, out.count.p, scratch, s);
+  ge_scan(counts, M, theta, pos, out.count.p, scratch, s);
   uint32_t F = 0;
   GPA_CUDA(cudaMemcpyAsync(&F, out.count.p, 4, cudaMemcpyDeviceToHost, s));
   stream_wait(s);
@@ -267,11 +267,15 @@ bool device_candgen_begin(const DeviceLevel& L, DeviceBatch& out, DeviceScratch&
   uint32_t* cnt = scratch.u32c(n, s);
   uint32_t* bound = scratch.u32d(n + 1, s);
   uint32_t* sizes = scratch.u32h(4, s);  // [0] = M, [1] = G
-  { run_start_kernel<<<grid_for(n, n_sms), kThreads, 0, s>>>(L.rows.p, n, w, flags, n_dev); note_launch(); }
+  {
+    const uint32_t tiles = scan_tiles(n);
+    const uint32_t ep = scan_epoch(scratch.scan, tiles, s);
+    run_scan_kernel<<<tiles, sd::kScanThreads, 0, s>>>(L.rows.p, n, w, flags, run_ex, bound, n_dev,
+                                                       scratch.scan.flags.p, scratch.scan.agg.p, scratch.scan.inc.p,
+                                                       ep);
+    note_launch();
+  }
   GPA_CUDA(cudaGetLastError());
-  exclusive_scan(flags, run_ex, n, nullptr, scratch, s);
-  { run_bound_kernel<<<grid_for(n, n_sms), kThreads, 0, s>>>(flags, run_ex, n, bound); note_launch(); }
-  { bound_sentinel_kernel<<<1, 32, 0, s>>>(flags, run_ex, n, bound, n_dev); note_launch(); }
   // hash set over L for the prune probes
   uint32_t cap = 16;
   while (cap < 2 * n + 1) cap <<= 1;
@@ -283,11 +287,9 @@ bool device_candgen_begin(const DeviceLevel& L, DeviceBatch& out, DeviceScratch&
         cap - 1, cnt, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, n_dev); note_launch(); }
   GPA_CUDA(cudaGetLastError());
   uint32_t* cand_off = scratch.u32e(n, s);
-  uint32_t* gflag = scratch.u32f(n, s);
   uint32_t* gidx = scratch.u32g(n, s);
-  exclusive_scan(cnt, cand_off, n, sizes, scratch, s);
-  { nonzero_kernel<<<grid_for(n, n_sms), kThreads, 0, s>>>(cnt, n, gflag); note_launch(); }
-  exclusive_scan(gflag, gidx, n, sizes + 1, scratch, s);
+  // candidate offsets and group indices in one scan: sizes = {M, G}
+  scan_excl_split(cnt, cand_off, gidx, n, sizes, scratch.scan, s);
   *d_sizes = sizes;
   return true;
 }

@@ -34,11 +34,11 @@
 #include <cstdint>
 #include <cstdlib>
 #include <map>
-#include <cub/device/device_scan.cuh>
 
 #include "../common.h"
 #include "../kernels.h"
 #include "proj_dev.cuh"
+#include "scan_dev.cuh"
 
 namespace gpa {
 namespace {
@@ -55,25 +55,34 @@ unsigned grid_for(uint64_t n, int n_sms, int per_sm = 16) {
 // A class = a run of entries with the same par_a (the left parent = the (k-2)-prefix).
 // n_dev (device-sized level): the entry count lives on the device, n is its host upper bound; the
 // flags are zero past the count (the scans run over n)
-__global__ void cls_flag_kernel(const uint32_t* __restrict__ par_a, uint32_t n, uint32_t* __restrict__ flag,
-                                const uint32_t* __restrict__ n_dev) {
+// class starts (entries whose left parent differs from the previous entry's; zero past the device
+// count) in one launch: flag, its exclusive scan ex, bound[c] = the first entry of class c,
+// bound[#classes] = |L| and *n_cls = #classes
+__global__ void __launch_bounds__(sd::kScanThreads, 1) cls_scan_kernel(const uint32_t* __restrict__ par_a, uint32_t n,
+                                                                       uint32_t* __restrict__ flag,
+                                                                       uint32_t* __restrict__ ex,
+                                                                       uint32_t* __restrict__ bound,
+                                                                       uint32_t* __restrict__ n_cls,
+                                                                       const uint32_t* __restrict__ n_dev,
+                                                                       uint32_t* sflags, uint64_t* agg, uint64_t* inc,
+                                                                       uint32_t epoch) {
   const uint32_t ne = n_dev ? min(*n_dev, n) : n;
-  for (uint32_t j = blockIdx.x * blockDim.x + threadIdx.x; j < n; j += gridDim.x * blockDim.x)
-    flag[j] = j < ne && (j == 0 || par_a[j] != par_a[j - 1]);
-}
-
-__global__ void cls_bound_kernel(const uint32_t* __restrict__ flag, const uint32_t* __restrict__ ex, uint32_t n,
-                                 uint32_t* __restrict__ bound, uint32_t* __restrict__ n_cls,
-                                 const uint32_t* __restrict__ n_dev) {
-  n = n_dev ? min(*n_dev, n) : n;   // n_cls stays 0 (zeroed by the caller) when the level is empty
-  for (uint32_t j = blockIdx.x * blockDim.x + threadIdx.x; j < n; j += gridDim.x * blockDim.x) {
-    if (flag[j]) bound[ex[j]] = j;
-    if (j == n - 1) {
-      const uint32_t C = ex[j] + flag[j];
-      bound[C] = n;
-      *n_cls = C;
-    }
-  }
+  sd::scan_tile<uint32_t>(
+      n,
+      [&](uint32_t j) {
+        const uint32_t f = j < ne && (j == 0 || par_a[j] != par_a[j - 1]);
+        flag[j] = f;
+        return f;
+      },
+      [&](uint32_t j, uint32_t e, uint32_t f) {
+        ex[j] = e;
+        if (f) bound[e] = j;
+      },
+      [&](uint32_t C) {
+        bound[C] = ne;
+        *n_cls = C;
+      },
+      sflags, agg, inc, epoch);
 }
 
 __global__ void seg_popc_kernel(Src src, const uint32_t* __restrict__ par_a, const uint32_t* __restrict__ bound,
@@ -572,24 +581,7 @@ __global__ void __launch_bounds__(kT) count_proj_kernel(const uint32_t* __restri
   }
 }
 
-template <class T>
-void scan_excl(const T* in, T* out, uint32_t n, PBuf<uint8_t>& tmpbuf, cudaStream_t s) {
-  size_t bytes = 0;
-  GPA_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, bytes, in, out, n, s));
-  void* tmp = tmpbuf.ensure(bytes);
-  GPA_CUDA(cub::DeviceScan::ExclusiveSum(tmp, bytes, in, out, n, s));
-  note_launch(2);
-}
 
-// totals: tot[0] = pext items, tot[1] = vector words
-__global__ void proj_totals_kernel(const uint32_t* __restrict__ items, const uint32_t* __restrict__ item_off,
-                                   uint32_t n_pairs, const uint64_t* __restrict__ cw, const uint64_t* __restrict__ cb,
-                                   uint32_t cmax, uint64_t* __restrict__ tot) {
-  if (threadIdx.x == 0 && blockIdx.x == 0) {
-    tot[0] = (uint64_t)item_off[n_pairs - 1] + items[n_pairs - 1];
-    tot[1] = cb[cmax - 1] + cw[cmax - 1];
-  }
-}
 
 // generation 3 by bit gather (pext3_kernel); GPA_PROJ_K3_PEXT=1 keeps the set-bit-walk pext (comparisons)
 bool gather3() {
@@ -605,7 +597,7 @@ bool gather3() {
 struct ProjWork {
   PBuf<uint32_t> flag, ex, bound, small, words, loc, items, item_off, item_pair, nwc;
   PBuf<uint64_t> cls_words, cls_base, tot;
-  PBuf<uint8_t> tmp;   // CUB temporary storage of its own: proj_build_begin may run beside the join's scans
+  ScanState scan;      // scan status words of its own: proj_build_begin runs beside the join's scans
   DeviceProj lists[2];
 };
 ProjWork& work_for(int device) {
@@ -664,10 +656,13 @@ bool proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, 
   W.bound.ensure(n + 1);
   W.small.ensure(4);
   GPA_CUDA(cudaMemsetAsync(W.small.p, 0, 16, s));
-  { cls_flag_kernel<<<grid_for(n, n_sms), kT, 0, s>>>(par_a, n, W.flag.p, n_dev); note_launch(); }
-  scan_excl<uint32_t>(W.flag.p, W.ex.p, n, W.tmp, s);
-  { cls_bound_kernel<<<grid_for(n, n_sms), kT, 0, s>>>(W.flag.p, W.ex.p, n, W.bound.p, W.small.p, n_dev);
-    note_launch(); }
+  {
+    const uint32_t tiles = scan_tiles(n);
+    const uint32_t ep = scan_epoch(W.scan, tiles, s);
+    cls_scan_kernel<<<tiles, sd::kScanThreads, 0, s>>>(par_a, n, W.flag.p, W.ex.p, W.bound.p, W.small.p, n_dev,
+                                                       W.scan.flags.p, W.scan.agg.p, W.scan.inc.p, ep);
+    note_launch();
+  }
   W.words.ensure((size_t)n_pairs * 32);
   W.loc.ensure((size_t)n_pairs * 32);
   W.items.ensure(n_pairs);
@@ -690,10 +685,9 @@ bool proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, 
           W.words.p, W.bound.p, W.small.p, cmax, nseg, W.loc.p, W.nwc.p, W.cls_words.p, W.items.p, W.small.p + 1);
       note_launch(); }
   }
-  scan_excl<uint32_t>(W.items.p, W.item_off.p, n_pairs, W.tmp, s);
-  scan_excl<uint64_t>(W.cls_words.p, W.cls_base.p, cmax, W.tmp, s);
-  { proj_totals_kernel<<<1, 32, 0, s>>>(W.items.p, W.item_off.p, n_pairs, W.cls_words.p, W.cls_base.p, cmax,
-                                        W.tot.p); note_launch(); }
+  // tot = {pext items, list words}: the totals of the two scans
+  scan_excl_u32(W.items.p, W.item_off.p, n_pairs, W.tot.p, W.scan, s);
+  scan_excl_u64(W.cls_words.p, W.cls_base.p, cmax, W.tot.p + 1, W.scan, s);
   GPA_CUDA(cudaGetLastError());
   pp.d_tot = W.tot.p;
   pp.d_small = W.small.p;
