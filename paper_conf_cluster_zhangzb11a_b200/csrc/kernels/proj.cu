@@ -96,25 +96,42 @@ __global__ void cls_pad_kernel(const uint32_t* __restrict__ words, const uint32_
                                const uint32_t* __restrict__ n_cls, uint32_t cmax, uint32_t nseg,
                                uint32_t* __restrict__ loc, uint32_t* __restrict__ nwc,
                                uint64_t* __restrict__ cls_words, uint32_t* __restrict__ items,
-                               uint32_t* __restrict__ max_lw) {
+                               uint32_t* __restrict__ max_lw, uint32_t* __restrict__ len) {
   const uint32_t c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  if (c < cmax) cls_pad_warp(c, words, bound, *n_cls, cmax, nseg, loc, nwc, cls_words, items, max_lw);
+  if (c < cmax) cls_pad_warp(c, words, bound, *n_cls, cmax, nseg, loc, nwc, cls_words, items, max_lw, len);
 }
 
-// entry j -> its vector (offset, words); entries of single-member classes get none
+// warp per entry j: its vector (offset, words; entries of single-member classes get none), and
+// the words past what the list build writes zeroed -- lane-interleaved lists (k >= 4): lane l's
+// tail len[c][l] .. Lw_c - 1; natural-order lists (generation 3): len[c][0] .. nwc - 1
 __global__ void entry_off_kernel(const uint32_t* __restrict__ flag, const uint32_t* __restrict__ ex,
                                  const uint32_t* __restrict__ bound, const uint32_t* __restrict__ nwc,
                                  const uint64_t* __restrict__ cls_base, uint32_t n, uint64_t* __restrict__ off,
-                                 uint32_t* __restrict__ nw) {
-  for (uint32_t j = blockIdx.x * blockDim.x + threadIdx.x; j < n; j += gridDim.x * blockDim.x) {
+                                 uint32_t* __restrict__ nw, const uint32_t* __restrict__ len, bool natural,
+                                 uint32_t* __restrict__ data) {
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t n_warps = (gridDim.x * blockDim.x) >> 5;
+  for (uint32_t j = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; j < n; j += n_warps) {
     const uint32_t c = ex[j] + flag[j] - 1;
     const uint32_t j0 = bound[c], m = bound[c + 1] - j0;
     if (m < 2) {
-      off[j] = 0;
-      nw[j] = 0;
+      if (lane == 0) {
+        off[j] = 0;
+        nw[j] = 0;
+      }
+      continue;
+    }
+    const uint32_t w = nwc[c];
+    const uint64_t o = cls_base[c] + (uint64_t)(j - j0) * w;
+    if (lane == 0) {
+      nw[j] = w;
+      off[j] = o;
+    }
+    if (natural) {
+      const uint32_t i = len[(uint64_t)c * 32] + lane;
+      if (i < w) data[o + i] = 0u;
     } else {
-      nw[j] = nwc[c];
-      off[j] = cls_base[c] + (uint64_t)(j - j0) * nwc[c];
+      for (uint32_t jj = len[(uint64_t)c * 32 + lane]; jj < w / 32u; ++jj) data[o + 32ull * jj + lane] = 0u;
     }
   }
 }
@@ -292,10 +309,10 @@ __global__ void cls3_pad_kernel(const uint32_t* __restrict__ w3, const uint32_t*
                                 const uint32_t* __restrict__ n_cls, uint32_t cmax, uint32_t nseg,
                                 uint32_t* __restrict__ loc3, uint32_t* __restrict__ nwc,
                                 uint64_t* __restrict__ cls_words, uint32_t* __restrict__ items,
-                                uint32_t* __restrict__ max_lw) {
+                                uint32_t* __restrict__ max_lw, uint32_t* __restrict__ len) {
   const uint32_t C = *n_cls;
   for (uint32_t c = blockIdx.x * blockDim.x + threadIdx.x; c < cmax; c += gridDim.x * blockDim.x)
-    cls3_pad_thread(c, w3, bound, C, cmax, nseg, loc3, nwc, cls_words, items, max_lw);
+    cls3_pad_thread(c, w3, bound, C, cmax, nseg, loc3, nwc, cls_words, items, max_lw, len);
 }
 
 // pext3 per-warp shared memory: a ring of three chunk slots of member words (set bits carried over
@@ -595,7 +612,7 @@ bool gather3() {
 // per-thread, per-device persistent workspace (grow-only): the class tables of proj_build and the
 // two generations of lists
 struct ProjWork {
-  PBuf<uint32_t> flag, ex, bound, small, words, loc, items, item_off, item_pair, nwc;
+  PBuf<uint32_t> flag, ex, bound, small, words, loc, items, item_off, item_pair, nwc, len;
   PBuf<uint64_t> cls_words, cls_base, tot;
   ScanState scan;      // scan status words of its own: proj_build_begin runs beside the join's scans
   DeviceProj lists[2];
@@ -670,19 +687,21 @@ bool proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, 
   W.nwc.ensure(cmax);
   W.cls_words.ensure(cmax);
   W.cls_base.ensure(cmax);
+  W.len.ensure((size_t)cmax * 32);
   W.tot.ensure(2);
   const unsigned wpb = kT / 32;
   if (!prev && gather3()) {  // generation 3: bit gather (pext3_kernel), natural-order lists
     { seg3_kernel<<<(n_pairs + wpb - 1) / wpb, kT, 0, s>>>(rows, pitch_words, par_a, W.bound.p, W.small.p, cmax, n_pairs,
           W.words.p, reinterpret_cast<unsigned long long*>(W.small.p + 2)); note_launch(); }
     { cls3_pad_kernel<<<grid_for(cmax, n_sms), kT, 0, s>>>(W.words.p, W.bound.p, W.small.p, cmax, nseg, W.loc.p,
-          W.nwc.p, W.cls_words.p, W.items.p, W.small.p + 1); note_launch(); }
+          W.nwc.p, W.cls_words.p, W.items.p, W.small.p + 1, W.len.p); note_launch(); }
   } else {
     { seg_popc_kernel<<<(n_pairs + wpb - 1) / wpb, kT, 0, s>>>(
           src, par_a, W.bound.p, W.small.p, cmax, nseg, n_pairs, W.words.p,
           reinterpret_cast<unsigned long long*>(W.small.p + 2)); note_launch(); }
     { cls_pad_kernel<<<(cmax + wpb - 1) / wpb, kT, 0, s>>>(
-          W.words.p, W.bound.p, W.small.p, cmax, nseg, W.loc.p, W.nwc.p, W.cls_words.p, W.items.p, W.small.p + 1);
+          W.words.p, W.bound.p, W.small.p, cmax, nseg, W.loc.p, W.nwc.p, W.cls_words.p, W.items.p, W.small.p + 1,
+          W.len.p);
       note_launch(); }
   }
   // tot = {pext items, list words}: the totals of the two scans
@@ -722,10 +741,10 @@ bool proj_build_finish(const ProjPending& pp, const uint64_t T[2], const uint32_
   out.words = T[1];
   out.max_lw = sm[1];
   out.in_words = (uint64_t)sm[2] | ((uint64_t)sm[3] << 32);
-  // lanes shorter than their class' Lw keep a zero tail
-  GPA_CUDA(cudaMemsetAsync(out.data.p, 0, std::max<uint64_t>(T[1], 1) * 4, s));
-  { entry_off_kernel<<<grid_for(n, n_sms), kT, 0, s>>>(W.flag.p, W.ex.p, W.bound.p, W.nwc.p, W.cls_base.p, n,
-                                                      out.off.p, out.nw.p); note_launch(); }
+  // offsets, and the zero tails of lanes shorter than their class' Lw (the list build writes the rest)
+  { entry_off_kernel<<<grid_for(32ull * n, n_sms), kT, 0, s>>>(W.flag.p, W.ex.p, W.bound.p, W.nwc.p, W.cls_base.p, n,
+                                                              out.off.p, out.nw.p, W.len.p,
+                                                              !pp.prev && gather3(), out.data.p); note_launch(); }
   if (ev_build) GPA_CUDA(cudaEventRecord(ev_build, s));  // start of the list build proper
   if (T[0]) {
     W.item_pair.ensure(T[0]);

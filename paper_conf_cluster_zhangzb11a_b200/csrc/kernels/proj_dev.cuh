@@ -64,7 +64,7 @@ __device__ __forceinline__ void cls_pad_warp(uint32_t c, const uint32_t* __restr
                                              const uint32_t* __restrict__ bound, uint32_t n_cls, uint32_t cmax,
                                              uint32_t nseg, uint32_t* __restrict__ loc, uint32_t* __restrict__ nwc,
                                              uint64_t* __restrict__ cls_words, uint32_t* __restrict__ items,
-                                             uint32_t* __restrict__ max_lw) {
+                                             uint32_t* __restrict__ max_lw, uint32_t* __restrict__ len) {
   const uint32_t lane = threadIdx.x & 31;
   uint32_t m = 0;
   if (c < n_cls) m = bound[c + 1] - bound[c];
@@ -79,6 +79,7 @@ __device__ __forceinline__ void cls_pad_warp(uint32_t c, const uint32_t* __restr
     if (lane == 0) items[p] = any ? groups : 0;
   }
   const uint32_t lw = __reduce_max_sync(0xffffffffu, acc);
+  len[(uint64_t)c * 32 + lane] = acc;   // lane words written by pext: the rest up to lw is zeroed
   if (lane == 0) {
     nwc[c] = groups ? 32u * lw : 0u;
     cls_words[c] = groups ? (uint64_t)32u * lw * m : 0ull;
@@ -138,7 +139,7 @@ __device__ __forceinline__ void cls3_pad_thread(uint32_t c, const uint32_t* __re
                                                 const uint32_t* __restrict__ bound, uint32_t n_cls, uint32_t cmax,
                                                 uint32_t nseg, uint32_t* __restrict__ loc3, uint32_t* __restrict__ nwc,
                                                 uint64_t* __restrict__ cls_words, uint32_t* __restrict__ items,
-                                                uint32_t* __restrict__ max_lw) {
+                                                uint32_t* __restrict__ max_lw, uint32_t* __restrict__ len) {
   const uint32_t m = c < n_cls ? bound[c + 1] - bound[c] : 0;
   const uint32_t groups = m >= 2 ? (m + kG3Group - 1) / kG3Group : 0;
   uint32_t acc = 0;
@@ -149,6 +150,7 @@ __device__ __forceinline__ void cls3_pad_thread(uint32_t c, const uint32_t* __re
     items[p] = w3[p] ? groups : 0;
   }
   const uint32_t words = groups ? (acc + 31u) & ~31u : 0u;
+  len[(uint64_t)c * 32] = acc;   // words written by pext3: the rest up to `words` is zeroed
   nwc[c] = words;
   cls_words[c] = (uint64_t)words * m;
   if (words) atomicMax(max_lw, words / 32u);
