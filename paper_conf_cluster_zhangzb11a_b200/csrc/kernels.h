@@ -112,8 +112,9 @@ struct ScanState {
   PBuf<uint64_t> agg, inc;
   uint32_t epoch = 0;
 };
-// fused scans (scan_dev.cuh): tiles of a scan of n values, and the epoch of the next scan on st
-uint32_t scan_tiles(uint32_t n);
+// fused scans (scan_dev.cuh): tiles of a scan of n values (items per thread), and the epoch of
+// the next scan on st
+uint32_t scan_tiles(uint32_t n, uint32_t items = 8);
 uint32_t scan_epoch(ScanState& st, uint32_t tiles, cudaStream_t s);
 void scan_excl_u32(const uint32_t* in, uint32_t* out, uint32_t n, uint32_t* tot, ScanState& st, cudaStream_t s);
 void scan_excl_u32(const uint32_t* in, uint32_t* out, uint32_t n, uint64_t* tot, ScanState& st, cudaStream_t s);

@@ -21,6 +21,7 @@ namespace {
 using namespace lvl;
 
 constexpr int kThreads = 256;
+constexpr int kRunScanItems = 2;   // run detection compares two rows per member: more CTAs in flight
 
 // n_dev (device-sized levels): the member count lives on the device; n is its host upper bound
 __device__ __forceinline__ uint32_t eff_n(uint32_t n, const uint32_t* n_dev) { return n_dev ? min(*n_dev, n) : n; }
@@ -107,7 +108,7 @@ __global__ void __launch_bounds__(sd::kScanThreads, 1) run_scan_kernel(const uin
                                                                        uint32_t* sflags, uint64_t* agg, uint64_t* inc,
                                                                        uint32_t epoch) {
   const uint32_t ne = eff_n(n, n_dev);
-  sd::scan_tile<uint32_t>(
+  sd::scan_tile<uint32_t, kRunScanItems>(
       n,
       [&](uint32_t i) {
         const uint32_t f = i < ne && (i == 0 || lex_cmp(L + (uint64_t)(i - 1) * w, L + (uint64_t)i * w, w - 1) != 0);
@@ -268,7 +269,7 @@ bool device_candgen_begin(const DeviceLevel& L, DeviceBatch& out, DeviceScratch&
   uint32_t* bound = scratch.u32d(n + 1, s);
   uint32_t* sizes = scratch.u32h(4, s);  // [0] = M, [1] = G
   {
-    const uint32_t tiles = scan_tiles(n);
+    const uint32_t tiles = scan_tiles(n, kRunScanItems);
     const uint32_t ep = scan_epoch(scratch.scan, tiles, s);
     run_scan_kernel<<<tiles, sd::kScanThreads, 0, s>>>(L.rows.p, n, w, flags, run_ex, bound, n_dev,
                                                        scratch.scan.flags.p, scratch.scan.agg.p, scratch.scan.inc.p,

@@ -86,6 +86,49 @@ __device__ __forceinline__ void join_warp(uint32_t x, const uint32_t* __restrict
   }
   const uint64_t p_last = pw;  // P^(w-1)
   uint32_t here = 0;  // survivors so far (warp-uniform)
+  const uint32_t np = w - 1;   // prune probes per sibling: the subsets dropping item d < w - 1
+  if (np >= 1 && np <= 16) {
+    // probes spread over the lanes: lane = (sibling g, item d) for G = 32 / np siblings per round,
+    // so a round waits for ONE probe chain instead of np in sequence
+    const uint32_t G = 32u / np, d = lane % np, g = lane / np;
+    uint64_t hd = 0, pp = 1;   // A_d + B_d: the items of px without d at positions 0 .. w - 2
+    for (uint32_t i = 0; i < w; ++i) {
+      if (i == d) continue;
+      hd += (uint64_t)(px[i] + 1) * pp;
+      pp *= kHashP;
+    }
+    const uint32_t pmask = (1u << np) - 1u;
+    for (uint32_t y0 = x + 1; y0 < end; y0 += G) {
+      const uint32_t y = y0 + g;
+      const bool on = g < G && y < end;
+      uint32_t b = 0;
+      bool found = true;
+      if (on) {
+        b = L[(uint64_t)y * w + w - 1];
+        uint32_t h = (uint32_t)hash_mix(hd + (uint64_t)(b + 1) * p_last) & mask;
+        for (;;) {
+          const uint32_t i = slots[h];
+          if (i == kEmpty) {
+            found = false;
+            break;
+          }
+          if (row_is_sub(L + (uint64_t)i * w, px, w, d, b)) break;
+          h = (h + 1) & mask;
+        }
+      }
+      const uint32_t probes = __ballot_sync(0xffffffffu, found);
+      // sibling j (lane j < G) survives iff all its np probes hit
+      const uint32_t bj = __shfl_sync(0xffffffffu, b, (lane < G ? lane : 0u) * np);
+      const bool keep = lane < G && y0 + lane < end && ((probes >> (lane * np)) & pmask) == pmask;
+      const uint32_t ballot = __ballot_sync(0xffffffffu, keep);
+      if (EMIT && keep) {
+        const uint32_t at = cand_off[x] + here + __popc(ballot & ((1u << lane) - 1u));
+        ext[at] = bj;
+        eidx[at] = y0 + lane;
+      }
+      here += __popc(ballot);
+    }
+  } else
   for (uint32_t y0 = x + 1; y0 < end; y0 += 32) {
     const uint32_t y = y0 + lane;
     bool keep = y < end;

@@ -66,7 +66,10 @@ uint32_t scan_epoch(ScanState& st, uint32_t tiles, cudaStream_t s) {
   if (st.epoch == 0) st.epoch = 1;
   return st.epoch;
 }
-uint32_t scan_tiles(uint32_t n) { return (n + kScanTile - 1) / kScanTile; }
+uint32_t scan_tiles(uint32_t n, uint32_t items) {
+  const uint32_t tile = kScanThreads * items;
+  return (n + tile - 1) / tile;
+}
 
 namespace {
 

@@ -1,11 +1,13 @@
 // The single-launch exclusive scan's device part (scan.cu), for kernels that fuse their own input
 // transform / output side effects into the scan (candgen.cu, proj.cu).  Internal.
 //
-// CTA = tile of kScanTile values (256 threads x 8), block scan in registers + shuffles, the tile's
+// CTA = tile of 256 x ITEMS values (8 by default; fewer for input transforms with dependent loads,
+// so that more CTAs are in flight), block scan in registers + shuffles, the tile's
 // prefix by decoupled look-back over the earlier tiles' published aggregate / inclusive values.
 // The status words carry the scan's epoch (ScanState, one per stream), so no init pass clears them
 // between scans.  Tiles are blockIdx order: a tile only waits for lower-indexed tiles, which the
-// hardware dispatches first.  Launch: scan_tiles(n) CTAs of kScanThreads with scan_epoch()'s epoch.
+// hardware dispatches first.  Launch: scan_tiles(n, ITEMS) CTAs of kScanThreads with scan_epoch()'s
+// epoch.
 #pragma once
 #include <cstdint>
 #include "../common.h"
@@ -37,17 +39,17 @@ __device__ __forceinline__ T warp_incl(T v, uint32_t lane) {
 }
 
 // in(i): value of element i < n; out(i, exclusive prefix, value); tot(total) by the last tile
-template <class T, class In, class Out, class Tot>
+template <class T, int ITEMS = kScanItems, class In, class Out, class Tot>
 __device__ __forceinline__ void scan_tile(uint32_t n, In in, Out out, Tot tot, uint32_t* __restrict__ flags,
                                           uint64_t* __restrict__ agg, uint64_t* __restrict__ inc, uint32_t epoch) {
   __shared__ T s_warp[kScanThreads / 32];
   __shared__ T s_prefix;
   const uint32_t tile = blockIdx.x, lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const uint32_t base = tile * kScanTile + threadIdx.x * kScanItems;
-  T v[kScanItems];
+  const uint32_t base = tile * (kScanThreads * ITEMS) + threadIdx.x * ITEMS;
+  T v[ITEMS];
   T sum = 0;
 #pragma unroll
-  for (int j = 0; j < kScanItems; ++j) {
+  for (int j = 0; j < ITEMS; ++j) {
     v[j] = base + j < n ? in(base + j) : T(0);
     sum += v[j];
   }
@@ -106,7 +108,7 @@ __device__ __forceinline__ void scan_tile(uint32_t n, In in, Out out, Tot tot, u
   __syncthreads();
   T run = s_prefix + s_warp[warp] + (wi - sum);
 #pragma unroll
-  for (int j = 0; j < kScanItems; ++j) {
+  for (int j = 0; j < ITEMS; ++j) {
     if (base + j < n) out(base + j, run, v[j]);
     run += v[j];
   }

@@ -445,10 +445,12 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
         if (trace_enabled()) GPA_CUDA(cudaEventRecord(trace_ev[1], aux_s.s));
         GPA_CUDA(cudaMemcpyAsync(hs, d_sizes, 8, cudaMemcpyDeviceToHost, s));
         if (Ld.n_dev) GPA_CUDA(cudaMemcpyAsync(hs + 10, Ld.n_dev, 4, cudaMemcpyDeviceToHost, s));
+        if (trace_enabled()) GPA_CUDA(cudaEventRecord(trace_ev[2], s));
         const double tw0 = now_ms();
         stream_wait(s);
         stream_wait(aux_s.s);
         const double tw1 = now_ms();
+        if (trace_enabled()) GPA_CUDA(cudaEventRecord(trace_ev[3], s));
         M = hs[0];
         G = hs[1];
         std::memcpy(pT, hs + 2, 16);
@@ -458,16 +460,21 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
           Ld.n_dev = nullptr;
           finalize(pending.back(), Ld.n);
         }
+        const double tw2 = now_ms();
         ppend.n = Ld.n;   // the class tables ran over the upper bound; the lists are for |L_{k-1}| entries
         device_candgen_finish(Ld, Bd, scratch, bs->n_sms, s, (uint32_t)M, (uint32_t)G, aux_s.s, aux_evs.e[0]);
         GPA_CUDA(cudaEventRecord(aux_evs.e[1], aux_s.s));
         aux_join = true;
+        const double tw3 = now_ms();
         if (trace_enabled()) {
-          float ja = 0, jb = 0;
+          float ja = 0, jb = 0, jc = 0, jd = 0;
           GPA_CUDA(cudaEventElapsedTime(&ja, ev.e[5], trace_ev[0]));
           GPA_CUDA(cudaEventElapsedTime(&jb, ev.e[5], trace_ev[1]));
+          GPA_CUDA(cudaEventElapsedTime(&jc, ev.e[5], trace_ev[2]));
+          GPA_CUDA(cudaEventElapsedTime(&jd, ev.e[5], trace_ev[3]));
           fprintf(stderr, "[gpa] k=%u host: enqueue %.3f, wait %.3f, after wait %.3f ms; device: join stage 1 %.3f, "
-                  "class tables %.3f ms\n", k, tw0 - t0, tw1 - tw0, now_ms() - tw1, ja, jb);
+                  "class tables + sizes %.3f, sizes on s %.3f, host awake %.3f ms (finalize %.3f, finish %.3f)\n", k,
+                  tw0 - t0, tw1 - tw0, now_ms() - tw1, ja, jb, jc, jd, tw2 - tw1, tw3 - tw2);
         }
       }
     } else {
