@@ -16,11 +16,34 @@
 #include "internal.h"
 #include "pool.h"
 
+// Allocator whose resize() leaves new elements uninitialised: F (tens of MB) is filled by parallel
+// copies right after the resize, so a zero-fill would be a serial pass (and every page fault on a
+// single thread) for nothing.
+template <class T>
+struct DefaultInitAlloc : std::allocator<T> {
+  template <class U>
+  struct rebind {
+    using other = DefaultInitAlloc<U>;
+  };
+  DefaultInitAlloc() = default;
+  template <class U>
+  DefaultInitAlloc(const DefaultInitAlloc<U>&) noexcept {}
+  template <class U>
+  void construct(U* p) noexcept {
+    ::new (static_cast<void*>(p)) U;
+  }
+  template <class U, class... A>
+  void construct(U* p, A&&... a) {
+    ::new (static_cast<void*>(p)) U(std::forward<A>(a)...);
+  }
+};
+using FVec = std::vector<uint32_t, DefaultInitAlloc<uint32_t>>;
+
 struct gpa_level_data {
   uint32_t k = 0;
   uint64_t n_cand = 0, n_freq = 0, n_groups = 0;
-  std::vector<uint32_t> freq_items;    // n_freq * k, original ids, lexicographic
-  std::vector<uint32_t> freq_support;  // n_freq
+  FVec freq_items;                     // n_freq * k, original ids, lexicographic
+  FVec freq_support;                   // n_freq
   std::vector<uint32_t> cand_items;    // n_cand * k (GPA_KEEP_CANDIDATES)
   std::vector<uint32_t> cand_counts;   // n_cand     (GPA_KEEP_CANDIDATES)
   bool kept = false;
@@ -47,7 +70,7 @@ double now_ms() {
 // GPA_KEEP_CANDIDATES the whole C_k (the host batch b, or all pairs for k = 2) and its counts
 // are recorded as well.
 void record_level(gpa_result* R, const gpa_bitset* bs, uint32_t k, const GroupedBatch* b, uint64_t M,
-                  std::vector<uint32_t>&& Litems, std::vector<uint32_t>&& Lsup, bool keep,
+                  FVec&& Litems, FVec&& Lsup, bool keep,
                   const std::vector<uint32_t>* counts) {
   gpa_level_data lv;
   lv.k = k;
