@@ -570,24 +570,55 @@ __global__ void __launch_bounds__(kT) count_proj_kernel(const uint32_t* __restri
       const bool h0 = w0 < n, h1 = w1 < n;
       const uint4 x0 = h0 ? *reinterpret_cast<const uint4*>(X + w0) : make_uint4(0, 0, 0, 0);
       const uint4 x1 = h1 ? *reinterpret_cast<const uint4*>(X + w1) : make_uint4(0, 0, 0, 0);
-      for (uint32_t i = 0; i < nb; i += 2) {
-        uint32_t c = 0;
+      if constexpr (WARP) {   // short lists, few siblings: two at a time
+        for (uint32_t i = 0; i < nb; i += 2) {
+          uint32_t c = 0;
 #pragma unroll
-        for (uint32_t q = 0; q < 2; ++q) {
-          if (i + q < nb) {
-            const uint64_t yo = __shfl_sync(0xffffffffu, my_off, i + q);
-            const uint32_t* Y = data + yo;
-            const uint4 y0 = h0 ? *reinterpret_cast<const uint4*>(Y + w0) : make_uint4(0, 0, 0, 0);
-            const uint4 y1 = h1 ? *reinterpret_cast<const uint4*>(Y + w1) : make_uint4(0, 0, 0, 0);
+          for (uint32_t q = 0; q < 2; ++q) {
+            if (i + q < nb) {
+              const uint64_t yo = __shfl_sync(0xffffffffu, my_off, i + q);
+              const uint32_t* Y = data + yo;
+              const uint4 y0 = h0 ? *reinterpret_cast<const uint4*>(Y + w0) : make_uint4(0, 0, 0, 0);
+              const uint4 y1 = h1 ? *reinterpret_cast<const uint4*>(Y + w1) : make_uint4(0, 0, 0, 0);
+              const uint32_t v = __popc(x0.x & y0.x) + __popc(x0.y & y0.y) + __popc(x0.z & y0.z) +
+                                 __popc(x0.w & y0.w) + __popc(x1.x & y1.x) + __popc(x1.y & y1.y) +
+                                 __popc(x1.z & y1.z) + __popc(x1.w & y1.w);
+              c |= v << (16 * q);
+            }
+          }
+          c = __reduce_add_sync(0xffffffffu, c);
+          if (lane == i) acc += c & 0xffffu;
+          if (lane == i + 1) acc += c >> 16;
+        }
+        continue;
+      }
+      // long lists: 4 siblings per step, their 8 loads issued together, then two packed reductions
+      for (uint32_t i = 0; i < nb; i += 4) {
+        uint4 ya[4], yb[4];
+#pragma unroll
+        for (uint32_t q = 0; q < 4; ++q) {
+          const uint64_t yo = __shfl_sync(0xffffffffu, my_off, (i + q) & 31u);
+          const bool ok = i + q < nb;
+          const uint32_t* Y = data + yo;
+          ya[q] = ok && h0 ? *reinterpret_cast<const uint4*>(Y + w0) : make_uint4(0, 0, 0, 0);
+          yb[q] = ok && h1 ? *reinterpret_cast<const uint4*>(Y + w1) : make_uint4(0, 0, 0, 0);
+        }
+#pragma unroll
+        for (uint32_t pq = 0; pq < 4; pq += 2) {
+          if (i + pq >= nb) break;   // warp-uniform
+          uint32_t c = 0;
+#pragma unroll
+          for (uint32_t q = 0; q < 2; ++q) {
+            const uint4 y0 = ya[pq + q], y1 = yb[pq + q];
             const uint32_t v = __popc(x0.x & y0.x) + __popc(x0.y & y0.y) + __popc(x0.z & y0.z) +
                                __popc(x0.w & y0.w) + __popc(x1.x & y1.x) + __popc(x1.y & y1.y) +
                                __popc(x1.z & y1.z) + __popc(x1.w & y1.w);
             c |= v << (16 * q);
           }
+          c = __reduce_add_sync(0xffffffffu, c);
+          if (lane == i + pq) acc += c & 0xffffu;
+          if (lane == i + pq + 1) acc += c >> 16;
         }
-        c = __reduce_add_sync(0xffffffffu, c);
-        if (lane == i) acc += c & 0xffffu;
-        if (lane == i + 1) acc += c >> 16;
       }
     }
     if (WARP) {
