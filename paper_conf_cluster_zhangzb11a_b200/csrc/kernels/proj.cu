@@ -315,113 +315,131 @@ __global__ void cls3_pad_kernel(const uint32_t* __restrict__ w3, const uint32_t*
     cls3_pad_thread(c, w3, bound, C, cmax, nseg, loc3, nwc, cls_words, items, max_lw, len);
 }
 
-// pext3 per-warp shared memory: a ring of three chunk slots of member words (set bits carried over
-// from chunk j - 1 still read its slot while chunk j's are packed and chunk j + 1's are stored),
-// the members' row / list offsets and the staged set bits not yet packed.
-constexpr uint32_t kP3Warps = 4;
-constexpr uint32_t kP3Blocks = kG3Group <= 16 ? 6 : 4;  // blocks/SM (shared memory)
-// A staged set bit is (word index in xs) << 5 | bit.  Member rows are 33 words apart: column 32 of
-// every row stays zero, so kP3None (slot 0, column 32, bit 0) packs a 0 for every member.
-constexpr uint32_t kP3Row = 33;
-constexpr uint16_t kP3None = 32u << 5;
+// pext3 per-warp shared memory: two stages of the group's member words of one 64-word chunk (the
+// chunk being packed, the next one arriving by cp.async) and the chunk's staged set bits.
+constexpr uint32_t kP3Warps = 8;
+constexpr uint32_t kP3Blocks = 3;     // blocks/SM (shared memory: 8 x 9.3 KB per block)
+constexpr uint32_t kP3Chunk = 64;     // mask words per chunk: two per lane
+constexpr uint32_t kP3Pos = 512;      // staged set bits per pass (a chunk holds up to 2,048)
 struct P3Warp {
-  uint32_t xs[3][kG3Group][kP3Row];
-  uint32_t so[kG3Group];    // member row: word offset of its bitset row
-  uint32_t oo[kG3Group];    // member list: word offset in data
-  uint16_t pos[1024 + 32];  // staged set bits not yet packed
+  uint32_t xs[2][kG3Group][kP3Chunk];  // member q's words of the chunk
+  uint16_t pos[kP3Pos];                // a pass of the chunk's set bits in rank order: word << 5 | bit
+  uint32_t oo[kG3Group];               // member list: word offset in data
 };
 
+__device__ __forceinline__ void cp_async16(uint32_t dst, const void* src) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst), "l"(src) : "memory");
+}
+
+// One item of pext3_kernel: a group of nm <= G members of a class over the mask segment's chunks
+// [ca, cb) (64 words each).  Per chunk: lane l holds mask words 2l, 2l + 1; a warp scan of their
+// popcounts ranks the chunk's C set bits, which are staged in rank order; output words are packed
+// by ballots over ranks.  Set bits carry across chunks: the word of a chunk's last pend (< 32) bits
+// is gathered at once (lanes >= pend vote 0) and stays in its output slot, and the next chunk's
+// first ballot ORs its bits in at lanes pend .. 31 -- the segment's bits are packed densely,
+// ceil(bits / 32) words (seg3_warp), and no chunk's words are needed after the chunk.  Per member
+// and output word: LDS + LOP3 (-> predicate) + VOTE + LOP3 (into lane slot's register).
 template <uint32_t G>
 __device__ __forceinline__ void pext3_item(P3Warp& w, const uint32_t* __restrict__ mrow,
-                                           const uint32_t* __restrict__ rows, uint32_t nm, uint32_t ja,
-                                           uint32_t jb, uint32_t ow0, uint32_t* __restrict__ data) {
+                                           const uint32_t* __restrict__ rows, uint32_t so_l, uint32_t nm,
+                                           uint32_t ca, uint32_t cb, uint32_t ow0, uint32_t* __restrict__ data) {
+  static_assert(G % 2 == 0 && G <= kG3Group, "members are staged two per cp.async instruction");
   const uint32_t lane = threadIdx.x & 31;
-  uint32_t* xsl = &w.xs[0][0][lane];
-  if (lane < G) w.xs[0][lane][32] = 0u;  // the zero column kP3None reads
-  uint32_t xn[G], keep[G];
+  // lane l stages 16 bytes of member 2i + (l >> 4): words 4 (l & 15) .. + 3 of the chunk
+  uint32_t my_so[G / 2];
+#pragma unroll
+  for (uint32_t i = 0; i < G / 2; ++i) my_so[i] = __shfl_sync(0xffffffffu, so_l, 2 * i + (lane >> 4)) + 4u * (lane & 15u);
+  const uint32_t xs_lane = (uint32_t)__cvta_generic_to_shared(&w.xs[0][lane >> 4][4u * (lane & 15u)]);
+  auto stage = [&](uint32_t c, uint32_t st) {
+    const uint32_t* cur = rows + (uint64_t)c * kP3Chunk;
+    const uint32_t dst = xs_lane + st * (uint32_t)sizeof(w.xs[0]);
+#pragma unroll
+    for (uint32_t i = 0; i < G / 2; ++i) cp_async16(dst + i * 2u * kP3Chunk * 4u, addr4(cur, my_so[i]));
+    asm volatile("cp.async.commit_group;" ::: "memory");
+  };
+  uint32_t keep[G];
 #pragma unroll
   for (uint32_t q = 0; q < G; ++q) keep[q] = 0;
-  uint32_t wc = 0;      // words packed in this segment (warp-uniform)
-  uint32_t pend = 0;    // staged set bits not yet packed, < 32 between chunks (P3Carry)
-  bool old = false;     // some of them are from the chunk before the last one
-
-  const uint32_t* mp = mrow + 32u * ja;
-  const uint32_t* cur = rows + 32u * ja;
-  uint32_t mn = __ldg(mp);
-#pragma unroll
-  for (uint32_t q = 0; q < G; ++q) xn[q] = __ldg(addr4(cur, w.so[q]));  // slots >= nm: member 0 again
-  uint32_t slot = 0;
-  // j == jb: a last step that only flushes the set bits still pending
-  for (uint32_t j = ja; j <= jb; ++j) {
-    const bool real = j < jb;
-    uint32_t mw = 0;
-    if (real) {
-#pragma unroll
-      for (uint32_t q = 0; q < G; ++q) xsl[(slot * kG3Group + q) * kP3Row] = xn[q];
-      mw = mn;
-      if (j + 1 < jb) {  // chunk j + 1's words in flight while chunk j is packed
-        mp += 32;
-        cur += 32;
-        mn = __ldg(mp);
-#pragma unroll
-        for (uint32_t q = 0; q < G; ++q) xn[q] = __ldg(addr4(cur, w.so[q]));
-      }
+  uint32_t wc = 0;    // whole words packed in this segment (warp-uniform)
+  uint32_t pend = 0;  // set bits in the open word (slot wc & 31), < 32
+  stage(ca, 0);
+  const uint2* mp = reinterpret_cast<const uint2*>(mrow) + lane;
+  uint2 mn = __ldg(mp + (uint64_t)ca * (kP3Chunk / 2));
+  for (uint32_t c = ca; c < cb; ++c) {
+    const uint32_t st = (c - ca) & 1u;
+    const uint2 m = mn;
+    asm volatile("cp.async.wait_group 0;" ::: "memory");
+    __syncwarp();  // chunk c's member words visible to the warp; chunk c - 1's reads are done
+    if (c + 1 < cb) {
+      stage(c + 1, st ^ 1u);
+      mn = __ldg(mp + (uint64_t)(c + 1) * (kP3Chunk / 2));
     }
-    // pending bits of chunk j - 2 (their slot takes chunk j + 1), or at the end: one partial word
-    uint32_t base = pend;
-    if (pend && (old || !real)) {
-      if (lane >= pend) w.pos[lane] = kP3None;
-      base = 32;
-    }
-    // ranks of this lane's set bits among the chunk's: warp scan of the popcounts
-    const uint32_t c = __popc(mw);
-    uint32_t o = c;
+    // ranks of this lane's set bits: warp scan of the popcounts
+    const uint32_t cnt = __popc(m.x) + __popc(m.y);
+    uint32_t o = cnt;
 #pragma unroll
     for (uint32_t d = 1; d < 32; d <<= 1) {
       const uint32_t t = __shfl_up_sync(0xffffffffu, o, d);
       if (lane >= d) o += t;
     }
-    const uint32_t C = __shfl_sync(0xffffffffu, o, 31);
-    o += base - c;
-    const uint32_t tag = (slot * kG3Group * kP3Row + lane) << 5;
-    uint16_t* pp = &w.pos[o];
-    for (uint32_t mm = mw; mm; mm &= mm - 1u) *pp++ = (uint16_t)(tag | (uint32_t)(__ffs(mm) - 1));
-    __syncwarp();  // chunk j's member words and set bits visible to the warp
-    const uint32_t t = base + C, nr = t >> 5;
-    for (uint32_t r = 0; r < nr; ++r) {  // one output word per member from set bits 32 r .. 32 r + 31
-      const uint32_t v = w.pos[32u * r + lane];
-      const uint32_t* xb = &w.xs[0][0][0] + (v >> 5);
-      const uint32_t bm = 1u << (v & 31u);
-      const bool mine = lane == (wc & 31u);
-#pragma unroll
-      for (uint32_t q = 0; q < G; ++q) {
-        const uint32_t b = __ballot_sync(0xffffffffu, (xb[q * kP3Row] & bm) != 0u);
-        if (mine) keep[q] = b;
+    const uint32_t Call = __shfl_sync(0xffffffffu, o, 31);
+    // the chunk's set bits in passes of at most kP3Pos ranks (one pass below 25 % density)
+    for (uint32_t lo = 0; lo < Call; lo += kP3Pos) {
+      const uint32_t C = min(Call - lo, kP3Pos);
+      {
+        // 32-bit walks (a 64-bit one costs ~2.5x the instructions per set bit)
+        const uint32_t code0 = lane * 64u;
+        if (Call <= kP3Pos) {
+          uint16_t* pp = &w.pos[o - cnt];
+          for (uint32_t mm = m.x; mm; mm &= mm - 1u) *pp++ = (uint16_t)(code0 + (uint32_t)(__ffs(mm) - 1));
+          for (uint32_t mm = m.y; mm; mm &= mm - 1u) *pp++ = (uint16_t)(code0 + 31u + (uint32_t)__ffs(mm));
+        } else {   // dense chunk: only the ranks of this pass
+          uint32_t r = o - cnt - lo;
+          for (uint32_t mm = m.x; mm; mm &= mm - 1u, ++r)
+            if (r < C) w.pos[r] = (uint16_t)(code0 + (uint32_t)(__ffs(mm) - 1));
+          for (uint32_t mm = m.y; mm; mm &= mm - 1u, ++r)
+            if (r < C) w.pos[r] = (uint16_t)(code0 + 31u + (uint32_t)__ffs(mm));
+        }
       }
-      if ((wc & 31u) == 31u) {
-#pragma unroll
-        for (uint32_t q = 0; q < G; ++q)
-          if (q < nm) data[w.oo[q] + ow0 + (wc - 31u) + lane] = keep[q];
-      }
-      ++wc;
-    }
-    pend = t & 31u;
-    old = pend > C;
-    if (nr && pend) {
-      const uint32_t v = lane < pend ? w.pos[32u * nr + lane] : 0u;
       __syncwarp();
-      if (lane < pend) w.pos[lane] = (uint16_t)v;
-    }
-    __syncwarp();
-    slot = slot == 2u ? 0u : slot + 1u;
-  }
-  if (wc & 31u) {
-    const uint32_t base = wc & ~31u;
-    if (lane < (wc & 31u)) {
+      const uint32_t tot = pend + C, full = tot >> 5;
+      const uint32_t nb = full + ((tot & 31u) ? 1u : 0u);
+      const uint32_t* xst = &w.xs[st][0][0];
+      for (uint32_t t = 0; t < nb; ++t) {
+        // lane r takes the pass' set bit of rank 32 t + r - pend (none outside [0, C))
+        const int rank = (int)(32u * t + lane) - (int)pend;
+        const bool valid = rank >= 0 && rank < (int)C;
+        const uint32_t code = w.pos[valid ? rank : 0];
+        const uint32_t bm = valid ? 1u << (code & 31u) : 0u;
+        const uint32_t* xb = xst + (code >> 5);
+        const uint32_t sel = lane == (wc & 31u) ? 0xffffffffu : 0u;
 #pragma unroll
-      for (uint32_t q = 0; q < G; ++q)
-        if (q < nm) data[w.oo[q] + ow0 + base + lane] = keep[q];
+        for (uint32_t q = 0; q < G; ++q) {
+          const uint32_t b = __ballot_sync(0xffffffffu, (xb[q * kP3Chunk] & bm) != 0u);
+          uint32_t r;
+          asm("lop3.b32 %0, %1, %2, %3, 0xF8;" : "=r"(r) : "r"(keep[q]), "r"(b), "r"(sel));  // keep | (b & sel)
+          keep[q] = r;
+        }
+        if (t < full) {  // a whole word: the next slot; 32 slots full -> one coalesced store per member
+          if ((++wc & 31u) == 0u) {
+#pragma unroll
+            for (uint32_t q = 0; q < G; ++q) {
+              if (q < nm) data[w.oo[q] + ow0 + (wc - 32u) + lane] = keep[q];
+              keep[q] = 0;
+            }
+          }
+        }
+      }
+      pend = tot & 31u;
+      __syncwarp();  // pos (and, after the chunk, this stage) are rewritten next
     }
+  }
+  // the last whole words and the open partial word (its high bits zero)
+  const uint32_t left = (wc & 31u) + (pend ? 1u : 0u);
+  if (lane < left) {
+#pragma unroll
+    for (uint32_t q = 0; q < G; ++q)
+      if (q < nm) data[w.oo[q] + ow0 + (wc & ~31u) + lane] = keep[q];
   }
 }
 
@@ -445,29 +463,25 @@ __global__ void __launch_bounds__(kP3Warps * 32, kP3Blocks) pext3_kernel(const u
   const uint32_t g = it - item_off[p];
   const uint32_t first = j0 + g * kG3Group;
   const uint32_t nm = min(kG3Group, m - g * kG3Group);
-  uint32_t ja, jb;
+  uint32_t ja, jb;   // the segment in 32-word steps (a multiple of 2: pitch is a multiple of 1,024 words)
   seg_range((uint32_t)(pitch / 32), s, ja, jb);
   if (ja >= jb) return;
-  if (lane < kG3Group) {
-    const uint32_t e = first + (lane < nm ? lane : 0u);
-    w.so[lane] = (uint32_t)((uint64_t)par_b[e] * pitch);
-    w.oo[lane] = (uint32_t)off[e];
-  }
+  // member row offsets (slots >= nm shadow member 0: staged and gathered, never stored)
+  const uint32_t e = first + (lane < nm ? lane : 0u);
+  const uint32_t so_l = (uint32_t)((uint64_t)par_b[e] * pitch);
+  if (lane < kG3Group) w.oo[lane] = (uint32_t)off[e];
   __syncwarp();
-  const uint32_t* mrow = rows + (uint64_t)par_a[j0] * pitch + lane;
+  const uint32_t* mrow = rows + (uint64_t)par_a[j0] * pitch;
   const uint32_t ow0 = loc3[p];
+  const uint32_t ca = ja / 2, cb = jb / 2;
   if (nm <= 4)
-    pext3_item<4>(w, mrow, rows + lane, nm, ja, jb, ow0, data);
+    pext3_item<4>(w, mrow, rows, so_l, nm, ca, cb, ow0, data);
   else if (nm <= 8)
-    pext3_item<8>(w, mrow, rows + lane, nm, ja, jb, ow0, data);
+    pext3_item<8>(w, mrow, rows, so_l, nm, ca, cb, ow0, data);
   else if (nm <= 12)
-    pext3_item<12>(w, mrow, rows + lane, nm, ja, jb, ow0, data);
-  else if (kG3Group > 16 && nm <= 16)
-    pext3_item<16>(w, mrow, rows + lane, nm, ja, jb, ow0, data);
-  else if (kG3Group > 24 && nm <= 24)
-    pext3_item<24>(w, mrow, rows + lane, nm, ja, jb, ow0, data);
+    pext3_item<12>(w, mrow, rows, so_l, nm, ca, cb, ow0, data);
   else
-    pext3_item<kG3Group>(w, mrow, rows + lane, nm, ja, jb, ow0, data);
+    pext3_item<16>(w, mrow, rows, so_l, nm, ca, cb, ow0, data);
 }
 
 // item -> its pair (items of pair p are item_off[p] .. + items[p])

@@ -87,27 +87,8 @@ __device__ __forceinline__ void cls_pad_warp(uint32_t c, const uint32_t* __restr
   }
 }
 
-// generation 3, warp per pair p = s * cmax + c: output words of row a's segment s (sum over its
-// 32-word chunks of ceil(set bits / 32))
-// Generation 3's output words of one (segment, class): the class' set bits in chunk order, packed
-// 32 per word.  A chunk's member words stay staged for two more chunks (pext3_kernel's ring of three
-// slots), so set bits still pending when their slot is reused are flushed as a partial word first.
-// chunk(C) returns the words completed by a chunk of C set bits; pext3_kernel runs the same steps.
-struct P3Carry {
-  uint32_t pend = 0;  // set bits not yet packed (< 32)
-  bool old = false;   // some of them are from the chunk before the last one
-  __device__ __forceinline__ uint32_t chunk(uint32_t C) {
-    uint32_t w = 0;
-    if (pend && old) { w = 1; pend = 0; }
-    const uint32_t t = pend + C;
-    w += t >> 5;
-    pend = t & 31u;
-    old = pend > C;
-    return w;
-  }
-  __device__ __forceinline__ uint32_t end() const { return pend ? 1u : 0u; }
-};
-
+// generation 3, warp per pair p = s * cmax + c: output words of row a's segment s -- pext3_kernel
+// packs the segment's set bits densely across its chunks: ceil(set bits / 32)
 __device__ __forceinline__ void seg3_warp(uint32_t p, const uint32_t* __restrict__ rows, uint64_t pitch,
                                           const uint32_t* __restrict__ par_a, const uint32_t* __restrict__ bound,
                                           uint32_t n_cls, uint32_t cmax, uint32_t* __restrict__ w3,
@@ -121,11 +102,9 @@ __device__ __forceinline__ void seg3_warp(uint32_t p, const uint32_t* __restrict
       const uint32_t* row = rows + (uint64_t)par_a[j0] * pitch + lane;
       uint32_t a, b;
       seg_range((uint32_t)(pitch / 32), s, a, b);
-      // pext3's word count: set bits carried across chunks, a partial word only where a carried bit
-      // would outlive its chunk's staging slot (P3Carry) and at the segment end
-      P3Carry cy;
-      for (uint32_t j = a; j < b; ++j) words += cy.chunk(__reduce_add_sync(0xffffffffu, (uint32_t)__popc(row[32ull * j])));
-      words += cy.end();
+      uint32_t bits = 0;
+      for (uint32_t j = a; j < b; ++j) bits += __popc(row[32ull * j]);
+      words = (__reduce_add_sync(0xffffffffu, bits) + 31u) / 32u;
       if (lane == 0 && b > a) atomicAdd(in_words, 32ull * (b - a) * m);
     }
   }

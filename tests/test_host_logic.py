@@ -249,87 +249,72 @@ def test_sparse_compress_matches_pext():
     assert [_sparse_compress(x, m) for x, m in zip(xs, ms)] == ref
 
 
-def _p3carry_words(counts):
-    """proj_dev.cuh P3Carry: words of one (segment, class) from its per-chunk set-bit counts."""
-    pend, old, words = 0, False, 0
-    for c in counts:
-        if pend and old:
-            words, pend = words + 1, 0
-        t = pend + c
-        words += t >> 5
-        pend = t & 31
-        old = pend > c
-    return words + (1 if pend else 0)
+def _seg3_words(counts):
+    """proj_dev.cuh seg3_warp: words of one (segment, class) -- its set bits packed densely."""
+    return (sum(counts) + 31) // 32
 
 
 def _pext3_pack(mask_chunks, member_chunks):
-    """pext3_kernel's packing of one (segment, class) written out: each chunk's set bits (lane-major,
-    ascending bits) are staged with the ring slot their member words sit in (3 slots: chunk j's
-    words replace chunk j - 3's); pending bits of chunk j - 2 are flushed as a zero-padded word
-    before chunk j's are staged, and at the end.  Returns (per-member words, per-word real-bit masks, every slot read still held
-    its chunk)."""
-    ring = [None, None, None]
-    staged, out, real, ok = [], [[] for _ in member_chunks], [], True
-
-    def pack(entries):
-        nonlocal ok
-        real.append(sum(1 << r for r, e in enumerate(entries) if e is not None))
-        for q, mem in enumerate(member_chunks):
-            w = 0
-            for r, e in enumerate(entries):
-                if e is None:
-                    continue
-                j, lane, bit = e
-                ok &= ring[j % 3] == j
-                w |= ((int(mem[j][lane]) >> bit) & 1) << r
-            out[q].append(w)
-
-    old = False
-    n = len(mask_chunks)
-    for j in range(n + 1):
-        if j < n:
-            ring[j % 3] = j                          # chunk j's words stored first, as in the kernel
-        if staged and (old or j == n):
-            pack(staged + [None] * (32 - len(staged)))
-            staged = []
-        if j == n:
-            break
-        new = [(j, lane, b) for lane in range(32) for b in range(32) if (int(mask_chunks[j][lane]) >> b) & 1]
-        staged += new
-        while len(staged) >= 32:
-            pack(staged[:32])
-            staged = staged[32:]
-        old = len(staged) > len(new)
-    return out, real, ok
+    """pext3_kernel's packing of one (segment, class) written out step by step: per 64-word chunk
+    (lane l holds words 2l, 2l + 1) the set bits are ranked in word order; ballot t takes rank
+    32 t + r - pend at lane r (nothing outside [0, C)); every ballot ORs into the open slot (slots
+    zeroed after each flush of 32 words); a ballot that fills its word moves to the next slot, the
+    last partial one stays open (pend bits) for the next chunk.  Returns per-member word lists."""
+    n_mem = len(member_chunks)
+    keep = [[0] * 32 for _ in range(n_mem)]
+    out = [[] for _ in range(n_mem)]
+    wc = pend = 0
+    for j, mw in enumerate(mask_chunks):
+        pos = [(wi << 5) | b for wi in range(64) for b in range(32) if (int(mw[wi]) >> b) & 1]
+        C = len(pos)
+        if C == 0:
+            continue
+        tot = pend + C
+        full, nb = tot >> 5, (tot >> 5) + (1 if tot & 31 else 0)
+        for t in range(nb):
+            for q in range(n_mem):
+                b = 0
+                for r in range(32):
+                    rank = 32 * t + r - pend
+                    if 0 <= rank < C:
+                        code = pos[rank]
+                        b |= ((int(member_chunks[q][j][code >> 5]) >> (code & 31)) & 1) << r
+                keep[q][wc & 31] |= b
+            if t < full:
+                wc += 1
+                if wc % 32 == 0:
+                    for q in range(n_mem):
+                        out[q] += keep[q]
+                        keep[q] = [0] * 32
+        pend = tot & 31
+    left = (wc & 31) + (1 if pend else 0)
+    for q in range(n_mem):
+        out[q] += keep[q][:left]
+    return out
 
 
-@pytest.mark.parametrize("density", [0.002, 0.02, 0.05, 0.3])
+@pytest.mark.parametrize("density", [0.002, 0.02, 0.05, 0.3, 0.9])
 def test_pext3_carry_packing(density):
-    """Generation 3's carried packing: every member's words hold exactly pext(member, mask) in order
-    (zero bits only in flushed words' padding), no staged bit is read after its ring slot was
-    reused, and the word count equals the size pass (P3Carry) -- sparse masks (many flushes)
-    through dense, with empty chunks that age carried bits."""
+    """Generation 3's carried packing: every member's words hold exactly pext(member, mask) over the
+    segment, packed densely (the last word zero above its bits), and the word count equals the
+    size pass (seg3_warp) -- sparse masks through dense, with empty chunks between."""
     rng = np.random.default_rng(int(density * 1000))
-    n_chunks, n_mem = 24, 3
-    mask = rng.random((n_chunks, 32, 32)) < density
+    n_chunks, n_mem = 40, 3
+    mask = rng.random((n_chunks, 64, 32)) < density
     mask[5] = False
     mask[6] = False
     mask[7] = False
     mask[7, 0, :3] = True
     pw = (mask * (1 << np.arange(32, dtype=np.uint64))).sum(axis=2).astype(np.uint32)
-    mem = rng.integers(0, 2 ** 32, (n_mem, n_chunks, 32), dtype=np.uint64).astype(np.uint32)
-    out, real, ok = _pext3_pack(pw, mem)
-    assert ok
+    mem = rng.integers(0, 2 ** 32, (n_mem, n_chunks, 64), dtype=np.uint64).astype(np.uint32)
+    out = _pext3_pack(pw, mem)
     counts = [int(mask[j].sum()) for j in range(n_chunks)]
-    assert len(out[0]) == _p3carry_words(counts) == len(real)
-    assert sum(bin(r).count("1") for r in real) == sum(counts)
+    total = sum(counts)
+    assert len(out[0]) == _seg3_words(counts)
     for q in range(n_mem):
-        want = [int((mem[q][j][l] >> b) & 1) for j in range(n_chunks) for l in range(32) for b in range(32)
-                if mask[j, l, b]]
-        got = [(w >> r) & 1 for w, rm in zip(out[q], real) for r in range(32) if (rm >> r) & 1]
-        assert got == want
-        assert all(w & ~rm == 0 for w, rm in zip(out[q], real))
-    # padding only in flushed words: a partial word is a prefix of real bits
-    assert all(((r + 1) & r) == 0 for r in real)
-    assert _p3carry_words([0] * 5) == 0 and _p3carry_words([32]) == 1 and _p3carry_words([33]) == 2
-    assert _p3carry_words([20, 0, 0]) == 1 and _p3carry_words([20, 5, 0, 0]) == 1
+        want = [int((mem[q][j][w] >> b) & 1) for j in range(n_chunks) for w in range(64) for b in range(32)
+                if mask[j, w, b]]
+        got = [(out[q][i >> 5] >> (i & 31)) & 1 for i in range(32 * len(out[q]))]
+        assert got[:total] == want and not any(got[total:])
+    assert _seg3_words([0] * 5) == 0 and _seg3_words([32]) == 1 and _seg3_words([33]) == 2
+    assert _seg3_words([20, 0, 0]) == 1 and _seg3_words([20, 5, 0, 13]) == 2
