@@ -146,19 +146,22 @@ __global__ void __launch_bounds__(kScanThreads) scan_build_kernel(const uint64_t
   const uint32_t n_it = soff[kChunkTx];
   // pieces: items [A + p kPiece, ...) copied from the 16-byte aligned index at or below (the
   // items pointer is 16-byte aligned, checked by the launcher), never past the last whole 16-byte
-  // group of the array: the last <= 3 items of the array are read from global memory directly
+  // group of the array: the last <= 3 items of the array are stored into the buffer by the issuer
   const uint64_t cend = nnz & ~3ull;
-  const uint32_t n_copy = cend > A ? (cend - A < (uint64_t)n_it ? (uint32_t)(cend - A) : n_it) : 0u;   // items [0, n_copy) in smem
   const uint32_t n_pieces = (n_it + kPiece - 1) / kPiece;
   auto issue = [&](uint32_t p) {
     const uint64_t first = A + (uint64_t)p * kPiece;
     const uint64_t last = A + min(n_it, (p + 1) * kPiece);       // exclusive
     const uint64_t a0 = first & ~3ull, a1r = (last + 3) & ~3ull;
     const uint64_t a1 = a1r < cend ? a1r : cend;
-    if (a1 <= a0) {   // nothing copyable: complete the phase without a copy
+    if (a1 <= a0) {   // nothing copyable (the array's tail only): complete the phase without a copy
+      for (uint64_t x = first; x < last; ++x) buf[(p & 1) * (kPiece + 4) + (uint32_t)(x - (first & ~3ull))] = __ldg(items + x);
       asm volatile("mbarrier.arrive.shared.b64 _, [%0];" ::"r"(smem_u32(&bar[p & 1])) : "memory");
       return;
     }
+    // the array's last items past the last whole 16-byte group (never bulk-copied) are stored by
+    // this thread before its arrive, so that every item of the piece is read from shared memory
+    for (uint64_t x = max(first, cend); x < last; ++x) buf[(p & 1) * (kPiece + 4) + (uint32_t)(x - a0)] = __ldg(items + x);
     const uint32_t bytes = (uint32_t)((a1 - a0) * 4);
     const uint32_t b = smem_u32(&bar[p & 1]);
     asm volatile("mbarrier.arrive.expect_tx.shared.b64 _, [%0], %1;" ::"r"(b), "r"(bytes) : "memory");
@@ -178,33 +181,39 @@ __global__ void __launch_bounds__(kScanThreads) scan_build_kernel(const uint64_t
     const uint32_t q0 = p * kPiece, q1 = min(n_it, q0 + kPiece);
     const uint4* pb = reinterpret_cast<const uint4*>(buf + (p & 1) * (kPiece + 4));   // 16-byte groups
     // warp step = 32 aligned 16-byte groups of the buffer (128 items, one conflict-free LDS.128 per
-    // lane); group g holds items q0 - head0 + 4g .. + 3 (chunk-relative, 32-bit); the step's first
-    // transaction by a warp-uniform binary search, each lane's by a short walk from there
+    // lane); group g holds items q0 - head0 + 4g .. + 3 (chunk-relative, 32-bit).  Each lane finds
+    // the transaction of its first item by a binary search over soff, the next ones by comparing
+    // with the next transaction's start (kept in a register)
     const uint32_t n_groups = (head0 + (q1 - q0) + 3) / 4;
-    for (uint32_t g0 = warp * 32; g0 < n_groups; g0 += (kScanThreads / 32) * 32) {
-      const uint32_t jw = q0 + (g0 * 4 > head0 ? g0 * 4 - head0 : 0u);   // first item of the step
-      uint32_t lo = 0, hi = kChunkTx;   // last tx with soff[tx] <= jw
-#pragma unroll
-      for (int it = 0; it < 9; ++it) {
-        const uint32_t mid = (lo + hi) >> 1;
-        const bool le = soff[mid] <= jw;
-        lo = le ? mid : lo;
-        hi = le ? hi : mid;
-      }
-      const uint32_t g = g0 + lane;
+    for (uint32_t g = warp * 32 + lane; g - lane < n_groups; g += kScanThreads) {
       if (g >= n_groups) continue;
       const uint4 v = pb[g];
       const uint32_t xs[4] = {v.x, v.y, v.z, v.w};
-      uint32_t tx = lo;
       const int32_t jr0 = (int32_t)(q0 + 4 * g) - (int32_t)head0;   // chunk-relative index of xs[0]
+      const uint32_t ja = (uint32_t)max(jr0, (int32_t)q0);
+      uint32_t lo = 0, hi = kChunkTx;   // last tx with soff[tx] <= ja
+#pragma unroll
+      for (int it = 0; it < 9; ++it) {
+        const uint32_t mid = (lo + hi) >> 1;
+        const bool le = soff[mid] <= ja;
+        lo = le ? mid : lo;
+        hi = le ? hi : mid;
+      }
+      uint32_t tx = lo, nxt = soff[lo + 1];   // soff[512] = n_it > any item stops the walk
+      uint32_t* trow = tile + (tx >> 5);
+      uint32_t bit = 1u << (tx & 31);
 #pragma unroll
       for (int i = 0; i < 4; ++i) {
         const int32_t jr = jr0 + i;
         if (jr < (int32_t)q0 || jr >= (int32_t)q1) continue;
         const uint32_t j = (uint32_t)jr;
-        while (soff[tx + 1] <= j) ++tx;   // soff[512] = n_it > j stops the walk
-        const uint32_t x = j < n_copy ? xs[i] : __ldg(items + A + j);
-        if (x < n_items) atomicOr(&tile[x * kScanStride + (tx >> 5)], 1u << (tx & 31));
+        if (j >= nxt) {
+          do nxt = soff[++tx + 1]; while (j >= nxt);
+          trow = tile + (tx >> 5);
+          bit = 1u << (tx & 31);
+        }
+        const uint32_t x = xs[i];
+        if (x < n_items) atomicOr(trow + x * kScanStride, bit);
         else my_flags |= kFlagBadItem;
       }
     }
