@@ -124,10 +124,15 @@ void scan_excl_u64(const uint64_t* in, uint64_t* out, uint32_t n, uint64_t* tot,
 void scan_excl_split(const uint32_t* cnt, uint32_t* off, uint32_t* idx, uint32_t n, uint32_t* tot2, ScanState& st,
                      cudaStream_t s);
 
+// Its scan status words persist per thread and device (scan_state()): they are cudaMalloc'd
+// (PBuf), and a per-call ScanState would allocate -- and on growth cudaFree, which synchronises
+// the device -- inside every mining call.
+ScanState& scan_state(int device);
 struct DeviceScratch {
+  explicit DeviceScratch(int device) : scan(scan_state(device)) {}
   DBuf<uint32_t> a, b, c, d, e, f, g, h, i;
   uint32_t hash_cap = 0;   // slots of the join's hash set (i), set by device_candgen_begin
-  ScanState scan;
+  ScanState& scan;
   uint32_t* u32a(size_t n, cudaStream_t s) { a.ensure(n ? n : 1, s); return a.p; }
   uint32_t* u32b(size_t n, cudaStream_t s) { b.ensure(n ? n : 1, s); return b.p; }
   uint32_t* u32c(size_t n, cudaStream_t s) { c.ensure(n ? n : 1, s); return c.p; }
@@ -166,11 +171,14 @@ uint32_t device_threshold(const uint32_t* counts, uint32_t M, uint32_t theta, ui
                           const uint32_t* sel, const uint32_t* prefix, const uint32_t* ext_off, const uint32_t* ext,
                           uint32_t G, const uint32_t* gpar, const uint32_t* eidx,
                           DeviceLevel& out, DeviceScratch& scratch, int n_sms, cudaStream_t s);
-// The same without a synchronisation: out becomes device-sized (n_dev = &|L_k|, n_max = M).
+// The same without a synchronisation: out becomes device-sized (n_dev = &|L_k|, n_max = M).  With
+// items / sup_out (>= M k / M words) the scatter also writes L_k's original item ids (ior: bitset
+// row -> item id) and supports for the result.
 void device_threshold_async(const uint32_t* counts, uint32_t M, uint32_t theta, uint32_t k, uint32_t n_rows,
                             const uint32_t* sel, const uint32_t* prefix, const uint32_t* ext_off, const uint32_t* ext,
                             uint32_t G, const uint32_t* gpar, const uint32_t* eidx,
-                            DeviceLevel& out, DeviceScratch& scratch, int n_sms, cudaStream_t s);
+                            DeviceLevel& out, DeviceScratch& scratch, int n_sms, cudaStream_t s,
+                            const uint32_t* ior = nullptr, uint32_t* items = nullptr, uint32_t* sup_out = nullptr);
 
 // ---- association rules (rules.cu): F as n itemsets in canonical order (items at
 // items + item_off[i], len[i] items, support sup[i]); the rules A => X \ A of the itemsets x0 .. n-1

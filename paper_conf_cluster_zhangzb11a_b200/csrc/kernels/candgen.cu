@@ -26,15 +26,6 @@ constexpr int kRunScanItems = 2;   // run detection compares two rows per member
 // n_dev (device-sized levels): the member count lives on the device; n is its host upper bound
 __device__ __forceinline__ uint32_t eff_n(uint32_t n, const uint32_t* n_dev) { return n_dev ? min(*n_dev, n) : n; }
 
-__global__ void hash_build_kernel(const uint32_t* __restrict__ L, uint32_t n, uint32_t w, uint32_t* slots,
-                                  uint32_t mask, const uint32_t* __restrict__ n_dev) {
-  n = eff_n(n, n_dev);
-  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
-    uint32_t h = (uint32_t)hash_mix(raw_hash(L + (uint64_t)i * w, w)) & mask;
-    while (atomicCAS(&slots[h], kEmpty, i) != kEmpty) h = (h + 1) & mask;
-  }
-}
-
 // L_k's positions: pos[m] = #{m' < m : count >= theta}, *count = |L_k| (one launch)
 __global__ void __launch_bounds__(sd::kScanThreads, 1) ge_scan_kernel(const uint32_t* __restrict__ counts, uint32_t M,
                                                                       uint32_t theta, uint32_t* __restrict__ pos,
@@ -46,10 +37,13 @@ __global__ void __launch_bounds__(sd::kScanThreads, 1) ge_scan_kernel(const uint
 }
 
 // k = 2: candidate m is the pair (a, b) of pair_index order over n rows
+// (every scatter also writes the entry's original item ids and support for the result: ior maps a
+// bitset row to its item id; items / sup_out may be null)
 __global__ void scatter_pairs_kernel(const uint32_t* __restrict__ counts, uint32_t theta,
                                      const uint32_t* __restrict__ pos, uint32_t M, uint32_t n,
                                      const uint32_t* __restrict__ sel, uint32_t* L,
-                                     uint32_t* sup, uint32_t* par_a, uint32_t* par_b) {
+                                     uint32_t* sup, uint32_t* par_a, uint32_t* par_b,
+                                     const uint32_t* __restrict__ ior, uint32_t* items, uint32_t* sup_out) {
   for (uint32_t m = blockIdx.x * blockDim.x + threadIdx.x; m < M; m += gridDim.x * blockDim.x) {
     if (counts[m] < theta) continue;
     uint32_t lo = 0, hi = n - 1;  // a = last row whose first pair index <= m
@@ -68,6 +62,11 @@ __global__ void scatter_pairs_kernel(const uint32_t* __restrict__ counts, uint32
     sup[p] = counts[m];
     par_a[p] = a;
     par_b[p] = b;
+    if (items) {
+      items[2ull * p] = ior[a];
+      items[2ull * p + 1] = ior[b];
+      sup_out[p] = counts[m];
+    }
   }
 }
 
@@ -77,7 +76,8 @@ __global__ void scatter_grouped_kernel(const uint32_t* __restrict__ counts, uint
                                        const uint32_t* __restrict__ prefix, const uint32_t* __restrict__ ext_off,
                                        const uint32_t* __restrict__ ext, uint32_t G, uint32_t km1,
                                        const uint32_t* __restrict__ gpar, const uint32_t* __restrict__ eidx,
-                                       uint32_t* L, uint32_t* sup, uint32_t* par_a, uint32_t* par_b) {
+                                       uint32_t* L, uint32_t* sup, uint32_t* par_a, uint32_t* par_b,
+                                       const uint32_t* __restrict__ ior, uint32_t* items, uint32_t* sup_out) {
   for (uint32_t m = blockIdx.x * blockDim.x + threadIdx.x; m < M; m += gridDim.x * blockDim.x) {
     if (counts[m] < theta) continue;
     uint32_t lo = 0, hi = G;  // g = last group with ext_off[g] <= m
@@ -87,9 +87,18 @@ __global__ void scatter_grouped_kernel(const uint32_t* __restrict__ counts, uint
     }
     const uint32_t p = pos[m];
     uint32_t* dst = L + (uint64_t)p * (km1 + 1);
-    for (uint32_t d = 0; d < km1; ++d) dst[d] = prefix[(uint64_t)lo * km1 + d];
+    uint32_t* it = items ? items + (uint64_t)p * (km1 + 1) : nullptr;
+    for (uint32_t d = 0; d < km1; ++d) {
+      const uint32_t r = prefix[(uint64_t)lo * km1 + d];
+      dst[d] = r;
+      if (it) it[d] = ior[r];
+    }
     dst[km1] = ext[m];
     sup[p] = counts[m];
+    if (it) {
+      it[km1] = ior[ext[m]];
+      sup_out[p] = counts[m];
+    }
     if (gpar) {
       par_a[p] = gpar[lo];
       par_b[p] = eidx[m];
@@ -105,6 +114,7 @@ __global__ void __launch_bounds__(sd::kScanThreads, 1) run_scan_kernel(const uin
                                                                        uint32_t* __restrict__ run_ex,
                                                                        uint32_t* __restrict__ bound,
                                                                        const uint32_t* __restrict__ n_dev,
+                                                                       uint32_t* slots, uint32_t mask,
                                                                        uint32_t* sflags, uint64_t* agg, uint64_t* inc,
                                                                        uint32_t epoch) {
   const uint32_t ne = eff_n(n, n_dev);
@@ -118,6 +128,12 @@ __global__ void __launch_bounds__(sd::kScanThreads, 1) run_scan_kernel(const uin
       [&](uint32_t i, uint32_t e, uint32_t f) {
         run_ex[i] = e;
         if (f) bound[e] = i;
+        // member i into the hash set of the prune probes (after the tile's look-back, so that the
+        // inserts do not delay the later tiles' prefixes)
+        if (i < ne) {
+          uint32_t h = (uint32_t)hash_mix(raw_hash(L + (uint64_t)i * w, w)) & mask;
+          while (atomicCAS(&slots[h], kEmpty, i) != kEmpty) h = (h + 1) & mask;
+        }
       },
       [&](uint32_t runs) { bound[runs] = ne; }, sflags, agg, inc, epoch);
 }
@@ -129,9 +145,10 @@ __global__ void join_kernel(const uint32_t* __restrict__ L, uint32_t n, uint32_t
                             const uint32_t* __restrict__ slots, uint32_t mask, uint32_t* cnt,
                             const uint32_t* __restrict__ cand_off, const uint32_t* __restrict__ gidx,
                             uint32_t* prefix, uint32_t* ext_off, uint32_t* ext, uint32_t* gpar, uint32_t* eidx,
-                            const uint32_t* __restrict__ n_dev) {
+                            const uint32_t* __restrict__ n_dev, const uint32_t* __restrict__ sizes) {
   const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, n_warps = (gridDim.x * blockDim.x) >> 5;
   const uint32_t ne = eff_n(n, n_dev);
+  if (EMIT && blockIdx.x == 0 && threadIdx.x == 0) ext_off[sizes[1]] = sizes[0];   // ext_off[G] = M
   for (uint32_t x = warp; x < n; x += n_warps) {
     if (x < ne)
       lvl::join_warp<EMIT>(x, L, w, flags, run_ex, bound, slots, mask, cnt, cand_off, gidx, prefix, ext_off, ext,
@@ -140,12 +157,6 @@ __global__ void join_kernel(const uint32_t* __restrict__ L, uint32_t n, uint32_t
       cnt[x] = 0;   // past the device count: no survivors (the scans run over the upper bound)
   }
 }
-
-// ext_off[G] = M
-__global__ void ext_end_kernel(const uint32_t* __restrict__ sizes, uint32_t* ext_off) {
-  if (threadIdx.x == 0 && blockIdx.x == 0) ext_off[sizes[1]] = sizes[0];
-}
-
 
 // L_k's rows -> item ids (n = entries x k words) and, with sup_in, its supports copied to sup_out;
 // a device-sized level stops at its count
@@ -186,7 +197,7 @@ namespace {
 void threshold_impl(const uint32_t* counts, uint32_t M, uint32_t theta, uint32_t k, uint32_t n_rows, const uint32_t* sel,
                     const uint32_t* prefix, const uint32_t* ext_off, const uint32_t* ext, uint32_t G,
                     const uint32_t* gpar, const uint32_t* eidx, DeviceLevel& out, DeviceScratch& scratch, int n_sms,
-                    cudaStream_t s, uint32_t cap) {
+                    cudaStream_t s, uint32_t cap, const uint32_t* ior, uint32_t* items, uint32_t* sup_out) {
   uint32_t* pos = scratch.u32b(M, s);
   out.count.ensure(1, s);
   ge_scan(counts, M, theta, pos, out.count.p, scratch, s);
@@ -196,11 +207,13 @@ void threshold_impl(const uint32_t* counts, uint32_t M, uint32_t theta, uint32_t
   out.par_b.ensure(std::max<uint32_t>(cap, 1), s);
   if (k == 2)
     { scatter_pairs_kernel<<<grid_for(M, n_sms), kThreads, 0, s>>>(counts, theta, pos, M, n_rows, sel, out.rows.p,
-                                                                out.sup.p, out.par_a.p, out.par_b.p); note_launch(); }
+                                                                out.sup.p, out.par_a.p, out.par_b.p, ior, items,
+                                                                sup_out); note_launch(); }
   else
     { scatter_grouped_kernel<<<grid_for(M, n_sms), kThreads, 0, s>>>(counts, theta, pos, M, prefix, ext_off, ext, G,
                                                                   k - 1, gpar, eidx, out.rows.p, out.sup.p,
-                                                                  out.par_a.p, out.par_b.p); note_launch(); }
+                                                                  out.par_a.p, out.par_b.p, ior, items, sup_out);
+    note_launch(); }
   GPA_CUDA(cudaGetLastError());
 }
 }  // namespace
@@ -222,7 +235,7 @@ uint32_t device_threshold(const uint32_t* counts, uint32_t M, uint32_t theta, ui
   GPA_CUDA(cudaMemcpyAsync(&F, out.count.p, 4, cudaMemcpyDeviceToHost, s));
   stream_wait(s);
   if (F) threshold_impl(counts, M, theta, k, n_rows, sel, prefix, ext_off, ext, G, gpar, eidx, out, scratch, n_sms, s,
-                        F);
+                        F, nullptr, nullptr, nullptr);
   out.n = F;
   return F;
 }
@@ -230,13 +243,15 @@ uint32_t device_threshold(const uint32_t* counts, uint32_t M, uint32_t theta, ui
 void device_threshold_async(const uint32_t* counts, uint32_t M, uint32_t theta, uint32_t k, uint32_t n_rows,
                             const uint32_t* sel, const uint32_t* prefix, const uint32_t* ext_off, const uint32_t* ext,
                             uint32_t G, const uint32_t* gpar, const uint32_t* eidx,
-                            DeviceLevel& out, DeviceScratch& scratch, int n_sms, cudaStream_t s) {
+                            DeviceLevel& out, DeviceScratch& scratch, int n_sms, cudaStream_t s,
+                            const uint32_t* ior, uint32_t* items, uint32_t* sup_out) {
   out.k = k;
   out.n = 0;
   out.n_dev = nullptr;
   out.n_max = 0;
   if (M == 0) return;
-  threshold_impl(counts, M, theta, k, n_rows, sel, prefix, ext_off, ext, G, gpar, eidx, out, scratch, n_sms, s, M);
+  threshold_impl(counts, M, theta, k, n_rows, sel, prefix, ext_off, ext, G, gpar, eidx, out, scratch, n_sms, s, M, ior,
+                 items, sup_out);
   out.n_dev = out.count.p;   // |L_k| stays on the device until the next generation's synchronisation
   out.n_max = M;
 }
@@ -268,24 +283,23 @@ bool device_candgen_begin(const DeviceLevel& L, DeviceBatch& out, DeviceScratch&
   uint32_t* cnt = scratch.u32c(n, s);
   uint32_t* bound = scratch.u32d(n + 1, s);
   uint32_t* sizes = scratch.u32h(4, s);  // [0] = M, [1] = G
-  {
-    const uint32_t tiles = scan_tiles(n, kRunScanItems);
-    const uint32_t ep = scan_epoch(scratch.scan, tiles, s);
-    run_scan_kernel<<<tiles, sd::kScanThreads, 0, s>>>(L.rows.p, n, w, flags, run_ex, bound, n_dev,
-                                                       scratch.scan.flags.p, scratch.scan.agg.p, scratch.scan.inc.p,
-                                                       ep);
-    note_launch();
-  }
-  GPA_CUDA(cudaGetLastError());
-  // hash set over L for the prune probes
+  // hash set over L for the prune probes (filled by run_scan_kernel)
   uint32_t cap = 16;
   while (cap < 2 * n + 1) cap <<= 1;
   uint32_t* slots = scratch.u32i(cap, s);
   scratch.hash_cap = cap;   // the emitting join (stage 2) probes the same table
   GPA_CUDA(cudaMemsetAsync(slots, 0xff, (size_t)cap * 4, s));
-  { hash_build_kernel<<<grid_for(n, n_sms), kThreads, 0, s>>>(L.rows.p, n, w, slots, cap - 1, n_dev); note_launch(); }
+  {
+    const uint32_t tiles = scan_tiles(n, kRunScanItems);
+    const uint32_t ep = scan_epoch(scratch.scan, tiles, s);
+    run_scan_kernel<<<tiles, sd::kScanThreads, 0, s>>>(L.rows.p, n, w, flags, run_ex, bound, n_dev, slots, cap - 1,
+                                                       scratch.scan.flags.p, scratch.scan.agg.p, scratch.scan.inc.p,
+                                                       ep);
+    note_launch();
+  }
+  GPA_CUDA(cudaGetLastError());
   { join_kernel<false><<<grid_for(32ull * n, n_sms), kThreads, 0, s>>>(L.rows.p, n, w, flags, run_ex, bound, slots,
-        cap - 1, cnt, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, n_dev); note_launch(); }
+        cap - 1, cnt, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, n_dev, nullptr); note_launch(); }
   GPA_CUDA(cudaGetLastError());
   uint32_t* cand_off = scratch.u32e(n, s);
   uint32_t* gidx = scratch.u32g(n, s);
@@ -314,9 +328,8 @@ void device_candgen_finish(const DeviceLevel& L, DeviceBatch& out, DeviceScratch
   const uint32_t cap = scratch.hash_cap;   // the table stage 1 built (sized for its upper bound)
   { join_kernel<true><<<grid_for(32ull * n, n_sms), kThreads, 0, run>>>(L.rows.p, n, w, scratch.a.p, scratch.b.p,
         scratch.d.p, scratch.i.p, cap - 1, scratch.c.p, scratch.e.p, scratch.g.p, out.prefix.p, out.ext_off.p,
-        out.ext.p, out.gpar.p, out.eidx.p, nullptr); note_launch(); }
+        out.ext.p, out.gpar.p, out.eidx.p, nullptr, scratch.h.p); note_launch(); }   // + ext_off[G] = M
   GPA_CUDA(cudaGetLastError());
-  { ext_end_kernel<<<1, 32, 0, run>>>(scratch.h.p, out.ext_off.p); note_launch(); }
   out.M = M;
   out.G = G;
 }

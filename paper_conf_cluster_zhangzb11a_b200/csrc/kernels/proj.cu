@@ -67,6 +67,9 @@ __global__ void __launch_bounds__(sd::kScanThreads, 1) cls_scan_kernel(const uin
                                                                        uint32_t* sflags, uint64_t* agg, uint64_t* inc,
                                                                        uint32_t epoch) {
   const uint32_t ne = n_dev ? min(*n_dev, n) : n;
+  // n_cls[1] (max lane words, atomicMax) and n_cls[2..3] (u64 compressed words, atomicAdd) start at
+  // zero for the class-table kernels that follow
+  if (blockIdx.x == 0 && threadIdx.x < 3) n_cls[1 + threadIdx.x] = 0u;
   sd::scan_tile<uint32_t>(
       n,
       [&](uint32_t j) {
@@ -104,11 +107,17 @@ __global__ void cls_pad_kernel(const uint32_t* __restrict__ words, const uint32_
 // warp per entry j: its vector (offset, words; entries of single-member classes get none), and
 // the words past what the list build writes zeroed -- lane-interleaved lists (k >= 4): lane l's
 // tail len[c][l] .. Lw_c - 1; natural-order lists (generation 3): len[c][0] .. nwc - 1
+// (and, thread per (segment, class) pair, item_pair[] = the pair of every list-build item: the items
+// of pair p are item_off[p] .. + items[p])
 __global__ void entry_off_kernel(const uint32_t* __restrict__ flag, const uint32_t* __restrict__ ex,
                                  const uint32_t* __restrict__ bound, const uint32_t* __restrict__ nwc,
                                  const uint64_t* __restrict__ cls_base, uint32_t n, uint64_t* __restrict__ off,
                                  uint32_t* __restrict__ nw, const uint32_t* __restrict__ len, bool natural,
-                                 uint32_t* __restrict__ data) {
+                                 uint32_t* __restrict__ data, const uint32_t* __restrict__ items,
+                                 const uint32_t* __restrict__ item_off, uint32_t n_pairs,
+                                 uint32_t* __restrict__ item_pair) {
+  for (uint32_t p = blockIdx.x * blockDim.x + threadIdx.x; p < n_pairs; p += gridDim.x * blockDim.x)
+    for (uint32_t i = 0; i < items[p]; ++i) item_pair[item_off[p] + i] = p;
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t n_warps = (gridDim.x * blockDim.x) >> 5;
   for (uint32_t j = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; j < n; j += n_warps) {
@@ -484,13 +493,6 @@ __global__ void __launch_bounds__(kP3Warps * 32, kP3Blocks) pext3_kernel(const u
     pext3_item<16>(w, mrow, rows, so_l, nm, ca, cb, ow0, data);
 }
 
-// item -> its pair (items of pair p are item_off[p] .. + items[p])
-__global__ void item_pair_kernel(const uint32_t* __restrict__ items, const uint32_t* __restrict__ item_off,
-                                 uint32_t n_pairs, uint32_t* __restrict__ item_pair) {
-  for (uint32_t p = blockIdx.x * blockDim.x + threadIdx.x; p < n_pairs; p += gridDim.x * blockDim.x)
-    for (uint32_t i = 0; i < items[p]; ++i) item_pair[item_off[p] + i] = p;
-}
-
 // Warp per item = (pair p = (segment, class), group of <= kMemberGroup members: full groups of 8,
 // the remainder in the class' last group).  Items run pair-major = segment-major, so the warps in
 // flight share the same bitset segments in L2.
@@ -716,8 +718,7 @@ bool proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, 
   W.flag.ensure(n);
   W.ex.ensure(n);
   W.bound.ensure(n + 1);
-  W.small.ensure(4);
-  GPA_CUDA(cudaMemsetAsync(W.small.p, 0, 16, s));
+  W.small.ensure(4);   // zeroed by cls_scan_kernel
   {
     const uint32_t tiles = scan_tiles(n);
     const uint32_t ep = scan_epoch(W.scan, tiles, s);
@@ -786,15 +787,15 @@ bool proj_build_finish(const ProjPending& pp, const uint64_t T[2], const uint32_
   out.words = T[1];
   out.max_lw = sm[1];
   out.in_words = (uint64_t)sm[2] | ((uint64_t)sm[3] << 32);
-  // offsets, and the zero tails of lanes shorter than their class' Lw (the list build writes the rest)
-  { entry_off_kernel<<<grid_for(32ull * n, n_sms), kT, 0, s>>>(W.flag.p, W.ex.p, W.bound.p, W.nwc.p, W.cls_base.p, n,
-                                                              out.off.p, out.nw.p, W.len.p,
-                                                              !pp.prev && gather3(), out.data.p); note_launch(); }
+  // offsets, the zero tails of lanes shorter than their class' Lw (the list build writes the rest)
+  // and the item -> pair map of the list build
+  W.item_pair.ensure(std::max<uint64_t>(T[0], 1));
+  { entry_off_kernel<<<grid_for(std::max<uint64_t>(32ull * n, pp.n_pairs), n_sms), kT, 0, s>>>(
+        W.flag.p, W.ex.p, W.bound.p, W.nwc.p, W.cls_base.p, n, out.off.p, out.nw.p, W.len.p, !pp.prev && gather3(),
+        out.data.p, W.items.p, W.item_off.p, T[0] ? pp.n_pairs : 0u, W.item_pair.p);
+    note_launch(); }
   if (ev_build) GPA_CUDA(cudaEventRecord(ev_build, s));  // start of the list build proper
   if (T[0]) {
-    W.item_pair.ensure(T[0]);
-    { item_pair_kernel<<<grid_for(pp.n_pairs, n_sms), kT, 0, s>>>(W.items.p, W.item_off.p, pp.n_pairs,
-                                                                 W.item_pair.p); note_launch(); }
     const uint64_t blocks = (T[0] + kT / 32 - 1) / (kT / 32);
     if (!pp.prev && gather3()) {
       const int smem = (int)(kP3Warps * sizeof(P3Warp));

@@ -5,6 +5,7 @@
 // costs ~3 us of idle GPU (profiles/r02_microbench_launch_gap.txt).  One kernel per scan here
 // (scan_dev.cuh: decoupled look-back, epoch-tagged status words, the total from the last tile).
 #include <algorithm>
+#include <map>
 #include <cstdint>
 #include "../common.h"
 #include "../kernels.h"
@@ -52,6 +53,11 @@ __global__ void __launch_bounds__(kScanThreads, 1) scan_split_kernel(const uint3
 }
 
 }  // namespace
+
+ScanState& scan_state(int device) {
+  thread_local std::map<int, ScanState> m;
+  return m[device];
+}
 
 uint32_t scan_epoch(ScanState& st, uint32_t tiles, cudaStream_t s) {
   if (st.flags.n < tiles) {   // grow-only (cudaMalloc): fresh flags are zero = no epoch

@@ -8,10 +8,15 @@
 // value results are copied back to main memory", P18@672), L_k = { c : count >= min_count }
 // (P13@474, ">=" per DESIGN.md Q1).  Stops when L_k or C_{k+1} is empty (P13@652).
 #include <algorithm>
+#include <array>
+#include <map>
+#include <memory>
+#include <mutex>
 #include <chrono>
 #include <cstdlib>
 #include <cstring>
 #include <deque>
+#include <string>
 
 #include "internal.h"
 #include "pool.h"
@@ -39,11 +44,49 @@ struct DefaultInitAlloc : std::allocator<T> {
 };
 using FVec = std::vector<uint32_t, DefaultInitAlloc<uint32_t>>;
 
+namespace gpa {
+// Page-locked blocks that a result owns: the frequent itemsets of a generation are copied from the
+// device straight into one (no host copy at the end of the loop), and a destroyed result returns
+// its blocks here for the next call (cudaHostAlloc costs ~1 ms per MB-sized block).
+struct PinnedCache {
+  std::mutex mu;
+  std::multimap<size_t, void*> free;
+  void* get(size_t& bytes) {
+    bytes = (bytes + (size_t(1) << 16) - 1) & ~((size_t(1) << 16) - 1);
+    {
+      std::lock_guard<std::mutex> lk(mu);
+      auto it = free.lower_bound(bytes);
+      if (it != free.end() && it->first <= 4 * bytes + (size_t(1) << 20)) {
+        void* p = it->second;
+        bytes = it->first;
+        free.erase(it);
+        return p;
+      }
+    }
+    void* p = nullptr;
+    GPA_CUDA(cudaHostAlloc(&p, bytes, cudaHostAllocDefault));
+    return p;
+  }
+  void put(void* p, size_t bytes) {
+    std::lock_guard<std::mutex> lk(mu);
+    free.emplace(bytes, p);
+  }
+};
+inline PinnedCache& pinned_cache() {
+  static PinnedCache* c = new PinnedCache();   // never destroyed: results may outlive static teardown
+  return *c;
+}
+}  // namespace gpa
+
 struct gpa_level_data {
   uint32_t k = 0;
   uint64_t n_cand = 0, n_freq = 0, n_groups = 0;
-  FVec freq_items;                     // n_freq * k, original ids, lexicographic
-  FVec freq_support;                   // n_freq
+  FVec freq_items;                     // n_freq * k, original ids, lexicographic (or in fi)
+  FVec freq_support;                   // n_freq (or in fs)
+  const uint32_t* fi = nullptr;        // when set: F in a page-locked block of the result
+  const uint32_t* fs = nullptr;
+  const uint32_t* items() const { return fi ? fi : freq_items.data(); }
+  const uint32_t* supports() const { return fs ? fs : freq_support.data(); }
   std::vector<uint32_t> cand_items;    // n_cand * k (GPA_KEEP_CANDIDATES)
   std::vector<uint32_t> cand_counts;   // n_cand     (GPA_KEEP_CANDIDATES)
   bool kept = false;
@@ -53,6 +96,13 @@ struct gpa_level_data {
 struct gpa_result {
   uint64_t n_tx = 0, min_count = 0;
   uint32_t n_items = 0;
+  std::vector<std::pair<void*, size_t>> pinned;   // page-locked blocks holding F (pinned_cache)
+  gpa_result() = default;
+  gpa_result(const gpa_result&) = delete;
+  gpa_result& operator=(const gpa_result&) = delete;
+  ~gpa_result() {
+    for (auto& b : pinned) gpa::pinned_cache().put(b.first, b.second);
+  }
   std::vector<gpa_level_data> levels;  // levels[0] is k = 1
   std::vector<uint64_t> freq_start;    // prefix sums of n_freq
   double phase_ms[GPA_PHASE_COUNT_] = {0};
@@ -64,6 +114,24 @@ namespace {
 double now_ms() {
   return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now().time_since_epoch()).count();
 }
+
+// GPA_HOST_TRACE=1: host timestamps of the level loop (no CUDA calls), printed after the loop
+struct HostTrace {
+  bool on = [] {
+    const char* e = std::getenv("GPA_HOST_TRACE");
+    return e && *e && *e != '0';
+  }();
+  std::vector<std::pair<std::string, double>> v;
+  void mark(const char* what, uint32_t k) {
+    if (on) v.emplace_back(std::string(what) + " k=" + std::to_string(k), now_ms());
+  }
+  void print() const {
+    if (!on || v.empty()) return;
+    for (size_t i = 0; i < v.size(); ++i)
+      fprintf(stderr, "[gpa-host] %9.3f (+%7.3f) %s\n", v[i].second - v[0].second,
+              i ? v[i].second - v[i - 1].second : 0.0, v[i].first.c_str());
+  }
+};
 
 // Record generation k from the device-side threshold: L_k (F rows of k row ids, lexicographic)
 // and supports come back from the GPU; they are mapped to original item ids in parallel.  With
@@ -153,52 +221,59 @@ uint32_t* host_sizes() {
   return h.p;
 }
 
-// Page-locked staging for the frequent itemsets: each generation's L_k (item ids, supports) is
-// copied to the host right after its threshold, overlapping the next generations, into blocks
-// that persist per thread across calls (grow-only); the result vectors are filled from them at
-// the end (a pageable D2H of all of F took ~3 ms at the end of the loop on T40I10D10M).
-struct PinnedArena {
-  std::vector<std::pair<uint8_t*, size_t>> blocks;
-  size_t cur = 0, used = 0;
-  void reset() { cur = 0; used = 0; }
-  void* get(size_t bytes) {
-    bytes = (bytes + 255) & ~size_t(255);
-    while (cur < blocks.size() && used + bytes > blocks[cur].second) {
-      ++cur;
-      used = 0;
-    }
-    if (cur == blocks.size()) {
-      const size_t sz = std::max<size_t>(bytes, size_t(64) << 20);
-      void* p = nullptr;
-      GPA_CUDA(cudaHostAlloc(&p, sz, cudaHostAllocDefault));
-      blocks.emplace_back(static_cast<uint8_t*>(p), sz);
-      used = 0;
-    }
-    void* r = blocks[cur].first + used;
-    used += bytes;
-    return r;
+}  // namespace
+
+// Per thread and device: the level loop's side streams and its events, created once.
+struct LoopWs {
+  static constexpr int kCopyEvents = 4;
+  static constexpr int kEv = 7;   // per generation: [5] start, [0] counting start, [1] counting end,
+                                  // [2] all-reduce end, [3, 4) list build, [6] threshold end
+  cudaStream_t copy_s = nullptr, aux_s = nullptr;
+  cudaEvent_t copy_ev[kCopyEvents] = {}, aux_ev[4] = {}, trace_ev[kEv] = {};
+  std::deque<std::array<cudaEvent_t, kEv>> sets;
+  explicit LoopWs(int device) {
+    use_device(device);
+    GPA_CUDA(cudaStreamCreateWithFlags(&copy_s, cudaStreamNonBlocking));
+    GPA_CUDA(cudaStreamCreateWithFlags(&aux_s, cudaStreamNonBlocking));
+    for (auto& x : copy_ev) GPA_CUDA(cudaEventCreateWithFlags(&x, cudaEventDisableTiming));
+    for (auto& x : aux_ev) GPA_CUDA(cudaEventCreateWithFlags(&x, cudaEventDisableTiming));
+    for (auto& x : trace_ev) GPA_CUDA(cudaEventCreate(&x));
   }
-  ~PinnedArena() {
-    for (auto& b : blocks) cudaFreeHost(b.first);
+  cudaEvent_t* evset(size_t i) {
+    while (sets.size() <= i) {
+      std::array<cudaEvent_t, kEv> a{};
+      for (auto& x : a) GPA_CUDA(cudaEventCreate(&x));
+      sets.push_back(a);
+    }
+    return sets[i].data();
+  }
+  ~LoopWs() {   // at thread exit (errors ignored: the context may be gone)
+    for (auto& a : sets)
+      for (auto x : a) cudaEventDestroy(x);
+    for (auto x : copy_ev) cudaEventDestroy(x);
+    for (auto x : aux_ev) cudaEventDestroy(x);
+    for (auto x : trace_ev) cudaEventDestroy(x);
+    if (copy_s) cudaStreamDestroy(copy_s);
+    if (aux_s) cudaStreamDestroy(aux_s);
   }
 };
-
-PinnedArena& pinned_arena() {
-  thread_local PinnedArena a;
-  return a;
+LoopWs& loop_ws(int device) {
+  thread_local std::map<int, std::unique_ptr<LoopWs>> m;
+  auto& p = m[device];
+  if (!p) p = std::make_unique<LoopWs>(device);
+  return *p;
 }
-
-}  // namespace
 
 gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist, const gpa_options* opt_in) {
   const double t_start = now_ms();
+  HostTrace ht;
+  ht.mark("enter", 0);
   gpa_options opt;
   gpa_options_default(&opt);
   if (opt_in) opt = *opt_in;
   GPA_REQUIRE(min_count >= 1, GPA_ERR_INVALID, "min_count must be >= 1");
   const bool keep = (opt.flags & GPA_KEEP_CANDIDATES) != 0;
   const bool fused_requested = opt.count_kernel == GPA_KERNEL_FUSED;
-  pinned_arena().reset();  // a previous call on this thread consumed its blocks before returning
   const bool host_candgen = (opt.flags & GPA_HOST_CANDGEN) != 0;
   const uint32_t max_k = opt.max_k ? opt.max_k : GPA_MAX_K;
   GPA_REQUIRE(min_count < (1ull << 32), GPA_ERR_INVALID, "min_count must be < 2^32");
@@ -210,12 +285,14 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
   use_device(dist ? dist->device : opt.device);
   // the ingest path is chosen collectively: every rank issues the same collective sequence
   const bool overlap = agree_input(db, dist, !(opt.flags & GPA_NO_OVERLAP_INGEST));
+  ht.mark("input agreed", 0);
   gpa_bitset* bs = overlap ? bitset_build_overlapped(db, min_count, dist, &opt, &pairs_ready, &pair_stats)
                            : bitset_build(db, min_count, dist, &opt, true, true);
   struct BsGuard {
     gpa_bitset* b;
     ~BsGuard() { bitset_free(b); }
   } bs_guard{bs};
+  ht.mark("bitset built", 0);
   auto* R = new gpa_result();
   struct RGuard {
     gpa_result* r;
@@ -254,7 +331,7 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
   // ---- the level loop stays on the device: threshold + compaction of the counts into L_k and
   // join + prune of C_{k+1} run as kernels (candgen.cu); only the sizes, the candidate batch (for
   // the trie kernel's host-side plan) and L_k (for the result) cross PCIe.
-  DeviceScratch scratch;
+  DeviceScratch scratch(bs->device);
   DeviceLevel Ld, Ln;   // L_{k-1}, L_k on the device
   DeviceBatch Bd;       // C_k on the device (k >= 3)
   DBuf<uint32_t> d_ior;  // row -> original item id
@@ -273,24 +350,21 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     uint32_t F = 0, k = 0;
     bool open = false;                  // |L_k| not yet read back (device-sized level)
     DBuf<uint32_t> items, sup;
-    const uint32_t* h_items = nullptr;  // page-locked copies (pinned_arena)
-    const uint32_t* h_sup = nullptr;
   };
   std::vector<Pending> pending;
-  struct CopyStream {
-    cudaStream_t s = nullptr;
-    CopyStream() { GPA_CUDA(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking)); }
-    ~CopyStream() {
-      if (s) { cudaStreamSynchronize(s); cudaStreamDestroy(s); }
+  // streams and events persist per thread and device (created once: stream and event creation
+  // cost ~10 us each, 7 events per generation)
+  LoopWs& lw = loop_ws(bs->device);
+  struct { cudaStream_t s; } copy_s{lw.copy_s};
+  struct SyncAtExit {   // the side streams read `pending` and the level buffers: drained before they go
+    cudaStream_t a, b;
+    ~SyncAtExit() {
+      cudaStreamSynchronize(a);
+      cudaStreamSynchronize(b);
     }
-  } copy_s;
-  constexpr int kCopyEvents = 4;   // re-recorded round robin: a wait captures the event's state at call time
-  struct Events {
-    cudaEvent_t e[kCopyEvents] = {};
-    Events() { for (auto& x : e) GPA_CUDA(cudaEventCreateWithFlags(&x, cudaEventDisableTiming)); }
-    ~Events() { for (auto x : e) if (x) cudaEventDestroy(x); }
-  } copy_evs;
-  cudaEvent_t* copy_ev = copy_evs.e;
+  } sync_at_exit{lw.copy_s, lw.aux_s};
+  constexpr int kCopyEvents = LoopWs::kCopyEvents;   // re-recorded round robin: a wait captures the event's state at call time
+  cudaEvent_t* copy_ev = lw.copy_ev;
   // |L_k| known on the host: record it and start the D2H of L_k (item ids, supports) on the copy
   // stream -- s has just been synchronised, so everything that produced L_k is complete
   auto finalize = [&](Pending& pd, uint32_t F) {
@@ -299,14 +373,19 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     R->levels[pd.level].n_freq = F;
     R->levels[pd.level].stats.n_freq = F;
     if (F) {
-      auto* hi = static_cast<uint32_t*>(pinned_arena().get((size_t)F * pd.k * 4));
-      auto* hs = static_cast<uint32_t*>(pinned_arena().get((size_t)F * 4));
+      // one page-locked block of the result: F x k item ids, then F supports
+      size_t bytes = (size_t)F * (pd.k + 1) * 4;
+      R->pinned.emplace_back(nullptr, 0);
+      void* blk = pinned_cache().get(bytes);
+      R->pinned.back() = {blk, bytes};
+      auto* hi = static_cast<uint32_t*>(blk);
+      auto* hs = hi + (size_t)F * pd.k;
       GPA_CUDA(cudaEventRecord(copy_ev[pd.k % kCopyEvents], s));
       GPA_CUDA(cudaStreamWaitEvent(copy_s.s, copy_ev[pd.k % kCopyEvents], 0));
       GPA_CUDA(cudaMemcpyAsync(hi, pd.items.p, (size_t)F * pd.k * 4, cudaMemcpyDeviceToHost, copy_s.s));
       GPA_CUDA(cudaMemcpyAsync(hs, pd.sup.p, (size_t)F * 4, cudaMemcpyDeviceToHost, copy_s.s));
-      pd.h_items = hi;
-      pd.h_sup = hs;
+      R->levels[pd.level].fi = hi;
+      R->levels[pd.level].fs = hs;
     }
   };
   // a device-sized L_{k-1}: read |L_{k-1}| now (a synchronisation of its own)
@@ -319,8 +398,8 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     L.n_dev = nullptr;
     finalize(pending.back(), L.n);
   };
-  CopyStream aux_s;          // the emitting join of C_k, overlapping the list build on s
-  Events aux_evs;            // [0] s -> aux (batch buffers sized), [1] aux done
+  struct { cudaStream_t s; } aux_s{lw.aux_s};   // the emitting join of C_k, overlapping the list build on s
+  struct { cudaEvent_t* e; } aux_evs{lw.aux_ev};  // [0] s -> aux (batch buffers sized), [1] aux done, [2] aux start
   ProjPending ppend;
   bool aux_join = false;     // this generation's batch was emitted on aux_s
   uint64_t pT[2] = {0, 0};
@@ -328,25 +407,18 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
   // deferred (device-side) timing of a generation on stream s: [5] generation start, [0] counting
   // start, [1] counting end, [2] all-reduce end, [3, 4) projected-list build, [6] threshold end
   struct EvTriple {
-    enum { kN = 7 };
-    cudaEvent_t e[kN] = {};
-    bool counted = false;   // e[0..2] recorded (not the generation counted during the overlapped ingest)
-    EvTriple() {
-      for (auto& x : e) GPA_CUDA(cudaEventCreate(&x));
-    }
-    EvTriple(EvTriple&& o) noexcept {
-      for (int i = 0; i < kN; ++i) std::swap(e[i], o.e[i]);
-      counted = o.counted;
-    }
-    EvTriple(const EvTriple&) = delete;
-    ~EvTriple() {
-      for (auto x : e)
-        if (x) cudaEventDestroy(x);
-    }
+    cudaEvent_t* e;           // LoopWs::EvSet::e (kN events)
+    bool counted = false;     // e[0..2] recorded (not the generation counted during the overlapped ingest)
   };
-  std::deque<EvTriple> events;
-  EvTriple trace_evs;        // GPA_TRACE: [0] end of join stage 1 (s), [1] of the class tables (aux_s)
-  cudaEvent_t* trace_ev = trace_evs.e;
+  struct EvQueue {            // events[i] uses the workspace's i-th event set
+    LoopWs& w;
+    std::deque<EvTriple> q;
+    EvTriple& emplace_back() { return q.emplace_back(EvTriple{w.evset(q.size())}); }
+    void pop_back() { q.pop_back(); }
+    EvTriple& operator[](size_t i) { return q[i]; }
+    size_t size() const { return q.size(); }
+  } events{lw, {}};
+  cudaEvent_t* trace_ev = lw.trace_ev;   // GPA_TRACE: [0] end of join stage 1 (s), [1] of the class tables (aux_s)
   std::vector<size_t> event_level;
   d_ior.alloc(std::max<uint32_t>(bs->n_rows, 1), s);
   if (bs->n_rows)
@@ -408,8 +480,10 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
       events.pop_back();
     }
   }
+  ht.mark("loop setup", 0);
   for (uint32_t k = 2; k <= max_k && nL > 0; ++k) {
     double t0 = now_ms();
+    ht.mark("top", k);
     EvTriple& ev = events.emplace_back();
     GPA_CUDA(cudaEventRecord(ev.e[5], s));
     CountStats cs;
@@ -470,9 +544,11 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
         if (Ld.n_dev) GPA_CUDA(cudaMemcpyAsync(hs + 10, Ld.n_dev, 4, cudaMemcpyDeviceToHost, s));
         if (trace_enabled()) GPA_CUDA(cudaEventRecord(trace_ev[2], s));
         const double tw0 = now_ms();
+        ht.mark("begin enqueued", k);
         stream_wait(s);
         stream_wait(aux_s.s);
         const double tw1 = now_ms();
+        ht.mark("sizes back", k);
         if (trace_enabled()) GPA_CUDA(cudaEventRecord(trace_ev[3], s));
         M = hs[0];
         G = hs[1];
@@ -488,6 +564,7 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
         device_candgen_finish(Ld, Bd, scratch, bs->n_sms, s, (uint32_t)M, (uint32_t)G, aux_s.s, aux_evs.e[0]);
         GPA_CUDA(cudaEventRecord(aux_evs.e[1], aux_s.s));
         aux_join = true;
+        ht.mark("join finished", k);
         const double tw3 = now_ms();
         if (trace_enabled()) {
           float ja = 0, jb = 0, jc = 0, jd = 0;
@@ -564,22 +641,22 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     }
     if (keep && k > 2) fetch_batch();
     double t2 = now_ms();
+    ht.mark("count enqueued", k);
 
     // L_k = { c in C_k : count >= min_count } on the device WITHOUT a synchronisation: |L_k| stays on
     // the device (Ln is device-sized) and comes back with the next generation's sizes (or settle())
-    device_threshold_async(bs->d_counts.p, (uint32_t)M, (uint32_t)min_count, k, l1_size(bs),
-                           k == 2 && bs->l1_sub ? bs->d_l1.p : nullptr, Bd.prefix.p, Bd.ext_off.p, Bd.ext.p,
-                           (uint32_t)G, host_candgen ? nullptr : Bd.gpar.p, host_candgen ? nullptr : Bd.eidx.p, Ln,
-                           scratch, bs->n_sms, s);
-    // the frequent itemsets of this generation (item ids) and supports, mapped on the device (over
-    // the upper bound M; the kernel stops at |L_k|); their D2H starts once |L_k| is known (finalize)
+    // the frequent itemsets of this generation (item ids) and supports for the result, written by
+    // the scatter (arrays sized for the upper bound M; the D2H starts once |L_k| is known: finalize)
     Pending pd;
     pd.level = R->levels.size();
     pd.k = k;
     pd.open = true;
     pd.items.alloc((size_t)M * k, s);
     pd.sup.alloc(M, s);
-    device_map_items(Ln.rows.p, (uint64_t)M * k, d_ior.p, pd.items.p, bs->n_sms, s, Ln.n_dev, k, Ln.sup.p, pd.sup.p);
+    device_threshold_async(bs->d_counts.p, (uint32_t)M, (uint32_t)min_count, k, l1_size(bs),
+                           k == 2 && bs->l1_sub ? bs->d_l1.p : nullptr, Bd.prefix.p, Bd.ext_off.p, Bd.ext.p,
+                           (uint32_t)G, host_candgen ? nullptr : Bd.gpar.p, host_candgen ? nullptr : Bd.eidx.p, Ln,
+                           scratch, bs->n_sms, s, d_ior.p, pd.items.p, pd.sup.p);
     ev.counted = cs.e0 != nullptr;
     GPA_CUDA(cudaEventRecord(ev.e[6], s));
     std::vector<uint32_t> counts;
@@ -589,6 +666,7 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
       stream_wait(s);
     }
     const double tr0 = now_ms();
+    ht.mark("threshold enqueued", k);
     record_level(R, bs, k, k > 2 ? &batch : nullptr, M, {}, {}, keep, keep ? &counts : nullptr);
     R->levels.back().n_freq = 0;   // set by finalize()
     pending.push_back(std::move(pd));
@@ -617,6 +695,7 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
   const double tf0 = now_ms();
   stream_wait(s);
   stream_wait(copy_s.s);
+  ht.mark("drained", 0);
   const double tf1 = now_ms();
   // phases of the level loop from the events on s (device time, contiguous per generation):
   // candidate generation = generation start -> counting start, counting (+ all-reduce) = counting
@@ -654,26 +733,9 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     R->phase_ms[GPA_PHASE_COUNT] += a + b;
     R->phase_ms[GPA_PHASE_THRESHOLD] += g - cg - a - b;
   }
-  // pinned staging -> the result's vectors: sized first, then copied in ~256 KB pieces over the pool
-  // (one generation can hold most of F)
-  struct Piece { size_t i; uint64_t a, b; };
-  std::vector<Piece> pieces;
-  for (size_t i = 0; i < pending.size(); ++i) {
-    const Pending& pd = pending[i];
-    gpa_level_data& lv = R->levels[pd.level];
-    lv.freq_items.resize((size_t)pd.F * pd.k);
-    lv.freq_support.resize(pd.F);
-    const uint64_t step = std::max<uint64_t>(1, (uint64_t)65536 / std::max<uint32_t>(pd.k, 1));
-    for (uint64_t a = 0; a < pd.F; a += step) pieces.push_back({i, a, std::min<uint64_t>(pd.F, a + step)});
-  }
-  parallel_for(pieces.size(), [&](size_t j) {
-    const Piece& pc = pieces[j];
-    const Pending& pd = pending[pc.i];
-    gpa_level_data& lv = R->levels[pd.level];
-    std::memcpy(lv.freq_items.data() + pc.a * pd.k, pd.h_items + pc.a * pd.k, (pc.b - pc.a) * pd.k * 4);
-    std::memcpy(lv.freq_support.data() + pc.a, pd.h_sup + pc.a, (pc.b - pc.a) * 4);
-  });
+  // F is already in the result's page-locked blocks (copy stream drained above)
   pending.clear();
+  ht.mark("F in the result", 0);
   if (trace_enabled())
     fprintf(stderr, "[gpa] end of loop: drain %.2f ms, F transfer %.2f ms\n", tf1 - tf0, now_ms() - tf1);
 
@@ -684,6 +746,8 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
   }
   R->freq_start.push_back(acc);
   R->phase_ms[GPA_PHASE_TOTAL] = now_ms() - t_start;
+  ht.mark("return", 0);
+  ht.print();
   r_guard.r = nullptr;
   return R;
 }
@@ -730,9 +794,9 @@ extern "C" gpa_status gpa_result_get(const gpa_result* r, uint64_t i, const uint
     size_t lvi = std::upper_bound(r->freq_start.begin(), r->freq_start.end(), i) - r->freq_start.begin() - 1;
     const gpa_level_data& lv = r->levels[lvi];
     const uint64_t j = i - r->freq_start[lvi];
-    if (items) *items = lv.freq_items.data() + j * lv.k;
+    if (items) *items = lv.items() + j * lv.k;
     if (k) *k = lv.k;
-    if (support) *support = lv.freq_support[j];
+    if (support) *support = lv.supports()[j];
   });
 }
 
@@ -749,8 +813,8 @@ extern "C" gpa_status gpa_result_frequent(const gpa_result* r, uint32_t k, uint6
     }
     const gpa_level_data& lv = r->levels[k - 1];
     if (n) *n = lv.n_freq;
-    if (items) *items = lv.freq_items.data();
-    if (supports) *supports = lv.freq_support.data();
+    if (items) *items = lv.items();
+    if (supports) *supports = lv.supports();
   });
 }
 
