@@ -36,7 +36,7 @@ last_end = t0
 agg = {}
 for e in ev:
     gap = e["ts"] - last_end
-    nm = e["name"].split("(")[0].replace("void ", "").replace("(anonymous namespace)::", "")[:40]
+    nm = e["name"].replace("(anonymous namespace)::", "").replace("void ", "").replace("gpa::", "").split("(")[0][:40]
     print(f"{(e['ts'] - t0) / 1e3:9.3f} gap {gap:8.1f} us  dur {e['dur']:8.1f} us  {e.get('cat')[:6]} {nm}")
     a = agg.setdefault(nm, [0, 0.0, 0.0])
     a[0] += 1
