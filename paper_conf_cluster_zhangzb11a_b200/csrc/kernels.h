@@ -265,7 +265,11 @@ struct FusedOut {
     uint64_t freq_word = 0, freq_entry = 0, cand_word = 0, cand_entry = 0;   // offsets into the arrays below
   };
   std::vector<Level> levels;               // generations 2 .. last
-  std::vector<uint32_t> items, sup;        // L_k item ids (F x k per generation) and supports, in order
+  // L_k item ids (F x k per generation) and supports, in order: copied from the device into one
+  // page-locked block from pinned_alloc (bytes in, rounded size out)
+  std::function<void*(size_t&)> pinned_alloc;
+  const uint32_t* items = nullptr;
+  const uint32_t* sup = nullptr;
   std::vector<uint32_t> cand_items, cand_counts;   // keep: every C_k (M x k) and its counts
 };
 // Levels k >= 2 of gpa_mine over the L_1 rows (n1 entries; d_sel: entry -> bitset row or nullptr;

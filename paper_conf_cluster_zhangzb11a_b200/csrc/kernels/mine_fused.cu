@@ -554,22 +554,26 @@ bool mine_fused(const uint32_t* rows, uint64_t pitch_words, uint64_t n_tx, uint3
   P.tstamp = trace ? tsb.ensure(64 * 16) : nullptr;
   if (trace) GPA_CUDA(cudaMemsetAsync(P.tstamp, 0, 64 * 16 * 8, s));
   P.level_tab = W.level_tab.ensure(8 * (GPA_MAX_K + 2));
-  P.status = W.status.ensure(4);
+  P.status = P.level_tab;   // words 0..3 of the table (generation rows start at 8 k, k >= 2)
   P.out_items = W.out_items.ensure(kCapOut);
   P.out_sup = W.out_sup.ensure(kCapOut);
   if (keep) {
     P.cand_items = W.cand_items.ensure(kCapOut);
     P.cand_counts = W.cand_counts.ensure(kCapOut);
   }
-  GPA_CUDA(cudaMemsetAsync(P.status, 0, 16, s));
   GPA_CUDA(cudaMemsetAsync(P.level_tab, 0, 8 * (GPA_MAX_K + 2) * 4, s));
   void* args[] = {&P};
   GPA_CUDA(cudaLaunchCooperativeKernel(reinterpret_cast<const void*>(mine_fused_kernel), W.grid, kFT, args, dsmem, s));
   note_launch();
   // sizes: status + per-generation (M, F, G)
-  std::vector<uint32_t> tab(8 * (GPA_MAX_K + 2)), st(4);
-  GPA_CUDA(cudaMemcpyAsync(st.data(), P.status, 16, cudaMemcpyDeviceToHost, s));
-  GPA_CUDA(cudaMemcpyAsync(tab.data(), P.level_tab, tab.size() * 4, cudaMemcpyDeviceToHost, s));
+  thread_local struct HostTab {   // page-locked: one D2H of the status words and the table
+    uint32_t* p = nullptr;
+    HostTab() { GPA_CUDA(cudaHostAlloc(reinterpret_cast<void**>(&p), 8 * (GPA_MAX_K + 2) * 4, cudaHostAllocDefault)); }
+    ~HostTab() { if (p) cudaFreeHost(p); }
+  } htab;
+  const uint32_t* tab = htab.p;
+  const uint32_t* st = htab.p;
+  GPA_CUDA(cudaMemcpyAsync(htab.p, P.level_tab, 8 * (GPA_MAX_K + 2) * 4, cudaMemcpyDeviceToHost, s));
   stream_wait(s);
   if (trace) {
     std::vector<uint64_t> ts(64 * 16);
@@ -602,12 +606,17 @@ bool mine_fused(const uint32_t* rows, uint64_t pitch_words, uint64_t n_tx, uint3
     }
     out.levels.push_back(lv);
   }
-  out.items.resize(fw);
-  out.sup.resize(fn);
+  out.items = out.sup = nullptr;
+  if (fw) {
+    size_t bytes = (fw + fn) * 4;
+    auto* blk = static_cast<uint32_t*>(out.pinned_alloc(bytes));
+    out.items = blk;
+    out.sup = blk + fw;
+    GPA_CUDA(cudaMemcpyAsync(blk, P.out_items, fw * 4, cudaMemcpyDeviceToHost, s));
+    GPA_CUDA(cudaMemcpyAsync(blk + fw, P.out_sup, fn * 4, cudaMemcpyDeviceToHost, s));
+  }
   out.cand_items.resize(cw);
   out.cand_counts.resize(cn);
-  if (fw) GPA_CUDA(cudaMemcpyAsync(out.items.data(), P.out_items, fw * 4, cudaMemcpyDeviceToHost, s));
-  if (fn) GPA_CUDA(cudaMemcpyAsync(out.sup.data(), P.out_sup, fn * 4, cudaMemcpyDeviceToHost, s));
   if (cw) GPA_CUDA(cudaMemcpyAsync(out.cand_items.data(), P.cand_items, cw * 4, cudaMemcpyDeviceToHost, s));
   if (cn) GPA_CUDA(cudaMemcpyAsync(out.cand_counts.data(), P.cand_counts, cn * 4, cudaMemcpyDeviceToHost, s));
   stream_wait(s);

@@ -6,6 +6,7 @@
 //   ascending item id -> device transpose of the CSR into the static bitset (P18@755).
 // count_grouped / count_all_pairs run the sm_100a counting kernels on a candidate batch and
 // leave the (rank-summed) counts in bs->d_counts.
+#include <cstring>
 #include <algorithm>
 #include <chrono>
 #include <cstdlib>
@@ -77,15 +78,11 @@ gpa_bitset* bitset_build(const gpa_tx_csr* db, uint64_t row_min_count, const gpa
   bs->opt = opt;
   bs->n_items = db->n_items;
   bs->n_tx_local = db->n_tx;
-  if (opt.stream) {
-    bs->stream = static_cast<cudaStream_t>(opt.stream);
-  } else {
-    GPA_CUDA(cudaStreamCreateWithFlags(&bs->stream, cudaStreamNonBlocking));
-    bs->own_stream = true;
-  }
-  GPA_CUDA(cudaEventCreate(&bs->ev0));
-  GPA_CUDA(cudaEventCreate(&bs->ev1));
-  GPA_CUDA(cudaEventCreate(&bs->ev2));
+  bs->bundle = acquire_bundle(bs->device);
+  bs->stream = opt.stream ? static_cast<cudaStream_t>(opt.stream) : bs->bundle->s;
+  bs->ev0 = bs->bundle->ev[0];
+  bs->ev1 = bs->bundle->ev[1];
+  bs->ev2 = bs->bundle->ev[2];
   cudaStream_t s = bs->stream;
 
   // ---- input on the device
@@ -124,14 +121,18 @@ gpa_bitset* bitset_build(const gpa_tx_csr* db, uint64_t row_min_count, const gpa
 
   // ---- validation + generation-1 histogram (+ n_tx) ; one all-reduce each
   const uint32_t n_items = db->n_items;
-  DBuf<uint32_t> d_hist, d_flags;
-  DBuf<uint64_t> d_ntx;
-  d_hist.alloc(std::max<uint32_t>(n_items, 1), s);
-  d_flags.alloc(1, s);
-  d_ntx.alloc(1, s);
-  GPA_CUDA(cudaMemsetAsync(d_hist.p, 0, std::max<uint32_t>(n_items, 1) * sizeof(uint32_t), s));
-  GPA_CUDA(cudaMemsetAsync(d_flags.p, 0, sizeof(uint32_t), s));
-  GPA_CUDA(cudaMemcpyAsync(d_ntx.p, &bs->n_tx_local, sizeof(uint64_t), cudaMemcpyHostToDevice, s));
+  // one block: the histogram (n_items words, rounded to even), the flags word + pad, n_tx (u64):
+  // one memset, one H2D of n_tx, one D2H of everything after the collectives
+  const size_t nh = (std::max<uint32_t>(n_items, 1) + 1) & ~size_t(1);
+  DBuf<uint32_t> d_blk;
+  d_blk.alloc(nh + 4, s);
+  uint32_t* const d_hist_p = d_blk.p;
+  uint32_t* const d_flags_p = d_blk.p + nh;
+  uint64_t* const d_ntx_p = reinterpret_cast<uint64_t*>(d_blk.p + nh + 2);
+  GPA_CUDA(cudaMemsetAsync(d_blk.p, 0, (nh + 2) * sizeof(uint32_t), s));
+  GPA_CUDA(cudaMemcpyAsync(d_ntx_p, &bs->n_tx_local, sizeof(uint64_t), cudaMemcpyHostToDevice, s));
+  struct { uint32_t* p; } d_hist{d_hist_p}, d_flags{d_flags_p};
+  struct { uint64_t* p; } d_ntx{d_ntx_p};
   bs->pitch_words = pitch_words_for(n_tx);
   // up to 1,024 item ids: ONE read of the CSR builds the rows of every item id and their popcounts
   // are the generation-1 counts (scan_build); the L_1 rows are compacted afterwards.  Otherwise a
@@ -153,12 +154,12 @@ gpa_bitset* bitset_build(const gpa_tx_csr* db, uint64_t row_min_count, const gpa
   allreduce_max_u32(dist, d_flags.p, 1, s);   // every rank takes the same accept / reject decision
   allreduce_sum_u32(dist, d_hist.p, n_items, s);
   allreduce_sum_u64(dist, d_ntx.p, 1, s);
-  bs->item_counts.assign(n_items, 0);
-  if (n_items)
-    GPA_CUDA(cudaMemcpyAsync(bs->item_counts.data(), d_hist.p, n_items * sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
-  GPA_CUDA(cudaMemcpyAsync(&flags, d_flags.p, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
-  GPA_CUDA(cudaMemcpyAsync(&bs->n_tx_global, d_ntx.p, sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+  std::vector<uint32_t> h_blk(nh + 4);
+  GPA_CUDA(cudaMemcpyAsync(h_blk.data(), d_blk.p, (nh + 4) * sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
   stream_wait(s);
+  bs->item_counts.assign(h_blk.begin(), h_blk.begin() + n_items);
+  flags = h_blk[nh];
+  std::memcpy(&bs->n_tx_global, h_blk.data() + nh + 2, sizeof(uint64_t));
   GPA_REQUIRE(!(flags & kFlagBadOffsets), GPA_ERR_INVALID, "offsets are not non-decreasing%s",
               dist ? " (on some rank)" : "");
   GPA_REQUIRE(!(flags & kFlagBadItem), GPA_ERR_INVALID, "an item id is >= n_items (%u)%s", n_items,
@@ -231,10 +232,10 @@ void bitset_free(gpa_bitset* bs) {
   bs->d_l1.reset();
   bs->d_pairs_all.reset();
   if (bs->stream) cudaStreamSynchronize(bs->stream);
-  if (bs->ev0) cudaEventDestroy(bs->ev0);
-  if (bs->ev1) cudaEventDestroy(bs->ev1);
-  if (bs->ev2) cudaEventDestroy(bs->ev2);
-  if (bs->own_stream && bs->stream) cudaStreamDestroy(bs->stream);
+  if (bs->bundle) {
+    cudaStreamSynchronize(bs->bundle->s);
+    release_bundle(bs->bundle);   // its stream is idle: reusable by the next bitset
+  }
   delete bs;
 }
 

@@ -125,6 +125,40 @@ DistScope::~DistScope() { t_scope = prev; }
 
 }  // namespace gpa
 
+namespace gpa {
+namespace {
+std::mutex g_bundle_mu;
+std::vector<StreamBundle*>& free_bundles() {
+  static auto* v = new std::vector<StreamBundle*>();   // never destroyed (used until process exit)
+  return *v;
+}
+}  // namespace
+
+StreamBundle* acquire_bundle(int device) {
+  {
+    std::lock_guard<std::mutex> lk(g_bundle_mu);
+    auto& v = free_bundles();
+    for (size_t i = 0; i < v.size(); ++i)
+      if (v[i]->device == device) {
+        StreamBundle* b = v[i];
+        v.erase(v.begin() + (long)i);
+        return b;
+      }
+  }
+  auto* b = new StreamBundle();
+  b->device = device;
+  GPA_CUDA(cudaStreamCreateWithFlags(&b->s, cudaStreamNonBlocking));
+  for (auto& e : b->ev) GPA_CUDA(cudaEventCreate(&e));
+  return b;
+}
+
+void release_bundle(StreamBundle* b) {
+  if (!b) return;
+  std::lock_guard<std::mutex> lk(g_bundle_mu);
+  free_bundles().push_back(b);
+}
+}  // namespace gpa
+
 void gpa::stream_wait(cudaStream_t s) {
   const gpa_dist* d = t_scope;
   if (!d || !d->comm) {

@@ -100,15 +100,11 @@ gpa_bitset* bitset_build_overlapped(const gpa_tx_csr* db, uint64_t row_min_count
   bs->opt = opt;
   bs->n_items = db->n_items;
   bs->n_tx_local = db->n_tx;
-  if (opt.stream) {
-    bs->stream = static_cast<cudaStream_t>(opt.stream);
-  } else {
-    GPA_CUDA(cudaStreamCreateWithFlags(&bs->stream, cudaStreamNonBlocking));
-    bs->own_stream = true;
-  }
-  GPA_CUDA(cudaEventCreate(&bs->ev0));
-  GPA_CUDA(cudaEventCreate(&bs->ev1));
-  GPA_CUDA(cudaEventCreate(&bs->ev2));
+  bs->bundle = acquire_bundle(bs->device);
+  bs->stream = opt.stream ? static_cast<cudaStream_t>(opt.stream) : bs->bundle->s;
+  bs->ev0 = bs->bundle->ev[0];
+  bs->ev1 = bs->bundle->ev[1];
+  bs->ev2 = bs->bundle->ev[2];
   cudaStream_t s = bs->stream;
   cudaStream_t cs = nullptr;
   GPA_CUDA(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));

@@ -121,13 +121,24 @@ struct CountStats {
   uint64_t build_bytes = 0, count_bytes = 0;   // GPA_KERNEL_PROJ: algorithmic bytes (gpa_level_stats)
 };
 
+// A stream + three timing events, recycled across bitsets (stream / event creation costs ~10 us
+// each, and the mining entry points create a bitset per call).  acquire() hands out a free bundle of
+// the device or creates one; release() returns it (its stream idle).
+struct StreamBundle {
+  int device = 0;
+  cudaStream_t s = nullptr;
+  cudaEvent_t ev[3] = {nullptr, nullptr, nullptr};
+};
+StreamBundle* acquire_bundle(int device);
+void release_bundle(StreamBundle* b);
+
 }  // namespace gpa
 
 struct gpa_bitset {
   int device = 0;
   int n_sms = 148;
   cudaStream_t stream = nullptr;
-  bool own_stream = false;
+  gpa::StreamBundle* bundle = nullptr;   // own stream (when opt.stream is null) and ev0..ev2
   const gpa_dist* dist = nullptr;
   gpa_options opt{};
   uint64_t n_tx_local = 0, n_tx_global = 0;

@@ -435,6 +435,11 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
                           fused_eligible((uint32_t)nL, bs->pitch_words);
   if (want_fused) {
     FusedOut fo;
+    fo.pinned_alloc = [&](size_t& bytes) {   // F lands in a page-locked block of the result
+      void* p = pinned_cache().get(bytes);
+      R->pinned.emplace_back(p, bytes);
+      return p;
+    };
     EvTriple& ev = events.emplace_back();
     GPA_CUDA(cudaEventRecord(ev.e[5], s));
     GPA_CUDA(cudaEventRecord(ev.e[0], s));
@@ -460,8 +465,10 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
         lv.n_freq = f.F;
         lv.n_groups = f.G;
         lv.kept = keep;
-        lv.freq_items.assign(fo.items.begin() + f.freq_word, fo.items.begin() + f.freq_word + (uint64_t)f.F * f.k);
-        lv.freq_support.assign(fo.sup.begin() + f.freq_entry, fo.sup.begin() + f.freq_entry + f.F);
+        if (f.F) {
+          lv.fi = fo.items + f.freq_word;
+          lv.fs = fo.sup + f.freq_entry;
+        }
         if (keep) {
           lv.cand_items.assign(fo.cand_items.begin() + f.cand_word,
                                fo.cand_items.begin() + f.cand_word + (uint64_t)f.M * f.k);
