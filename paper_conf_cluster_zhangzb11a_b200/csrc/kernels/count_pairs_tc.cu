@@ -9,7 +9,8 @@
 // Generation 2 is the one place where the hot path IS a dense contraction (every (a, b) is a
 // candidate), so it runs as an integer GEMM on tcgen05 (kind::i8, u8 x u8 -> s32 in TMEM):
 //   * CTA tile = 128 rows a (TMEM lanes, M = 128) x 256 rows b (TMEM columns, N = 256), only tiles
-//     that reach the upper triangle, times a split of the transaction axis (K): the grid is exactly
+//     that reach the upper triangle (the lower diagonal tiles, whose left 128 b rows lie below the
+//     diagonal, run N = 128 on the right half), times a split of the transaction axis (K): the grid is exactly
 //     4 waves of one CTA per SM, the live tiles get floor or ceil(grid / tiles) K-splits each (no
 //     tail wave, no idle CTAs);
 //   * one thread streams the tile's bit rows with TMA (cp.async.bulk.tensor.2d, boxes of 8 words x
@@ -58,6 +59,9 @@ constexpr size_t kSmemBytes = (size_t)kStages * kStageBytes + (size_t)kBitStages
 // instruction descriptor (kind::i8): D = S32 (bits 4-5 = 2), A = B = unsigned 8-bit (0), both
 // K-major, N >> 3 at bit 17, M >> 4 at bit 24
 constexpr uint32_t kIdesc = (2u << 4) | ((uint32_t)(kN >> 3) << 17) | ((uint32_t)(kM >> 4) << 24);
+// the lower diagonal tiles (row block bi = 2 bj + 1): their left 128 b columns lie entirely below the
+// diagonal, so they run N = 128 on the right half only
+constexpr uint32_t kIdescHalf = (2u << 4) | ((uint32_t)((kN / 2) >> 3) << 17) | ((uint32_t)(kM >> 4) << 24);
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 
@@ -87,11 +91,12 @@ __device__ __forceinline__ uint64_t umma_desc(uint32_t saddr) {
          (1ull << 46);
 }
 // D[tmem] (+)= A[tmem] . B[smem]^T
-__device__ __forceinline__ void umma_i8_ta(uint32_t tmem_d, uint32_t tmem_a, uint64_t db, uint32_t accumulate) {
+__device__ __forceinline__ void umma_i8_ta(uint32_t tmem_d, uint32_t tmem_a, uint64_t db, uint32_t accumulate,
+                                           uint32_t idesc) {
   asm volatile(
       "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
       "tcgen05.mma.cta_group::1.kind::i8 [%0], [%1], %2, %3, p;\n}\n" ::"r"(tmem_d),
-      "r"(tmem_a), "l"(db), "r"(kIdesc), "r"(accumulate)
+      "r"(tmem_a), "l"(db), "r"(idesc), "r"(accumulate)
       : "memory");
 }
 // w >> j as the high word of w * 2^(32 - j) (IMAD.HI on the FMA pipe) -- the expansion below is
@@ -166,8 +171,12 @@ __global__ void __launch_bounds__(kThreads, 1)
     t -= cnt;
   }
   const uint32_t bi = t;
-  const uint32_t a0 = bi * kM, b0 = bj * kN;
-  const uint32_t b_hi = min(n_rows, b0 + kN);
+  // lower diagonal tile: b columns [256 bj, 256 bj + 128) < a0 -- only the right half is counted
+  // (N = 128, the B half loaded as B rows 0..127)
+  const bool half = bi == 2 * bj + 1;
+  const uint32_t nN = half ? kN / 2 : kN;
+  const uint32_t a0 = bi * kM, b0 = bj * kN + (half ? kN / 2 : 0u);
+  const uint32_t b_hi = min(n_rows, b0 + nN);
   // K range of this split in whole bit stages (2 operand stages each)
   const uint32_t bs0 = (uint32_t)((uint64_t)n_bit_stages * si / S), bs1 = (uint32_t)((uint64_t)n_bit_stages * (si + 1) / S);
   if (bs0 >= bs1) return;
@@ -229,7 +238,9 @@ __global__ void __launch_bounds__(kThreads, 1)
       if (lane == 0) mbar_arrive(bempty0 + 8 * bslot);
       const uint32_t slot = i % kStages;
       mbar_wait(empty0 + 8 * slot, ((i / kStages) & 1) ^ 1);
-      if (is_a) {   // warp-uniform
+      if (half && !is_a && r >= kN / 2) {
+        // B rows past the half: not used by the N = 128 MMA (warp-uniform)
+      } else if (is_a) {   // warp-uniform
         const uint32_t ta = ta0 + slot * kAcolsPerStage;
         expand_word_tmem(v.x, ta, sh);
         expand_word_tmem(v.y, ta + 8, sh);
@@ -256,9 +267,10 @@ __global__ void __launch_bounds__(kThreads, 1)
         mbar_wait(full0 + 8 * slot, (i / kStages) & 1);
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
         const uint32_t sb = buf0 + slot * kStageBytes, ta = tmem + kAcol + slot * kAcolsPerStage;
+        const uint32_t idesc = half ? kIdescHalf : kIdesc;
 #pragma unroll
         for (int s = 0; s < kWords; ++s)
-          umma_i8_ta(tmem, ta + s * 8, umma_desc(sb + s * kN * 32), (i | s) ? 1u : 0u);
+          umma_i8_ta(tmem, ta + s * 8, umma_desc(sb + s * kN * 32), (i | s) ? 1u : 0u, idesc);
         umma_commit(empty0 + 8 * slot);
       }
       umma_commit(done);
@@ -271,11 +283,11 @@ __global__ void __launch_bounds__(kThreads, 1)
         const uint32_t bslot = j % kBitStages;
         mbar_wait(bempty0 + 8 * bslot, ((j / kBitStages) & 1) ^ 1);
         const uint32_t bar = bfull0 + 8 * bslot, dst = bits0 + bslot * kBitStageBytes;
-        mbar_arrive_expect_tx(bar, kBitStageBytes);
+        mbar_arrive_expect_tx(bar, half ? (uint32_t)(kM + kBoxRows) * kBitWords * 4 : kBitStageBytes);
         const int c = w0 + (int)(j * kBitWords);
         tma_load_2d(dst, &tmap, c, (int)a0, bar);
         tma_load_2d(dst + kM * 32, &tmap, c, (int)b0, bar);
-        tma_load_2d(dst + (kM + kBoxRows) * 32, &tmap, c, (int)(b0 + kBoxRows), bar);
+        if (!half) tma_load_2d(dst + (kM + kBoxRows) * 32, &tmap, c, (int)(b0 + kBoxRows), bar);
       }
     }
     __syncwarp();
@@ -284,7 +296,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
     const uint32_t a = a0 + warp * 32 + lane;
     const uint64_t n = n_rows;
-    for (uint32_t c0 = 0; c0 < (uint32_t)kN; c0 += 32) {
+    for (uint32_t c0 = 0; c0 < nN; c0 += 32) {
       if (b0 + c0 >= b_hi) break;                                 // warp-uniform
       if (b0 + c0 + 31 <= a0 + warp * 32) continue;               // whole chunk at or below the diagonal
       uint32_t v[32];

@@ -329,10 +329,11 @@ __global__ void cls3_pad_kernel(const uint32_t* __restrict__ w3, const uint32_t*
 constexpr uint32_t kP3Warps = 8;
 constexpr uint32_t kP3Blocks = 3;     // blocks/SM (shared memory: 8 x 9.3 KB per block)
 constexpr uint32_t kP3Chunk = 64;     // mask words per chunk: two per lane
-constexpr uint32_t kP3Pos = 512;      // staged set bits per pass (a chunk holds up to 2,048)
+constexpr uint32_t kP3Pos = 448;      // staged set bits per pass (a chunk holds up to 2,048)
+constexpr uint16_t kP3None = 32;      // staged code of "no bit": word 0, shift 32 -> empty mask
 struct P3Warp {
   uint32_t xs[2][kG3Group][kP3Chunk];  // member q's words of the chunk
-  uint16_t pos[kP3Pos];                // a pass of the chunk's set bits in rank order: word << 5 | bit
+  uint16_t pos[32 + kP3Pos + 32];      // a pass of the chunk's set bits in rank order: word << 6 | bit
   uint32_t oo[kG3Group];               // member list: word offset in data
 };
 
@@ -392,35 +393,40 @@ __device__ __forceinline__ void pext3_item(P3Warp& w, const uint32_t* __restrict
       if (lane >= d) o += t;
     }
     const uint32_t Call = __shfl_sync(0xffffffffu, o, 31);
-    // the chunk's set bits in passes of at most kP3Pos ranks (one pass below 25 % density)
+    // the chunk's set bits in passes of at most kP3Pos ranks (one pass below 22 % density).  A pass
+    // stages pos[pend + r] = the code (word << 6 | bit) of its rank r, with kP3None -- bit 32, i.e.
+    // an empty bit mask -- in the pend slots before and the 32 after, so that ballot t reads
+    // pos[32 t + lane] with no range test (the carried lanes and the tail vote 0)
     for (uint32_t lo = 0; lo < Call; lo += kP3Pos) {
       const uint32_t C = min(Call - lo, kP3Pos);
       {
         // 32-bit walks (a 64-bit one costs ~2.5x the instructions per set bit)
-        const uint32_t code0 = lane * 64u;
+        const uint32_t code0 = lane * 128u;   // word 2 lane, bit 0
+        if (lane < pend) w.pos[lane] = kP3None;
+        w.pos[pend + C + lane] = kP3None;
         if (Call <= kP3Pos) {
-          uint16_t* pp = &w.pos[o - cnt];
+          uint16_t* pp = &w.pos[pend + o - cnt];
           for (uint32_t mm = m.x; mm; mm &= mm - 1u) *pp++ = (uint16_t)(code0 + (uint32_t)(__ffs(mm) - 1));
-          for (uint32_t mm = m.y; mm; mm &= mm - 1u) *pp++ = (uint16_t)(code0 + 31u + (uint32_t)__ffs(mm));
+          for (uint32_t mm = m.y; mm; mm &= mm - 1u) *pp++ = (uint16_t)(code0 + 63u + (uint32_t)__ffs(mm));
         } else {   // dense chunk: only the ranks of this pass
           uint32_t r = o - cnt - lo;
           for (uint32_t mm = m.x; mm; mm &= mm - 1u, ++r)
-            if (r < C) w.pos[r] = (uint16_t)(code0 + (uint32_t)(__ffs(mm) - 1));
+            if (r < C) w.pos[pend + r] = (uint16_t)(code0 + (uint32_t)(__ffs(mm) - 1));
           for (uint32_t mm = m.y; mm; mm &= mm - 1u, ++r)
-            if (r < C) w.pos[r] = (uint16_t)(code0 + 31u + (uint32_t)__ffs(mm));
+            if (r < C) w.pos[pend + r] = (uint16_t)(code0 + 63u + (uint32_t)__ffs(mm));
         }
       }
       __syncwarp();
       const uint32_t tot = pend + C, full = tot >> 5;
       const uint32_t nb = full + ((tot & 31u) ? 1u : 0u);
       const uint32_t* xst = &w.xs[st][0][0];
+      const uint16_t* pl = &w.pos[lane];
       for (uint32_t t = 0; t < nb; ++t) {
-        // lane r takes the pass' set bit of rank 32 t + r - pend (none outside [0, C))
-        const int rank = (int)(32u * t + lane) - (int)pend;
-        const bool valid = rank >= 0 && rank < (int)C;
-        const uint32_t code = w.pos[valid ? rank : 0];
-        const uint32_t bm = valid ? 1u << (code & 31u) : 0u;
-        const uint32_t* xb = xst + (code >> 5);
+        // lane r takes the pass' set bit of rank 32 t + r - pend
+        const uint32_t code = pl[32u * t];
+        uint32_t bm;
+        asm("shl.b32 %0, 1, %1;" : "=r"(bm) : "r"(code & 63u));   // bit 32 (kP3None): 0
+        const uint32_t* xb = xst + (code >> 6);
         const uint32_t sel = lane == (wc & 31u) ? 0xffffffffu : 0u;
 #pragma unroll
         for (uint32_t q = 0; q < G; ++q) {
