@@ -402,6 +402,12 @@ def main():
         b0, b1 = shard_range(cfg.n_tx, 0, args.emulate_shard, cfg.kind == "quest")
         theta = max(1, theta * (b1 - b0) // cfg.n_tx)
     ds = gen.make(cfg.name, tx_begin=b0, tx_end=b1)
+    # SHA-256 of this rank's CSR bytes (offsets then items): the identity of the synthetic input
+    import hashlib
+    sha = hashlib.sha256()
+    sha.update(np.ascontiguousarray(ds.offsets, dtype=np.uint64).data)
+    sha.update(np.ascontiguousarray(ds.items, dtype=np.uint32).data)
+    dataset_sha256 = sha.hexdigest()
     kern = {"auto": gpa.KERNEL_AUTO, "v0": gpa.KERNEL_V0, "prefix": gpa.KERNEL_PREFIX,
             "pairs": gpa.KERNEL_PAIRS, "trie": gpa.KERNEL_TRIE, "pairs_tc": gpa.KERNEL_PAIRS_TC,
             "proj": gpa.KERNEL_PROJ}[args.kernel]
@@ -531,7 +537,8 @@ def main():
                        "frequent_itemsets": sum(lv.n_freq for lv in res.levels),
                        "l2_flush": "not needed: bitset 1.25 GB and CSR 1.6 GB exceed the 126 MB L2"
                        if cfg.name == "t40i10d10m" else "none (small config)",
-                       "parallelism": f"tx-shard x{world}", "kernel": args.kernel},
+                       "parallelism": f"tx-shard x{world}", "kernel": args.kernel,
+                       "dataset_sha256": dataset_sha256},
             "roofline": roof,
             "roofline_by_kernel": roof_all,
             "cpu_baseline": cpu,

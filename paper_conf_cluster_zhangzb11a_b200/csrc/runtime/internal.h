@@ -1,5 +1,6 @@
 // Runtime-internal declarations (handles, device buffers, counting engine).
 #pragma once
+#include <nvtx3/nvToolsExt.h>
 #include <cstdint>
 #include <cstring>
 #include <string>
@@ -27,6 +28,14 @@ struct gpa_dist {
 };
 
 namespace gpa {
+// NVTX range (header-only NVTX v3: a no-op unless a profiler is attached): phases of gpa_mine show
+// up by name in Nsight Systems / ncu --nvtx
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  NvtxRange(const NvtxRange&) = delete;
+  NvtxRange& operator=(const NvtxRange&) = delete;
+  ~NvtxRange() { nvtxRangePop(); }
+};
 
 struct DeviceInfo {
   int device;

@@ -266,6 +266,7 @@ LoopWs& loop_ws(int device) {
 
 gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist, const gpa_options* opt_in) {
   const double t_start = now_ms();
+  NvtxRange nv_mine("gpa_mine");
   HostTrace ht;
   ht.mark("enter", 0);
   gpa_options opt;
@@ -286,12 +287,14 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
   // the ingest path is chosen collectively: every rank issues the same collective sequence
   const bool overlap = agree_input(db, dist, !(opt.flags & GPA_NO_OVERLAP_INGEST));
   ht.mark("input agreed", 0);
+  nvtxRangePushA(overlap ? "gpa_bitset_build (overlapped ingest)" : "gpa_bitset_build");
   gpa_bitset* bs = overlap ? bitset_build_overlapped(db, min_count, dist, &opt, &pairs_ready, &pair_stats)
                            : bitset_build(db, min_count, dist, &opt, true, true);
   struct BsGuard {
     gpa_bitset* b;
     ~BsGuard() { bitset_free(b); }
   } bs_guard{bs};
+  nvtxRangePop();
   ht.mark("bitset built", 0);
   auto* R = new gpa_result();
   struct RGuard {
@@ -490,6 +493,9 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
   ht.mark("loop setup", 0);
   for (uint32_t k = 2; k <= max_k && nL > 0; ++k) {
     double t0 = now_ms();
+    char nv_name[32];
+    snprintf(nv_name, sizeof nv_name, "gpa_generation %u", k);
+    NvtxRange nv_gen(nv_name);
     ht.mark("top", k);
     EvTriple& ev = events.emplace_back();
     GPA_CUDA(cudaEventRecord(ev.e[5], s));
