@@ -131,7 +131,8 @@ ScanState& scan_state(int device);
 struct DeviceScratch {
   explicit DeviceScratch(int device) : scan(scan_state(device)) {}
   DBuf<uint32_t> a, b, c, d, e, f, g, h, i;
-  uint32_t hash_cap = 0;   // slots of the join's hash set (i), set by device_candgen_begin
+  uint32_t hash_cap = 0;   // slots of the join's hash set (i), filled by the scatter of L (threshold)
+  uint32_t hash_n = 0;     // the level size (upper bound) that set was built for
   ScanState& scan;
   uint32_t* u32a(size_t n, cudaStream_t s) { a.ensure(n ? n : 1, s); return a.p; }
   uint32_t* u32b(size_t n, cudaStream_t s) { b.ensure(n ? n : 1, s); return b.p; }

@@ -26,6 +26,14 @@ constexpr int kRunScanItems = 2;   // run detection compares two rows per member
 // n_dev (device-sized levels): the member count lives on the device; n is its host upper bound
 __device__ __forceinline__ uint32_t eff_n(uint32_t n, const uint32_t* n_dev) { return n_dev ? min(*n_dev, n) : n; }
 
+// entry p (its w row ids at row) into the hash set of the next join's prune probes -- done by the
+// scatter that writes L_k, so the set needs no pass of its own (slots cleared to kEmpty first)
+__device__ __forceinline__ void hash_insert(const uint32_t* row, uint32_t w, uint32_t p, uint32_t* slots,
+                                            uint32_t mask) {
+  uint32_t h = (uint32_t)hash_mix(raw_hash(row, w)) & mask;
+  while (atomicCAS(&slots[h], kEmpty, p) != kEmpty) h = (h + 1) & mask;
+}
+
 // L_k's positions: pos[m] = #{m' < m : count >= theta}, *count = |L_k| (one launch)
 __global__ void __launch_bounds__(sd::kScanThreads, 1) ge_scan_kernel(const uint32_t* __restrict__ counts, uint32_t M,
                                                                       uint32_t theta, uint32_t* __restrict__ pos,
@@ -43,7 +51,8 @@ __global__ void scatter_pairs_kernel(const uint32_t* __restrict__ counts, uint32
                                      const uint32_t* __restrict__ pos, uint32_t M, uint32_t n,
                                      const uint32_t* __restrict__ sel, uint32_t* L,
                                      uint32_t* sup, uint32_t* par_a, uint32_t* par_b,
-                                     const uint32_t* __restrict__ ior, uint32_t* items, uint32_t* sup_out) {
+                                     const uint32_t* __restrict__ ior, uint32_t* items, uint32_t* sup_out,
+                                     uint32_t* slots, uint32_t mask) {
   for (uint32_t m = blockIdx.x * blockDim.x + threadIdx.x; m < M; m += gridDim.x * blockDim.x) {
     if (counts[m] < theta) continue;
     uint32_t lo = 0, hi = n - 1;  // a = last row whose first pair index <= m
@@ -67,6 +76,7 @@ __global__ void scatter_pairs_kernel(const uint32_t* __restrict__ counts, uint32
       items[2ull * p + 1] = ior[b];
       sup_out[p] = counts[m];
     }
+    if (slots) hash_insert(L + 2ull * p, 2, p, slots, mask);
   }
 }
 
@@ -77,7 +87,8 @@ __global__ void scatter_grouped_kernel(const uint32_t* __restrict__ counts, uint
                                        const uint32_t* __restrict__ ext, uint32_t G, uint32_t km1,
                                        const uint32_t* __restrict__ gpar, const uint32_t* __restrict__ eidx,
                                        uint32_t* L, uint32_t* sup, uint32_t* par_a, uint32_t* par_b,
-                                       const uint32_t* __restrict__ ior, uint32_t* items, uint32_t* sup_out) {
+                                       const uint32_t* __restrict__ ior, uint32_t* items, uint32_t* sup_out,
+                                       uint32_t* slots, uint32_t mask) {
   for (uint32_t m = blockIdx.x * blockDim.x + threadIdx.x; m < M; m += gridDim.x * blockDim.x) {
     if (counts[m] < theta) continue;
     uint32_t lo = 0, hi = G;  // g = last group with ext_off[g] <= m
@@ -99,6 +110,7 @@ __global__ void scatter_grouped_kernel(const uint32_t* __restrict__ counts, uint
       it[km1] = ior[ext[m]];
       sup_out[p] = counts[m];
     }
+    if (slots) hash_insert(dst, km1 + 1, p, slots, mask);
     if (gpar) {
       par_a[p] = gpar[lo];
       par_b[p] = eidx[m];
@@ -114,7 +126,6 @@ __global__ void __launch_bounds__(sd::kScanThreads, 1) run_scan_kernel(const uin
                                                                        uint32_t* __restrict__ run_ex,
                                                                        uint32_t* __restrict__ bound,
                                                                        const uint32_t* __restrict__ n_dev,
-                                                                       uint32_t* slots, uint32_t mask,
                                                                        uint32_t* sflags, uint64_t* agg, uint64_t* inc,
                                                                        uint32_t epoch) {
   const uint32_t ne = eff_n(n, n_dev);
@@ -128,12 +139,6 @@ __global__ void __launch_bounds__(sd::kScanThreads, 1) run_scan_kernel(const uin
       [&](uint32_t i, uint32_t e, uint32_t f) {
         run_ex[i] = e;
         if (f) bound[e] = i;
-        // member i into the hash set of the prune probes (after the tile's look-back, so that the
-        // inserts do not delay the later tiles' prefixes)
-        if (i < ne) {
-          uint32_t h = (uint32_t)hash_mix(raw_hash(L + (uint64_t)i * w, w)) & mask;
-          while (atomicCAS(&slots[h], kEmpty, i) != kEmpty) h = (h + 1) & mask;
-        }
       },
       [&](uint32_t runs) { bound[runs] = ne; }, sflags, agg, inc, epoch);
 }
@@ -205,14 +210,22 @@ void threshold_impl(const uint32_t* counts, uint32_t M, uint32_t theta, uint32_t
   out.sup.ensure(std::max<uint32_t>(cap, 1), s);
   out.par_a.ensure(std::max<uint32_t>(cap, 1), s);
   out.par_b.ensure(std::max<uint32_t>(cap, 1), s);
+  // the next join's hash set over L_k (sized for the upper bound cap), filled by the scatter
+  uint32_t hcap = 16;
+  while (hcap < 2 * cap + 1) hcap <<= 1;
+  uint32_t* slots = scratch.u32i(hcap, s);
+  scratch.hash_cap = hcap;
+  scratch.hash_n = cap;
+  GPA_CUDA(cudaMemsetAsync(slots, 0xff, (size_t)hcap * 4, s));
   if (k == 2)
     { scatter_pairs_kernel<<<grid_for(M, n_sms), kThreads, 0, s>>>(counts, theta, pos, M, n_rows, sel, out.rows.p,
                                                                 out.sup.p, out.par_a.p, out.par_b.p, ior, items,
-                                                                sup_out); note_launch(); }
+                                                                sup_out, slots, hcap - 1); note_launch(); }
   else
     { scatter_grouped_kernel<<<grid_for(M, n_sms), kThreads, 0, s>>>(counts, theta, pos, M, prefix, ext_off, ext, G,
                                                                   k - 1, gpar, eidx, out.rows.p, out.sup.p,
-                                                                  out.par_a.p, out.par_b.p, ior, items, sup_out);
+                                                                  out.par_a.p, out.par_b.p, ior, items, sup_out,
+                                                                  slots, hcap - 1);
     note_launch(); }
   GPA_CUDA(cudaGetLastError());
 }
@@ -283,16 +296,15 @@ bool device_candgen_begin(const DeviceLevel& L, DeviceBatch& out, DeviceScratch&
   uint32_t* cnt = scratch.u32c(n, s);
   uint32_t* bound = scratch.u32d(n + 1, s);
   uint32_t* sizes = scratch.u32h(4, s);  // [0] = M, [1] = G
-  // hash set over L for the prune probes (filled by run_scan_kernel)
-  uint32_t cap = 16;
-  while (cap < 2 * n + 1) cap <<= 1;
-  uint32_t* slots = scratch.u32i(cap, s);
-  scratch.hash_cap = cap;   // the emitting join (stage 2) probes the same table
-  GPA_CUDA(cudaMemsetAsync(slots, 0xff, (size_t)cap * 4, s));
+  // the hash set over L for the prune probes was filled by the scatter that wrote L (threshold_impl)
+  GPA_REQUIRE(scratch.hash_cap >= 2 * n + 1 && scratch.hash_n == n && scratch.i.p, GPA_ERR_STATE,
+              "join: no hash set over this level");
+  const uint32_t cap = scratch.hash_cap;   // the emitting join (stage 2) probes the same table
+  uint32_t* slots = scratch.i.p;
   {
     const uint32_t tiles = scan_tiles(n, kRunScanItems);
     const uint32_t ep = scan_epoch(scratch.scan, tiles, s);
-    run_scan_kernel<<<tiles, sd::kScanThreads, 0, s>>>(L.rows.p, n, w, flags, run_ex, bound, n_dev, slots, cap - 1,
+    run_scan_kernel<<<tiles, sd::kScanThreads, 0, s>>>(L.rows.p, n, w, flags, run_ex, bound, n_dev,
                                                        scratch.scan.flags.p, scratch.scan.agg.p, scratch.scan.inc.p,
                                                        ep);
     note_launch();
