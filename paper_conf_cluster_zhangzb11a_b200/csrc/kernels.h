@@ -143,6 +143,9 @@ struct DeviceScratch {
   uint32_t* u32g(size_t n, cudaStream_t s) { g.ensure(n ? n : 1, s); return g.p; }
   uint32_t* u32h(size_t n, cudaStream_t s) { h.ensure(n ? n : 1, s); return h.p; }
   uint32_t* u32i(size_t n, cudaStream_t s) { i.ensure(n ? n : 1, s); return i.p; }
+  // the join's per-member survivor masks (stage 1 -> stage 2, lvl::join_warp)
+  DBuf<unsigned long long> surv;
+  unsigned long long* surv64(size_t n, cudaStream_t s) { surv.ensure(n ? n : 1, s); return surv.p; }
 };
 // L_k on the device: n rows of k row ids (lexicographic) and their supports
 // par_a[p] / par_b[p]: index in L_{k-1} of the entry's left parent (its first k-1 items) and

@@ -150,14 +150,15 @@ __global__ void join_kernel(const uint32_t* __restrict__ L, uint32_t n, uint32_t
                             const uint32_t* __restrict__ slots, uint32_t mask, uint32_t* cnt,
                             const uint32_t* __restrict__ cand_off, const uint32_t* __restrict__ gidx,
                             uint32_t* prefix, uint32_t* ext_off, uint32_t* ext, uint32_t* gpar, uint32_t* eidx,
-                            const uint32_t* __restrict__ n_dev, const uint32_t* __restrict__ sizes) {
+                            const uint32_t* __restrict__ n_dev, const uint32_t* __restrict__ sizes,
+                            unsigned long long* surv) {
   const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, n_warps = (gridDim.x * blockDim.x) >> 5;
   const uint32_t ne = eff_n(n, n_dev);
   if (EMIT && blockIdx.x == 0 && threadIdx.x == 0) ext_off[sizes[1]] = sizes[0];   // ext_off[G] = M
   for (uint32_t x = warp; x < n; x += n_warps) {
     if (x < ne)
       lvl::join_warp<EMIT>(x, L, w, flags, run_ex, bound, slots, mask, cnt, cand_off, gidx, prefix, ext_off, ext,
-                           gpar, eidx);
+                           gpar, eidx, surv);
     else if (!EMIT && (threadIdx.x & 31) == 0)
       cnt[x] = 0;   // past the device count: no survivors (the scans run over the upper bound)
   }
@@ -311,7 +312,8 @@ bool device_candgen_begin(const DeviceLevel& L, DeviceBatch& out, DeviceScratch&
   }
   GPA_CUDA(cudaGetLastError());
   { join_kernel<false><<<grid_for(32ull * n, n_sms), kThreads, 0, s>>>(L.rows.p, n, w, flags, run_ex, bound, slots,
-        cap - 1, cnt, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, n_dev, nullptr); note_launch(); }
+        cap - 1, cnt, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, n_dev, nullptr,
+        scratch.surv64(n, s)); note_launch(); }
   GPA_CUDA(cudaGetLastError());
   uint32_t* cand_off = scratch.u32e(n, s);
   uint32_t* gidx = scratch.u32g(n, s);
@@ -340,7 +342,7 @@ void device_candgen_finish(const DeviceLevel& L, DeviceBatch& out, DeviceScratch
   const uint32_t cap = scratch.hash_cap;   // the table stage 1 built (sized for its upper bound)
   { join_kernel<true><<<grid_for(32ull * n, n_sms), kThreads, 0, run>>>(L.rows.p, n, w, scratch.a.p, scratch.b.p,
         scratch.d.p, scratch.i.p, cap - 1, scratch.c.p, scratch.e.p, scratch.g.p, out.prefix.p, out.ext_off.p,
-        out.ext.p, out.gpar.p, out.eidx.p, nullptr, scratch.h.p); note_launch(); }   // + ext_off[G] = M
+        out.ext.p, out.gpar.p, out.eidx.p, nullptr, scratch.h.p, scratch.surv.p); note_launch(); }   // + ext_off[G] = M
   GPA_CUDA(cudaGetLastError());
   out.M = M;
   out.G = G;

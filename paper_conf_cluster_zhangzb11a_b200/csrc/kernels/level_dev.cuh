@@ -60,23 +60,60 @@ __device__ __forceinline__ bool row_is_sub(const uint32_t* __restrict__ row, con
   return row[w - 1] == b;
 }
 
+// surv (optional): stage 1 leaves, per member with at most kSurvBits siblings, the bit mask of its
+// surviving siblings (bit j: sibling x + 1 + j), kSurvNone otherwise; stage 2 then emits from the
+// mask instead of probing the hash set again.
+constexpr uint32_t kSurvBits = 63;
+constexpr unsigned long long kSurvNone = ~0ull;
+
 template <bool EMIT>
 __device__ __forceinline__ void join_warp(uint32_t x, const uint32_t* __restrict__ L, uint32_t w,
                                           const uint32_t* __restrict__ flags, const uint32_t* __restrict__ run_ex,
                                           const uint32_t* __restrict__ bound, const uint32_t* __restrict__ slots,
                                           uint32_t mask, uint32_t* cnt, const uint32_t* __restrict__ cand_off,
                                           const uint32_t* __restrict__ gidx, uint32_t* prefix, uint32_t* ext_off,
-                                          uint32_t* ext, uint32_t* gpar, uint32_t* eidx) {
+                                          uint32_t* ext, uint32_t* gpar, uint32_t* eidx,
+                                          unsigned long long* surv = nullptr) {
   const uint32_t lane = threadIdx.x & 31;
   if (EMIT && cnt[x] == 0) return;  // warp-uniform
+  const uint32_t* px = L + (uint64_t)x * w;
+  if (EMIT && surv) {
+    const unsigned long long sm = surv[x];
+    if (sm != kSurvNone) {   // the survivors of stage 1: no probes
+      const uint32_t base = cand_off[x];
+      uint32_t here = 0;
+#pragma unroll
+      for (uint32_t hf = 0; hf < 2; ++hf) {
+        const uint32_t bits = (uint32_t)(sm >> (32 * hf));
+        if ((bits >> lane) & 1u) {
+          const uint32_t y = x + 1 + 32 * hf + lane;
+          const uint32_t at = base + here + __popc(bits & ((1u << lane) - 1u));
+          ext[at] = L[(uint64_t)y * w + w - 1];
+          eidx[at] = y;
+        }
+        here += __popc(bits);
+      }
+      const uint32_t g = gidx[x];
+      for (uint32_t i = lane; i < w; i += 32) prefix[(uint64_t)g * w + i] = px[i];
+      if (lane == 0) {
+        ext_off[g] = base;
+        gpar[g] = x;
+      }
+      return;
+    }
+  }
   // run index of x = (#run starts <= x) - 1
   const uint32_t r = run_ex[x] + flags[x] - 1;
   const uint32_t end = bound[r + 1];  // bound[n_runs] = n (sentinel end of the last run)
   if (!EMIT && end == x + 1) {
-    if (lane == 0) cnt[x] = 0;
+    if (lane == 0) {
+      cnt[x] = 0;
+      if (surv) surv[x] = 0ull;
+    }
     return;
   }
-  const uint32_t* px = L + (uint64_t)x * w;
+  const bool track = !EMIT && surv && end - x - 1 <= kSurvBits;   // warp-uniform
+  unsigned long long smask = 0ull;
   // hash of the subset "px without item d, then b" = A_d + B_d + (b + 1) P^(w-1) with
   // A_d = sum_{i<d} (x_i+1) P^i, B_d = sum_{i>d} (x_i+1) P^(i-1): both walked with d below
   uint64_t B0 = 0, pw = 1;
@@ -126,6 +163,7 @@ __device__ __forceinline__ void join_warp(uint32_t x, const uint32_t* __restrict
         ext[at] = bj;
         eidx[at] = y0 + lane;
       }
+      if (track) smask |= (unsigned long long)ballot << (y0 - x - 1);   // bits 0 .. G-1 = siblings y0 ..
       here += __popc(ballot);
     }
   } else
@@ -162,8 +200,10 @@ __device__ __forceinline__ void join_warp(uint32_t x, const uint32_t* __restrict
       ext[at] = b;
       eidx[at] = y;
     }
+    if (track) smask |= (unsigned long long)ballot << (y0 - x - 1);
     here += __popc(ballot);
   }
+  if (!EMIT && surv && lane == 0) surv[x] = track ? smask : kSurvNone;
   if (EMIT) {
     const uint32_t g = gidx[x];
     for (uint32_t i = lane; i < w; i += 32) prefix[(uint64_t)g * w + i] = px[i];
