@@ -17,6 +17,9 @@ namespace gpa {
 void launch_hist_validate(const uint64_t* offsets, const uint32_t* items, uint64_t n_tx, uint64_t nnz,
                           uint32_t n_items, uint32_t* hist, uint32_t* flags, int n_sms, cudaStream_t stream);
 // same over transactions [tx_begin, tx_end) (offsets / items are the whole arrays)
+// items[j] of a bit-packed upload (bits per item, little-endian 32-bit words) -> out[j] (u32), j < n
+void launch_unpack_items(const uint32_t* packed, uint64_t n, uint32_t bits, uint32_t* out, int n_sms,
+                         cudaStream_t stream);
 void launch_hist_validate_range(const uint64_t* offsets, const uint32_t* items, uint64_t tx_begin, uint64_t tx_end,
                                 uint64_t nnz, uint32_t n_items, uint32_t* hist, uint32_t* flags, int n_sms,
                                 cudaStream_t stream);

@@ -16,6 +16,10 @@
 // rebuilt for L_1 from the device copy of the CSR and generation 2 is counted afresh.  Either way
 // the result is identical to the sequential path (same counts, same rows).
 #include <algorithm>
+#include <array>
+#include <cstdlib>
+#include <utility>
+#include <map>
 
 #include "internal.h"
 #include "pool.h"
@@ -25,6 +29,110 @@ namespace gpa {
 namespace {
 constexpr uint64_t kIngestAlign = 8192;   // transactions: one bitset stripe (256 words)
 constexpr uint32_t kIngestChunks = 8;
+
+// Bit-packed upload of the item ids (the PCIe transfer bounds gpa_mine on host input): with
+// n_items <= 2^16 every id fits in b = ceil(log2 n_items) bits, so host threads pack a chunk's
+// items into b-bit fields (32 items = b whole words per block: blocks pack independently) in a
+// page-locked staging buffer, the copy stream moves b/32 of the bytes, and unpack.cu widens them
+// in place in the device CSR.  An id >= 2^b (invalid input) sends that chunk as raw u32, so the
+// validation kernel sees and rejects it as before.  GPA_NO_PACKED_UPLOAD=1 disables it.
+uint32_t pack_bits(uint32_t n_items) {
+  if (const char* e = getenv("GPA_NO_PACKED_UPLOAD"))
+    if (*e && *e != '0') return 0;
+  uint32_t b = 1;
+  while (b < 32 && (1ull << b) < n_items) ++b;
+  return b <= 16 ? b : 0;
+}
+
+struct PackStage {   // per thread and device: three host staging buffers + one device buffer
+  uint32_t* h[3] = {nullptr, nullptr, nullptr};
+  cudaEvent_t ev[3] = {nullptr, nullptr, nullptr};   // the H2D out of h[i] done
+  bool pending[3] = {false, false, false};
+  size_t cap = 0;                                    // words per buffer
+  PBuf<uint32_t> d;
+  void ensure(size_t words) {
+    if (!ev[0])
+      for (auto& e : ev) GPA_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    if (words <= cap) return;
+    for (int i = 0; i < 3; ++i) {
+      if (pending[i]) GPA_CUDA(cudaEventSynchronize(ev[i]));
+      pending[i] = false;
+      if (h[i]) cudaFreeHost(h[i]);
+      h[i] = nullptr;
+    }
+    cap = 0;
+    for (auto& x : h) GPA_CUDA(cudaHostAlloc(reinterpret_cast<void**>(&x), words * 4, cudaHostAllocDefault));
+    cap = words;
+    d.ensure(words);
+  }
+  ~PackStage() {
+    for (int i = 0; i < 3; ++i) {
+      if (pending[i]) cudaEventSynchronize(ev[i]);
+      if (h[i]) cudaFreeHost(h[i]);
+      if (ev[i]) cudaEventDestroy(ev[i]);
+    }
+  }
+};
+PackStage& pack_stage(int device) {
+  thread_local std::map<int, PackStage> m;
+  return m[device];
+}
+
+// one block of 32 ids -> B words (B a compile-time constant: straight-line shifts and ORs)
+template <uint32_t B>
+inline uint32_t pack_block(const uint32_t* __restrict__ src, uint32_t* __restrict__ dst) {
+  uint32_t orv = 0;
+  uint64_t acc = 0;
+  uint32_t nb = 0, k = 0;
+#pragma GCC unroll 32
+  for (uint32_t i = 0; i < 32; ++i) {
+    const uint32_t v = src[i];
+    orv |= v;
+    acc |= (uint64_t)v << nb;
+    nb += B;
+    if (nb >= 32) {
+      dst[k++] = (uint32_t)acc;
+      acc >>= 32;
+      nb -= 32;
+    }
+  }
+  return orv;
+}
+
+template <uint32_t B>
+uint32_t pack_range(const uint32_t* items, uint64_t n, uint64_t blk0, uint64_t blk1, uint32_t* words) {
+  uint32_t orv = 0;
+  for (uint64_t blk = blk0; blk < blk1; ++blk) {
+    const uint64_t j0 = blk * 32;
+    if (j0 + 32 <= n) {
+      orv |= pack_block<B>(items + j0, words + blk * B);
+    } else {   // the ragged last block: zero-padded copy
+      uint32_t tmp[32] = {};
+      for (uint64_t j = j0; j < n; ++j) tmp[j - j0] = items[j];
+      orv |= pack_block<B>(tmp, words + blk * B);
+    }
+  }
+  return orv;
+}
+
+using PackFn = uint32_t (*)(const uint32_t*, uint64_t, uint64_t, uint64_t, uint32_t*);
+template <uint32_t... Bs>
+constexpr std::array<PackFn, sizeof...(Bs)> pack_table(std::integer_sequence<uint32_t, Bs...>) {
+  return {&pack_range<Bs + 1>...};
+}
+
+// items[0, n) -> b-bit fields in words (ceil(n / 32) * b words); returns false if an id >= 2^b
+bool pack_items(const uint32_t* items, uint64_t n, uint32_t b, uint32_t* words) {
+  static constexpr auto table = pack_table(std::make_integer_sequence<uint32_t, 16>{});
+  const PackFn fn = table[b - 1];
+  const uint64_t nblk = (n + 31) / 32;
+  const size_t T = std::max<size_t>(1, std::min<uint64_t>(pool_threads() * 4, (nblk + 1023) / 1024));
+  std::vector<uint32_t> ors(T, 0);
+  parallel_for(T, [&](size_t t) { ors[t] = fn(items, n, nblk * t / T, nblk * (t + 1) / T, words); });
+  uint32_t o = 0;
+  for (uint32_t v : ors) o |= v;
+  return (o >> b) == 0;
+}
 }  // namespace
 
 bool ingest_overlap_eligible(const gpa_tx_csr* db) {
@@ -140,11 +248,36 @@ gpa_bitset* bitset_build_overlapped(const gpa_tx_csr* db, uint64_t row_min_count
     std::vector<cudaEvent_t>& v;
     ~EvGuard() { for (auto e : v) if (e) cudaEventDestroy(e); }
   } ev_guard{up};
+  const uint32_t pbits = pack_bits(n_items);
+  PackStage* ps = nullptr;
+  if (pbits) {
+    uint64_t max_items = 0;
+    for (size_t c = 0; c < C; ++c) max_items = std::max<uint64_t>(max_items, db->offsets[cut[c + 1]] - db->offsets[cut[c]]);
+    ps = &pack_stage(bs->device);
+    ps->ensure((max_items + 31) / 32 * pbits + 1);
+  }
+  uint64_t packed_bytes = 0;
   auto upload = [&](size_t c) {
     const uint64_t a = cut[c], b = cut[c + 1];
     const uint64_t ia = db->offsets[a], ib = db->offsets[b];
     GPA_CUDA(cudaMemcpyAsync(d_off.p + a, db->offsets + a, (b - a + 1) * 8, cudaMemcpyHostToDevice, cs));
-    if (ib > ia) GPA_CUDA(cudaMemcpyAsync(d_items.p + ia, db->items + ia, (ib - ia) * 4, cudaMemcpyHostToDevice, cs));
+    bool raw = ib > ia;
+    if (ib > ia && ps) {
+      const int slot = (int)(c % 3);
+      if (ps->pending[slot]) GPA_CUDA(cudaEventSynchronize(ps->ev[slot]));   // chunk c - 3's H2D is done
+      ps->pending[slot] = false;
+      const uint64_t n = ib - ia, words = (n + 31) / 32 * pbits;
+      if (pack_items(db->items + ia, n, pbits, ps->h[slot])) {
+        GPA_CUDA(cudaMemcpyAsync(ps->d.p, ps->h[slot], words * 4, cudaMemcpyHostToDevice, cs));
+        GPA_CUDA(cudaEventRecord(ps->ev[slot], cs));
+        ps->pending[slot] = true;
+        // (the single device buffer is reused by the next chunk's H2D after this kernel: stream order)
+        launch_unpack_items(ps->d.p, n, pbits, d_items.p + ia, bs->n_sms, cs);
+        packed_bytes += words * 4;
+        raw = false;
+      }
+    }
+    if (raw) GPA_CUDA(cudaMemcpyAsync(d_items.p + ia, db->items + ia, (ib - ia) * 4, cudaMemcpyHostToDevice, cs));
     GPA_CUDA(cudaEventCreateWithFlags(&up[c], cudaEventDisableTiming));
     GPA_CUDA(cudaEventRecord(up[c], cs));
   };
@@ -316,8 +449,9 @@ gpa_bitset* bitset_build_overlapped(const gpa_tx_csr* db, uint64_t row_min_count
   bs->build_ms[2] = wall_ms() - t2;
   if (trace_enabled())
     fprintf(stderr, "[gpa] overlapped ingest: %zu chunks, R0 = %u rows, L1 = %u rows (%s), upload+hist+build+pairs "
-            "%.2f ms (pairs kernels %.2f ms), finish %.2f ms\n", C, nr0, bs->n_rows, subset ? "subset" : "rebuilt",
-            t1 - t0, pairs_ms, wall_ms() - t1);
+            "%.2f ms (pairs kernels %.2f ms), finish %.2f ms; items sent as %u-bit fields (%.1f MB)\n", C, nr0,
+            bs->n_rows, subset ? "subset" : "rebuilt", t1 - t0, pairs_ms, wall_ms() - t1, pbits ? pbits : 32,
+            (pbits ? packed_bytes : nnz * 4) / 1e6);
   guard.b = nullptr;
   return bs;
 }

@@ -433,6 +433,26 @@ def test_overlapped_ingest_row_estimate_miss():
     assert_mine_equal(res, ref)
 
 
+def test_packed_upload_invalid_and_unpacked_paths(monkeypatch):
+    """Host input on the overlapped path uploads the item ids bit-packed (b = ceil(log2 n_items)
+    bits): results equal the oracle with packing and with GPA_NO_PACKED_UPLOAD (read per call); an id
+    >= n_items that still fits in b bits, and one that does not (the chunk then goes raw), are both
+    rejected by the validation -- in a late chunk, not only chunk 0."""
+    ds = gen.make("accidents")          # 468 item ids -> 9-bit fields
+    theta = oracle.min_count(ds.n_tx, "0.30")
+    ref = oracle.mine_ds(ds, theta)
+    assert_mine_equal(gpa.mine(ds, min_count=theta, keep_candidates=True), ref)
+    monkeypatch.setenv("GPA_NO_PACKED_UPLOAD", "1")
+    assert_mine_equal(gpa.mine(ds, min_count=theta, keep_candidates=True), ref)
+    monkeypatch.delenv("GPA_NO_PACKED_UPLOAD")
+    for bad in (ds.n_items, 1 << 12):   # in range of 9 bits (>= n_items) / out of 9 bits
+        items = ds.items.copy()
+        items[len(items) - 5] = bad
+        with pytest.raises(gpa.GpaError) as e:
+            gpa.mine(ds.offsets, items, ds.n_items, min_count=theta)
+        assert e.value.status == 1
+
+
 def test_c_example_fimi_roundtrip(tmp_path, fig2):
     """The C example (C ABI only) on the Fig. 2 database written as a FIMI file: every frequent
     itemset and support as the oracle computes them."""
