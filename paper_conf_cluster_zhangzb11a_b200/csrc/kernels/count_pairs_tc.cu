@@ -198,7 +198,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     mbar_init(done, 1);
     for (int s = 0; s < kBitStages; ++s) {
       mbar_init(bfull0 + 8 * s, 1);
-      mbar_init(bempty0 + 8 * s, kProducerGroups * kProducerWarps);
+      mbar_init(bempty0 + 8 * s, kProducerWarps);   // a bit stage is expanded by one producer group
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
@@ -213,9 +213,9 @@ __global__ void __launch_bounds__(kThreads, 1)
   const uint32_t tmem = s_tmem;
 
   if (warp >= kEpiWarps) {
-    // ---------------- producers: group g = 0, 1 (warps 4..15, 16..27) expands the operand stages
-    // i = g mod 2, i.e. half g of every bit stage; thread p owns tile row p (A rows 0..127, then
-    // B rows 0..255) -- two groups keep two stages in flight per row
+    // ---------------- producers: group g = 0, 1 (warps 4..15, 16..27) expands the bit stages
+    // j = g mod 2 (both of their operand stages); thread p owns tile row p (A rows 0..127, then
+    // B rows 0..255) -- two groups keep two bit stages in flight per row
     const uint32_t g = (uint32_t)(warp - kEpiWarps) / kProducerWarps;
     const uint32_t p = threadIdx.x - (kEpiWarps + g * kProducerWarps) * 32;
     const bool is_a = p < kM;
@@ -230,12 +230,19 @@ __global__ void __launch_bounds__(kThreads, 1)
     Shr sh;
 #pragma unroll
     for (int j = 0; j < 8; ++j) sh.m[j] = j ? one << (32 - j) : 0u;
-    for (uint32_t i = g; i < n_st; i += 2) {
-      const uint32_t j = i >> 1, h = i & 1, bslot = j % kBitStages;
+    // group g expands the bit stages j = g mod 2, both operand stages (halves) of each: one bit-ring
+    // wait / release per two operand stages
+    for (uint32_t j = g; j < n_bst; j += 2) {
+      const uint32_t bslot = j % kBitStages;
       mbar_wait(bfull0 + 8 * bslot, (j / kBitStages) & 1);
-      const uint4 v = lds128(brow + bslot * kBitStageBytes + ((h ^ bsw) << 4));
+      const uint32_t brs = brow + bslot * kBitStageBytes;
+      const uint4 v0 = lds128(brs + (bsw << 4)), v1 = lds128(brs + ((bsw ^ 1u) << 4));
       __syncwarp();
       if (lane == 0) mbar_arrive(bempty0 + 8 * bslot);
+#pragma unroll
+      for (uint32_t h = 0; h < 2; ++h) {
+      const uint32_t i = 2 * j + h;
+      const uint4 v = h ? v1 : v0;
       const uint32_t slot = i % kStages;
       mbar_wait(empty0 + 8 * slot, ((i / kStages) & 1) ^ 1);
       if (half && !is_a && r >= kN / 2) {
@@ -258,6 +265,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       }
       __syncwarp();
       if (lane == 0) mbar_arrive(full0 + 8 * slot);
+      }
     }
   } else {
     // ---------------- warp 0 lane 0: MMA issue
