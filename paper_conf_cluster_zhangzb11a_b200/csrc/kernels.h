@@ -146,6 +146,11 @@ struct DeviceScratch {
   uint32_t* u32g(size_t n, cudaStream_t s) { g.ensure(n ? n : 1, s); return g.p; }
   uint32_t* u32h(size_t n, cudaStream_t s) { h.ensure(n ? n : 1, s); return h.p; }
   uint32_t* u32i(size_t n, cudaStream_t s) { i.ensure(n ? n : 1, s); return i.p; }
+  // one generation's sizes, read by the host in ONE copy: [0] |C_k|, [1] groups, [2..5] the lists'
+  // totals (u64 x 2: build items, words), [6..9] class-table counters (classes, max lane words,
+  // u64 compressed words), [10] |L_{k-1}|
+  DBuf<uint32_t> blk;
+  uint32_t* size_block(cudaStream_t s) { blk.ensure(16, s); return blk.p; }
   // the join's per-member survivor masks (stage 1 -> stage 2, lvl::join_warp)
   DBuf<unsigned long long> surv;
   unsigned long long* surv64(size_t n, cudaStream_t s) { surv.ensure(n ? n : 1, s); return surv.p; }
@@ -235,9 +240,11 @@ struct ProjPending {
 // too many classes): use complete intersection.
 // n_dev: L is device-sized (n = its host upper bound, the count at *n_dev); set pp.n to the count
 // before proj_build_finish.
+// d_block (optional): the generation's size block (DeviceScratch::size_block): the totals and the
+// class-table counters are written to words 2..9 of it instead of the workspace's own
 bool proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const DeviceProj* prev,
                       const uint32_t* rows, uint64_t pitch_words, uint32_t n_rows, DeviceScratch& scratch, int n_sms,
-                      cudaStream_t s, ProjPending& pp, const uint32_t* n_dev = nullptr);
+                      cudaStream_t s, ProjPending& pp, const uint32_t* n_dev = nullptr, uint32_t* d_block = nullptr);
 bool proj_build_finish(const ProjPending& pp, const uint64_t T[2], const uint32_t sm[4], DeviceProj& out, int n_sms,
                        cudaStream_t s, cudaEvent_t ev_build);
 // counts[m] += popc(V_gpar[g] & V_eidx[m]) for every candidate m of group g (counts zeroed by the caller)

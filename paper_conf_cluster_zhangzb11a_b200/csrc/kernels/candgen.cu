@@ -37,11 +37,15 @@ __device__ __forceinline__ void hash_insert(const uint32_t* row, uint32_t w, uin
 // L_k's positions: pos[m] = #{m' < m : count >= theta}, *count = |L_k| (one launch)
 __global__ void __launch_bounds__(sd::kScanThreads, 1) ge_scan_kernel(const uint32_t* __restrict__ counts, uint32_t M,
                                                                       uint32_t theta, uint32_t* __restrict__ pos,
-                                                                      uint32_t* count, uint32_t* sflags, uint64_t* agg,
-                                                                      uint64_t* inc, uint32_t epoch) {
+                                                                      uint32_t* count, uint32_t* count2, uint32_t* sflags,
+                                                                      uint64_t* agg, uint64_t* inc, uint32_t epoch) {
   sd::scan_tile<uint32_t>(
       M, [&](uint32_t m) { return counts[m] >= theta ? 1u : 0u; }, [&](uint32_t m, uint32_t e, uint32_t) { pos[m] = e; },
-      [&](uint32_t t) { *count = t; }, sflags, agg, inc, epoch);
+      [&](uint32_t t) {
+        *count = t;
+        if (count2) *count2 = t;   // |L_k| into the next generation's size block as well
+      },
+      sflags, agg, inc, epoch);
 }
 
 // k = 2: candidate m is the pair (a, b) of pair_index order over n rows
@@ -189,10 +193,10 @@ void exclusive_scan(const uint32_t* in, uint32_t* out, uint32_t n, uint32_t* tot
 }
 
 void ge_scan(const uint32_t* counts, uint32_t M, uint32_t theta, uint32_t* pos, uint32_t* count, DeviceScratch& scratch,
-             cudaStream_t s) {
+             cudaStream_t s, uint32_t* count2 = nullptr) {
   const uint32_t tiles = scan_tiles(M);
   const uint32_t ep = scan_epoch(scratch.scan, tiles, s);
-  { ge_scan_kernel<<<tiles, sd::kScanThreads, 0, s>>>(counts, M, theta, pos, count, scratch.scan.flags.p,
+  { ge_scan_kernel<<<tiles, sd::kScanThreads, 0, s>>>(counts, M, theta, pos, count, count2, scratch.scan.flags.p,
                                                       scratch.scan.agg.p, scratch.scan.inc.p, ep); note_launch(); }
   GPA_CUDA(cudaGetLastError());
 }
@@ -203,10 +207,11 @@ namespace {
 void threshold_impl(const uint32_t* counts, uint32_t M, uint32_t theta, uint32_t k, uint32_t n_rows, const uint32_t* sel,
                     const uint32_t* prefix, const uint32_t* ext_off, const uint32_t* ext, uint32_t G,
                     const uint32_t* gpar, const uint32_t* eidx, DeviceLevel& out, DeviceScratch& scratch, int n_sms,
-                    cudaStream_t s, uint32_t cap, const uint32_t* ior, uint32_t* items, uint32_t* sup_out) {
+                    cudaStream_t s, uint32_t cap, const uint32_t* ior, uint32_t* items, uint32_t* sup_out,
+                    uint32_t* count2) {
   uint32_t* pos = scratch.u32b(M, s);
   out.count.ensure(1, s);
-  ge_scan(counts, M, theta, pos, out.count.p, scratch, s);
+  ge_scan(counts, M, theta, pos, out.count.p, scratch, s, count2);
   out.rows.ensure((size_t)std::max<uint32_t>(cap, 1) * k, s);
   out.sup.ensure(std::max<uint32_t>(cap, 1), s);
   out.par_a.ensure(std::max<uint32_t>(cap, 1), s);
@@ -249,7 +254,7 @@ uint32_t device_threshold(const uint32_t* counts, uint32_t M, uint32_t theta, ui
   GPA_CUDA(cudaMemcpyAsync(&F, out.count.p, 4, cudaMemcpyDeviceToHost, s));
   stream_wait(s);
   if (F) threshold_impl(counts, M, theta, k, n_rows, sel, prefix, ext_off, ext, G, gpar, eidx, out, scratch, n_sms, s,
-                        F, nullptr, nullptr, nullptr);
+                        F, nullptr, nullptr, nullptr, nullptr);
   out.n = F;
   return F;
 }
@@ -265,7 +270,7 @@ void device_threshold_async(const uint32_t* counts, uint32_t M, uint32_t theta, 
   out.n_max = 0;
   if (M == 0) return;
   threshold_impl(counts, M, theta, k, n_rows, sel, prefix, ext_off, ext, G, gpar, eidx, out, scratch, n_sms, s, M, ior,
-                 items, sup_out);
+                 items, sup_out, scratch.size_block(s) + 10);
   out.n_dev = out.count.p;   // |L_k| stays on the device until the next generation's synchronisation
   out.n_max = M;
 }
@@ -296,7 +301,7 @@ bool device_candgen_begin(const DeviceLevel& L, DeviceBatch& out, DeviceScratch&
   uint32_t* run_ex = scratch.u32b(n, s);
   uint32_t* cnt = scratch.u32c(n, s);
   uint32_t* bound = scratch.u32d(n + 1, s);
-  uint32_t* sizes = scratch.u32h(4, s);  // [0] = M, [1] = G
+  uint32_t* sizes = scratch.size_block(s);  // [0] = M, [1] = G
   // the hash set over L for the prune probes was filled by the scatter that wrote L (threshold_impl)
   GPA_REQUIRE(scratch.hash_cap >= 2 * n + 1 && scratch.hash_n == n && scratch.i.p, GPA_ERR_STATE,
               "join: no hash set over this level");
@@ -342,7 +347,7 @@ void device_candgen_finish(const DeviceLevel& L, DeviceBatch& out, DeviceScratch
   const uint32_t cap = scratch.hash_cap;   // the table stage 1 built (sized for its upper bound)
   { join_kernel<true><<<grid_for(32ull * n, n_sms), kThreads, 0, run>>>(L.rows.p, n, w, scratch.a.p, scratch.b.p,
         scratch.d.p, scratch.i.p, cap - 1, scratch.c.p, scratch.e.p, scratch.g.p, out.prefix.p, out.ext_off.p,
-        out.ext.p, out.gpar.p, out.eidx.p, nullptr, scratch.h.p, scratch.surv.p); note_launch(); }   // + ext_off[G] = M
+        out.ext.p, out.gpar.p, out.eidx.p, nullptr, scratch.blk.p, scratch.surv.p); note_launch(); }   // + ext_off[G] = M
   GPA_CUDA(cudaGetLastError());
   out.M = M;
   out.G = G;

@@ -696,7 +696,7 @@ Src make_src(const ProjPending& pp) {
 
 bool proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const DeviceProj* prev,
                       const uint32_t* rows, uint64_t pitch_words, uint32_t n_rows, DeviceScratch& scratch, int n_sms,
-                      cudaStream_t s, ProjPending& pp, const uint32_t* n_dev) {
+                      cudaStream_t s, ProjPending& pp, const uint32_t* n_dev, uint32_t* d_block) {
   pp = ProjPending();
   pp.n = n;
   pp.par_a = par_a;
@@ -725,10 +725,14 @@ bool proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, 
   W.ex.ensure(n);
   W.bound.ensure(n + 1);
   W.small.ensure(4);   // zeroed by cls_scan_kernel
+  W.tot.ensure(2);
+  // counters and totals in the caller's size block (one host read per generation) or our own
+  uint32_t* const small = d_block ? d_block + 6 : W.small.p;
+  uint64_t* const tot = d_block ? reinterpret_cast<uint64_t*>(d_block + 2) : W.tot.p;
   {
     const uint32_t tiles = scan_tiles(n);
     const uint32_t ep = scan_epoch(W.scan, tiles, s);
-    cls_scan_kernel<<<tiles, sd::kScanThreads, 0, s>>>(par_a, n, W.flag.p, W.ex.p, W.bound.p, W.small.p, n_dev,
+    cls_scan_kernel<<<tiles, sd::kScanThreads, 0, s>>>(par_a, n, W.flag.p, W.ex.p, W.bound.p, small, n_dev,
                                                        W.scan.flags.p, W.scan.agg.p, W.scan.inc.p, ep);
     note_launch();
   }
@@ -740,28 +744,27 @@ bool proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, 
   W.cls_words.ensure(cmax);
   W.cls_base.ensure(cmax);
   W.len.ensure((size_t)cmax * 32);
-  W.tot.ensure(2);
   const unsigned wpb = kT / 32;
   if (!prev && gather3()) {  // generation 3: bit gather (pext3_kernel), natural-order lists
-    { seg3_kernel<<<(n_pairs + wpb - 1) / wpb, kT, 0, s>>>(rows, pitch_words, par_a, W.bound.p, W.small.p, cmax, n_pairs,
-          W.words.p, reinterpret_cast<unsigned long long*>(W.small.p + 2)); note_launch(); }
-    { cls3_pad_kernel<<<grid_for(cmax, n_sms), kT, 0, s>>>(W.words.p, W.bound.p, W.small.p, cmax, nseg, W.loc.p,
-          W.nwc.p, W.cls_words.p, W.items.p, W.small.p + 1, W.len.p); note_launch(); }
+    { seg3_kernel<<<(n_pairs + wpb - 1) / wpb, kT, 0, s>>>(rows, pitch_words, par_a, W.bound.p, small, cmax, n_pairs,
+          W.words.p, reinterpret_cast<unsigned long long*>(small + 2)); note_launch(); }
+    { cls3_pad_kernel<<<grid_for(cmax, n_sms), kT, 0, s>>>(W.words.p, W.bound.p, small, cmax, nseg, W.loc.p,
+          W.nwc.p, W.cls_words.p, W.items.p, small + 1, W.len.p); note_launch(); }
   } else {
     { seg_popc_kernel<<<(n_pairs + wpb - 1) / wpb, kT, 0, s>>>(
-          src, par_a, W.bound.p, W.small.p, cmax, nseg, n_pairs, W.words.p,
-          reinterpret_cast<unsigned long long*>(W.small.p + 2)); note_launch(); }
+          src, par_a, W.bound.p, small, cmax, nseg, n_pairs, W.words.p,
+          reinterpret_cast<unsigned long long*>(small + 2)); note_launch(); }
     { cls_pad_kernel<<<(cmax + wpb - 1) / wpb, kT, 0, s>>>(
-          W.words.p, W.bound.p, W.small.p, cmax, nseg, W.loc.p, W.nwc.p, W.cls_words.p, W.items.p, W.small.p + 1,
+          W.words.p, W.bound.p, small, cmax, nseg, W.loc.p, W.nwc.p, W.cls_words.p, W.items.p, small + 1,
           W.len.p);
       note_launch(); }
   }
   // tot = {pext items, list words}: the totals of the two scans
-  scan_excl_u32(W.items.p, W.item_off.p, n_pairs, W.tot.p, W.scan, s);
-  scan_excl_u64(W.cls_words.p, W.cls_base.p, cmax, W.tot.p + 1, W.scan, s);
+  scan_excl_u32(W.items.p, W.item_off.p, n_pairs, tot, W.scan, s);
+  scan_excl_u64(W.cls_words.p, W.cls_base.p, cmax, tot + 1, W.scan, s);
   GPA_CUDA(cudaGetLastError());
-  pp.d_tot = W.tot.p;
-  pp.d_small = W.small.p;
+  pp.d_tot = tot;
+  pp.d_small = small;
   return true;
 }
 

@@ -537,29 +537,26 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
       // emitting join runs on aux_s while the lists are built on s
       const uint32_t* d_sizes = nullptr;
       // the class tables (aux_s) are independent of the join's stage 1 (s): both read L_{k-1}
+      // the generation's sizes (|C_k|, groups, list totals, class-table counters, |L_{k-1}|) land in
+      // one device block: ONE copy and ONE synchronisation per generation
+      uint32_t* blk = scratch.size_block(s);
       GPA_CUDA(cudaEventRecord(aux_evs.e[2], s));
       GPA_CUDA(cudaStreamWaitEvent(aux_s.s, aux_evs.e[2], 0));
-      // L_{k-1} is device-sized: |L_{k-1}| comes back with the sizes of C_k and of the lists -- ONE
-      // synchronisation per generation
       const uint32_t n_up = Ld.n_dev ? Ld.n_max : Ld.n;
       if (device_candgen_begin(Ld, Bd, scratch, bs->n_sms, s, &d_sizes)) {
         if (trace_enabled()) GPA_CUDA(cudaEventRecord(trace_ev[0], s));
         uint32_t* hs = host_sizes();
-        if (proj_build_begin(n_up, Ld.par_a.p, Ld.par_b.p, k == 3 ? nullptr : Pprev, bs->rows.p, bs->pitch_words,
-                             bs->n_rows, scratch, bs->n_sms, aux_s.s, ppend, Ld.n_dev)) {
-          GPA_CUDA(cudaMemcpyAsync(hs + 2, ppend.d_tot, 16, cudaMemcpyDeviceToHost, aux_s.s));
-          GPA_CUDA(cudaMemcpyAsync(hs + 6, ppend.d_small, 16, cudaMemcpyDeviceToHost, aux_s.s));
-        } else {
+        if (!proj_build_begin(n_up, Ld.par_a.p, Ld.par_b.p, k == 3 ? nullptr : Pprev, bs->rows.p, bs->pitch_words,
+                              bs->n_rows, scratch, bs->n_sms, aux_s.s, ppend, Ld.n_dev, blk))
           proj_on = false;   // lists not addressable: complete intersection from this generation on
-        }
         if (trace_enabled()) GPA_CUDA(cudaEventRecord(trace_ev[1], aux_s.s));
-        GPA_CUDA(cudaMemcpyAsync(hs, d_sizes, 8, cudaMemcpyDeviceToHost, s));
-        if (Ld.n_dev) GPA_CUDA(cudaMemcpyAsync(hs + 10, Ld.n_dev, 4, cudaMemcpyDeviceToHost, s));
+        GPA_CUDA(cudaEventRecord(aux_evs.e[3], aux_s.s));   // the class tables are done
+        GPA_CUDA(cudaStreamWaitEvent(s, aux_evs.e[3], 0));
+        GPA_CUDA(cudaMemcpyAsync(hs, blk, 16 * 4, cudaMemcpyDeviceToHost, s));
         if (trace_enabled()) GPA_CUDA(cudaEventRecord(trace_ev[2], s));
         const double tw0 = now_ms();
         ht.mark("begin enqueued", k);
         stream_wait(s);
-        stream_wait(aux_s.s);
         const double tw1 = now_ms();
         ht.mark("sizes back", k);
         if (trace_enabled()) GPA_CUDA(cudaEventRecord(trace_ev[3], s));
@@ -595,8 +592,7 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
       const uint32_t* d_sizes = nullptr;
       if (device_candgen_begin(Ld, Bd, scratch, bs->n_sms, s, &d_sizes)) {
         uint32_t* hs = host_sizes();
-        GPA_CUDA(cudaMemcpyAsync(hs, d_sizes, 8, cudaMemcpyDeviceToHost, s));
-        if (Ld.n_dev) GPA_CUDA(cudaMemcpyAsync(hs + 10, Ld.n_dev, 4, cudaMemcpyDeviceToHost, s));
+        GPA_CUDA(cudaMemcpyAsync(hs, d_sizes, 16 * 4, cudaMemcpyDeviceToHost, s));   // the size block: [10] = |L_{k-1}|
         stream_wait(s);
         if (Ld.n_dev) {
           Ld.n = hs[10];
