@@ -335,12 +335,15 @@ void device_candgen_finish(const DeviceLevel& L, DeviceBatch& out, DeviceScratch
   const uint32_t n = L.n, w = L.k;
   out.M = out.G = 0;
   if (M == 0) return;
-  out.prefix.ensure((size_t)G * w, s);
-  out.ext_off.ensure(G + 1, s);
-  out.ext.ensure(M, s);
-  out.gpar.ensure(G, s);
-  out.eidx.ensure(M, s);
-  if (run != s) {
+  // run != s with ev == nullptr: the caller already made `run` wait for s at the end of stage 1, and s
+  // may hold later work -- the batch is then allocated (stream-ordered) on `run` itself
+  const cudaStream_t as = run != s && !ev ? run : s;
+  out.prefix.ensure((size_t)G * w, as);
+  out.ext_off.ensure(G + 1, as);
+  out.ext.ensure(M, as);
+  out.gpar.ensure(G, as);
+  out.eidx.ensure(M, as);
+  if (run != s && ev) {
     GPA_CUDA(cudaEventRecord(ev, s));
     GPA_CUDA(cudaStreamWaitEvent(run, ev, 0));
   }

@@ -183,18 +183,25 @@ void record_level(gpa_result* R, const gpa_bitset* bs, uint32_t k, const Grouped
 // proj_build_begin shared the generation's one host synchronisation with the join
 // (the sizes T, sm came back with |C_k|): the list build (pext) on s, overlapping the emitting
 // join on the auxiliary stream; the supports wait for both (aux_done).
-bool count_projected_staged(gpa_bitset* bs, uint32_t k, const DeviceBatch& B, DeviceProj& cur, const ProjPending& pp,
-                            const uint64_t T[2], const uint32_t sm[4], cudaEvent_t aux_done, CountStats* cs,
-                            uint64_t src_words) {
+// The projected lists of L_{k-1} (entry offsets, list build) on the mining stream, right after the
+// generation's size read -- before the emitting join is enqueued, so the build starts first.
+bool proj_build_stage(gpa_bitset* bs, uint32_t k, DeviceProj& cur, const ProjPending& pp, const uint64_t T[2],
+                      const uint32_t sm[4], CountStats* cs) {
   cudaStream_t s = bs->stream;
-  const double t0 = now_ms();
   GPA_CUDA(cudaEventRecord(cs->e0, s));
   // GPA_PROJ_TEST_MAX_K=k: behave as if the lists of generations > k did not fit (tests drive the
   // mid-run fallback to complete intersection with it)
   const char* tk = getenv("GPA_PROJ_TEST_MAX_K");
-  const bool ok = !(tk && k > (uint32_t)atoi(tk)) && proj_build_finish(pp, T, sm, cur, bs->n_sms, s, cs->ep);
+  return !(tk && k > (uint32_t)atoi(tk)) && proj_build_finish(pp, T, sm, cur, bs->n_sms, s, cs->ep);
+}
+
+// The supports of C_k from the lists (count_proj), once the emitting join (aux stream) is done.
+bool proj_count_stage(gpa_bitset* bs, uint32_t k, const DeviceBatch& B, DeviceProj& cur, const ProjPending& pp,
+                      bool built, cudaEvent_t aux_done, CountStats* cs, uint64_t src_words) {
+  cudaStream_t s = bs->stream;
+  const double t0 = now_ms();
   GPA_CUDA(cudaStreamWaitEvent(s, aux_done, 0));
-  if (!ok) return false;
+  if (!built) return false;
   bs->d_counts.ensure(B.M, s);
   GPA_CUDA(cudaMemsetAsync(bs->d_counts.p, 0, (size_t)B.M * 4, s));
   GPA_CUDA(cudaEventRecord(cs->eb, s));
@@ -500,6 +507,7 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
     EvTriple& ev = events.emplace_back();
     GPA_CUDA(cudaEventRecord(ev.e[5], s));
     CountStats cs;
+    bool lists_built = false;   // proj_build_stage ran for this generation
     GroupedBatch batch;
     uint64_t M = 0, G = 0;
     if (k == 2) {
@@ -553,6 +561,10 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
         GPA_CUDA(cudaEventRecord(aux_evs.e[3], aux_s.s));   // the class tables are done
         GPA_CUDA(cudaStreamWaitEvent(s, aux_evs.e[3], 0));
         GPA_CUDA(cudaMemcpyAsync(hs, blk, 16 * 4, cudaMemcpyDeviceToHost, s));
+        // the emitting join (aux) depends on stage 1 only: ordered here, before the list build that
+        // s runs right after the read
+        GPA_CUDA(cudaEventRecord(aux_evs.e[0], s));
+        GPA_CUDA(cudaStreamWaitEvent(aux_s.s, aux_evs.e[0], 0));
         if (trace_enabled()) GPA_CUDA(cudaEventRecord(trace_ev[2], s));
         const double tw0 = now_ms();
         ht.mark("begin enqueued", k);
@@ -564,16 +576,22 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
         G = hs[1];
         std::memcpy(pT, hs + 2, 16);
         std::memcpy(psm, hs + 6, 16);
-        if (Ld.n_dev) {
+        const bool l_open = Ld.n_dev != nullptr;
+        if (l_open) {
           Ld.n = hs[10];
           Ld.n_dev = nullptr;
-          finalize(pending.back(), Ld.n);
         }
         const double tw2 = now_ms();
         ppend.n = Ld.n;   // the class tables ran over the upper bound; the lists are for |L_{k-1}| entries
-        device_candgen_finish(Ld, Bd, scratch, bs->n_sms, s, (uint32_t)M, (uint32_t)G, aux_s.s, aux_evs.e[0]);
+        // the list build first (the critical path), then the emitting join on the side stream
+        cs.e0 = ev.e[0];
+        cs.ep = ev.e[3];
+        cs.eb = ev.e[4];
+        if (proj_on && M > 0) lists_built = proj_build_stage(bs, k, *Pcur, ppend, pT, psm, &cs);
+        device_candgen_finish(Ld, Bd, scratch, bs->n_sms, s, (uint32_t)M, (uint32_t)G, aux_s.s, nullptr);
         GPA_CUDA(cudaEventRecord(aux_evs.e[1], aux_s.s));
         aux_join = true;
+        if (l_open) finalize(pending.back(), Ld.n);   // L_{k-1}'s D2H on the copy stream
         ht.mark("join finished", k);
         const double tw3 = now_ms();
         if (trace_enabled()) {
@@ -635,7 +653,7 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
       count_all_pairs(bs, opt.count_kernel, &cs);
     } else {
       const uint64_t src_words = k == 3 ? (uint64_t)bs->n_rows * bs->pitch_words : Pprev->words;
-      if (proj_on && count_projected_staged(bs, k, Bd, *Pcur, ppend, pT, psm, aux_evs.e[1], &cs, src_words)) {
+      if (proj_on && proj_count_stage(bs, k, Bd, *Pcur, ppend, lists_built, aux_evs.e[1], &cs, src_words)) {
         std::swap(Pprev, Pcur);
       } else {
         // complete intersection from the static bitset (requested, or the projected lists did not
