@@ -91,8 +91,9 @@ __global__ void __launch_bounds__(sd::kScanThreads, 1) cls_scan_kernel(const uin
 __global__ void seg_popc_kernel(Src src, const uint32_t* __restrict__ par_a, const uint32_t* __restrict__ bound,
                                 const uint32_t* __restrict__ n_cls, uint32_t cmax, uint32_t nseg, uint32_t n_pairs,
                                 uint32_t* __restrict__ words, unsigned long long* __restrict__ in_words) {
-  const uint32_t p = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  if (p < n_pairs) seg_popc_warp(p, src, par_a, bound, *n_cls, cmax, words, in_words);
+  const uint32_t nc = *n_cls, n_warps = (gridDim.x * blockDim.x) >> 5;
+  for (uint32_t p = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; p < n_pairs; p += n_warps)
+    seg_popc_warp(p, src, par_a, bound, nc, cmax, words, in_words);
 }
 
 __global__ void cls_pad_kernel(const uint32_t* __restrict__ words, const uint32_t* __restrict__ bound,
@@ -100,8 +101,9 @@ __global__ void cls_pad_kernel(const uint32_t* __restrict__ words, const uint32_
                                uint32_t* __restrict__ loc, uint32_t* __restrict__ nwc,
                                uint64_t* __restrict__ cls_words, uint32_t* __restrict__ items,
                                uint32_t* __restrict__ max_lw, uint32_t* __restrict__ len) {
-  const uint32_t c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  if (c < cmax) cls_pad_warp(c, words, bound, *n_cls, cmax, nseg, loc, nwc, cls_words, items, max_lw, len);
+  const uint32_t nc = *n_cls, n_warps = (gridDim.x * blockDim.x) >> 5;
+  for (uint32_t c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < cmax; c += n_warps)
+    cls_pad_warp(c, words, bound, nc, cmax, nseg, loc, nwc, cls_words, items, max_lw, len);
 }
 
 // warp per entry j: its vector (offset, words; entries of single-member classes get none), and
@@ -310,8 +312,9 @@ __device__ __forceinline__ void pext_item(const uint32_t* __restrict__ mp, const
 __global__ void seg3_kernel(const uint32_t* __restrict__ rows, uint64_t pitch, const uint32_t* __restrict__ par_a,
                             const uint32_t* __restrict__ bound, const uint32_t* __restrict__ n_cls, uint32_t cmax,
                             uint32_t n_pairs, uint32_t* __restrict__ w3, unsigned long long* __restrict__ in_words) {
-  const uint32_t p = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  if (p < n_pairs) seg3_warp(p, rows, pitch, par_a, bound, *n_cls, cmax, w3, in_words);
+  const uint32_t nc = *n_cls, n_warps = (gridDim.x * blockDim.x) >> 5;
+  for (uint32_t p = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; p < n_pairs; p += n_warps)
+    seg3_warp(p, rows, pitch, par_a, bound, nc, cmax, w3, in_words);
 }
 
 __global__ void cls3_pad_kernel(const uint32_t* __restrict__ w3, const uint32_t* __restrict__ bound,
@@ -746,15 +749,15 @@ bool proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, 
   W.len.ensure((size_t)cmax * 32);
   const unsigned wpb = kT / 32;
   if (!prev && gather3()) {  // generation 3: bit gather (pext3_kernel), natural-order lists
-    { seg3_kernel<<<(n_pairs + wpb - 1) / wpb, kT, 0, s>>>(rows, pitch_words, par_a, W.bound.p, small, cmax, n_pairs,
+    { seg3_kernel<<<grid_for(32ull * n_pairs, n_sms), kT, 0, s>>>(rows, pitch_words, par_a, W.bound.p, small, cmax, n_pairs,
           W.words.p, reinterpret_cast<unsigned long long*>(small + 2)); note_launch(); }
     { cls3_pad_kernel<<<grid_for(cmax, n_sms), kT, 0, s>>>(W.words.p, W.bound.p, small, cmax, nseg, W.loc.p,
           W.nwc.p, W.cls_words.p, W.items.p, small + 1, W.len.p); note_launch(); }
   } else {
-    { seg_popc_kernel<<<(n_pairs + wpb - 1) / wpb, kT, 0, s>>>(
+    { seg_popc_kernel<<<grid_for(32ull * n_pairs, n_sms), kT, 0, s>>>(
           src, par_a, W.bound.p, small, cmax, nseg, n_pairs, W.words.p,
           reinterpret_cast<unsigned long long*>(small + 2)); note_launch(); }
-    { cls_pad_kernel<<<(cmax + wpb - 1) / wpb, kT, 0, s>>>(
+    { cls_pad_kernel<<<grid_for(32ull * cmax, n_sms), kT, 0, s>>>(
           W.words.p, W.bound.p, small, cmax, nseg, W.loc.p, W.nwc.p, W.cls_words.p, W.items.p, small + 1,
           W.len.p);
       note_launch(); }
