@@ -445,6 +445,10 @@ def test_packed_upload_invalid_and_unpacked_paths(monkeypatch):
     monkeypatch.setenv("GPA_NO_PACKED_UPLOAD", "1")
     assert_mine_equal(gpa.mine(ds, min_count=theta, keep_candidates=True), ref)
     monkeypatch.delenv("GPA_NO_PACKED_UPLOAD")
+    for every in ("0", "1", "2"):        # every chunk packed / every chunk raw / alternating
+        monkeypatch.setenv("GPA_PACK_RAW_EVERY", every)
+        assert_mine_equal(gpa.mine(ds, min_count=theta, keep_candidates=True), ref)
+    monkeypatch.delenv("GPA_PACK_RAW_EVERY")
     for bad in (ds.n_items, 1 << 12):   # in range of 9 bits (>= n_items) / out of 9 bits
         items = ds.items.copy()
         items[len(items) - 5] = bad
