@@ -247,7 +247,9 @@ bool proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, 
                       cudaStream_t s, ProjPending& pp, const uint32_t* n_dev = nullptr, uint32_t* d_block = nullptr);
 bool proj_build_finish(const ProjPending& pp, const uint64_t T[2], const uint32_t sm[4], DeviceProj& out, int n_sms,
                        cudaStream_t s, cudaEvent_t ev_build);
-// counts[m] += popc(V_gpar[g] & V_eidx[m]) for every candidate m of group g (counts zeroed by the caller)
+// counts[m] += popc(V_gpar[g] & V_eidx[m]) for every candidate m of group g (counts zeroed by the caller,
+// unless count_proj_stores_all(P): the warp-per-group variant of short lists stores every count)
+bool count_proj_stores_all(const DeviceProj& P);
 void launch_count_proj(const DeviceProj& P, const uint32_t* gpar, const uint32_t* ext_off, const uint32_t* eidx,
                        uint32_t G, uint32_t* counts, cudaStream_t s);
 // items[i] = item_of_row[rows[i]] (row ids -> original item ids) for i < n, or for i < *n_dev * k

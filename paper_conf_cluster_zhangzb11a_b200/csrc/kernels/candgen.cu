@@ -51,75 +51,90 @@ __global__ void __launch_bounds__(sd::kScanThreads, 1) ge_scan_kernel(const uint
 // k = 2: candidate m is the pair (a, b) of pair_index order over n rows
 // (every scatter also writes the entry's original item ids and support for the result: ior maps a
 // bitset row to its item id; items / sup_out may be null)
-__global__ void scatter_pairs_kernel(const uint32_t* __restrict__ counts, uint32_t theta,
-                                     const uint32_t* __restrict__ pos, uint32_t M, uint32_t n,
-                                     const uint32_t* __restrict__ sel, uint32_t* L,
-                                     uint32_t* sup, uint32_t* par_a, uint32_t* par_b,
-                                     const uint32_t* __restrict__ ior, uint32_t* items, uint32_t* sup_out,
-                                     uint32_t* slots, uint32_t mask) {
-  for (uint32_t m = blockIdx.x * blockDim.x + threadIdx.x; m < M; m += gridDim.x * blockDim.x) {
-    if (counts[m] < theta) continue;
-    uint32_t lo = 0, hi = n - 1;  // a = last row whose first pair index <= m
-    while (lo + 1 < hi) {
-      const uint32_t mid = (lo + hi) >> 1;
-      if (pair_index(mid, mid + 1, n) <= m) lo = mid; else hi = mid;
-    }
-    uint32_t a = lo, b = (uint32_t)(m - pair_index(a, a + 1, n)) + a + 1;
-    if (sel) {   // logical L_1 indices -> bitset rows
-      a = sel[a];
-      b = sel[b];
-    }
-    const uint32_t p = pos[m];
-    L[2ull * p] = a;
-    L[2ull * p + 1] = b;
-    sup[p] = counts[m];
-    par_a[p] = a;
-    par_b[p] = b;
-    if (items) {
-      items[2ull * p] = ior[a];
-      items[2ull * p + 1] = ior[b];
-      sup_out[p] = counts[m];
-    }
-    if (slots) hash_insert(L + 2ull * p, 2, p, slots, mask);
+struct ScatterOut {   // L_k and the side outputs one frequent candidate is scattered into
+  uint32_t *L, *sup, *par_a, *par_b;
+  const uint32_t* ior;
+  uint32_t *items, *sup_out, *slots;
+  uint32_t mask;
+};
+
+__device__ __forceinline__ void scatter_pair(uint32_t m, uint32_t p, uint32_t c, uint32_t n,
+                                             const uint32_t* __restrict__ sel, const ScatterOut& o) {
+  uint32_t lo = 0, hi = n - 1;  // a = last row whose first pair index <= m
+  while (lo + 1 < hi) {
+    const uint32_t mid = (lo + hi) >> 1;
+    if (pair_index(mid, mid + 1, n) <= m) lo = mid; else hi = mid;
   }
+  uint32_t a = lo, b = (uint32_t)(m - pair_index(a, a + 1, n)) + a + 1;
+  if (sel) {   // logical L_1 indices -> bitset rows
+    a = sel[a];
+    b = sel[b];
+  }
+  o.L[2ull * p] = a;
+  o.L[2ull * p + 1] = b;
+  o.sup[p] = c;
+  o.par_a[p] = a;
+  o.par_b[p] = b;
+  if (o.items) {
+    o.items[2ull * p] = o.ior[a];
+    o.items[2ull * p + 1] = o.ior[b];
+    o.sup_out[p] = c;
+  }
+  if (o.slots) hash_insert(o.L + 2ull * p, 2, p, o.slots, o.mask);
 }
 
 // k >= 3: candidate m = prefix[g] ++ ext[m] with g the group holding m
-__global__ void scatter_grouped_kernel(const uint32_t* __restrict__ counts, uint32_t theta,
-                                       const uint32_t* __restrict__ pos, uint32_t M,
-                                       const uint32_t* __restrict__ prefix, const uint32_t* __restrict__ ext_off,
-                                       const uint32_t* __restrict__ ext, uint32_t G, uint32_t km1,
-                                       const uint32_t* __restrict__ gpar, const uint32_t* __restrict__ eidx,
-                                       uint32_t* L, uint32_t* sup, uint32_t* par_a, uint32_t* par_b,
-                                       const uint32_t* __restrict__ ior, uint32_t* items, uint32_t* sup_out,
-                                       uint32_t* slots, uint32_t mask) {
-  for (uint32_t m = blockIdx.x * blockDim.x + threadIdx.x; m < M; m += gridDim.x * blockDim.x) {
-    if (counts[m] < theta) continue;
-    uint32_t lo = 0, hi = G;  // g = last group with ext_off[g] <= m
-    while (lo + 1 < hi) {
-      const uint32_t mid = (lo + hi) >> 1;
-      if (ext_off[mid] <= m) lo = mid; else hi = mid;
-    }
-    const uint32_t p = pos[m];
-    uint32_t* dst = L + (uint64_t)p * (km1 + 1);
-    uint32_t* it = items ? items + (uint64_t)p * (km1 + 1) : nullptr;
-    for (uint32_t d = 0; d < km1; ++d) {
-      const uint32_t r = prefix[(uint64_t)lo * km1 + d];
-      dst[d] = r;
-      if (it) it[d] = ior[r];
-    }
-    dst[km1] = ext[m];
-    sup[p] = counts[m];
-    if (it) {
-      it[km1] = ior[ext[m]];
-      sup_out[p] = counts[m];
-    }
-    if (slots) hash_insert(dst, km1 + 1, p, slots, mask);
-    if (gpar) {
-      par_a[p] = gpar[lo];
-      par_b[p] = eidx[m];
-    }
+__device__ __forceinline__ void scatter_grouped(uint32_t m, uint32_t p, uint32_t c,
+                                                const uint32_t* __restrict__ prefix,
+                                                const uint32_t* __restrict__ ext_off, const uint32_t* __restrict__ ext,
+                                                uint32_t G, uint32_t km1, const uint32_t* __restrict__ gpar,
+                                                const uint32_t* __restrict__ eidx, const ScatterOut& o) {
+  uint32_t lo = 0, hi = G;  // g = last group with ext_off[g] <= m
+  while (lo + 1 < hi) {
+    const uint32_t mid = (lo + hi) >> 1;
+    if (ext_off[mid] <= m) lo = mid; else hi = mid;
   }
+  uint32_t* dst = o.L + (uint64_t)p * (km1 + 1);
+  uint32_t* it = o.items ? o.items + (uint64_t)p * (km1 + 1) : nullptr;
+  for (uint32_t d = 0; d < km1; ++d) {
+    const uint32_t r = prefix[(uint64_t)lo * km1 + d];
+    dst[d] = r;
+    if (it) it[d] = o.ior[r];
+  }
+  dst[km1] = ext[m];
+  o.sup[p] = c;
+  if (it) {
+    it[km1] = o.ior[ext[m]];
+    o.sup_out[p] = c;
+  }
+  if (o.slots) hash_insert(dst, km1 + 1, p, o.slots, o.mask);
+  if (gpar) {
+    o.par_a[p] = gpar[lo];
+    o.par_b[p] = eidx[m];
+  }
+}
+
+// The threshold in ONE launch: the flag scan of counts >= theta, each frequent candidate scattered
+// at its exclusive rank in the scan's output phase (after the tile's look-back: the scatters do not
+// delay later tiles), |L_k| from the last tile.  k2: pair order (generation 2), else grouped.
+template <bool K2>
+__global__ void __launch_bounds__(sd::kScanThreads, 1) ge_scatter_kernel(
+    const uint32_t* __restrict__ counts, uint32_t M, uint32_t theta, uint32_t n, const uint32_t* __restrict__ sel,
+    const uint32_t* __restrict__ prefix, const uint32_t* __restrict__ ext_off, const uint32_t* __restrict__ ext,
+    uint32_t G, uint32_t km1, const uint32_t* __restrict__ gpar, const uint32_t* __restrict__ eidx, ScatterOut o,
+    uint32_t* count, uint32_t* count2, uint32_t* sflags, uint64_t* agg, uint64_t* inc, uint32_t epoch) {
+  sd::scan_tile<uint32_t, 4>(
+      M, [&](uint32_t m) { return counts[m] >= theta ? 1u : 0u; },
+      [&](uint32_t m, uint32_t e, uint32_t f) {
+        if (!f) return;
+        if constexpr (K2) scatter_pair(m, e, counts[m], n, sel, o);
+        else scatter_grouped(m, e, counts[m], prefix, ext_off, ext, G, km1, gpar, eidx, o);
+      },
+      [&](uint32_t t) {
+        *count = t;
+        if (count2) *count2 = t;
+      },
+      sflags, agg, inc, epoch);
 }
 
 // run starts (members whose first w-1 items differ from the previous member's; zero past the
@@ -209,9 +224,7 @@ void threshold_impl(const uint32_t* counts, uint32_t M, uint32_t theta, uint32_t
                     const uint32_t* gpar, const uint32_t* eidx, DeviceLevel& out, DeviceScratch& scratch, int n_sms,
                     cudaStream_t s, uint32_t cap, const uint32_t* ior, uint32_t* items, uint32_t* sup_out,
                     uint32_t* count2) {
-  uint32_t* pos = scratch.u32b(M, s);
   out.count.ensure(1, s);
-  ge_scan(counts, M, theta, pos, out.count.p, scratch, s, count2);
   out.rows.ensure((size_t)std::max<uint32_t>(cap, 1) * k, s);
   out.sup.ensure(std::max<uint32_t>(cap, 1), s);
   out.par_a.ensure(std::max<uint32_t>(cap, 1), s);
@@ -223,16 +236,20 @@ void threshold_impl(const uint32_t* counts, uint32_t M, uint32_t theta, uint32_t
   scratch.hash_cap = hcap;
   scratch.hash_n = cap;
   GPA_CUDA(cudaMemsetAsync(slots, 0xff, (size_t)hcap * 4, s));
-  if (k == 2)
-    { scatter_pairs_kernel<<<grid_for(M, n_sms), kThreads, 0, s>>>(counts, theta, pos, M, n_rows, sel, out.rows.p,
-                                                                out.sup.p, out.par_a.p, out.par_b.p, ior, items,
-                                                                sup_out, slots, hcap - 1); note_launch(); }
-  else
-    { scatter_grouped_kernel<<<grid_for(M, n_sms), kThreads, 0, s>>>(counts, theta, pos, M, prefix, ext_off, ext, G,
-                                                                  k - 1, gpar, eidx, out.rows.p, out.sup.p,
-                                                                  out.par_a.p, out.par_b.p, ior, items, sup_out,
-                                                                  slots, hcap - 1);
-    note_launch(); }
+  const ScatterOut o{out.rows.p, out.sup.p, out.par_a.p, out.par_b.p, ior, items, sup_out, slots, hcap - 1};
+  {   // scan + scatter in one launch
+    const uint32_t tiles = scan_tiles(M, 4);
+    const uint32_t ep = scan_epoch(scratch.scan, tiles, s);
+    if (k == 2)
+      ge_scatter_kernel<true><<<tiles, sd::kScanThreads, 0, s>>>(counts, M, theta, n_rows, sel, nullptr, nullptr,
+          nullptr, 0, 1, nullptr, nullptr, o, out.count.p, count2, scratch.scan.flags.p, scratch.scan.agg.p,
+          scratch.scan.inc.p, ep);
+    else
+      ge_scatter_kernel<false><<<tiles, sd::kScanThreads, 0, s>>>(counts, M, theta, n_rows, sel, prefix, ext_off,
+          ext, G, k - 1, gpar, eidx, o, out.count.p, count2, scratch.scan.flags.p, scratch.scan.agg.p,
+          scratch.scan.inc.p, ep);
+    note_launch();
+  }
   GPA_CUDA(cudaGetLastError());
 }
 }  // namespace

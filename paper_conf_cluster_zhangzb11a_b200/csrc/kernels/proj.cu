@@ -840,10 +840,12 @@ bool proj_build(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const 
   return proj_build_finish(pp, T, sm, out, n_sms, s, ev_build);
 }
 
+bool count_proj_stores_all(const DeviceProj& P) { return (uint64_t)P.max_lw * 32 <= 8192; }
+
 void launch_count_proj(const DeviceProj& P, const uint32_t* gpar, const uint32_t* ext_off, const uint32_t* eidx,
                        uint32_t G, uint32_t* counts, cudaStream_t s) {
   if (G == 0) return;
-  if ((uint64_t)P.max_lw * 32 <= 8192)
+  if (count_proj_stores_all(P))
     { count_proj_kernel<true><<<(G + kT / 32 - 1) / (kT / 32), kT, 0, s>>>(P.data.p, P.off.p, P.nw.p, gpar, ext_off,
                                                                           eidx, counts, G); note_launch(); }
   else

@@ -203,7 +203,7 @@ bool proj_count_stage(gpa_bitset* bs, uint32_t k, const DeviceBatch& B, DevicePr
   GPA_CUDA(cudaStreamWaitEvent(s, aux_done, 0));
   if (!built) return false;
   bs->d_counts.ensure(B.M, s);
-  GPA_CUDA(cudaMemsetAsync(bs->d_counts.p, 0, (size_t)B.M * 4, s));
+  if (!count_proj_stores_all(cur)) GPA_CUDA(cudaMemsetAsync(bs->d_counts.p, 0, (size_t)B.M * 4, s));
   GPA_CUDA(cudaEventRecord(cs->eb, s));
   cs->build_words = cur.in_words;
   cs->build_bytes = (src_words + cur.words) * 4;            // sources read once, lists written once
