@@ -122,6 +122,9 @@ uint32_t scan_epoch(ScanState& st, uint32_t tiles, cudaStream_t s);
 void scan_excl_u32(const uint32_t* in, uint32_t* out, uint32_t n, uint32_t* tot, ScanState& st, cudaStream_t s);
 void scan_excl_u32(const uint32_t* in, uint32_t* out, uint32_t n, uint64_t* tot, ScanState& st, cudaStream_t s);
 void scan_excl_u64(const uint64_t* in, uint64_t* out, uint32_t n, uint64_t* tot, ScanState& st, cudaStream_t s);
+// the two above in one launch (independent inputs)
+void scan_excl_dual(const uint32_t* in1, uint32_t* out1, uint32_t n1, uint64_t* tot1, const uint64_t* in2,
+                    uint64_t* out2, uint32_t n2, uint64_t* tot2, ScanState& st, cudaStream_t s);
 // (cnt << 32 | cnt != 0) scanned as one: off = exclusive sums of cnt, idx = exclusive count of the
 // non-zero cnt, tot2 = {sum, non-zero count}
 void scan_excl_split(const uint32_t* cnt, uint32_t* off, uint32_t* idx, uint32_t n, uint32_t* tot2, ScanState& st,

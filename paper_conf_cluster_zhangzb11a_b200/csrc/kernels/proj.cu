@@ -763,8 +763,7 @@ bool proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, 
       note_launch(); }
   }
   // tot = {pext items, list words}: the totals of the two scans
-  scan_excl_u32(W.items.p, W.item_off.p, n_pairs, tot, W.scan, s);
-  scan_excl_u64(W.cls_words.p, W.cls_base.p, cmax, tot + 1, W.scan, s);
+  scan_excl_dual(W.items.p, W.item_off.p, n_pairs, tot, W.cls_words.p, W.cls_base.p, cmax, tot + 1, W.scan, s);
   GPA_CUDA(cudaGetLastError());
   pp.d_tot = tot;
   pp.d_small = small;

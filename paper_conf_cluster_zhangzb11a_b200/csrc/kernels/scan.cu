@@ -52,6 +52,26 @@ __global__ void __launch_bounds__(kScanThreads, 1) scan_split_kernel(const uint3
       flags, agg, inc, epoch);
 }
 
+// two independent exclusive scans in one launch (u32 -> u32 with a u64 total, u64 -> u64): blocks
+// [0, t1) run the first, [t1, t1 + t2) the second on status words offset by t1 (a block only waits
+// for lower-indexed blocks of its own scan, dispatched first)
+__global__ void __launch_bounds__(kScanThreads, 1) dual_scan_kernel(const uint32_t* __restrict__ in1,
+                                                                  uint32_t* __restrict__ out1, uint32_t n1,
+                                                                  uint64_t* tot1, uint32_t t1,
+                                                                  const uint64_t* __restrict__ in2,
+                                                                  uint64_t* __restrict__ out2, uint32_t n2,
+                                                                  uint64_t* tot2, uint32_t t2, uint32_t* flags,
+                                                                  uint64_t* agg, uint64_t* inc, uint32_t epoch) {
+  if (blockIdx.x < t1)
+    scan_tile<uint32_t>(
+        n1, [&](uint32_t i) { return in1[i]; }, [&](uint32_t i, uint32_t x, uint32_t) { out1[i] = x; },
+        [&](uint32_t t) { *tot1 = t; }, flags, agg, inc, epoch, 0, t1);
+  else
+    scan_tile<uint64_t>(
+        n2, [&](uint32_t i) { return in2[i]; }, [&](uint32_t i, uint64_t x, uint64_t) { out2[i] = x; },
+        [&](uint64_t t) { *tot2 = t; }, flags + t1, agg + t1, inc + t1, epoch, t1, t2);
+}
+
 }  // namespace
 
 ScanState& scan_state(int device) {
@@ -113,6 +133,20 @@ void scan_excl_split(const uint32_t* cnt, uint32_t* off, uint32_t* idx, uint32_t
   const uint32_t ep = scan_epoch(st, tiles, s);
   { scan_split_kernel<<<tiles, kScanThreads, 0, s>>>(cnt, off, idx, n, tot2, st.flags.p, st.agg.p, st.inc.p, ep);
     note_launch(); }
+  GPA_CUDA(cudaGetLastError());
+}
+
+void scan_excl_dual(const uint32_t* in1, uint32_t* out1, uint32_t n1, uint64_t* tot1, const uint64_t* in2,
+                    uint64_t* out2, uint32_t n2, uint64_t* tot2, ScanState& st, cudaStream_t s) {
+  if (n1 == 0 || n2 == 0) {   // (not on the mining path: both are >= 1 there)
+    scan_excl_u32(in1, out1, n1, tot1, st, s);
+    scan_excl_u64(in2, out2, n2, tot2, st, s);
+    return;
+  }
+  const uint32_t t1 = (n1 + kScanTile - 1) / kScanTile, t2 = (n2 + kScanTile - 1) / kScanTile;
+  const uint32_t ep = scan_epoch(st, t1 + t2, s);
+  { dual_scan_kernel<<<t1 + t2, kScanThreads, 0, s>>>(in1, out1, n1, tot1, t1, in2, out2, n2, tot2, t2, st.flags.p,
+                                                     st.agg.p, st.inc.p, ep); note_launch(); }
   GPA_CUDA(cudaGetLastError());
 }
 

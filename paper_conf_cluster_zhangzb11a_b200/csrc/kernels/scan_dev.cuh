@@ -38,13 +38,17 @@ __device__ __forceinline__ T warp_incl(T v, uint32_t lane) {
   return v;
 }
 
-// in(i): value of element i < n; out(i, exclusive prefix, value); tot(total) by the last tile
+// in(i): value of element i < n; out(i, exclusive prefix, value); tot(total) by the last tile.
+// Several scans in one launch: blocks [tile0, tile0 + n_tiles) run this one (its own status words:
+// flags / agg / inc already offset by the caller); n_tiles = 0: the whole grid.
 template <class T, int ITEMS = kScanItems, class In, class Out, class Tot>
 __device__ __forceinline__ void scan_tile(uint32_t n, In in, Out out, Tot tot, uint32_t* __restrict__ flags,
-                                          uint64_t* __restrict__ agg, uint64_t* __restrict__ inc, uint32_t epoch) {
+                                          uint64_t* __restrict__ agg, uint64_t* __restrict__ inc, uint32_t epoch,
+                                          uint32_t tile0 = 0, uint32_t n_tiles = 0) {
   __shared__ T s_warp[kScanThreads / 32];
   __shared__ T s_prefix;
-  const uint32_t tile = blockIdx.x, lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const uint32_t tile = blockIdx.x - tile0, lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const uint32_t last_tile = (n_tiles ? n_tiles : gridDim.x) - 1;
   const uint32_t base = tile * (kScanThreads * ITEMS) + threadIdx.x * ITEMS;
   T v[ITEMS];
   T sum = 0;
@@ -102,7 +106,7 @@ __device__ __forceinline__ void scan_tile(uint32_t n, In in, Out out, Tot tot, u
     }
     if (lane == 0) {
       s_prefix = prefix;
-      if (tile == gridDim.x - 1) tot(prefix + aggregate);
+      if (tile == last_tile) tot(prefix + aggregate);
     }
   }
   __syncthreads();
