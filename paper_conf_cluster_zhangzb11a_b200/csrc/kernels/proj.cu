@@ -88,22 +88,15 @@ __global__ void __launch_bounds__(sd::kScanThreads, 1) cls_scan_kernel(const uin
       sflags, agg, inc, epoch);
 }
 
-__global__ void seg_popc_kernel(Src src, const uint32_t* __restrict__ par_a, const uint32_t* __restrict__ bound,
-                                const uint32_t* __restrict__ n_cls, uint32_t cmax, uint32_t nseg, uint32_t n_pairs,
-                                uint32_t* __restrict__ words, unsigned long long* __restrict__ in_words) {
-  const uint32_t nc = *n_cls, n_warps = (gridDim.x * blockDim.x) >> 5;
-  for (uint32_t p = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; p < n_pairs; p += n_warps)
-    seg_popc_warp(p, src, par_a, bound, nc, cmax, words, in_words);
-}
-
-__global__ void cls_pad_kernel(const uint32_t* __restrict__ words, const uint32_t* __restrict__ bound,
+__global__ void seg_pad_kernel(Src src, const uint32_t* __restrict__ par_a, const uint32_t* __restrict__ bound,
                                const uint32_t* __restrict__ n_cls, uint32_t cmax, uint32_t nseg,
                                uint32_t* __restrict__ loc, uint32_t* __restrict__ nwc,
                                uint64_t* __restrict__ cls_words, uint32_t* __restrict__ items,
-                               uint32_t* __restrict__ max_lw, uint32_t* __restrict__ len) {
+                               uint32_t* __restrict__ max_lw, uint32_t* __restrict__ len,
+                               unsigned long long* __restrict__ in_words) {
   const uint32_t nc = *n_cls, n_warps = (gridDim.x * blockDim.x) >> 5;
   for (uint32_t c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < cmax; c += n_warps)
-    cls_pad_warp(c, words, bound, nc, cmax, nseg, loc, nwc, cls_words, items, max_lw, len);
+    seg_pad_warp(c, src, par_a, bound, nc, cmax, nseg, loc, nwc, cls_words, items, max_lw, len, in_words);
 }
 
 // warp per entry j: its vector (offset, words; entries of single-member classes get none), and
@@ -754,12 +747,9 @@ bool proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, 
     { cls3_pad_kernel<<<grid_for(cmax, n_sms), kT, 0, s>>>(W.words.p, W.bound.p, small, cmax, nseg, W.loc.p,
           W.nwc.p, W.cls_words.p, W.items.p, small + 1, W.len.p); note_launch(); }
   } else {
-    { seg_popc_kernel<<<grid_for(32ull * n_pairs, n_sms), kT, 0, s>>>(
-          src, par_a, W.bound.p, small, cmax, nseg, n_pairs, W.words.p,
-          reinterpret_cast<unsigned long long*>(small + 2)); note_launch(); }
-    { cls_pad_kernel<<<grid_for(32ull * cmax, n_sms), kT, 0, s>>>(
-          W.words.p, W.bound.p, small, cmax, nseg, W.loc.p, W.nwc.p, W.cls_words.p, W.items.p, small + 1,
-          W.len.p);
+    { seg_pad_kernel<<<grid_for(32ull * cmax, n_sms), kT, 0, s>>>(
+          src, par_a, W.bound.p, small, cmax, nseg, W.loc.p, W.nwc.p, W.cls_words.p, W.items.p, small + 1, W.len.p,
+          reinterpret_cast<unsigned long long*>(small + 2));
       note_launch(); }
   }
   // tot = {pext items, list words}: the totals of the two scans

@@ -35,45 +35,34 @@ __device__ __forceinline__ void seg_range(uint32_t lw, uint32_t s, uint32_t& j0,
   j1 = min(lw, j0 + kSegJ);
 }
 
-// warp per (segment s, class c) pair p = s * cmax + c: lane l's mask popcount in the segment ->
-// words[p][l] = its output words (bits rounded up to whole words)
-__device__ __forceinline__ void seg_popc_warp(uint32_t p, Src src, const uint32_t* __restrict__ par_a,
-                                              const uint32_t* __restrict__ bound, uint32_t n_cls, uint32_t cmax,
-                                              uint32_t* __restrict__ words,
-                                              unsigned long long* __restrict__ in_words) {
+// warp per class c (k >= 4: few segments per class): lane l's output words of every mask segment (the
+// lane's set bits rounded up to whole words), their prefix (loc: the lane's word offset of every
+// segment), Lw_c = max over lanes of the lane's total, words per member nwc = 32 Lw_c, the class'
+// words and its pext items (one per segment with words and group of kMemberGroup members)
+__device__ __forceinline__ void seg_pad_warp(uint32_t c, Src src, const uint32_t* __restrict__ par_a,
+                                             const uint32_t* __restrict__ bound, uint32_t n_cls, uint32_t cmax,
+                                             uint32_t nseg, uint32_t* __restrict__ loc, uint32_t* __restrict__ nwc,
+                                             uint64_t* __restrict__ cls_words, uint32_t* __restrict__ items,
+                                             uint32_t* __restrict__ max_lw, uint32_t* __restrict__ len,
+                                             unsigned long long* __restrict__ in_words) {
   const uint32_t lane = threadIdx.x & 31;
-  const uint32_t c = p % cmax, s = p / cmax;
-  uint32_t cnt = 0;
-  if (c < n_cls) {
-    const uint32_t j0 = bound[c], m = bound[c + 1] - j0;
-    if (m >= 2) {
-      const VecRef mk = src.vec(par_a[j0]);
+  uint32_t m = 0;
+  if (c < n_cls) m = bound[c + 1] - bound[c];
+  const uint32_t groups = m >= 2 ? (m + kMemberGroup - 1) / kMemberGroup : 0;
+  VecRef mk{nullptr, 0};
+  if (groups) mk = src.vec(par_a[bound[c]]);
+  uint32_t acc = 0;
+  for (uint32_t s = 0; s < nseg; ++s) {
+    const uint64_t p = (uint64_t)s * cmax + c;
+    uint32_t cnt = 0;
+    if (groups) {
       uint32_t a, b;
       seg_range(mk.lw, s, a, b);
       for (uint32_t j = a; j < b; ++j) cnt += __popc(mk.p[32ull * j + lane]);
       if (lane == 0 && b > a) atomicAdd(in_words, 32ull * (b - a) * m);
     }
-  }
-  words[(uint64_t)p * 32 + lane] = (cnt + 31) / 32;
-}
-
-// warp per class: lane l's word offset of every segment (loc), Lw_c = max over lanes of the
-// lane's total, words per member nwc = 32 Lw_c, the class' words and its pext items (one per
-// segment and group of kMemberGroup members)
-__device__ __forceinline__ void cls_pad_warp(uint32_t c, const uint32_t* __restrict__ words,
-                                             const uint32_t* __restrict__ bound, uint32_t n_cls, uint32_t cmax,
-                                             uint32_t nseg, uint32_t* __restrict__ loc, uint32_t* __restrict__ nwc,
-                                             uint64_t* __restrict__ cls_words, uint32_t* __restrict__ items,
-                                             uint32_t* __restrict__ max_lw, uint32_t* __restrict__ len) {
-  const uint32_t lane = threadIdx.x & 31;
-  uint32_t m = 0;
-  if (c < n_cls) m = bound[c + 1] - bound[c];
-  const uint32_t groups = m >= 2 ? (m + kMemberGroup - 1) / kMemberGroup : 0;
-  uint32_t acc = 0;
-  for (uint32_t s = 0; s < nseg; ++s) {
-    const uint64_t p = (uint64_t)s * cmax + c;
+    const uint32_t w = (cnt + 31) / 32;
     loc[p * 32 + lane] = acc;
-    const uint32_t w = words[p * 32 + lane];
     acc += w;
     const bool any = __any_sync(0xffffffffu, w != 0);
     if (lane == 0) items[p] = any ? groups : 0;
