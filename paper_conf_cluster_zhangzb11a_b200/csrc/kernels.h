@@ -138,6 +138,9 @@ struct DeviceScratch {
   explicit DeviceScratch(int device) : scan(scan_state(device)) {}
   DBuf<uint32_t> a, b, c, d, e, f, g, h, i;
   uint32_t hash_cap = 0;   // slots of the join's hash set (i), filled by the scatter of L (threshold)
+  // the run structure stage 1 used (its own run scan, or the class scan of the projected lists: a
+  // class of L -- entries with one left parent -- IS a run of L), for stage 2
+  const uint32_t *rflags = nullptr, *rex = nullptr, *rbound = nullptr;
   uint32_t hash_n = 0;     // the level size (upper bound) that set was built for
   ScanState& scan;
   uint32_t* u32a(size_t n, cudaStream_t s) { a.ensure(n ? n : 1, s); return a.p; }
@@ -238,6 +241,7 @@ struct ProjPending {
   uint64_t pitch = 0;
   const uint64_t* d_tot = nullptr;
   const uint32_t* d_small = nullptr;
+  const uint32_t *flag = nullptr, *ex = nullptr, *bound = nullptr;   // the class scan (null: not run)
 };
 // begin returns false (nothing enqueued) when the lists cannot be addressed (bitset >= 2^32 words,
 // too many classes): use complete intersection.
@@ -245,9 +249,12 @@ struct ProjPending {
 // before proj_build_finish.
 // d_block (optional): the generation's size block (DeviceScratch::size_block): the totals and the
 // class-table counters are written to words 2..9 of it instead of the workspace's own
+// pre / fork (optional): the class scan runs on `pre`, then s waits for `fork` recorded after it (the
+// class scan's flag / ex / bound arrays -- pp.flag, pp.ex, pp.bound -- are L's runs as well)
 bool proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const DeviceProj* prev,
                       const uint32_t* rows, uint64_t pitch_words, uint32_t n_rows, DeviceScratch& scratch, int n_sms,
-                      cudaStream_t s, ProjPending& pp, const uint32_t* n_dev = nullptr, uint32_t* d_block = nullptr);
+                      cudaStream_t s, ProjPending& pp, const uint32_t* n_dev = nullptr, uint32_t* d_block = nullptr,
+                      cudaStream_t pre = nullptr, cudaEvent_t fork = nullptr);
 bool proj_build_finish(const ProjPending& pp, const uint64_t T[2], const uint32_t sm[4], DeviceProj& out, int n_sms,
                        cudaStream_t s, cudaEvent_t ev_build);
 // counts[m] += popc(V_gpar[g] & V_eidx[m]) for every candidate m of group g (counts zeroed by the caller,
@@ -269,8 +276,11 @@ void device_candgen(const DeviceLevel& L, DeviceBatch& out, DeviceScratch& scrat
 // projected lists' class tables -- can share the synchronisation): begin leaves (M, G) at
 // *d_sizes on the device; finish sizes the batch on s and runs the emitting join on `run`
 // (waiting for s through ev when run != s).  begin returns false when |L| < 2 (no candidates).
+// runs (optional): flags / exclusive counts / bounds of L's runs already on the device (the class
+// scan of proj_build_begin, ordered before on s): no run-detection scan of its own
 bool device_candgen_begin(const DeviceLevel& L, DeviceBatch& out, DeviceScratch& scratch, int n_sms, cudaStream_t s,
-                          const uint32_t** d_sizes);
+                          const uint32_t** d_sizes, const uint32_t* run_flags = nullptr,
+                          const uint32_t* run_ex = nullptr, const uint32_t* run_bound = nullptr);
 void device_candgen_finish(const DeviceLevel& L, DeviceBatch& out, DeviceScratch& scratch, int n_sms, cudaStream_t s,
                            uint32_t M, uint32_t G, cudaStream_t run, cudaEvent_t ev);
 

@@ -308,31 +308,38 @@ void device_map_items(const uint32_t* rows, uint64_t n, const uint32_t* item_of_
 // Stage 1: run detection, hash set, survivor counts and their scans; the sizes (M, G) are left on
 // the device (sizes[0], sizes[1]) -- no synchronisation.  Returns false when L has < 2 members.
 bool device_candgen_begin(const DeviceLevel& L, DeviceBatch& out, DeviceScratch& scratch, int n_sms, cudaStream_t s,
-                          const uint32_t** d_sizes) {
+                          const uint32_t** d_sizes, const uint32_t* run_flags, const uint32_t* run_ex_in,
+                          const uint32_t* run_bound) {
   const uint32_t* n_dev = L.n_dev;
   const uint32_t n = n_dev ? L.n_max : L.n, w = L.k;   // device-sized level: n = the host upper bound
   out.k = w + 1;
   out.M = out.G = 0;
   if (n < 2) return false;
-  uint32_t* flags = scratch.u32a(n, s);
-  uint32_t* run_ex = scratch.u32b(n, s);
   uint32_t* cnt = scratch.u32c(n, s);
-  uint32_t* bound = scratch.u32d(n + 1, s);
   uint32_t* sizes = scratch.size_block(s);  // [0] = M, [1] = G
   // the hash set over L for the prune probes was filled by the scatter that wrote L (threshold_impl)
   GPA_REQUIRE(scratch.hash_cap >= 2 * n + 1 && scratch.hash_n == n && scratch.i.p, GPA_ERR_STATE,
               "join: no hash set over this level");
   const uint32_t cap = scratch.hash_cap;   // the emitting join (stage 2) probes the same table
   uint32_t* slots = scratch.i.p;
-  {
+  const uint32_t *flags = run_flags, *run_ex = run_ex_in, *bound = run_bound;
+  if (!flags) {
+    uint32_t* f = scratch.u32a(n, s);
+    uint32_t* e = scratch.u32b(n, s);
+    uint32_t* b = scratch.u32d(n + 1, s);
     const uint32_t tiles = scan_tiles(n, kRunScanItems);
     const uint32_t ep = scan_epoch(scratch.scan, tiles, s);
-    run_scan_kernel<<<tiles, sd::kScanThreads, 0, s>>>(L.rows.p, n, w, flags, run_ex, bound, n_dev,
-                                                       scratch.scan.flags.p, scratch.scan.agg.p, scratch.scan.inc.p,
-                                                       ep);
+    run_scan_kernel<<<tiles, sd::kScanThreads, 0, s>>>(L.rows.p, n, w, f, e, b, n_dev, scratch.scan.flags.p,
+                                                       scratch.scan.agg.p, scratch.scan.inc.p, ep);
     note_launch();
+    GPA_CUDA(cudaGetLastError());
+    flags = f;
+    run_ex = e;
+    bound = b;
   }
-  GPA_CUDA(cudaGetLastError());
+  scratch.rflags = flags;
+  scratch.rex = run_ex;
+  scratch.rbound = bound;
   { join_kernel<false><<<grid_for(32ull * n, n_sms), kThreads, 0, s>>>(L.rows.p, n, w, flags, run_ex, bound, slots,
         cap - 1, cnt, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, n_dev, nullptr,
         scratch.surv64(n, s)); note_launch(); }
@@ -365,8 +372,8 @@ void device_candgen_finish(const DeviceLevel& L, DeviceBatch& out, DeviceScratch
     GPA_CUDA(cudaStreamWaitEvent(run, ev, 0));
   }
   const uint32_t cap = scratch.hash_cap;   // the table stage 1 built (sized for its upper bound)
-  { join_kernel<true><<<grid_for(32ull * n, n_sms), kThreads, 0, run>>>(L.rows.p, n, w, scratch.a.p, scratch.b.p,
-        scratch.d.p, scratch.i.p, cap - 1, scratch.c.p, scratch.e.p, scratch.g.p, out.prefix.p, out.ext_off.p,
+  { join_kernel<true><<<grid_for(32ull * n, n_sms), kThreads, 0, run>>>(L.rows.p, n, w, scratch.rflags, scratch.rex,
+        scratch.rbound, scratch.i.p, cap - 1, scratch.c.p, scratch.e.p, scratch.g.p, out.prefix.p, out.ext_off.p,
         out.ext.p, out.gpar.p, out.eidx.p, nullptr, scratch.blk.p, scratch.surv.p); note_launch(); }   // + ext_off[G] = M
   GPA_CUDA(cudaGetLastError());
   out.M = M;

@@ -692,7 +692,8 @@ Src make_src(const ProjPending& pp) {
 
 bool proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, const DeviceProj* prev,
                       const uint32_t* rows, uint64_t pitch_words, uint32_t n_rows, DeviceScratch& scratch, int n_sms,
-                      cudaStream_t s, ProjPending& pp, const uint32_t* n_dev, uint32_t* d_block) {
+                      cudaStream_t s, ProjPending& pp, const uint32_t* n_dev, uint32_t* d_block, cudaStream_t pre,
+                      cudaEvent_t fork) {
   pp = ProjPending();
   pp.n = n;
   pp.par_a = par_a;
@@ -727,11 +728,19 @@ bool proj_build_begin(uint32_t n, const uint32_t* par_a, const uint32_t* par_b, 
   uint64_t* const tot = d_block ? reinterpret_cast<uint64_t*>(d_block + 2) : W.tot.p;
   {
     const uint32_t tiles = scan_tiles(n);
-    const uint32_t ep = scan_epoch(W.scan, tiles, s);
-    cls_scan_kernel<<<tiles, sd::kScanThreads, 0, s>>>(par_a, n, W.flag.p, W.ex.p, W.bound.p, small, n_dev,
-                                                       W.scan.flags.p, W.scan.agg.p, W.scan.inc.p, ep);
+    const uint32_t ep = scan_epoch(W.scan, tiles, pre ? pre : s);
+    cls_scan_kernel<<<tiles, sd::kScanThreads, 0, pre ? pre : s>>>(par_a, n, W.flag.p, W.ex.p, W.bound.p, small,
+                                                                   n_dev, W.scan.flags.p, W.scan.agg.p, W.scan.inc.p,
+                                                                   ep);
     note_launch();
   }
+  if (pre) {   // the rest of the class tables on s, after the class scan on pre
+    GPA_CUDA(cudaEventRecord(fork, pre));
+    GPA_CUDA(cudaStreamWaitEvent(s, fork, 0));
+  }
+  pp.flag = W.flag.p;
+  pp.ex = W.ex.p;
+  pp.bound = W.bound.p;
   W.words.ensure((size_t)n_pairs * 32);
   W.loc.ensure((size_t)n_pairs * 32);
   W.items.ensure(n_pairs);

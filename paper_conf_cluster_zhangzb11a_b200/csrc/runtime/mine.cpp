@@ -548,15 +548,18 @@ gpa_result* mine(const gpa_tx_csr* db, uint64_t min_count, const gpa_dist* dist,
       // the generation's sizes (|C_k|, groups, list totals, class-table counters, |L_{k-1}|) land in
       // one device block: ONE copy and ONE synchronisation per generation
       uint32_t* blk = scratch.size_block(s);
-      GPA_CUDA(cudaEventRecord(aux_evs.e[2], s));
-      GPA_CUDA(cudaStreamWaitEvent(aux_s.s, aux_evs.e[2], 0));
       const uint32_t n_up = Ld.n_dev ? Ld.n_max : Ld.n;
-      if (device_candgen_begin(Ld, Bd, scratch, bs->n_sms, s, &d_sizes)) {
+      // the class scan on s -- a class of L_{k-1} (entries with one left parent) IS a run, so it is
+      // the join's run structure too -- then the rest of the class tables on aux beside the join
+      const bool lists_ok = proj_build_begin(n_up, Ld.par_a.p, Ld.par_b.p, k == 3 ? nullptr : Pprev, bs->rows.p,
+                                             bs->pitch_words, bs->n_rows, scratch, bs->n_sms, aux_s.s, ppend,
+                                             Ld.n_dev, blk, s, aux_evs.e[2]);
+      if (!lists_ok) proj_on = false;   // lists not addressable: complete intersection from this generation on
+      const bool runs = lists_ok && ppend.flag;
+      if (device_candgen_begin(Ld, Bd, scratch, bs->n_sms, s, &d_sizes, runs ? ppend.flag : nullptr,
+                               runs ? ppend.ex : nullptr, runs ? ppend.bound : nullptr)) {
         if (trace_enabled()) GPA_CUDA(cudaEventRecord(trace_ev[0], s));
         uint32_t* hs = host_sizes();
-        if (!proj_build_begin(n_up, Ld.par_a.p, Ld.par_b.p, k == 3 ? nullptr : Pprev, bs->rows.p, bs->pitch_words,
-                              bs->n_rows, scratch, bs->n_sms, aux_s.s, ppend, Ld.n_dev, blk))
-          proj_on = false;   // lists not addressable: complete intersection from this generation on
         if (trace_enabled()) GPA_CUDA(cudaEventRecord(trace_ev[1], aux_s.s));
         GPA_CUDA(cudaEventRecord(aux_evs.e[3], aux_s.s));   // the class tables are done
         GPA_CUDA(cudaStreamWaitEvent(s, aux_evs.e[3], 0));
