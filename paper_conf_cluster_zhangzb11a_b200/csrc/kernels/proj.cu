@@ -498,7 +498,8 @@ __global__ void __launch_bounds__(kP3Warps * 32, kP3Blocks) pext3_kernel(const u
 // Warp per item = (pair p = (segment, class), group of <= kMemberGroup members: full groups of 8,
 // the remainder in the class' last group).  Items run pair-major = segment-major, so the warps in
 // flight share the same bitset segments in L2.
-__global__ void __launch_bounds__(kT, 4) pext_kernel(Src src, const uint32_t* __restrict__ par_a,
+constexpr int kPextT = 128;   // pext_kernel block (8 blocks/SM: the same 32 warps, finer scheduling)
+__global__ void __launch_bounds__(kPextT, 8) pext_kernel(Src src, const uint32_t* __restrict__ par_a,
                                                      const uint32_t* __restrict__ par_b,
                                                      const uint32_t* __restrict__ bound, uint32_t cmax,
                                                      const uint32_t* __restrict__ item_pair,
@@ -523,7 +524,7 @@ __global__ void __launch_bounds__(kT, 4) pext_kernel(Src src, const uint32_t* __
     uint32_t ja, jb;
     seg_range(mk.lw, s, ja, jb);
     if (ja >= jb) return;
-    __shared__ uint32_t s_oo[kT / 32][kMemberGroup];
+    __shared__ uint32_t s_oo[kPextT / 32][kMemberGroup];
     uint32_t* oo = s_oo[threadIdx.x >> 5];
     uint32_t so[kMemberGroup];
 #pragma unroll
@@ -806,7 +807,7 @@ bool proj_build_finish(const ProjPending& pp, const uint64_t T[2], const uint32_
     note_launch(); }
   if (ev_build) GPA_CUDA(cudaEventRecord(ev_build, s));  // start of the list build proper
   if (T[0]) {
-    const uint64_t blocks = (T[0] + kT / 32 - 1) / (kT / 32);
+    const uint64_t blocks = (T[0] + kPextT / 32 - 1) / (kPextT / 32);
     if (!pp.prev && gather3()) {
       const int smem = (int)(kP3Warps * sizeof(P3Warp));
       ensure_smem_attr((const void*)pext3_kernel, smem);
@@ -815,7 +816,7 @@ bool proj_build_finish(const ProjPending& pp, const uint64_t T[2], const uint32_
           W.loc.p, out.off.p, out.data.p);
       note_launch();
     } else
-      { pext_kernel<<<(unsigned)blocks, kT, 0, s>>>(src, pp.par_a, pp.par_b, W.bound.p, pp.cmax, W.item_pair.p,
+      { pext_kernel<<<(unsigned)blocks, kPextT, 0, s>>>(src, pp.par_a, pp.par_b, W.bound.p, pp.cmax, W.item_pair.p,
                                                     W.item_off.p, (uint32_t)T[0], W.loc.p, out.off.p, out.data.p, 4u);
         note_launch(); }
   }
