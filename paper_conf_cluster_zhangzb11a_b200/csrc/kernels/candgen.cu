@@ -20,7 +20,7 @@ namespace gpa {
 namespace {
 using namespace lvl;
 
-constexpr int kThreads = 256;
+constexpr int kThreads = 128;
 constexpr int kRunScanItems = 2;   // run detection compares two rows per member: more CTAs in flight
 
 // n_dev (device-sized levels): the member count lives on the device; n is its host upper bound
