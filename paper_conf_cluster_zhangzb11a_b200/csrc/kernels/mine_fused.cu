@@ -38,7 +38,7 @@ namespace gpa {
 namespace {
 
 constexpr int kFT = 1024;                // threads per CTA (one CTA per SM: cheap grid syncs)
-constexpr uint32_t kFusedStageWords = 8192;   // staged tile words per CTA when |L_1| <= 256
+constexpr uint32_t kFusedStageWords = 2048;   // staged tile words per CTA (tile batches of 2,048 / (32 |L_1|) tiles; measured 1,024 / 2,048 / 4,096 / 8,192 / 32,768: 2,048 best overall)
 constexpr uint32_t kNoSlot = 0xffffffffu, kClaimed = 0xfffffffeu;
 constexpr uint32_t kWarps = kFT / 32;
 
