@@ -250,7 +250,7 @@ __device__ GenState generation(const Team& T, const FusedParams& P, GenState S) 
   // ---- count C_k: (tile batch, group range) items, about two per CTA
   const uint32_t n_tiles = (P.W + 31) / 32;
   const uint32_t nu = S.n_used;   // rows C_k uses (slots assigned while L_{k-1} was scattered)
-  const uint32_t tb = max(1u, kFusedStageWords / (32 * max(nu, 1u)));   // tiles per batch (>= 8,192 staged words)
+  const uint32_t tb = max(1u, kFusedStageWords / (32 * max(nu, 1u)));   // tiles per batch (>= kFusedStageWords staged words)
   const uint32_t n_batches = (n_tiles + tb - 1) / tb;
   const uint32_t n_cta = n_threads / kFT;
   const uint32_t n_ranges = max(1u, min(G, (2 * n_cta + n_batches - 1) / n_batches));
