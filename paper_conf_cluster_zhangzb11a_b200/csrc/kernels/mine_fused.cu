@@ -174,7 +174,7 @@ struct GridTeam {
 };
 // counts[m] += popcount of the AND of candidate m's rows over a batch of 32-word tiles: work item
 // = (tile batch, range of prefix groups); the CTA stages the batch of EVERY L_1 row in shared
-// memory (8,192 words: 256 / |L_1| tiles, or one tile of |L_1| x 32 words), then a warp per group: its structure (prefix rows,
+// memory (kFusedStageWords words: 64 / |L_1| tiles, or one tile of |L_1| x 32 words), then a warp per group: its structure (prefix rows,
 // extensions) loaded once into lanes, per tile the prefix AND from shared memory (lane = word),
 // one AND + POPC per extension, warp-reduced (redux.sync), accumulated per extension in the lane
 // of that extension; one atomic per (candidate, item).  counts must be zero.
