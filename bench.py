@@ -202,6 +202,27 @@ def all_configs_table(args):
         print(json.dumps(rows[-1]), flush=True)
 
 
+def wire_bytes(offsets: np.ndarray, n_items: int, raw_every: int = 4) -> int:
+    """Host-to-device bytes of gpa_mine on host input: the library's overlapped ingest (>= 262,144
+    transactions, <= 16,384 item ids; runtime/ingest.cpp) sends the offsets and, per chunk (8 chunks
+    of whole 8,192-transaction stripes), the item ids as ceil(log2 n_items)-bit fields in blocks of 32
+    ids -- every raw_every-th chunk from chunk 0 raw (u32); otherwise everything goes raw."""
+    n_tx = len(offsets) - 1
+    o = offsets.astype(np.int64)
+    raw = int(offsets.nbytes) + 4 * int(o[-1])
+    b = max(1, int(n_items - 1).bit_length())
+    if not (n_tx >= 8 * 4 * 8192 and 2 <= n_items <= 16384 and b <= 16):
+        return raw
+    ct = -(-n_tx // 8)
+    ct = -(-ct // 8192) * 8192
+    cuts = list(range(0, n_tx, ct)) + [n_tx]
+    total = int(offsets.nbytes)
+    for c in range(len(cuts) - 1):
+        n = int(o[cuts[c + 1]] - o[cuts[c]])
+        total += 4 * n if raw_every and c % raw_every == 0 else -(-n // 32) * b * 4
+    return total
+
+
 def load_peaks() -> dict:
     try:
         return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
@@ -495,20 +516,7 @@ def main():
         e2e_ms = max_over_ranks(e0.elapsed_time(e1) / args.steps)
         assert r2.frequent() == res.frequent()
         h2d = int(ds.offsets.nbytes + ds.items.nbytes)
-        # bytes on the wire: the library's overlapped ingest (>= 262,144 transactions, <= 16,384
-        # item ids) sends the item ids as ceil(log2 n_items)-bit fields, chunk by chunk (8 chunks,
-        # 8,192-transaction aligned: runtime/ingest.cpp) -- the same formula here
-        wire = h2d
-        b = max(1, int(ds.n_items - 1).bit_length())
-        if ds.n_tx >= 8 * 4 * 8192 and ds.n_items <= 16384 and b <= 16:
-            ct = -(-ds.n_tx // 8)
-            ct = -(-ct // 8192) * 8192
-            cuts = list(range(0, ds.n_tx, ct)) + [ds.n_tx]
-            o = ds.offsets.astype(np.int64)
-            raw_every = int(os.environ.get("GPA_PACK_RAW_EVERY", "4"))   # every raw_every-th chunk goes raw
-            wire = int(ds.offsets.nbytes) + sum(
-                (int(o[cuts[c + 1]] - o[cuts[c]]) * 4 if raw_every and c % raw_every == 0
-                 else -(-int(o[cuts[c + 1]] - o[cuts[c]]) // 32) * b * 4) for c in range(len(cuts) - 1))
+        wire = wire_bytes(ds.offsets, ds.n_items, int(os.environ.get("GPA_PACK_RAW_EVERY", "4")))
         # the histogram, and every generation's frequent itemsets (k item ids + support each)
         d2h = 4 * ds.n_items + 4 * sum(lv.n_freq * (lv.k + 1) for lv in r2.levels[1:])
         e2e = {"value": cand_tx / (e2e_ms * 1e-3), "unit": "cand*tx/s", "ms_per_step": e2e_ms,

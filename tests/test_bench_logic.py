@@ -50,3 +50,23 @@ def test_pitch_bytes_matches_library_rule():
     assert bench.pitch_bytes(32768) == 4096
     assert bench.pitch_bytes(32769) == 8192
     assert bench.pitch_bytes(10_000_000) == 1_253_376
+
+
+def test_wire_bytes_follow_the_packed_upload():
+    """The bench's e2e wire bytes: offsets + per chunk either 4 bytes per id (raw) or ceil(n / 32) blocks
+    of b words (b = ceil(log2 n_items) = 10 for 1,000 ids); small inputs and > 16,384 ids go raw."""
+    import numpy as np
+    n_tx = 300_000
+    lens = np.full(n_tx, 7, np.uint64)
+    offsets = np.zeros(n_tx + 1, np.uint64)
+    np.cumsum(lens, out=offsets[1:])
+    raw = offsets.nbytes + 4 * 7 * n_tx
+    assert bench.wire_bytes(offsets, 20_000) == raw                 # > 16,384 ids
+    assert bench.wire_bytes(offsets[:1001], 1000) == offsets[:1001].nbytes + 4 * 7 * 1000   # small input
+    # 8 chunks of 40,960 transactions (37,500 rounded up to 8,192), the last one 13,280
+    chunks = [40_960] * 7 + [n_tx - 7 * 40_960]
+    packed = lambda n: -(-7 * n // 32) * 10 * 4
+    assert bench.wire_bytes(offsets, 1000, 0) == offsets.nbytes + sum(packed(n) for n in chunks)
+    assert bench.wire_bytes(offsets, 1000, 4) == offsets.nbytes + sum(
+        4 * 7 * n if c % 4 == 0 else packed(n) for c, n in enumerate(chunks))
+    assert bench.wire_bytes(offsets, 1000, 1) == raw
